@@ -1,0 +1,397 @@
+"""Pins of the CPU oracle against what the paper and mathematics fix
+(worked examples, closed forms, brute force, invariants).  CPU only."""
+from __future__ import annotations
+
+import os
+
+import numpy as np
+import pytest
+
+import bruteforce as bf
+import oracle as orc
+import workloads as wl
+from oracle import NONE
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _lines(name):
+    with open(os.path.join(GOLD, name)) as f:
+        return [l.strip() for l in f if l.strip() and not l.startswith("#")]
+
+
+def _feed(o: orc.Oracle, hashes, lists):
+    offs = np.zeros(len(lists) + 1, dtype=np.uint64)
+    offs[1:] = np.cumsum([len(l) for l in lists])
+    flat = np.array([b for l in lists for b in l], dtype=np.uint32)
+    ex = o.record_faults(np.array(hashes, dtype=np.uint64), offs, flat)
+    o.build_tables()
+    return ex
+
+
+def _state(o: orc.Oracle, what=orc.EXEC | orc.CORR | orc.BLK | orc.WALK | orc.HIST):
+    return orc.parse_dump(o.dump(what), what, o.num_exec, o.R, o.A, o.S)
+
+
+# ----------------------------------------------------------------------------
+# Fig. 7 + the chaining example of PAPER.md L222
+# ----------------------------------------------------------------------------
+def _fig7():
+    exp = {}
+    launches = {}
+    window = None
+    cur = None
+    for l in _lines("fig7_block_tables.txt"):
+        if l.startswith("EXEC"):
+            cur = int(l.split()[1])
+            exp[cur] = {"rows": {}}
+        elif l.startswith("START"):
+            exp[cur]["start"] = l.split()[1]
+        elif l.startswith("END"):
+            exp[cur]["end"] = l.split()[1]
+        elif l.startswith("LAUNCHES"):
+            parts = [p.split() for p in l[len("LAUNCHES"):].split("|")]
+            launches[int(parts[0][0])] = parts[1:]
+        elif l.startswith("WINDOW"):
+            head, tail = l[len("WINDOW"):].split("|")
+            e0, anchor, nxt = head.split()
+            window = (int(e0), anchor, int(nxt), [(x.split(":")[0], int(x.split(":")[1])) for x in tail.split()])
+        else:
+            blk, succ = l.split("|")
+            exp[cur]["rows"][blk.strip()] = succ.split()
+    return exp, launches, window
+
+
+def test_fig7_block_tables_and_l222_window():
+    exp, launches, (e0, anchor, nxt_exec, win) = _fig7()
+    letters = sorted({c for ls in launches.values() for l in ls for c in l})
+    bid = {c: 100 + i for i, c in enumerate(letters)}   # distinct small ids, distinct sets
+    name = {v: k for k, v in bid.items()}
+    # interleave exec 0 and exec 1 launches: 0,1,0,1,0,1,0,1,1
+    order = []
+    i0 = i1 = 0
+    while i0 < len(launches[0]) or i1 < len(launches[1]):
+        if i0 < len(launches[0]):
+            order.append((0, launches[0][i0])); i0 += 1
+        if i1 < len(launches[1]):
+            order.append((1, launches[1][i1])); i1 += 1
+    o = orc.Oracle(R=2048, A=2, S=4, N=4, W=4096, C=16)     # Config9
+    ex = _feed(o, [1000 + e for e, _ in order], [[bid[c] for c in l] for _, l in order])
+    assert list(ex[:2]) == [0, 1]
+    st = _state(o)
+    for e in (0, 1):
+        rows = orc.table_rows(st["blk"][e])
+        for blk, succ in exp[e]["rows"].items():
+            assert [name[s] for s in rows[bid[blk]]] == succ, (e, blk)
+        assert name[int(st["start"][e])] == exp[e]["start"]
+        assert name[int(st["end"][e])] == exp[e]["end"]
+    # the last 0 -> 1 transition was recorded with history (1, 0, 1)
+    t = len(order) - 2
+    hist = tuple(int(x) for x in ex[t - 4:t - 1])
+    assert ex[t] == 1 and ex[t - 1] == 0 and hist == (1, 0, 1)
+    q = np.array([[e0, *hist, bid[anchor], 1]], dtype=np.uint32)
+    off, pairs, ko, ch = o.predict(q)
+    assert ch[0, 0] == 0 and ch[0, 1] == nxt_exec
+    got = [(name[int(b)], int(e)) for b, e in pairs]
+    assert got == win
+    # kern_off: 2 pairs for the current kernel, 6 for the next
+    assert list(ko[0][:3]) == [0, 2, 8]
+
+
+# ----------------------------------------------------------------------------
+# Fig. 6
+# ----------------------------------------------------------------------------
+def test_fig6_execution_table():
+    lines = _lines("fig6_exec_table.txt")
+    seq = [int(x) for x in lines[-1].split()[1:]]
+    exp = {}
+    for l in lines[:-1]:
+        parts = l.split("|")
+        exp[int(parts[0])] = [tuple(int(x) for x in p.split()) for p in parts[1:]]
+    o = orc.Oracle(R=16, A=1, S=1, N=4, W=64, C=4)
+    ex = _feed(o, seq, [[] for _ in seq])   # exec-ID behaviour only: empty fault lists
+    st = _state(o)
+    label = {i: int(h) for i, h in enumerate(st["exec_hash"])}
+    assert bf.dense_exec_ids(seq) == list(ex)
+    idof = {v: k for k, v in label.items()}
+    L = lambda x: NONE if x == NONE else label[x]
+    got = {lab: [tuple(L(x) for x in r) for r in st["corr"][idof[lab]]] for lab in exp}
+    assert got[0] == exp[0]                         # exact
+    assert got[2] == exp[2]                         # exact
+    assert set(exp[1]) <= set(got[1])               # superset (see fixture comment)
+    # entry 0 with history (7, 9, 92) predicts 75
+    q = np.array([[idof[0], idof[7], idof[9], idof[92], NONE, 1]], dtype=np.uint32)
+    _, _, _, ch = o.predict(q)
+    assert label[int(ch[0, 1])] == 75
+
+
+# ----------------------------------------------------------------------------
+# Fig. 5 reconstructed (pair-based, one level + chaining)
+# ----------------------------------------------------------------------------
+def test_fig5_pair_based_prefetch_set():
+    d = {l.split()[0]: l.split()[1:] for l in _lines("fig5_pair_based.txt")}
+    bid = {c: i + 1 for i, c in enumerate("abcdefgh")}
+    o = orc.Oracle(R=2048, A=1, S=4, N=0, W=64, C=4)
+    _feed(o, [7], [[bid[c] for c in d["MISSES"]]])
+    q = np.array([[0, NONE, NONE, NONE, bid[d["REMISS"][0]], 0]], dtype=np.uint32)
+    _, pairs, _, _ = o.predict(q)
+    inv = {v: k for k, v in bid.items()}
+    assert [inv[int(b)] for b in pairs[:, 0]] == d["PREFETCH"]
+
+
+# ----------------------------------------------------------------------------
+# Config T closed form (SURVEY.md Sec. 8c "Config T closed form")
+# ----------------------------------------------------------------------------
+def test_config_T_closed_form():
+    tr = wl.make_T()
+    assert tr.n_fault == 2576
+    assert [tr.faults_in_iteration(i) for i in range(10)] == [272] + [256] * 9
+    o = orc.Oracle(R=2048, A=2, S=4, N=32, W=tr.W, C=tr.C)
+    ex_all = []
+    for i in range(tr.n_iter):
+        h, off, f = tr.iteration(i)
+        ex_all += list(o.record_faults(h, off, f))
+        o.build_tables()
+        if i >= 1:
+            st = _state(o)
+            for k in range(4):
+                e = ex_all[k]
+                assert st["start"][e] == 64 * k + 16
+                assert st["end"][e] == 64 * ((k + 1) % 4) + 15
+                steady = list(range(64 * k + 16, 64 * k + 64)) + list(range(64 * ((k + 1) % 4), 64 * ((k + 1) % 4) + 16))
+                assert list(st["walk"][e]) == steady
+    assert ex_all[:4] == [0, 1, 2, 3]
+    st = _state(o)
+    N_ = NONE
+    assert st["corr"][0] == [(N_, N_, N_, 1), (1, 2, 3, 1)]
+    assert st["corr"][1] == [(N_, N_, 0, 2), (2, 3, 0, 2)]
+    assert st["corr"][2] == [(N_, 0, 1, 3), (3, 0, 1, 3)]
+    assert st["corr"][3] == [(0, 1, 2, 0)]
+    assert st["hist"] == (0, 1, 2, 3) and st["launches"] == 40
+    q = np.array([[1, 2, 3, 0, NONE, 2]], dtype=np.uint32)
+    off, pairs, ko, ch = o.predict(q)
+    assert list(ch[0, :3]) == [1, 2, 3] and len(pairs) == 192
+    assert list(ko[0, :4]) == [0, 64, 128, 192]
+
+
+# ----------------------------------------------------------------------------
+# brute-force statistics on random tiny traces
+# ----------------------------------------------------------------------------
+@pytest.mark.parametrize("seed", range(12))
+def test_successor_lists_without_replacement(seed):
+    """No set ever overflows (every block owns its set: W <= R, low-bit index),
+    so each row must equal the S most recent distinct successors."""
+    rng = np.random.default_rng(seed)
+    S = int(rng.choice([1, 2, 4, 8]))
+    h, off, f = wl.random_trace(rng, n_launch=60, n_kernels=5, W=64, max_faults=12)
+    o = orc.Oracle(R=64, A=1, S=S, N=4, W=64, C=8)
+    ex = o.record_faults(h, off, f)
+    o.build_tables()
+    assert list(ex) == bf.dense_exec_ids(h)
+    st = _state(o)
+    for e in range(o.num_exec):
+        lists = [bf.dedupe_first(f[int(off[k]):int(off[k + 1])]) for k in range(len(h)) if ex[k] == e]
+        lists_nz = [l for l in lists if l]
+        rows = orc.table_rows(st["blk"][e])
+        assert rows == bf.successor_lists(lists, S)
+        if lists_nz:
+            assert st["start"][e] == lists_nz[-1][0] and st["end"][e] == lists_nz[-1][-1]
+        else:
+            assert st["start"][e] == NONE and st["end"][e] == NONE
+
+
+@pytest.mark.parametrize("seed", range(8))
+@pytest.mark.parametrize("A", [1, 2, 3, 4])
+def test_single_row_is_textbook_lru(seed, A):
+    """R = 1: the table is one set, i.e. an A-entry LRU cache of the blocks in
+    TOUCH order (D8)."""
+    rng = np.random.default_rng(100 + seed)
+    h, off, f = wl.random_trace(rng, n_launch=40, n_kernels=3, W=20, max_faults=10)
+    o = orc.Oracle(R=1, A=A, S=2, N=2, W=20, C=4)
+    ex = o.record_faults(h, off, f)
+    o.build_tables()
+    st = _state(o)
+    for e in range(o.num_exec):
+        touches = [b for k in range(len(h)) if ex[k] == e for b in bf.dedupe_first(f[int(off[k]):int(off[k + 1])])]
+        tags = [int(t) for t in st["blk"][e][0, :, 0] if t != NONE]
+        assert tags == bf.lru_tags(touches, A)
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_exec_prediction_is_last_successor_of_4gram(seed):
+    rng = np.random.default_rng(200 + seed)
+    n = 80
+    labels = [int(x) for x in rng.integers(0, 6, n)]
+    o = orc.Oracle(R=16, A=1, S=1, N=1, W=16, C=2)
+    ex = list(_feed(o, labels, [[] for _ in labels]))
+    E = o.num_exec
+    qs = []
+    expect = []
+    for _ in range(200):
+        e = int(rng.integers(0, E))
+        hh = tuple(int(x) if x < E else NONE for x in rng.integers(0, E + 1, 3))
+        qs.append([e, *hh, NONE, 1])
+        expect.append(bf.next_exec(ex, e, hh))
+    for k in range(3, n):  # every context that occurred
+        e, hh = ex[k], tuple(([NONE] * 3 + ex)[k:k + 3])
+        qs.append([e, *hh, NONE, 1])
+        expect.append(bf.next_exec(ex, e, hh))
+    _, _, _, ch = o.predict(np.array(qs, dtype=np.uint32))
+    assert [int(x) for x in ch[:, 1]] == expect
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_select_matches_sort_filter_take(seed):
+    rng = np.random.default_rng(300 + seed)
+    W, C = 64, 24
+    o = orc.Oracle(R=64, A=2, S=2, N=4, W=W, C=C)
+    n_res = int(rng.integers(0, C + 1))
+    lrm = [int(x) for x in rng.permutation(W)[:n_res]]
+    o.load_residency(lrm)
+    inact = set(int(x) for x in rng.permutation(W)[: W // 3])
+    o.mark_inactive(sorted(inact))
+    qoff = [0]
+    pairs = []
+    anchors = []
+    for _ in range(20):
+        k = int(rng.integers(0, 30))
+        win = [int(x) for x in rng.permutation(W)[:k]]
+        pairs += [[b, 0] for b in win]
+        qoff.append(len(pairs))
+        anchors.append(int(rng.integers(0, W)) if rng.random() < 0.5 else NONE)
+    wb_off, wb, inv_off, inv = o.select(np.array(qoff), np.array(pairs).reshape(-1, 2), np.array(anchors))
+    res = set(lrm)
+    for i in range(20):
+        win = [p[0] for p in pairs[qoff[i]:qoff[i + 1]]]
+        ew, ei = bf.select_victims(lrm, C - n_res, win, anchors[i], res, inact)
+        assert list(wb[wb_off[i]:wb_off[i + 1]]) == ew
+        assert list(inv[inv_off[i]:inv_off[i + 1]]) == ei
+        # I7: no victim is in the window or is the anchor
+        assert not (set(ew) | set(ei)) & (set(win) | {anchors[i]})
+
+
+# ----------------------------------------------------------------------------
+# periodic-trace closed form (walk = the kernel's list;
+# window = first-occurrence dedupe of the next N kernels' lists)
+# ----------------------------------------------------------------------------
+@pytest.mark.parametrize("seed", range(6))
+def test_periodic_trace_closed_form(seed):
+    rng = np.random.default_rng(400 + seed)
+    K = int(rng.integers(5, 12))
+    W = 512
+    lists = [[int(x) for x in rng.permutation(W)[: int(rng.integers(0, 20))]] for _ in range(K)]
+    N = int(rng.integers(0, 2 * K))
+    o = orc.Oracle(R=512, A=2, S=4, N=N, W=W, C=8)
+    hashes = [5000 + i for i in range(K)]
+    for it in range(3):
+        _feed(o, hashes, lists)
+    st = _state(o)
+    for e in range(K):
+        assert list(st["walk"][e]) == lists[e]
+    qs = [[k, (k - 3) % K, (k - 2) % K, (k - 1) % K, NONE, N] for k in range(K)]
+    off, pairs, ko, ch = o.predict(np.array(qs, dtype=np.uint32))
+    for k in range(K):
+        kern = [(k + d) % K for d in range(N + 1)]
+        assert list(ch[k, : N + 1]) == kern
+        exp, seen = [], set()
+        for e in kern:
+            for b in lists[e]:
+                if b not in seen:
+                    seen.add(b)
+                    exp.append((b, e))
+        got = [(int(b), int(e)) for b, e in pairs[int(off[k]):int(off[k + 1])]]
+        assert got == exp
+
+
+# ----------------------------------------------------------------------------
+# invariants I1-I6, I9 on a random trace with replacement pressure
+# ----------------------------------------------------------------------------
+@pytest.mark.parametrize("geom", [(16, 1, 1), (16, 2, 4), (4, 2, 2), (2048, 2, 4), (128, 4, 4)])
+def test_invariants_under_pressure(geom):
+    R, A, S = geom
+    rng = np.random.default_rng(R * 31 + A * 7 + S)
+    h, off, f = wl.random_trace(rng, n_launch=120, n_kernels=7, W=300, max_faults=60)
+    o = orc.Oracle(R=R, A=A, S=S, N=6, W=300, C=10)
+    ex = o.record_faults(h, off, f)
+    o.build_tables()
+    st = _state(o)
+    E = o.num_exec
+    assert list(ex) == bf.dense_exec_ids(h)                               # I3
+    for e in range(E):
+        blk = st["blk"][e]
+        for r in range(R):
+            tags = [int(t) for t in blk[r, :, 0] if t != NONE]
+            assert len(tags) == len(set(tags))                             # I1
+            assert all((t & (R - 1)) == r for t in tags)
+            valid = [w for w in range(A) if blk[r, w, 0] != NONE]
+            assert valid == list(range(len(valid)))                       # ways packed MRU-first
+            for w in valid:
+                s = [int(x) for x in blk[r, w, 1:]]
+                k = s.index(NONE) if NONE in s else S
+                assert all(x == NONE for x in s[k:])                      # I2 no holes
+                assert len(set(s[:k])) == k and blk[r, w, 0] not in s[:k]  # I2 distinct, no self
+        keys = [r[:3] for r in st["corr"][e]]
+        assert len(keys) == len(set(keys))                                 # I4
+        lists = [bf.dedupe_first(f[int(off[k]):int(off[k + 1])]) for k in range(len(h)) if ex[k] == e]
+        lists = [l for l in lists if l]
+        if lists:                                                          # I5
+            assert st["start"][e] == lists[-1][0] and st["end"][e] == lists[-1][-1]
+        w = list(st["walk"][e])
+        assert len(w) == len(set(w))                                       # I6
+        if lists:
+            assert w[0] == lists[-1][0]
+    qs = [[int(ex[k]), *([NONE] * 3 + list(ex))[k:k + 3], NONE, 6] for k in range(len(h))]
+    off_, pairs, ko, ch = o.predict(np.array(qs, dtype=np.uint32))
+    for i in range(len(qs)):
+        p = pairs[int(off_[i]):int(off_[i + 1])]
+        assert len(set(int(b) for b in p[:, 0])) == len(p)                 # I6
+        chain = [int(x) for x in ch[i] if x != NONE]
+        assert set(int(e) for e in p[:, 1]) <= set(chain) and len(chain) <= 7
+        assert ko[i, -1] == len(p) and all(np.diff(ko[i].astype(np.int64)) >= 0)
+
+
+def test_migration_bookkeeping():
+    """I9 residency bijection, lowest-free-frame-first (D21), LRM stamps (D19),
+    compaction leaves a contiguous free tail."""
+    o = orc.Oracle(R=16, A=1, S=1, N=1, W=32, C=8)
+    assert o.migrate(orc.H2D, [5, 9, 2]) == 0
+    st = orc.parse_dump(o.dump(orc.RES), orc.RES, 0, 16, 1, 1)
+    assert list(st["block_of_frame"][:3]) == [5, 9, 2] and list(st["lrm"]) == [5, 9, 2]
+    assert o.migrate(orc.D2H, [9]) == 0
+    assert o.migrate(orc.INVALIDATE, [5]) == 0
+    assert o.migrate(orc.H2D, [7, 8, 1]) == 0            # fills frames 0, 1, 3
+    st = orc.parse_dump(o.dump(orc.RES), orc.RES, 0, 16, 1, 1)
+    assert list(st["block_of_frame"][:4]) == [7, 8, 2, 1] and list(st["lrm"]) == [2, 7, 8, 1]
+    assert o.migrate(orc.H2D, [2]) != 0                  # already resident
+    assert o.migrate(orc.D2H, [2]) == 0                  # hole at frame 2
+    assert o.migrate(orc.D2D, None) == 0                 # compaction
+    st = orc.parse_dump(o.dump(orc.RES), orc.RES, 0, 16, 1, 1)
+    bof = list(st["block_of_frame"])
+    assert bof[:3] == [7, 8, 1] and all(x == NONE for x in bof[3:])
+    assert o.free_frames == 5
+    assert o.migrate(orc.H2D, list(range(10, 16))) != 0  # not enough frames
+
+
+# ----------------------------------------------------------------------------
+# Config T closed loop (all five calls) vs the survey's independent derivation
+# ----------------------------------------------------------------------------
+def _loop_rows():
+    rows = []
+    for l in _lines("T_integration_loop.txt"):
+        n, faults, h2d, d2h = [p.strip() for p in l.split("|")]
+        rows.append((int(n), [int(x) for x in faults.split()], int(h2d), int(d2h)))
+    return rows
+
+
+@pytest.mark.parametrize("row", _loop_rows(), ids=lambda r: "N%d" % r[0])
+def test_T_integration_loop(row):
+    import integration_loop as il
+    N, faults, h2d, d2h = row
+    tr = wl.make_T()
+
+    def check(k, eng):   # I7/I9 after every launch
+        res = eng.resident()
+        assert len(res) == len(set(res)) and len(res) + eng.free() == tr.C
+
+    r = il.run_loop(il.OracleLoop(tr, N), tr, N, check=check)
+    assert r["faults_per_iter"] == faults and r["h2d"] == h2d and r["d2h"] == d2h
