@@ -1,0 +1,309 @@
+/*
+ * include/deepum_b200.h -- C-ABI of the B200-native DeepUM correlation-prefetch
+ * and tensor-migration engine (libdeepum_b200.so).
+ *
+ * The five calls of the hot path follow the paper's statement of the problem
+ * (DeepUM, Jung, Kim and Lee, ASPLOS '23; "P:Lnnn" = /root/reference/PAPER.md
+ * line nnn):
+ *
+ *   dum_record_faults     a1+a2  fault records grouped per kernel launch, the
+ *                                launch's exec ID from the hash of its name and
+ *                                arguments (P:L124 step 2)
+ *   dum_build_tables      a3-a6  execution ID correlation table (P:L176,
+ *                                P:L208-L210), per-exec-ID set-associative UM
+ *                                block correlation tables with Start/End
+ *                                (P:L164-L174), walk cache
+ *   dum_predict_prefetch  a7     chained prefetch window of the current kernel
+ *                                plus the next N predicted kernels, as
+ *                                (block, exec ID) commands
+ *   dum_select_evictions  a8     pre-eviction victims: least recently migrated
+ *                                and not in the window; split into write-back
+ *                                and invalidate by PT-block inactivity
+ *
+ *   dum_migrate_blocks    a9     batched 2 MiB block moves between pinned host
+ *                                memory and HBM (P:L124 steps 4-7), plus
+ *                                HBM->HBM compaction
+ *
+ * Semantics where the paper is silent follow the readings D1-D22 listed in
+ * DESIGN.md ("Readings").  Every state-changing call is bit-exact with the
+ * sequential CPU oracle in oracle/ (tests/test_gpu_parity.py).
+ *
+ * Conventions (all calls):
+ *   - Return 0 (DUM_OK) or a negative DUM_E* code; dum_last_error() has text.
+ *   - All calls are asynchronous and stream-ordered on the given CUDA stream
+ *     (cudaStream_t passed as dum_stream_t), except dum_create, dum_destroy,
+ *     dum_dump_state, dum_sync, dum_get_stats, dum_read_counters and
+ *     dum_read_timing, which synchronize.
+ *   - Ownership: the caller owns every input/output buffer and must keep it
+ *     valid until the stream work completes; the engine owns all tables,
+ *     residency state and scratch (device memory on cfg.device).
+ *   - Pointers are device pointers unless a call says otherwise.  With
+ *     DUM_HOST_PTRS, dum_record_faults copies host inputs to the device itself.
+ *   - Errors detected on the device (a block id >= max_blocks, an exceeded
+ *     capacity) are sticky; dum_sync() returns them (and the required capacity
+ *     through *needed).  Outputs of a call that raised DUM_ECAPACITY on the
+ *     device are unspecified.
+ *   - Identifiers: UM block ids are uint32 in [0, max_blocks) (block =
+ *     (va - um_base) >> 21, D1); exec IDs are dense uint32 from 0 in
+ *     first-seen order (D3); DUM_NONE = 0xFFFFFFFF marks absence.
+ *   - Thread safety: one engine per host thread; engines share nothing.
+ */
+#ifndef DEEPUM_B200_H
+#define DEEPUM_B200_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct dum_engine dum_engine;
+typedef struct CUstream_st *dum_stream_t; /* == cudaStream_t */
+
+#define DUM_NONE 0xFFFFFFFFu
+#define DUM_BLOCK_BYTES (2ull << 20) /* 4 KB x 512 pages */
+
+enum {
+  DUM_OK = 0,
+  DUM_EINVAL = -1,    /* bad geometry / argument / alignment / block id */
+  DUM_ECAPACITY = -2, /* an output or engine capacity is too small */
+  DUM_ENOMEM = -3,
+  DUM_ECUDA = -4,
+  DUM_ESTATE = -5     /* call not valid in the engine's current state */
+};
+
+/* flags */
+#define DUM_HOST_PTRS 0x1u /* dum_record_faults: inputs are host pointers */
+
+typedef struct {
+  /* UM block correlation table geometry, Table 6;
+   * default Config9 = 2048 rows, 2-way, 4 successors.
+   * num_rows: power of two <= 8192; assoc <= 32; num_succs <= 32. */
+  uint32_t num_rows, assoc, num_succs;
+  /* degree of prefetching N: window = current + next N kernels (P:L224,
+   * P:L465; default 32) */
+  uint32_t degree_n;           /* <= 128 */
+  uint32_t max_blocks;         /* W: block-id space; <= 2^20 (window bitmaps) */
+  uint32_t max_exec_ids;       /* table capacity; DUM_ECAPACITY beyond */
+  uint32_t hbm_frames;         /* C: HBM capacity in 2 MiB frames */
+  uint32_t row_index;          /* 0 = low bits b & (R-1) (D7), 1 = fmix32 */
+  uint32_t max_batch_launches; /* staging capacity between build calls (0 = 65536) */
+  uint64_t max_batch_faults;   /* staging capacity in fault records (0 = 16 Mi) */
+  uint32_t corr_capacity;      /* exec-correlation records (0 = 16 * max_exec_ids) */
+  int device;                  /* CUDA device ordinal */
+  /* Data plane (optional; NULL = metadata-only engine, migrate -> DUM_ESTATE):
+   * host_arena: pinned (cudaHostAlloc / cudaHostRegister) host memory holding
+   *             block b at byte offset b * 2 MiB, max_blocks blocks;
+   * frame_pool: device memory holding frame f at f * 2 MiB, hbm_frames frames. */
+  void *host_arena;
+  uint64_t host_arena_bytes;
+  void *frame_pool;
+  uint64_t frame_pool_bytes;
+} dum_config;
+
+/* Fill *cfg with the defaults (Config9, N = 32). */
+void dum_config_default(dum_config *cfg);
+
+int dum_create(const dum_config *cfg, dum_engine **out);
+int dum_destroy(dum_engine *eng);
+/* Clear exec map, correlation tables, block tables, walk cache, history,
+ * staging, residency (all frames free, no inactive blocks). Keeps allocations. */
+int dum_reset(dum_engine *eng, dum_stream_t stream);
+
+/* ---- a1 + a2 ------------------------------------------------------------
+ * Stage one batch of whole kernel launches.  Launch i has hash launch_hash[i]
+ * ("hash value of the kernel's name and arguments") and the fault
+ * records fault_block[launch_off[i] .. launch_off[i+1]) (block ids, in fault
+ * order, duplicates allowed).  Requires launch_off[0] == 0 and
+ * launch_off[n_launch] == n_fault.  Records are normalised to the first
+ * occurrence of each block per launch (P:L124 step 2; D2).  Exec IDs: same
+ * hash -> same ID, else the next dense ID in first-seen order (D3);
+ * written to out_exec[i] if out_exec != NULL (device).  Staged launches are
+ * applied by the next dum_build_tables. */
+int dum_record_faults(dum_engine *eng, const uint64_t *launch_hash, const uint64_t *launch_off,
+                      uint32_t n_launch, const uint32_t *fault_block, uint64_t n_fault,
+                      uint32_t *out_exec, uint32_t flags, dum_stream_t stream);
+
+/* ---- a3 - a6 ------------------------------------------------------------
+ * Apply every staged launch, in order:
+ *  a3  record (e_{k-4}, e_{k-3}, e_{k-2} -> e_k) in entry e_{k-1} of the
+ *      execution ID correlation table (D4, D5);
+ *  a4  per normalised fault b_j of launch k (exec e): INSERT b_j as the MRU
+ *      successor in the row of b_{j-1}, then TOUCH b_j (allocate / make MRU)
+ *      in block table e (D7-D10);
+ *  a5  Start/End of e = first/last normalised fault of e's latest faulting
+ *      launch (D11);
+ *  a6  rebuild the walk cache WALK(e, NONE) of every exec ID touched
+ *      (D13). */
+int dum_build_tables(dum_engine *eng, dum_stream_t stream);
+
+/* A prefetch query: the kernel running now (exec), the three exec IDs that ran
+ * before it (hist[0] oldest; DUM_NONE allowed, D4), the faulted block the walk
+ * starts from (anchor) or DUM_NONE for a kernel-transition query that starts at
+ * Start (D14), and the degree n <= cfg.degree_n (D15). */
+typedef struct {
+  uint32_t exec;
+  uint32_t hist[3];
+  uint32_t anchor;
+  uint32_t n;
+} dum_query;
+
+/* Build transition queries for launches first..n_seq-1 of an exec-ID sequence
+ * (device array exec_seq[0..n_seq)): q[i-first] = {exec_seq[i],
+ * exec_seq[i-3..i-1] (DUM_NONE before 0), DUM_NONE, degree}. */
+int dum_make_queries(dum_engine *eng, const uint32_t *exec_seq, uint32_t n_seq, uint32_t first,
+                     uint32_t degree, dum_query *out, dum_stream_t stream);
+
+/* ---- a6 + a7 ------------------------------------------------------------
+ * For each query q (device array): chain up to q.n next-kernel predictions
+ * through the execution ID correlation table (D16), then
+ * concatenate WALK(exec, anchor) and WALK(e_d, NONE) of each predicted kernel,
+ * keeping the first occurrence of every block (D17).  Reads the state left by
+ * the last dum_build_tables.
+ *   out_pairs      pool of (block, exec) uint32 pairs, out_cap_pairs entries;
+ *   out_range      2 * n_query uint64: query i's pairs are
+ *                  out_pairs[2*out_range[2i] .. 2*out_range[2i+1]) -- each query
+ *                  owns a contiguous range; ranges are disjoint but not ordered;
+ *   out_kern_off   n_query * (degree_n + 2) uint32 or NULL: kern_off[0] = 0,
+ *                  kern_off[d+1] = pairs emitted after kernel d (padded);
+ *   out_chain      n_query * (degree_n + 1) uint32 or NULL: the predicted
+ *                  kernels (DUM_NONE padded);
+ *   out_needed     device uint64 or NULL: pool entries the call required. */
+int dum_predict_prefetch(dum_engine *eng, const dum_query *queries, uint32_t n_query, uint32_t *out_pairs,
+                         uint64_t out_cap_pairs, uint64_t *out_range, uint32_t *out_kern_off,
+                         uint32_t *out_chain, uint64_t *out_needed, dum_stream_t stream);
+
+/* ---- a8 -----------------------------------------------------------------
+ * Pre-eviction selection per query window (D18-D20): need =
+ * max(0, #window blocks without a frame - #free frames); victims = the first
+ * `need` resident blocks in least-recently-migrated order that are neither in
+ * the window nor the anchor.  Victims whose UM block is inactive (P:L285,
+ * dum_mark_inactive) go to out_invalidate, the rest to out_writeback, both in
+ * LRM order.  query_range/pairs as produced by dum_predict_prefetch; anchors
+ * are read from queries[i].anchor (queries may be NULL: no anchors).
+ *   out_range: 4 * n_query uint64 = {wb_begin, wb_end, inv_begin, inv_end}
+ *   out_needed: device uint64 or NULL (entries required per pool). */
+int dum_select_evictions(dum_engine *eng, const uint64_t *query_range, const uint32_t *pairs,
+                         uint32_t n_query, const dum_query *queries, uint32_t *out_writeback,
+                         uint32_t *out_invalidate, uint64_t out_cap, uint64_t *out_range,
+                         uint64_t *out_needed, dum_stream_t stream);
+
+/* Mark UM blocks as belonging to inactive (inactive != 0) or active PyTorch
+ * blocks (D20: a block is invalidatable iff every PT block overlapping
+ * it is inactive -- the caller resolves overlap). */
+int dum_mark_inactive(dum_engine *eng, const uint32_t *blocks, uint32_t n, int inactive,
+                      dum_stream_t stream);
+
+/* Replace the residency with a snapshot: lrm_blocks[i] resident in frame i with
+ * migration stamp i (oldest first); frames n_resident.. free. */
+int dum_load_residency(dum_engine *eng, const uint32_t *lrm_blocks, uint32_t n_resident,
+                       dum_stream_t stream);
+
+/* ---- a9 -----------------------------------------------------------------
+ * DUM_H2D:        blocks (non-resident) get the lowest free frames in list
+ *                 order (D21), are copied host -> HBM and stamped (D19).
+ * DUM_D2H:        resident blocks are copied HBM -> host and freed.
+ * DUM_INVALIDATE: resident blocks are freed without a copy.
+ * DUM_D2D:        blocks_or_src == NULL: compaction -- the resident blocks in
+ *                 the highest frames move into the lowest free frames until
+ *                 the free frames form a contiguous tail; otherwise block
+ *                 blocks_or_src[i] moves to the free frame dst_frames[i].
+ * method: 0 = auto, 1 = SM copy kernel, 2 = copy engines (cudaMemcpyAsync runs).
+ * Invalid lists (duplicates, wrong residency, not enough free frames) set a
+ * sticky DUM_EINVAL / DUM_ECAPACITY and move nothing. */
+typedef enum { DUM_H2D = 0, DUM_D2H = 1, DUM_INVALIDATE = 2, DUM_D2D = 3 } dum_dir;
+int dum_migrate_blocks(dum_engine *eng, dum_dir dir, const uint32_t *blocks_or_src, const uint32_t *dst_frames,
+                       uint32_t n, uint32_t method, dum_stream_t stream);
+
+/* 64-bit position-weighted checksums (sum_w word_w * (2w+1) mod 2^64) of 2 MiB
+ * blocks: where = 0 -> HBM frames ids[i]; 1 -> host-arena blocks ids[i]. */
+int dum_block_checksums(dum_engine *eng, int where, const uint32_t *ids, uint32_t n, uint64_t *out,
+                        dum_stream_t stream);
+
+/* ---- inspection ---------------------------------------------------------
+ * Canonical state dump (identical byte format to
+ * the oracle's).  `what` is a bitwise OR of DUM_DUMP_*.  Synchronizes.  If cap
+ * is too small nothing is written, *needed holds the size and DUM_ECAPACITY is
+ * returned. */
+#define DUM_DUMP_EXEC 1u
+#define DUM_DUMP_CORR 2u
+#define DUM_DUMP_BLK 4u
+#define DUM_DUMP_WALK 8u
+#define DUM_DUMP_RES 16u
+#define DUM_DUMP_HIST 32u
+int dum_dump_state(dum_engine *eng, uint32_t what, void *host_buf, uint64_t cap, uint64_t *needed);
+
+/* Synchronize `stream`, then return the sticky device error (clearing it) and
+ * the largest capacity a failed call required (*needed, may be NULL). */
+int dum_sync(dum_engine *eng, dum_stream_t stream, uint64_t *needed);
+
+typedef struct {
+  uint32_t num_exec;        /* exec IDs assigned */
+  uint32_t corr_records;    /* execution-correlation records */
+  uint32_t free_frames;
+  uint32_t staged_launches; /* recorded, not yet built */
+  uint64_t launches;        /* launches recorded since reset */
+  uint64_t staged_faults;
+  uint32_t slow_walks;      /* walks that took the sequential fallback in the last build */
+  uint32_t n_resident;
+} dum_stats;
+/* Synchronizes. */
+int dum_get_stats(dum_engine *eng, dum_stats *out);
+
+/* ---- instrumentation (bench / profiling; not needed for correctness) ------
+ * Work counters accumulated on the device by the kernels (one atomic per CTA);
+ * the bench derives each kernel's algorithmic bytes from them (DESIGN.md
+ * "Roofline accounting").  Reading synchronizes the device. */
+enum {
+  DUM_CTR_RAW_RECORDS = 0,  /* fault records ingested                    */
+  DUM_CTR_NORM_RECORDS,     /* after first-occurrence dedupe             */
+  DUM_CTR_LAUNCHES,         /* launches ingested                         */
+  DUM_CTR_CORR_UPSERTS,     /* exec-correlation upserts                  */
+  DUM_CTR_EXEC_BUILT,       /* exec IDs whose block table was updated    */
+  DUM_CTR_OPS,              /* fused INSERT+TOUCH ops applied            */
+  DUM_CTR_SETS,             /* (exec, set) pairs read-modified-written   */
+  DUM_CTR_WALK_ROWS,        /* rows read by walk rebuilds                */
+  DUM_CTR_WALK_OUT,         /* walk-cache entries written                */
+  DUM_CTR_QUERIES,          /* prefetch queries answered                 */
+  DUM_CTR_CHAIN,            /* kernels in predicted windows              */
+  DUM_CTR_GATHERED,         /* walk-list entries gathered by predict     */
+  DUM_CTR_EMITTED,          /* (block, exec) pairs emitted               */
+  DUM_CTR_SEL_WINDOW,       /* window entries read by select             */
+  DUM_CTR_SEL_SCANNED,      /* LRM-log entries scanned by select         */
+  DUM_CTR_SEL_VICTIMS,      /* victims selected                          */
+  DUM_CTR_MIG_BLOCKS,       /* 2 MiB blocks copied                       */
+  DUM_NCOUNTERS = 24
+};
+int dum_read_counters(dum_engine *eng, uint64_t out[DUM_NCOUNTERS], int reset);
+
+/* Per-kernel CUDA-event timing on the launching stream (off by default).
+ * dum_read_timing synchronizes and returns the summed milliseconds and launch
+ * counts per kernel since the last reset. */
+enum {
+  DUM_T_INGEST = 0,
+  DUM_T_EXEC_ASSIGN,
+  DUM_T_BUILD_PREP,
+  DUM_T_APPLY_WALK,
+  DUM_T_WALK_SLOW,
+  DUM_T_MAKE_QUERIES,
+  DUM_T_ANCHOR_WALK,
+  DUM_T_PREDICT,
+  DUM_T_SELECT,
+  DUM_T_MIG_PLAN,
+  DUM_T_COPY,
+  DUM_T_RESIDENCY,
+  DUM_NTIMERS = 16
+};
+int dum_set_timing(dum_engine *eng, int enable);
+int dum_read_timing(dum_engine *eng, double ms[DUM_NTIMERS], uint64_t count[DUM_NTIMERS], int reset);
+
+const char *dum_last_error(const dum_engine *eng);
+
+/* Number of the library's own kernel launches issued so far (for bench
+ * launch counting). */
+uint64_t dum_kernel_launches(const dum_engine *eng);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DEEPUM_B200_H */

@@ -1,0 +1,612 @@
+// libdeepum_b200.so: the C-ABI (include/deepum_b200.h) and the host engine that
+// owns the device state, validates calls and launches the kernels of
+// k_record.cu, k_build.cu, k_predict.cu, k_select.cu and k_migrate.cu in stream
+// order.  Every step of the hot path runs in those kernels; this file only
+// allocates, validates, launches, and (for dum_dump_state) canonicalises a
+// device snapshot for inspection.
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <vector>
+
+#include "device_util.cuh"
+#include "kernels.cuh"
+
+using namespace dum;
+
+namespace {
+
+__global__ void k_fill_u32(uint32_t *p, uint64_t n, uint32_t v) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    p[i] = v;
+}
+
+__global__ void k_init_corr(CorrSlot *c, uint32_t n) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    c[i].key[0] = c[i].key[1] = c[i].key[2] = c[i].key[3] = NONE;
+    c[i].last = 0;
+    c[i].first = ~0ull;
+  }
+}
+
+__global__ void k_init_state(DevState *st) {
+  st->E = 0;
+  for (int q = 0; q < 4; ++q) st->hist[q] = NONE;
+  st->err = 0;
+  st->needed = 0;
+  st->pool_pairs = st->pool_wb = st->pool_inv = st->pool_anchor = st->pool_big = 0;
+  st->n_slow = 0;
+  st->corr_used = 0;
+  st->mig_ok = 0;
+  st->mig_n = 0;
+  for (int c = 0; c < DUM_NCOUNTERS; ++c) st->ctr[c] = 0;
+}
+
+uint32_t pow2ceil_h(uint64_t x) {
+  uint64_t p = 1;
+  while (p < x) p <<= 1;
+  return (uint32_t)p;
+}
+
+int fail(dum_engine *e, int code, const char *msg) {
+  if (e) e->last_error = msg;
+  return code;
+}
+
+int cuda_fail(dum_engine *e, cudaError_t err, const char *where) {
+  if (e) {
+    e->last_error = std::string(where) + ": " + cudaGetErrorString(err);
+  }
+  return DUM_ECUDA;
+}
+
+#define CK(call)                                  \
+  do {                                            \
+    cudaError_t _e = (call);                      \
+    if (_e != cudaSuccess) return cuda_fail(e, _e, #call); \
+  } while (0)
+
+template <class T>
+cudaError_t dmalloc(T **p, uint64_t count) {
+  return cudaMalloc((void **)p, std::max<uint64_t>(count, 1) * sizeof(T));
+}
+
+cudaError_t fill(uint32_t *p, uint64_t n, uint32_t v, cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  uint64_t blocks = std::min<uint64_t>((n + 255) / 256, 4096);
+  k_fill_u32<<<(unsigned)blocks, 256, 0, s>>>(p, n, v);
+  return cudaGetLastError();
+}
+
+int reset_state(dum_engine *e, cudaStream_t s) {
+  const Geo &g = e->g;
+  CK(fill((uint32_t *)e->d_exec_keys, 2ull * (e->exec_cap + 1), NONE, s));
+  CK(cudaMemsetAsync(e->d_exec_keys + e->exec_cap, 0, 8, s));  // sentinel slot: absent
+  CK(fill(e->d_exec_vals, e->exec_cap + 1, PENDING, s));
+  CK(fill(e->d_exec_minpos, e->exec_cap + 1, NONE, s));
+  k_init_corr<<<1024, 256, 0, s>>>(e->d_corr, e->corr_cap);
+  CK(cudaGetLastError());
+  CK(fill(e->d_tbl, (uint64_t)g.Emax * g.R * g.stride, NONE, s));
+  CK(fill(e->d_start_end, 2ull * g.Emax, NONE, s));
+  CK(cudaMemsetAsync(e->d_walk_len, 0, 4ull * g.Emax, s));
+  CK(fill(e->d_head, g.Emax, NONE, s));
+  k_init_state<<<1, 1, 0, s>>>(e->d_state);
+  CK(cudaGetLastError());
+  CK(launch_reset_residency(e, s));
+  e->n_staged = 0;
+  e->staged_faults = 0;
+  e->launches = 0;
+  e->built_launches = 0;
+  e->kernel_launches += 8;
+  return DUM_OK;
+}
+
+void free_all(dum_engine *e) {
+  void *ptrs[] = {e->d_exec_keys, e->d_exec_vals, e->d_exec_minpos, e->d_exec_hash, e->d_corr, e->d_tbl,
+                  e->d_start_end, e->d_walk, e->d_walk_len, e->d_in_hash, e->d_in_off, e->d_in_faults,
+                  e->d_stage_hash, e->d_stage_norm, e->d_stage_cnt, e->d_stage_exec, e->d_stage_slot,
+                  e->d_stage_off, e->d_head, e->d_next, e->d_slow_list, e->d_big_pool, e->d_walk_seen,
+                  e->d_walk_chain, e->d_walk_tmp, e->d_walk_out, e->d_anchor_pool, e->d_anchor_range,
+                  e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits, e->d_inactive_bits, e->d_lrm_blk,
+                  e->d_lrm_stamp, e->d_mig_frames, e->d_mig_src, e->d_mig_blocks, e->d_state};
+  for (void *p : ptrs)
+    if (p) cudaFree(p);
+  if (e->h_state) cudaFreeHost(e->h_state);
+  for (auto &t : e->pending) {
+    cudaEventDestroy(t.a);
+    cudaEventDestroy(t.b);
+  }
+  for (auto ev : e->event_pool) cudaEventDestroy(ev);
+}
+
+cudaEvent_t get_event(dum_engine *e) {
+  if (!e->event_pool.empty()) {
+    cudaEvent_t ev = e->event_pool.back();
+    e->event_pool.pop_back();
+    return ev;
+  }
+  cudaEvent_t ev = nullptr;
+  cudaEventCreate(&ev);
+  return ev;
+}
+
+}  // namespace
+
+namespace dum {
+TimerScope::TimerScope(dum_engine *e_, int id_, cudaStream_t s_) : e(e_), id(id_), s(s_), b(nullptr) {
+  if (!e->timing) return;
+  cudaEvent_t a = get_event(e);
+  b = get_event(e);
+  cudaEventRecord(a, s);
+  e->pending.push_back({id, a, b});
+}
+TimerScope::~TimerScope() {
+  if (b) cudaEventRecord(b, s);
+}
+}  // namespace dum
+
+extern "C" {
+
+void dum_config_default(dum_config *c) {
+  std::memset(c, 0, sizeof(*c));
+  c->num_rows = 2048;  // Config9
+  c->assoc = 2;
+  c->num_succs = 4;
+  c->degree_n = 32;
+  c->max_blocks = 1u << 16;
+  c->max_exec_ids = 8192;
+  c->hbm_frames = 1024;
+  c->row_index = 0;
+  c->device = 0;
+}
+
+int dum_create(const dum_config *cfg, dum_engine **out) {
+  if (!cfg || !out) return DUM_EINVAL;
+  *out = nullptr;
+  const uint32_t R = cfg->num_rows, A = cfg->assoc, S = cfg->num_succs;
+  if (R == 0 || (R & (R - 1)) || R > 8192 || A == 0 || A > 32 || S == 0 || S > 32 || cfg->degree_n > 128 ||
+      cfg->max_blocks == 0 || cfg->max_blocks > (1u << 20) || cfg->max_exec_ids == 0 || cfg->hbm_frames == 0 ||
+      cfg->row_index > 1)
+    return DUM_EINVAL;
+  dum_engine *e = new (std::nothrow) dum_engine();
+  if (!e) return DUM_ENOMEM;
+  e->cfg = *cfg;
+  e->device = cfg->device;
+  e->timing = false;
+  for (int i = 0; i < DUM_NTIMERS; ++i) {
+    e->t_ms[i] = 0;
+    e->t_cnt[i] = 0;
+  }
+  Geo &g = e->g;
+  g.R = R;
+  g.A = A;
+  g.S = S;
+  g.N = cfg->degree_n;
+  g.W = cfg->max_blocks;
+  g.C = cfg->hbm_frames;
+  g.Emax = cfg->max_exec_ids;
+  g.row_index = cfg->row_index;
+  g.set_u32 = A * (1 + S);
+  g.stride = (g.set_u32 + 7) / 8 * 8;  // 32 B sectors
+  g.walk_cap = 1 + S * (R * A + 1);
+  if (cudaSetDevice(cfg->device) != cudaSuccess) {
+    delete e;
+    return DUM_ECUDA;
+  }
+  e->exec_cap = std::max<uint32_t>(64, pow2ceil_h(2ull * g.Emax));
+  const uint64_t corr_records = cfg->corr_capacity ? cfg->corr_capacity : 16ull * g.Emax;
+  e->corr_cap = pow2ceil_h(2 * corr_records);
+  e->stage_launch_cap = cfg->max_batch_launches ? cfg->max_batch_launches : 65536;
+  e->stage_fault_cap = cfg->max_batch_faults ? cfg->max_batch_faults : (16ull << 20);
+  e->big_pool_entries = 4 * e->stage_fault_cap;
+  e->n_walk_slots = 64;
+  e->walk_hash_cap = pow2ceil_h(2ull * g.walk_cap);
+  e->anchor_range_cap = 1u << 20;
+  e->anchor_pool_entries = 16ull << 20;
+  e->lrm_cap = 4 * g.C + 1024;
+  e->mig_cap = g.C + 32;
+  const uint64_t tmp_cap = g.walk_cap + (uint64_t)g.R * g.A + 4;
+  cudaError_t err = cudaSuccess;
+  auto A_ = [&](cudaError_t x) {
+    if (err == cudaSuccess) err = x;
+  };
+  A_(dmalloc(&e->d_exec_keys, e->exec_cap + 1));
+  A_(dmalloc(&e->d_exec_vals, e->exec_cap + 1));
+  A_(dmalloc(&e->d_exec_minpos, e->exec_cap + 1));
+  A_(dmalloc(&e->d_exec_hash, g.Emax));
+  A_(dmalloc(&e->d_corr, e->corr_cap));
+  A_(dmalloc(&e->d_tbl, (uint64_t)g.Emax * g.R * g.stride));
+  A_(dmalloc(&e->d_start_end, 2ull * g.Emax));
+  A_(dmalloc(&e->d_walk, (uint64_t)g.Emax * g.walk_cap));
+  A_(dmalloc(&e->d_walk_len, g.Emax));
+  A_(dmalloc(&e->d_in_hash, e->stage_launch_cap));
+  A_(dmalloc(&e->d_in_off, e->stage_launch_cap + 1ull));
+  A_(dmalloc(&e->d_in_faults, e->stage_fault_cap));
+  A_(dmalloc(&e->d_stage_hash, e->stage_launch_cap));
+  A_(dmalloc(&e->d_stage_norm, e->stage_fault_cap));
+  A_(dmalloc(&e->d_stage_cnt, e->stage_launch_cap));
+  A_(dmalloc(&e->d_stage_exec, e->stage_launch_cap));
+  A_(dmalloc(&e->d_stage_slot, e->stage_launch_cap));
+  A_(dmalloc(&e->d_stage_off, e->stage_launch_cap));
+  A_(dmalloc(&e->d_head, g.Emax));
+  A_(dmalloc(&e->d_next, e->stage_launch_cap));
+  A_(dmalloc(&e->d_slow_list, e->stage_launch_cap));
+  A_(dmalloc(&e->d_big_pool, 2 * e->big_pool_entries));
+  A_(dmalloc(&e->d_walk_seen, (uint64_t)e->n_walk_slots * e->walk_hash_cap));
+  A_(dmalloc(&e->d_walk_chain, (uint64_t)e->n_walk_slots * e->walk_hash_cap));
+  A_(dmalloc(&e->d_walk_tmp, (uint64_t)e->n_walk_slots * tmp_cap));
+  A_(dmalloc(&e->d_walk_out, (uint64_t)e->n_walk_slots * g.walk_cap));
+  A_(dmalloc(&e->d_anchor_pool, e->anchor_pool_entries));
+  A_(dmalloc(&e->d_anchor_range, 2ull * e->anchor_range_cap));
+  A_(dmalloc(&e->d_frame_of, g.W));
+  A_(dmalloc(&e->d_stamp_of, g.W));
+  A_(dmalloc(&e->d_block_of, g.C));
+  A_(dmalloc(&e->d_free_bits, (g.C + 31) / 32));
+  A_(dmalloc(&e->d_inactive_bits, (g.W + 31) / 32));
+  A_(dmalloc(&e->d_lrm_blk, e->lrm_cap));
+  A_(dmalloc(&e->d_lrm_stamp, e->lrm_cap));
+  A_(dmalloc(&e->d_mig_frames, e->mig_cap));
+  A_(dmalloc(&e->d_mig_src, e->mig_cap));
+  A_(dmalloc(&e->d_mig_blocks, e->mig_cap));
+  A_(dmalloc(&e->d_state, 1));
+  A_(cudaMallocHost((void **)&e->h_state, sizeof(DevState)));
+  if (err != cudaSuccess) {
+    free_all(e);
+    delete e;
+    return err == cudaErrorMemoryAllocation ? DUM_ENOMEM : DUM_ECUDA;
+  }
+  // walker scratch starts empty (NONE) and is kept empty by the walkers
+  fill(e->d_walk_seen, (uint64_t)e->n_walk_slots * e->walk_hash_cap, NONE, 0);
+  fill(e->d_walk_chain, (uint64_t)e->n_walk_slots * e->walk_hash_cap, NONE, 0);
+  fill(e->d_walk_tmp, (uint64_t)e->n_walk_slots * tmp_cap, NONE, 0);
+  if (cfg->host_arena) {
+    if (cfg->host_arena_bytes < (uint64_t)g.W * DUM_BLOCK_BYTES) {
+      free_all(e);
+      delete e;
+      return DUM_EINVAL;
+    }
+    void *dp = nullptr;
+    if (cudaHostGetDevicePointer(&dp, cfg->host_arena, 0) != cudaSuccess) {
+      cudaGetLastError();
+      free_all(e);
+      delete e;
+      return DUM_EINVAL;  // not pinned / not mapped
+    }
+    e->host_arena = (char *)cfg->host_arena;
+    e->host_arena_dev = (char *)dp;
+  }
+  if (cfg->frame_pool) {
+    if (cfg->frame_pool_bytes < (uint64_t)g.C * DUM_BLOCK_BYTES) {
+      free_all(e);
+      delete e;
+      return DUM_EINVAL;
+    }
+    e->frame_pool = (char *)cfg->frame_pool;
+  }
+  int rc = reset_state(e, 0);
+  if (rc == DUM_OK && cudaDeviceSynchronize() != cudaSuccess) rc = DUM_ECUDA;
+  if (rc != DUM_OK) {
+    free_all(e);
+    delete e;
+    return rc;
+  }
+  *out = e;
+  return DUM_OK;
+}
+
+int dum_destroy(dum_engine *e) {
+  if (!e) return DUM_EINVAL;
+  cudaSetDevice(e->device);
+  cudaDeviceSynchronize();
+  free_all(e);
+  delete e;
+  return DUM_OK;
+}
+
+int dum_reset(dum_engine *e, dum_stream_t stream) {
+  if (!e) return DUM_EINVAL;
+  cudaSetDevice(e->device);
+  return reset_state(e, (cudaStream_t)stream);
+}
+
+int dum_record_faults(dum_engine *e, const uint64_t *launch_hash, const uint64_t *launch_off, uint32_t n_launch,
+                      const uint32_t *fault_block, uint64_t n_fault, uint32_t *out_exec, uint32_t flags,
+                      dum_stream_t stream) {
+  if (!e) return DUM_EINVAL;
+  if (n_launch == 0) return DUM_OK;
+  if (!launch_hash || !launch_off || (n_fault && !fault_block)) return fail(e, DUM_EINVAL, "null input");
+  if ((uint64_t)e->n_staged + n_launch > e->stage_launch_cap || e->staged_faults + n_fault > e->stage_fault_cap)
+    return fail(e, DUM_ECAPACITY, "staging capacity exceeded: call dum_build_tables or raise max_batch_*");
+  if (e->launches + n_launch > 0xFFFFFFFFull) return fail(e, DUM_ECAPACITY, "launch counter exceeds 2^32");
+  cudaSetDevice(e->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  const uint64_t *h = launch_hash, *o = launch_off;
+  const uint32_t *f = fault_block;
+  if (flags & DUM_HOST_PTRS) {
+    if (launch_off[0] != 0 || launch_off[n_launch] != n_fault) return fail(e, DUM_EINVAL, "batch not launch-aligned");
+    for (uint32_t i = 0; i < n_launch; ++i)
+      if (launch_off[i + 1] < launch_off[i]) return fail(e, DUM_EINVAL, "launch_off not monotone");
+    for (uint64_t i = 0; i < n_fault; ++i)
+      if (fault_block[i] >= e->g.W) return fail(e, DUM_EINVAL, "block id >= max_blocks");
+    CK(cudaMemcpyAsync(e->d_in_hash, launch_hash, 8ull * n_launch, cudaMemcpyHostToDevice, s));
+    CK(cudaMemcpyAsync(e->d_in_off, launch_off, 8ull * (n_launch + 1), cudaMemcpyHostToDevice, s));
+    if (n_fault) CK(cudaMemcpyAsync(e->d_in_faults, fault_block, 4ull * n_fault, cudaMemcpyHostToDevice, s));
+    h = e->d_in_hash;
+    o = e->d_in_off;
+    f = e->d_in_faults;
+  } else if ((reinterpret_cast<uintptr_t>(launch_hash) | reinterpret_cast<uintptr_t>(launch_off)) & 7 ||
+             reinterpret_cast<uintptr_t>(fault_block) & 3) {
+    return fail(e, DUM_EINVAL, "unaligned pointer");
+  }
+  CK(launch_record(e, h, o, n_launch, f, out_exec, s));
+  e->n_staged += n_launch;
+  e->staged_faults += n_fault;
+  e->launches += n_launch;
+  return DUM_OK;
+}
+
+int dum_build_tables(dum_engine *e, dum_stream_t stream) {
+  if (!e) return DUM_EINVAL;
+  cudaSetDevice(e->device);
+  CK(launch_build(e, (cudaStream_t)stream));
+  e->n_staged = 0;
+  e->staged_faults = 0;
+  e->built_launches = e->launches;
+  return DUM_OK;
+}
+
+int dum_make_queries(dum_engine *e, const uint32_t *exec_seq, uint32_t n_seq, uint32_t first, uint32_t degree,
+                     dum_query *out, dum_stream_t stream) {
+  if (!e || (!exec_seq && n_seq) || (!out && first < n_seq)) return DUM_EINVAL;
+  cudaSetDevice(e->device);
+  CK(launch_make_queries(e, exec_seq, n_seq, first, degree, out, (cudaStream_t)stream));
+  return DUM_OK;
+}
+
+int dum_predict_prefetch(dum_engine *e, const dum_query *q, uint32_t n_query, uint32_t *out_pairs,
+                         uint64_t out_cap_pairs, uint64_t *out_range, uint32_t *out_kern_off, uint32_t *out_chain,
+                         uint64_t *out_needed, dum_stream_t stream) {
+  if (!e) return DUM_EINVAL;
+  if (n_query == 0) return DUM_OK;
+  if (!q || !out_range || (!out_pairs && out_cap_pairs)) return fail(e, DUM_EINVAL, "null argument");
+  if (n_query > e->anchor_range_cap) return fail(e, DUM_EINVAL, "too many queries in one call (max 2^20)");
+  if (reinterpret_cast<uintptr_t>(out_pairs) & 7) return fail(e, DUM_EINVAL, "out_pairs must be 8-byte aligned");
+  cudaSetDevice(e->device);
+  CK(launch_predict(e, q, n_query, out_pairs, out_cap_pairs, out_range, out_kern_off, out_chain, out_needed,
+                    (cudaStream_t)stream));
+  return DUM_OK;
+}
+
+int dum_select_evictions(dum_engine *e, const uint64_t *query_range, const uint32_t *pairs, uint32_t n_query,
+                         const dum_query *queries, uint32_t *out_writeback, uint32_t *out_invalidate,
+                         uint64_t out_cap, uint64_t *out_range, uint64_t *out_needed, dum_stream_t stream) {
+  if (!e) return DUM_EINVAL;
+  if (n_query == 0) return DUM_OK;
+  if (!query_range || !out_range) return fail(e, DUM_EINVAL, "null argument");
+  cudaSetDevice(e->device);
+  CK(launch_select(e, query_range, pairs, n_query, queries, out_writeback, out_invalidate, out_cap, out_range,
+                   out_needed, (cudaStream_t)stream));
+  return DUM_OK;
+}
+
+int dum_mark_inactive(dum_engine *e, const uint32_t *blocks, uint32_t n, int inactive, dum_stream_t stream) {
+  if (!e || (n && !blocks)) return DUM_EINVAL;
+  cudaSetDevice(e->device);
+  CK(launch_mark_inactive(e, blocks, n, inactive, (cudaStream_t)stream));
+  return DUM_OK;
+}
+
+int dum_load_residency(dum_engine *e, const uint32_t *lrm_blocks, uint32_t n_resident, dum_stream_t stream) {
+  if (!e || (n_resident && !lrm_blocks)) return DUM_EINVAL;
+  if (n_resident > e->g.C) return fail(e, DUM_ECAPACITY, "more resident blocks than frames");
+  cudaSetDevice(e->device);
+  CK(launch_load_residency(e, lrm_blocks, n_resident, (cudaStream_t)stream));
+  return DUM_OK;
+}
+
+int dum_migrate_blocks(dum_engine *e, dum_dir dir, const uint32_t *blocks_or_src, const uint32_t *dst_frames,
+                       uint32_t n, uint32_t method, dum_stream_t stream) {
+  if (!e) return DUM_EINVAL;
+  if ((int)dir < 0 || (int)dir > 3 || method > 2) return fail(e, DUM_EINVAL, "bad direction or method");
+  if (n > e->g.C) return fail(e, DUM_EINVAL, "list longer than the frame count");
+  if (dir != DUM_D2D && n && !blocks_or_src) return fail(e, DUM_EINVAL, "null block list");
+  if (dir == DUM_D2D && blocks_or_src && !dst_frames) return fail(e, DUM_EINVAL, "D2D needs dst_frames");
+  if (dir != DUM_INVALIDATE && (!e->frame_pool || (dir != DUM_D2D && !e->host_arena)))
+    return fail(e, DUM_ESTATE, "metadata-only engine: no host arena / frame pool configured");
+  if (n == 0 && !(dir == DUM_D2D && !blocks_or_src)) return DUM_OK;
+  cudaSetDevice(e->device);
+  CK(launch_migrate(e, (int)dir, blocks_or_src, dst_frames, n, method, (cudaStream_t)stream));
+  return DUM_OK;
+}
+
+int dum_block_checksums(dum_engine *e, int where, const uint32_t *ids, uint32_t n, uint64_t *out,
+                        dum_stream_t stream) {
+  if (!e || (n && (!ids || !out))) return DUM_EINVAL;
+  if ((where == 0 && !e->frame_pool) || (where == 1 && !e->host_arena) || where < 0 || where > 1)
+    return fail(e, DUM_ESTATE, "no such arena");
+  cudaSetDevice(e->device);
+  CK(launch_checksums(e, where, ids, n, out, (cudaStream_t)stream));
+  return DUM_OK;
+}
+
+int dum_sync(dum_engine *e, dum_stream_t stream, uint64_t *needed) {
+  if (!e) return DUM_EINVAL;
+  cudaSetDevice(e->device);
+  CK(cudaStreamSynchronize((cudaStream_t)stream));
+  CK(cudaMemcpy(e->h_state, e->d_state, sizeof(DevState), cudaMemcpyDeviceToHost));
+  const uint32_t err = e->h_state->err;
+  if (needed) *needed = e->h_state->needed;
+  if (err) {
+    CK(cudaMemset(&e->d_state->err, 0, 4));
+    CK(cudaMemset(&e->d_state->needed, 0, 8));
+    if (err & ERR_EINVAL) return fail(e, DUM_EINVAL, "device-side validation failed (block id / list / alignment)");
+    return fail(e, DUM_ECAPACITY, "device-side capacity exceeded (see *needed)");
+  }
+  return DUM_OK;
+}
+
+int dum_get_stats(dum_engine *e, dum_stats *out) {
+  if (!e || !out) return DUM_EINVAL;
+  cudaSetDevice(e->device);
+  CK(cudaDeviceSynchronize());
+  CK(cudaMemcpy(e->h_state, e->d_state, sizeof(DevState), cudaMemcpyDeviceToHost));
+  out->num_exec = e->h_state->E;
+  out->corr_records = e->h_state->corr_used;
+  out->free_frames = e->h_state->free_count;
+  out->staged_launches = e->n_staged;
+  out->launches = e->launches;
+  out->staged_faults = e->staged_faults;
+  out->slow_walks = e->h_state->n_slow;
+  out->n_resident = e->h_state->n_resident;
+  return DUM_OK;
+}
+
+const char *dum_last_error(const dum_engine *e) { return e ? e->last_error.c_str() : "null engine"; }
+
+int dum_read_counters(dum_engine *e, uint64_t out[DUM_NCOUNTERS], int reset) {
+  if (!e || !out) return DUM_EINVAL;
+  cudaSetDevice(e->device);
+  CK(cudaDeviceSynchronize());
+  CK(cudaMemcpy(out, e->d_state->ctr, sizeof(uint64_t) * DUM_NCOUNTERS, cudaMemcpyDeviceToHost));
+  if (reset) CK(cudaMemset(e->d_state->ctr, 0, sizeof(uint64_t) * DUM_NCOUNTERS));
+  return DUM_OK;
+}
+
+int dum_set_timing(dum_engine *e, int enable) {
+  if (!e) return DUM_EINVAL;
+  e->timing = enable != 0;
+  return DUM_OK;
+}
+
+int dum_read_timing(dum_engine *e, double ms[DUM_NTIMERS], uint64_t count[DUM_NTIMERS], int reset) {
+  if (!e) return DUM_EINVAL;
+  cudaSetDevice(e->device);
+  CK(cudaDeviceSynchronize());
+  for (auto &t : e->pending) {
+    float x = 0.f;
+    CK(cudaEventElapsedTime(&x, t.a, t.b));
+    e->t_ms[t.id] += x;
+    e->t_cnt[t.id] += 1;
+    e->event_pool.push_back(t.a);
+    e->event_pool.push_back(t.b);
+  }
+  e->pending.clear();
+  for (int i = 0; i < DUM_NTIMERS; ++i) {
+    if (ms) ms[i] = e->t_ms[i];
+    if (count) count[i] = e->t_cnt[i];
+    if (reset) {
+      e->t_ms[i] = 0;
+      e->t_cnt[i] = 0;
+    }
+  }
+  return DUM_OK;
+}
+
+uint64_t dum_kernel_launches(const dum_engine *e) { return e ? e->kernel_launches : 0; }
+
+// ---------------------------------------------------------------------------
+// canonical dump (host-side canonicalisation of a device snapshot)
+// ---------------------------------------------------------------------------
+static void put32(std::vector<uint8_t> &o, uint32_t v) {
+  const size_t n = o.size();
+  o.resize(n + 4);
+  std::memcpy(o.data() + n, &v, 4);
+}
+static void put64(std::vector<uint8_t> &o, uint64_t v) {
+  const size_t n = o.size();
+  o.resize(n + 8);
+  std::memcpy(o.data() + n, &v, 8);
+}
+
+int dum_dump_state(dum_engine *e, uint32_t what, void *host_buf, uint64_t cap, uint64_t *needed) {
+  if (!e) return DUM_EINVAL;
+  cudaSetDevice(e->device);
+  CK(cudaDeviceSynchronize());
+  DevState st;
+  CK(cudaMemcpy(&st, e->d_state, sizeof(st), cudaMemcpyDeviceToHost));
+  const Geo &g = e->g;
+  const uint32_t E = st.E;
+  std::vector<uint8_t> o;
+  if (what & DUM_DUMP_EXEC) {
+    std::vector<uint64_t> h(E);
+    if (E) CK(cudaMemcpy(h.data(), e->d_exec_hash, 8ull * E, cudaMemcpyDeviceToHost));
+    put32(o, E);
+    for (auto x : h) put64(o, x);
+  }
+  if (what & DUM_DUMP_CORR) {
+    std::vector<CorrSlot> c(e->corr_cap);
+    CK(cudaMemcpy(c.data(), e->d_corr, sizeof(CorrSlot) * e->corr_cap, cudaMemcpyDeviceToHost));
+    std::vector<std::vector<const CorrSlot *>> per(E);
+    for (auto &sl : c)
+      if (sl.key[0] != NONE && sl.key[0] < E) per[sl.key[0]].push_back(&sl);
+    for (uint32_t x = 0; x < E; ++x) {
+      auto &v = per[x];
+      std::sort(v.begin(), v.end(), [](const CorrSlot *a, const CorrSlot *b) { return a->first < b->first; });
+      put32(o, (uint32_t)v.size());
+      for (auto *sl : v) {
+        put32(o, sl->key[1]);
+        put32(o, sl->key[2]);
+        put32(o, sl->key[3]);
+        put32(o, (uint32_t)(sl->last & 0xFFFFFFFFull));
+      }
+    }
+  }
+  if (what & DUM_DUMP_BLK) {
+    std::vector<uint32_t> t((uint64_t)g.R * g.stride), se(2ull * std::max<uint32_t>(E, 1));
+    if (E) CK(cudaMemcpy(se.data(), e->d_start_end, 8ull * E, cudaMemcpyDeviceToHost));
+    for (uint32_t x = 0; x < E; ++x) {
+      CK(cudaMemcpy(t.data(), e->d_tbl + (uint64_t)x * g.R * g.stride, 4ull * g.R * g.stride,
+                    cudaMemcpyDeviceToHost));
+      const size_t n = o.size();
+      o.resize(n + 4ull * g.R * g.set_u32);
+      uint8_t *dst = o.data() + n;
+      for (uint32_t r = 0; r < g.R; ++r) std::memcpy(dst + 4ull * r * g.set_u32, &t[(uint64_t)r * g.stride], 4ull * g.set_u32);
+      put32(o, se[2 * x]);
+      put32(o, se[2 * x + 1]);
+    }
+  }
+  if (what & DUM_DUMP_WALK) {
+    std::vector<uint32_t> len(std::max<uint32_t>(E, 1));
+    if (E) CK(cudaMemcpy(len.data(), e->d_walk_len, 4ull * E, cudaMemcpyDeviceToHost));
+    std::vector<uint32_t> w;
+    for (uint32_t x = 0; x < E; ++x) {
+      w.resize(len[x]);
+      if (len[x])
+        CK(cudaMemcpy(w.data(), e->d_walk + (uint64_t)x * g.walk_cap, 4ull * len[x], cudaMemcpyDeviceToHost));
+      put32(o, len[x]);
+      for (auto b : w) put32(o, b);
+    }
+  }
+  if (what & DUM_DUMP_RES) {
+    std::vector<uint32_t> bof(g.C), fof(g.W), sof(g.W);
+    CK(cudaMemcpy(bof.data(), e->d_block_of, 4ull * g.C, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(fof.data(), e->d_frame_of, 4ull * g.W, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(sof.data(), e->d_stamp_of, 4ull * g.W, cudaMemcpyDeviceToHost));
+    const uint32_t nlog = st.lrm_tail - st.lrm_head;
+    std::vector<uint32_t> lb(nlog), ls(nlog);
+    if (nlog) {
+      CK(cudaMemcpy(lb.data(), e->d_lrm_blk + st.lrm_head, 4ull * nlog, cudaMemcpyDeviceToHost));
+      CK(cudaMemcpy(ls.data(), e->d_lrm_stamp + st.lrm_head, 4ull * nlog, cudaMemcpyDeviceToHost));
+    }
+    put32(o, g.C);
+    for (auto b : bof) put32(o, b);
+    std::vector<uint32_t> lrm;
+    for (uint32_t i = 0; i < nlog; ++i) {
+      const uint32_t b = lb[i];
+      if (b < g.W && fof[b] != NONE && sof[b] == ls[i]) lrm.push_back(b);
+    }
+    put32(o, (uint32_t)lrm.size());
+    for (auto b : lrm) put32(o, b);
+  }
+  if (what & DUM_DUMP_HIST) {
+    for (int q = 0; q < 4; ++q) put32(o, st.hist[q]);
+    put64(o, e->launches);
+  }
+  if (needed) *needed = o.size();
+  if (o.size() > cap) return fail(e, DUM_ECAPACITY, "dump buffer too small");
+  if (!o.empty()) std::memcpy(host_buf, o.data(), o.size());
+  return DUM_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,180 @@
+// Internal definitions of libdeepum_b200.so (not part of the C-ABI).
+//
+// HBM layout:
+//   exec map     open-addressing u64 keys / u32 ids / u32 min-position, pow2
+//                capacity >= 2 * max_exec_ids (+1 slot for the sentinel key)
+//   exec_hash    u64[max_exec_ids]   hash of exec ID e (canonical dump)
+//   corr         CorrSlot[corr_cap]  32 B: key {owner e, h1, h2, h3} (16 B,
+//                claimed with a 128-bit CAS), max(k<<32|succ), min(k)
+//   tbl          u32[E][R][stride]   set = A ways x (tag, S succ), MRU first,
+//                                    NONE-padded; stride = A(1+S) rounded up to
+//                                    a 32 B sector
+//   start_end    u32[E][2]
+//   walk         u32[E][walk_cap], walk_len u32[E]
+//   residency    frame_of u32[W], stamp_of u32[W], block_of u32[C],
+//                free bitmap u32[C/32], inactive bitmap u32[W/32],
+//                LRM log (blk u32, stamp u32)[log_cap] ordered by stamp
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "../../include/deepum_b200.h"
+
+namespace dum {
+
+// enumerators (not constexpr variables) so that device code never odr-uses them
+enum : uint32_t { NONE = 0xFFFFFFFFu, PENDING = 0xFFFFFFFEu, CLAIM = 0xFFFFFFFDu, CLAIM_DST = 0xFFFFFFFCu };
+enum : unsigned long long { EMPTY64 = 0xFFFFFFFFFFFFFFFFull };
+
+// sticky device error bits
+enum : uint32_t {
+  ERR_EINVAL = 1u,
+  ERR_ECAPACITY = 2u,
+};
+
+struct __align__(32) CorrSlot {
+  uint32_t key[4];      // owner, h1, h2, h3 ; owner == NONE -> empty
+  unsigned long long last;   // max over observations of (k << 32 | succ)
+  unsigned long long first;  // min over observations of k
+};
+
+// Device-resident engine scalars (one struct in device memory).
+struct DevState {
+  uint32_t E;                 // exec IDs assigned
+  uint32_t hist[4];           // last four exec IDs applied by build, oldest first
+  uint32_t err;               // sticky ERR_* bits
+  unsigned long long needed;  // largest capacity a failed call required
+  unsigned long long pool_pairs;   // predict output bump pointer
+  unsigned long long pool_wb, pool_inv;
+  unsigned long long pool_anchor;  // anchored-walk scratch bump pointer
+  unsigned long long pool_big;     // build-walk global hash scratch bump pointer
+  uint32_t n_slow;            // exec IDs queued for the sequential walk
+  uint32_t free_count;        // free HBM frames
+  uint32_t mig_counter;       // next migration stamp (D19)
+  uint32_t lrm_head, lrm_tail;// LRM log [head, tail)
+  uint32_t n_resident;
+  uint32_t corr_used;
+  uint32_t mig_ok;            // last migrate validated
+  uint32_t mig_n;             // blocks moved by the last migrate
+  uint32_t pad;
+  unsigned long long ctr[DUM_NCOUNTERS];  // work counters (instrumentation)
+};
+
+struct Geo {
+  uint32_t R, A, S, N, W, C, Emax;
+  uint32_t row_index;
+  uint32_t set_u32;     // A * (1 + S)
+  uint32_t stride;      // set stride in u32 (multiple of 8)
+  uint32_t walk_cap;    // per-exec walk capacity
+};
+
+__host__ __device__ inline uint32_t fmix32(uint32_t h) {
+  h ^= h >> 16;
+  h *= 0x85ebca6bu;
+  h ^= h >> 13;
+  h *= 0xc2b2ae35u;
+  h ^= h >> 16;
+  return h;
+}
+__host__ __device__ inline uint64_t fmix64(uint64_t k) {
+  k ^= k >> 33;
+  k *= 0xff51afd7ed558ccdull;
+  k ^= k >> 33;
+  k *= 0xc4ceb9fe1a85ec53ull;
+  k ^= k >> 33;
+  return k;
+}
+__host__ __device__ inline uint32_t row_of(const Geo &g, uint32_t b) {
+  return (g.row_index ? fmix32(b) : b) & (g.R - 1);
+}
+
+__device__ __forceinline__ void ctr_add(DevState *st, int c, unsigned long long v) {
+#ifdef __CUDA_ARCH__
+  if (v) atomicAdd(&st->ctr[c], v);
+#endif
+}
+
+}  // namespace dum
+
+struct dum_engine;
+namespace dum {
+// RAII event pair around a kernel launch when timing is enabled.
+struct TimerScope {
+  dum_engine *e;
+  int id;
+  cudaStream_t s;
+  cudaEvent_t b;
+  TimerScope(dum_engine *e_, int id_, cudaStream_t s_);
+  ~TimerScope();
+};
+}  // namespace dum
+
+struct dum_engine {
+  dum_config cfg;
+  dum::Geo g;
+  int device;
+  // exec map
+  uint32_t exec_cap;   // pow2; slot exec_cap is the sentinel-key slot
+  unsigned long long *d_exec_keys;
+  uint32_t *d_exec_vals, *d_exec_minpos;
+  uint64_t *d_exec_hash;
+  // corr
+  uint32_t corr_cap;
+  dum::CorrSlot *d_corr;
+  // block tables / walk cache
+  uint32_t *d_tbl, *d_start_end, *d_walk, *d_walk_len;
+  // staging
+  uint32_t stage_launch_cap;
+  uint64_t stage_fault_cap;
+  uint64_t *d_in_hash, *d_in_off;   // host-pointer inputs are copied here
+  uint32_t *d_in_faults;
+  uint64_t *d_stage_hash;
+  uint32_t *d_stage_norm, *d_stage_cnt, *d_stage_exec, *d_stage_slot;
+  uint64_t *d_stage_off;  // offset of launch j's records in d_stage_norm
+  uint32_t n_staged;
+  uint64_t staged_faults;
+  uint64_t launches;      // recorded since reset (global launch index base)
+  uint64_t built_launches;
+  // build scratch
+  uint32_t *d_head, *d_next, *d_slow_list;
+  uint32_t *d_big_pool;   // u32 pairs for large-walk hash tables
+  uint64_t big_pool_entries;
+  // walk scratch for the sequential walker (per CTA slot)
+  uint32_t n_walk_slots;
+  uint32_t walk_hash_cap; // pow2 per table
+  uint32_t *d_walk_seen, *d_walk_chain, *d_walk_tmp, *d_walk_out;
+  // predict anchored walks
+  uint32_t *d_anchor_pool;
+  uint64_t anchor_pool_entries;
+  uint64_t *d_anchor_range;   // per query (begin, len)
+  uint32_t anchor_range_cap;
+  // residency
+  uint32_t *d_frame_of, *d_stamp_of, *d_block_of, *d_free_bits, *d_inactive_bits;
+  uint32_t *d_lrm_blk, *d_lrm_stamp;
+  uint32_t lrm_cap;
+  uint32_t *d_mig_frames;     // destination frames of the last migrate
+  uint32_t *d_mig_src;        // source frames (D2D)
+  uint32_t *d_mig_blocks;     // blocks of the last migrate
+  uint32_t mig_cap;
+  // data plane
+  char *host_arena, *host_arena_dev, *frame_pool;
+  // state
+  dum::DevState *d_state;
+  dum::DevState *h_state;     // pinned mirror for dum_sync / stats
+  std::string last_error;
+  uint64_t kernel_launches;
+  // per-kernel event timing
+  bool timing;
+  struct TimedLaunch {
+    int id;
+    cudaEvent_t a, b;
+  };
+  std::vector<TimedLaunch> pending;
+  std::vector<cudaEvent_t> event_pool;
+  double t_ms[DUM_NTIMERS];
+  uint64_t t_cnt[DUM_NTIMERS];
+  int predict_smem, select_smem, build_smem;
+};

@@ -1,0 +1,583 @@
+// a3 - a6: table build.
+//
+//  k_build_prep   one thread per staged launch k: upsert the record
+//                 (e_{k-4}, e_{k-3}, e_{k-2} -> e_k) into entry e_{k-1} of the
+//                 execution ID correlation table (PAPER.md; D5): key claimed
+//                 with a 128-bit CAS, successor = max(k<<32 | e_k) ("last
+//                 wins"), order = min(k) ("first seen") -- order-independent
+//                 (SURVEY P4).  Links the launch into its exec ID's group.
+//  k_apply_walk   one CTA per exec ID with faults in the batch (the group
+//                 leader).  Applies the block-table operations of all its
+//                 launches (D7-D11): per fault b_j,
+//                 INSERT b_j into row(b_{j-1}) then TOUCH b_j.  Tables of
+//                 different exec IDs are independent (P1) and operations on
+//                 different sets commute (P2), so the ops are counting-sorted by
+//                 set in shared memory and each set's ops are applied in order
+//                 by one thread, with the set held in registers.  Then it
+//                 rebuilds the walk cache WALK(e, NONE) (
+//                 D13) in parallel -- see walk_fast() -- and records Start/End.
+//  k_walk_slow    sequential one-warp walker; takes the exec IDs whose walk
+//                 exceeded the parallel path's scratch (never on the configs
+//                 measured; kept for exactness on any input).
+#include "device_util.cuh"
+#include "kernels.cuh"
+#include "walk_seq.cuh"
+
+namespace dum {
+
+constexpr int BUILD_NT = 256;
+constexpr uint32_t GCAP = 1024;   // launches of one exec ID per build batch
+constexpr uint32_t OPCAP = 2048;  // ops per apply round
+constexpr uint32_t QCAP = 4096;   // smem walk-dedupe hash capacity (|Q| <= 2048)
+constexpr uint32_t WCAP = 2048;   // smem per-row counts (latest launch <= 2048 faults)
+
+// ---------------------------------------------------------------------------
+// k_build_prep
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void corr_upsert(CorrSlot *corr, uint32_t cap, uint32_t owner, uint32_t h1, uint32_t h2,
+                                            uint32_t h3, uint32_t succ, uint32_t k, DevState *st) {
+  const unsigned long long k0 = (unsigned long long)owner | ((unsigned long long)h1 << 32);
+  const unsigned long long k1 = (unsigned long long)h2 | ((unsigned long long)h3 << 32);
+  uint32_t s = (uint32_t)fmix64(k0 * 0x9E3779B97F4A7C15ull ^ fmix64(k1)) & (cap - 1);
+  for (uint32_t p = 0; p < cap; ++p) {
+    CorrSlot *sl = corr + s;
+    const volatile uint32_t *kv = sl->key;
+    uint32_t c0 = kv[0];
+    bool mine = false;
+    if (c0 == NONE) {
+      unsigned long long o0, o1;
+      cas128(sl->key, EMPTY64, EMPTY64, k0, k1, o0, o1);
+      if (o0 == EMPTY64 && o1 == EMPTY64) {
+        atomicAdd(&st->corr_used, 1u);
+        mine = true;
+      } else {
+        mine = (o0 == k0 && o1 == k1);
+      }
+    } else {
+      mine = c0 == owner && kv[1] == h1 && kv[2] == h2 && kv[3] == h3;
+    }
+    if (mine) {
+      atomicMax(&sl->last, ((unsigned long long)k << 32) | succ);
+      atomicMin(&sl->first, (unsigned long long)k);
+      return;
+    }
+    s = (s + 1) & (cap - 1);
+  }
+  set_err(st, ERR_ECAPACITY, 2ull * cap);
+}
+
+__global__ void k_build_prep(uint32_t n_staged, uint32_t k0, const uint32_t *__restrict__ stage_exec,
+                             const uint32_t *__restrict__ stage_cnt, CorrSlot *corr, uint32_t corr_cap,
+                             uint32_t *head, uint32_t *__restrict__ next, DevState *st) {
+  const uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
+  if (j == 0) {
+    st->pool_big = 0;
+    st->n_slow = 0;
+  }
+  if (j >= n_staged) return;
+  auto prev = [&](int m) -> uint32_t {
+    long jj = (long)j - m;
+    return jj >= 0 ? stage_exec[jj] : st->hist[4 + jj];
+  };
+  const uint32_t e = stage_exec[j];
+  const uint32_t owner = prev(1);
+  const bool up = owner != NONE && e != NONE;
+  if (up) corr_upsert(corr, corr_cap, owner, prev(4), prev(3), prev(2), e, k0 + j, st);
+  const uint32_t nup = __popc(__ballot_sync(__activemask(), up));
+  if ((threadIdx.x & 31) == __ffs(__activemask()) - 1) ctr_add(st, DUM_CTR_CORR_UPSERTS, nup);
+  if (e != NONE && stage_cnt[j] > 0) next[j] = atomicExch(&head[e], j);
+}
+
+// ---------------------------------------------------------------------------
+// set operations in registers (MAXA ways x MAXS successors, runtime A <= MAXA,
+// S <= MAXS; all indices static so the set stays in registers)
+// ---------------------------------------------------------------------------
+template <int MAXA, int MAXS>
+struct RegSet {
+  uint32_t tag[MAXA];
+  uint32_t sc[MAXA][MAXS];
+
+  __device__ __forceinline__ void load(const uint32_t *p, uint32_t A, uint32_t S) {
+#pragma unroll
+    for (int w = 0; w < MAXA; ++w) {
+      tag[w] = NONE;
+#pragma unroll
+      for (int j = 0; j < MAXS; ++j) sc[w][j] = NONE;
+      if (w < (int)A) {
+        tag[w] = p[w * (1 + S)];
+#pragma unroll
+        for (int j = 0; j < MAXS; ++j)
+          if (j < (int)S) sc[w][j] = p[w * (1 + S) + 1 + j];
+      }
+    }
+  }
+  __device__ __forceinline__ void store(uint32_t *p, uint32_t A, uint32_t S) const {
+#pragma unroll
+    for (int w = 0; w < MAXA; ++w) {
+      if (w < (int)A) {
+        p[w * (1 + S)] = tag[w];
+#pragma unroll
+        for (int j = 0; j < MAXS; ++j)
+          if (j < (int)S) p[w * (1 + S) + 1 + j] = sc[w][j];
+      }
+    }
+  }
+  // TOUCH: the block's row becomes MRU; allocate on a miss, dropping the LRU
+  // way (D8, D10).
+  __device__ __forceinline__ void touch(uint32_t b, uint32_t A) {
+    int hit = -1;
+#pragma unroll
+    for (int w = 0; w < MAXA; ++w)
+      if (w < (int)A && tag[w] == b) hit = w;
+    const int lim = hit < 0 ? (int)A - 1 : hit;  // ways [0, lim) shift down by one
+    uint32_t st = b;
+    uint32_t ss[MAXS];
+#pragma unroll
+    for (int j = 0; j < MAXS; ++j) ss[j] = NONE;
+    if (hit >= 0) {
+#pragma unroll
+      for (int w = 0; w < MAXA; ++w)
+        if (w == hit) {
+#pragma unroll
+          for (int j = 0; j < MAXS; ++j) ss[j] = sc[w][j];
+        }
+    }
+#pragma unroll
+    for (int w = MAXA - 1; w >= 1; --w) {
+      if (w <= lim) {
+        tag[w] = tag[w - 1];
+#pragma unroll
+        for (int j = 0; j < MAXS; ++j) sc[w][j] = sc[w - 1][j];
+      }
+    }
+    tag[0] = st;
+#pragma unroll
+    for (int j = 0; j < MAXS; ++j) sc[0][j] = ss[j];
+  }
+  // INSERT s as the MRU successor of the row in way 0 (D9).
+  __device__ __forceinline__ void insert0(uint32_t s, uint32_t S) {
+    if (s == tag[0]) return;
+    int pos = -1;
+#pragma unroll
+    for (int j = 0; j < MAXS; ++j)
+      if (j < (int)S && sc[0][j] == s) pos = j;
+    const int lim = pos < 0 ? (int)S - 1 : pos;
+#pragma unroll
+    for (int j = MAXS - 1; j >= 1; --j)
+      if (j <= lim) sc[0][j] = sc[0][j - 1];
+    sc[0][0] = s;
+  }
+};
+
+// ---------------------------------------------------------------------------
+// k_apply_walk
+// ---------------------------------------------------------------------------
+struct BuildArgs {
+  Geo g;
+  uint32_t n_staged;
+  const uint32_t *stage_exec, *stage_cnt, *stage_norm;
+  const uint64_t *stage_off;
+  uint32_t *head, *next;
+  uint32_t *tbl, *start_end, *walk, *walk_len;
+  uint32_t *big_pool;
+  uint64_t big_entries;
+  uint32_t *slow_list;
+  DevState *st;
+};
+
+// Parallel WALK(e, NONE) right after the build (D13).  Let C = the latest
+// faulting launch of e in this batch (deduplicated, n = |C|); then Start =
+// C[0], End = C[n-1] (D11).  After the build, the row of C[i] (if still
+// present) has C[i+1] as its MRU successor: INSERT(C[i] -> C[i+1]) was the last
+// operation on that row, because C is duplicate-free and no later launch of e
+// is in the batch.  C[i+1] is not among the chained nodes C[0..i], so the
+// sequential walk's next chain node is exactly C[i+1] until the first i at
+// which the row is missing or a successor equals End.  With t that index, the
+// walk is the first-occurrence dedupe of
+//   Q = [C[0]] ++ succ(row C[0]) ++ ... ++ succ(row C[t])   (row C[t] only if
+//                                                            present).
+// The speculation is still verified (succ[0] == C[i+1]); any violation sends e
+// to the sequential walker.
+template <int MAXA, int MAXS>
+__global__ void __launch_bounds__(BUILD_NT) k_apply_walk(BuildArgs a) {
+  extern __shared__ uint32_t sm[];
+  __shared__ uint32_t ws[BUILD_NT / 32];
+  __shared__ uint32_t s_ng, s_tev, s_flag;
+  const Geo &g = a.g;
+  const uint32_t tid = threadIdx.x;
+  const uint32_t j = blockIdx.x;
+  if (j == 0 && tid == 0) {
+    // history shift register after this batch: the last four exec IDs of
+    // (old history ++ staged launches); read by k_build_prep only.
+    uint32_t h[4];
+    for (int q = 0; q < 4; ++q) {
+      const long jj = (long)a.n_staged - 4 + q;
+      h[q] = jj >= 0 ? a.stage_exec[jj] : a.st->hist[4 + jj];
+    }
+    for (int q = 0; q < 4; ++q) a.st->hist[q] = h[q];
+  }
+  const uint32_t e = a.stage_exec[j];
+  if (e == NONE || a.stage_cnt[j] == 0) return;
+  if (__ldcg(&a.head[e]) != j) return;  // not this exec ID's group leader
+
+  uint32_t *grp = sm;              // [GCAP]
+  uint32_t *seg = grp + GCAP;      // [GCAP + 1]
+  uint32_t *U = seg + GCAP + 1;    // union region
+  const uint32_t R = g.R, A = g.A, S = g.S;
+
+  // ---- collect and order the group's launches ----
+  if (tid == 0) {
+    uint32_t x = j, n = 0;
+    while (x != NONE && n < GCAP) {
+      grp[n++] = x;
+      x = __ldcg(&a.next[x]);
+    }
+    if (x != NONE) set_err(a.st, ERR_ECAPACITY, GCAP + 1);
+    s_ng = n;
+    a.head[e] = NONE;
+  }
+  __syncthreads();
+  const uint32_t ng = s_ng;
+  {
+    // rank sort (ascending launch index)
+    uint32_t *tmp = U;
+    for (uint32_t p = tid; p < ng; p += BUILD_NT) {
+      uint32_t v = grp[p], r = 0;
+      for (uint32_t q = 0; q < ng; ++q) r += grp[q] < v;
+      tmp[r] = v;
+    }
+    __syncthreads();
+    for (uint32_t p = tid; p < ng; p += BUILD_NT) grp[p] = tmp[p];
+    __syncthreads();
+    if (tid == 0) {
+      uint32_t acc = 0;
+      for (uint32_t p = 0; p < ng; ++p) {
+        seg[p] = acc;
+        acc += a.stage_cnt[grp[p]];
+      }
+      seg[ng] = acc;
+    }
+    __syncthreads();
+  }
+  const uint32_t n_ops = seg[ng];
+  __shared__ uint32_t s_sets;
+  if (tid == 0) s_sets = 0;
+  uint32_t *tbl_e = a.tbl + (uint64_t)e * R * g.stride;
+
+  // ---- apply: rounds of up to OPCAP ops, counting-sorted by set ----
+  uint32_t *cnt_s = U, *off_s = U + R;
+  uint32_t *opb = off_s + R, *opn = opb + OPCAP, *opset = opn + OPCAP, *sorted = opset + OPCAP;
+  for (uint32_t r0 = 0; r0 < n_ops; r0 += OPCAP) {
+    const uint32_t m = min(OPCAP, n_ops - r0);
+    for (uint32_t s = tid; s < R; s += BUILD_NT) {
+      cnt_s[s] = 0;
+      off_s[s] = 0;
+    }
+    __syncthreads();
+    for (uint32_t p = tid; p < m; p += BUILD_NT) {
+      const uint32_t gp = r0 + p;
+      uint32_t lo = 0, hi = ng;  // seg[lo] <= gp < seg[lo+1]
+      while (hi - lo > 1) {
+        uint32_t mid = (lo + hi) >> 1;
+        if (seg[mid] <= gp) lo = mid;
+        else hi = mid;
+      }
+      const uint32_t L = grp[lo];
+      const uint64_t base = a.stage_off[L];
+      const uint32_t idx = gp - seg[lo];
+      const uint32_t b = a.stage_norm[base + idx];
+      const uint32_t nx = (gp + 1 < seg[lo + 1]) ? a.stage_norm[base + idx + 1] : NONE;
+      const uint32_t s = row_of(g, b);
+      opb[p] = b;
+      opn[p] = nx;
+      opset[p] = s;
+      atomicAdd(&cnt_s[s], 1u);
+    }
+    __syncthreads();
+    {
+      // exclusive scan of cnt_s over R sets (each thread a contiguous chunk)
+      const uint32_t per = (R + BUILD_NT - 1) / BUILD_NT;
+      const uint32_t s0 = tid * per, s1 = min(R, s0 + per);
+      uint32_t loc = 0;
+      for (uint32_t s = s0; s < s1; ++s) loc += cnt_s[s];
+      uint32_t tot;
+      uint32_t pre = block_excl_scan(loc, ws, &tot);
+      for (uint32_t s = s0; s < s1; ++s) {
+        off_s[s] = pre;
+        pre += cnt_s[s];
+      }
+    }
+    __syncthreads();
+    for (uint32_t p = tid; p < m; p += BUILD_NT) {
+      const uint32_t s = opset[p];
+      const uint32_t pos = atomicAdd(&off_s[s], 1u);  // off_s becomes the bucket end
+      sorted[pos] = p;
+    }
+    __syncthreads();
+    for (uint32_t s = tid; s < R; s += BUILD_NT) {
+      const uint32_t c = cnt_s[s];
+      if (c == 0) continue;
+      const uint32_t e1 = off_s[s], b0 = e1 - c;
+      // insertion sort of the bucket by op position (buckets are tiny)
+      for (uint32_t u = b0 + 1; u < e1; ++u) {
+        uint32_t v = sorted[u];
+        uint32_t w = u;
+        while (w > b0 && sorted[w - 1] > v) {
+          sorted[w] = sorted[w - 1];
+          --w;
+        }
+        sorted[w] = v;
+      }
+      atomicAdd(&s_sets, 1u);
+      RegSet<MAXA, MAXS> rs;
+      uint32_t *sp = tbl_e + (uint64_t)s * g.stride;
+      rs.load(sp, A, S);
+      for (uint32_t u = b0; u < e1; ++u) {
+        const uint32_t p = sorted[u];
+        rs.touch(opb[p], A);
+        if (opn[p] != NONE) rs.insert0(opn[p], S);
+      }
+      rs.store(sp, A, S);
+    }
+    __syncthreads();
+  }
+
+  if (tid == 0) {
+    ctr_add(a.st, DUM_CTR_EXEC_BUILT, 1);
+    ctr_add(a.st, DUM_CTR_OPS, n_ops);
+    ctr_add(a.st, DUM_CTR_SETS, s_sets);
+  }
+  // ---- Start / End from the latest launch (D11) ----
+  const uint32_t Llast = grp[ng - 1];
+  const uint64_t cbase = a.stage_off[Llast];
+  const uint32_t n = a.stage_cnt[Llast];
+  const uint32_t *C = a.stage_norm + cbase;
+  const uint32_t start = C[0], end = C[n - 1];
+  if (tid == 0) {
+    a.start_end[2 * e] = start;
+    a.start_end[2 * e + 1] = end;
+  }
+  uint32_t *wout = a.walk + (uint64_t)e * g.walk_cap;
+  if (n == 1) {  // x == End: the walk is [Start]
+    if (tid == 0) {
+      wout[0] = start;
+      a.walk_len[e] = 1;
+      ctr_add(a.st, DUM_CTR_WALK_OUT, 1);
+    }
+    return;
+  }
+  __syncthreads();  // table writes of this CTA visible to its own reads below
+
+  // ---- pass A: per chain position i < n-1: row present? stop? successor count ----
+  uint32_t *cq;
+  if (n <= WCAP) {
+    cq = U;
+  } else {
+    unsigned long long need = n;
+    unsigned long long off = 0;
+    if (tid == 0) {
+      off = atomicAdd(&a.st->pool_big, need);
+      s_flag = off + need <= a.big_entries * 2 ? (uint32_t)0 : 1u;
+      s_tev = (uint32_t)off;  // temporarily
+    }
+    __syncthreads();
+    if (s_flag) {
+      if (tid == 0) a.slow_list[atomicAdd(&a.st->n_slow, 1u)] = e;
+      return;
+    }
+    cq = a.big_pool + s_tev;
+    __syncthreads();
+  }
+  if (tid == 0) s_tev = NONE;
+  __syncthreads();
+  for (uint32_t i = tid; i < n - 1; i += BUILD_NT) {
+    const uint32_t x = C[i];
+    const uint32_t *set = tbl_e + (uint64_t)row_of(g, x) * g.stride;
+    int w = -1;
+    for (uint32_t q = 0; q < A; ++q)
+      if (w < 0 && __ldcg(set + q * (1 + S)) == x) w = (int)q;
+    uint32_t ev = 0, cnt = 0;
+    if (w < 0) {
+      ev = 1;  // row missing: stop, nothing emitted at this step
+    } else {
+      const uint32_t *sc = set + w * (1 + S) + 1;
+      bool hit = false;
+      for (uint32_t q = 0; q < S; ++q) {
+        uint32_t v = __ldcg(sc + q);
+        if (v == NONE) break;
+        hit |= v == end;
+        ++cnt;
+      }
+      const uint32_t s0 = cnt ? __ldcg(sc) : NONE;
+      if (hit) ev = 2;                      // a successor is End: stop after emitting
+      else if (s0 != C[i + 1]) ev = 3;      // speculation violated -> sequential walker
+    }
+    cq[i] = cnt;
+    if (ev) atomicMin(&s_tev, (i << 2) | ev);
+  }
+  __syncthreads();
+  const uint32_t tev = s_tev;
+  if (tev == NONE || (tev & 3) == 3) {
+    if (tid == 0) a.slow_list[atomicAdd(&a.st->n_slow, 1u)] = e;
+    return;
+  }
+  const uint32_t t = tev >> 2;
+  if ((tev & 3) == 1 && tid == 0) cq[t] = 0;
+  __syncthreads();
+  // ---- pass B: Q positions (qpos[i] = 1 + sum cq[0..i)) in place ----
+  uint32_t run = 1;
+  for (uint32_t c = 0; c <= t; c += BUILD_NT) {
+    const uint32_t i = c + tid;
+    const uint32_t v = i <= t ? cq[i] : 0;
+    uint32_t tot;
+    const uint32_t pre = block_excl_scan(v, ws, &tot);
+    if (i <= t) cq[i] = run + pre;
+    run += tot;
+  }
+  const uint32_t qlen = run;  // |Q|
+  // dedupe map block -> min Q position
+  uint32_t *qk, *qv;
+  uint32_t qcap = pow2ceil(2 * qlen);
+  if (qcap <= QCAP) {
+    qk = U + WCAP;
+    qv = qk + qcap;
+  } else {
+    if (tid == 0) {
+      unsigned long long off = atomicAdd(&a.st->pool_big, 2ull * qcap);
+      s_flag = off + 2ull * qcap <= a.big_entries * 2 ? 0u : 1u;
+      s_tev = (uint32_t)off;
+    }
+    __syncthreads();
+    if (s_flag) {
+      if (tid == 0) a.slow_list[atomicAdd(&a.st->n_slow, 1u)] = e;
+      return;
+    }
+    qk = a.big_pool + s_tev;
+    qv = qk + qcap;
+  }
+  for (uint32_t p = tid; p < qcap; p += BUILD_NT) {
+    qk[p] = NONE;
+    qv[p] = NONE;
+  }
+  __syncthreads();
+  if (tid == 0) hmap_insert_min(qk, qv, qcap, start, 0);
+  for (uint32_t i = tid; i <= t; i += BUILD_NT) {
+    const uint32_t q0 = cq[i];
+    const uint32_t qn = (i < t ? cq[i + 1] : qlen) - q0;
+    if (qn == 0) continue;
+    const uint32_t x = C[i];
+    const uint32_t *set = tbl_e + (uint64_t)row_of(g, x) * g.stride;
+    uint32_t w = 0;
+    for (uint32_t q = 0; q < A; ++q)
+      if (__ldcg(set + q * (1 + S)) == x) w = q;
+    const uint32_t *sc = set + w * (1 + S) + 1;
+    for (uint32_t q = 0; q < qn; ++q) hmap_insert_min(qk, qv, qcap, __ldcg(sc + q), q0 + q);
+  }
+  __syncthreads();
+  // ---- pass C: ordered compaction of first occurrences ----
+  uint32_t outn = 0;
+  for (uint32_t c = 0; c < qlen; c += BUILD_NT) {
+    const uint32_t p = c + tid;
+    uint32_t val = NONE, keep = 0;
+    if (p < qlen) {
+      if (p == 0) {
+        val = start;
+      } else {
+        uint32_t lo = 0, hi = t + 1;  // cq[lo] <= p < next
+        while (hi - lo > 1) {
+          uint32_t mid = (lo + hi) >> 1;
+          if (cq[mid] <= p) lo = mid;
+          else hi = mid;
+        }
+        const uint32_t x = C[lo];
+        const uint32_t *set = tbl_e + (uint64_t)row_of(g, x) * g.stride;
+        uint32_t w = 0;
+        for (uint32_t q = 0; q < A; ++q)
+          if (__ldcg(set + q * (1 + S)) == x) w = q;
+        val = __ldcg(set + w * (1 + S) + 1 + (p - cq[lo]));
+      }
+      keep = hmap_get(qk, qv, qcap, val) == p;
+    }
+    uint32_t tot;
+    const uint32_t pre = block_excl_scan(keep, ws, &tot);
+    if (keep && outn + pre < g.walk_cap) wout[outn + pre] = val;
+    outn += tot;
+  }
+  if (tid == 0) {
+    if (outn > g.walk_cap) set_err(a.st, ERR_ECAPACITY, outn);
+    a.walk_len[e] = outn;
+    ctr_add(a.st, DUM_CTR_WALK_ROWS, t + 1);
+    ctr_add(a.st, DUM_CTR_WALK_OUT, outn);
+  }
+}
+
+__global__ void k_walk_slow(Geo g, const uint32_t *tbl, const uint32_t *start_end, uint32_t *walk,
+                            uint32_t *walk_len, const uint32_t *slow_list, WalkScratch ws, DevState *st) {
+  const uint32_t nslow = *(volatile uint32_t *)&st->n_slow;
+  for (uint32_t q = blockIdx.x; q < nslow; q += gridDim.x) {
+    const uint32_t e = slow_list[q];
+    const uint32_t *tbl_e = tbl + (uint64_t)e * g.R * g.stride;
+    uint32_t n = walk_seq(g, tbl_e, start_end[2 * e], start_end[2 * e + 1], NONE, walk + (uint64_t)e * g.walk_cap,
+                          g.walk_cap, ws, blockIdx.x);
+    if (threadIdx.x == 0) {
+      if (n == NONE) {
+        set_err(st, ERR_ECAPACITY, g.walk_cap + 1ull);
+        n = 0;
+      }
+      walk_len[e] = n;
+    }
+  }
+}
+
+template <int MA, int MS>
+static cudaError_t launch_apply(dum_engine *e, const BuildArgs &ba, cudaStream_t s) {
+  const size_t smem = (size_t)(2 * GCAP + 1) * 4 +
+                      (size_t)std::max<uint32_t>(2 * ba.g.R + 4 * OPCAP, WCAP + 2 * QCAP) * 4;
+  cudaFuncSetAttribute(k_apply_walk<MA, MS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  k_apply_walk<MA, MS><<<ba.n_staged, BUILD_NT, smem, s>>>(ba);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
+  const uint32_t n = e->n_staged;
+  if (n == 0) return cudaSuccess;
+  {
+  TimerScope t(e, DUM_T_BUILD_PREP, s);
+  k_build_prep<<<(n + 255) / 256, 256, 0, s>>>(n, (uint32_t)e->built_launches, e->d_stage_exec, e->d_stage_cnt,
+                                                e->d_corr, e->corr_cap, e->d_head, e->d_next, e->d_state);
+  }
+  BuildArgs ba;
+  ba.g = e->g;
+  ba.n_staged = n;
+  ba.stage_exec = e->d_stage_exec;
+  ba.stage_cnt = e->d_stage_cnt;
+  ba.stage_norm = e->d_stage_norm;
+  ba.stage_off = e->d_stage_off;
+  ba.head = e->d_head;
+  ba.next = e->d_next;
+  ba.tbl = e->d_tbl;
+  ba.start_end = e->d_start_end;
+  ba.walk = e->d_walk;
+  ba.walk_len = e->d_walk_len;
+  ba.big_pool = e->d_big_pool;
+  ba.big_entries = e->big_pool_entries;
+  ba.slow_list = e->d_slow_list;
+  ba.st = e->d_state;
+  cudaError_t err;
+  {
+  TimerScope t(e, DUM_T_APPLY_WALK, s);
+  if (e->g.A <= 2 && e->g.S <= 4) err = launch_apply<2, 4>(e, ba, s);
+  else if (e->g.A <= 4 && e->g.S <= 8) err = launch_apply<4, 8>(e, ba, s);
+  else err = launch_apply<32, 32>(e, ba, s);
+  }
+  if (err != cudaSuccess) return err;
+  WalkScratch ws{e->d_walk_seen, e->d_walk_chain, e->d_walk_tmp, e->walk_hash_cap,
+                 e->g.walk_cap + e->g.R * e->g.A + 4};
+  TimerScope t(e, DUM_T_WALK_SLOW, s);
+  k_walk_slow<<<e->n_walk_slots, 32, 0, s>>>(e->g, e->d_tbl, e->d_start_end, e->d_walk, e->d_walk_len,
+                                             e->d_slow_list, ws, e->d_state);
+  e->kernel_launches += 3;
+  return cudaGetLastError();
+}
+
+}  // namespace dum

@@ -1,0 +1,180 @@
+// a1 + a2: fault-trace ingest and the execution ID table.
+//
+//  k_ingest        one CTA per launch: first-occurrence dedupe of the launch's
+//                  fault records (PAPER.md L124 step (2): the driver "removes the
+//                  duplicate addresses and groups them according to their UM
+//                  blocks"; reading D2) with an order-preserving block scan, and
+//                  the launch's probe of the execution ID table (PAPER.md:
+//                  "looks up the execution ID table to find the command of the
+//                  same hash value").
+//  k_exec_assign   one CTA: new hashes get dense IDs in first-seen order
+//                  ("Otherwise, it assigns a new execution ID", PAPER.md L136;
+//                  D3) = rank of each new hash by its minimum launch position
+//                  (order-independent).
+#include "device_util.cuh"
+#include "kernels.cuh"
+
+namespace dum {
+
+constexpr int INGEST_NT = 256;
+constexpr uint32_t INGEST_HCAP = 4096;  // smem hash capacity (n <= 2048 in smem)
+
+__global__ void __launch_bounds__(INGEST_NT) k_ingest(
+    const uint64_t *__restrict__ hash, const uint64_t *__restrict__ off, const uint32_t *__restrict__ faults,
+    uint32_t n_launch, uint32_t W, uint32_t l0, uint64_t f0, uint64_t *__restrict__ stage_hash,
+    uint64_t *__restrict__ stage_off, uint32_t *__restrict__ stage_norm, uint32_t *__restrict__ stage_cnt,
+    uint32_t *__restrict__ stage_slot, unsigned long long *exec_keys, uint32_t *exec_vals, uint32_t *exec_minpos,
+    uint32_t exec_cap, uint32_t *big_pool, uint64_t big_entries, DevState *st) {
+  __shared__ uint32_t hk[INGEST_HCAP];
+  __shared__ uint32_t hv[INGEST_HCAP];
+  __shared__ uint32_t ws[INGEST_NT / 32];
+  const uint32_t i = blockIdx.x;
+  if (i >= n_launch) return;
+  const uint64_t a = off[i], b = off[i + 1];
+  const uint32_t n = (uint32_t)(b - a);
+  if (threadIdx.x == 0) {
+    // execution ID table probe (insert if absent)
+    const uint64_t h = hash[i];
+    stage_hash[l0 + i] = h;
+    stage_off[l0 + i] = f0 + a;
+    uint32_t slot = NONE;
+    if (h == EMPTY64) {
+      slot = exec_cap;  // sentinel-key slot; exec_keys[exec_cap] is a presence word
+      atomicCAS(&exec_keys[exec_cap], 0ull, 1ull);
+    } else {
+      uint32_t s = (uint32_t)fmix64(h) & (exec_cap - 1);
+      for (uint32_t p = 0; p < exec_cap; ++p) {
+        unsigned long long old = atomicCAS(&exec_keys[s], EMPTY64, (unsigned long long)h);
+        if (old == EMPTY64 || old == h) {
+          slot = s;
+          break;
+        }
+        s = (s + 1) & (exec_cap - 1);
+      }
+    }
+    if (slot == NONE) {
+      set_err(st, ERR_ECAPACITY, 2ull * exec_cap);
+    } else if (((volatile uint32_t *)exec_vals)[slot] == PENDING) {
+      atomicMin(&exec_minpos[slot], i);
+    }
+    stage_slot[l0 + i] = slot;
+  }
+  if (threadIdx.x == 0) ctr_add(st, DUM_CTR_LAUNCHES, 1);
+  if (n == 0) {
+    if (threadIdx.x == 0) stage_cnt[l0 + i] = 0;
+    return;
+  }
+  // hash of (block -> first position) in shared memory, or in a private
+  // region of the global pool for launches with > INGEST_HCAP/2 records
+  uint32_t *keys = hk, *vals = hv;
+  uint32_t cap = INGEST_HCAP;
+  if (n > INGEST_HCAP / 2) {
+    cap = pow2ceil(2 * n);
+    uint64_t base = 4ull * (f0 + a);  // region [4(f0+a), 4(f0+b)) holds >= cap entries
+    if (2ull * (base + cap) > 2ull * big_entries) {
+      if (threadIdx.x == 0) set_err(st, ERR_ECAPACITY, base + cap);
+      return;
+    }
+    keys = big_pool + 2ull * base;
+    vals = keys + cap;
+  }
+  for (uint32_t t = threadIdx.x; t < cap; t += INGEST_NT) {
+    keys[t] = NONE;
+    vals[t] = NONE;
+  }
+  __syncthreads();
+  for (uint32_t j = threadIdx.x; j < n; j += INGEST_NT) {
+    uint32_t blk = faults[a + j];
+    if (blk >= W) {
+      set_err(st, ERR_EINVAL);
+      continue;
+    }
+    hmap_insert_min(keys, vals, cap, blk, j);
+  }
+  __syncthreads();
+  // order-preserving compaction of first occurrences
+  uint32_t run = 0;
+  for (uint32_t c = 0; c < n; c += INGEST_NT) {
+    const uint32_t j = c + threadIdx.x;
+    uint32_t blk = NONE, keep = 0;
+    if (j < n) {
+      blk = faults[a + j];
+      keep = blk < W && hmap_get(keys, vals, cap, blk) == j;
+    }
+    uint32_t tot;
+    uint32_t pre = block_excl_scan(keep, ws, &tot);
+    if (keep) stage_norm[f0 + a + run + pre] = blk;
+    run += tot;
+  }
+  if (threadIdx.x == 0) {
+    stage_cnt[l0 + i] = run;
+    ctr_add(st, DUM_CTR_RAW_RECORDS, n);
+    ctr_add(st, DUM_CTR_NORM_RECORDS, run);
+  }
+}
+
+constexpr int ASSIGN_NT = 1024;
+
+__global__ void __launch_bounds__(ASSIGN_NT) k_exec_assign(
+    uint32_t n_launch, uint32_t l0, const uint32_t *__restrict__ stage_slot, const uint64_t *__restrict__ stage_hash,
+    uint32_t *exec_vals, uint32_t *exec_minpos, uint64_t *exec_hash, uint32_t *__restrict__ stage_exec,
+    uint32_t *__restrict__ out_exec, uint32_t Emax, DevState *st) {
+  __shared__ uint32_t ws[ASSIGN_NT / 32];
+  const uint32_t E0 = st->E;
+  uint32_t base = 0;
+  for (uint32_t c = 0; c < n_launch; c += ASSIGN_NT) {
+    const uint32_t i = c + threadIdx.x;
+    uint32_t flag = 0, slot = NONE;
+    if (i < n_launch) {
+      slot = stage_slot[l0 + i];
+      if (slot != NONE)
+        flag = ((volatile uint32_t *)exec_vals)[slot] == PENDING &&
+               ((volatile uint32_t *)exec_minpos)[slot] == i;
+    }
+    uint32_t tot;
+    uint32_t pre = block_excl_scan(flag, ws, &tot);
+    if (flag) {
+      uint32_t id = E0 + base + pre;
+      exec_vals[slot] = id;
+      exec_minpos[slot] = NONE;
+      if (id < Emax) exec_hash[id] = stage_hash[l0 + i];
+    }
+    base += tot;
+  }
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < n_launch; i += ASSIGN_NT) {
+    uint32_t slot = stage_slot[l0 + i];
+    uint32_t id = slot == NONE ? NONE : ((volatile uint32_t *)exec_vals)[slot];
+    if (id != NONE && id >= Emax) id = NONE;
+    stage_exec[l0 + i] = id;
+    if (out_exec) out_exec[i] = id;
+  }
+  if (threadIdx.x == 0) {
+    uint32_t E = E0 + base;
+    if (E > Emax) {
+      set_err(st, ERR_ECAPACITY, E);
+      E = Emax;
+    }
+    st->E = E;
+  }
+}
+
+cudaError_t launch_record(dum_engine *e, const uint64_t *hash, const uint64_t *off, uint32_t n_launch,
+                          const uint32_t *faults, uint32_t *out_exec, cudaStream_t s) {
+  if (n_launch == 0) return cudaSuccess;
+  {
+  TimerScope t(e, DUM_T_INGEST, s);
+  k_ingest<<<n_launch, INGEST_NT, 0, s>>>(hash, off, faults, n_launch, e->g.W, e->n_staged, e->staged_faults,
+                                          e->d_stage_hash, e->d_stage_off, e->d_stage_norm, e->d_stage_cnt,
+                                          e->d_stage_slot, e->d_exec_keys, e->d_exec_vals, e->d_exec_minpos,
+                                          e->exec_cap, e->d_big_pool, e->big_pool_entries, e->d_state);
+  }
+  TimerScope t(e, DUM_T_EXEC_ASSIGN, s);
+  k_exec_assign<<<1, ASSIGN_NT, 0, s>>>(n_launch, e->n_staged, e->d_stage_slot, e->d_stage_hash, e->d_exec_vals,
+                                        e->d_exec_minpos, e->d_exec_hash, e->d_stage_exec, out_exec, e->g.Emax,
+                                        e->d_state);
+  e->kernel_launches += 2;
+  return cudaGetLastError();
+}
+
+}  // namespace dum

@@ -1,0 +1,211 @@
+"""GPU parity: the CUDA engine (through the C-ABI) against the CPU oracle on
+the same seeded inputs.  Integer state -> bit-exact comparisons of canonical
+dumps, per-query prefetch lists and eviction sets."""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+import torch
+
+pytestmark = pytest.mark.gpu
+
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("needs a GPU", allow_module_level=True)
+
+import oracle as orc  # noqa: E402
+import workloads as wl  # noqa: E402
+from gpu_helpers import (ALL_TABLES, NONE, assert_same_predictions, assert_same_state, build_both,  # noqa: E402
+                         dev, make_pair, predict_both, record_both, select_both, transition_queries)
+from paper_conf_asplos_jungkl23_b200 import binding as B  # noqa: E402
+
+TABLE6 = {  # PAPER.md Table 6 (L429-L443): name -> (Assoc, NumSuccs, NumRows)
+    "Config0": (2, 4, 128), "Config1": (2, 8, 128), "Config2": (4, 4, 128), "Config3": (2, 4, 512),
+    "Config4": (2, 8, 512), "Config5": (4, 4, 512), "Config6": (2, 4, 1024), "Config7": (2, 8, 1024),
+    "Config8": (4, 4, 1024), "Config9": (2, 4, 2048), "Config10": (2, 8, 2048), "Config11": (4, 4, 2048),
+    "Config12": (2, 4, 4096),
+}
+
+
+def _run_trace_per_iteration(eng, o, tr, N, check_every=True, host_ptrs=False, queries=True, select=True):
+    """Bench schedule per iteration i: record(i) -> predict(i) on
+    the state built through i-1 -> select -> build(i)."""
+    ex_all = []
+    for i in range(tr.n_iter):
+        h, off, f = tr.iteration(i)
+        exo, exg = record_both(eng, o, h, off, f, host_ptrs=host_ptrs)
+        assert np.array_equal(exo, exg), "exec ids iteration %d" % i
+        ex_all += [int(x) for x in exo]
+        if queries and i >= 1:
+            qs = transition_queries(ex_all, i * tr.K, tr.K, N)
+            ro, rg, (gp, grng, qd) = predict_both(eng, o, qs)
+            assert_same_predictions(ro, rg, msg="iteration %d" % i)
+            if select:
+                select_both(eng, o, gp, grng, qd, qs, ro)
+        build_both(eng, o)
+        if check_every:
+            assert_same_state(eng, o, msg="iteration %d" % i)
+    return ex_all
+
+
+def test_config_T_all_calls_parity():
+    tr = wl.make_T()
+    eng, o = make_pair(W=tr.W, C=tr.C, N=32)
+    # a residency snapshot for select: the generator's LRM snapshot at iteration 5
+    snap = tr.snap_blk[5][: int(tr.snap_cnt[5])]
+    o.load_residency(snap)
+    eng.load_residency(dev(snap))
+    _run_trace_per_iteration(eng, o, tr, N=32)
+    assert_same_state(eng, o, what=ALL_TABLES | orc.RES)
+
+
+@pytest.mark.parametrize("N", [0, 1, 2, 4])
+def test_config_T_degrees(N):
+    tr = wl.make_T()
+    eng, o = make_pair(W=tr.W, C=tr.C, N=max(N, 1))
+    _run_trace_per_iteration(eng, o, tr, N=N, check_every=False, select=False)
+    assert_same_state(eng, o)
+
+
+@pytest.mark.parametrize("name", sorted(TABLE6))
+def test_table6_geometries_on_T(name):
+    A, S, R = TABLE6[name]
+    tr = wl.make_T(dup_ppm=200_000)
+    eng, o = make_pair(R=R, A=A, S=S, W=tr.W, C=tr.C, N=8)
+    _run_trace_per_iteration(eng, o, tr, N=8, check_every=False, select=False)
+    assert_same_state(eng, o)
+
+
+@pytest.mark.parametrize("geom", [(16, 1, 1), (16, 2, 4), (16, 1, 4), (16, 2, 1), (1, 3, 2), (1, 1, 1),
+                                  (4, 4, 8), (8, 5, 3), (2048, 2, 4)])
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_random_traces_stress_geometries(geom, seed):
+    """Replacement pressure, duplicates, empty launches, repeated exec IDs in one
+    batch, several record calls per build, fault-anchored queries."""
+    R, A, S = geom
+    rng = np.random.default_rng(1000 * seed + R + 7 * A + 13 * S)
+    W = 300
+    eng, o = make_pair(R=R, A=A, S=S, W=W, C=40, N=6)
+    ex_all = []
+    for batch in range(6):
+        n_rec = int(rng.integers(1, 4))
+        for _ in range(n_rec):
+            h, off, f = wl.random_trace(rng, n_launch=int(rng.integers(1, 40)), n_kernels=6, W=W, max_faults=80)
+            exo, exg = record_both(eng, o, h, off, f, host_ptrs=bool(rng.integers(0, 2)))
+            assert np.array_equal(exo, exg)
+            ex_all += [int(x) for x in exo]
+        build_both(eng, o)
+        assert_same_state(eng, o, msg="batch %d" % batch)
+        qs = transition_queries(ex_all, 0, len(ex_all), 6)
+        # mix in fault-anchored queries (anchor = a random block) and n < N
+        anch = qs.copy()
+        anch[:, 4] = rng.integers(0, W, len(anch))
+        anch[:, 5] = rng.integers(0, 7, len(anch))
+        allq = np.concatenate([qs, anch])
+        ro, rg, (gp, grng, qd) = predict_both(eng, o, allq)
+        assert_same_predictions(ro, rg, msg="batch %d" % batch)
+        n_res = int(rng.integers(0, 41))
+        snap = rng.permutation(W)[:n_res].astype(np.uint32)
+        o.load_residency(snap)
+        eng.load_residency(dev(snap))
+        inact = rng.permutation(W)[: W // 4].astype(np.uint32)
+        o.mark_inactive(inact, True)
+        eng.mark_inactive(dev(inact), True)
+        select_both(eng, o, gp, grng, qd, allq, ro)
+
+
+def test_block_ids_near_limit_and_fmix_index():
+    W = 1 << 20
+    rng = np.random.default_rng(5)
+    eng, o = make_pair(R=64, A=2, S=4, W=W, C=16, N=4, row_index=1)
+    hi = np.arange(W - 200, W, dtype=np.uint32)
+    lists = [list(rng.choice(hi, 30)) for _ in range(20)]
+    h = np.array([wl.fnv1a64(b"k%d" % (i % 5)) for i in range(20)], dtype=np.uint64)
+    off = np.zeros(21, dtype=np.uint64)
+    off[1:] = np.cumsum([len(x) for x in lists])
+    f = np.array([b for x in lists for b in x], dtype=np.uint32)
+    exo, exg = record_both(eng, o, h, off, f)
+    assert np.array_equal(exo, exg)
+    build_both(eng, o)
+    assert_same_state(eng, o)
+    qs = transition_queries([int(x) for x in exo], 0, 20, 4)
+    ro, rg, _ = predict_both(eng, o, qs)
+    assert_same_predictions(ro, rg)
+
+
+def test_hash_sentinel_and_collisions():
+    """Two launches with the same hash share an ID; the all-ones hash is a
+    legal key (D3)."""
+    eng, o = make_pair(W=64, C=8, N=2)
+    h = np.array([0xFFFFFFFFFFFFFFFF, 7, 0xFFFFFFFFFFFFFFFF, 7, 0, 0], dtype=np.uint64)
+    off = np.array([0, 2, 2, 5, 6, 6, 8], dtype=np.uint64)
+    f = np.array([1, 2, 3, 4, 3, 9, 1, 1], dtype=np.uint32)
+    exo, exg = record_both(eng, o, h, off, f)
+    assert list(exo) == [0, 1, 0, 1, 2, 2] and np.array_equal(exo, exg)
+    build_both(eng, o)
+    assert_same_state(eng, o)
+
+
+@pytest.mark.parametrize("config", ["B", "G"])
+def test_full_size_tables_and_sampled_predictions(config):
+    """BASELINE.json configs[1] / configs[2] at full size (3 iterations): the
+    complete table state is compared byte for byte; predictions and selections
+    on a seeded sample of queries in the bench's launch configuration."""
+    tr = wl.make(config, n_iter=3)
+    eng, o = make_pair(W=tr.W, C=tr.C, N=32, Emax=8192)
+    ex_all = []
+    for i in range(tr.n_iter):
+        h, off, f = tr.iteration(i)
+        exo, exg = record_both(eng, o, h, off, f)
+        assert np.array_equal(exo, exg)
+        ex_all += [int(x) for x in exo]
+        build_both(eng, o)
+    st = eng.stats()
+    assert st.slow_walks == 0
+    assert_same_state(eng, o)
+    rng = np.random.default_rng(11)
+    pick = np.sort(rng.choice(np.arange(2 * tr.K, 3 * tr.K), 64, replace=False))
+    allq = transition_queries(ex_all, 0, len(ex_all), 32)[pick]
+    ro, rg, (gp, grng, qd) = predict_both(eng, o, allq)
+    assert_same_predictions(ro, rg)
+    snap = tr.snap_blk[2][: int(tr.snap_cnt[2])]
+    o.load_residency(snap)
+    eng.load_residency(dev(snap))
+    o.mark_inactive(tr.inactive_blocks, True)
+    eng.mark_inactive(dev(tr.inactive_blocks), True)
+    select_both(eng, o, gp, grng, qd, allq, ro)
+
+
+def test_full_batch_of_ten_iterations_in_one_build():
+    """Config T recorded as one 40-launch batch, built once (multi-launch groups
+    per exec ID inside one build)."""
+    tr = wl.make_T(dup_ppm=300_000)
+    eng, o = make_pair(W=tr.W, C=tr.C, N=32)
+    exo, exg = record_both(eng, o, tr.launch_hash, tr.launch_off, tr.fault_block)
+    assert np.array_equal(exo, exg)
+    build_both(eng, o)
+    assert_same_state(eng, o)
+
+
+def test_errors_are_reported():
+    eng, o = make_pair(W=64, C=8, N=2)
+    with pytest.raises(B.EngineError):
+        eng.record_faults(np.array([1], np.uint64), np.array([0, 1], np.uint64), np.array([64], np.uint32))
+    # device-side detection of an out-of-range block id
+    eng.record_faults(dev(np.array([1], np.uint64), np.uint64), dev(np.array([0, 1], np.uint64), np.uint64),
+                      dev(np.array([99], np.uint32)))
+    with pytest.raises(B.EngineError):
+        eng.sync()
+    eng.build_tables()
+    eng.sync()
+    # predict capacity too small -> ECAPACITY with the needed size
+    eng2, o2 = make_pair(W=64, C=8, N=2)
+    h = np.array([5, 6, 5, 6, 5, 6], np.uint64)
+    off = np.array([0, 3, 6, 9, 12, 15, 18], np.uint64)
+    f = np.arange(18, dtype=np.uint32) % 12
+    record_both(eng2, o2, h, off, f)
+    build_both(eng2, o2)
+    q = dev(transition_queries([0, 1, 0, 1, 0, 1], 3, 3, 2).reshape(-1)).reshape(-1, 6)
+    eng2.predict_prefetch(q, 1)
+    with pytest.raises(B.EngineError) as ei:
+        eng2.sync()
+    assert getattr(ei.value, "needed", 0) > 1
