@@ -70,10 +70,17 @@ class Clocks:
         self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
         try:
             self.p = subprocess.Popen(["nvidia-smi", "-i", str(gpu), "--query-gpu=" + self.FIELDS,
-                                       "--format=csv,noheader,nounits", "-lms", "200"], stdout=self.f,
+                                       "--format=csv,noheader,nounits", "-lms", "100"], stdout=self.f,
                                       stderr=subprocess.DEVNULL)
         except Exception:
             self.p = None
+        # wait (<= 5 s) until the sampler produces output so the window covers the run
+        t0 = time.time()
+        while self.p is not None and time.time() - t0 < 5:
+            self.f.flush()
+            if os.path.getsize(self.f.name) > 0:
+                break
+            time.sleep(0.05)
 
     def stop(self):
         if self.p is None:
@@ -100,7 +107,8 @@ class Clocks:
                 if r[4 + k].lower() == "active":
                     reasons.add(nm)
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(rows)}
+                "reasons": sorted(reasons), "samples": len(rows),
+                "window": "nvidia-smi -lms 100 from the start of warm-up to the end of the timed steps"}
 
 
 # ---------------------------------------------------------------------------
@@ -283,6 +291,7 @@ def run_ours(args, rank, world, local_rank):
     # (predict and select never modify tables, so an overflow in warm-up only
     # invalidates that step's lists)
     grow(4 << 20)
+    clk = Clocks(local_rank) if rank == 0 else None
     for i in range(1, 1 + args.warmup):
         pre_step(i)
         step(i)
@@ -302,7 +311,6 @@ def run_ours(args, rank, world, local_rank):
     eng.read_timing(reset=True)
     eng.set_timing(True)
     launches0 = eng.kernel_launches
-    clk = Clocks(local_rank) if rank == 0 else None
     stream = torch.cuda.current_stream(dev)
     evs = []
     records = 0
