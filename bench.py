@@ -55,6 +55,7 @@ def parse():
     ap.add_argument("--no-migration", action="store_true")
     ap.add_argument("--cpu-launches", type=int, default=0, help="oracle sample size in launches")
     ap.add_argument("--json-out", default="")
+    ap.add_argument("--unfused", action="store_true", help="separate predict / select calls")
     return ap.parse_args()
 
 
@@ -114,20 +115,25 @@ class Clocks:
 # ---------------------------------------------------------------------------
 # algorithmic bytes per kernel
 # ---------------------------------------------------------------------------
-def algorithmic_bytes(ctr, geo, N):
+def algorithmic_bytes(ctr, geo, N, fused=True):
+    """Bytes each kernel must move at minimum for the work it did (counters
+    from the engine).  DESIGN.md "Roofline accounting" states every term."""
     from paper_conf_asplos_jungkl23_b200.binding import CTR
     c = {k: int(ctr[v]) for k, v in CTR.items()}
     set_bytes = 4 * geo["A"] * (1 + geo["S"])
+    predict = (24 * c["QUERIES"] + 32 * c["CHAIN"] + 4 * c["GATHERED"] + 8 * c["EMITTED"]
+               + c["QUERIES"] * (16 + 4 * (N + 2) + 4 * (N + 1)))
+    select_core = 4 * c["SEL_SCANNED"] + 4 * c["SEL_VICTIMS"] + 32 * c["QUERIES"]
+    if fused:  # window set reused from predict: residency lookups per emitted pair
+        predict += 4 * c["EMITTED"] + select_core
     return {
         "k_ingest": 4 * c["RAW_RECORDS"] + 4 * c["NORM_RECORDS"] + 28 * c["LAUNCHES"],
         "k_exec_assign": 16 * c["LAUNCHES"],
         "k_build_prep": 8 * c["LAUNCHES"] + 2 * 32 * c["CORR_UPSERTS"],
         "k_apply_walk": (4 * c["OPS"] + 2 * set_bytes * c["SETS"] + set_bytes * c["WALK_ROWS"]
                          + 4 * c["WALK_OUT"] + 16 * c["EXEC_BUILT"]),
-        "k_predict": (24 * c["QUERIES"] + 32 * c["CHAIN"] + 4 * c["GATHERED"] + 8 * c["EMITTED"]
-                      + c["QUERIES"] * (16 + 4 * (N + 2) + 4 * (N + 1))),
-        "k_select": (8 * c["SEL_WINDOW"] + 4 * c["SEL_WINDOW"] + 12 * c["SEL_SCANNED"] + 4 * c["SEL_VICTIMS"]
-                     + 48 * c["QUERIES"]),
+        "k_predict": predict,
+        "k_select": 8 * c["SEL_WINDOW"] + 4 * c["SEL_WINDOW"] + select_core,
     }
 
 
@@ -273,8 +279,13 @@ def run_ours(args, rank, world, local_rank):
             eng.record_faults(host[0][i], host[1][i], host[2][i], out_exec)
         if i >= 1:
             eng.make_queries(exec_all[i * K: 3 + (i + 1) * K], 3, N, out=qbuf)
-            eng.predict_prefetch(qbuf, cap[0], pairs=pairs[0], rng=rng, kern_off=ko, chain=ch, needed=need_p)
-            eng.select_evictions(rng, pairs[0], qbuf, cap[0], wb=wb[0], inv=inv[0], out_rng=srng, needed=need_s)
+            if args.unfused:
+                eng.predict_prefetch(qbuf, cap[0], pairs=pairs[0], rng=rng, kern_off=ko, chain=ch, needed=need_p)
+                eng.select_evictions(rng, pairs[0], qbuf, cap[0], wb=wb[0], inv=inv[0], out_rng=srng,
+                                     needed=need_s)
+            else:
+                eng.predict_select(qbuf, cap[0], cap[0], pairs=pairs[0], rng=rng, kern_off=ko, chain=ch,
+                                   needed=need_p, wb=wb[0], inv=inv[0], sel_rng=srng, sel_needed=need_s)
         eng.build_tables()
 
     def pre_step(i):
@@ -351,7 +362,7 @@ def run_ours(args, rank, world, local_rank):
 
     # ---- roofline of the dominant kernel ----
     peak, peak_src = load_peaks()
-    abytes = algorithmic_bytes(ctr, geo, N)
+    abytes = algorithmic_bytes(ctr, geo, N, fused=not args.unfused)
     per_kernel = {}
     for name, idx in B.TIMER.items():
         if kcnt[idx]:

@@ -188,6 +188,16 @@ int dum_select_evictions(dum_engine *eng, const uint64_t *query_range, const uin
                          uint32_t *out_invalidate, uint64_t out_cap, uint64_t *out_range,
                          uint64_t *out_needed, dum_stream_t stream);
 
+/* ---- a7 + a8 fused ------------------------------------------------------
+ * dum_predict_prefetch followed by dum_select_evictions on the same windows,
+ * in one kernel: the window set built for the prefetch list is reused for the
+ * victim search instead of being re-read from HBM.  Outputs and semantics are
+ * exactly those of the two calls (same arguments, same layouts). */
+int dum_predict_select(dum_engine *eng, const dum_query *queries, uint32_t n_query, uint32_t *out_pairs,
+                       uint64_t out_cap_pairs, uint64_t *out_range, uint32_t *out_kern_off, uint32_t *out_chain,
+                       uint64_t *out_needed, uint32_t *out_writeback, uint32_t *out_invalidate, uint64_t sel_cap,
+                       uint64_t *sel_range, uint64_t *sel_needed, dum_stream_t stream);
+
 /* Mark UM blocks as belonging to inactive (inactive != 0) or active PyTorch
  * blocks (D20: a block is invalidatable iff every PT block overlapping
  * it is inactive -- the caller resolves overlap). */

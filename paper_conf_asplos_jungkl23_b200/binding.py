@@ -82,6 +82,7 @@ def load_library() -> ctypes.CDLL:
         "dum_make_queries": (I, [P, P, U32, U32, U32, P, P]),
         "dum_predict_prefetch": (I, [P, P, U32, P, U64, P, P, P, P, P]),
         "dum_select_evictions": (I, [P, P, P, U32, P, P, P, U64, P, P, P]),
+        "dum_predict_select": (I, [P, P, U32, P, U64, P, P, P, P, P, P, U64, P, P, P]),
         "dum_mark_inactive": (I, [P, P, U32, I, P]),
         "dum_load_residency": (I, [P, P, U32, P]),
         "dum_migrate_blocks": (I, [P, I, P, P, U32, U32, P]),
@@ -249,6 +250,37 @@ class Engine:
                                                _dev(wb, 4), _dev(inv, 4), cap, _dev(out_rng, 8), _dev(needed, 8),
                                                self._stream()), "dum_select_evictions")
         return wb, inv, out_rng, needed
+
+    def predict_select(self, queries: torch.Tensor, cap: int, sel_cap: Optional[int] = None, pairs=None, rng=None,
+                       kern_off=None, chain=None, needed=None, wb=None, inv=None, sel_rng=None, sel_needed=None,
+                       want_kern_off: bool = True, want_chain: bool = True):
+        """Fused a7 + a8 (dum_predict_select)."""
+        nq = queries.shape[0]
+        sel_cap = cap if sel_cap is None else sel_cap
+        d = self.device
+        if pairs is None:
+            pairs = torch.empty((max(cap, 1), 2), dtype=torch.int32, device=d)
+        if rng is None:
+            rng = torch.empty((nq, 2), dtype=torch.int64, device=d)
+        if kern_off is None and want_kern_off:
+            kern_off = torch.empty((nq, self.N + 2), dtype=torch.int32, device=d)
+        if chain is None and want_chain:
+            chain = torch.empty((nq, self.N + 1), dtype=torch.int32, device=d)
+        if needed is None:
+            needed = torch.zeros(1, dtype=torch.int64, device=d)
+        if wb is None:
+            wb = torch.empty(max(sel_cap, 1), dtype=torch.int32, device=d)
+        if inv is None:
+            inv = torch.empty(max(sel_cap, 1), dtype=torch.int32, device=d)
+        if sel_rng is None:
+            sel_rng = torch.empty((nq, 4), dtype=torch.int64, device=d)
+        if sel_needed is None:
+            sel_needed = torch.zeros(1, dtype=torch.int64, device=d)
+        self._ck(self.lib.dum_predict_select(self._h, _dev(queries, 4), nq, _dev(pairs, 4), cap, _dev(rng, 8),
+                                             _dev(kern_off, 4), _dev(chain, 4), _dev(needed, 8), _dev(wb, 4),
+                                             _dev(inv, 4), sel_cap, _dev(sel_rng, 8), _dev(sel_needed, 8),
+                                             self._stream()), "dum_predict_select")
+        return pairs, rng, kern_off, chain, needed, wb, inv, sel_rng, sel_needed
 
     def mark_inactive(self, blocks: torch.Tensor, inactive: bool = True):
         self._ck(self.lib.dum_mark_inactive(self._h, _dev(blocks, 4), blocks.numel(), 1 if inactive else 0,

@@ -12,6 +12,7 @@
 
 #include "device_util.cuh"
 #include "kernels.cuh"
+#include "select_tail.cuh"
 
 using namespace dum;
 
@@ -374,7 +375,23 @@ int dum_predict_prefetch(dum_engine *e, const dum_query *q, uint32_t n_query, ui
   if (reinterpret_cast<uintptr_t>(out_pairs) & 7) return fail(e, DUM_EINVAL, "out_pairs must be 8-byte aligned");
   cudaSetDevice(e->device);
   CK(launch_predict(e, q, n_query, out_pairs, out_cap_pairs, out_range, out_kern_off, out_chain, out_needed,
-                    (cudaStream_t)stream));
+                    nullptr, nullptr, (cudaStream_t)stream));
+  return DUM_OK;
+}
+
+int dum_predict_select(dum_engine *e, const dum_query *q, uint32_t n_query, uint32_t *out_pairs,
+                       uint64_t out_cap_pairs, uint64_t *out_range, uint32_t *out_kern_off, uint32_t *out_chain,
+                       uint64_t *out_needed, uint32_t *out_writeback, uint32_t *out_invalidate, uint64_t sel_cap,
+                       uint64_t *sel_range, uint64_t *sel_needed, dum_stream_t stream) {
+  if (!e) return DUM_EINVAL;
+  if (n_query == 0) return DUM_OK;
+  if (!q || !out_range || !sel_range || (!out_pairs && out_cap_pairs)) return fail(e, DUM_EINVAL, "null argument");
+  if (n_query > e->anchor_range_cap) return fail(e, DUM_EINVAL, "too many queries in one call (max 2^20)");
+  if (reinterpret_cast<uintptr_t>(out_pairs) & 7) return fail(e, DUM_EINVAL, "out_pairs must be 8-byte aligned");
+  cudaSetDevice(e->device);
+  SelectOut so = make_select_out(e, out_writeback, out_invalidate, sel_cap, sel_range);
+  CK(launch_predict(e, q, n_query, out_pairs, out_cap_pairs, out_range, out_kern_off, out_chain, out_needed, &so,
+                    sel_needed, (cudaStream_t)stream));
   return DUM_OK;
 }
 

@@ -59,7 +59,7 @@ struct DevState {
   uint32_t corr_used;
   uint32_t mig_ok;            // last migrate validated
   uint32_t mig_n;             // blocks moved by the last migrate
-  uint32_t pad;
+  uint32_t log_dirty;         // LRM log may hold entries of evicted blocks
   unsigned long long ctr[DUM_NCOUNTERS];  // work counters (instrumentation)
 };
 

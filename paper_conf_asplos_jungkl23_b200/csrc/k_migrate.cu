@@ -43,6 +43,7 @@ __global__ void k_res_reset(uint32_t W, uint32_t C, uint32_t *frame_of, uint32_t
     for (uint32_t w = t; w < (W + 31) / 32; w += nt) inactive[w] = 0;
   if (t == 0) {
     st->lrm_head = st->lrm_tail = 0;
+    st->log_dirty = 0;
     st->free_count = C;
     st->mig_counter = 0;
     st->n_resident = 0;
@@ -176,6 +177,7 @@ __global__ void __launch_bounds__(PLAN_NT) k_mig_plan(MigArgs a) {
       }
       head = 0;
       tail = outp;
+      if (tid == 0) st->log_dirty = 0;
       if (tail + n > a.lrm_cap) {
         if (tid == 0) set_err(st, ERR_ECAPACITY, tail + n);
         for (uint32_t i = tid; i < n; i += PLAN_NT) a.frame_of[a.blocks[i]] = NONE;
@@ -226,6 +228,7 @@ __global__ void __launch_bounds__(PLAN_NT) k_mig_plan(MigArgs a) {
     if (tid == 0) {
       st->free_count += n;
       st->n_resident -= n;
+      st->log_dirty = 1;
     }
   } else if (a.dir == DUM_D2D && a.blocks != nullptr) {
     for (uint32_t i = tid; i < n; i += PLAN_NT) {

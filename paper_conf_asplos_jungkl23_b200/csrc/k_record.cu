@@ -67,7 +67,8 @@ __global__ void __launch_bounds__(INGEST_NT) k_ingest(
   // hash of (block -> first position) in shared memory, or in a private
   // region of the global pool for launches with > INGEST_HCAP/2 records
   uint32_t *keys = hk, *vals = hv;
-  uint32_t cap = INGEST_HCAP;
+  uint32_t cap = pow2ceil(2 * n);
+  if (cap < 64) cap = 64;
   if (n > INGEST_HCAP / 2) {
     cap = pow2ceil(2 * n);
     uint64_t base = 4ull * (f0 + a);  // region [4(f0+a), 4(f0+b)) holds >= cap entries

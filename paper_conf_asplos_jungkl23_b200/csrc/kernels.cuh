@@ -12,9 +12,10 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s);
 // k_predict.cu (a6 + a7)
 cudaError_t launch_make_queries(dum_engine *e, const uint32_t *exec_seq, uint32_t n_seq, uint32_t first,
                                 uint32_t degree, dum_query *out, cudaStream_t s);
+struct SelectOut;
 cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint32_t *pairs, uint64_t cap,
                            uint64_t *range, uint32_t *kern_off, uint32_t *chain, uint64_t *needed,
-                           cudaStream_t s);
+                           const SelectOut *sel, uint64_t *sel_needed, cudaStream_t s);
 // k_select.cu  (a8)
 cudaError_t launch_select(dum_engine *e, const uint64_t *range, const uint32_t *pairs, uint32_t nq,
                           const dum_query *q, uint32_t *wb, uint32_t *inv, uint64_t cap, uint64_t *out_range,

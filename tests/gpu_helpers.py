@@ -126,6 +126,38 @@ def select_both(eng: Engine, o: orc.Oracle, gp, grng, qd, queries: np.ndarray, r
     return wb, iv
 
 
+def fused_both(eng: Engine, o: orc.Oracle, queries: np.ndarray):
+    """dum_predict_select (fused a7+a8) vs the oracle's predict then select."""
+    q = np.ascontiguousarray(queries, dtype=np.uint32).reshape(-1, 6)
+    off, pairs, ko, ch = o.predict(q)
+    wo, wb, io, iv = o.select(off, pairs, q[:, 4])
+    qd = dev(q.reshape(-1)).reshape(-1, 6)
+    cap = int(off[-1]) + 16
+    while True:
+        out = eng.predict_select(qd, cap, sel_cap=cap)
+        try:
+            eng.sync()
+            break
+        except B.EngineError as e:
+            assert e.code == -2 and e.needed > cap, e
+            cap = int(e.needed)
+    gp, grng, gko, gch, _, gwb, ginv, gsr, _ = out
+    gp = B.u32(gp).reshape(-1, 2)
+    grng = B.u64(grng).reshape(-1, 2)
+    gko = B.u32(gko).reshape(len(q), -1)
+    gch = B.u32(gch).reshape(len(q), -1)
+    gwb, ginv, r = B.u32(gwb), B.u32(ginv), B.u64(gsr).reshape(-1, 4)
+    for i in range(len(q)):
+        po = pairs[int(off[i]):int(off[i + 1])]
+        pg = gp[int(grng[i, 0]):int(grng[i, 1])]
+        assert np.array_equal(po, pg) and np.array_equal(ko[i], gko[i]) and np.array_equal(ch[i], gch[i]), \
+            "fused predict query %d: n gpu=%d orc=%d" % (i, len(pg), len(po))
+        ew, ei = wb[int(wo[i]):int(wo[i + 1])], iv[int(io[i]):int(io[i + 1])]
+        aw, ai = gwb[int(r[i, 0]):int(r[i, 1])], ginv[int(r[i, 2]):int(r[i, 3])]
+        assert np.array_equal(ew, aw) and np.array_equal(ei, ai), \
+            "fused select query %d: wb gpu=%d orc=%d inv gpu=%d orc=%d" % (i, len(aw), len(ew), len(ai), len(ei))
+
+
 def transition_queries(exec_seq: List[int], first: int, n: int, N: int) -> np.ndarray:
     pad = [NONE, NONE, NONE] + list(exec_seq)
     qs = []

@@ -15,7 +15,7 @@ if not torch.cuda.is_available():  # pragma: no cover
 import oracle as orc  # noqa: E402
 import workloads as wl  # noqa: E402
 from gpu_helpers import (ALL_TABLES, NONE, assert_same_predictions, assert_same_state, build_both,  # noqa: E402
-                         dev, make_pair, predict_both, record_both, select_both, transition_queries)
+                         dev, fused_both, make_pair, predict_both, record_both, select_both, transition_queries)
 from paper_conf_asplos_jungkl23_b200 import binding as B  # noqa: E402
 
 TABLE6 = {  # PAPER.md Table 6 (L429-L443): name -> (Assoc, NumSuccs, NumRows)
@@ -41,6 +41,7 @@ def _run_trace_per_iteration(eng, o, tr, N, check_every=True, host_ptrs=False, q
             assert_same_predictions(ro, rg, msg="iteration %d" % i)
             if select:
                 select_both(eng, o, gp, grng, qd, qs, ro)
+                fused_both(eng, o, qs)
         build_both(eng, o)
         if check_every:
             assert_same_state(eng, o, msg="iteration %d" % i)
@@ -111,6 +112,7 @@ def test_random_traces_stress_geometries(geom, seed):
         o.mark_inactive(inact, True)
         eng.mark_inactive(dev(inact), True)
         select_both(eng, o, gp, grng, qd, allq, ro)
+        fused_both(eng, o, allq)
 
 
 def test_block_ids_near_limit_and_fmix_index():
@@ -173,6 +175,7 @@ def test_full_size_tables_and_sampled_predictions(config):
     o.mark_inactive(tr.inactive_blocks, True)
     eng.mark_inactive(dev(tr.inactive_blocks), True)
     select_both(eng, o, gp, grng, qd, allq, ro)
+    fused_both(eng, o, allq)
 
 
 def test_full_batch_of_ten_iterations_in_one_build():
