@@ -289,9 +289,12 @@ def run_ours(args, rank, world, local_rank):
         eng.build_tables()
 
     def pre_step(i):
+        eng.set_timing(False)
         eng.load_residency(snaps[i])
         flush.zero_()
+        eng.set_timing(timing_on[0])
 
+    timing_on = [False]
     # iteration 0 (cold build, untimed) + capacity sizing on iteration 1
     eng.mark_inactive(inactive, True)
     pre_step(0)
@@ -320,6 +323,7 @@ def run_ours(args, rank, world, local_rank):
     # ---- timed region ----
     eng.read_counters(reset=True)
     eng.read_timing(reset=True)
+    timing_on[0] = True
     eng.set_timing(True)
     launches0 = eng.kernel_launches
     stream = torch.cuda.current_stream(dev)
@@ -337,6 +341,7 @@ def run_ours(args, rank, world, local_rank):
         records += tr.faults_in_iteration(i)
     torch.cuda.synchronize()
     clocks = clk.stop() if clk else None
+    timing_on[0] = False
     eng.set_timing(False)
     launches = eng.kernel_launches - launches0
     try:

@@ -302,6 +302,7 @@ enum {
   DUM_T_MIG_PLAN,
   DUM_T_COPY,
   DUM_T_RESIDENCY,
+  DUM_T_CHAIN,
   DUM_NTIMERS = 16
 };
 int dum_set_timing(dum_engine *eng, int enable);

@@ -110,7 +110,8 @@ void free_all(dum_engine *e) {
                   e->d_stage_off, e->d_head, e->d_next, e->d_slow_list, e->d_big_pool, e->d_walk_seen,
                   e->d_walk_chain, e->d_walk_tmp, e->d_walk_out, e->d_anchor_pool, e->d_anchor_range,
                   e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits, e->d_inactive_bits, e->d_lrm_blk,
-                  e->d_lrm_stamp, e->d_mig_frames, e->d_mig_src, e->d_mig_blocks, e->d_state};
+                  e->d_lrm_stamp, e->d_mig_frames, e->d_mig_src, e->d_mig_blocks, e->d_state, e->d_qkern,
+                  e->d_qloff, e->d_qnk, e->d_qbase};
   for (void *p : ptrs)
     if (p) cudaFree(p);
   if (e->h_state) cudaFreeHost(e->h_state);
@@ -203,7 +204,7 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   e->big_pool_entries = 4 * e->stage_fault_cap;
   e->n_walk_slots = 64;
   e->walk_hash_cap = pow2ceil_h(2ull * g.walk_cap);
-  e->anchor_range_cap = 1u << 20;
+  e->anchor_range_cap = 1u << 16;
   e->anchor_pool_entries = 16ull << 20;
   e->lrm_cap = 4 * g.C + 1024;
   e->mig_cap = g.C + 32;
@@ -240,6 +241,10 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_walk_out, (uint64_t)e->n_walk_slots * g.walk_cap));
   A_(dmalloc(&e->d_anchor_pool, e->anchor_pool_entries));
   A_(dmalloc(&e->d_anchor_range, 2ull * e->anchor_range_cap));
+  A_(dmalloc(&e->d_qkern, (uint64_t)e->anchor_range_cap * (g.N + 1)));
+  A_(dmalloc(&e->d_qloff, (uint64_t)e->anchor_range_cap * (g.N + 2)));
+  A_(dmalloc(&e->d_qnk, e->anchor_range_cap));
+  A_(dmalloc(&e->d_qbase, e->anchor_range_cap));
   A_(dmalloc(&e->d_frame_of, g.W));
   A_(dmalloc(&e->d_stamp_of, g.W));
   A_(dmalloc(&e->d_block_of, g.C));
@@ -371,7 +376,7 @@ int dum_predict_prefetch(dum_engine *e, const dum_query *q, uint32_t n_query, ui
   if (!e) return DUM_EINVAL;
   if (n_query == 0) return DUM_OK;
   if (!q || !out_range || (!out_pairs && out_cap_pairs)) return fail(e, DUM_EINVAL, "null argument");
-  if (n_query > e->anchor_range_cap) return fail(e, DUM_EINVAL, "too many queries in one call (max 2^20)");
+  if (n_query > e->anchor_range_cap) return fail(e, DUM_EINVAL, "too many queries in one call (max 65536)");
   if (reinterpret_cast<uintptr_t>(out_pairs) & 7) return fail(e, DUM_EINVAL, "out_pairs must be 8-byte aligned");
   cudaSetDevice(e->device);
   CK(launch_predict(e, q, n_query, out_pairs, out_cap_pairs, out_range, out_kern_off, out_chain, out_needed,
@@ -386,7 +391,7 @@ int dum_predict_select(dum_engine *e, const dum_query *q, uint32_t n_query, uint
   if (!e) return DUM_EINVAL;
   if (n_query == 0) return DUM_OK;
   if (!q || !out_range || !sel_range || (!out_pairs && out_cap_pairs)) return fail(e, DUM_EINVAL, "null argument");
-  if (n_query > e->anchor_range_cap) return fail(e, DUM_EINVAL, "too many queries in one call (max 2^20)");
+  if (n_query > e->anchor_range_cap) return fail(e, DUM_EINVAL, "too many queries in one call (max 65536)");
   if (reinterpret_cast<uintptr_t>(out_pairs) & 7) return fail(e, DUM_EINVAL, "out_pairs must be 8-byte aligned");
   cudaSetDevice(e->device);
   SelectOut so = make_select_out(e, out_writeback, out_invalidate, sel_cap, sel_range);

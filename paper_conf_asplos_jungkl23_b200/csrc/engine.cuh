@@ -150,7 +150,9 @@ struct dum_engine {
   uint32_t *d_anchor_pool;
   uint64_t anchor_pool_entries;
   uint64_t *d_anchor_range;   // per query (begin, len)
-  uint32_t anchor_range_cap;
+  uint32_t anchor_range_cap;  // max queries per predict call
+  uint32_t *d_qkern, *d_qloff, *d_qnk;  // per-query chain scratch (k_chain -> k_predict)
+  unsigned long long *d_qbase;
   // residency
   uint32_t *d_frame_of, *d_stamp_of, *d_block_of, *d_free_bits, *d_inactive_bits;
   uint32_t *d_lrm_blk, *d_lrm_stamp;

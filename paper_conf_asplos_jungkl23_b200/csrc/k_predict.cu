@@ -1,28 +1,38 @@
-// a6 + a7: prefetch-window prediction.
+// a6 + a7 (+ fused a8): prefetch-window prediction.
 //
 //  k_make_queries  transition queries from an exec-ID sequence.
 //  k_anchor_walk   WALK(e, anchor) for fault-anchored queries (PAPER.md L156:
 //                  "calculates the UM block addresses for prefetching with the
 //                  faulted block address"; D14) with the sequential walker.
-//  k_predict       one CTA per query: chain up to n next-kernel predictions
+//  k_chain         one thread per query: chain up to n next-kernel predictions
 //                  through the execution ID correlation table (PAPER.md,
-//                  L220; D15, D16), then gather the walk lists of the window's
+//                  L220; D15, D16); window layout (per-kernel offsets) and the
+//                  query's output reservation.  All queries' chains run
+//                  concurrently, so the serial lookup latency is paid once per
+//                  call instead of once per query.
+//  k_predict       one CTA per query: gather the walk lists of the window's
 //                  kernels and keep the first occurrence of every block (D17),
 //                  emitting (block, exec ID) prefetch commands.
-//                  The window set lives in a shared-memory bitmap over the
-//                  block-id space; duplicates inside one gather chunk are
-//                  resolved by a chunk-local min-position hash so any chunking
-//                  gives the sequential order's result.
+//                  Fast path: one pass writes every element at its concatenated
+//                  position while a warp-aggregated atomicOr into a shared-memory
+//                  bitmap over the block-id space detects whether any block
+//                  occurs twice; only then (never on the measured traces) the
+//                  exact order-free dedupe (min-position hash) and an ordered
+//                  re-compaction overwrite the output.
+//                  SELECT: the fused pre-eviction selection of a8 reuses the
+//                  window bitmap (select_tail.cuh).
 #include "device_util.cuh"
 #include "kernels.cuh"
-#include "walk_seq.cuh"
 #include "select_tail.cuh"
+#include "walk_seq.cuh"
 
 namespace dum {
 
 constexpr int PRED_NT = 512;
-constexpr uint32_t MAXN = 128;  // degree_n limit
-constexpr uint32_t CH_CAP = 2 * PRED_NT;
+constexpr int NWARP = PRED_NT / 32;
+constexpr uint32_t MAXN = 128;   // degree_n limit
+constexpr uint32_t DCAP = 2048;  // duplicate-block hash (window-wide)
+constexpr uint32_t CH_CAP = 1024;
 
 __global__ void k_make_queries(const uint32_t *__restrict__ seq, uint32_t n_seq, uint32_t first, uint32_t degree,
                                dum_query *__restrict__ out) {
@@ -38,17 +48,19 @@ __global__ void k_make_queries(const uint32_t *__restrict__ seq, uint32_t n_seq,
   out[i - first] = q;
 }
 
-// lookup(e, h1, h2, h3) -> successor or NONE (A9)
+// lookup(e, h1, h2, h3) -> successor or NONE (A9).  The 32 B slot is read with
+// two independent 16 B loads (one round trip per probe).
 __device__ __forceinline__ uint32_t corr_lookup(const CorrSlot *corr, uint32_t cap, uint32_t owner, uint32_t h1,
                                                 uint32_t h2, uint32_t h3) {
   const unsigned long long k0 = (unsigned long long)owner | ((unsigned long long)h1 << 32);
   const unsigned long long k1 = (unsigned long long)h2 | ((unsigned long long)h3 << 32);
   uint32_t s = (uint32_t)fmix64(k0 * 0x9E3779B97F4A7C15ull ^ fmix64(k1)) & (cap - 1);
   for (uint32_t p = 0; p < cap; ++p) {
-    const uint4 kk = __ldcg(reinterpret_cast<const uint4 *>(corr[s].key));
+    const uint4 *sp = reinterpret_cast<const uint4 *>(corr + s);
+    const uint4 kk = __ldcg(sp);
+    const uint4 vv = __ldcg(sp + 1);
     if (kk.x == NONE) return NONE;
-    if (kk.x == owner && kk.y == h1 && kk.z == h2 && kk.w == h3)
-      return (uint32_t)(__ldcg(&corr[s].last) & 0xFFFFFFFFull);
+    if (kk.x == owner && kk.y == h1 && kk.z == h2 && kk.w == h3) return vv.x;  // low word of `last`
     s = (s + 1) & (cap - 1);
   }
   return NONE;
@@ -102,202 +114,186 @@ struct PredArgs {
   uint32_t *kern_off, *chain;
   DevState *st;
   uint32_t nwords;  // bitmap words
-  // fused select (a8) outputs; unused unless SELECT
-  SelectOut so;
+  // per-query scratch written by k_chain
+  uint32_t *qkern;  // [nq][N+1]
+  uint32_t *qloff;  // [nq][N+2]
+  uint32_t *qnk;    // [nq]
+  unsigned long long *qbase;  // [nq]
+  SelectOut so;     // fused a8 outputs (SELECT only)
 };
 
-constexpr uint32_t DCAP = 2048;       // duplicate-block hash (window-wide)
-constexpr uint32_t UCAP = 65536;      // keep-bit capacity (window elements)
-constexpr int NWARP = PRED_NT / 32;
+constexpr int CHAIN_NT = 128;
 
-// Element t of the window's concatenated walk lists; d advances monotonically.
-struct WinSrc {
-  const uint32_t *walk, *apool;
-  const uint32_t *kern, *loff;
-  uint32_t nk, walk_cap;
-  uint64_t abase;
-  bool anchored;
-  __device__ __forceinline__ uint32_t get(uint32_t t, uint32_t &d) const {
-    while (d + 1 < nk && loff[d + 1] <= t) ++d;
-    const uint32_t idx = t - loff[d];
-    return (d == 0 && anchored) ? apool[abase + idx] : __ldg(walk + (uint64_t)kern[d] * walk_cap + idx);
+__global__ void __launch_bounds__(CHAIN_NT) k_chain(PredArgs a) {
+  const uint32_t qi = blockIdx.x * CHAIN_NT + threadIdx.x;
+  const uint32_t lane = threadIdx.x & 31;
+  const Geo &g = a.g;
+  uint32_t U = 0;
+  if (qi < a.nq) {
+    const dum_query Q = a.q[qi];
+    const bool anchored = Q.anchor != NONE;
+    const uint32_t E = *(volatile uint32_t *)&a.st->E;
+    uint32_t *kern = a.qkern + (uint64_t)qi * (g.N + 1);
+    uint32_t *loff = a.qloff + (uint64_t)qi * (g.N + 2);
+    uint32_t nk = 0;
+    loff[0] = 0;
+    auto add = [&](uint32_t e) {
+      uint32_t len = (nk == 0 && anchored) ? (uint32_t)a.anchor_range[2 * qi + 1] : a.walk_len[e];
+      // a kernel met earlier in the chain with the same (unanchored) walk
+      // cannot add anything (exact; keeps the reservation tight)
+      for (uint32_t d2 = anchored ? 1u : 0u; d2 < nk && len; ++d2)
+        if (kern[d2] == e) len = 0;
+      kern[nk] = e;
+      U += len;
+      loff[++nk] = U;
+    };
+    if (Q.exec < E) {
+      const uint32_t n = Q.n < g.N ? Q.n : g.N;
+      uint32_t cur = Q.exec, h1 = Q.hist[0], h2 = Q.hist[1], h3 = Q.hist[2];
+      add(cur);
+      for (uint32_t i = 0; i < n; ++i) {
+        const uint32_t nx = corr_lookup(a.corr, a.corr_cap, cur, h1, h2, h3);
+        if (nx == NONE) break;
+        add(nx);
+        h1 = h2;  // D16: shift register over predicted IDs
+        h2 = h3;
+        h3 = cur;
+        cur = nx;
+      }
+    }
+    a.qnk[qi] = nk;
   }
-};
+  // warp-aggregated output reservation
+  uint32_t incl = U;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= (uint32_t)o) incl += y;
+  }
+  unsigned long long wbase = 0;
+  if (lane == 31 && incl) wbase = atomicAdd(&a.st->pool_pairs, (unsigned long long)incl);
+  wbase = __shfl_sync(0xffffffffu, wbase, 31);
+  if (qi < a.nq) {
+    const unsigned long long base = wbase + incl - U;
+    a.qbase[qi] = base;
+    if (base + U > a.cap) set_err(a.st, ERR_ECAPACITY, base + U);
+  }
+}
 
-// One CTA per query.
-//  phase 1  warp 0 lane 0 chains the next-kernel predictions (serial corr
-//           lookups) and publishes kernel d as soon as it is known; warps 1..15
-//           meanwhile insert the published kernels' walk lists into the window
-//           bitmap (order-free atomicOr).  An element that finds its bit
-//           already set marks its block as duplicated (hash: block -> min
-//           position).
-//  phase 2  (only if duplicates exist) every element of a duplicated block
-//           lowers that block's min position to its own.
-//  phase 3  keep(t) = block not duplicated, or t is its min position (the
-//           anchor is pre-seeded at position 0 so it is never kept): exactly
-//           the first-occurrence rule of D17 regardless of processing order.
-//  phase 4  ordered compaction: per-warp contiguous segments, ballots, one
-//           block scan of 16 warp totals; (block, exec) pairs written.
-//  SELECT   (fused a8) the window set is the phase-1 bitmap: count window
-//           blocks without a frame, then scan the LRM log for victims.
+// Warp-aggregated test-and-set of bit b in a shared bitmap: lanes hitting the
+// same 32-bit word combine into one atomicOr.  Returns true if the block was
+// already present (set before, or by a lower lane of this warp step).
+__device__ __forceinline__ bool warp_test_and_set(uint32_t *bitmap, uint32_t b, bool valid) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t w = valid ? (b >> 5) : 0xFFFFFFFFu;
+  const uint32_t bit = valid ? 1u << (b & 31) : 0u;
+  const uint32_t grp = __match_any_sync(0xffffffffu, w);
+  const uint32_t comb = __reduce_or_sync(grp, bit);
+  const uint32_t leader = __ffs(grp) - 1;
+  uint32_t old = 0;
+  if (lane == leader && valid) old = atomicOr(&bitmap[w], comb);
+  old = __shfl_sync(0xffffffffu, old, leader);
+  bool dup = valid && (old & bit);
+  if (__popc(comb) < __popc(grp) && valid) {
+    // two lanes carry the same block: all but the lowest are duplicates
+    const uint32_t same = __match_any_sync(grp, b);
+    dup |= lane != (uint32_t)(__ffs(same) - 1);
+  }
+  return dup;
+}
+
 template <bool SELECT>
 __global__ void __launch_bounds__(PRED_NT) k_predict(PredArgs a) {
   extern __shared__ uint32_t bitmap[];
   __shared__ uint32_t kern[MAXN + 1], loff[MAXN + 2], kcnt[MAXN + 1];
   __shared__ uint32_t dk[DCAP], dv[DCAP];
-  __shared__ uint32_t keepbits[UCAP / 32];
   __shared__ uint32_t ws[NWARP], wtot[NWARP];
-  __shared__ volatile uint32_t s_ready, s_done;
-  __shared__ uint32_t s_ndup, s_ovf, s_ok, s_nonres;
-  __shared__ unsigned long long s_base;
+  __shared__ uint32_t s_ndup, s_ovf, s_nonres;
   const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const uint32_t qi = blockIdx.x;
   const Geo &g = a.g;
-  const dum_query Q = a.q[qi];
-  const bool anchored = Q.anchor != NONE;
+  const uint32_t anchor = a.q[qi].anchor;
+  const bool anchored = anchor != NONE;
+  const uint32_t nk = a.qnk[qi];
+  const unsigned long long base = a.qbase[qi];
   for (uint32_t w = tid; w < a.nwords; w += PRED_NT) bitmap[w] = 0;
   for (uint32_t p = tid; p < DCAP; p += PRED_NT) {
     dk[p] = NONE;
     dv[p] = NONE;
   }
-  for (uint32_t p = tid; p <= g.N; p += PRED_NT) kcnt[p] = 0;
+  for (uint32_t d = tid; d <= nk; d += PRED_NT) {
+    loff[d] = a.qloff[(uint64_t)qi * (g.N + 2) + d];
+    if (d < nk) kern[d] = a.qkern[(uint64_t)qi * (g.N + 1) + d];
+  }
   if (tid == 0) {
-    s_ready = 0;
-    s_done = 0;
     s_ndup = 0;
     s_ovf = 0;
     s_nonres = 0;
-    loff[0] = 0;
   }
   __syncthreads();
-  if (tid == 0 && anchored && Q.anchor < g.W) {
-    bitmap[Q.anchor >> 5] |= 1u << (Q.anchor & 31);
-    hmap_insert_min(dk, dv, DCAP, Q.anchor, 0);  // position 0: never kept
-    s_ndup = 1;
+  const uint32_t U = nk ? loff[nk] : 0;
+  const bool ok = base + U <= a.cap;
+  if (tid == 0 && anchored && anchor < g.W) {
+    bitmap[anchor >> 5] |= 1u << (anchor & 31);
+    hmap_insert_min(dk, dv, DCAP, anchor, 0);  // position 0: never kept
   }
   __syncthreads();
-  WinSrc src{a.walk, a.anchor_pool, kern, loff, 0, g.walk_cap, anchored ? a.anchor_range[2 * qi] : 0, anchored};
-  // ---------------- phase 1 ----------------
-  if (wid == 0) {
-    if (lane == 0) {
-      const uint32_t E = *(volatile uint32_t *)&a.st->E;
-      uint32_t nk = 0, tot = 0;
-      auto publish = [&](uint32_t e, uint32_t d) {
-        uint32_t len = (d == 0 && anchored) ? (uint32_t)a.anchor_range[2 * qi + 1] : a.walk_len[e];
-        // a kernel met earlier in the chain with the same (unanchored) walk
-        // cannot add anything (exact; keeps the reservation tight)
-        for (uint32_t d2 = anchored ? 1u : 0u; d2 < d && len; ++d2)
-          if (kern[d2] == e) len = 0;
-        kern[d] = e;
-        tot += len;
-        loff[d + 1] = tot;
-        __threadfence_block();
-        s_ready = d + 1;
-      };
-      if (Q.exec < E) {
-        const uint32_t n = Q.n < g.N ? Q.n : g.N;
-        uint32_t cur = Q.exec, h1 = Q.hist[0], h2 = Q.hist[1], h3 = Q.hist[2];
-        publish(cur, nk++);
-        for (uint32_t i = 0; i < n; ++i) {
-          const uint32_t nx = corr_lookup(a.corr, a.corr_cap, cur, h1, h2, h3);
-          if (nx == NONE) break;
-          publish(nx, nk++);
-          h1 = h2;  // D16: shift register over predicted IDs
-          h2 = h3;
-          h3 = cur;
-          cur = nx;
-        }
-      }
-      __threadfence_block();
-      s_done = 1;
-    }
-  } else {
+  const uint32_t *apool = a.anchor_pool + (anchored ? a.anchor_range[2 * qi] : 0);
+  auto elem = [&](uint32_t t, uint32_t &d) -> uint32_t {
+    while (d + 1 < nk && loff[d + 1] <= t) ++d;
+    const uint32_t idx = t - loff[d];
+    return (d == 0 && anchored) ? apool[idx] : __ldg(a.walk + (uint64_t)kern[d] * g.walk_cap + idx);
+  };
+  // ---------------- fast path: one pass ----------------
+  // warp w owns the contiguous segment [t0, t1); 4 loads in flight per lane
+  const uint32_t seg = ((U + NWARP - 1) / NWARP + 127) & ~127u;
+  const uint32_t t0 = min(U, wid * seg), t1 = min(U, t0 + seg);
+  uint32_t nonres = 0, ndup = 0;
+  {
     uint32_t d = 0;
-    for (;;) {
-      uint32_t ready = s_ready;
-      if (d >= ready) {
-        if (s_done) {
-          __threadfence_block();
-          ready = s_ready;
-          if (d >= ready) break;
-        } else {
-          __nanosleep(64);
-          continue;
+    for (uint32_t c = t0; c < t1; c += 128) {
+      uint32_t b[4];
+      uint32_t dd[4];
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const uint32_t t = c + 32 * k + lane;
+        b[k] = t < t1 ? elem(t, d) : NONE;
+        dd[k] = d;
+      }
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const uint32_t t = c + 32 * k + lane;
+        const bool valid = t < t1;
+        const bool dup = warp_test_and_set(bitmap, b[k], valid);
+        if (dup) {
+          ++ndup;
+          if (!hmap_insert_min(dk, dv, DCAP, b[k], t + 1)) s_ovf = 1;
+        }
+        if (valid) {
+          if (ok) reinterpret_cast<uint2 *>(a.pairs)[base + t] = make_uint2(b[k], kern[dd[k]]);
+          if (SELECT) nonres += __ldg(&a.so.frame_of[b[k]]) == NONE;
         }
       }
-      const uint32_t L = loff[d + 1] - loff[d];
-      const uint32_t e = kern[d];
-      const uint32_t *lst = (d == 0 && anchored) ? a.anchor_pool + src.abase : a.walk + (uint64_t)e * g.walk_cap;
-      for (uint32_t idx = (wid - 1) * 32 + lane; idx < L; idx += (NWARP - 1) * 32) {
-        const uint32_t b = __ldg(lst + idx);
-        const uint32_t bit = 1u << (b & 31);
-        const uint32_t old = atomicOr(&bitmap[b >> 5], bit);
-        if (old & bit) {
-          if (!hmap_insert_min(dk, dv, DCAP, b, loff[d] + idx + 1)) s_ovf = 1;
-          atomicAdd(&s_ndup, 1u);
-        }
-      }
-      ++d;
     }
+  }
+  if (ndup) atomicAdd(&s_ndup, ndup);
+  if (SELECT) {
+#pragma unroll
+    for (int o = 16; o; o >>= 1) nonres += __shfl_xor_sync(0xffffffffu, nonres, o);
+    if (lane == 0 && nonres) atomicAdd(&s_nonres, nonres);
   }
   __syncthreads();
-  uint32_t nk = s_ready;
-  const uint32_t U = loff[nk];
-  src.nk = nk;
-  if (tid == 0) {
-    const unsigned long long base = atomicAdd(&a.st->pool_pairs, (unsigned long long)U);
-    s_base = base;
-    s_ok = base + U <= a.cap;
-    if (!s_ok) set_err(a.st, ERR_ECAPACITY, base + U);
-  }
-  const bool ndup = s_ndup != 0;
-  if (s_ovf) {
-    // too many duplicated blocks for the window-wide hash: exact chunked
-    // fallback (ordered chunks, chunk-local min-position hash)
-    for (uint32_t w = tid; w < a.nwords; w += PRED_NT) bitmap[w] = 0;
+  uint32_t run = U;
+  if (s_ndup) {
+    // ---------------- exact slow path (some block occurs twice) ----------------
+    if (tid == 0) s_nonres = 0;
+    for (uint32_t d = tid; d <= nk; d += PRED_NT) kcnt[d] = 0;
     __syncthreads();
-    if (tid == 0 && anchored && Q.anchor < g.W) bitmap[Q.anchor >> 5] |= 1u << (Q.anchor & 31);
-    for (uint32_t p = tid; p < CH_CAP; p += PRED_NT) {
-      dk[p] = NONE;
-      dv[p] = NONE;
-    }
-    __syncthreads();
-    const unsigned long long base = s_base;
-    const bool ok = s_ok;
-    uint32_t run = 0, d = 0;
-    for (uint32_t c = 0; c < U; c += PRED_NT) {
-      const uint32_t t = c + tid;
-      uint32_t b = NONE;
-      bool fresh = false;
-      if (t < U) {
-        b = src.get(t, d);
-        fresh = !(bitmap[b >> 5] & (1u << (b & 31)));
-        if (fresh) hmap_insert_min(dk, dv, CH_CAP, b, t);
-      }
-      __syncthreads();
-      const uint32_t keep = fresh && hmap_get(dk, dv, CH_CAP, b) == t;
-      if (keep) {
-        atomicOr(&bitmap[b >> 5], 1u << (b & 31));
-        atomicAdd(&kcnt[d], 1u);
-        if (SELECT && __ldg(&a.so.frame_of[b]) == NONE) atomicAdd(&s_nonres, 1u);
-      }
-      uint32_t tot;
-      const uint32_t pre = block_excl_scan(keep, ws, &tot);
-      if (keep && ok) reinterpret_cast<uint2 *>(a.pairs)[base + run + pre] = make_uint2(b, kern[d]);
-      run += tot;
-      for (uint32_t p = tid; p < CH_CAP; p += PRED_NT) {
-        dk[p] = NONE;
-        dv[p] = NONE;
-      }
-      __syncthreads();
-    }
-    if (tid == 0) wtot[0] = run;
-  } else {
-    // ---------------- phase 2 ----------------
-    if (ndup) {
+    if (!s_ovf) {
+      // phase 2: every occurrence of a duplicated block lowers its min position
       uint32_t d = 0;
       for (uint32_t t = tid; t < U; t += PRED_NT) {
-        const uint32_t b = src.get(t, d);
+        const uint32_t b = elem(t, d);
         const uint32_t s0 = hslot(b, DCAP);
         for (uint32_t p = 0, s = s0; p < DCAP; ++p, s = (s + 1) & (DCAP - 1)) {
           const uint32_t k = dk[s];
@@ -309,91 +305,108 @@ __global__ void __launch_bounds__(PRED_NT) k_predict(PredArgs a) {
         }
       }
       __syncthreads();
-    }
-    // ---------------- phase 3: keep bits and per-warp counts ----------------
-    const uint32_t seg = ((U + NWARP - 1) / NWARP + 31) & ~31u;
-    const uint32_t t0 = wid * seg, t1 = min(U, t0 + seg);
-    const bool bits = U <= UCAP;
-    uint32_t cnt = 0;
-    {
-      uint32_t d = 0;
-      for (uint32_t c = t0; c < t1; c += 32) {
-        const uint32_t t = c + lane;
-        bool keep = false;
-        if (t < t1) {
-          const uint32_t b = src.get(t, d);
-          keep = !ndup;
-          if (ndup) {
+      // phase 3: per-warp keep counts
+      uint32_t cnt = 0;
+      {
+        uint32_t dd = 0;
+        for (uint32_t c = t0; c < t1; c += 32) {
+          const uint32_t t = c + lane;
+          bool keep = false;
+          if (t < t1) {
+            const uint32_t b = elem(t, dd);
             const uint32_t m = hmap_get(dk, dv, DCAP, b);
             keep = (m == NONE) || (m == t + 1);
           }
+          cnt += __popc(__ballot_sync(0xffffffffu, keep));
         }
-        const uint32_t mask = __ballot_sync(0xffffffffu, keep);
-        if (bits && lane == 0) keepbits[c >> 5] = mask;
-        cnt += __popc(mask);
       }
-    }
-    if (lane == 0) wtot[wid] = cnt;
-    __syncthreads();
-    if (tid == 0) {
-      uint32_t acc = 0;
-      for (int w = 0; w < NWARP; ++w) {
-        const uint32_t v = wtot[w];
-        wtot[w] = acc;
-        acc += v;
+      if (lane == 0) wtot[wid] = cnt;
+      __syncthreads();
+      if (tid == 0) {
+        uint32_t acc = 0;
+        for (int w = 0; w < NWARP; ++w) {
+          const uint32_t v = wtot[w];
+          wtot[w] = acc;
+          acc += v;
+        }
+        ws[0] = acc;
       }
-      ws[0] = acc;
-    }
-    __syncthreads();
-    // ---------------- phase 4: ordered write ----------------
-    const unsigned long long base = s_base;
-    const bool ok = s_ok;
-    uint32_t pos = wtot[wid];
-    uint32_t nonres = 0;
-    {
-      uint32_t d = 0;
-      for (uint32_t c = t0; c < t1; c += 32) {
-        const uint32_t t = c + lane;
-        uint32_t b = NONE;
-        bool keep = false;
-        if (t < t1) {
-          b = src.get(t, d);
-          if (bits) {
-            keep = (keepbits[c >> 5] >> lane) & 1u;
-          } else {
-            keep = !ndup;
-            if (ndup) {
-              const uint32_t m = hmap_get(dk, dv, DCAP, b);
-              keep = (m == NONE) || (m == t + 1);
-            }
+      __syncthreads();
+      // phase 4: ordered re-write
+      uint32_t pos = wtot[wid], nr = 0;
+      {
+        uint32_t dd = 0;
+        for (uint32_t c = t0; c < t1; c += 32) {
+          const uint32_t t = c + lane;
+          uint32_t b = NONE;
+          bool keep = false;
+          if (t < t1) {
+            b = elem(t, dd);
+            const uint32_t m = hmap_get(dk, dv, DCAP, b);
+            keep = (m == NONE) || (m == t + 1);
           }
+          const uint32_t mask = __ballot_sync(0xffffffffu, keep);
+          if (keep) {
+            if (ok) reinterpret_cast<uint2 *>(a.pairs)[base + pos + __popc(mask & ((1u << lane) - 1))] =
+                make_uint2(b, kern[dd]);
+            if (SELECT) nr += __ldg(&a.so.frame_of[b]) == NONE;
+          }
+          const uint32_t grp = __match_any_sync(0xffffffffu, keep ? dd : 0xFFFFFFFFu);
+          if (keep && lane == __ffs(grp) - 1) atomicAdd(&kcnt[dd], __popc(grp));
+          pos += __popc(mask);
         }
-        const uint32_t mask = __ballot_sync(0xffffffffu, keep);
-        if (keep) {
-          if (ok) reinterpret_cast<uint2 *>(a.pairs)[base + pos + __popc(mask & ((1u << lane) - 1))] =
-              make_uint2(b, kern[d]);
-          if (SELECT) nonres += __ldg(&a.so.frame_of[b]) == NONE;
-        }
-        // per-kernel counts (kern_off): one add per distinct kernel among kept lanes
-        const uint32_t grp = __match_any_sync(0xffffffffu, keep ? d : 0xFFFFFFFFu);
-        if (keep && lane == __ffs(grp) - 1) atomicAdd(&kcnt[d], __popc(grp));
-        pos += __popc(mask);
       }
-    }
-    if (SELECT) {
+      if (SELECT) {
 #pragma unroll
-      for (int o = 16; o; o >>= 1) nonres += __shfl_xor_sync(0xffffffffu, nonres, o);
-      if (lane == 0 && nonres) atomicAdd(&s_nonres, nonres);
+        for (int o = 16; o; o >>= 1) nr += __shfl_xor_sync(0xffffffffu, nr, o);
+        if (lane == 0 && nr) atomicAdd(&s_nonres, nr);
+      }
+      __syncthreads();
+      run = ws[0];
+    } else {
+      // too many duplicated blocks for the window-wide hash: ordered chunks
+      // with a chunk-local min-position hash
+      for (uint32_t w = tid; w < a.nwords; w += PRED_NT) bitmap[w] = 0;
+      for (uint32_t p = tid; p < CH_CAP; p += PRED_NT) {
+        dk[p] = NONE;
+        dv[p] = NONE;
+      }
+      __syncthreads();
+      if (tid == 0 && anchored && anchor < g.W) bitmap[anchor >> 5] |= 1u << (anchor & 31);
+      __syncthreads();
+      uint32_t r = 0, d = 0;
+      for (uint32_t c = 0; c < U; c += PRED_NT) {
+        const uint32_t t = c + tid;
+        uint32_t b = NONE;
+        bool fresh = false;
+        if (t < U) {
+          b = elem(t, d);
+          fresh = !(bitmap[b >> 5] & (1u << (b & 31)));
+          if (fresh) hmap_insert_min(dk, dv, CH_CAP, b, t);
+        }
+        __syncthreads();
+        const uint32_t keep = fresh && hmap_get(dk, dv, CH_CAP, b) == t;
+        if (keep) {
+          atomicOr(&bitmap[b >> 5], 1u << (b & 31));
+          atomicAdd(&kcnt[d], 1u);
+          if (SELECT && __ldg(&a.so.frame_of[b]) == NONE) atomicAdd(&s_nonres, 1u);
+        }
+        uint32_t tot;
+        const uint32_t pre = block_excl_scan(keep, ws, &tot);
+        if (keep && ok) reinterpret_cast<uint2 *>(a.pairs)[base + r + pre] = make_uint2(b, kern[d]);
+        r += tot;
+        for (uint32_t p = tid; p < CH_CAP; p += PRED_NT) {
+          dk[p] = NONE;
+          dv[p] = NONE;
+        }
+        __syncthreads();
+      }
+      run = r;
     }
-    __syncthreads();
-    if (tid == 0) wtot[0] = ws[0];
   }
-  __syncthreads();
-  const uint32_t run = wtot[0];
-  const unsigned long long base = s_base;
   if (tid == 0) {
     a.range[2 * qi] = base;
-    a.range[2 * qi + 1] = base + (s_ok ? run : 0);
+    a.range[2 * qi + 1] = base + (ok ? run : 0);
     ctr_add(a.st, DUM_CTR_QUERIES, 1);
     ctr_add(a.st, DUM_CTR_CHAIN, nk);
     ctr_add(a.st, DUM_CTR_GATHERED, U);
@@ -401,13 +414,16 @@ __global__ void __launch_bounds__(PRED_NT) k_predict(PredArgs a) {
   }
   if (a.kern_off) {
     uint32_t *ko = a.kern_off + (uint64_t)qi * (g.N + 2);
-    if (tid == 0) {
-      uint32_t acc = 0;
-      ko[0] = 0;
-      for (uint32_t d = 0; d <= g.N; ++d) {
-        if (d < nk) acc += kcnt[d];
-        ko[d + 1] = acc;
+    const bool dedup = s_ndup != 0;
+    for (uint32_t d = tid; d <= g.N + 1; d += PRED_NT) {
+      uint32_t v;
+      if (!dedup) {
+        v = d <= nk ? loff[d] : U;
+      } else {
+        v = 0;
+        for (uint32_t x = 0; x < d && x < nk; ++x) v += kcnt[x];
       }
+      ko[d] = v;
     }
   }
   if (a.chain) {
@@ -437,9 +453,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
                            const SelectOut *sel, uint64_t *sel_needed, cudaStream_t s) {
   if (nq == 0) return cudaSuccess;
   if (nq > e->anchor_range_cap) return cudaErrorInvalidValue;
-  cudaMemsetAsync(&e->d_state->pool_pairs, 0, sizeof(unsigned long long), s);
-  cudaMemsetAsync(&e->d_state->pool_anchor, 0, sizeof(unsigned long long), s);
-  if (sel) cudaMemsetAsync(&e->d_state->pool_wb, 0, 2 * sizeof(unsigned long long), s);
+  cudaMemsetAsync(&e->d_state->pool_pairs, 0, 2 * sizeof(unsigned long long) * 2, s);  // pairs, wb, inv, anchor
   WalkScratch ws{e->d_walk_seen, e->d_walk_chain, e->d_walk_tmp, e->walk_hash_cap,
                  e->g.walk_cap + e->g.R * e->g.A + 4};
   {
@@ -465,7 +479,15 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   a.chain = chain;
   a.st = e->d_state;
   a.nwords = (e->g.W + 31) / 32;
+  a.qkern = e->d_qkern;
+  a.qloff = e->d_qloff;
+  a.qnk = e->d_qnk;
+  a.qbase = e->d_qbase;
   if (sel) a.so = *sel;
+  {
+    TimerScope t(e, DUM_T_CHAIN, s);
+    k_chain<<<(nq + CHAIN_NT - 1) / CHAIN_NT, CHAIN_NT, 0, s>>>(a);
+  }
   const size_t smem = (size_t)a.nwords * 4;
   if (sel) {
     cudaFuncSetAttribute(k_predict<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -476,7 +498,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
     TimerScope t(e, DUM_T_PREDICT, s);
     k_predict<false><<<nq, PRED_NT, smem, s>>>(a);
   }
-  e->kernel_launches += 2;
+  e->kernel_launches += 3;
   if (needed) {
     k_copy_counter<<<1, 1, 0, s>>>(&e->d_state->pool_pairs, needed);
     e->kernel_launches += 1;

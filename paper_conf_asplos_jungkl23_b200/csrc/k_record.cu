@@ -28,15 +28,95 @@ __global__ void __launch_bounds__(INGEST_NT) k_ingest(
   __shared__ uint32_t hk[INGEST_HCAP];
   __shared__ uint32_t hv[INGEST_HCAP];
   __shared__ uint32_t ws[INGEST_NT / 32];
+  __shared__ uint32_t s_dups;
   const uint32_t i = blockIdx.x;
   if (i >= n_launch) return;
   const uint64_t a = off[i], b = off[i + 1];
   const uint32_t n = (uint32_t)(b - a);
   if (threadIdx.x == 0) {
-    // execution ID table probe (insert if absent)
-    const uint64_t h = hash[i];
-    stage_hash[l0 + i] = h;
+    stage_hash[l0 + i] = hash[i];
     stage_off[l0 + i] = f0 + a;
+    ctr_add(st, DUM_CTR_LAUNCHES, 1);
+    s_dups = 0;
+  }
+  if (n > 0) {
+    // hash of (block -> first position) in shared memory, or in a private
+    // region of the global pool for launches with > INGEST_HCAP/2 records
+    uint32_t *keys = hk, *vals = hv;
+    uint32_t cap = pow2ceil(2 * n);
+    if (cap < 64) cap = 64;
+    bool fits = true;
+    if (n > INGEST_HCAP / 2) {
+      const uint64_t pbase = 4ull * (f0 + a);  // region [4(f0+a), 4(f0+b)) holds >= cap entries
+      if (pbase + cap > big_entries) {
+        if (threadIdx.x == 0) set_err(st, ERR_ECAPACITY, pbase + cap);
+        fits = false;
+      }
+      keys = big_pool + 2ull * pbase;
+      vals = keys + cap;
+    }
+    if (fits) {
+      for (uint32_t t = threadIdx.x; t < cap; t += INGEST_NT) {
+        keys[t] = NONE;
+        vals[t] = NONE;
+      }
+      __syncthreads();
+      bool dup = false;
+      for (uint32_t j = threadIdx.x; j < n; j += INGEST_NT) {
+        const uint32_t blk = faults[a + j];
+        if (blk >= W) {
+          set_err(st, ERR_EINVAL);
+          dup = true;  // dropped: take the compaction path
+          continue;
+        }
+        // first-occurrence test: insert (block -> min position)
+        uint32_t s = hslot(blk, cap);
+        for (uint32_t p = 0; p < cap; ++p) {
+          const uint32_t old = atomicCAS(&keys[s], NONE, blk);
+          if (old == NONE || old == blk) {
+            dup |= old == blk;
+            atomicMin(&vals[s], j);
+            break;
+          }
+          s = (s + 1) & (cap - 1);
+        }
+      }
+      if (dup) s_dups = 1;
+      __syncthreads();
+      uint32_t run = n;
+      if (!s_dups) {
+        // no duplicate record in this launch: the normalised list is the input
+        for (uint32_t j = threadIdx.x; j < n; j += INGEST_NT) stage_norm[f0 + a + j] = faults[a + j];
+      } else {
+        // order-preserving compaction of first occurrences
+        run = 0;
+        for (uint32_t c = 0; c < n; c += INGEST_NT) {
+          const uint32_t j = c + threadIdx.x;
+          uint32_t blk = NONE, keep = 0;
+          if (j < n) {
+            blk = faults[a + j];
+            keep = blk < W && hmap_get(keys, vals, cap, blk) == j;
+          }
+          uint32_t tot;
+          const uint32_t pre = block_excl_scan(keep, ws, &tot);
+          if (keep) stage_norm[f0 + a + run + pre] = blk;
+          run += tot;
+        }
+      }
+      if (threadIdx.x == 0) {
+        stage_cnt[l0 + i] = run;
+        ctr_add(st, DUM_CTR_RAW_RECORDS, n);
+        ctr_add(st, DUM_CTR_NORM_RECORDS, run);
+      }
+    } else if (threadIdx.x == 0) {
+      stage_cnt[l0 + i] = 0;
+    }
+  } else if (threadIdx.x == 0) {
+    stage_cnt[l0 + i] = 0;
+  }
+  if (threadIdx.x == 0) {
+    // execution ID table probe (insert if absent), PAPER.md L136
+    const uint64_t h = hash[i];
     uint32_t slot = NONE;
     if (h == EMPTY64) {
       slot = exec_cap;  // sentinel-key slot; exec_keys[exec_cap] is a presence word
@@ -44,7 +124,7 @@ __global__ void __launch_bounds__(INGEST_NT) k_ingest(
     } else {
       uint32_t s = (uint32_t)fmix64(h) & (exec_cap - 1);
       for (uint32_t p = 0; p < exec_cap; ++p) {
-        unsigned long long old = atomicCAS(&exec_keys[s], EMPTY64, (unsigned long long)h);
+        const unsigned long long old = atomicCAS(&exec_keys[s], EMPTY64, (unsigned long long)h);
         if (old == EMPTY64 || old == h) {
           slot = s;
           break;
@@ -58,59 +138,6 @@ __global__ void __launch_bounds__(INGEST_NT) k_ingest(
       atomicMin(&exec_minpos[slot], i);
     }
     stage_slot[l0 + i] = slot;
-  }
-  if (threadIdx.x == 0) ctr_add(st, DUM_CTR_LAUNCHES, 1);
-  if (n == 0) {
-    if (threadIdx.x == 0) stage_cnt[l0 + i] = 0;
-    return;
-  }
-  // hash of (block -> first position) in shared memory, or in a private
-  // region of the global pool for launches with > INGEST_HCAP/2 records
-  uint32_t *keys = hk, *vals = hv;
-  uint32_t cap = pow2ceil(2 * n);
-  if (cap < 64) cap = 64;
-  if (n > INGEST_HCAP / 2) {
-    cap = pow2ceil(2 * n);
-    uint64_t base = 4ull * (f0 + a);  // region [4(f0+a), 4(f0+b)) holds >= cap entries
-    if (2ull * (base + cap) > 2ull * big_entries) {
-      if (threadIdx.x == 0) set_err(st, ERR_ECAPACITY, base + cap);
-      return;
-    }
-    keys = big_pool + 2ull * base;
-    vals = keys + cap;
-  }
-  for (uint32_t t = threadIdx.x; t < cap; t += INGEST_NT) {
-    keys[t] = NONE;
-    vals[t] = NONE;
-  }
-  __syncthreads();
-  for (uint32_t j = threadIdx.x; j < n; j += INGEST_NT) {
-    uint32_t blk = faults[a + j];
-    if (blk >= W) {
-      set_err(st, ERR_EINVAL);
-      continue;
-    }
-    hmap_insert_min(keys, vals, cap, blk, j);
-  }
-  __syncthreads();
-  // order-preserving compaction of first occurrences
-  uint32_t run = 0;
-  for (uint32_t c = 0; c < n; c += INGEST_NT) {
-    const uint32_t j = c + threadIdx.x;
-    uint32_t blk = NONE, keep = 0;
-    if (j < n) {
-      blk = faults[a + j];
-      keep = blk < W && hmap_get(keys, vals, cap, blk) == j;
-    }
-    uint32_t tot;
-    uint32_t pre = block_excl_scan(keep, ws, &tot);
-    if (keep) stage_norm[f0 + a + run + pre] = blk;
-    run += tot;
-  }
-  if (threadIdx.x == 0) {
-    stage_cnt[l0 + i] = run;
-    ctr_add(st, DUM_CTR_RAW_RECORDS, n);
-    ctr_add(st, DUM_CTR_NORM_RECORDS, run);
   }
 }
 

@@ -5,7 +5,7 @@
 # serialised: compare SHARES) and gpurun_out/<tag>_<kernel>.ncu-rep (--set full).
 set -u
 TAG=${1:-r01}
-KERNELS=${KERNELS:-"k_predict k_apply_walk k_select"}
+KERNELS=${KERNELS:-"k_predict k_apply_walk k_ingest k_chain"}
 B="python bench.py --steps 2 --warmup 3 --no-e2e --no-migration --no-cpu-baseline"
 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv \
     --log-file gpurun_out/${TAG}_launches.csv $B > gpurun_out/${TAG}_launches.log 2>&1
