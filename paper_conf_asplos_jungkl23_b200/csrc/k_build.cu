@@ -25,7 +25,7 @@
 
 namespace dum {
 
-constexpr int BUILD_NT = 256;
+constexpr int BUILD_NT = 512;
 constexpr uint32_t GCAP = 1024;   // launches of one exec ID per build batch
 constexpr uint32_t OPCAP = 2048;  // ops per apply round
 constexpr uint32_t QCAP = 4096;   // smem walk-dedupe hash capacity (|Q| <= 2048)
@@ -154,6 +154,27 @@ struct RegSet {
 #pragma unroll
     for (int j = 0; j < MAXS; ++j) sc[0][j] = ss[j];
   }
+  // Row of block b (count + successors, or NONE count when absent) -> out[0..S].
+  __device__ __forceinline__ void export_row(uint32_t b, uint32_t A, uint32_t S, uint32_t *out) const {
+    int hit = -1;
+#pragma unroll
+    for (int w = 0; w < MAXA; ++w)
+      if (w < (int)A && tag[w] == b) hit = w;
+    uint32_t cnt = hit < 0 ? NONE : 0;
+#pragma unroll
+    for (int w = 0; w < MAXA; ++w) {
+      if (w == hit) {
+#pragma unroll
+        for (int jj = 0; jj < MAXS; ++jj) {
+          if (jj < (int)S) {
+            out[1 + jj] = sc[w][jj];
+            cnt += sc[w][jj] != NONE;
+          }
+        }
+      }
+    }
+    out[0] = cnt;
+  }
   // INSERT s as the MRU successor of the row in way 0 (D9).
   __device__ __forceinline__ void insert0(uint32_t s, uint32_t S) {
     if (s == tag[0]) return;
@@ -198,11 +219,25 @@ struct BuildArgs {
 //                                                            present).
 // The speculation is still verified (succ[0] == C[i+1]); any violation sends e
 // to the sequential walker.
+//
+// Shared-memory plan (u32 words): grp/seg | row cache of C (count + S succ
+// per position, filled by the set owners right after applying the ops, so the
+// walk never re-reads the table) | per-row Q offsets | a union of the apply
+// arrays (per-set counts/offsets, non-empty-set list, ops, op order) and the
+// walk's dedupe hash.
+constexpr uint32_t RCCAP = 10240;  // row-cache words: n * (1 + S) <= RCCAP
+
+__host__ __device__ inline uint32_t apply_union_words(uint32_t R) {
+  const uint32_t ap = 3 * R + 2 * OPCAP, wk = 2 * QCAP;
+  return ap > wk ? ap : wk;
+}
+
 template <int MAXA, int MAXS>
 __global__ void __launch_bounds__(BUILD_NT) k_apply_walk(BuildArgs a) {
+  constexpr int OWN_B = (MAXA * (1 + MAXS) <= 10) ? 4 : 1;  // sets loaded per owner batch
   extern __shared__ uint32_t sm[];
   __shared__ uint32_t ws[BUILD_NT / 32];
-  __shared__ uint32_t s_ng, s_tev, s_flag;
+  __shared__ uint32_t s_ng, s_tev, s_flag, s_sets, s_nnz;
   const Geo &g = a.g;
   const uint32_t tid = threadIdx.x;
   const uint32_t j = blockIdx.x;
@@ -220,10 +255,12 @@ __global__ void __launch_bounds__(BUILD_NT) k_apply_walk(BuildArgs a) {
   if (e == NONE || a.stage_cnt[j] == 0) return;
   if (__ldcg(&a.head[e]) != j) return;  // not this exec ID's group leader
 
-  uint32_t *grp = sm;              // [GCAP]
-  uint32_t *seg = grp + GCAP;      // [GCAP + 1]
-  uint32_t *U = seg + GCAP + 1;    // union region
   const uint32_t R = g.R, A = g.A, S = g.S;
+  uint32_t *grp = sm;             // [GCAP]
+  uint32_t *seg = grp + GCAP;     // [GCAP + 1]
+  uint32_t *rc = seg + GCAP + 1;  // [RCCAP]
+  uint32_t *cqs = rc + RCCAP;     // [WCAP]
+  uint32_t *U = cqs + WCAP;       // union region
 
   // ---- collect and order the group's launches ----
   if (tid == 0) {
@@ -234,13 +271,13 @@ __global__ void __launch_bounds__(BUILD_NT) k_apply_walk(BuildArgs a) {
     }
     if (x != NONE) set_err(a.st, ERR_ECAPACITY, GCAP + 1);
     s_ng = n;
+    s_sets = 0;
     a.head[e] = NONE;
   }
   __syncthreads();
   const uint32_t ng = s_ng;
-  {
-    // rank sort (ascending launch index)
-    uint32_t *tmp = U;
+  if (ng > 1) {
+    uint32_t *tmp = U;  // rank sort (ascending launch index)
     for (uint32_t p = tid; p < ng; p += BUILD_NT) {
       uint32_t v = grp[p], r = 0;
       for (uint32_t q = 0; q < ng; ++q) r += grp[q] < v;
@@ -249,109 +286,134 @@ __global__ void __launch_bounds__(BUILD_NT) k_apply_walk(BuildArgs a) {
     __syncthreads();
     for (uint32_t p = tid; p < ng; p += BUILD_NT) grp[p] = tmp[p];
     __syncthreads();
-    if (tid == 0) {
-      uint32_t acc = 0;
-      for (uint32_t p = 0; p < ng; ++p) {
-        seg[p] = acc;
-        acc += a.stage_cnt[grp[p]];
-      }
-      seg[ng] = acc;
-    }
-    __syncthreads();
   }
+  if (tid == 0) {
+    uint32_t acc = 0;
+    for (uint32_t p = 0; p < ng; ++p) {
+      seg[p] = acc;
+      acc += a.stage_cnt[grp[p]];
+    }
+    seg[ng] = acc;
+  }
+  __syncthreads();
   const uint32_t n_ops = seg[ng];
-  __shared__ uint32_t s_sets;
-  if (tid == 0) s_sets = 0;
+  const uint32_t last_seg = seg[ng - 1];
+  const uint32_t Llast = grp[ng - 1];
+  const uint32_t n = a.stage_cnt[Llast];
+  const bool single_round = n_ops <= OPCAP;
+  const bool use_rc = single_round && n <= WCAP && n * (1 + S) <= RCCAP;
   uint32_t *tbl_e = a.tbl + (uint64_t)e * R * g.stride;
 
   // ---- apply: rounds of up to OPCAP ops, counting-sorted by set ----
-  uint32_t *cnt_s = U, *off_s = U + R;
-  uint32_t *opb = off_s + R, *opn = opb + OPCAP, *opset = opn + OPCAP, *sorted = opset + OPCAP;
+  uint32_t *cnt_s = U, *off_s = U + R, *nz = U + 2 * R;
+  uint32_t *opb = U + 3 * R, *sorted = opb + OPCAP;
   for (uint32_t r0 = 0; r0 < n_ops; r0 += OPCAP) {
     const uint32_t m = min(OPCAP, n_ops - r0);
-    for (uint32_t s = tid; s < R; s += BUILD_NT) {
-      cnt_s[s] = 0;
-      off_s[s] = 0;
-    }
+    for (uint32_t s = tid; s < R; s += BUILD_NT) cnt_s[s] = 0;
     __syncthreads();
     for (uint32_t p = tid; p < m; p += BUILD_NT) {
       const uint32_t gp = r0 + p;
       uint32_t lo = 0, hi = ng;  // seg[lo] <= gp < seg[lo+1]
       while (hi - lo > 1) {
-        uint32_t mid = (lo + hi) >> 1;
+        const uint32_t mid = (lo + hi) >> 1;
         if (seg[mid] <= gp) lo = mid;
         else hi = mid;
       }
-      const uint32_t L = grp[lo];
-      const uint64_t base = a.stage_off[L];
-      const uint32_t idx = gp - seg[lo];
-      const uint32_t b = a.stage_norm[base + idx];
-      const uint32_t nx = (gp + 1 < seg[lo + 1]) ? a.stage_norm[base + idx + 1] : NONE;
-      const uint32_t s = row_of(g, b);
+      const uint32_t b = a.stage_norm[a.stage_off[grp[lo]] + (gp - seg[lo])];
       opb[p] = b;
-      opn[p] = nx;
-      opset[p] = s;
-      atomicAdd(&cnt_s[s], 1u);
+      atomicAdd(&cnt_s[row_of(g, b)], 1u);
     }
     __syncthreads();
     {
-      // exclusive scan of cnt_s over R sets (each thread a contiguous chunk)
+      // exclusive scan of op counts and of non-empty sets (packed), each
+      // thread a contiguous chunk of sets; non-empty sets listed in set order
       const uint32_t per = (R + BUILD_NT - 1) / BUILD_NT;
-      const uint32_t s0 = tid * per, s1 = min(R, s0 + per);
-      uint32_t loc = 0;
-      for (uint32_t s = s0; s < s1; ++s) loc += cnt_s[s];
-      uint32_t tot;
-      uint32_t pre = block_excl_scan(loc, ws, &tot);
+      const uint32_t s0 = min(R, tid * per), s1 = min(R, s0 + per);
+      uint32_t lo_ops = 0, lo_nz = 0;
       for (uint32_t s = s0; s < s1; ++s) {
-        off_s[s] = pre;
-        pre += cnt_s[s];
+        lo_ops += cnt_s[s];
+        lo_nz += cnt_s[s] != 0;
       }
+      uint32_t tot;
+      const uint32_t pre = block_excl_scan((lo_nz << 16) | lo_ops, ws, &tot);
+      uint32_t po = pre & 0xFFFFu, pz = pre >> 16;
+      for (uint32_t s = s0; s < s1; ++s) {
+        const uint32_t c = cnt_s[s];
+        off_s[s] = po;
+        po += c;
+        if (c) nz[pz++] = s;
+      }
+      if (tid == 0) s_nnz = tot >> 16;
     }
     __syncthreads();
     for (uint32_t p = tid; p < m; p += BUILD_NT) {
-      const uint32_t s = opset[p];
-      const uint32_t pos = atomicAdd(&off_s[s], 1u);  // off_s becomes the bucket end
+      const uint32_t pos = atomicAdd(&off_s[row_of(g, opb[p])], 1u);  // off_s becomes the bucket end
       sorted[pos] = p;
     }
     __syncthreads();
-    for (uint32_t s = tid; s < R; s += BUILD_NT) {
-      const uint32_t c = cnt_s[s];
-      if (c == 0) continue;
-      const uint32_t e1 = off_s[s], b0 = e1 - c;
-      // insertion sort of the bucket by op position (buckets are tiny)
-      for (uint32_t u = b0 + 1; u < e1; ++u) {
-        uint32_t v = sorted[u];
-        uint32_t w = u;
-        while (w > b0 && sorted[w - 1] > v) {
-          sorted[w] = sorted[w - 1];
-          --w;
+    const uint32_t n_nz = s_nnz;
+    if (tid == 0) s_sets += n_nz;
+    for (uint32_t k0 = tid; k0 < n_nz; k0 += BUILD_NT * OWN_B) {
+      RegSet<MAXA, MAXS> rs[OWN_B];
+      uint32_t sid[OWN_B];
+#pragma unroll
+      for (int q = 0; q < OWN_B; ++q) {  // issue every set load of the batch first
+        const uint32_t k = k0 + q * BUILD_NT;
+        sid[q] = k < n_nz ? nz[k] : NONE;
+        if (sid[q] != NONE) rs[q].load(tbl_e + (uint64_t)sid[q] * g.stride, A, S);
+      }
+#pragma unroll
+      for (int q = 0; q < OWN_B; ++q) {
+        if (sid[q] == NONE) continue;
+        const uint32_t sset = sid[q];
+        const uint32_t e1 = off_s[sset], b0 = e1 - cnt_s[sset];
+        for (uint32_t u = b0 + 1; u < e1; ++u) {  // insertion sort of the (tiny) bucket
+          const uint32_t v = sorted[u];
+          uint32_t w = u;
+          while (w > b0 && sorted[w - 1] > v) {
+            sorted[w] = sorted[w - 1];
+            --w;
+          }
+          sorted[w] = v;
         }
-        sorted[w] = v;
+        for (uint32_t u = b0; u < e1; ++u) {
+          const uint32_t p = sorted[u];
+          const uint32_t gp = r0 + p;
+          rs[q].touch(opb[p], A);
+          // the next record of the same launch (ops of a launch are contiguous)
+          uint32_t lo = 0, hi = ng;
+          while (hi - lo > 1) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (seg[mid] <= gp) lo = mid;
+            else hi = mid;
+          }
+          if (gp + 1 < seg[lo + 1]) {
+            const uint32_t nx = (p + 1 < m) ? opb[p + 1]
+                                            : a.stage_norm[a.stage_off[grp[lo]] + (gp + 1 - seg[lo])];
+            rs[q].insert0(nx, S);
+          }
+        }
+        rs[q].store(tbl_e + (uint64_t)sset * g.stride, A, S);
+        if (use_rc) {
+          // row cache for the walk: final rows of the latest launch's blocks
+          for (uint32_t u = b0; u < e1; ++u) {
+            const uint32_t p = sorted[u];
+            if (r0 + p < last_seg) continue;
+            const uint32_t i = r0 + p - last_seg;
+            rs[q].export_row(opb[p], A, S, rc + i * (1 + S));
+          }
+        }
       }
-      atomicAdd(&s_sets, 1u);
-      RegSet<MAXA, MAXS> rs;
-      uint32_t *sp = tbl_e + (uint64_t)s * g.stride;
-      rs.load(sp, A, S);
-      for (uint32_t u = b0; u < e1; ++u) {
-        const uint32_t p = sorted[u];
-        rs.touch(opb[p], A);
-        if (opn[p] != NONE) rs.insert0(opn[p], S);
-      }
-      rs.store(sp, A, S);
     }
     __syncthreads();
   }
-
   if (tid == 0) {
     ctr_add(a.st, DUM_CTR_EXEC_BUILT, 1);
     ctr_add(a.st, DUM_CTR_OPS, n_ops);
     ctr_add(a.st, DUM_CTR_SETS, s_sets);
   }
   // ---- Start / End from the latest launch (D11) ----
-  const uint32_t Llast = grp[ng - 1];
-  const uint64_t cbase = a.stage_off[Llast];
-  const uint32_t n = a.stage_cnt[Llast];
-  const uint32_t *C = a.stage_norm + cbase;
+  const uint32_t *C = a.stage_norm + a.stage_off[Llast];
   const uint32_t start = C[0], end = C[n - 1];
   if (tid == 0) {
     a.start_end[2 * e] = start;
@@ -366,19 +428,34 @@ __global__ void __launch_bounds__(BUILD_NT) k_apply_walk(BuildArgs a) {
     }
     return;
   }
-  __syncthreads();  // table writes of this CTA visible to its own reads below
+  // row i of the chain: pointer to its successor list (row cache or table)
+  // and its successor count; NONE count = row missing
+  auto row_at = [&](uint32_t i, const uint32_t *&sc) -> uint32_t {
+    if (use_rc) {
+      sc = rc + i * (1 + S) + 1;
+      return rc[i * (1 + S)];
+    }
+    const uint32_t x = C[i];
+    const uint32_t *set = tbl_e + (uint64_t)row_of(g, x) * g.stride;
+    int w = -1;
+    for (uint32_t q = 0; q < A; ++q)
+      if (w < 0 && __ldcg(set + q * (1 + S)) == x) w = (int)q;
+    if (w < 0) return NONE;
+    sc = set + w * (1 + S) + 1;
+    uint32_t cnt = 0;
+    while (cnt < S && __ldcg(sc + cnt) != NONE) ++cnt;
+    return cnt;
+  };
 
   // ---- pass A: per chain position i < n-1: row present? stop? successor count ----
   uint32_t *cq;
   if (n <= WCAP) {
-    cq = U;
+    cq = cqs;
   } else {
-    unsigned long long need = n;
-    unsigned long long off = 0;
     if (tid == 0) {
-      off = atomicAdd(&a.st->pool_big, need);
-      s_flag = off + need <= a.big_entries * 2 ? (uint32_t)0 : 1u;
-      s_tev = (uint32_t)off;  // temporarily
+      const unsigned long long off = atomicAdd(&a.st->pool_big, (unsigned long long)n);
+      s_flag = off + n <= a.big_entries * 2 ? 0u : 1u;
+      s_tev = (uint32_t)off;
     }
     __syncthreads();
     if (s_flag) {
@@ -391,28 +468,19 @@ __global__ void __launch_bounds__(BUILD_NT) k_apply_walk(BuildArgs a) {
   if (tid == 0) s_tev = NONE;
   __syncthreads();
   for (uint32_t i = tid; i < n - 1; i += BUILD_NT) {
-    const uint32_t x = C[i];
-    const uint32_t *set = tbl_e + (uint64_t)row_of(g, x) * g.stride;
-    int w = -1;
-    for (uint32_t q = 0; q < A; ++q)
-      if (w < 0 && __ldcg(set + q * (1 + S)) == x) w = (int)q;
-    uint32_t ev = 0, cnt = 0;
-    if (w < 0) {
+    const uint32_t *sc = nullptr;
+    const uint32_t cnt = row_at(i, sc);
+    uint32_t ev = 0;
+    if (cnt == NONE) {
       ev = 1;  // row missing: stop, nothing emitted at this step
+      cq[i] = 0;
     } else {
-      const uint32_t *sc = set + w * (1 + S) + 1;
       bool hit = false;
-      for (uint32_t q = 0; q < S; ++q) {
-        uint32_t v = __ldcg(sc + q);
-        if (v == NONE) break;
-        hit |= v == end;
-        ++cnt;
-      }
-      const uint32_t s0 = cnt ? __ldcg(sc) : NONE;
-      if (hit) ev = 2;                      // a successor is End: stop after emitting
-      else if (s0 != C[i + 1]) ev = 3;      // speculation violated -> sequential walker
+      for (uint32_t q = 0; q < cnt; ++q) hit |= sc[q] == end;
+      if (hit) ev = 2;                                   // a successor is End: stop after emitting
+      else if (cnt == 0 || sc[0] != C[i + 1]) ev = 3;    // speculation violated -> sequential walker
+      cq[i] = cnt;
     }
-    cq[i] = cnt;
     if (ev) atomicMin(&s_tev, (i << 2) | ev);
   }
   __syncthreads();
@@ -422,8 +490,6 @@ __global__ void __launch_bounds__(BUILD_NT) k_apply_walk(BuildArgs a) {
     return;
   }
   const uint32_t t = tev >> 2;
-  if ((tev & 3) == 1 && tid == 0) cq[t] = 0;
-  __syncthreads();
   // ---- pass B: Q positions (qpos[i] = 1 + sum cq[0..i)) in place ----
   uint32_t run = 1;
   for (uint32_t c = 0; c <= t; c += BUILD_NT) {
@@ -437,13 +503,13 @@ __global__ void __launch_bounds__(BUILD_NT) k_apply_walk(BuildArgs a) {
   const uint32_t qlen = run;  // |Q|
   // dedupe map block -> min Q position
   uint32_t *qk, *qv;
-  uint32_t qcap = pow2ceil(2 * qlen);
+  const uint32_t qcap = pow2ceil(2 * qlen);
   if (qcap <= QCAP) {
-    qk = U + WCAP;
+    qk = U;
     qv = qk + qcap;
   } else {
     if (tid == 0) {
-      unsigned long long off = atomicAdd(&a.st->pool_big, 2ull * qcap);
+      const unsigned long long off = atomicAdd(&a.st->pool_big, 2ull * qcap);
       s_flag = off + 2ull * qcap <= a.big_entries * 2 ? 0u : 1u;
       s_tev = (uint32_t)off;
     }
@@ -465,13 +531,9 @@ __global__ void __launch_bounds__(BUILD_NT) k_apply_walk(BuildArgs a) {
     const uint32_t q0 = cq[i];
     const uint32_t qn = (i < t ? cq[i + 1] : qlen) - q0;
     if (qn == 0) continue;
-    const uint32_t x = C[i];
-    const uint32_t *set = tbl_e + (uint64_t)row_of(g, x) * g.stride;
-    uint32_t w = 0;
-    for (uint32_t q = 0; q < A; ++q)
-      if (__ldcg(set + q * (1 + S)) == x) w = q;
-    const uint32_t *sc = set + w * (1 + S) + 1;
-    for (uint32_t q = 0; q < qn; ++q) hmap_insert_min(qk, qv, qcap, __ldcg(sc + q), q0 + q);
+    const uint32_t *sc = nullptr;
+    row_at(i, sc);
+    for (uint32_t q = 0; q < qn; ++q) hmap_insert_min(qk, qv, qcap, sc[q], q0 + q);
   }
   __syncthreads();
   // ---- pass C: ordered compaction of first occurrences ----
@@ -483,18 +545,15 @@ __global__ void __launch_bounds__(BUILD_NT) k_apply_walk(BuildArgs a) {
       if (p == 0) {
         val = start;
       } else {
-        uint32_t lo = 0, hi = t + 1;  // cq[lo] <= p < next
+        uint32_t lo = 0, hi = t + 1;  // largest lo with cq[lo] <= p
         while (hi - lo > 1) {
-          uint32_t mid = (lo + hi) >> 1;
+          const uint32_t mid = (lo + hi) >> 1;
           if (cq[mid] <= p) lo = mid;
           else hi = mid;
         }
-        const uint32_t x = C[lo];
-        const uint32_t *set = tbl_e + (uint64_t)row_of(g, x) * g.stride;
-        uint32_t w = 0;
-        for (uint32_t q = 0; q < A; ++q)
-          if (__ldcg(set + q * (1 + S)) == x) w = q;
-        val = __ldcg(set + w * (1 + S) + 1 + (p - cq[lo]));
+        const uint32_t *sc = nullptr;
+        row_at(lo, sc);
+        val = sc[p - cq[lo]];
       }
       keep = hmap_get(qk, qv, qcap, val) == p;
     }
@@ -531,8 +590,7 @@ __global__ void k_walk_slow(Geo g, const uint32_t *tbl, const uint32_t *start_en
 
 template <int MA, int MS>
 static cudaError_t launch_apply(dum_engine *e, const BuildArgs &ba, cudaStream_t s) {
-  const size_t smem = (size_t)(2 * GCAP + 1) * 4 +
-                      (size_t)std::max<uint32_t>(2 * ba.g.R + 4 * OPCAP, WCAP + 2 * QCAP) * 4;
+  const size_t smem = (size_t)(2 * GCAP + 1 + RCCAP + WCAP + apply_union_words(ba.g.R)) * 4;
   cudaFuncSetAttribute(k_apply_walk<MA, MS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   k_apply_walk<MA, MS><<<ba.n_staged, BUILD_NT, smem, s>>>(ba);
   return cudaGetLastError();

@@ -71,7 +71,18 @@ __global__ void k_anchor_walk(Geo g, const dum_query *__restrict__ q, uint32_t n
                               uint64_t *range, WalkScratch ws, DevState *st) {
   const uint32_t E = *(volatile uint32_t *)&st->E;
   uint32_t *out = slot_out + (uint64_t)blockIdx.x * g.walk_cap;
-  for (uint32_t qi = blockIdx.x; qi < nq; qi += gridDim.x) {
+  const uint32_t lane = threadIdx.x & 31;
+  for (uint32_t q0 = blockIdx.x * 32; q0 < nq; q0 += gridDim.x * 32) {
+   // lanes test 32 queries at once; anchored ones are walked one after another
+   const bool anch = q0 + lane < nq && q[q0 + lane].anchor != NONE;
+   if (!anch && q0 + lane < nq) {
+     range[2 * (q0 + lane)] = 0;
+     range[2 * (q0 + lane) + 1] = 0;
+   }
+   uint32_t todo = __ballot_sync(0xffffffffu, anch);
+   while (todo) {
+    const uint32_t qi = q0 + __ffs(todo) - 1;
+    todo &= todo - 1;
     const dum_query Q = q[qi];
     uint32_t n = 0;
     if (Q.anchor != NONE && Q.exec < E) {
@@ -96,6 +107,7 @@ __global__ void k_anchor_walk(Geo g, const dum_query *__restrict__ q, uint32_t n
       range[2 * qi + 1] = n;
     }
     __syncwarp();
+   }
   }
 }
 
@@ -122,9 +134,10 @@ struct PredArgs {
   SelectOut so;     // fused a8 outputs (SELECT only)
 };
 
-constexpr int CHAIN_NT = 128;
+constexpr int CHAIN_NT = 64;
 
 __global__ void __launch_bounds__(CHAIN_NT) k_chain(PredArgs a) {
+  __shared__ uint32_t skern[CHAIN_NT][MAXN + 1];  // per-thread chain (repeat check stays on chip)
   const uint32_t qi = blockIdx.x * CHAIN_NT + threadIdx.x;
   const uint32_t lane = threadIdx.x & 31;
   const Geo &g = a.g;
@@ -133,33 +146,37 @@ __global__ void __launch_bounds__(CHAIN_NT) k_chain(PredArgs a) {
     const dum_query Q = a.q[qi];
     const bool anchored = Q.anchor != NONE;
     const uint32_t E = *(volatile uint32_t *)&a.st->E;
-    uint32_t *kern = a.qkern + (uint64_t)qi * (g.N + 1);
+    uint32_t *kern = skern[threadIdx.x];
+    uint32_t *gkern = a.qkern + (uint64_t)qi * (g.N + 1);
     uint32_t *loff = a.qloff + (uint64_t)qi * (g.N + 2);
     uint32_t nk = 0;
-    loff[0] = 0;
-    auto add = [&](uint32_t e) {
-      uint32_t len = (nk == 0 && anchored) ? (uint32_t)a.anchor_range[2 * qi + 1] : a.walk_len[e];
-      // a kernel met earlier in the chain with the same (unanchored) walk
-      // cannot add anything (exact; keeps the reservation tight)
-      for (uint32_t d2 = anchored ? 1u : 0u; d2 < nk && len; ++d2)
-        if (kern[d2] == e) len = 0;
-      kern[nk] = e;
-      U += len;
-      loff[++nk] = U;
-    };
     if (Q.exec < E) {
+      // the serial part: only the dependent lookups
       const uint32_t n = Q.n < g.N ? Q.n : g.N;
       uint32_t cur = Q.exec, h1 = Q.hist[0], h2 = Q.hist[1], h3 = Q.hist[2];
-      add(cur);
+      kern[nk++] = cur;
       for (uint32_t i = 0; i < n; ++i) {
         const uint32_t nx = corr_lookup(a.corr, a.corr_cap, cur, h1, h2, h3);
         if (nx == NONE) break;
-        add(nx);
+        kern[nk++] = nx;
         h1 = h2;  // D16: shift register over predicted IDs
         h2 = h3;
         h3 = cur;
         cur = nx;
       }
+    }
+    // window layout: walk lengths (independent loads), a kernel met earlier in
+    // the chain with the same (unanchored) walk adds nothing (exact; keeps the
+    // reservation tight)
+    loff[0] = 0;
+    for (uint32_t d = 0; d < nk; ++d) {
+      const uint32_t e = kern[d];
+      uint32_t len = (d == 0 && anchored) ? (uint32_t)a.anchor_range[2 * qi + 1] : __ldg(a.walk_len + e);
+      for (uint32_t d2 = anchored ? 1u : 0u; d2 < d && len; ++d2)
+        if (kern[d2] == e) len = 0;
+      gkern[d] = e;
+      U += len;
+      loff[d + 1] = U;
     }
     a.qnk[qi] = nk;
   }
