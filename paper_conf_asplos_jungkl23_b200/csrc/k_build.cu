@@ -26,7 +26,7 @@
 namespace dum {
 
 constexpr int BUILD_NT = 512;
-constexpr uint32_t GCAP = 1024;   // launches of one exec ID per build batch
+constexpr uint32_t GCAP = 512;    // launches of one exec ID per build batch
 constexpr uint32_t OPCAP = 2048;  // ops per apply round
 constexpr uint32_t QCAP = 4096;   // smem walk-dedupe hash capacity (|Q| <= 2048)
 constexpr uint32_t WCAP = 2048;   // smem per-row counts (latest launch <= 2048 faults)
@@ -226,15 +226,21 @@ struct BuildArgs {
 // arrays (per-set counts/offsets, non-empty-set list, ops, op order) and the
 // walk's dedupe hash.
 constexpr uint32_t RCCAP = 10240;  // row-cache words: n * (1 + S) <= RCCAP
+constexpr uint32_t HCAPMAX = 2 * OPCAP;  // set-hash capacity for a full round
 
-__host__ __device__ inline uint32_t apply_union_words(uint32_t R) {
-  const uint32_t ap = 3 * R + 2 * OPCAP, wk = 2 * QCAP;
+__host__ __device__ inline uint32_t apply_union_words(uint32_t) {
+  const uint32_t ap = 2 * HCAPMAX + 3 * OPCAP, wk = 2 * QCAP;
   return ap > wk ? ap : wk;
 }
 
+// link op p at the head of its set's list (order fixed up by the owner)
+__device__ __forceinline__ void sorted_link(uint32_t p, uint32_t slot, uint32_t *hh, uint32_t *lnk) {
+  lnk[p] = atomicExch(&hh[slot], p);
+}
+
 template <int MAXA, int MAXS>
-__global__ void __launch_bounds__(BUILD_NT) k_apply_walk(BuildArgs a) {
-  constexpr int OWN_B = (MAXA * (1 + MAXS) <= 10) ? 4 : 1;  // sets loaded per owner batch
+__global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
+  constexpr int OWN_B = (MAXA * (1 + MAXS) <= 10) ? 2 : 1;  // sets loaded per owner batch
   extern __shared__ uint32_t sm[];
   __shared__ uint32_t ws[BUILD_NT / 32];
   __shared__ uint32_t s_ng, s_tev, s_flag, s_sets, s_nnz;
@@ -304,12 +310,21 @@ __global__ void __launch_bounds__(BUILD_NT) k_apply_walk(BuildArgs a) {
   const bool use_rc = single_round && n <= WCAP && n * (1 + S) <= RCCAP;
   uint32_t *tbl_e = a.tbl + (uint64_t)e * R * g.stride;
 
-  // ---- apply: rounds of up to OPCAP ops, counting-sorted by set ----
-  uint32_t *cnt_s = U, *off_s = U + R, *nz = U + 2 * R;
-  uint32_t *opb = U + 3 * R, *sorted = opb + OPCAP;
+  // ---- apply: rounds of up to OPCAP ops, grouped by set ----
+  // Each op (fused TOUCH b_p + INSERT b_p -> b_{p+1}) is linked into its set's
+  // list through a shared hash keyed by set index (O(ops), independent of R);
+  // the owner of a set collects the set's ops, orders them by position (lists
+  // are tiny), loads the set into registers, applies them and stores it.
+  uint32_t *hk = U, *hh = U + HCAPMAX;          // set key, list head
+  uint32_t *opb = U + 2 * HCAPMAX, *onx = opb + OPCAP;
   for (uint32_t r0 = 0; r0 < n_ops; r0 += OPCAP) {
     const uint32_t m = min(OPCAP, n_ops - r0);
-    for (uint32_t s = tid; s < R; s += BUILD_NT) cnt_s[s] = 0;
+    uint32_t hcap = pow2ceil(2 * m);
+    if (hcap < 64) hcap = 64;
+    for (uint32_t p = tid; p < hcap; p += BUILD_NT) {
+      hk[p] = NONE;
+      hh[p] = NONE;
+    }
     __syncthreads();
     for (uint32_t p = tid; p < m; p += BUILD_NT) {
       const uint32_t gp = r0 + p;
@@ -319,92 +334,62 @@ __global__ void __launch_bounds__(BUILD_NT) k_apply_walk(BuildArgs a) {
         if (seg[mid] <= gp) lo = mid;
         else hi = mid;
       }
-      const uint32_t b = a.stage_norm[a.stage_off[grp[lo]] + (gp - seg[lo])];
+      const uint64_t base = a.stage_off[grp[lo]] + (gp - seg[lo]);
+      const uint32_t b = a.stage_norm[base];
+      // successor within the same launch (ops of a launch are contiguous)
+      const uint32_t nx = (gp + 1 < seg[lo + 1]) ? a.stage_norm[base + 1] : NONE;
       opb[p] = b;
-      atomicAdd(&cnt_s[row_of(g, b)], 1u);
-    }
-    __syncthreads();
-    {
-      // exclusive scan of op counts and of non-empty sets (packed), each
-      // thread a contiguous chunk of sets; non-empty sets listed in set order
-      const uint32_t per = (R + BUILD_NT - 1) / BUILD_NT;
-      const uint32_t s0 = min(R, tid * per), s1 = min(R, s0 + per);
-      uint32_t lo_ops = 0, lo_nz = 0;
-      for (uint32_t s = s0; s < s1; ++s) {
-        lo_ops += cnt_s[s];
-        lo_nz += cnt_s[s] != 0;
+      const uint32_t key = row_of(g, b);
+      uint32_t sl = hslot(key, hcap);
+      for (;;) {
+        const uint32_t old = atomicCAS(&hk[sl], NONE, key);
+        if (old == NONE || old == key) break;
+        sl = (sl + 1) & (hcap - 1);
       }
-      uint32_t tot;
-      const uint32_t pre = block_excl_scan((lo_nz << 16) | lo_ops, ws, &tot);
-      uint32_t po = pre & 0xFFFFu, pz = pre >> 16;
-      for (uint32_t s = s0; s < s1; ++s) {
-        const uint32_t c = cnt_s[s];
-        off_s[s] = po;
-        po += c;
-        if (c) nz[pz++] = s;
-      }
-      if (tid == 0) s_nnz = tot >> 16;
+      onx[p] = nx;
+      sorted_link(p, sl, hh, U + 2 * HCAPMAX + 2 * OPCAP);
     }
     __syncthreads();
-    for (uint32_t p = tid; p < m; p += BUILD_NT) {
-      const uint32_t pos = atomicAdd(&off_s[row_of(g, opb[p])], 1u);  // off_s becomes the bucket end
-      sorted[pos] = p;
-    }
-    __syncthreads();
-    const uint32_t n_nz = s_nnz;
-    if (tid == 0) s_sets += n_nz;
-    for (uint32_t k0 = tid; k0 < n_nz; k0 += BUILD_NT * OWN_B) {
+    uint32_t *lnk = U + 2 * HCAPMAX + 2 * OPCAP;  // per-op next pointer of its set list
+    uint32_t nsets = 0;
+    for (uint32_t k0 = tid; k0 < hcap; k0 += BUILD_NT * OWN_B) {
       RegSet<MAXA, MAXS> rs[OWN_B];
-      uint32_t sid[OWN_B];
+      uint32_t sid[OWN_B], head[OWN_B];
 #pragma unroll
       for (int q = 0; q < OWN_B; ++q) {  // issue every set load of the batch first
         const uint32_t k = k0 + q * BUILD_NT;
-        sid[q] = k < n_nz ? nz[k] : NONE;
+        sid[q] = k < hcap ? hk[k] : NONE;
+        head[q] = k < hcap ? hh[k] : NONE;
         if (sid[q] != NONE) rs[q].load(tbl_e + (uint64_t)sid[q] * g.stride, A, S);
       }
 #pragma unroll
       for (int q = 0; q < OWN_B; ++q) {
         if (sid[q] == NONE) continue;
-        const uint32_t sset = sid[q];
-        const uint32_t e1 = off_s[sset], b0 = e1 - cnt_s[sset];
-        for (uint32_t u = b0 + 1; u < e1; ++u) {  // insertion sort of the (tiny) bucket
-          const uint32_t v = sorted[u];
-          uint32_t w = u;
-          while (w > b0 && sorted[w - 1] > v) {
-            sorted[w] = sorted[w - 1];
-            --w;
-          }
-          sorted[w] = v;
+        ++nsets;
+        // the set's ops in position order: repeatedly take the smallest
+        // remaining position from the (short) list
+        uint32_t last = 0xFFFFFFFFu;
+        for (;;) {
+          uint32_t best = NONE;
+          for (uint32_t x = head[q]; x != NONE; x = lnk[x])
+            if ((last == 0xFFFFFFFFu || x > last) && (best == NONE || x < best)) best = x;
+          if (best == NONE) break;
+          rs[q].touch(opb[best], A);
+          if (onx[best] != NONE) rs[q].insert0(onx[best], S);
+          last = best;
         }
-        for (uint32_t u = b0; u < e1; ++u) {
-          const uint32_t p = sorted[u];
-          const uint32_t gp = r0 + p;
-          rs[q].touch(opb[p], A);
-          // the next record of the same launch (ops of a launch are contiguous)
-          uint32_t lo = 0, hi = ng;
-          while (hi - lo > 1) {
-            const uint32_t mid = (lo + hi) >> 1;
-            if (seg[mid] <= gp) lo = mid;
-            else hi = mid;
-          }
-          if (gp + 1 < seg[lo + 1]) {
-            const uint32_t nx = (p + 1 < m) ? opb[p + 1]
-                                            : a.stage_norm[a.stage_off[grp[lo]] + (gp + 1 - seg[lo])];
-            rs[q].insert0(nx, S);
-          }
-        }
-        rs[q].store(tbl_e + (uint64_t)sset * g.stride, A, S);
+        rs[q].store(tbl_e + (uint64_t)sid[q] * g.stride, A, S);
         if (use_rc) {
           // row cache for the walk: final rows of the latest launch's blocks
-          for (uint32_t u = b0; u < e1; ++u) {
-            const uint32_t p = sorted[u];
-            if (r0 + p < last_seg) continue;
-            const uint32_t i = r0 + p - last_seg;
-            rs[q].export_row(opb[p], A, S, rc + i * (1 + S));
+          for (uint32_t x = head[q]; x != NONE; x = lnk[x]) {
+            if (r0 + x < last_seg) continue;
+            const uint32_t i = r0 + x - last_seg;
+            rs[q].export_row(opb[x], A, S, rc + i * (1 + S));
           }
         }
       }
     }
+    if (nsets) atomicAdd(&s_sets, nsets);
     __syncthreads();
   }
   if (tid == 0) {
@@ -592,6 +577,8 @@ template <int MA, int MS>
 static cudaError_t launch_apply(dum_engine *e, const BuildArgs &ba, cudaStream_t s) {
   const size_t smem = (size_t)(2 * GCAP + 1 + RCCAP + WCAP + apply_union_words(ba.g.R)) * 4;
   cudaFuncSetAttribute(k_apply_walk<MA, MS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaFuncSetAttribute(k_apply_walk<MA, MS>, cudaFuncAttributePreferredSharedMemoryCarveout,
+                       cudaSharedmemCarveoutMaxShared);
   k_apply_walk<MA, MS><<<ba.n_staged, BUILD_NT, smem, s>>>(ba);
   return cudaGetLastError();
 }
