@@ -56,6 +56,7 @@ def parse():
     ap.add_argument("--cpu-launches", type=int, default=0, help="oracle sample size in launches")
     ap.add_argument("--json-out", default="")
     ap.add_argument("--unfused", action="store_true", help="separate predict / select calls")
+    ap.add_argument("--debug", action="store_true", help="synchronize and check after every call")
     return ap.parse_args()
 
 
@@ -270,15 +271,25 @@ def run_ours(args, rank, world, local_rank):
         wb[0] = torch.empty(cap[0], dtype=torch.int32, device=dev)
         inv[0] = torch.empty(cap[0], dtype=torch.int32, device=dev)
 
+    def dbg(what):
+        if args.debug:
+            try:
+                eng.sync()
+            except B.EngineError as e:
+                raise SystemExit("device error after %s (iteration %d): %s" % (what, dbg.i, e))
+
     def step(i, host=None):
         """record(i) -> queries -> predict(i) -> select(i) -> build(i)"""
+        dbg.i = i
         out_exec = exec_all[3 + i * K: 3 + (i + 1) * K]
         if host is None:
             eng.record_faults(hs[i], offs[i], fs[i], out_exec)
         else:
             eng.record_faults(host[0][i], host[1][i], host[2][i], out_exec)
+        dbg("record_faults")
         if i >= 1:
             eng.make_queries(exec_all[i * K: 3 + (i + 1) * K], 3, N, out=qbuf)
+            dbg("make_queries")
             if args.unfused:
                 eng.predict_prefetch(qbuf, cap[0], pairs=pairs[0], rng=rng, kern_off=ko, chain=ch, needed=need_p)
                 eng.select_evictions(rng, pairs[0], qbuf, cap[0], wb=wb[0], inv=inv[0], out_rng=srng,
@@ -286,7 +297,9 @@ def run_ours(args, rank, world, local_rank):
             else:
                 eng.predict_select(qbuf, cap[0], cap[0], pairs=pairs[0], rng=rng, kern_off=ko, chain=ch,
                                    needed=need_p, wb=wb[0], inv=inv[0], sel_rng=srng, sel_needed=need_s)
+            dbg("predict")
         eng.build_tables()
+        dbg("build_tables")
 
     def pre_step(i):
         eng.set_timing(False)

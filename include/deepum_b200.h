@@ -256,6 +256,8 @@ typedef struct {
   uint64_t staged_faults;
   uint32_t slow_walks;      /* walks that took the sequential fallback in the last build */
   uint32_t n_resident;
+  uint32_t guard_line;      /* first failed internal consistency guard (0 = none) */
+  uint32_t guard_val;
 } dum_stats;
 /* Synchronizes. */
 int dum_get_stats(dum_engine *eng, dum_stats *out);

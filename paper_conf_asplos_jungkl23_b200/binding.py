@@ -11,7 +11,7 @@ import numpy as np
 import torch
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-_LIBPATH = os.path.join(HERE, "libdeepum_b200.so")
+_LIBPATH = os.environ.get("DUM_LIB") or os.path.join(HERE, "libdeepum_b200.so")
 
 DUM_NONE = NONE = 0xFFFFFFFF
 DUM_HOST_PTRS = 0x1
@@ -54,6 +54,7 @@ class DumStats(ctypes.Structure):
         ("num_exec", ctypes.c_uint32), ("corr_records", ctypes.c_uint32), ("free_frames", ctypes.c_uint32),
         ("staged_launches", ctypes.c_uint32), ("launches", ctypes.c_uint64), ("staged_faults", ctypes.c_uint64),
         ("slow_walks", ctypes.c_uint32), ("n_resident", ctypes.c_uint32),
+        ("guard_line", ctypes.c_uint32), ("guard_val", ctypes.c_uint32),
     ]
 
 

@@ -36,15 +36,17 @@ def up_to_date() -> bool:
     return all(os.path.getmtime(p) <= t for p in _deps())
 
 
-def build(force: bool = False, verbose: bool = False, ptxas_v: bool = False) -> str:
-    if not force and up_to_date():
+def build(force: bool = False, verbose: bool = False, ptxas_v: bool = False, checks: bool = False) -> str:
+    out = OUT if not checks else OUT.replace(".so", "_checks.so")
+    if not force and not checks and up_to_date():
         return OUT
-    os.makedirs(BUILD, exist_ok=True)
+    bdir = BUILD if not checks else BUILD + "_checks"
+    os.makedirs(bdir, exist_ok=True)
     objs = []
 
     def one(src):
-        obj = os.path.join(BUILD, os.path.basename(src) + ".o")
-        cmd = [NVCC, *ARCH, *FLAGS, "-c", src, "-o", obj]
+        obj = os.path.join(bdir, os.path.basename(src) + ".o")
+        cmd = [NVCC, *ARCH, *FLAGS, "-c", src, "-o", obj] + (["-DDUM_CHECKS", "-DDUM_POISON"] if checks else [])
         if ptxas_v:
             cmd[1:1] = ["-Xptxas", "-v"]
         r = subprocess.run(cmd, capture_output=True, text=True)
@@ -56,14 +58,15 @@ def build(force: bool = False, verbose: bool = False, ptxas_v: bool = False) -> 
 
     with cf.ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 2)) as ex:
         objs = list(ex.map(one, _sources()))
-    tmp = OUT + ".tmp%d" % os.getpid()
+    tmp = out + ".tmp%d" % os.getpid()
     cmd = [NVCC, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError("link failed:\n%s\n%s" % (r.stdout, r.stderr))
-    os.replace(tmp, OUT)
-    return OUT
+    os.replace(tmp, out)
+    return out
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="--verbose" in sys.argv, ptxas_v="-v" in sys.argv))
+    print(build(force="--force" in sys.argv, verbose="--verbose" in sys.argv, ptxas_v="-v" in sys.argv,
+                checks="--checks" in sys.argv))

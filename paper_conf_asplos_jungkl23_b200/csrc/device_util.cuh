@@ -7,6 +7,29 @@
 
 namespace dum {
 
+#ifdef DUM_CHECKS
+#define DCHECK(cond, ...)                                                        \
+  do {                                                                           \
+    if (!(cond)) {                                                               \
+      printf("DCHECK %s:%d block %d thread %d: %s\n", __FILE__, __LINE__,        \
+             (int)blockIdx.x, (int)threadIdx.x, #cond);                          \
+      printf(__VA_ARGS__);                                                       \
+      __trap();                                                                  \
+    }                                                                            \
+  } while (0)
+#else
+#define DCHECK(cond, ...) \
+  do {                    \
+  } while (0)
+#endif
+
+// Internal consistency guard: records the first failure (line, value) in the
+// device state; the caller clamps/skips the offending access.
+#define GUARD(st, cond, val)                                          \
+  ((cond) ? true : (atomicCAS(&(st)->dbg_line, 0u, (uint32_t)__LINE__) == 0u \
+                        ? ((st)->dbg_val = (uint32_t)(val), false)    \
+                        : false))
+
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31; }
 __device__ __forceinline__ uint32_t warp_id() { return threadIdx.x >> 5; }
 

@@ -6,6 +6,7 @@
 // device snapshot for inspection.
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <vector>
@@ -41,6 +42,7 @@ __global__ void k_init_state(DevState *st) {
   st->corr_used = 0;
   st->mig_ok = 0;
   st->mig_n = 0;
+  st->dbg_line = st->dbg_val = 0;
   for (int c = 0; c < DUM_NCOUNTERS; ++c) st->ctr[c] = 0;
 }
 
@@ -145,6 +147,15 @@ TimerScope::TimerScope(dum_engine *e_, int id_, cudaStream_t s_) : e(e_), id(id_
 }
 TimerScope::~TimerScope() {
   if (b) cudaEventRecord(b, s);
+  static const bool sync_each = getenv("DUM_SYNC_EACH") != nullptr;
+  if (sync_each) {
+    cudaError_t err = cudaStreamSynchronize(s);
+    if (err == cudaSuccess) err = cudaGetLastError();
+    if (err != cudaSuccess) {
+      fprintf(stderr, "DUM_SYNC_EACH: kernel timer id %d failed: %s\n", id, cudaGetErrorString(err));
+      fflush(stderr);
+    }
+  }
 }
 }  // namespace dum
 
@@ -481,6 +492,8 @@ int dum_get_stats(dum_engine *e, dum_stats *out) {
   out->staged_faults = e->staged_faults;
   out->slow_walks = e->h_state->n_slow;
   out->n_resident = e->h_state->n_resident;
+  out->guard_line = e->h_state->dbg_line;
+  out->guard_val = e->h_state->dbg_val;
   return DUM_OK;
 }
 

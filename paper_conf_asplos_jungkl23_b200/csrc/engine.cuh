@@ -60,6 +60,7 @@ struct DevState {
   uint32_t mig_ok;            // last migrate validated
   uint32_t mig_n;             // blocks moved by the last migrate
   uint32_t log_dirty;         // LRM log may hold entries of evicted blocks
+  uint32_t dbg_line, dbg_val; // first failed internal guard (GUARD macro)
   unsigned long long ctr[DUM_NCOUNTERS];  // work counters (instrumentation)
 };
 

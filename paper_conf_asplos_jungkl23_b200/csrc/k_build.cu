@@ -259,7 +259,11 @@ __global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
   }
   const uint32_t e = a.stage_exec[j];
   if (e == NONE || a.stage_cnt[j] == 0) return;
-  if (__ldcg(&a.head[e]) != j) return;  // not this exec ID's group leader
+  // Leader test, decided once per CTA: thread 0 resets head[e] below, so a
+  // per-thread read could see the reset and drop part of the CTA.
+  if (tid == 0) s_flag = __ldcg(&a.head[e]) == j;
+  __syncthreads();
+  if (!s_flag) return;  // not this exec ID's group leader
 
   const uint32_t R = g.R, A = g.A, S = g.S;
   uint32_t *grp = sm;             // [GCAP]
@@ -267,11 +271,19 @@ __global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
   uint32_t *rc = seg + GCAP + 1;  // [RCCAP]
   uint32_t *cqs = rc + RCCAP;     // [WCAP]
   uint32_t *U = cqs + WCAP;       // union region
+#ifdef DUM_POISON
+  {
+    const uint32_t words = 2 * GCAP + 1 + RCCAP + WCAP + apply_union_words(R);
+    for (uint32_t w = tid; w < words; w += BUILD_NT) sm[w] = 0xDEAD0000u | (w & 0xFFFF);
+    __syncthreads();
+  }
+#endif
 
   // ---- collect and order the group's launches ----
   if (tid == 0) {
     uint32_t x = j, n = 0;
     while (x != NONE && n < GCAP) {
+      if (!GUARD(a.st, x < a.n_staged && a.stage_exec[x] == e, x)) break;
       grp[n++] = x;
       x = __ldcg(&a.next[x]);
     }
@@ -335,7 +347,8 @@ __global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
         else hi = mid;
       }
       const uint64_t base = a.stage_off[grp[lo]] + (gp - seg[lo]);
-      const uint32_t b = a.stage_norm[base];
+      uint32_t b = a.stage_norm[base];
+      if (!GUARD(a.st, b < g.W, b)) b = 0;
       // successor within the same launch (ops of a launch are contiguous)
       const uint32_t nx = (gp + 1 < seg[lo + 1]) ? a.stage_norm[base + 1] : NONE;
       opb[p] = b;
@@ -374,6 +387,7 @@ __global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
           for (uint32_t x = head[q]; x != NONE; x = lnk[x])
             if ((last == 0xFFFFFFFFu || x > last) && (best == NONE || x < best)) best = x;
           if (best == NONE) break;
+          if (!GUARD(a.st, best < m, best)) break;
           rs[q].touch(opb[best], A);
           if (onx[best] != NONE) rs[q].insert0(onx[best], S);
           last = best;
@@ -384,6 +398,7 @@ __global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
           for (uint32_t x = head[q]; x != NONE; x = lnk[x]) {
             if (r0 + x < last_seg) continue;
             const uint32_t i = r0 + x - last_seg;
+            if (!GUARD(a.st, i < n && (i + 1) * (1 + S) <= RCCAP, i)) continue;
             rs[q].export_row(opb[x], A, S, rc + i * (1 + S));
           }
         }
@@ -418,6 +433,7 @@ __global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
   auto row_at = [&](uint32_t i, const uint32_t *&sc) -> uint32_t {
     if (use_rc) {
       sc = rc + i * (1 + S) + 1;
+      DCHECK(rc[i * (1 + S)] == NONE || rc[i * (1 + S)] <= S, "rc[%u]=%x n=%u e=%u\n", i, rc[i * (1 + S)], n, e);
       return rc[i * (1 + S)];
     }
     const uint32_t x = C[i];
@@ -475,6 +491,10 @@ __global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
     return;
   }
   const uint32_t t = tev >> 2;
+  if (!GUARD(a.st, t + 1 < n, t)) {
+    if (tid == 0) a.slow_list[atomicAdd(&a.st->n_slow, 1u)] = e;
+    return;
+  }
   // ---- pass B: Q positions (qpos[i] = 1 + sum cq[0..i)) in place ----
   uint32_t run = 1;
   for (uint32_t c = 0; c <= t; c += BUILD_NT) {
@@ -486,6 +506,10 @@ __global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
     run += tot;
   }
   const uint32_t qlen = run;  // |Q|
+  if (!GUARD(a.st, qlen <= 1 + (t + 1) * S, qlen)) {
+    if (tid == 0) a.slow_list[atomicAdd(&a.st->n_slow, 1u)] = e;
+    return;
+  }
   // dedupe map block -> min Q position
   uint32_t *qk, *qv;
   const uint32_t qcap = pow2ceil(2 * qlen);
@@ -537,8 +561,8 @@ __global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
           else hi = mid;
         }
         const uint32_t *sc = nullptr;
-        row_at(lo, sc);
-        val = sc[p - cq[lo]];
+        const uint32_t cnt_lo = row_at(lo, sc);
+        val = GUARD(a.st, cnt_lo != NONE && p - cq[lo] < cnt_lo, (lo << 16) | (p - cq[lo])) ? sc[p - cq[lo]] : start;
       }
       keep = hmap_get(qk, qv, qcap, val) == p;
     }
