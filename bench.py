@@ -229,12 +229,13 @@ def run_ours(args, rank, world, local_rank):
     import torch
     import workloads as wl
     from paper_conf_asplos_jungkl23_b200 import Engine, binding as B
+    from paper_conf_asplos_jungkl23_b200.replicas import aggregate, replica_seed
 
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
     n_iter = 1 + args.warmup + args.steps
     shape_seed = {"G": 3, "B": 2, "T": 1}[args.workload]
-    seed = shape_seed + 1000 * rank
+    seed = replica_seed(shape_seed, rank)
     tr = wl.make(args.workload, n_iter=n_iter, seed=seed)
     K, N = tr.K, args.degree
     eng = Engine(num_rows=2048, assoc=2, num_succs=4, degree_n=N, max_blocks=tr.W, max_exec_ids=8192,
@@ -368,14 +369,7 @@ def run_ours(args, rank, world, local_rank):
     ctr = eng.read_counters(reset=True)
     kms, kcnt = eng.read_timing(reset=True)
     # max over ranks (time), sum over ranks (records)
-    if world > 1:
-        t = torch.tensor([tot_ms], dtype=torch.float64, device=dev)
-        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-        r = torch.tensor([records], dtype=torch.float64, device=dev)
-        torch.distributed.all_reduce(r, op=torch.distributed.ReduceOp.SUM)
-        tot_ms_max, records_all = float(t.item()), float(r.item())
-    else:
-        tot_ms_max, records_all = tot_ms, float(records)
+    tot_ms_max, records_all = aggregate(tot_ms, records, device=dev)
     value = records_all / (tot_ms_max / 1000.0)
 
     # ---- roofline of the dominant kernel ----
