@@ -109,9 +109,9 @@ void free_all(dum_engine *e) {
   void *ptrs[] = {e->d_exec_keys, e->d_exec_vals, e->d_exec_minpos, e->d_exec_hash, e->d_corr, e->d_tbl,
                   e->d_start_end, e->d_walk, e->d_walk_len, e->d_in_hash, e->d_in_off, e->d_in_faults,
                   e->d_stage_hash, e->d_stage_norm, e->d_stage_cnt, e->d_stage_exec, e->d_stage_slot,
-                  e->d_stage_off, e->d_head, e->d_next, e->d_slow_list, e->d_big_pool, e->d_walk_seen,
+                  e->d_stage_off, e->d_head, e->d_next, e->d_order, e->d_slow_list, e->d_big_pool, e->d_walk_seen,
                   e->d_walk_chain, e->d_walk_tmp, e->d_walk_out, e->d_anchor_pool, e->d_anchor_range,
-                  e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits, e->d_inactive_bits, e->d_lrm_blk,
+                  e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits, e->d_inactive_bits, e->d_res_bits, e->d_lrm_blk,
                   e->d_lrm_stamp, e->d_mig_frames, e->d_mig_src, e->d_mig_blocks, e->d_state, e->d_qkern,
                   e->d_qloff, e->d_qnk, e->d_qbase};
   for (void *p : ptrs)
@@ -244,6 +244,7 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_stage_off, e->stage_launch_cap));
   A_(dmalloc(&e->d_head, g.Emax));
   A_(dmalloc(&e->d_next, e->stage_launch_cap));
+  A_(dmalloc(&e->d_order, 3ull * e->stage_launch_cap));
   A_(dmalloc(&e->d_slow_list, e->stage_launch_cap));
   A_(dmalloc(&e->d_big_pool, 2 * e->big_pool_entries));
   A_(dmalloc(&e->d_walk_seen, (uint64_t)e->n_walk_slots * e->walk_hash_cap));
@@ -261,6 +262,7 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_block_of, g.C));
   A_(dmalloc(&e->d_free_bits, (g.C + 31) / 32));
   A_(dmalloc(&e->d_inactive_bits, (g.W + 31) / 32));
+  A_(dmalloc(&e->d_res_bits, (g.W + 31) / 32));
   A_(dmalloc(&e->d_lrm_blk, e->lrm_cap));
   A_(dmalloc(&e->d_lrm_stamp, e->lrm_cap));
   A_(dmalloc(&e->d_mig_frames, e->mig_cap));

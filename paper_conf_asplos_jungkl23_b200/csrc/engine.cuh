@@ -61,6 +61,7 @@ struct DevState {
   uint32_t mig_n;             // blocks moved by the last migrate
   uint32_t log_dirty;         // LRM log may hold entries of evicted blocks
   uint32_t dbg_line, dbg_val; // first failed internal guard (GUARD macro)
+  uint32_t cls_cnt[4];        // build: faulting launches per size class
   unsigned long long ctr[DUM_NCOUNTERS];  // work counters (instrumentation)
 };
 
@@ -140,7 +141,7 @@ struct dum_engine {
   uint64_t launches;      // recorded since reset (global launch index base)
   uint64_t built_launches;
   // build scratch
-  uint32_t *d_head, *d_next, *d_slow_list;
+  uint32_t *d_head, *d_next, *d_slow_list, *d_order;
   uint32_t *d_big_pool;   // u32 pairs for large-walk hash tables
   uint64_t big_pool_entries;
   // walk scratch for the sequential walker (per CTA slot)
@@ -155,7 +156,7 @@ struct dum_engine {
   uint32_t *d_qkern, *d_qloff, *d_qnk;  // per-query chain scratch (k_chain -> k_predict)
   unsigned long long *d_qbase;
   // residency
-  uint32_t *d_frame_of, *d_stamp_of, *d_block_of, *d_free_bits, *d_inactive_bits;
+  uint32_t *d_frame_of, *d_stamp_of, *d_block_of, *d_free_bits, *d_inactive_bits, *d_res_bits;
   uint32_t *d_lrm_blk, *d_lrm_stamp;
   uint32_t lrm_cap;
   uint32_t *d_mig_frames;     // destination frames of the last migrate

@@ -28,7 +28,8 @@ constexpr int PLAN_NT = 1024;
 constexpr uint64_t BLK = 2ull << 20;
 
 __global__ void k_res_reset(uint32_t W, uint32_t C, uint32_t *frame_of, uint32_t *stamp_of, uint32_t *block_of,
-                            uint32_t *free_bits, uint32_t *inactive, bool clear_inactive, DevState *st) {
+                            uint32_t *free_bits, uint32_t *inactive, uint32_t *res_bits, bool clear_inactive,
+                            DevState *st) {
   const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x, nt = gridDim.x * blockDim.x;
   for (uint32_t i = t; i < W; i += nt) {
     frame_of[i] = NONE;
@@ -39,8 +40,10 @@ __global__ void k_res_reset(uint32_t W, uint32_t C, uint32_t *frame_of, uint32_t
     const uint32_t lo = w * 32;
     free_bits[w] = C - lo >= 32 ? 0xFFFFFFFFu : ((1u << (C - lo)) - 1u);
   }
-  if (clear_inactive)
-    for (uint32_t w = t; w < (W + 31) / 32; w += nt) inactive[w] = 0;
+  for (uint32_t w = t; w < (W + 31) / 32; w += nt) {
+    res_bits[w] = 0;
+    if (clear_inactive) inactive[w] = 0;
+  }
   if (t == 0) {
     st->lrm_head = st->lrm_tail = 0;
     st->log_dirty = 0;
@@ -52,7 +55,7 @@ __global__ void k_res_reset(uint32_t W, uint32_t C, uint32_t *frame_of, uint32_t
 
 __global__ void k_load_res(const uint32_t *__restrict__ lrm, uint32_t n, uint32_t W, uint32_t *frame_of,
                            uint32_t *stamp_of, uint32_t *block_of, uint32_t *free_bits, uint32_t *lrm_blk,
-                           uint32_t *lrm_stamp, DevState *st) {
+                           uint32_t *lrm_stamp, uint32_t *res_bits, DevState *st) {
   const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i == 0) {
     st->lrm_head = 0;
@@ -72,6 +75,7 @@ __global__ void k_load_res(const uint32_t *__restrict__ lrm, uint32_t n, uint32_
   lrm_blk[i] = b;
   lrm_stamp[i] = i;
   atomicAnd(&free_bits[i >> 5], ~(1u << (i & 31)));
+  atomicOr(&res_bits[b >> 5], 1u << (b & 31));
 }
 
 __global__ void k_mark_inactive(const uint32_t *__restrict__ blocks, uint32_t n, int flag, uint32_t W,
@@ -92,7 +96,7 @@ struct MigArgs {
   const uint32_t *blocks, *dst;
   uint32_t n;
   uint32_t W, C;
-  uint32_t *frame_of, *stamp_of, *block_of, *free_bits, *lrm_blk, *lrm_stamp;
+  uint32_t *frame_of, *stamp_of, *block_of, *free_bits, *lrm_blk, *lrm_stamp, *res_bits;
   uint32_t lrm_cap;
   uint32_t *mig_frames, *mig_src, *mig_blocks;
   DevState *st;
@@ -195,6 +199,7 @@ __global__ void __launch_bounds__(PLAN_NT) k_mig_plan(MigArgs a) {
       a.lrm_blk[tail + i] = b;
       a.lrm_stamp[tail + i] = mc + i;
       atomicAnd(&a.free_bits[f >> 5], ~(1u << (f & 31)));
+      atomicOr(&a.res_bits[b >> 5], 1u << (b & 31));
     }
     if (tid == 0) {
       st->free_count -= n;
@@ -224,6 +229,7 @@ __global__ void __launch_bounds__(PLAN_NT) k_mig_plan(MigArgs a) {
       a.block_of[f] = NONE;
       a.mig_blocks[i] = b;
       atomicOr(&a.free_bits[f >> 5], 1u << (f & 31));
+      atomicAnd(&a.res_bits[b >> 5], ~(1u << (b & 31)));
     }
     if (tid == 0) {
       st->free_count += n;
@@ -361,7 +367,7 @@ __global__ void __launch_bounds__(SUM_NT) k_checksums(const uint32_t *__restrict
 // ---------------------------------------------------------------------------
 cudaError_t launch_reset_residency(dum_engine *e, cudaStream_t s) {
   k_res_reset<<<256, 256, 0, s>>>(e->g.W, e->g.C, e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits,
-                                  e->d_inactive_bits, true, e->d_state);
+                                  e->d_inactive_bits, e->d_res_bits, true, e->d_state);
   e->kernel_launches += 1;
   return cudaGetLastError();
 }
@@ -369,9 +375,10 @@ cudaError_t launch_reset_residency(dum_engine *e, cudaStream_t s) {
 cudaError_t launch_load_residency(dum_engine *e, const uint32_t *lrm, uint32_t n, cudaStream_t s) {
   TimerScope t(e, DUM_T_RESIDENCY, s);
   k_res_reset<<<256, 256, 0, s>>>(e->g.W, e->g.C, e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits,
-                                  e->d_inactive_bits, false, e->d_state);
+                                  e->d_inactive_bits, e->d_res_bits, false, e->d_state);
   k_load_res<<<(n + 255) / 256 + 1, 256, 0, s>>>(lrm, n, e->g.W, e->d_frame_of, e->d_stamp_of, e->d_block_of,
-                                                  e->d_free_bits, e->d_lrm_blk, e->d_lrm_stamp, e->d_state);
+                                                  e->d_free_bits, e->d_lrm_blk, e->d_lrm_stamp, e->d_res_bits,
+                                                  e->d_state);
   e->kernel_launches += 2;
   return cudaGetLastError();
 }
@@ -407,6 +414,7 @@ cudaError_t launch_migrate(dum_engine *e, int dir, const uint32_t *blocks, const
   a.free_bits = e->d_free_bits;
   a.lrm_blk = e->d_lrm_blk;
   a.lrm_stamp = e->d_lrm_stamp;
+  a.res_bits = e->d_res_bits;
   a.lrm_cap = e->lrm_cap;
   a.mig_frames = e->d_mig_frames;
   a.mig_src = e->d_mig_src;

@@ -31,8 +31,6 @@ namespace dum {
 constexpr int PRED_NT = 512;
 constexpr int NWARP = PRED_NT / 32;
 constexpr uint32_t MAXN = 128;   // degree_n limit
-constexpr uint32_t DCAP = 2048;  // duplicate-block hash (window-wide)
-constexpr uint32_t CH_CAP = 1024;
 
 __global__ void k_make_queries(const uint32_t *__restrict__ seq, uint32_t n_seq, uint32_t first, uint32_t degree,
                                dum_query *__restrict__ out) {
@@ -131,6 +129,8 @@ struct PredArgs {
   uint32_t *qloff;  // [nq][N+2]
   uint32_t *qnk;    // [nq]
   unsigned long long *qbase;  // [nq]
+  uint32_t *big_pool;         // scratch for the exact slow path
+  uint64_t big_entries;
   SelectOut so;     // fused a8 outputs (SELECT only)
 };
 
@@ -220,12 +220,12 @@ __device__ __forceinline__ bool warp_test_and_set(uint32_t *bitmap, uint32_t b, 
 }
 
 template <bool SELECT>
-__global__ void __launch_bounds__(PRED_NT) k_predict(PredArgs a) {
+__global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
   extern __shared__ uint32_t bitmap[];
   __shared__ uint32_t kern[MAXN + 1], loff[MAXN + 2], kcnt[MAXN + 1];
-  __shared__ uint32_t dk[DCAP], dv[DCAP];
   __shared__ uint32_t ws[NWARP], wtot[NWARP];
-  __shared__ uint32_t s_ndup, s_ovf, s_nonres;
+  __shared__ uint32_t s_ndup, s_nonres, s_flag;
+  __shared__ unsigned long long s_hoff;
   const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const uint32_t qi = blockIdx.x;
   const Geo &g = a.g;
@@ -233,10 +233,10 @@ __global__ void __launch_bounds__(PRED_NT) k_predict(PredArgs a) {
   const bool anchored = anchor != NONE;
   const uint32_t nk = a.qnk[qi];
   const unsigned long long base = a.qbase[qi];
-  for (uint32_t w = tid; w < a.nwords; w += PRED_NT) bitmap[w] = 0;
-  for (uint32_t p = tid; p < DCAP; p += PRED_NT) {
-    dk[p] = NONE;
-    dv[p] = NONE;
+  {
+    uint4 *b4 = reinterpret_cast<uint4 *>(bitmap);
+    for (uint32_t w = tid; w < a.nwords / 4; w += PRED_NT) b4[w] = make_uint4(0, 0, 0, 0);
+    for (uint32_t w = (a.nwords & ~3u) + tid; w < a.nwords; w += PRED_NT) bitmap[w] = 0;
   }
   for (uint32_t d = tid; d <= nk; d += PRED_NT) {
     loff[d] = a.qloff[(uint64_t)qi * (g.N + 2) + d];
@@ -244,51 +244,48 @@ __global__ void __launch_bounds__(PRED_NT) k_predict(PredArgs a) {
   }
   if (tid == 0) {
     s_ndup = 0;
-    s_ovf = 0;
     s_nonres = 0;
   }
   __syncthreads();
   const uint32_t U = nk ? loff[nk] : 0;
   const bool ok = base + U <= a.cap;
-  if (tid == 0 && anchored && anchor < g.W) {
-    bitmap[anchor >> 5] |= 1u << (anchor & 31);
-    hmap_insert_min(dk, dv, DCAP, anchor, 0);  // position 0: never kept
-  }
+  if (tid == 0 && anchored && anchor < g.W) bitmap[anchor >> 5] |= 1u << (anchor & 31);
   __syncthreads();
   const uint32_t *apool = a.anchor_pool + (anchored ? a.anchor_range[2 * qi] : 0);
-  auto elem = [&](uint32_t t, uint32_t &d) -> uint32_t {
-    while (d + 1 < nk && loff[d + 1] <= t) ++d;
-    const uint32_t idx = t - loff[d];
-    return (d == 0 && anchored) ? apool[idx] : __ldg(a.walk + (uint64_t)kern[d] * g.walk_cap + idx);
+  auto list_of = [&](uint32_t d) -> const uint32_t * {
+    return (d == 0 && anchored) ? apool : a.walk + (uint64_t)kern[d] * g.walk_cap;
   };
   // ---------------- fast path: one pass ----------------
-  // warp w owns the contiguous segment [t0, t1); 4 loads in flight per lane
+  // warp w owns the contiguous segment [t0, t1), walked kernel by kernel
+  // (no per-element kernel search), 4 loads in flight per lane
   const uint32_t seg = ((U + NWARP - 1) / NWARP + 127) & ~127u;
   const uint32_t t0 = min(U, wid * seg), t1 = min(U, t0 + seg);
   uint32_t nonres = 0, ndup = 0;
-  {
+  if (t0 < t1) {
     uint32_t d = 0;
-    for (uint32_t c = t0; c < t1; c += 128) {
-      uint32_t b[4];
-      uint32_t dd[4];
+    while (d + 1 < nk && loff[d + 1] <= t0) ++d;
+    for (; d < nk && loff[d] < t1; ++d) {
+      const uint32_t k0 = max(t0, loff[d]), k1 = min(t1, loff[d + 1]);
+      if (k0 >= k1) continue;
+      const uint32_t *lst = list_of(d) - loff[d];  // indexed by window position
+      const uint32_t kd = kern[d];
+      for (uint32_t c = k0; c < k1; c += 128) {
+        uint32_t b[4];
 #pragma unroll
-      for (int k = 0; k < 4; ++k) {
-        const uint32_t t = c + 32 * k + lane;
-        b[k] = t < t1 ? elem(t, d) : NONE;
-        dd[k] = d;
-      }
-#pragma unroll
-      for (int k = 0; k < 4; ++k) {
-        const uint32_t t = c + 32 * k + lane;
-        const bool valid = t < t1;
-        const bool dup = warp_test_and_set(bitmap, b[k], valid);
-        if (dup) {
-          ++ndup;
-          if (!hmap_insert_min(dk, dv, DCAP, b[k], t + 1)) s_ovf = 1;
+        for (int k = 0; k < 4; ++k) {
+          const uint32_t t = c + 32 * k + lane;
+          b[k] = t < k1 ? __ldg(lst + t) : NONE;
         }
-        if (valid) {
-          if (ok) reinterpret_cast<uint2 *>(a.pairs)[base + t] = make_uint2(b[k], kern[dd[k]]);
-          if (SELECT) nonres += __ldg(&a.so.frame_of[b[k]]) == NONE;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const uint32_t t = c + 32 * k + lane;
+          const bool valid = t < k1;
+          if (c + 32 * k >= k1) break;  // warp-uniform
+          ndup += warp_test_and_set(bitmap, b[k], valid);
+          if (valid) {
+            if (ok) reinterpret_cast<uint2 *>(a.pairs)[base + t] = make_uint2(b[k], kd);
+            if (SELECT) nonres += !((__ldg(&a.so.res_bits[b[k] >> 5]) >> (b[k] & 31)) & 1u);
+          }
         }
       }
     }
@@ -301,124 +298,87 @@ __global__ void __launch_bounds__(PRED_NT) k_predict(PredArgs a) {
   }
   __syncthreads();
   uint32_t run = U;
-  if (s_ndup) {
+  const bool dedup = s_ndup != 0;
+  if (dedup) {
     // ---------------- exact slow path (some block occurs twice) ----------------
-    if (tid == 0) s_nonres = 0;
+    // keep(t) = t is the minimum window position of its block, the anchor
+    // pre-seeded at position 0 (D17); min positions in a global scratch hash
+    const uint32_t hcap = pow2ceil(2 * (U + 1));
+    if (tid == 0) {
+      s_nonres = 0;
+      const unsigned long long o = atomicAdd(&a.st->pool_big, 2ull * hcap);
+      s_flag = o + 2ull * hcap <= a.big_entries * 2;
+      s_hoff = o;
+      if (!s_flag) set_err(a.st, ERR_ECAPACITY, o + 2ull * hcap);
+    }
     for (uint32_t d = tid; d <= nk; d += PRED_NT) kcnt[d] = 0;
     __syncthreads();
-    if (!s_ovf) {
-      // phase 2: every occurrence of a duplicated block lowers its min position
-      uint32_t d = 0;
-      for (uint32_t t = tid; t < U; t += PRED_NT) {
-        const uint32_t b = elem(t, d);
-        const uint32_t s0 = hslot(b, DCAP);
-        for (uint32_t p = 0, s = s0; p < DCAP; ++p, s = (s + 1) & (DCAP - 1)) {
-          const uint32_t k = dk[s];
-          if (k == NONE) break;
-          if (k == b) {
-            atomicMin(&dv[s], t + 1);
-            break;
-          }
-        }
+    if (s_flag) {
+      uint32_t *hk = a.big_pool + s_hoff, *hv = hk + hcap;
+      for (uint32_t p = tid; p < hcap; p += PRED_NT) {
+        hk[p] = NONE;
+        hv[p] = NONE;
       }
       __syncthreads();
-      // phase 3: per-warp keep counts
-      uint32_t cnt = 0;
-      {
-        uint32_t dd = 0;
-        for (uint32_t c = t0; c < t1; c += 32) {
-          const uint32_t t = c + lane;
-          bool keep = false;
-          if (t < t1) {
-            const uint32_t b = elem(t, dd);
-            const uint32_t m = hmap_get(dk, dv, DCAP, b);
-            keep = (m == NONE) || (m == t + 1);
-          }
-          cnt += __popc(__ballot_sync(0xffffffffu, keep));
-        }
-      }
-      if (lane == 0) wtot[wid] = cnt;
-      __syncthreads();
-      if (tid == 0) {
-        uint32_t acc = 0;
-        for (int w = 0; w < NWARP; ++w) {
-          const uint32_t v = wtot[w];
-          wtot[w] = acc;
-          acc += v;
-        }
-        ws[0] = acc;
+      if (tid == 0 && anchored) hmap_insert_min(hk, hv, hcap, anchor, 0);
+      for (uint32_t d = 0; d < nk; ++d) {
+        const uint32_t *lst = list_of(d);
+        for (uint32_t i = tid; i < loff[d + 1] - loff[d]; i += PRED_NT)
+          hmap_insert_min(hk, hv, hcap, __ldg(lst + i), loff[d] + i + 1);
       }
       __syncthreads();
-      // phase 4: ordered re-write
-      uint32_t pos = wtot[wid], nr = 0;
-      {
-        uint32_t dd = 0;
-        for (uint32_t c = t0; c < t1; c += 32) {
-          const uint32_t t = c + lane;
-          uint32_t b = NONE;
-          bool keep = false;
-          if (t < t1) {
-            b = elem(t, dd);
-            const uint32_t m = hmap_get(dk, dv, DCAP, b);
-            keep = (m == NONE) || (m == t + 1);
+      // per-warp keep counts over the warp segments, then ordered writes
+      for (int pass = 0; pass < 2; ++pass) {
+        uint32_t pos = pass ? wtot[wid] : 0, nr = 0;
+        if (t0 < t1) {
+          uint32_t d = 0;
+          while (d + 1 < nk && loff[d + 1] <= t0) ++d;
+          for (; d < nk && loff[d] < t1; ++d) {
+            const uint32_t k0 = max(t0, loff[d]), k1 = min(t1, loff[d + 1]);
+            if (k0 >= k1) continue;
+            const uint32_t *lst = list_of(d) - loff[d];
+            for (uint32_t c = k0; c < k1; c += 32) {
+              const uint32_t t = c + lane;
+              uint32_t bb = NONE;
+              bool keep = false;
+              if (t < k1) {
+                bb = __ldg(lst + t);
+                keep = hmap_get(hk, hv, hcap, bb) == t + 1;
+              }
+              const uint32_t mask = __ballot_sync(0xffffffffu, keep);
+              if (pass && keep) {
+                if (ok) reinterpret_cast<uint2 *>(a.pairs)[base + pos + __popc(mask & ((1u << lane) - 1))] =
+                    make_uint2(bb, kern[d]);
+                if (SELECT) nr += !((__ldg(&a.so.res_bits[bb >> 5]) >> (bb & 31)) & 1u);
+              }
+              if (pass && lane == 0) atomicAdd(&kcnt[d], __popc(mask));
+              pos += __popc(mask);
+            }
           }
-          const uint32_t mask = __ballot_sync(0xffffffffu, keep);
-          if (keep) {
-            if (ok) reinterpret_cast<uint2 *>(a.pairs)[base + pos + __popc(mask & ((1u << lane) - 1))] =
-                make_uint2(b, kern[dd]);
-            if (SELECT) nr += __ldg(&a.so.frame_of[b]) == NONE;
-          }
-          const uint32_t grp = __match_any_sync(0xffffffffu, keep ? dd : 0xFFFFFFFFu);
-          if (keep && lane == __ffs(grp) - 1) atomicAdd(&kcnt[dd], __popc(grp));
-          pos += __popc(mask);
         }
-      }
-      if (SELECT) {
+        if (!pass) {
+          if (lane == 0) wtot[wid] = pos;
+          __syncthreads();
+          if (tid == 0) {
+            uint32_t acc = 0;
+            for (int w = 0; w < NWARP; ++w) {
+              const uint32_t v = wtot[w];
+              wtot[w] = acc;
+              acc += v;
+            }
+            ws[0] = acc;
+          }
+          __syncthreads();
+        } else if (SELECT) {
 #pragma unroll
-        for (int o = 16; o; o >>= 1) nr += __shfl_xor_sync(0xffffffffu, nr, o);
-        if (lane == 0 && nr) atomicAdd(&s_nonres, nr);
+          for (int o = 16; o; o >>= 1) nr += __shfl_xor_sync(0xffffffffu, nr, o);
+          if (lane == 0 && nr) atomicAdd(&s_nonres, nr);
+        }
       }
       __syncthreads();
       run = ws[0];
     } else {
-      // too many duplicated blocks for the window-wide hash: ordered chunks
-      // with a chunk-local min-position hash
-      for (uint32_t w = tid; w < a.nwords; w += PRED_NT) bitmap[w] = 0;
-      for (uint32_t p = tid; p < CH_CAP; p += PRED_NT) {
-        dk[p] = NONE;
-        dv[p] = NONE;
-      }
-      __syncthreads();
-      if (tid == 0 && anchored && anchor < g.W) bitmap[anchor >> 5] |= 1u << (anchor & 31);
-      __syncthreads();
-      uint32_t r = 0, d = 0;
-      for (uint32_t c = 0; c < U; c += PRED_NT) {
-        const uint32_t t = c + tid;
-        uint32_t b = NONE;
-        bool fresh = false;
-        if (t < U) {
-          b = elem(t, d);
-          fresh = !(bitmap[b >> 5] & (1u << (b & 31)));
-          if (fresh) hmap_insert_min(dk, dv, CH_CAP, b, t);
-        }
-        __syncthreads();
-        const uint32_t keep = fresh && hmap_get(dk, dv, CH_CAP, b) == t;
-        if (keep) {
-          atomicOr(&bitmap[b >> 5], 1u << (b & 31));
-          atomicAdd(&kcnt[d], 1u);
-          if (SELECT && __ldg(&a.so.frame_of[b]) == NONE) atomicAdd(&s_nonres, 1u);
-        }
-        uint32_t tot;
-        const uint32_t pre = block_excl_scan(keep, ws, &tot);
-        if (keep && ok) reinterpret_cast<uint2 *>(a.pairs)[base + r + pre] = make_uint2(b, kern[d]);
-        r += tot;
-        for (uint32_t p = tid; p < CH_CAP; p += PRED_NT) {
-          dk[p] = NONE;
-          dv[p] = NONE;
-        }
-        __syncthreads();
-      }
-      run = r;
+      run = 0;
     }
   }
   if (tid == 0) {
@@ -431,7 +391,6 @@ __global__ void __launch_bounds__(PRED_NT) k_predict(PredArgs a) {
   }
   if (a.kern_off) {
     uint32_t *ko = a.kern_off + (uint64_t)qi * (g.N + 2);
-    const bool dedup = s_ndup != 0;
     for (uint32_t d = tid; d <= g.N + 1; d += PRED_NT) {
       uint32_t v;
       if (!dedup) {
@@ -471,6 +430,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   if (nq == 0) return cudaSuccess;
   if (nq > e->anchor_range_cap) return cudaErrorInvalidValue;
   cudaMemsetAsync(&e->d_state->pool_pairs, 0, 2 * sizeof(unsigned long long) * 2, s);  // pairs, wb, inv, anchor
+  cudaMemsetAsync(&e->d_state->pool_big, 0, sizeof(unsigned long long), s);
   WalkScratch ws{e->d_walk_seen, e->d_walk_chain, e->d_walk_tmp, e->walk_hash_cap,
                  e->g.walk_cap + e->g.R * e->g.A + 4};
   {
@@ -500,7 +460,13 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   a.qloff = e->d_qloff;
   a.qnk = e->d_qnk;
   a.qbase = e->d_qbase;
-  if (sel) a.so = *sel;
+  a.big_pool = e->d_big_pool;
+  a.big_entries = e->big_pool_entries;
+  if (sel) {
+    a.so = *sel;
+  } else {
+    a.so.res_bits = e->d_res_bits;
+  }
   {
     TimerScope t(e, DUM_T_CHAIN, s);
     k_chain<<<(nq + CHAIN_NT - 1) / CHAIN_NT, CHAIN_NT, 0, s>>>(a);

@@ -9,7 +9,7 @@
 namespace dum {
 
 struct SelectOut {
-  const uint32_t *frame_of, *stamp_of, *inactive, *lrm_blk, *lrm_stamp;
+  const uint32_t *frame_of, *stamp_of, *inactive, *res_bits, *lrm_blk, *lrm_stamp;
   uint32_t *wb, *inv;
   uint64_t cap;
   uint64_t *out_range;  // 4 per query
@@ -19,15 +19,19 @@ struct SelectOut {
 // = the first `need` entries of the LRM log (oldest migration first) that are
 // still resident with that stamp and not in the window bitmap; split into
 // write-back / invalidate by the inactive bitmap, both in LRM order.
-// Each thread examines ITEMS consecutive log entries per chunk, so one block
-// scan covers NT * ITEMS entries.
+// Chunks of NT * 4 log entries; warp w owns 128 consecutive entries of a
+// chunk (4 coalesced steps of 32), counts its eligible active / inactive
+// entries with ballots, and the 32 warp totals are scanned by one warp -- one
+// barrier pair per chunk.
 template <int NT>
 __device__ void select_tail(const SelectOut &so, uint32_t qi, uint32_t nonres, const uint32_t *bitmap, uint32_t W,
                             DevState *st, uint32_t *ws) {
+  constexpr int NW = NT / 32;
   constexpr int ITEMS = 4;
-  __shared__ uint32_t s_ok, s_cwb, s_cinv;
+  constexpr uint32_t CHUNK = NT * ITEMS;
+  __shared__ uint32_t s_ok, s_wcnt[NW], s_icnt[NW], s_tw, s_ti, s_aw, s_ai, s_split, s_rem;
   __shared__ unsigned long long s_bwb, s_binv;
-  const uint32_t tid = threadIdx.x;
+  const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const uint32_t nfree = *(volatile uint32_t *)&st->free_count;
   const uint32_t need = nonres > nfree ? nonres - nfree : 0;
   const bool clean = *(volatile uint32_t *)&st->log_dirty == 0;
@@ -48,59 +52,120 @@ __device__ void select_tail(const SelectOut &so, uint32_t qi, uint32_t nonres, c
   const bool ok = s_ok;
   uint32_t run_wb = 0, run_inv = 0, scanned = 0;
   const uint32_t head = *(volatile uint32_t *)&st->lrm_head, tail = *(volatile uint32_t *)&st->lrm_tail;
-  for (uint32_t c = head; c < tail && run_wb + run_inv < need; c += NT * ITEMS) {
-    scanned += min((uint32_t)(NT * ITEMS), tail - c);
-    uint32_t blk[ITEMS];
-    uint32_t flags = 0;  // bit k: eligible, bit 8+k: inactive
+  const uint32_t lt = (1u << lane) - 1;
+  for (uint32_t c = head; c < tail && run_wb + run_inv < need; c += CHUNK) {
+    scanned += min(CHUNK, tail - c);
+    uint32_t blk[ITEMS], me[ITEMS], mi[ITEMS];
     uint32_t cw = 0, ci = 0;
 #pragma unroll
     for (int k = 0; k < ITEMS; ++k) {
-      const uint32_t i = c + tid * ITEMS + k;
-      blk[k] = NONE;
-      if (i < tail) {
-        const uint32_t b = so.lrm_blk[i];
-        blk[k] = b;
-        bool elig = !(bitmap[b >> 5] & (1u << (b & 31)));
-        if (elig && !clean) elig = __ldg(&so.frame_of[b]) != NONE && __ldg(&so.stamp_of[b]) == so.lrm_stamp[i];
-        if (elig) {
-          const bool ina = (__ldg(&so.inactive[b >> 5]) >> (b & 31)) & 1u;
-          flags |= (1u << k) | (ina ? (1u << (8 + k)) : 0u);
-          ci += ina;
-          cw += !ina;
-        }
-      }
+      const uint32_t i = c + wid * (32 * ITEMS) + 32 * k + lane;
+      blk[k] = i < tail ? so.lrm_blk[i] : NONE;
     }
-    uint32_t tot;
-    const uint32_t pre = block_excl_scan((ci << 16) | cw, ws, &tot);
-    const uint32_t left = need - run_wb - run_inv;
-    uint32_t pw = pre & 0xFFFFu, pi = pre >> 16;
-    uint32_t tw = 0, ti = 0;
 #pragma unroll
     for (int k = 0; k < ITEMS; ++k) {
-      if (flags & (1u << k)) {
-        const bool ina = flags & (1u << (8 + k));
-        if (pw + pi < left) {
-          if (ok) {
-            if (ina) so.inv[binv + run_inv + pi] = blk[k];
-            else so.wb[bwb + run_wb + pw] = blk[k];
-          }
-          if (ina) ++ti;
-          else ++tw;
-        }
-        if (ina) ++pi;
-        else ++pw;
+      const uint32_t i = c + wid * (32 * ITEMS) + 32 * k + lane;
+      const uint32_t b = blk[k];
+      bool elig = false, ina = false;
+      if (i < tail) {
+        elig = !(bitmap[b >> 5] & (1u << (b & 31)));
+        if (elig && !clean) elig = __ldg(&so.frame_of[b]) != NONE && __ldg(&so.stamp_of[b]) == so.lrm_stamp[i];
+        if (elig) ina = (__ldg(&so.inactive[b >> 5]) >> (b & 31)) & 1u;
       }
+      me[k] = __ballot_sync(0xffffffffu, elig && !ina);
+      mi[k] = __ballot_sync(0xffffffffu, elig && ina);
+      cw += __popc(me[k]);
+      ci += __popc(mi[k]);
     }
-    if (tid == 0) {
-      s_cwb = 0;
-      s_cinv = 0;
+    if (lane == 0) {
+      s_wcnt[wid] = cw;
+      s_icnt[wid] = ci;
     }
     __syncthreads();
-    if (tw) atomicAdd(&s_cwb, tw);
-    if (ti) atomicAdd(&s_cinv, ti);
-    __syncthreads();
-    run_wb += s_cwb;
-    run_inv += s_cinv;
+    // exclusive prefix of the warp totals (in log order = warp order)
+    uint32_t pw = 0, pi = 0, tw = 0, ti = 0;
+#pragma unroll
+    for (int w = 0; w < NW; ++w) {
+      const uint32_t a = s_wcnt[w], b2 = s_icnt[w];
+      if (w < (int)wid) {
+        pw += a;
+        pi += b2;
+      }
+      tw += a;
+      ti += b2;
+    }
+    const uint32_t left = need - run_wb - run_inv;
+#pragma unroll
+    for (int k = 0; k < ITEMS; ++k) {
+      const uint32_t i = c + wid * (32 * ITEMS) + 32 * k + lane;
+      const bool ew = (me[k] >> lane) & 1u, ei = (mi[k] >> lane) & 1u;
+      const uint32_t rw = pw + __popc(me[k] & lt), ri = pi + __popc(mi[k] & lt);
+      if ((ew || ei) && rw + ri < left && ok) {
+        if (ei) so.inv[binv + run_inv + ri] = blk[k];
+        else so.wb[bwb + run_wb + rw] = blk[k];
+      }
+      (void)i;
+      pw += __popc(me[k]);
+      pi += __popc(mi[k]);
+    }
+    // the taken entries are the first `left` eligible ones of the chunk; how
+    // many of them are write-back vs invalidate
+    uint32_t take_w = tw, take_i = ti;
+    if (tw + ti > left) {
+      // find the split inside the chunk: the warp holding eligible entry `left`
+      if (tid == 0) {
+        uint32_t aw = 0, ai = 0;
+        s_split = NONE;
+        for (int w = 0; w < NW; ++w) {
+          if (aw + ai + s_wcnt[w] + s_icnt[w] > left) {
+            s_split = w;
+            s_rem = left - aw - ai;  // eligible entries of warp w that are taken
+            break;
+          }
+          aw += s_wcnt[w];
+          ai += s_icnt[w];
+        }
+        s_aw = aw;  // totals of the warps before the split warp
+        s_ai = ai;
+      }
+      __syncthreads();
+      const uint32_t w_split = s_split, rem = s_rem;
+      const uint32_t aw = s_aw, ai = s_ai;
+      if (wid == w_split) {
+        // walk this warp's 4 steps in order; lanes count taken entries
+        uint32_t r = rem, cw2 = 0, ci2 = 0;
+#pragma unroll
+        for (int k = 0; k < ITEMS; ++k) {
+          const uint32_t all = me[k] | mi[k];
+          const uint32_t nall = __popc(all);
+          if (r >= nall) {
+            cw2 += __popc(me[k]);
+            ci2 += __popc(mi[k]);
+            r -= nall;
+          } else if (r > 0) {
+            // first r set bits of `all`
+            uint32_t m = all, sel = 0;
+            for (uint32_t q = 0; q < r; ++q) {
+              const uint32_t bit = m & (~m + 1u);
+              sel |= bit;
+              m &= m - 1;
+            }
+            cw2 += __popc(me[k] & sel);
+            ci2 += __popc(mi[k] & sel);
+            r = 0;
+          }
+        }
+        if (lane == 0) {
+          s_tw = aw + cw2;
+          s_ti = ai + ci2;
+        }
+      }
+      __syncthreads();
+      take_w = s_tw;
+      take_i = s_ti;
+    }
+    run_wb += take_w;
+    run_inv += take_i;
     __syncthreads();
   }
   if (tid == 0) {
@@ -119,6 +184,7 @@ inline SelectOut make_select_out(dum_engine *e, uint32_t *wb, uint32_t *inv, uin
   so.frame_of = e->d_frame_of;
   so.stamp_of = e->d_stamp_of;
   so.inactive = e->d_inactive_bits;
+  so.res_bits = e->d_res_bits;
   so.lrm_blk = e->d_lrm_blk;
   so.lrm_stamp = e->d_lrm_stamp;
   so.wb = wb;
