@@ -31,6 +31,7 @@ namespace dum {
 constexpr int PRED_NT = 512;
 constexpr int NWARP = PRED_NT / 32;
 constexpr uint32_t MAXN = 128;   // degree_n limit
+constexpr uint32_t DCAP = 2048;  // shared hash of duplicated blocks (block -> min window position)
 
 __global__ void k_make_queries(const uint32_t *__restrict__ seq, uint32_t n_seq, uint32_t first, uint32_t degree,
                                dum_query *__restrict__ out) {
@@ -221,10 +222,10 @@ __device__ __forceinline__ bool warp_test_and_set(uint32_t *bitmap, uint32_t b, 
 
 template <bool SELECT>
 __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
-  extern __shared__ uint32_t bitmap[];
+  extern __shared__ uint32_t bitmap[];  // [nwords] window set | dk[DCAP] | dv[DCAP]
   __shared__ uint32_t kern[MAXN + 1], loff[MAXN + 2], kcnt[MAXN + 1];
   __shared__ uint32_t ws[NWARP], wtot[NWARP];
-  __shared__ uint32_t s_ndup, s_nonres, s_flag;
+  __shared__ uint32_t s_ndup, s_nonres, s_flag, s_ovf;
   __shared__ unsigned long long s_hoff;
   const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const uint32_t qi = blockIdx.x;
@@ -233,10 +234,13 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
   const bool anchored = anchor != NONE;
   const uint32_t nk = a.qnk[qi];
   const unsigned long long base = a.qbase[qi];
+  uint32_t *dk = bitmap + ((a.nwords + 3) & ~3u), *dv = dk + DCAP;
   {
     uint4 *b4 = reinterpret_cast<uint4 *>(bitmap);
     for (uint32_t w = tid; w < a.nwords / 4; w += PRED_NT) b4[w] = make_uint4(0, 0, 0, 0);
     for (uint32_t w = (a.nwords & ~3u) + tid; w < a.nwords; w += PRED_NT) bitmap[w] = 0;
+    uint4 *d4 = reinterpret_cast<uint4 *>(dk);
+    for (uint32_t w = tid; w < 2 * DCAP / 4; w += PRED_NT) d4[w] = make_uint4(NONE, NONE, NONE, NONE);
   }
   for (uint32_t d = tid; d <= nk; d += PRED_NT) {
     loff[d] = a.qloff[(uint64_t)qi * (g.N + 2) + d];
@@ -245,11 +249,15 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
   if (tid == 0) {
     s_ndup = 0;
     s_nonres = 0;
+    s_ovf = 0;
   }
   __syncthreads();
   const uint32_t U = nk ? loff[nk] : 0;
   const bool ok = base + U <= a.cap;
-  if (tid == 0 && anchored && anchor < g.W) bitmap[anchor >> 5] |= 1u << (anchor & 31);
+  if (tid == 0 && anchored && anchor < g.W) {
+    bitmap[anchor >> 5] |= 1u << (anchor & 31);
+    hmap_insert_min(dk, dv, DCAP, anchor, 0);  // position 0: never kept
+  }
   __syncthreads();
   const uint32_t *apool = a.anchor_pool + (anchored ? a.anchor_range[2 * qi] : 0);
   auto list_of = [&](uint32_t d) -> const uint32_t * {
@@ -281,7 +289,10 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
           const uint32_t t = c + 32 * k + lane;
           const bool valid = t < k1;
           if (c + 32 * k >= k1) break;  // warp-uniform
-          ndup += warp_test_and_set(bitmap, b[k], valid);
+          if (warp_test_and_set(bitmap, b[k], valid)) {
+            ++ndup;
+            if (!hmap_insert_min(dk, dv, DCAP, b[k], t + 1)) s_ovf = 1;
+          }
           if (valid) {
             if (ok) reinterpret_cast<uint2 *>(a.pairs)[base + t] = make_uint2(b[k], kd);
             if (SELECT) nonres += !((__ldg(&a.so.res_bits[b[k] >> 5]) >> (b[k] & 31)) & 1u);
@@ -302,29 +313,58 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
   if (dedup) {
     // ---------------- exact slow path (some block occurs twice) ----------------
     // keep(t) = t is the minimum window position of its block, the anchor
-    // pre-seeded at position 0 (D17); min positions in a global scratch hash
-    const uint32_t hcap = pow2ceil(2 * (U + 1));
+    // pre-seeded at position 0 (D17).  Normally only the duplicated blocks
+    // (found in the fast pass) sit in the shared hash and every occurrence of
+    // them lowers the min position; if that hash overflowed, all elements go
+    // into a global scratch hash instead.
+    const bool ovf = s_ovf != 0;
+    uint32_t hcap = DCAP;
+    uint32_t *hk = dk, *hv = dv;
     if (tid == 0) {
       s_nonres = 0;
-      const unsigned long long o = atomicAdd(&a.st->pool_big, 2ull * hcap);
-      s_flag = o + 2ull * hcap <= a.big_entries * 2;
-      s_hoff = o;
-      if (!s_flag) set_err(a.st, ERR_ECAPACITY, o + 2ull * hcap);
+      s_flag = 1;
+      if (ovf) {
+        const uint32_t hc = pow2ceil(2 * (U + 1));
+        const unsigned long long o = atomicAdd(&a.st->pool_big, 2ull * hc);
+        s_flag = o + 2ull * hc <= a.big_entries * 2;
+        s_hoff = o;
+        if (!s_flag) set_err(a.st, ERR_ECAPACITY, o + 2ull * hc);
+      }
     }
     for (uint32_t d = tid; d <= nk; d += PRED_NT) kcnt[d] = 0;
     __syncthreads();
+    if (ovf) {
+      hcap = pow2ceil(2 * (U + 1));
+      hk = a.big_pool + s_hoff;
+      hv = hk + hcap;
+    }
     if (s_flag) {
-      uint32_t *hk = a.big_pool + s_hoff, *hv = hk + hcap;
-      for (uint32_t p = tid; p < hcap; p += PRED_NT) {
-        hk[p] = NONE;
-        hv[p] = NONE;
+      if (ovf) {
+        for (uint32_t p = tid; p < hcap; p += PRED_NT) {
+          hk[p] = NONE;
+          hv[p] = NONE;
+        }
+        __syncthreads();
+        if (tid == 0 && anchored) hmap_insert_min(hk, hv, hcap, anchor, 0);
       }
-      __syncthreads();
-      if (tid == 0 && anchored) hmap_insert_min(hk, hv, hcap, anchor, 0);
       for (uint32_t d = 0; d < nk; ++d) {
         const uint32_t *lst = list_of(d);
-        for (uint32_t i = tid; i < loff[d + 1] - loff[d]; i += PRED_NT)
-          hmap_insert_min(hk, hv, hcap, __ldg(lst + i), loff[d] + i + 1);
+        for (uint32_t i = tid; i < loff[d + 1] - loff[d]; i += PRED_NT) {
+          const uint32_t bb = __ldg(lst + i), pos = loff[d] + i + 1;
+          if (ovf) {
+            hmap_insert_min(hk, hv, hcap, bb, pos);
+          } else {
+            // lower the min position of duplicated blocks only
+            for (uint32_t pp = 0, sl = hslot(bb, hcap); pp < hcap; ++pp, sl = (sl + 1) & (hcap - 1)) {
+              const uint32_t kk = hk[sl];
+              if (kk == NONE) break;
+              if (kk == bb) {
+                atomicMin(&hv[sl], pos);
+                break;
+              }
+            }
+          }
+        }
       }
       __syncthreads();
       // per-warp keep counts over the warp segments, then ordered writes
@@ -343,7 +383,8 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
               bool keep = false;
               if (t < k1) {
                 bb = __ldg(lst + t);
-                keep = hmap_get(hk, hv, hcap, bb) == t + 1;
+                const uint32_t mp = hmap_get(hk, hv, hcap, bb);
+                keep = ovf ? mp == t + 1 : (mp == NONE || mp == t + 1);
               }
               const uint32_t mask = __ballot_sync(0xffffffffu, keep);
               if (pass && keep) {
@@ -471,7 +512,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
     TimerScope t(e, DUM_T_CHAIN, s);
     k_chain<<<(nq + CHAIN_NT - 1) / CHAIN_NT, CHAIN_NT, 0, s>>>(a);
   }
-  const size_t smem = (size_t)a.nwords * 4;
+  const size_t smem = (size_t)((a.nwords + 3) & ~3u) * 4 + 2 * DCAP * 4;
   if (sel) {
     cudaFuncSetAttribute(k_predict<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     TimerScope t(e, DUM_T_PREDICT, s);
