@@ -111,7 +111,7 @@ void free_all(dum_engine *e) {
                   e->d_stage_hash, e->d_stage_norm, e->d_stage_cnt, e->d_stage_exec, e->d_stage_slot,
                   e->d_stage_off, e->d_head, e->d_next, e->d_order, e->d_slow_list, e->d_big_pool, e->d_walk_seen,
                   e->d_walk_chain, e->d_walk_tmp, e->d_walk_out, e->d_anchor_pool, e->d_anchor_range,
-                  e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits, e->d_inactive_bits, e->d_res_bits, e->d_lrm_blk,
+                  e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits, e->d_inactive_bits, e->d_res_bits, e->d_logpos, e->d_lrm_blk,
                   e->d_lrm_stamp, e->d_mig_frames, e->d_mig_src, e->d_mig_blocks, e->d_state, e->d_qkern,
                   e->d_qloff, e->d_qnk, e->d_qbase};
   for (void *p : ptrs)
@@ -264,6 +264,7 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_inactive_bits, (g.W + 31) / 32));
   A_(dmalloc(&e->d_res_bits, (g.W + 31) / 32));
   A_(dmalloc(&e->d_lrm_blk, e->lrm_cap));
+  A_(dmalloc(&e->d_logpos, g.W));
   A_(dmalloc(&e->d_lrm_stamp, e->lrm_cap));
   A_(dmalloc(&e->d_mig_frames, e->mig_cap));
   A_(dmalloc(&e->d_mig_src, e->mig_cap));
@@ -630,7 +631,7 @@ int dum_dump_state(dum_engine *e, uint32_t what, void *host_buf, uint64_t cap, u
     for (auto b : bof) put32(o, b);
     std::vector<uint32_t> lrm;
     for (uint32_t i = 0; i < nlog; ++i) {
-      const uint32_t b = lb[i];
+      const uint32_t b = lb[i] & 0x7FFFFFFFu;
       if (b < g.W && fof[b] != NONE && sof[b] == ls[i]) lrm.push_back(b);
     }
     put32(o, (uint32_t)lrm.size());

@@ -157,7 +157,8 @@ struct dum_engine {
   unsigned long long *d_qbase;
   // residency
   uint32_t *d_frame_of, *d_stamp_of, *d_block_of, *d_free_bits, *d_inactive_bits, *d_res_bits;
-  uint32_t *d_lrm_blk, *d_lrm_stamp;
+  uint32_t *d_lrm_blk, *d_lrm_stamp;   // LRM log: block | inactive << 31, migration stamp
+  uint32_t *d_logpos;                  // log position of each resident block
   uint32_t lrm_cap;
   uint32_t *d_mig_frames;     // destination frames of the last migrate
   uint32_t *d_mig_src;        // source frames (D2D)

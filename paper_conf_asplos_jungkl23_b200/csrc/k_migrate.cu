@@ -55,7 +55,8 @@ __global__ void k_res_reset(uint32_t W, uint32_t C, uint32_t *frame_of, uint32_t
 
 __global__ void k_load_res(const uint32_t *__restrict__ lrm, uint32_t n, uint32_t W, uint32_t *frame_of,
                            uint32_t *stamp_of, uint32_t *block_of, uint32_t *free_bits, uint32_t *lrm_blk,
-                           uint32_t *lrm_stamp, uint32_t *res_bits, DevState *st) {
+                           uint32_t *lrm_stamp, uint32_t *res_bits, const uint32_t *inactive, uint32_t *logpos,
+                           DevState *st) {
   const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i == 0) {
     st->lrm_head = 0;
@@ -72,14 +73,16 @@ __global__ void k_load_res(const uint32_t *__restrict__ lrm, uint32_t n, uint32_
   }
   block_of[i] = b;
   stamp_of[b] = i;
-  lrm_blk[i] = b;
+  lrm_blk[i] = b | (((inactive[b >> 5] >> (b & 31)) & 1u) << 31);  // inactive flag packed in bit 31
+  logpos[b] = i;
   lrm_stamp[i] = i;
   atomicAnd(&free_bits[i >> 5], ~(1u << (i & 31)));
   atomicOr(&res_bits[b >> 5], 1u << (b & 31));
 }
 
 __global__ void k_mark_inactive(const uint32_t *__restrict__ blocks, uint32_t n, int flag, uint32_t W,
-                                uint32_t *inactive, DevState *st) {
+                                uint32_t *inactive, const uint32_t *frame_of, const uint32_t *logpos,
+                                uint32_t *lrm_blk, DevState *st) {
   const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   const uint32_t b = blocks[i];
@@ -89,6 +92,8 @@ __global__ void k_mark_inactive(const uint32_t *__restrict__ blocks, uint32_t n,
   }
   if (flag) atomicOr(&inactive[b >> 5], 1u << (b & 31));
   else atomicAnd(&inactive[b >> 5], ~(1u << (b & 31)));
+  // resident blocks carry the flag in their LRM-log entry (bit 31)
+  if (frame_of[b] != NONE) lrm_blk[logpos[b]] = b | ((flag ? 1u : 0u) << 31);
 }
 
 struct MigArgs {
@@ -96,7 +101,8 @@ struct MigArgs {
   const uint32_t *blocks, *dst;
   uint32_t n;
   uint32_t W, C;
-  uint32_t *frame_of, *stamp_of, *block_of, *free_bits, *lrm_blk, *lrm_stamp, *res_bits;
+  uint32_t *frame_of, *stamp_of, *block_of, *free_bits, *lrm_blk, *lrm_stamp, *res_bits, *logpos;
+  const uint32_t *inactive;
   uint32_t lrm_cap;
   uint32_t *mig_frames, *mig_src, *mig_blocks;
   DevState *st;
@@ -167,14 +173,15 @@ __global__ void __launch_bounds__(PLAN_NT) k_mig_plan(MigArgs a) {
         if (i < tail) {
           b = a.lrm_blk[i];
           s = a.lrm_stamp[i];
-          const uint32_t f = a.frame_of[b];
-          keep = f != NONE && f != CLAIM && a.stamp_of[b] == s;
+          const uint32_t f = a.frame_of[b & 0x7FFFFFFFu];
+          keep = f != NONE && f != CLAIM && a.stamp_of[b & 0x7FFFFFFFu] == s;
         }
         uint32_t tot;
         const uint32_t pre = block_excl_scan(keep, ws, &tot);  // syncs: reads done before writes
         if (keep) {
           a.lrm_blk[outp + pre] = b;
           a.lrm_stamp[outp + pre] = s;
+          a.logpos[b & 0x7FFFFFFFu] = outp + pre;
         }
         outp += tot;
         __syncthreads();
@@ -196,7 +203,8 @@ __global__ void __launch_bounds__(PLAN_NT) k_mig_plan(MigArgs a) {
       a.frame_of[b] = f;
       a.block_of[f] = b;
       a.stamp_of[b] = mc + i;
-      a.lrm_blk[tail + i] = b;
+      a.lrm_blk[tail + i] = b | (((a.inactive[b >> 5] >> (b & 31)) & 1u) << 31);
+      a.logpos[b] = tail + i;
       a.lrm_stamp[tail + i] = mc + i;
       atomicAnd(&a.free_bits[f >> 5], ~(1u << (f & 31)));
       atomicOr(&a.res_bits[b >> 5], 1u << (b & 31));
@@ -378,14 +386,15 @@ cudaError_t launch_load_residency(dum_engine *e, const uint32_t *lrm, uint32_t n
                                   e->d_inactive_bits, e->d_res_bits, false, e->d_state);
   k_load_res<<<(n + 255) / 256 + 1, 256, 0, s>>>(lrm, n, e->g.W, e->d_frame_of, e->d_stamp_of, e->d_block_of,
                                                   e->d_free_bits, e->d_lrm_blk, e->d_lrm_stamp, e->d_res_bits,
-                                                  e->d_state);
+                                                  e->d_inactive_bits, e->d_logpos, e->d_state);
   e->kernel_launches += 2;
   return cudaGetLastError();
 }
 
 cudaError_t launch_mark_inactive(dum_engine *e, const uint32_t *blocks, uint32_t n, int flag, cudaStream_t s) {
   if (n == 0) return cudaSuccess;
-  k_mark_inactive<<<(n + 255) / 256, 256, 0, s>>>(blocks, n, flag, e->g.W, e->d_inactive_bits, e->d_state);
+  k_mark_inactive<<<(n + 255) / 256, 256, 0, s>>>(blocks, n, flag, e->g.W, e->d_inactive_bits, e->d_frame_of,
+                                                  e->d_logpos, e->d_lrm_blk, e->d_state);
   e->kernel_launches += 1;
   return cudaGetLastError();
 }
@@ -415,6 +424,8 @@ cudaError_t launch_migrate(dum_engine *e, int dir, const uint32_t *blocks, const
   a.lrm_blk = e->d_lrm_blk;
   a.lrm_stamp = e->d_lrm_stamp;
   a.res_bits = e->d_res_bits;
+  a.logpos = e->d_logpos;
+  a.inactive = e->d_inactive_bits;
   a.lrm_cap = e->lrm_cap;
   a.mig_frames = e->d_mig_frames;
   a.mig_src = e->d_mig_src;

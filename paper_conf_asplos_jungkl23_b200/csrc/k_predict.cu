@@ -205,7 +205,17 @@ __device__ __forceinline__ bool warp_test_and_set(uint32_t *bitmap, uint32_t b, 
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t w = valid ? (b >> 5) : 0xFFFFFFFFu;
   const uint32_t bit = valid ? 1u << (b & 31) : 0u;
-  const uint32_t grp = __match_any_sync(0xffffffffu, w);
+  // walk lists are mostly runs of consecutive blocks: when the warp's words
+  // are lane 0's word and the next one, two ballots group the lanes (no MATCH)
+  const uint32_t w0 = __shfl_sync(0xffffffffu, w, 0);
+  const bool in0 = w == w0;
+  uint32_t grp;
+  if (__all_sync(0xffffffffu, in0 || w == w0 + 1 || w == 0xFFFFFFFFu)) {
+    const uint32_t m0 = __ballot_sync(0xffffffffu, in0), m1 = __ballot_sync(0xffffffffu, w == w0 + 1);
+    grp = in0 ? m0 : (w == w0 + 1 ? m1 : ~(m0 | m1));
+  } else {
+    grp = __match_any_sync(0xffffffffu, w);
+  }
   const uint32_t comb = __reduce_or_sync(grp, bit);
   const uint32_t leader = __ffs(grp) - 1;
   uint32_t old = 0;

@@ -65,13 +65,14 @@ __device__ void select_tail(const SelectOut &so, uint32_t qi, uint32_t nonres, c
 #pragma unroll
     for (int k = 0; k < ITEMS; ++k) {
       const uint32_t i = c + wid * (32 * ITEMS) + 32 * k + lane;
-      const uint32_t b = blk[k];
+      const uint32_t b = blk[k] & 0x7FFFFFFFu;  // log entry: block | inactive << 31
       bool elig = false, ina = false;
       if (i < tail) {
         elig = !(bitmap[b >> 5] & (1u << (b & 31)));
         if (elig && !clean) elig = __ldg(&so.frame_of[b]) != NONE && __ldg(&so.stamp_of[b]) == so.lrm_stamp[i];
-        if (elig) ina = (__ldg(&so.inactive[b >> 5]) >> (b & 31)) & 1u;
+        ina = blk[k] >> 31;
       }
+      blk[k] = b;
       me[k] = __ballot_sync(0xffffffffu, elig && !ina);
       mi[k] = __ballot_sync(0xffffffffu, elig && ina);
       cw += __popc(me[k]);
@@ -82,17 +83,23 @@ __device__ void select_tail(const SelectOut &so, uint32_t qi, uint32_t nonres, c
       s_icnt[wid] = ci;
     }
     __syncthreads();
-    // exclusive prefix of the warp totals (in log order = warp order)
-    uint32_t pw = 0, pi = 0, tw = 0, ti = 0;
+    // exclusive prefix of the warp totals (log order = warp order): one
+    // packed warp scan over the NW totals (counts <= 128 fit 16 bits)
+    uint32_t pw, pi, tw, ti;
+    {
+      const uint32_t v = lane < NW ? (s_icnt[lane] << 16) | s_wcnt[lane] : 0;
+      uint32_t x = v;
 #pragma unroll
-    for (int w = 0; w < NW; ++w) {
-      const uint32_t a = s_wcnt[w], b2 = s_icnt[w];
-      if (w < (int)wid) {
-        pw += a;
-        pi += b2;
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= (uint32_t)o) x += y;
       }
-      tw += a;
-      ti += b2;
+      const uint32_t ex = __shfl_sync(0xffffffffu, x - v, wid);
+      const uint32_t tot = __shfl_sync(0xffffffffu, x, NW - 1);
+      pw = ex & 0xFFFFu;
+      pi = ex >> 16;
+      tw = tot & 0xFFFFu;
+      ti = tot >> 16;
     }
     const uint32_t left = need - run_wb - run_inv;
 #pragma unroll
