@@ -239,7 +239,7 @@ def run_ours(args, rank, world, local_rank):
     tr = wl.make(args.workload, n_iter=n_iter, seed=seed)
     K, N = tr.K, args.degree
     eng = Engine(num_rows=2048, assoc=2, num_succs=4, degree_n=N, max_blocks=tr.W, max_exec_ids=8192,
-                 hbm_frames=tr.C, device=local_rank,
+                 hbm_frames=tr.C, device=local_rank, corr_capacity=1 << 16,
                  max_batch_faults=max(1 << 20, int(max(tr.faults_in_iteration(i) for i in range(n_iter)) * 1.2)),
                  max_batch_launches=max(K * 2, 4096))
     geo = {"A": 2, "S": 4, "R": 2048}

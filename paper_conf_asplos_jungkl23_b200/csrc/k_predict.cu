@@ -143,6 +143,15 @@ __global__ void __launch_bounds__(CHAIN_NT) k_chain(PredArgs a) {
   const uint32_t lane = threadIdx.x & 31;
   const Geo &g = a.g;
   uint32_t U = 0;
+  {
+    // Pull the (small) correlation table into L2 first: every query's chain
+    // is a sequence of dependent lookups, which then hit L2 instead of HBM.
+    const uint64_t lines = (uint64_t)a.corr_cap * sizeof(CorrSlot) / 128;
+    const uint64_t nthr = (uint64_t)gridDim.x * CHAIN_NT;
+    if (lines <= (16ull << 20) / 128)
+      for (uint64_t l = qi; l < lines; l += nthr)
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(reinterpret_cast<const char *>(a.corr) + l * 128));
+  }
   if (qi < a.nq) {
     const dum_query Q = a.q[qi];
     const bool anchored = Q.anchor != NONE;
@@ -196,38 +205,6 @@ __global__ void __launch_bounds__(CHAIN_NT) k_chain(PredArgs a) {
     a.qbase[qi] = base;
     if (base + U > a.cap) set_err(a.st, ERR_ECAPACITY, base + U);
   }
-}
-
-// Warp-aggregated test-and-set of bit b in a shared bitmap: lanes hitting the
-// same 32-bit word combine into one atomicOr.  Returns true if the block was
-// already present (set before, or by a lower lane of this warp step).
-__device__ __forceinline__ bool warp_test_and_set(uint32_t *bitmap, uint32_t b, bool valid) {
-  const uint32_t lane = threadIdx.x & 31;
-  const uint32_t w = valid ? (b >> 5) : 0xFFFFFFFFu;
-  const uint32_t bit = valid ? 1u << (b & 31) : 0u;
-  // walk lists are mostly runs of consecutive blocks: when the warp's words
-  // are lane 0's word and the next one, two ballots group the lanes (no MATCH)
-  const uint32_t w0 = __shfl_sync(0xffffffffu, w, 0);
-  const bool in0 = w == w0;
-  uint32_t grp;
-  if (__all_sync(0xffffffffu, in0 || w == w0 + 1 || w == 0xFFFFFFFFu)) {
-    const uint32_t m0 = __ballot_sync(0xffffffffu, in0), m1 = __ballot_sync(0xffffffffu, w == w0 + 1);
-    grp = in0 ? m0 : (w == w0 + 1 ? m1 : ~(m0 | m1));
-  } else {
-    grp = __match_any_sync(0xffffffffu, w);
-  }
-  const uint32_t comb = __reduce_or_sync(grp, bit);
-  const uint32_t leader = __ffs(grp) - 1;
-  uint32_t old = 0;
-  if (lane == leader && valid) old = atomicOr(&bitmap[w], comb);
-  old = __shfl_sync(0xffffffffu, old, leader);
-  bool dup = valid && (old & bit);
-  if (__popc(comb) < __popc(grp) && valid) {
-    // two lanes carry the same block: all but the lowest are duplicates
-    const uint32_t same = __match_any_sync(grp, b);
-    dup |= lane != (uint32_t)(__ffs(same) - 1);
-  }
-  return dup;
 }
 
 template <bool SELECT>

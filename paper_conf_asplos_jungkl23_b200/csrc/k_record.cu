@@ -11,6 +11,8 @@
 //                  ("Otherwise, it assigns a new execution ID", PAPER.md L136;
 //                  D3) = rank of each new hash by its minimum launch position
 //                  (order-independent).
+#include <algorithm>
+
 #include "device_util.cuh"
 #include "kernels.cuh"
 
@@ -18,17 +20,18 @@ namespace dum {
 
 constexpr int INGEST_NT = 256;
 constexpr uint32_t INGEST_HCAP = 4096;  // smem hash capacity (n <= 2048 in smem)
+constexpr uint32_t IDCAP = 1024;        // repeated-block hash of the bitmap path
+constexpr uint32_t INGEST_SMEM_MAX = 64 * 1024;
 
 __global__ void __launch_bounds__(INGEST_NT) k_ingest(
     const uint64_t *__restrict__ hash, const uint64_t *__restrict__ off, const uint32_t *__restrict__ faults,
     uint32_t n_launch, uint32_t W, uint32_t l0, uint64_t f0, uint64_t *__restrict__ stage_hash,
     uint64_t *__restrict__ stage_off, uint32_t *__restrict__ stage_norm, uint32_t *__restrict__ stage_cnt,
     uint32_t *__restrict__ stage_slot, unsigned long long *exec_keys, uint32_t *exec_vals, uint32_t *exec_minpos,
-    uint32_t exec_cap, uint32_t *big_pool, uint64_t big_entries, DevState *st) {
-  __shared__ uint32_t hk[INGEST_HCAP];
-  __shared__ uint32_t hv[INGEST_HCAP];
+    uint32_t exec_cap, uint32_t *big_pool, uint64_t big_entries, uint32_t bm_words, DevState *st) {
+  extern __shared__ uint32_t dyn[];  // hash (2 x INGEST_HCAP) or bitmap + small dup hash
   __shared__ uint32_t ws[INGEST_NT / 32];
-  __shared__ uint32_t s_dups;
+  __shared__ uint32_t s_dups, s_ovf;
   const uint32_t i = blockIdx.x;
   if (i >= n_launch) return;
   const uint64_t a = off[i], b = off[i + 1];
@@ -39,10 +42,84 @@ __global__ void __launch_bounds__(INGEST_NT) k_ingest(
     ctr_add(st, DUM_CTR_LAUNCHES, 1);
     s_dups = 0;
   }
-  if (n > 0) {
+  // Big launches (> INGEST_HCAP/2 records) dedupe through a bitmap over the
+  // block-id space when it fits the shared-memory budget: an order-free
+  // warp-aggregated test-and-set finds whether any block repeats (normally
+  // not: the input is then copied), and only repeated blocks go through a
+  // small min-position hash.  Otherwise a private global-pool hash is used.
+  const bool use_bitmap = n > INGEST_HCAP / 2 && bm_words != 0;
+  if (n > 0 && use_bitmap) {
+    uint32_t *bm = dyn, *dk = dyn + ((bm_words + 3) & ~3u), *dv = dk + IDCAP;
+    for (uint32_t t = threadIdx.x; t < bm_words; t += INGEST_NT) bm[t] = 0;
+    for (uint32_t t = threadIdx.x; t < IDCAP; t += INGEST_NT) {
+      dk[t] = NONE;
+      dv[t] = NONE;
+    }
+    if (threadIdx.x == 0) s_ovf = 0;
+    __syncthreads();
+    uint32_t ndup = 0;
+    for (uint32_t c = 0; c < n; c += INGEST_NT) {
+      const uint32_t j = c + threadIdx.x;
+      uint32_t blk = j < n ? faults[a + j] : NONE;
+      const bool inr = j < n && blk < W;
+      if (j < n && blk >= W) {
+        set_err(st, ERR_EINVAL);
+        ++ndup;  // dropped: take the compaction path
+      }
+      if (warp_test_and_set(bm, blk, inr)) {
+        ++ndup;
+        if (!hmap_insert_min(dk, dv, IDCAP, blk, j)) s_ovf = 1;
+      }
+    }
+    if (ndup) s_dups = 1;
+    __syncthreads();
+    uint32_t run = n;
+    if (!s_dups) {
+      for (uint32_t j = threadIdx.x; j < n; j += INGEST_NT) stage_norm[f0 + a + j] = faults[a + j];
+    } else if (!s_ovf) {
+      // every occurrence of a repeated block lowers that block's min position
+      for (uint32_t j = threadIdx.x; j < n; j += INGEST_NT) {
+        const uint32_t blk = faults[a + j];
+        if (blk >= W) continue;
+        for (uint32_t p = 0, sl = hslot(blk, IDCAP); p < IDCAP; ++p, sl = (sl + 1) & (IDCAP - 1)) {
+          const uint32_t kk = dk[sl];
+          if (kk == NONE) break;
+          if (kk == blk) {
+            atomicMin(&dv[sl], j);
+            break;
+          }
+        }
+      }
+      __syncthreads();
+      run = 0;
+      for (uint32_t c = 0; c < n; c += INGEST_NT) {
+        const uint32_t j = c + threadIdx.x;
+        uint32_t blk = NONE, keep = 0;
+        if (j < n) {
+          blk = faults[a + j];
+          if (blk < W) {
+            const uint32_t m = hmap_get(dk, dv, IDCAP, blk);
+            keep = m == NONE || m == j;
+          }
+        }
+        uint32_t tot;
+        const uint32_t pre = block_excl_scan(keep, ws, &tot);
+        if (keep) stage_norm[f0 + a + run + pre] = blk;
+        run += tot;
+      }
+    }
+    if (!s_dups || !s_ovf) {
+      if (threadIdx.x == 0) {
+        stage_cnt[l0 + i] = run;
+        ctr_add(st, DUM_CTR_RAW_RECORDS, n);
+        ctr_add(st, DUM_CTR_NORM_RECORDS, run);
+      }
+    }
+  }
+  if (n > 0 && (!use_bitmap || (s_dups && s_ovf))) {
     // hash of (block -> first position) in shared memory, or in a private
     // region of the global pool for launches with > INGEST_HCAP/2 records
-    uint32_t *keys = hk, *vals = hv;
+    uint32_t *keys = dyn, *vals = dyn + INGEST_HCAP;
     uint32_t cap = pow2ceil(2 * n);
     if (cap < 64) cap = 64;
     bool fits = true;
@@ -55,6 +132,8 @@ __global__ void __launch_bounds__(INGEST_NT) k_ingest(
       keys = big_pool + 2ull * pbase;
       vals = keys + cap;
     }
+    __syncthreads();
+    if (threadIdx.x == 0) s_dups = 0;
     if (fits) {
       for (uint32_t t = threadIdx.x; t < cap; t += INGEST_NT) {
         keys[t] = NONE;
@@ -111,7 +190,7 @@ __global__ void __launch_bounds__(INGEST_NT) k_ingest(
     } else if (threadIdx.x == 0) {
       stage_cnt[l0 + i] = 0;
     }
-  } else if (threadIdx.x == 0) {
+  } else if (n == 0 && threadIdx.x == 0) {
     stage_cnt[l0 + i] = 0;
   }
   if (threadIdx.x == 0) {
@@ -192,10 +271,16 @@ cudaError_t launch_record(dum_engine *e, const uint64_t *hash, const uint64_t *o
   if (n_launch == 0) return cudaSuccess;
   {
   TimerScope t(e, DUM_T_INGEST, s);
-  k_ingest<<<n_launch, INGEST_NT, 0, s>>>(hash, off, faults, n_launch, e->g.W, e->n_staged, e->staged_faults,
-                                          e->d_stage_hash, e->d_stage_off, e->d_stage_norm, e->d_stage_cnt,
-                                          e->d_stage_slot, e->d_exec_keys, e->d_exec_vals, e->d_exec_minpos,
-                                          e->exec_cap, e->d_big_pool, e->big_pool_entries, e->d_state);
+  const uint32_t bmw = (e->g.W + 31) / 32;
+  const size_t bm_bytes = (size_t)((bmw + 3) & ~3u) * 4 + 2 * IDCAP * 4;
+  const bool bm_ok = bm_bytes <= INGEST_SMEM_MAX;
+  const size_t smem = std::max<size_t>(2 * INGEST_HCAP * 4, bm_ok ? bm_bytes : 0);
+  cudaFuncSetAttribute(k_ingest, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  k_ingest<<<n_launch, INGEST_NT, smem, s>>>(hash, off, faults, n_launch, e->g.W, e->n_staged, e->staged_faults,
+                                             e->d_stage_hash, e->d_stage_off, e->d_stage_norm, e->d_stage_cnt,
+                                             e->d_stage_slot, e->d_exec_keys, e->d_exec_vals, e->d_exec_minpos,
+                                             e->exec_cap, e->d_big_pool, e->big_pool_entries, bm_ok ? bmw : 0,
+                                             e->d_state);
   }
   TimerScope t(e, DUM_T_EXEC_ASSIGN, s);
   k_exec_assign<<<1, ASSIGN_NT, 0, s>>>(n_launch, e->n_staged, e->d_stage_slot, e->d_stage_hash, e->d_exec_vals,
