@@ -179,14 +179,37 @@ __global__ void __launch_bounds__(CHAIN_NT) k_chain(PredArgs a) {
     // the chain with the same (unanchored) walk adds nothing (exact; keeps the
     // reservation tight)
     loff[0] = 0;
-    for (uint32_t d = 0; d < nk; ++d) {
-      const uint32_t e = kern[d];
-      uint32_t len = (d == 0 && anchored) ? (uint32_t)a.anchor_range[2 * qi + 1] : __ldg(a.walk_len + e);
-      for (uint32_t d2 = anchored ? 1u : 0u; d2 < d && len; ++d2)
-        if (kern[d2] == e) len = 0;
-      gkern[d] = e;
-      U += len;
-      loff[d + 1] = U;
+    uint32_t lens[4];
+    unsigned long long seen_lo = 0, seen_hi = 0;  // 128-bit filter of the chain's exec IDs
+    for (uint32_t d0 = 0; d0 < nk; d0 += 4) {
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {  // independent loads first
+        const uint32_t d = d0 + k;
+        lens[k] = d < nk ? ((d == 0 && anchored) ? (uint32_t)a.anchor_range[2 * qi + 1]
+                                                 : __ldg(a.walk_len + kern[d]))
+                         : 0u;
+      }
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const uint32_t d = d0 + k;
+        if (d >= nk) break;
+        const uint32_t e = kern[d];
+        uint32_t len = lens[k];
+        const uint32_t hb = fmix32(e) & 127;
+        const unsigned long long bit = 1ull << (hb & 63);
+        const bool maybe = hb < 64 ? (seen_lo & bit) : (seen_hi & bit);
+        if (maybe) {  // exact check only on a filter hit
+          for (uint32_t d2 = anchored ? 1u : 0u; d2 < d && len; ++d2)
+            if (kern[d2] == e) len = 0;
+        }
+        if (!(d == 0 && anchored)) {
+          if (hb < 64) seen_lo |= bit;
+          else seen_hi |= bit;
+        }
+        gkern[d] = e;
+        U += len;
+        loff[d + 1] = U;
+      }
     }
     a.qnk[qi] = nk;
   }
