@@ -113,9 +113,12 @@ void free_all(dum_engine *e) {
                   e->d_walk_chain, e->d_walk_tmp, e->d_walk_out, e->d_anchor_pool, e->d_anchor_range,
                   e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits, e->d_inactive_bits, e->d_res_bits, e->d_logpos, e->d_lrm_blk,
                   e->d_lrm_stamp, e->d_mig_frames, e->d_mig_src, e->d_mig_blocks, e->d_state, e->d_qkern,
-                  e->d_qloff, e->d_qnk, e->d_qbase};
+                  e->d_qloff, e->d_qnk, e->d_qbase, e->d_rec_slot, e->d_jump};
   for (void *p : ptrs)
     if (p) cudaFree(p);
+  if (e->ev_fork) cudaEventDestroy(e->ev_fork);
+  if (e->ev_join) cudaEventDestroy(e->ev_join);
+  if (e->side) cudaStreamDestroy(e->side);
   if (e->h_state) cudaFreeHost(e->h_state);
   for (auto &t : e->pending) {
     cudaEventDestroy(t.a);
@@ -210,6 +213,8 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   e->exec_cap = std::max<uint32_t>(64, pow2ceil_h(2ull * g.Emax));
   const uint64_t corr_records = cfg->corr_capacity ? cfg->corr_capacity : 16ull * g.Emax;
   e->corr_cap = pow2ceil_h(2 * corr_records);
+  e->jump_levels = 1;
+  while ((1u << e->jump_levels) < g.N) ++e->jump_levels;  // d <= N - 1 needs bits 0..levels-1
   e->stage_launch_cap = cfg->max_batch_launches ? cfg->max_batch_launches : 65536;
   e->stage_fault_cap = cfg->max_batch_faults ? cfg->max_batch_faults : (16ull << 20);
   e->big_pool_entries = 4 * e->stage_fault_cap;
@@ -229,6 +234,11 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_exec_minpos, e->exec_cap + 1));
   A_(dmalloc(&e->d_exec_hash, g.Emax));
   A_(dmalloc(&e->d_corr, e->corr_cap));
+  A_(dmalloc(&e->d_rec_slot, e->corr_cap));
+  A_(dmalloc(&e->d_jump, (uint64_t)e->jump_levels * e->corr_cap));
+  A_(cudaStreamCreateWithFlags(&e->side, cudaStreamNonBlocking));
+  A_(cudaEventCreateWithFlags(&e->ev_fork, cudaEventDisableTiming));
+  A_(cudaEventCreateWithFlags(&e->ev_join, cudaEventDisableTiming));
   A_(dmalloc(&e->d_tbl, (uint64_t)g.Emax * g.R * g.stride));
   A_(dmalloc(&e->d_start_end, 2ull * g.Emax));
   A_(dmalloc(&e->d_walk, (uint64_t)g.Emax * g.walk_cap));

@@ -126,6 +126,11 @@ struct dum_engine {
   // corr
   uint32_t corr_cap;
   dum::CorrSlot *d_corr;
+  uint32_t *d_rec_slot;   // [corr_cap] slots of the records in insertion order
+  uint32_t *d_jump;       // [jump_levels][corr_cap] J_k = next^(2^k) over record slots (k_jump.cu)
+  uint32_t jump_levels;
+  cudaStream_t side;      // jump-table build runs here, overlapping the block-table apply
+  cudaEvent_t ev_fork, ev_join;
   // block tables / walk cache
   uint32_t *d_tbl, *d_start_end, *d_walk, *d_walk_len;
   // staging

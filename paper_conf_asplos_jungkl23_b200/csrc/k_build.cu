@@ -25,6 +25,7 @@
 
 #include "device_util.cuh"
 #include "kernels.cuh"
+#include "corr.cuh"
 #include "walk_seq.cuh"
 
 namespace dum {
@@ -38,42 +39,10 @@ constexpr uint32_t WCAP = 2048;   // smem per-row counts (latest launch <= 2048 
 // ---------------------------------------------------------------------------
 // k_build_prep
 // ---------------------------------------------------------------------------
-__device__ __forceinline__ void corr_upsert(CorrSlot *corr, uint32_t cap, uint32_t owner, uint32_t h1, uint32_t h2,
-                                            uint32_t h3, uint32_t succ, uint32_t k, DevState *st) {
-  const unsigned long long k0 = (unsigned long long)owner | ((unsigned long long)h1 << 32);
-  const unsigned long long k1 = (unsigned long long)h2 | ((unsigned long long)h3 << 32);
-  uint32_t s = (uint32_t)fmix64(k0 * 0x9E3779B97F4A7C15ull ^ fmix64(k1)) & (cap - 1);
-  for (uint32_t p = 0; p < cap; ++p) {
-    CorrSlot *sl = corr + s;
-    const volatile uint32_t *kv = sl->key;
-    uint32_t c0 = kv[0];
-    bool mine = false;
-    if (c0 == NONE) {
-      unsigned long long o0, o1;
-      cas128(sl->key, EMPTY64, EMPTY64, k0, k1, o0, o1);
-      if (o0 == EMPTY64 && o1 == EMPTY64) {
-        atomicAdd(&st->corr_used, 1u);
-        mine = true;
-      } else {
-        mine = (o0 == k0 && o1 == k1);
-      }
-    } else {
-      mine = c0 == owner && kv[1] == h1 && kv[2] == h2 && kv[3] == h3;
-    }
-    if (mine) {
-      atomicMax(&sl->last, ((unsigned long long)k << 32) | succ);
-      atomicMin(&sl->first, (unsigned long long)k);
-      return;
-    }
-    s = (s + 1) & (cap - 1);
-  }
-  set_err(st, ERR_ECAPACITY, 2ull * cap);
-}
-
 __global__ void k_build_prep(uint32_t n_staged, uint32_t k0, const uint32_t *__restrict__ stage_exec,
                              const uint32_t *__restrict__ stage_cnt, CorrSlot *corr, uint32_t corr_cap,
-                             uint32_t *head, uint32_t *__restrict__ next, uint32_t *__restrict__ order,
-                             DevState *st) {
+                             uint32_t *rec_slot, uint32_t *head, uint32_t *__restrict__ next,
+                             uint32_t *__restrict__ order, DevState *st) {
   const uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
   if (j == 0) {
     st->pool_big = 0;
@@ -87,7 +56,7 @@ __global__ void k_build_prep(uint32_t n_staged, uint32_t k0, const uint32_t *__r
   const uint32_t e = stage_exec[j];
   const uint32_t owner = prev(1);
   const bool up = owner != NONE && e != NONE;
-  if (up) corr_upsert(corr, corr_cap, owner, prev(4), prev(3), prev(2), e, k0 + j, st);
+  if (up) corr_upsert(corr, corr_cap, rec_slot, owner, prev(4), prev(3), prev(2), e, k0 + j, st);
   const uint32_t nup = __popc(__ballot_sync(__activemask(), up));
   if ((threadIdx.x & 31) == __ffs(__activemask()) - 1) ctr_add(st, DUM_CTR_CORR_UPSERTS, nup);
   if (e != NONE && stage_cnt[j] > 0) {
@@ -701,8 +670,17 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   TimerScope t(e, DUM_T_BUILD_PREP, s);
   cudaMemsetAsync(e->d_state->cls_cnt, 0, sizeof(e->d_state->cls_cnt), s);
   k_build_prep<<<(n + 255) / 256, 256, 0, s>>>(n, (uint32_t)e->built_launches, e->d_stage_exec, e->d_stage_cnt,
-                                                e->d_corr, e->corr_cap, e->d_head, e->d_next, e->d_order,
+                                                e->d_corr, e->corr_cap, e->d_rec_slot, e->d_head, e->d_next,
+                                                e->d_order,
                                                 e->d_state);
+  }
+  // the jump tables depend only on the correlation table, final here
+  cudaEventRecord(e->ev_fork, s);
+  cudaStreamWaitEvent(e->side, e->ev_fork, 0);
+  {
+    const cudaError_t je = launch_jump_tables(e, e->side);
+    cudaEventRecord(e->ev_join, e->side);
+    if (je != cudaSuccess) return je;
   }
   BuildArgs ba;
   ba.g = e->g;
@@ -757,6 +735,7 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
       fclose(f);
     }
   }
+  cudaStreamWaitEvent(s, e->ev_join, 0);
   e->kernel_launches += 3;
   return cudaGetLastError();
 }

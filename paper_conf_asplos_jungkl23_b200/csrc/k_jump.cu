@@ -1,0 +1,56 @@
+// Jump tables over the execution ID correlation table, so that a query's
+// chain of up to N next-kernel predictions (D16)
+// costs O(log N) dependent loads instead of N.
+//
+// For record r = (owner e; h1, h2, h3 -> succ n), the next lookup of the chain
+// is the record (n; h2, h3, e) (D16: the history shifts in the predicted ID),
+// so next(r) is a function of r alone.  J_0 = next, J_{k+1} = J_k o J_k;
+// the chain of a query whose first record is r0 is succ(next^d(r0)) for
+// d = 0, 1, ... until next^d(r0) is absent.  Rebuilt after every build on a
+// side stream (it only reads the correlation table) while the block tables
+// are applied.
+#include "corr.cuh"
+#include "device_util.cuh"
+#include "kernels.cuh"
+
+namespace dum {
+
+constexpr int JUMP_NT = 256;
+
+__global__ void __launch_bounds__(JUMP_NT) k_jump0(const CorrSlot *corr, uint32_t cap, const uint32_t *rec_slot,
+                                                   uint32_t *j0, const DevState *st) {
+  const uint32_t nrec = min(*(const volatile uint32_t *)&st->corr_used, cap);
+  for (uint32_t r = blockIdx.x * JUMP_NT + threadIdx.x; r < nrec; r += gridDim.x * JUMP_NT) {
+    const uint32_t s = rec_slot[r];
+    const uint4 kk = __ldcg(reinterpret_cast<const uint4 *>(corr + s));
+    const uint32_t succ = (uint32_t)(__ldcg(&corr[s].last) & 0xFFFFFFFFull);
+    uint32_t dummy;
+    j0[s] = corr_find(corr, cap, succ, kk.z, kk.w, kk.x, &dummy);
+  }
+}
+
+__global__ void __launch_bounds__(JUMP_NT) k_jumpk(uint32_t cap, const uint32_t *rec_slot, const uint32_t *jprev,
+                                                   uint32_t *jnext, const DevState *st) {
+  const uint32_t nrec = min(*(const volatile uint32_t *)&st->corr_used, cap);
+  for (uint32_t r = blockIdx.x * JUMP_NT + threadIdx.x; r < nrec; r += gridDim.x * JUMP_NT) {
+    const uint32_t s = rec_slot[r];
+    const uint32_t m = __ldcg(jprev + s);
+    jnext[s] = m == NONE ? NONE : __ldcg(jprev + m);
+  }
+}
+
+cudaError_t launch_jump_tables(dum_engine *e, cudaStream_t s) {
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const uint32_t grid = (uint32_t)sms * 4;
+  TimerScope t(e, DUM_T_JUMP, s);
+  k_jump0<<<grid, JUMP_NT, 0, s>>>(e->d_corr, e->corr_cap, e->d_rec_slot, e->d_jump, e->d_state);
+  for (uint32_t k = 1; k < e->jump_levels; ++k)
+    k_jumpk<<<grid, JUMP_NT, 0, s>>>(e->corr_cap, e->d_rec_slot, e->d_jump + (uint64_t)(k - 1) * e->corr_cap,
+                                     e->d_jump + (uint64_t)k * e->corr_cap, e->d_state);
+  e->kernel_launches += e->jump_levels;
+  return cudaGetLastError();
+}
+
+}  // namespace dum

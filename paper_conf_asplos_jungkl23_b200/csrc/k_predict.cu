@@ -4,12 +4,13 @@
 //  k_anchor_walk   WALK(e, anchor) for fault-anchored queries (PAPER.md L156:
 //                  "calculates the UM block addresses for prefetching with the
 //                  faulted block address"; D14) with the sequential walker.
-//  k_chain         one thread per query: chain up to n next-kernel predictions
+//  k_chain         one warp per query: chain up to n next-kernel predictions
 //                  through the execution ID correlation table (PAPER.md,
-//                  L220; D15, D16); window layout (per-kernel offsets) and the
-//                  query's output reservation.  All queries' chains run
-//                  concurrently, so the serial lookup latency is paid once per
-//                  call instead of once per query.
+//                  L220; D15, D16); lane d reaches the record of step d with
+//                  popcount(d) loads from the jump tables (k_jump.cu), so the
+//                  chain costs O(log n) dependent loads instead of n; window
+//                  layout (per-kernel offsets) and the query's output
+//                  reservation.
 //  k_predict       one CTA per query: gather the walk lists of the window's
 //                  kernels and keep the first occurrence of every block (D17),
 //                  emitting (block, exec ID) prefetch commands.
@@ -21,6 +22,7 @@
 //                  re-compaction overwrite the output.
 //                  SELECT: the fused pre-eviction selection of a8 reuses the
 //                  window bitmap (select_tail.cuh).
+#include "corr.cuh"
 #include "device_util.cuh"
 #include "kernels.cuh"
 #include "select_tail.cuh"
@@ -45,24 +47,6 @@ __global__ void k_make_queries(const uint32_t *__restrict__ seq, uint32_t n_seq,
   q.anchor = NONE;
   q.n = degree;
   out[i - first] = q;
-}
-
-// lookup(e, h1, h2, h3) -> successor or NONE (A9).  The 32 B slot is read with
-// two independent 16 B loads (one round trip per probe).
-__device__ __forceinline__ uint32_t corr_lookup(const CorrSlot *corr, uint32_t cap, uint32_t owner, uint32_t h1,
-                                                uint32_t h2, uint32_t h3) {
-  const unsigned long long k0 = (unsigned long long)owner | ((unsigned long long)h1 << 32);
-  const unsigned long long k1 = (unsigned long long)h2 | ((unsigned long long)h3 << 32);
-  uint32_t s = (uint32_t)fmix64(k0 * 0x9E3779B97F4A7C15ull ^ fmix64(k1)) & (cap - 1);
-  for (uint32_t p = 0; p < cap; ++p) {
-    const uint4 *sp = reinterpret_cast<const uint4 *>(corr + s);
-    const uint4 kk = __ldcg(sp);
-    const uint4 vv = __ldcg(sp + 1);
-    if (kk.x == NONE) return NONE;
-    if (kk.x == owner && kk.y == h1 && kk.z == h2 && kk.w == h3) return vv.x;  // low word of `last`
-    s = (s + 1) & (cap - 1);
-  }
-  return NONE;
 }
 
 __global__ void k_anchor_walk(Geo g, const dum_query *__restrict__ q, uint32_t nq, const uint32_t *tbl,
@@ -116,6 +100,7 @@ struct PredArgs {
   uint32_t nq;
   const CorrSlot *corr;
   uint32_t corr_cap;
+  const uint32_t *jump;  // [levels][corr_cap]
   const uint32_t *walk, *walk_len;
   const uint32_t *anchor_pool;
   const uint64_t *anchor_range;
@@ -135,96 +120,92 @@ struct PredArgs {
   SelectOut so;     // fused a8 outputs (SELECT only)
 };
 
-constexpr int CHAIN_NT = 64;
+constexpr int CHAIN_WARPS = 8;
 
-__global__ void __launch_bounds__(CHAIN_NT) k_chain(PredArgs a) {
-  __shared__ uint32_t skern[CHAIN_NT][MAXN + 1];  // per-thread chain (repeat check stays on chip)
-  const uint32_t qi = blockIdx.x * CHAIN_NT + threadIdx.x;
-  const uint32_t lane = threadIdx.x & 31;
+__global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
+  __shared__ uint32_t skern[CHAIN_WARPS][MAXN + 1];
+  __shared__ uint32_t s_u[CHAIN_WARPS];
+  __shared__ unsigned long long s_base;
+  const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const uint32_t qi = blockIdx.x * CHAIN_WARPS + w;
+  const uint32_t below = (1u << lane) - 1;
   const Geo &g = a.g;
   uint32_t U = 0;
-  {
-    // Pull the (small) correlation table into L2 first: every query's chain
-    // is a sequence of dependent lookups, which then hit L2 instead of HBM.
-    const uint64_t lines = (uint64_t)a.corr_cap * sizeof(CorrSlot) / 128;
-    const uint64_t nthr = (uint64_t)gridDim.x * CHAIN_NT;
-    if (lines <= (16ull << 20) / 128)
-      for (uint64_t l = qi; l < lines; l += nthr)
-        asm volatile("prefetch.global.L2 [%0];" ::"l"(reinterpret_cast<const char *>(a.corr) + l * 128));
-  }
   if (qi < a.nq) {
     const dum_query Q = a.q[qi];
     const bool anchored = Q.anchor != NONE;
     const uint32_t E = *(volatile uint32_t *)&a.st->E;
-    uint32_t *kern = skern[threadIdx.x];
-    uint32_t *gkern = a.qkern + (uint64_t)qi * (g.N + 1);
-    uint32_t *loff = a.qloff + (uint64_t)qi * (g.N + 2);
+    uint32_t *kern = skern[w];
     uint32_t nk = 0;
     if (Q.exec < E) {
-      // the serial part: only the dependent lookups
       const uint32_t n = Q.n < g.N ? Q.n : g.N;
-      uint32_t cur = Q.exec, h1 = Q.hist[0], h2 = Q.hist[1], h3 = Q.hist[2];
-      kern[nk++] = cur;
-      for (uint32_t i = 0; i < n; ++i) {
-        const uint32_t nx = corr_lookup(a.corr, a.corr_cap, cur, h1, h2, h3);
-        if (nx == NONE) break;
-        kern[nk++] = nx;
-        h1 = h2;  // D16: shift register over predicted IDs
-        h2 = h3;
-        h3 = cur;
-        cur = nx;
+      uint32_t dummy = 0;
+      // record of step 0: (e; h1, h2, h3) (D15); every lane reads the same slots
+      const uint32_t r0 = n ? corr_find(a.corr, a.corr_cap, Q.exec, Q.hist[0], Q.hist[1], Q.hist[2], &dummy) : NONE;
+      if (lane == 0) kern[0] = Q.exec;
+      nk = 1;
+      for (uint32_t d0 = 0; d0 < n && r0 != NONE; d0 += 32) {
+        // lane d: record of step d = next^d(r0) (D16's shifted history), via
+        // the binary digits of d; absent anywhere on the way -> NONE
+        const uint32_t d = d0 + lane;
+        uint32_t s = d < n ? r0 : NONE;
+        for (uint32_t k = 0; s != NONE && (d >> k); ++k)
+          if ((d >> k) & 1u) s = __ldcg(a.jump + (uint64_t)k * a.corr_cap + s);
+        if (s != NONE) kern[d + 1] = (uint32_t)(__ldcg(&a.corr[s].last) & 0xFFFFFFFFull);
+        const uint32_t valid = __ballot_sync(0xffffffffu, s != NONE);  // a prefix of the lanes
+        const uint32_t cnt = valid == 0xffffffffu ? 32u : (uint32_t)__ffs(~valid) - 1;
+        nk += cnt;
+        if (cnt < 32) break;
       }
     }
-    // window layout: walk lengths (independent loads), a kernel met earlier in
-    // the chain with the same (unanchored) walk adds nothing (exact; keeps the
-    // reservation tight)
-    loff[0] = 0;
-    uint32_t lens[4];
-    unsigned long long seen_lo = 0, seen_hi = 0;  // 128-bit filter of the chain's exec IDs
-    for (uint32_t d0 = 0; d0 < nk; d0 += 4) {
+    __syncwarp();
+    // window layout: walk lengths; a kernel met earlier in the chain with the
+    // same (unanchored) walk adds nothing (exact; keeps the reservation tight)
+    uint32_t *gkern = a.qkern + (uint64_t)qi * (g.N + 1);
+    uint32_t *loff = a.qloff + (uint64_t)qi * (g.N + 2);
+    for (uint32_t d0 = 0; d0 < nk; d0 += 32) {
+      const uint32_t d = d0 + lane;
+      const bool v = d < nk, anc0 = d == 0 && anchored;
+      const uint32_t e = v ? kern[d] : NONE;
+      uint32_t len = v ? (anc0 ? (uint32_t)a.anchor_range[2 * qi + 1] : __ldg(a.walk_len + e)) : 0u;
+      const uint32_t key = (v && !anc0) ? e : NONE;
+      const uint32_t m = __match_any_sync(0xffffffffu, key);
+      if (key != NONE && (m & below)) len = 0;  // an earlier step of this pass
+      if (len)
+        for (uint32_t d2 = anchored ? 1u : 0u; d2 < d0; ++d2)
+          if (kern[d2] == e) {
+            len = 0;
+            break;
+          }
+      uint32_t incl = len;
 #pragma unroll
-      for (int k = 0; k < 4; ++k) {  // independent loads first
-        const uint32_t d = d0 + k;
-        lens[k] = d < nk ? ((d == 0 && anchored) ? (uint32_t)a.anchor_range[2 * qi + 1]
-                                                 : __ldg(a.walk_len + kern[d]))
-                         : 0u;
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= (uint32_t)o) incl += y;
       }
-#pragma unroll
-      for (int k = 0; k < 4; ++k) {
-        const uint32_t d = d0 + k;
-        if (d >= nk) break;
-        const uint32_t e = kern[d];
-        uint32_t len = lens[k];
-        const uint32_t hb = fmix32(e) & 127;
-        const unsigned long long bit = 1ull << (hb & 63);
-        const bool maybe = hb < 64 ? (seen_lo & bit) : (seen_hi & bit);
-        if (maybe) {  // exact check only on a filter hit
-          for (uint32_t d2 = anchored ? 1u : 0u; d2 < d && len; ++d2)
-            if (kern[d2] == e) len = 0;
-        }
-        if (!(d == 0 && anchored)) {
-          if (hb < 64) seen_lo |= bit;
-          else seen_hi |= bit;
-        }
+      if (v) {
         gkern[d] = e;
-        U += len;
-        loff[d + 1] = U;
+        loff[d + 1] = U + incl;
       }
+      U += __shfl_sync(0xffffffffu, incl, 31);
     }
-    a.qnk[qi] = nk;
+    if (lane == 0) {
+      loff[0] = 0;
+      a.qnk[qi] = nk;
+    }
   }
-  // warp-aggregated output reservation
-  uint32_t incl = U;
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
-    if (lane >= (uint32_t)o) incl += y;
+  // CTA-aggregated output reservation
+  if (lane == 0) s_u[w] = U;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long tot = 0;
+    for (int i = 0; i < CHAIN_WARPS; ++i) tot += s_u[i];
+    s_base = tot ? atomicAdd(&a.st->pool_pairs, tot) : 0ull;
   }
-  unsigned long long wbase = 0;
-  if (lane == 31 && incl) wbase = atomicAdd(&a.st->pool_pairs, (unsigned long long)incl);
-  wbase = __shfl_sync(0xffffffffu, wbase, 31);
-  if (qi < a.nq) {
-    const unsigned long long base = wbase + incl - U;
+  __syncthreads();
+  if (qi < a.nq && lane == 0) {
+    unsigned long long base = s_base;
+    for (uint32_t i = 0; i < w; ++i) base += s_u[i];
     a.qbase[qi] = base;
     if (base + U > a.cap) set_err(a.st, ERR_ECAPACITY, base + U);
   }
@@ -496,6 +477,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   a.nq = nq;
   a.corr = e->d_corr;
   a.corr_cap = e->corr_cap;
+  a.jump = e->d_jump;
   a.walk = e->d_walk;
   a.walk_len = e->d_walk_len;
   a.anchor_pool = e->d_anchor_pool;
@@ -520,7 +502,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   }
   {
     TimerScope t(e, DUM_T_CHAIN, s);
-    k_chain<<<(nq + CHAIN_NT - 1) / CHAIN_NT, CHAIN_NT, 0, s>>>(a);
+    k_chain<<<(nq + CHAIN_WARPS - 1) / CHAIN_WARPS, CHAIN_WARPS * 32, 0, s>>>(a);
   }
   const size_t smem = (size_t)((a.nwords + 3) & ~3u) * 4 + 2 * DCAP * 4;
   if (sel) {
