@@ -122,11 +122,15 @@ def algorithmic_bytes(ctr, geo, N, fused=True):
     from paper_conf_asplos_jungkl23_b200.binding import CTR
     c = {k: int(ctr[v]) for k, v in CTR.items()}
     set_bytes = 4 * geo["A"] * (1 + geo["S"])
-    predict = (24 * c["QUERIES"] + 32 * c["CHAIN"] + 4 * c["GATHERED"] + 8 * c["EMITTED"]
-               + c["QUERIES"] * (16 + 4 * (N + 2) + 4 * (N + 1)))
-    select_core = 4 * c["SEL_SCANNED"] + 4 * c["SEL_VICTIMS"] + 32 * c["QUERIES"]
-    if fused:  # window set reused from predict: residency lookups per emitted pair
-        predict += 4 * c["EMITTED"] + select_core
+    # predict: minimal HBM traffic = its outputs (pairs, per-query ranges,
+    # kern_off, chain) + the per-query scratch written by k_chain + one read of
+    # each run entry; re-reads of L2-resident shared inputs (walk lists, the
+    # residency bitmap, the LRM log) are not counted
+    predict = (8 * c["EMITTED"] + 8 * c["RUNS"] + 4 * c["CHAIN"]
+               + c["QUERIES"] * (16 + 24 + 12 + 4 * (N + 2) + 4 * (N + 1)))
+    select_core = 4 * c["SEL_VICTIMS"] + 32 * c["QUERIES"]
+    if fused:
+        predict += select_core
     return {
         "k_ingest": 4 * c["RAW_RECORDS"] + 4 * c["NORM_RECORDS"] + 28 * c["LAUNCHES"],
         "k_exec_assign": 16 * c["LAUNCHES"],
@@ -134,7 +138,7 @@ def algorithmic_bytes(ctr, geo, N, fused=True):
         "k_apply_walk": (4 * c["OPS"] + 2 * set_bytes * c["SETS"] + set_bytes * c["WALK_ROWS"]
                          + 4 * c["WALK_OUT"] + 16 * c["EXEC_BUILT"]),
         "k_predict": predict,
-        "k_select": 8 * c["SEL_WINDOW"] + 4 * c["SEL_WINDOW"] + select_core,
+        "k_select": 8 * c["SEL_WINDOW"] + select_core,
     }
 
 

@@ -284,6 +284,7 @@ enum {
   DUM_CTR_SEL_SCANNED,      /* LRM-log entries scanned by select         */
   DUM_CTR_SEL_VICTIMS,      /* victims selected                          */
   DUM_CTR_MIG_BLOCKS,       /* 2 MiB blocks copied                       */
+  DUM_CTR_RUNS,             /* walk bitmap runs inserted by predict      */
   DUM_NCOUNTERS = 24
 };
 int dum_read_counters(dum_engine *eng, uint64_t out[DUM_NCOUNTERS], int reset);

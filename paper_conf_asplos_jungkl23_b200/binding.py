@@ -20,7 +20,7 @@ H2D, D2H, INVALIDATE, D2D = 0, 1, 2, 3
 NCOUNTERS, NTIMERS = 24, 16
 CTR = {n: i for i, n in enumerate(["RAW_RECORDS", "NORM_RECORDS", "LAUNCHES", "CORR_UPSERTS", "EXEC_BUILT", "OPS",
                                    "SETS", "WALK_ROWS", "WALK_OUT", "QUERIES", "CHAIN", "GATHERED", "EMITTED",
-                                   "SEL_WINDOW", "SEL_SCANNED", "SEL_VICTIMS", "MIG_BLOCKS"])}
+                                   "SEL_WINDOW", "SEL_SCANNED", "SEL_VICTIMS", "MIG_BLOCKS", "RUNS"])}
 TIMER = {n: i for i, n in enumerate(["INGEST", "EXEC_ASSIGN", "BUILD_PREP", "APPLY_WALK", "WALK_SLOW",
                                      "MAKE_QUERIES", "ANCHOR_WALK", "PREDICT", "SELECT", "MIG_PLAN", "COPY",
                                      "RESIDENCY", "CHAIN", "JUMP"])}

@@ -93,6 +93,7 @@ int reset_state(dum_engine *e, cudaStream_t s) {
   CK(fill(e->d_tbl, (uint64_t)g.Emax * g.R * g.stride, NONE, s));
   CK(fill(e->d_start_end, 2ull * g.Emax, NONE, s));
   CK(cudaMemsetAsync(e->d_walk_len, 0, 4ull * g.Emax, s));
+  CK(cudaMemsetAsync(e->d_wrun_len, 0, 4ull * g.Emax, s));
   CK(fill(e->d_head, g.Emax, NONE, s));
   k_init_state<<<1, 1, 0, s>>>(e->d_state);
   CK(cudaGetLastError());
@@ -113,7 +114,7 @@ void free_all(dum_engine *e) {
                   e->d_walk_chain, e->d_walk_tmp, e->d_walk_out, e->d_anchor_pool, e->d_anchor_range,
                   e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits, e->d_inactive_bits, e->d_res_bits, e->d_logpos, e->d_lrm_blk,
                   e->d_lrm_stamp, e->d_mig_frames, e->d_mig_src, e->d_mig_blocks, e->d_state, e->d_qkern,
-                  e->d_qloff, e->d_qnk, e->d_qbase, e->d_rec_slot, e->d_jump};
+                  e->d_qloff, e->d_qnk, e->d_qbase, e->d_rec_slot, e->d_jump, e->d_wrun, e->d_wrun_len, e->d_qeoff, e->d_qgoff};
   for (void *p : ptrs)
     if (p) cudaFree(p);
   if (e->ev_fork) cudaEventDestroy(e->ev_fork);
@@ -205,7 +206,9 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   g.row_index = cfg->row_index;
   g.set_u32 = A * (1 + S);
   g.stride = (g.set_u32 + 7) / 8 * 8;  // 32 B sectors
-  g.walk_cap = 1 + S * (R * A + 1);
+  // a walk has at most 1 + S(RA + 1) blocks; rounded up to 8 so that every
+  // walk (and its run list) starts 32 B aligned (vector loads in k_predict)
+  g.walk_cap = (1 + S * (R * A + 1) + 7) / 8 * 8;
   if (cudaSetDevice(cfg->device) != cudaSuccess) {
     delete e;
     return DUM_ECUDA;
@@ -236,13 +239,21 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_corr, e->corr_cap));
   A_(dmalloc(&e->d_rec_slot, e->corr_cap));
   A_(dmalloc(&e->d_jump, (uint64_t)e->jump_levels * e->corr_cap));
-  A_(cudaStreamCreateWithFlags(&e->side, cudaStreamNonBlocking));
+  {
+    // the jump tables are on the critical path of the next predict and tiny:
+    // their CTAs go ahead of the block-table apply they overlap
+    int lo = 0, hi = 0;
+    cudaDeviceGetStreamPriorityRange(&lo, &hi);
+    A_(cudaStreamCreateWithPriority(&e->side, cudaStreamNonBlocking, hi));
+  }
   A_(cudaEventCreateWithFlags(&e->ev_fork, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_join, cudaEventDisableTiming));
   A_(dmalloc(&e->d_tbl, (uint64_t)g.Emax * g.R * g.stride));
   A_(dmalloc(&e->d_start_end, 2ull * g.Emax));
   A_(dmalloc(&e->d_walk, (uint64_t)g.Emax * g.walk_cap));
   A_(dmalloc(&e->d_walk_len, g.Emax));
+  A_(dmalloc(&e->d_wrun, 2ull * g.Emax * g.walk_cap));
+  A_(dmalloc(&e->d_wrun_len, g.Emax));
   A_(dmalloc(&e->d_in_hash, e->stage_launch_cap));
   A_(dmalloc(&e->d_in_off, e->stage_launch_cap + 1ull));
   A_(dmalloc(&e->d_in_faults, e->stage_fault_cap));
@@ -265,6 +276,8 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_anchor_range, 2ull * e->anchor_range_cap));
   A_(dmalloc(&e->d_qkern, (uint64_t)e->anchor_range_cap * (g.N + 1)));
   A_(dmalloc(&e->d_qloff, (uint64_t)e->anchor_range_cap * (g.N + 2)));
+  A_(dmalloc(&e->d_qeoff, (uint64_t)e->anchor_range_cap * (g.N + 2)));
+  A_(dmalloc(&e->d_qgoff, (uint64_t)e->anchor_range_cap * (g.N + 2)));
   A_(dmalloc(&e->d_qnk, e->anchor_range_cap));
   A_(dmalloc(&e->d_qbase, e->anchor_range_cap));
   A_(dmalloc(&e->d_frame_of, g.W));

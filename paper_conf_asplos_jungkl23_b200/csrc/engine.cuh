@@ -11,6 +11,8 @@
 //                                    a 32 B sector
 //   start_end    u32[E][2]
 //   walk         u32[E][walk_cap], walk_len u32[E]
+//   walk runs    (word, mask) u32x2[E][walk_cap], wrun_len u32[E]: the walk
+//                as bitmap words, consecutive blocks of one 32-block word merged
 //   residency    frame_of u32[W], stamp_of u32[W], block_of u32[C],
 //                free bitmap u32[C/32], inactive bitmap u32[W/32],
 //                LRM log (blk u32, stamp u32)[log_cap] ordered by stamp
@@ -133,6 +135,7 @@ struct dum_engine {
   cudaEvent_t ev_fork, ev_join;
   // block tables / walk cache
   uint32_t *d_tbl, *d_start_end, *d_walk, *d_walk_len;
+  uint32_t *d_wrun, *d_wrun_len;   // walk as (word, mask) runs (k_apply_walk / k_walk_slow)
   // staging
   uint32_t stage_launch_cap;
   uint64_t stage_fault_cap;
@@ -158,7 +161,7 @@ struct dum_engine {
   uint64_t anchor_pool_entries;
   uint64_t *d_anchor_range;   // per query (begin, len)
   uint32_t anchor_range_cap;  // max queries per predict call
-  uint32_t *d_qkern, *d_qloff, *d_qnk;  // per-query chain scratch (k_chain -> k_predict)
+  uint32_t *d_qkern, *d_qloff, *d_qeoff, *d_qgoff, *d_qnk;  // per-query chain scratch (k_chain -> k_predict)
   unsigned long long *d_qbase;
   // residency
   uint32_t *d_frame_of, *d_stamp_of, *d_block_of, *d_free_bits, *d_inactive_bits, *d_res_bits;

@@ -219,6 +219,7 @@ struct BuildArgs {
   uint32_t *big_pool;
   uint64_t big_entries;
   uint32_t *slow_list;
+  uint32_t *wrun, *wrun_len;   // walk bitmap runs (read by k_predict)
   const uint32_t *order;       // [3][n_staged] faulting launches by size class
   DevState *st;
   unsigned long long *cta_clk;  // debug: per-CTA (start, end, n_ops | n << 32) or null
@@ -267,7 +268,7 @@ __global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
   constexpr int OWN_B = (MAXA * (1 + MAXS) <= 10) ? 2 : 1;  // sets loaded per owner batch
   extern __shared__ uint32_t sm[];
   __shared__ uint32_t ws[BUILD_NT / 32];
-  __shared__ uint32_t s_ng, s_tev, s_flag, s_sets, s_nnz;
+  __shared__ uint32_t s_ng, s_tev, s_flag, s_sets, s_nnz, s_nrun;
   __shared__ unsigned long long goff[GCAP];  // stage offset of each group launch
   const Geo &g = a.g;
   const uint32_t tid = threadIdx.x;
@@ -463,6 +464,8 @@ __global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
     if (tid == 0) {
       wout[0] = start;
       a.walk_len[e] = 1;
+      reinterpret_cast<uint2 *>(a.wrun)[(uint64_t)e * g.walk_cap] = make_uint2(start >> 5, 1u << (start & 31));
+      a.wrun_len[e] = 1;
       ctr_add(a.st, DUM_CTR_WALK_OUT, 1);
     }
     return;
@@ -597,7 +600,12 @@ __global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
   __syncthreads();
   if (a.cta_clk && tid == 0) a.cta_clk[10 * j + 8] = gtimer();
   // ---- pass C: ordered compaction of first occurrences ----
+  // The kept blocks of each warp step are also grouped by bitmap word into
+  // runs (word, mask) for k_predict (any grouping that puts every block in
+  // exactly one run will do; runs of one walk are disjoint).
   uint32_t outn = 0;
+  uint2 *wrun = reinterpret_cast<uint2 *>(a.wrun) + (uint64_t)e * g.walk_cap;
+  if (tid == 0) s_nrun = 0;
   for (uint32_t c = 0; c < qlen; c += BUILD_NT) {
     const uint32_t p = c + tid;
     uint32_t val = NONE, keep = 0;
@@ -620,11 +628,25 @@ __global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
     uint32_t tot;
     const uint32_t pre = block_excl_scan(keep, ws, &tot);
     if (keep && outn + pre < g.walk_cap) wout[outn + pre] = val;
+    {
+      const uint32_t lane = tid & 31;
+      const uint32_t wkey = keep ? val >> 5 : NONE;
+      const uint32_t grp = __match_any_sync(0xffffffffu, wkey);
+      const uint32_t msk = __reduce_or_sync(grp, keep ? 1u << (val & 31) : 0u);
+      const bool lead = keep && lane == (uint32_t)(__ffs(grp) - 1);
+      const uint32_t lm = __ballot_sync(0xffffffffu, lead);
+      uint32_t rb = 0;
+      if (lane == 0 && lm) rb = atomicAdd(&s_nrun, (uint32_t)__popc(lm));
+      rb = __shfl_sync(0xffffffffu, rb, 0) + __popc(lm & ((1u << lane) - 1));
+      if (lead && rb < g.walk_cap) wrun[rb] = make_uint2(wkey, msk);
+    }
     outn += tot;
   }
+  __syncthreads();  // every warp's run count is in s_nrun
   if (tid == 0) {
     if (outn > g.walk_cap) set_err(a.st, ERR_ECAPACITY, outn);
     a.walk_len[e] = outn;
+    a.wrun_len[e] = s_nrun;
     ctr_add(a.st, DUM_CTR_WALK_ROWS, t + 1);
     ctr_add(a.st, DUM_CTR_WALK_OUT, outn);
     if (a.cta_clk) {
@@ -636,7 +658,8 @@ __global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
 }
 
 __global__ void k_walk_slow(Geo g, const uint32_t *tbl, const uint32_t *start_end, uint32_t *walk,
-                            uint32_t *walk_len, const uint32_t *slow_list, WalkScratch ws, DevState *st) {
+                            uint32_t *walk_len, uint32_t *wrun, uint32_t *wrun_len, const uint32_t *slow_list,
+                            WalkScratch ws, DevState *st) {
   const uint32_t nslow = *(volatile uint32_t *)&st->n_slow;
   for (uint32_t q = blockIdx.x; q < nslow; q += gridDim.x) {
     const uint32_t e = slow_list[q];
@@ -650,6 +673,26 @@ __global__ void k_walk_slow(Geo g, const uint32_t *tbl, const uint32_t *start_en
       }
       walk_len[e] = n;
     }
+    __syncwarp();
+    // bitmap runs of the new walk (see pass C of k_apply_walk)
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t *w = walk + (uint64_t)e * g.walk_cap;
+    uint2 *out = reinterpret_cast<uint2 *>(wrun) + (uint64_t)e * g.walk_cap;
+    const uint32_t len = *(volatile uint32_t *)&walk_len[e];
+    uint32_t nr = 0;
+    for (uint32_t c = 0; c < len; c += 32) {
+      const bool v = c + lane < len;
+      const uint32_t b = v ? w[c + lane] : NONE;
+      const uint32_t word = v ? b >> 5 : NONE;
+      const uint32_t grp = __match_any_sync(0xffffffffu, word);
+      const uint32_t mask = __reduce_or_sync(grp, v ? 1u << (b & 31) : 0u);
+      const bool lead = v && lane == (uint32_t)(__ffs(grp) - 1);
+      const uint32_t lm = __ballot_sync(0xffffffffu, lead);
+      if (lead) out[nr + __popc(lm & ((1u << lane) - 1))] = make_uint2(word, mask);
+      nr += __popc(lm);
+    }
+    if (lane == 0) wrun_len[e] = nr;
+    __syncwarp();
   }
 }
 
@@ -698,6 +741,8 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   ba.big_pool = e->d_big_pool;
   ba.big_entries = e->big_pool_entries;
   ba.slow_list = e->d_slow_list;
+  ba.wrun = e->d_wrun;
+  ba.wrun_len = e->d_wrun_len;
   ba.order = e->d_order;
   ba.st = e->d_state;
   ba.cta_clk = nullptr;
@@ -721,9 +766,11 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   if (err != cudaSuccess) return err;
   WalkScratch ws{e->d_walk_seen, e->d_walk_chain, e->d_walk_tmp, e->walk_hash_cap,
                  e->g.walk_cap + e->g.R * e->g.A + 4};
-  TimerScope t(e, DUM_T_WALK_SLOW, s);
-  k_walk_slow<<<e->n_walk_slots, 32, 0, s>>>(e->g, e->d_tbl, e->d_start_end, e->d_walk, e->d_walk_len,
-                                             e->d_slow_list, ws, e->d_state);
+  {
+    TimerScope t(e, DUM_T_WALK_SLOW, s);
+    k_walk_slow<<<e->n_walk_slots, 32, 0, s>>>(e->g, e->d_tbl, e->d_start_end, e->d_walk, e->d_walk_len,
+                                               e->d_wrun, e->d_wrun_len, e->d_slow_list, ws, e->d_state);
+  }
   if (clk_path) {
     std::vector<unsigned long long> h(10ull * n);
     cudaStreamSynchronize(s);

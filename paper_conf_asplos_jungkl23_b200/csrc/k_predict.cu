@@ -22,6 +22,10 @@
 //                  re-compaction overwrite the output.
 //                  SELECT: the fused pre-eviction selection of a8 reuses the
 //                  window bitmap (select_tail.cuh).
+#include <cstdio>
+#include <cstdlib>
+#include <vector>
+
 #include "corr.cuh"
 #include "device_util.cuh"
 #include "kernels.cuh"
@@ -33,7 +37,9 @@ namespace dum {
 constexpr int PRED_NT = 512;
 constexpr int NWARP = PRED_NT / 32;
 constexpr uint32_t MAXN = 128;   // degree_n limit
-constexpr uint32_t DCAP = 2048;  // shared hash of duplicated blocks (block -> min window position)
+constexpr uint32_t DLCAP = 512;   // duplicated blocks recorded by pass 1 (more: hash every element)
+constexpr uint32_t DHCAP = 2048;  // shared hash of the duplicated blocks (block -> min position + 1)
+static_assert(2 * DHCAP >= SEL_CHUNK, "the dup hash region doubles as the selection stage");
 
 __global__ void k_make_queries(const uint32_t *__restrict__ seq, uint32_t n_seq, uint32_t first, uint32_t degree,
                                dum_query *__restrict__ out) {
@@ -102,6 +108,7 @@ struct PredArgs {
   uint32_t corr_cap;
   const uint32_t *jump;  // [levels][corr_cap]
   const uint32_t *walk, *walk_len;
+  const uint32_t *wrun, *wrun_len;  // walk bitmap runs (k_apply_walk pass C / k_walk_slow)
   const uint32_t *anchor_pool;
   const uint64_t *anchor_range;
   uint32_t *pairs;
@@ -113,14 +120,24 @@ struct PredArgs {
   // per-query scratch written by k_chain
   uint32_t *qkern;  // [nq][N+1]
   uint32_t *qloff;  // [nq][N+2]
+  uint32_t *qeoff;  // [nq][N+2] run-entry offsets of the window's lists
+  uint32_t *qgoff;  // [nq][N+2] 128-block copy-chunk offsets of the window's lists
   uint32_t *qnk;    // [nq]
   unsigned long long *qbase;  // [nq]
   uint32_t *big_pool;         // scratch for the exact slow path
   uint64_t big_entries;
   SelectOut so;     // fused a8 outputs (SELECT only)
+  unsigned long long *cta_clk;  // debug (DUM_CTA_CLOCK): per CTA 8 x u64 timestamps, or null
 };
 
+__device__ __forceinline__ unsigned long long pred_timer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
 constexpr int CHAIN_WARPS = 8;
+constexpr uint32_t CHUNK_B = 128;  // window blocks per copy chunk (one warp: 4 coalesced steps)
 
 __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
   __shared__ uint32_t skern[CHAIN_WARPS][MAXN + 1];
@@ -163,6 +180,10 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
     // same (unanchored) walk adds nothing (exact; keeps the reservation tight)
     uint32_t *gkern = a.qkern + (uint64_t)qi * (g.N + 1);
     uint32_t *loff = a.qloff + (uint64_t)qi * (g.N + 2);
+    uint32_t *eoff = a.qeoff + (uint64_t)qi * (g.N + 2);
+    uint32_t *goff = a.qgoff + (uint64_t)qi * (g.N + 2);
+    uint32_t RU = 0;  // bitmap-run entries of the window (k_predict pass 1)
+    uint32_t GU = 0;  // 128-block copy chunks of the window (k_predict copy)
     for (uint32_t d0 = 0; d0 < nk; d0 += 32) {
       const uint32_t d = d0 + lane;
       const bool v = d < nk, anc0 = d == 0 && anchored;
@@ -177,20 +198,35 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
             len = 0;
             break;
           }
-      uint32_t incl = len;
+      // an anchored query's own walk has no runs: its blocks enter one by one
+      const uint32_t rl = len ? (anc0 ? len : __ldg(a.wrun_len + e)) : 0u;
+      const uint32_t gl = (len + CHUNK_B - 1) / CHUNK_B;
+      uint32_t incl = len, rincl = rl, gincl = gl;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
         const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
-        if (lane >= (uint32_t)o) incl += y;
+        const uint32_t z = __shfl_up_sync(0xffffffffu, rincl, o);
+        const uint32_t u = __shfl_up_sync(0xffffffffu, gincl, o);
+        if (lane >= (uint32_t)o) {
+          incl += y;
+          rincl += z;
+          gincl += u;
+        }
       }
       if (v) {
         gkern[d] = e;
         loff[d + 1] = U + incl;
+        eoff[d + 1] = RU + rincl;
+        goff[d + 1] = GU + gincl;
       }
       U += __shfl_sync(0xffffffffu, incl, 31);
+      RU += __shfl_sync(0xffffffffu, rincl, 31);
+      GU += __shfl_sync(0xffffffffu, gincl, 31);
     }
     if (lane == 0) {
       loff[0] = 0;
+      eoff[0] = 0;
+      goff[0] = 0;
       a.qnk[qi] = nk;
     }
   }
@@ -211,12 +247,30 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
   }
 }
 
+// Warp-specialised: warps [0, GRP_W) build the window set from the runs
+// (pass 1) and then run the selection (a8) on it; warps [GRP_W, NWARP) stream
+// the (block, exec) pairs meanwhile.  Duplicates (rare) are only known after
+// pass 1: the duplicate path then rewrites the pairs and redoes the selection
+// with the whole CTA.
+constexpr int GRP_W = NWARP / 2;
+constexpr int GRP_NT = GRP_W * 32;
+constexpr uint32_t OCCAP = 1024;   // duplicate occurrences (list, block) tracked by the duplicate path
+constexpr uint32_t DWCAP = 1024;   // duplicate-word hash slots (word -> mask of duplicated blocks)
+constexpr uint32_t DBCAP = 1024;   // duplicate-block hash slots (block -> first list + 1)
+static_assert(2 * DWCAP + 2 * DBCAP <= 2 * DHCAP, "duplicate hashes live in the dup/stage region");
+static_assert(OCCAP >= DLCAP, "s_dup doubles as the occurrence list");
+
 template <bool SELECT>
 __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
-  extern __shared__ uint32_t bitmap[];  // [nwords] window set | dk[DCAP] | dv[DCAP]
-  __shared__ uint32_t kern[MAXN + 1], loff[MAXN + 2], kcnt[MAXN + 1];
-  __shared__ uint32_t ws[NWARP], wtot[NWARP];
-  __shared__ uint32_t s_ndup, s_nonres, s_flag, s_ovf;
+  extern __shared__ uint4 sm4[];  // [nwords rounded up to 4] window set bitmap | dup hashes / select stage
+  uint32_t *bitmap = reinterpret_cast<uint32_t *>(sm4);
+  uint32_t *dk = bitmap + ((a.nwords + 3) & ~3u);  // [2 * DHCAP]
+  __shared__ SelShared ss;
+  __shared__ uint32_t kern[MAXN + 1], loff[MAXN + 2], kcnt[MAXN + 1], eoff[MAXN + 2], goff[MAXN + 2];
+  __shared__ uint32_t noff[MAXN + 2];
+  __shared__ uint32_t ws[NWARP];
+  __shared__ uint32_t s_ndup, s_nonres, s_flag, s_nocc, s_dnr;
+  __shared__ uint32_t s_dup[2 * OCCAP];  // pass 1: duplicated blocks; duplicate path: occurrences (list, block)
   __shared__ unsigned long long s_hoff;
   const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const uint32_t qi = blockIdx.x;
@@ -225,192 +279,347 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
   const bool anchored = anchor != NONE;
   const uint32_t nk = a.qnk[qi];
   const unsigned long long base = a.qbase[qi];
-  uint32_t *dk = bitmap + ((a.nwords + 3) & ~3u), *dv = dk + DCAP;
-  {
-    uint4 *b4 = reinterpret_cast<uint4 *>(bitmap);
-    for (uint32_t w = tid; w < a.nwords / 4; w += PRED_NT) b4[w] = make_uint4(0, 0, 0, 0);
-    for (uint32_t w = (a.nwords & ~3u) + tid; w < a.nwords; w += PRED_NT) bitmap[w] = 0;
-    uint4 *d4 = reinterpret_cast<uint4 *>(dk);
-    for (uint32_t w = tid; w < 2 * DCAP / 4; w += PRED_NT) d4[w] = make_uint4(NONE, NONE, NONE, NONE);
+  unsigned long long *clk = a.cta_clk ? a.cta_clk + 12ull * qi : nullptr;
+  if (clk && tid == 0) {
+    unsigned int smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    clk[0] = pred_timer();
+    clk[7] = smid;
   }
+  for (uint32_t w = tid; w < (a.nwords + 3) / 4; w += PRED_NT) sm4[w] = make_uint4(0, 0, 0, 0);
   for (uint32_t d = tid; d <= nk; d += PRED_NT) {
     loff[d] = a.qloff[(uint64_t)qi * (g.N + 2) + d];
+    eoff[d] = a.qeoff[(uint64_t)qi * (g.N + 2) + d];
+    goff[d] = a.qgoff[(uint64_t)qi * (g.N + 2) + d];
+    kcnt[d] = 0;
     if (d < nk) kern[d] = a.qkern[(uint64_t)qi * (g.N + 1) + d];
   }
   if (tid == 0) {
     s_ndup = 0;
     s_nonres = 0;
-    s_ovf = 0;
+    s_nocc = 0;
+    s_dnr = 0;
   }
   __syncthreads();
   const uint32_t U = nk ? loff[nk] : 0;
   const bool ok = base + U <= a.cap;
-  if (tid == 0 && anchored && anchor < g.W) {
-    bitmap[anchor >> 5] |= 1u << (anchor & 31);
-    hmap_insert_min(dk, dv, DCAP, anchor, 0);  // position 0: never kept
-  }
-  __syncthreads();
+  if (clk && tid == 0) clk[1] = pred_timer();
   const uint32_t *apool = a.anchor_pool + (anchored ? a.anchor_range[2 * qi] : 0);
   auto list_of = [&](uint32_t d) -> const uint32_t * {
     return (d == 0 && anchored) ? apool : a.walk + (uint64_t)kern[d] * g.walk_cap;
   };
-  // ---------------- fast path: one pass ----------------
-  // warp w owns the contiguous segment [t0, t1), walked kernel by kernel
-  // (no per-element kernel search), 4 loads in flight per lane
-  const uint32_t seg = ((U + NWARP - 1) / NWARP + 127) & ~127u;
-  const uint32_t t0 = min(U, wid * seg), t1 = min(U, t0 + seg);
-  uint32_t nonres = 0, ndup = 0;
-  if (t0 < t1) {
-    uint32_t d = 0;
-    while (d + 1 < nk && loff[d + 1] <= t0) ++d;
-    for (; d < nk && loff[d] < t1; ++d) {
-      const uint32_t k0 = max(t0, loff[d]), k1 = min(t1, loff[d + 1]);
-      if (k0 >= k1) continue;
-      const uint32_t *lst = list_of(d) - loff[d];  // indexed by window position
-      const uint32_t kd = kern[d];
-      for (uint32_t c = k0; c < k1; c += 128) {
-        uint32_t b[4];
+  auto search = [&](const uint32_t *off, uint32_t x) -> uint32_t {  // largest d < nk with off[d] <= x
+    uint32_t lo = 0, hi = nk;
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (off[mid] <= x) lo = mid;
+      else hi = mid;
+    }
+    return lo;
+  };
+  // run entry x of the window: (word, mask) of list `lo`
+  auto run_at = [&](uint32_t x, uint32_t &lo, uint32_t &w, uint32_t &m) {
+    lo = search(eoff, x);
+    const uint32_t i = x - eoff[lo];
+    if (lo == 0 && anchored) {
+      const uint32_t b = apool[i];
+      w = b >> 5;
+      m = 1u << (b & 31);
+    } else {
+      const uint2 r = __ldg(reinterpret_cast<const uint2 *>(a.wrun) + (uint64_t)kern[lo] * g.walk_cap + i);
+      w = r.x;
+      m = r.y;
+    }
+  };
+  // Copy of whole lists: flat over the window's 128-block chunks (chunks
+  // never straddle lists); warp-uniform chunk lookup, lane-consecutive 4 B
+  // loads and 8 B streaming stores (128 B / 256 B per warp instruction), two
+  // chunks in flight.  List d goes to pairs[base + oofs[d] ...]; lists with
+  // skip[d] != 0 are left out.
+  auto copy_lists = [&](uint32_t cw, uint32_t ncw, const uint32_t *oofs, const uint32_t *skip) {
+    constexpr uint32_t UN = 2;
+    const uint32_t G = nk ? goff[nk] : 0;
+    uint2 *out = reinterpret_cast<uint2 *>(a.pairs) + base;
+    for (uint32_t c0 = cw; c0 < G; c0 += ncw * UN) {
+      uint32_t b[UN][4], dd[UN], i0[UN], L[UN];
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
-          const uint32_t t = c + 32 * k + lane;
-          b[k] = t < k1 ? __ldg(lst + t) : NONE;
-        }
+      for (uint32_t u = 0; u < UN; ++u) {
+        const uint32_t c = c0 + u * ncw;
+        dd[u] = NONE;
+        if (c < G) {
+          const uint32_t lo = search(goff, c);
+          if (skip && skip[lo]) continue;
+          dd[u] = lo;
+          i0[u] = (c - goff[lo]) * CHUNK_B;
+          L[u] = loff[lo + 1] - loff[lo];
+          const uint32_t *lst = list_of(lo);
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
-          const uint32_t t = c + 32 * k + lane;
-          const bool valid = t < k1;
-          if (c + 32 * k >= k1) break;  // warp-uniform
-          if (warp_test_and_set(bitmap, b[k], valid)) {
-            ++ndup;
-            if (!hmap_insert_min(dk, dv, DCAP, b[k], t + 1)) s_ovf = 1;
-          }
-          if (valid) {
-            if (ok) reinterpret_cast<uint2 *>(a.pairs)[base + t] = make_uint2(b[k], kd);
-            if (SELECT) nonres += !((__ldg(&a.so.res_bits[b[k] >> 5]) >> (b[k] & 31)) & 1u);
+          for (uint32_t k = 0; k < 4; ++k) {
+            const uint32_t i = i0[u] + 32 * k + lane;
+            b[u][k] = i < L[u] ? __ldg(lst + i) : NONE;
           }
         }
       }
-    }
-  }
-  if (ndup) atomicAdd(&s_ndup, ndup);
-  if (SELECT) {
 #pragma unroll
-    for (int o = 16; o; o >>= 1) nonres += __shfl_xor_sync(0xffffffffu, nonres, o);
-    if (lane == 0 && nonres) atomicAdd(&s_nonres, nonres);
+      for (uint32_t u = 0; u < UN; ++u) {
+        if (dd[u] == NONE) continue;
+        const uint32_t kd = kern[dd[u]];
+        uint2 *o = out + oofs[dd[u]];
+#pragma unroll
+        for (uint32_t k = 0; k < 4; ++k) {
+          const uint32_t i = i0[u] + 32 * k + lane;
+          if (i < L[u]) __stcs(o + i, make_uint2(b[u][k], kd));
+        }
+      }
+    }
+  };
+  auto record_dup = [&](uint32_t w, uint32_t dup) {
+    while (dup) {  // rare
+      const uint32_t bit = __ffs(dup) - 1;
+      dup &= dup - 1;
+      const uint32_t k = atomicAdd(&s_ndup, 1u);
+      if (k < DLCAP) s_dup[k] = w * 32 + bit;
+    }
+  };
+  if (wid < GRP_W) {
+    // ---------------- pass 1: window set, duplicate test, non-resident count ----------------
+    // One shared atomicOr per run.  Within one walk the runs are disjoint, so
+    // a bit found already set means the block occurs in two lists of the
+    // window, or is the anchor (in the window set, never emitted; D14).
+    const uint32_t etot = nk ? eoff[nk] : 0;
+    uint32_t nonres = 0;
+    if (tid == 0 && anchored && anchor < g.W) {
+      const uint32_t m = 1u << (anchor & 31);
+      record_dup(anchor >> 5, atomicOr(&bitmap[anchor >> 5], m) & m);
+    }
+    for (uint32_t x = tid; x < etot; x += GRP_NT) {
+      uint32_t lo, w, m;
+      run_at(x, lo, w, m);
+      record_dup(w, atomicOr(&bitmap[w], m) & m);
+      if (SELECT) nonres += __popc(m & ~__ldg(&a.so.res_bits[w]));
+    }
+    if (SELECT) {
+#pragma unroll
+      for (int o = 16; o; o >>= 1) nonres += __shfl_xor_sync(0xffffffffu, nonres, o);
+      if (lane == 0 && nonres) atomicAdd(&s_nonres, nonres);
+      group_sync<1, GRP_NT>();
+      if (clk && tid == 0) clk[2] = pred_timer();
+      if (s_ndup == 0) {  // uniform over the group
+        if (tid == 0) select_reserve(a.so, s_nonres, a.st, ss);
+        group_sync<1, GRP_NT>();
+        if (clk && tid == 0) clk[3] = pred_timer();
+        select_tail<GRP_NT, 1>(a.so, qi, ss, bitmap, a.st, tid, dk);
+      }
+    }
+    if (clk && tid == 0) clk[4] = pred_timer();
+  } else if (ok) {
+    // ---------------- streaming copy (valid unless pass 1 finds a duplicate) ----------------
+    copy_lists(wid - GRP_W, NWARP - GRP_W, loff, nullptr);
   }
+  if (clk && tid == GRP_NT) clk[5] = pred_timer();
   __syncthreads();
+  const uint32_t ndup = s_ndup;
   uint32_t run = U;
-  const bool dedup = s_ndup != 0;
-  if (dedup) {
-    // ---------------- exact slow path (some block occurs twice) ----------------
-    // keep(t) = t is the minimum window position of its block, the anchor
-    // pre-seeded at position 0 (D17).  Normally only the duplicated blocks
-    // (found in the fast pass) sit in the shared hash and every occurrence of
-    // them lowers the min position; if that hash overflowed, all elements go
-    // into a global scratch hash instead.
-    const bool ovf = s_ovf != 0;
-    uint32_t hcap = DCAP;
-    uint32_t *hk = dk, *hv = dv;
-    if (tid == 0) {
-      s_nonres = 0;
-      s_flag = 1;
-      if (ovf) {
-        const uint32_t hc = pow2ceil(2 * (U + 1));
-        const unsigned long long o = atomicAdd(&a.st->pool_big, 2ull * hc);
-        s_flag = o + 2ull * hc <= a.big_entries * 2;
-        s_hoff = o;
-        if (!s_flag) set_err(a.st, ERR_ECAPACITY, o + 2ull * hc);
+  if (ndup) {
+    // ---------------- duplicate path (D17: first occurrence wins) ----------------
+    // The window is the concatenation of the lists; a list holds a block at
+    // most once, so an occurrence is kept iff no earlier list holds the block
+    // (and it is not the anchor, "list -1").  Per duplicated block the first
+    // list is found from the runs (a word hash filters the runs that hold
+    // duplicated blocks), every other occurrence is dropped, the lists keep
+    // their order and shift left; the few lists that lose blocks are
+    // compacted by one warp each, the others are copied again.
+    uint32_t *wk = dk, *wm = dk + DWCAP;                      // word -> duplicated-block mask
+    uint32_t *bk = dk + 2 * DWCAP, *bv = bk + DBCAP;          // block -> first list + 1 (anchor: 0)
+    bool fallback = ndup > DLCAP;
+    if (!fallback) {
+      for (uint32_t p = tid; p < 2 * DHCAP; p += PRED_NT) dk[p] = NONE;
+      __syncthreads();
+      for (uint32_t p = tid; p < ndup; p += PRED_NT) {
+        const uint32_t b = s_dup[p];
+        hmap_insert_min(bk, bv, DBCAP, b, NONE);
+        // word -> mask: claim the word's slot, then OR the bit in
+        for (uint32_t sl = hslot(b >> 5, DWCAP);; sl = (sl + 1) & (DWCAP - 1)) {
+          const uint32_t old = atomicCAS(&wk[sl], NONE, b >> 5);
+          if (old == NONE || old == (b >> 5)) break;
+        }
       }
+      __syncthreads();
+      // claimed words: clear the mask, then set the duplicated bits
+      for (uint32_t p = tid; p < DWCAP; p += PRED_NT)
+        if (wk[p] != NONE) wm[p] = 0;
+      __syncthreads();
+      for (uint32_t p = tid; p < ndup; p += PRED_NT) {
+        const uint32_t b = s_dup[p];
+        for (uint32_t sl = hslot(b >> 5, DWCAP);; sl = (sl + 1) & (DWCAP - 1))
+          if (wk[sl] == (b >> 5)) {
+            atomicOr(&wm[sl], 1u << (b & 31));
+            break;
+          }
+      }
+      if (tid == 0 && anchored) hmap_insert_min(bk, bv, DBCAP, anchor, 0);
+      __syncthreads();
+      // occurrences: runs holding duplicated blocks -> (list, block); first list per block
+      const uint32_t etot = nk ? eoff[nk] : 0;
+      for (uint32_t x = tid; x < etot; x += PRED_NT) {
+        uint32_t lo, w, m;
+        run_at(x, lo, w, m);
+        uint32_t hit = 0;
+        for (uint32_t sl = hslot(w, DWCAP);; sl = (sl + 1) & (DWCAP - 1)) {
+          const uint32_t kk = wk[sl];
+          if (kk == NONE) break;
+          if (kk == w) {
+            hit = m & wm[sl];
+            break;
+          }
+        }
+        while (hit) {
+          const uint32_t bit = __ffs(hit) - 1;
+          hit &= hit - 1;
+          const uint32_t b = w * 32 + bit;
+          hmap_insert_min(bk, bv, DBCAP, b, lo + 1);
+          const uint32_t k = atomicAdd(&s_nocc, 1u);
+          if (k < OCCAP) {
+            s_dup[2 * k] = lo;
+            s_dup[2 * k + 1] = b;
+          }
+        }
+      }
+      __syncthreads();
+      fallback = s_nocc > OCCAP;
     }
-    for (uint32_t d = tid; d <= nk; d += PRED_NT) kcnt[d] = 0;
-    __syncthreads();
-    if (ovf) {
-      hcap = pow2ceil(2 * (U + 1));
-      hk = a.big_pool + s_hoff;
-      hv = hk + hcap;
-    }
-    if (s_flag) {
-      if (ovf) {
+    if (!fallback) {
+      // dropped occurrences: per-list counts (kcnt) and the non-resident ones
+      const uint32_t nocc = s_nocc;
+      for (uint32_t k = tid; k < nocc; k += PRED_NT) {
+        const uint32_t d = s_dup[2 * k], b = s_dup[2 * k + 1];
+        if (hmap_get(bk, bv, DBCAP, b) != d + 1) {
+          atomicAdd(&kcnt[d], 1u);
+          if (SELECT && !((__ldg(&a.so.res_bits[b >> 5]) >> (b & 31)) & 1u)) atomicAdd(&s_dnr, 1u);
+        }
+      }
+      __syncthreads();
+      // output offsets of the shifted lists (warp 0)
+      if (wid == 0) {
+        uint32_t acc = 0;
+        for (uint32_t d0 = 0; d0 < nk; d0 += 32) {
+          const uint32_t d = d0 + lane;
+          const uint32_t len = d < nk ? loff[d + 1] - loff[d] - kcnt[d] : 0;
+          uint32_t incl = len;
+#pragma unroll
+          for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= (uint32_t)o) incl += y;
+          }
+          if (d < nk) noff[d] = acc + incl - len;
+          acc += __shfl_sync(0xffffffffu, incl, 31);
+        }
+        if (lane == 0) noff[nk] = acc;
+      }
+      __syncthreads();
+      run = noff[nk];
+      if (ok) {
+        // lists that lose blocks: one warp each, ordered ballot compaction
+        for (uint32_t d = wid; d < nk; d += NWARP) {
+          if (!kcnt[d]) continue;
+          const uint32_t *lst = list_of(d);
+          const uint32_t L = loff[d + 1] - loff[d], kd = kern[d];
+          uint2 *o = reinterpret_cast<uint2 *>(a.pairs) + base + noff[d];
+          uint32_t pos = 0;
+          for (uint32_t c = 0; c < L; c += 32) {
+            const uint32_t i = c + lane;
+            uint32_t b = NONE;
+            bool keep = false;
+            if (i < L) {
+              b = __ldg(lst + i);
+              const uint32_t f = hmap_get(bk, bv, DBCAP, b);
+              keep = f == NONE || f == d + 1;
+            }
+            const uint32_t mask = __ballot_sync(0xffffffffu, keep);
+            if (keep) __stcs(o + pos + __popc(mask & ((1u << lane) - 1)), make_uint2(b, kd));
+            pos += __popc(mask);
+          }
+        }
+        // the other lists at their shifted offsets
+        copy_lists(wid, NWARP, noff, kcnt);
+      }
+      if (SELECT && tid == 0) s_nonres -= s_dnr;
+      if (clk && tid == 0) clk[8] = pred_timer();
+    } else {
+      // ---------------- fallback: min-position hash over every element ----------------
+      const uint32_t hcap = pow2ceil(2 * (U + 1));
+      if (tid == 0) {
+        s_nonres = 0;
+        const unsigned long long o = atomicAdd(&a.st->pool_big, 2ull * hcap);
+        s_flag = o + 2ull * hcap <= a.big_entries * 2;
+        s_hoff = o;
+        if (!s_flag) set_err(a.st, ERR_ECAPACITY, o + 2ull * hcap);
+      }
+      for (uint32_t d = tid; d <= nk; d += PRED_NT) kcnt[d] = 0;
+      __syncthreads();
+      if (s_flag) {
+        uint32_t *hk = a.big_pool + s_hoff, *hv = hk + hcap;
         for (uint32_t p = tid; p < hcap; p += PRED_NT) {
           hk[p] = NONE;
           hv[p] = NONE;
         }
         __syncthreads();
         if (tid == 0 && anchored) hmap_insert_min(hk, hv, hcap, anchor, 0);
-      }
-      for (uint32_t d = 0; d < nk; ++d) {
-        const uint32_t *lst = list_of(d);
-        for (uint32_t i = tid; i < loff[d + 1] - loff[d]; i += PRED_NT) {
-          const uint32_t bb = __ldg(lst + i), pos = loff[d] + i + 1;
-          if (ovf) {
-            hmap_insert_min(hk, hv, hcap, bb, pos);
-          } else {
-            // lower the min position of duplicated blocks only
-            for (uint32_t pp = 0, sl = hslot(bb, hcap); pp < hcap; ++pp, sl = (sl + 1) & (hcap - 1)) {
-              const uint32_t kk = hk[sl];
-              if (kk == NONE) break;
-              if (kk == bb) {
-                atomicMin(&hv[sl], pos);
-                break;
-              }
-            }
-          }
+        for (uint32_t t = tid; t < U; t += PRED_NT) {
+          const uint32_t d = search(loff, t);
+          hmap_insert_min(hk, hv, hcap, __ldg(list_of(d) + (t - loff[d])), t + 1);
         }
-      }
-      __syncthreads();
-      // per-warp keep counts over the warp segments, then ordered writes
-      for (int pass = 0; pass < 2; ++pass) {
-        uint32_t pos = pass ? wtot[wid] : 0, nr = 0;
-        if (t0 < t1) {
-          uint32_t d = 0;
-          while (d + 1 < nk && loff[d + 1] <= t0) ++d;
-          for (; d < nk && loff[d] < t1; ++d) {
-            const uint32_t k0 = max(t0, loff[d]), k1 = min(t1, loff[d + 1]);
-            if (k0 >= k1) continue;
-            const uint32_t *lst = list_of(d) - loff[d];
-            for (uint32_t c = k0; c < k1; c += 32) {
-              const uint32_t t = c + lane;
-              uint32_t bb = NONE;
-              bool keep = false;
-              if (t < k1) {
-                bb = __ldg(lst + t);
-                const uint32_t mp = hmap_get(hk, hv, hcap, bb);
-                keep = ovf ? mp == t + 1 : (mp == NONE || mp == t + 1);
-              }
-              const uint32_t mask = __ballot_sync(0xffffffffu, keep);
-              if (pass && keep) {
-                if (ok) reinterpret_cast<uint2 *>(a.pairs)[base + pos + __popc(mask & ((1u << lane) - 1))] =
-                    make_uint2(bb, kern[d]);
-                if (SELECT) nr += !((__ldg(&a.so.res_bits[bb >> 5]) >> (bb & 31)) & 1u);
-              }
-              if (pass && lane == 0) atomicAdd(&kcnt[d], __popc(mask));
-              pos += __popc(mask);
+        __syncthreads();
+        // ordered compaction: chunks of 4 * PRED_NT positions, thread tid owns
+        // 4 consecutive ones; one block scan of the keep counts per chunk
+        uint32_t outn = 0, nr = 0;
+        for (uint32_t c = 0; c < U; c += 4 * PRED_NT) {
+          const uint32_t t0 = c + 4 * tid;
+          uint32_t bb[4], dd[4], keep = 0;
+#pragma unroll
+          for (uint32_t u = 0; u < 4; ++u) {
+            const uint32_t t = t0 + u;
+            dd[u] = NONE;
+            bb[u] = NONE;
+            if (t < U) {
+              dd[u] = search(loff, t);
+              bb[u] = __ldg(list_of(dd[u]) + (t - loff[dd[u]]));
+              if (hmap_get(hk, hv, hcap, bb[u]) == t + 1) keep |= 1u << u;
             }
           }
+          uint32_t tot;
+          const uint32_t pre = block_excl_scan(__popc(keep), ws, &tot);
+          uint32_t r = 0;
+#pragma unroll
+          for (uint32_t u = 0; u < 4; ++u) {
+            if (!((keep >> u) & 1u)) continue;
+            if (ok) reinterpret_cast<uint2 *>(a.pairs)[base + outn + pre + r] = make_uint2(bb[u], kern[dd[u]]);
+            if (SELECT) nr += !((__ldg(&a.so.res_bits[bb[u] >> 5]) >> (bb[u] & 31)) & 1u);
+            atomicAdd(&kcnt[dd[u]], 1u);  // kept per list
+            ++r;
+          }
+          outn += tot;
         }
-        if (!pass) {
-          if (lane == 0) wtot[wid] = pos;
-          __syncthreads();
-          if (tid == 0) {
-            uint32_t acc = 0;
-            for (int w = 0; w < NWARP; ++w) {
-              const uint32_t v = wtot[w];
-              wtot[w] = acc;
-              acc += v;
-            }
-            ws[0] = acc;
-          }
-          __syncthreads();
-        } else if (SELECT) {
+        if (SELECT) {
 #pragma unroll
           for (int o = 16; o; o >>= 1) nr += __shfl_xor_sync(0xffffffffu, nr, o);
           if (lane == 0 && nr) atomicAdd(&s_nonres, nr);
         }
+        __syncthreads();
+        // kept per list -> dropped per list (kern_off below uses the same form)
+        for (uint32_t d = tid; d < nk; d += PRED_NT) kcnt[d] = loff[d + 1] - loff[d] - kcnt[d];
+        run = outn;
+      } else {
+        run = 0;
       }
+      if (clk && tid == 0) clk[9] = pred_timer();
+    }
+    __syncthreads();
+    if (SELECT) {
+      if (tid == 0) select_reserve(a.so, s_nonres, a.st, ss);
       __syncthreads();
-      run = ws[0];
-    } else {
-      run = 0;
+      select_tail<PRED_NT, 0>(a.so, qi, ss, bitmap, a.st, tid, dk);
+      if (clk && tid == 0) clk[11] = pred_timer();
     }
   }
   if (tid == 0) {
@@ -420,16 +629,18 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
     ctr_add(a.st, DUM_CTR_CHAIN, nk);
     ctr_add(a.st, DUM_CTR_GATHERED, U);
     ctr_add(a.st, DUM_CTR_EMITTED, run);
+    ctr_add(a.st, DUM_CTR_RUNS, nk ? eoff[nk] : 0);
   }
   if (a.kern_off) {
+    // kern_off[d] = pairs emitted before kernel d (kcnt = occurrences dropped per list)
     uint32_t *ko = a.kern_off + (uint64_t)qi * (g.N + 2);
     for (uint32_t d = tid; d <= g.N + 1; d += PRED_NT) {
       uint32_t v;
-      if (!dedup) {
+      if (ndup == 0) {
         v = d <= nk ? loff[d] : U;
       } else {
         v = 0;
-        for (uint32_t x = 0; x < d && x < nk; ++x) v += kcnt[x];
+        for (uint32_t x = 0; x < d && x < nk; ++x) v += loff[x + 1] - loff[x] - kcnt[x];
       }
       ko[d] = v;
     }
@@ -438,7 +649,7 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
     uint32_t *ch = a.chain + (uint64_t)qi * (g.N + 1);
     for (uint32_t d = tid; d <= g.N; d += PRED_NT) ch[d] = d < nk ? kern[d] : NONE;
   }
-  if (SELECT) select_tail<PRED_NT>(a.so, qi, s_nonres, bitmap, g.W, a.st, ws);
+  if (clk && tid == 0) clk[6] = pred_timer() | ((unsigned long long)(ndup != 0) << 63);
 }
 
 __global__ void k_copy_counter(const unsigned long long *src, uint64_t *dst) { *dst = *src; }
@@ -480,6 +691,8 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   a.jump = e->d_jump;
   a.walk = e->d_walk;
   a.walk_len = e->d_walk_len;
+  a.wrun = e->d_wrun;
+  a.wrun_len = e->d_wrun_len;
   a.anchor_pool = e->d_anchor_pool;
   a.anchor_range = e->d_anchor_range;
   a.pairs = pairs;
@@ -491,6 +704,8 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   a.nwords = (e->g.W + 31) / 32;
   a.qkern = e->d_qkern;
   a.qloff = e->d_qloff;
+  a.qeoff = e->d_qeoff;
+  a.qgoff = e->d_qgoff;
   a.qnk = e->d_qnk;
   a.qbase = e->d_qbase;
   a.big_pool = e->d_big_pool;
@@ -500,11 +715,20 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   } else {
     a.so.res_bits = e->d_res_bits;
   }
+  a.cta_clk = nullptr;
+  static const char *clk_path = getenv("DUM_PRED_CLOCK");
+  static unsigned long long *d_clk = nullptr;
+  static int clk_calls = 0;
+  if (clk_path) {
+    if (!d_clk) cudaMalloc(&d_clk, 12ull * 8 * e->anchor_range_cap);
+    cudaMemsetAsync(d_clk, 0, 12ull * 8 * nq, s);
+    a.cta_clk = d_clk;
+  }
   {
     TimerScope t(e, DUM_T_CHAIN, s);
     k_chain<<<(nq + CHAIN_WARPS - 1) / CHAIN_WARPS, CHAIN_WARPS * 32, 0, s>>>(a);
   }
-  const size_t smem = (size_t)((a.nwords + 3) & ~3u) * 4 + 2 * DCAP * 4;
+  const size_t smem = (size_t)((a.nwords + 3) & ~3u) * 4 + 2 * DHCAP * 4;
   if (sel) {
     cudaFuncSetAttribute(k_predict<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     TimerScope t(e, DUM_T_PREDICT, s);
@@ -515,6 +739,17 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
     k_predict<false><<<nq, PRED_NT, smem, s>>>(a);
   }
   e->kernel_launches += 3;
+  if (clk_path) {
+    std::vector<unsigned long long> h(12ull * nq);
+    cudaStreamSynchronize(s);
+    cudaMemcpy(h.data(), d_clk, 12ull * 8 * nq, cudaMemcpyDeviceToHost);
+    char fn[512];
+    snprintf(fn, sizeof fn, "%s.%d", clk_path, clk_calls++);
+    if (FILE *f = fopen(fn, "wb")) {
+      fwrite(h.data(), 8, h.size(), f);
+      fclose(f);
+    }
+  }
   if (needed) {
     k_copy_counter<<<1, 1, 0, s>>>(&e->d_state->pool_pairs, needed);
     e->kernel_launches += 1;

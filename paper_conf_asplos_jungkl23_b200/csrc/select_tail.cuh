@@ -15,165 +15,169 @@ struct SelectOut {
   uint64_t *out_range;  // 4 per query
 };
 
-// All threads of the CTA must call it.  need = max(0, nonres - free); victims
-// = the first `need` entries of the LRM log (oldest migration first) that are
-// still resident with that stamp and not in the window bitmap; split into
-// write-back / invalidate by the inactive bitmap, both in LRM order.
-// Chunks of NT * 4 log entries; warp w owns 128 consecutive entries of a
-// chunk (4 coalesced steps of 32), counts its eligible active / inactive
-// entries with ballots, and the 32 warp totals are scanned by one warp -- one
-// barrier pair per chunk.
-template <int NT>
-__device__ void select_tail(const SelectOut &so, uint32_t qi, uint32_t nonres, const uint32_t *bitmap, uint32_t W,
-                            DevState *st, uint32_t *ws) {
-  constexpr int NW = NT / 32;
-  constexpr int ITEMS = 4;
-  constexpr uint32_t CHUNK = NT * ITEMS;
-  __shared__ uint32_t s_ok, s_wcnt[NW], s_icnt[NW], s_tw, s_ti, s_aw, s_ai, s_split, s_rem;
-  __shared__ unsigned long long s_bwb, s_binv;
-  const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+// Per-CTA selection state, filled by select_reserve (one thread) before the
+// barrier that precedes select_tail.
+struct SelShared {
+  unsigned long long bwb, binv;  // reserved output offsets (write-back, invalidate)
+  uint32_t need, ok, head, tail, clean;
+};
+
+// One thread: need = max(0, nonres - free frames) (D18); reserve `need`
+// entries in both output lists.  Issued as early as possible so that the
+// contended bump-pointer atomics overlap other work of the CTA.
+__device__ __forceinline__ void select_reserve(const SelectOut &so, uint32_t nonres, DevState *st, SelShared &ss) {
   const uint32_t nfree = *(volatile uint32_t *)&st->free_count;
   const uint32_t need = nonres > nfree ? nonres - nfree : 0;
-  const bool clean = *(volatile uint32_t *)&st->log_dirty == 0;
-  if (tid == 0) {
-    s_ok = 1;
-    s_bwb = s_binv = 0;
-    if (need) {
-      s_bwb = atomicAdd(&st->pool_wb, (unsigned long long)need);
-      s_binv = atomicAdd(&st->pool_inv, (unsigned long long)need);
-      if (s_bwb + need > so.cap || s_binv + need > so.cap) {
-        s_ok = 0;
-        set_err(st, ERR_ECAPACITY, (s_bwb > s_binv ? s_bwb : s_binv) + need);
-      }
+  ss.need = need;
+  ss.ok = 1;
+  ss.bwb = ss.binv = 0;
+  ss.head = *(volatile uint32_t *)&st->lrm_head;
+  ss.tail = *(volatile uint32_t *)&st->lrm_tail;
+  ss.clean = *(volatile uint32_t *)&st->log_dirty == 0;
+  if (need) {
+    ss.bwb = atomicAdd(&st->pool_wb, (unsigned long long)need);
+    ss.binv = atomicAdd(&st->pool_inv, (unsigned long long)need);
+    if (ss.bwb + need > so.cap || ss.binv + need > so.cap) {
+      ss.ok = 0;
+      set_err(st, ERR_ECAPACITY, (ss.bwb > ss.binv ? ss.bwb : ss.binv) + need);
     }
   }
-  __syncthreads();
-  const unsigned long long bwb = s_bwb, binv = s_binv;
-  const bool ok = s_ok;
+}
+
+// Barrier over the NT threads [0, NT) of the CTA: id 0 with NT = blockDim is
+// __syncthreads; other ids are named barriers of a warp group.
+template <int ID, int NT>
+__device__ __forceinline__ void group_sync() {
+  if (ID == 0) __syncthreads();
+  else asm volatile("bar.sync %0, %1;" ::"n"(ID), "n"(NT) : "memory");
+}
+
+// Called by the NT threads tid = [0, NT) of a warp group synchronised by
+// barrier BAR, after select_reserve and a barrier.  Victims = the first `need`
+// entries of the LRM log (oldest migration first) that are still resident
+// with that stamp and not in the window bitmap; split into write-back /
+// invalidate by the inactive bit of the log entry, both in LRM order.
+// The log is scanned in chunks of SEL_CHUNK entries aligned to 4: thread t
+// owns IT consecutive entries (16 B loads) and keeps its eligible active /
+// inactive entries as two bit masks; one group scan of the packed counts
+// (inactive << 16 | active) ranks them; the taken entries are staged in
+// shared memory (write-back from the front, invalidate from the back) and
+// copied out with coalesced stores.  Warp totals are double-buffered: a chunk
+// costs two barriers (three in the last one).
+constexpr uint32_t SEL_CHUNK = 4096;
+
+template <int NT, int BAR>
+__device__ void select_tail(const SelectOut &so, uint32_t qi, const SelShared &ss, const uint32_t *bitmap,
+                            DevState *st, uint32_t tid, uint32_t *stage /* SEL_CHUNK words of shared memory */) {
+  constexpr int NW = NT / 32;
+  constexpr uint32_t IT = SEL_CHUNK / NT;
+  static_assert(NW <= 32 && IT % 4 == 0 && IT <= 16, "one warp scans the warp totals; 16 B loads");
+  __shared__ uint32_t s_wt[2][NW], s_tw, s_ti;
+  const uint32_t lane = tid & 31, wid = tid >> 5;
+  const uint32_t need = ss.need, head = ss.head, tail = ss.tail;
+  const bool clean = ss.clean;
+  const unsigned long long bwb = ss.bwb, binv = ss.binv;
+  const bool ok = ss.ok;
   uint32_t run_wb = 0, run_inv = 0, scanned = 0;
-  const uint32_t head = *(volatile uint32_t *)&st->lrm_head, tail = *(volatile uint32_t *)&st->lrm_tail;
-  const uint32_t lt = (1u << lane) - 1;
-  for (uint32_t c = head; c < tail && run_wb + run_inv < need; c += CHUNK) {
-    scanned += min(CHUNK, tail - c);
-    uint32_t blk[ITEMS], me[ITEMS], mi[ITEMS];
-    uint32_t cw = 0, ci = 0;
+  int buf = 0;
+  for (uint32_t c = head & ~3u; c < tail && run_wb + run_inv < need; c += SEL_CHUNK, buf ^= 1) {
+    scanned += min(c + SEL_CHUNK, tail) - max(c, head);
+    const uint32_t i0 = c + IT * tid;
+    uint32_t v[IT];
+    const uint4 *p = reinterpret_cast<const uint4 *>(so.lrm_blk + i0);
 #pragma unroll
-    for (int k = 0; k < ITEMS; ++k) {
-      const uint32_t i = c + wid * (32 * ITEMS) + 32 * k + lane;
-      blk[k] = i < tail ? so.lrm_blk[i] : NONE;
+    for (uint32_t k = 0; k < IT / 4; ++k) {
+      uint4 x = make_uint4(0, 0, 0, 0);
+      if (i0 + 4 * k < tail) x = p[k];  // log capacity is a multiple of 4: never past the allocation
+      v[4 * k] = x.x;
+      v[4 * k + 1] = x.y;
+      v[4 * k + 2] = x.z;
+      v[4 * k + 3] = x.w;
     }
+    // entries of this thread inside [head, tail)
+    uint32_t valid = 0;
+    if (i0 < tail && i0 + IT > head) {
+      const uint32_t lo = i0 < head ? head - i0 : 0, hi = min(IT, tail - i0);
+      valid = (hi >= 32 ? 0xFFFFFFFFu : (1u << hi) - 1) & ~((1u << lo) - 1);
+    }
+    uint32_t em = 0, im = 0;  // eligible active / inactive entries (bit k = entry i0 + k)
 #pragma unroll
-    for (int k = 0; k < ITEMS; ++k) {
-      const uint32_t i = c + wid * (32 * ITEMS) + 32 * k + lane;
-      const uint32_t b = blk[k] & 0x7FFFFFFFu;  // log entry: block | inactive << 31
-      bool elig = false, ina = false;
-      if (i < tail) {
-        elig = !(bitmap[b >> 5] & (1u << (b & 31)));
-        if (elig && !clean) elig = __ldg(&so.frame_of[b]) != NONE && __ldg(&so.stamp_of[b]) == so.lrm_stamp[i];
-        ina = blk[k] >> 31;
-      }
-      blk[k] = b;
-      me[k] = __ballot_sync(0xffffffffu, elig && !ina);
-      mi[k] = __ballot_sync(0xffffffffu, elig && ina);
-      cw += __popc(me[k]);
-      ci += __popc(mi[k]);
+    for (uint32_t k = 0; k < IT; ++k) {
+      const uint32_t b = v[k] & 0x7FFFFFFFu;
+      uint32_t e = ((valid >> k) & 1u) & ~(bitmap[b >> 5] >> (b & 31));
+      if (!clean && (e & 1u))
+        e = __ldg(&so.frame_of[b]) != NONE && __ldg(&so.stamp_of[b]) == so.lrm_stamp[i0 + k];
+      const uint32_t ina = v[k] >> 31;
+      em |= (e & ~ina & 1u) << k;
+      im |= (e & ina & 1u) << k;
+      v[k] = b;
     }
-    if (lane == 0) {
-      s_wcnt[wid] = cw;
-      s_icnt[wid] = ci;
+    // group exclusive scan of (popc(im) << 16 | popc(em))
+    const uint32_t cnt = (__popc(im) << 16) | __popc(em);
+    uint32_t x = cnt;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= (uint32_t)o) x += y;
     }
-    __syncthreads();
-    // exclusive prefix of the warp totals (log order = warp order): one
-    // packed warp scan over the NW totals (counts <= 128 fit 16 bits)
-    uint32_t pw, pi, tw, ti;
+    if (lane == 31) s_wt[buf][wid] = x;
+    group_sync<BAR, NT>();
+    uint32_t wpre = 0, tot = 0;
     {
-      const uint32_t v = lane < NW ? (s_icnt[lane] << 16) | s_wcnt[lane] : 0;
-      uint32_t x = v;
+      const uint32_t t = lane < (uint32_t)NW ? s_wt[buf][lane] : 0;
+      uint32_t z = t;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-        if (lane >= (uint32_t)o) x += y;
+        const uint32_t y = __shfl_up_sync(0xffffffffu, z, o);
+        if (lane >= (uint32_t)o) z += y;
       }
-      const uint32_t ex = __shfl_sync(0xffffffffu, x - v, wid);
-      const uint32_t tot = __shfl_sync(0xffffffffu, x, NW - 1);
-      pw = ex & 0xFFFFu;
-      pi = ex >> 16;
-      tw = tot & 0xFFFFu;
-      ti = tot >> 16;
+      wpre = __shfl_sync(0xffffffffu, z - t, wid);
+      tot = __shfl_sync(0xffffffffu, z, NW - 1);
     }
+    const uint32_t pre = wpre + x - cnt;
+    const uint32_t pw = pre & 0xFFFFu, pi = pre >> 16;
+    const uint32_t tw = tot & 0xFFFFu, ti = tot >> 16;
     const uint32_t left = need - run_wb - run_inv;
+    // stage this thread's eligible entries of combined rank < left
+    {
+      uint32_t rw = pw, ri = pi;
 #pragma unroll
-    for (int k = 0; k < ITEMS; ++k) {
-      const uint32_t i = c + wid * (32 * ITEMS) + 32 * k + lane;
-      const bool ew = (me[k] >> lane) & 1u, ei = (mi[k] >> lane) & 1u;
-      const uint32_t rw = pw + __popc(me[k] & lt), ri = pi + __popc(mi[k] & lt);
-      if ((ew || ei) && rw + ri < left && ok) {
-        if (ei) so.inv[binv + run_inv + ri] = blk[k];
-        else so.wb[bwb + run_wb + rw] = blk[k];
+      for (uint32_t k = 0; k < IT; ++k) {
+        const uint32_t ew = (em >> k) & 1u, ei = (im >> k) & 1u;
+        if ((ew | ei) && rw + ri < left) stage[ei ? SEL_CHUNK - 1 - ri : rw] = v[k];
+        rw += ew;
+        ri += ei;
       }
-      (void)i;
-      pw += __popc(me[k]);
-      pi += __popc(mi[k]);
     }
-    // the taken entries are the first `left` eligible ones of the chunk; how
-    // many of them are write-back vs invalidate
     uint32_t take_w = tw, take_i = ti;
     if (tw + ti > left) {
-      // find the split inside the chunk: the warp holding eligible entry `left`
-      if (tid == 0) {
-        uint32_t aw = 0, ai = 0;
-        s_split = NONE;
-        for (int w = 0; w < NW; ++w) {
-          if (aw + ai + s_wcnt[w] + s_icnt[w] > left) {
-            s_split = w;
-            s_rem = left - aw - ai;  // eligible entries of warp w that are taken
-            break;
-          }
-          aw += s_wcnt[w];
-          ai += s_icnt[w];
-        }
-        s_aw = aw;  // totals of the warps before the split warp
-        s_ai = ai;
-      }
-      __syncthreads();
-      const uint32_t w_split = s_split, rem = s_rem;
-      const uint32_t aw = s_aw, ai = s_ai;
-      if (wid == w_split) {
-        // walk this warp's 4 steps in order; lanes count taken entries
-        uint32_t r = rem, cw2 = 0, ci2 = 0;
+      // the last chunk: the thread holding combined rank `left` reports how
+      // many of the taken entries are of each kind
+      const uint32_t p0 = pw + pi, nall = __popc(em | im);
+      if (p0 <= left && left < p0 + nall) {
+        uint32_t aw = pw, ai = pi;
 #pragma unroll
-        for (int k = 0; k < ITEMS; ++k) {
-          const uint32_t all = me[k] | mi[k];
-          const uint32_t nall = __popc(all);
-          if (r >= nall) {
-            cw2 += __popc(me[k]);
-            ci2 += __popc(mi[k]);
-            r -= nall;
-          } else if (r > 0) {
-            // first r set bits of `all`
-            uint32_t m = all, sel = 0;
-            for (uint32_t q = 0; q < r; ++q) {
-              const uint32_t bit = m & (~m + 1u);
-              sel |= bit;
-              m &= m - 1;
-            }
-            cw2 += __popc(me[k] & sel);
-            ci2 += __popc(mi[k] & sel);
-            r = 0;
+        for (uint32_t k = 0; k < IT; ++k) {
+          if (aw + ai < left) {
+            aw += (em >> k) & 1u;
+            ai += (im >> k) & 1u;
           }
         }
-        if (lane == 0) {
-          s_tw = aw + cw2;
-          s_ti = ai + ci2;
-        }
+        s_tw = aw;
+        s_ti = ai;
       }
-      __syncthreads();
+      group_sync<BAR, NT>();
       take_w = s_tw;
       take_i = s_ti;
+    } else {
+      group_sync<BAR, NT>();
+    }
+    if (ok) {
+      for (uint32_t j = tid; j < take_w; j += NT) so.wb[bwb + run_wb + j] = stage[j];
+      for (uint32_t j = tid; j < take_i; j += NT) so.inv[binv + run_inv + j] = stage[SEL_CHUNK - 1 - j];
     }
     run_wb += take_w;
     run_inv += take_i;
-    __syncthreads();
   }
   if (tid == 0) {
     uint64_t *o = so.out_range + 4ull * qi;
