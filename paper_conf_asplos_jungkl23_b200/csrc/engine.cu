@@ -114,7 +114,7 @@ void free_all(dum_engine *e) {
                   e->d_walk_chain, e->d_walk_tmp, e->d_walk_out, e->d_anchor_pool, e->d_anchor_range,
                   e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits, e->d_inactive_bits, e->d_res_bits, e->d_logpos, e->d_lrm_blk,
                   e->d_lrm_stamp, e->d_mig_frames, e->d_mig_src, e->d_mig_blocks, e->d_state, e->d_qkern,
-                  e->d_qloff, e->d_qnk, e->d_qbase, e->d_rec_slot, e->d_jump, e->d_wrun, e->d_wrun_len, e->d_qeoff, e->d_qgoff};
+                  e->d_qloff, e->d_qnk, e->d_qbase, e->d_rec_slot, e->d_jump, e->d_wrun, e->d_wrun_len, e->d_qeoff, e->d_qgoff, e->d_qrank, e->d_qperm};
   for (void *p : ptrs)
     if (p) cudaFree(p);
   if (e->ev_fork) cudaEventDestroy(e->ev_fork);
@@ -278,6 +278,8 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_qloff, (uint64_t)e->anchor_range_cap * (g.N + 2)));
   A_(dmalloc(&e->d_qeoff, (uint64_t)e->anchor_range_cap * (g.N + 2)));
   A_(dmalloc(&e->d_qgoff, (uint64_t)e->anchor_range_cap * (g.N + 2)));
+  A_(dmalloc(&e->d_qrank, e->anchor_range_cap));
+  A_(dmalloc(&e->d_qperm, e->anchor_range_cap));
   A_(dmalloc(&e->d_qnk, e->anchor_range_cap));
   A_(dmalloc(&e->d_qbase, e->anchor_range_cap));
   A_(dmalloc(&e->d_frame_of, g.W));

@@ -64,6 +64,8 @@ struct DevState {
   uint32_t log_dirty;         // LRM log may hold entries of evicted blocks
   uint32_t dbg_line, dbg_val; // first failed internal guard (GUARD macro)
   uint32_t cls_cnt[4];        // build: faulting launches per size class
+  uint32_t q_cls[8];          // predict: queries per window-size class (k_chain)
+  uint32_t chain_done;        // predict: k_chain CTAs finished
   unsigned long long ctr[DUM_NCOUNTERS];  // work counters (instrumentation)
 };
 
@@ -161,7 +163,8 @@ struct dum_engine {
   uint64_t anchor_pool_entries;
   uint64_t *d_anchor_range;   // per query (begin, len)
   uint32_t anchor_range_cap;  // max queries per predict call
-  uint32_t *d_qkern, *d_qloff, *d_qeoff, *d_qgoff, *d_qnk;  // per-query chain scratch (k_chain -> k_predict)
+  uint32_t *d_qkern, *d_qloff, *d_qeoff, *d_qgoff, *d_qnk;
+  uint32_t *d_qrank, *d_qperm;  // window-size class rank per query; predict CTA order (largest first)  // per-query chain scratch (k_chain -> k_predict)
   unsigned long long *d_qbase;
   // residency
   uint32_t *d_frame_of, *d_stamp_of, *d_block_of, *d_free_bits, *d_inactive_bits, *d_res_bits;

@@ -123,6 +123,8 @@ struct PredArgs {
   uint32_t *qeoff;  // [nq][N+2] run-entry offsets of the window's lists
   uint32_t *qgoff;  // [nq][N+2] 128-block copy-chunk offsets of the window's lists
   uint32_t *qnk;    // [nq]
+  uint32_t *qrank;  // [nq] class << 24 | rank within the window-size class
+  uint32_t *qperm;  // [nq] k_predict CTA b answers query qperm[b] (largest windows first)
   unsigned long long *qbase;  // [nq]
   uint32_t *big_pool;         // scratch for the exact slow path
   uint64_t big_entries;
@@ -137,6 +139,7 @@ __device__ __forceinline__ unsigned long long pred_timer() {
 }
 
 constexpr int CHAIN_WARPS = 8;
+constexpr int NQCLS = 5;  // window-size classes of the predict CTA order
 constexpr uint32_t CHUNK_B = 128;  // window blocks per copy chunk (one warp: 4 coalesced steps)
 
 __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
@@ -244,6 +247,34 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
     for (uint32_t i = 0; i < w; ++i) base += s_u[i];
     a.qbase[qi] = base;
     if (base + U > a.cap) set_err(a.st, ERR_ECAPACITY, base + U);
+    // window-size class (largest first) for k_predict's CTA order: the big
+    // windows start first instead of forming the tail
+    const uint32_t c = U >= 14336 ? 0u : U >= 10240 ? 1u : U >= 6144 ? 2u : U >= 2048 ? 3u : 4u;
+    a.qrank[qi] = (c << 24) | atomicAdd(&a.st->q_cls[c], 1u);
+  }
+  // the last CTA turns (class, rank) into the permutation
+  __shared__ bool s_last;
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) s_last = atomicAdd(&a.st->chain_done, 1u) == gridDim.x - 1;
+  __syncthreads();
+  if (s_last) {
+    __threadfence();
+    uint32_t pre[NQCLS];
+    uint32_t acc = 0;
+#pragma unroll
+    for (int c = 0; c < NQCLS; ++c) {
+      pre[c] = acc;
+      acc += *(volatile uint32_t *)&a.st->q_cls[c];
+    }
+    for (uint32_t q = threadIdx.x; q < a.nq; q += blockDim.x) {
+      const uint32_t r = __ldcg(a.qrank + q);
+      uint32_t p = r & 0xFFFFFFu;
+#pragma unroll
+      for (int c = 0; c < NQCLS; ++c)
+        if ((r >> 24) == (uint32_t)c) p += pre[c];
+      a.qperm[p] = q;
+    }
   }
 }
 
@@ -252,7 +283,7 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
 // the (block, exec) pairs meanwhile.  Duplicates (rare) are only known after
 // pass 1: the duplicate path then rewrites the pairs and redoes the selection
 // with the whole CTA.
-constexpr int GRP_W = NWARP / 2;
+constexpr int GRP_W = 10;  // window set + selection warps; the other NWARP - GRP_W copy
 constexpr int GRP_NT = GRP_W * 32;
 constexpr uint32_t OCCAP = 1024;   // duplicate occurrences (list, block) tracked by the duplicate path
 constexpr uint32_t DWCAP = 1024;   // duplicate-word hash slots (word -> mask of duplicated blocks)
@@ -273,7 +304,7 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
   __shared__ uint32_t s_dup[2 * OCCAP];  // pass 1: duplicated blocks; duplicate path: occurrences (list, block)
   __shared__ unsigned long long s_hoff;
   const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  const uint32_t qi = blockIdx.x;
+  const uint32_t qi = a.qperm[blockIdx.x];
   const Geo &g = a.g;
   const uint32_t anchor = a.q[qi].anchor;
   const bool anchored = anchor != NONE;
@@ -340,6 +371,7 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
     constexpr uint32_t UN = 2;
     const uint32_t G = nk ? goff[nk] : 0;
     uint2 *out = reinterpret_cast<uint2 *>(a.pairs) + base;
+    uint32_t cur = 0;  // list of the chunk (chunks only grow: a running cursor)
     for (uint32_t c0 = cw; c0 < G; c0 += ncw * UN) {
       uint32_t b[UN][4], dd[UN], i0[UN], L[UN];
 #pragma unroll
@@ -347,7 +379,8 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
         const uint32_t c = c0 + u * ncw;
         dd[u] = NONE;
         if (c < G) {
-          const uint32_t lo = search(goff, c);
+          while (goff[cur + 1] <= c) ++cur;
+          const uint32_t lo = cur;
           if (skip && skip[lo]) continue;
           dd[u] = lo;
           i0[u] = (c - goff[lo]) * CHUNK_B;
@@ -392,9 +425,20 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
       const uint32_t m = 1u << (anchor & 31);
       record_dup(anchor >> 5, atomicOr(&bitmap[anchor >> 5], m) & m);
     }
+    uint32_t lo = 0;  // list of run x (x only grows: a running cursor, no search)
     for (uint32_t x = tid; x < etot; x += GRP_NT) {
-      uint32_t lo, w, m;
-      run_at(x, lo, w, m);
+      while (eoff[lo + 1] <= x) ++lo;
+      const uint32_t i = x - eoff[lo];
+      uint32_t w, m;
+      if (lo == 0 && anchored) {
+        const uint32_t b = apool[i];
+        w = b >> 5;
+        m = 1u << (b & 31);
+      } else {
+        const uint2 r = __ldg(reinterpret_cast<const uint2 *>(a.wrun) + (uint64_t)kern[lo] * g.walk_cap + i);
+        w = r.x;
+        m = r.y;
+      }
       record_dup(w, atomicOr(&bitmap[w], m) & m);
       if (SELECT) nonres += __popc(m & ~__ldg(&a.so.res_bits[w]));
     }
@@ -674,6 +718,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   if (nq > e->anchor_range_cap) return cudaErrorInvalidValue;
   cudaMemsetAsync(&e->d_state->pool_pairs, 0, 2 * sizeof(unsigned long long) * 2, s);  // pairs, wb, inv, anchor
   cudaMemsetAsync(&e->d_state->pool_big, 0, sizeof(unsigned long long), s);
+  cudaMemsetAsync(e->d_state->q_cls, 0, sizeof(e->d_state->q_cls) + sizeof(e->d_state->chain_done), s);
   WalkScratch ws{e->d_walk_seen, e->d_walk_chain, e->d_walk_tmp, e->walk_hash_cap,
                  e->g.walk_cap + e->g.R * e->g.A + 4};
   {
@@ -706,6 +751,8 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   a.qloff = e->d_qloff;
   a.qeoff = e->d_qeoff;
   a.qgoff = e->d_qgoff;
+  a.qrank = e->d_qrank;
+  a.qperm = e->d_qperm;
   a.qnk = e->d_qnk;
   a.qbase = e->d_qbase;
   a.big_pool = e->d_big_pool;

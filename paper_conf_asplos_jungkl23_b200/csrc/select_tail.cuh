@@ -64,14 +64,15 @@ __device__ __forceinline__ void group_sync() {
 // shared memory (write-back from the front, invalidate from the back) and
 // copied out with coalesced stores.  Warp totals are double-buffered: a chunk
 // costs two barriers (three in the last one).
-constexpr uint32_t SEL_CHUNK = 4096;
+constexpr uint32_t SEL_CHUNK = 4096;  // stage capacity (words); a chunk is NT * IT <= SEL_CHUNK entries
 
 template <int NT, int BAR>
 __device__ void select_tail(const SelectOut &so, uint32_t qi, const SelShared &ss, const uint32_t *bitmap,
                             DevState *st, uint32_t tid, uint32_t *stage /* SEL_CHUNK words of shared memory */) {
   constexpr int NW = NT / 32;
-  constexpr uint32_t IT = SEL_CHUNK / NT;
-  static_assert(NW <= 32 && IT % 4 == 0 && IT <= 16, "one warp scans the warp totals; 16 B loads");
+  constexpr uint32_t IT = NT >= 512 ? 8 : NT >= 320 ? 12 : 16;
+  constexpr uint32_t CHUNK = NT * IT;
+  static_assert(NW <= 32 && IT % 4 == 0 && CHUNK <= SEL_CHUNK, "one warp scans the warp totals; 16 B loads");
   __shared__ uint32_t s_wt[2][NW], s_tw, s_ti;
   const uint32_t lane = tid & 31, wid = tid >> 5;
   const uint32_t need = ss.need, head = ss.head, tail = ss.tail;
@@ -80,8 +81,8 @@ __device__ void select_tail(const SelectOut &so, uint32_t qi, const SelShared &s
   const bool ok = ss.ok;
   uint32_t run_wb = 0, run_inv = 0, scanned = 0;
   int buf = 0;
-  for (uint32_t c = head & ~3u; c < tail && run_wb + run_inv < need; c += SEL_CHUNK, buf ^= 1) {
-    scanned += min(c + SEL_CHUNK, tail) - max(c, head);
+  for (uint32_t c = head & ~3u; c < tail && run_wb + run_inv < need; c += CHUNK, buf ^= 1) {
+    scanned += min(c + CHUNK, tail) - max(c, head);
     const uint32_t i0 = c + IT * tid;
     uint32_t v[IT];
     const uint4 *p = reinterpret_cast<const uint4 *>(so.lrm_blk + i0);
@@ -144,7 +145,7 @@ __device__ void select_tail(const SelectOut &so, uint32_t qi, const SelShared &s
 #pragma unroll
       for (uint32_t k = 0; k < IT; ++k) {
         const uint32_t ew = (em >> k) & 1u, ei = (im >> k) & 1u;
-        if ((ew | ei) && rw + ri < left) stage[ei ? SEL_CHUNK - 1 - ri : rw] = v[k];
+        if ((ew | ei) && rw + ri < left) stage[ei ? CHUNK - 1 - ri : rw] = v[k];
         rw += ew;
         ri += ei;
       }
@@ -174,7 +175,7 @@ __device__ void select_tail(const SelectOut &so, uint32_t qi, const SelShared &s
     }
     if (ok) {
       for (uint32_t j = tid; j < take_w; j += NT) so.wb[bwb + run_wb + j] = stage[j];
-      for (uint32_t j = tid; j < take_i; j += NT) so.inv[binv + run_inv + j] = stage[SEL_CHUNK - 1 - j];
+      for (uint32_t j = tid; j < take_i; j += NT) so.inv[binv + run_inv + j] = stage[CHUNK - 1 - j];
     }
     run_wb += take_w;
     run_inv += take_i;
