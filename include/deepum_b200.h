@@ -307,6 +307,7 @@ enum {
   DUM_T_RESIDENCY,
   DUM_T_CHAIN,
   DUM_T_JUMP,         /* jump tables over the correlation table (side stream, in dum_build_tables) */
+  DUM_T_WALK,         /* parallel walk-cache rebuild (in dum_build_tables) */
   DUM_NTIMERS = 16
 };
 int dum_set_timing(dum_engine *eng, int enable);

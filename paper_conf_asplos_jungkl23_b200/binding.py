@@ -23,14 +23,14 @@ CTR = {n: i for i, n in enumerate(["RAW_RECORDS", "NORM_RECORDS", "LAUNCHES", "C
                                    "SEL_WINDOW", "SEL_SCANNED", "SEL_VICTIMS", "MIG_BLOCKS", "RUNS"])}
 TIMER = {n: i for i, n in enumerate(["INGEST", "EXEC_ASSIGN", "BUILD_PREP", "APPLY_WALK", "WALK_SLOW",
                                      "MAKE_QUERIES", "ANCHOR_WALK", "PREDICT", "SELECT", "MIG_PLAN", "COPY",
-                                     "RESIDENCY", "CHAIN", "JUMP"])}
+                                     "RESIDENCY", "CHAIN", "JUMP", "WALK"])}
 KERNEL_OF_TIMER = {"INGEST": "k_ingest", "EXEC_ASSIGN": "k_exec_assign", "BUILD_PREP": "k_build_prep",
-                   "APPLY_WALK": "k_apply_walk", "WALK_SLOW": "k_walk_slow", "MAKE_QUERIES": "k_make_queries",
+                   "APPLY_WALK": "k_apply", "WALK": "k_walk", "WALK_SLOW": "k_walk_slow", "MAKE_QUERIES": "k_make_queries",
                    "ANCHOR_WALK": "k_anchor_walk", "PREDICT": "k_predict", "SELECT": "k_select",
                    "MIG_PLAN": "k_mig_plan", "COPY": "k_copy_blocks", "RESIDENCY": "k_load_res",
                    "CHAIN": "k_chain", "JUMP": "k_jump0"}
 # timers of kernels launched on the engine's side stream (overlapping others)
-SIDE_TIMERS = {"JUMP": "side stream, overlaps k_apply_walk (k_jump0 + k_jumpk levels)"}
+SIDE_TIMERS = {"JUMP": "side stream, overlaps k_apply / k_walk (k_jump0 + k_jumpk levels)"}
 _ERR = {0: "DUM_OK", -1: "DUM_EINVAL", -2: "DUM_ECAPACITY", -3: "DUM_ENOMEM", -4: "DUM_ECUDA", -5: "DUM_ESTATE"}
 
 

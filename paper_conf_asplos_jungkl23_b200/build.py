@@ -44,8 +44,13 @@ def build(force: bool = False, verbose: bool = False, ptxas_v: bool = False, che
     os.makedirs(bdir, exist_ok=True)
     objs = []
 
+    hdr_t = max(os.path.getmtime(p) for p in _deps() if not p.endswith(".cu"))
+
     def one(src):
         obj = os.path.join(bdir, os.path.basename(src) + ".o")
+        if (not force and os.path.exists(obj) and os.path.getmtime(obj) >= os.path.getmtime(src)
+                and os.path.getmtime(obj) >= hdr_t):
+            return obj  # incremental: object newer than its source and every header
         cmd = [NVCC, *ARCH, *FLAGS, "-c", src, "-o", obj] + (["-DDUM_CHECKS", "-DDUM_POISON"] if checks else [])
         if ptxas_v:
             cmd[1:1] = ["-Xptxas", "-v"]

@@ -84,6 +84,7 @@ cudaError_t fill(uint32_t *p, uint64_t n, uint32_t v, cudaStream_t s) {
 
 int reset_state(dum_engine *e, cudaStream_t s) {
   const Geo &g = e->g;
+  if (e->ev_join) CK(cudaStreamWaitEvent(s, e->ev_join, 0));  // jump tables still building on the side stream
   CK(fill((uint32_t *)e->d_exec_keys, 2ull * (e->exec_cap + 1), NONE, s));
   CK(cudaMemsetAsync(e->d_exec_keys + e->exec_cap, 0, 8, s));  // sentinel slot: absent
   CK(fill(e->d_exec_vals, e->exec_cap + 1, PENDING, s));
@@ -95,6 +96,8 @@ int reset_state(dum_engine *e, cudaStream_t s) {
   CK(cudaMemsetAsync(e->d_walk_len, 0, 4ull * g.Emax, s));
   CK(cudaMemsetAsync(e->d_wrun_len, 0, 4ull * g.Emax, s));
   CK(fill(e->d_head, g.Emax, NONE, s));
+  CK(cudaMemsetAsync(e->d_e_ops, 0, 4ull * g.Emax, s));
+  CK(cudaMemsetAsync(e->d_e_last, 0, 4ull * g.Emax, s));
   k_init_state<<<1, 1, 0, s>>>(e->d_state);
   CK(cudaGetLastError());
   CK(launch_reset_residency(e, s));
@@ -110,7 +113,8 @@ void free_all(dum_engine *e) {
   void *ptrs[] = {e->d_exec_keys, e->d_exec_vals, e->d_exec_minpos, e->d_exec_hash, e->d_corr, e->d_tbl,
                   e->d_start_end, e->d_walk, e->d_walk_len, e->d_in_hash, e->d_in_off, e->d_in_faults,
                   e->d_stage_hash, e->d_stage_norm, e->d_stage_cnt, e->d_stage_exec, e->d_stage_slot,
-                  e->d_stage_off, e->d_head, e->d_next, e->d_order, e->d_slow_list, e->d_big_pool, e->d_walk_seen,
+                  e->d_stage_off, e->d_head, e->d_next, e->d_order, e->d_slow_list,
+                  e->d_e_ops, e->d_e_last, e->d_lead, e->d_items, e->d_rowc, e->d_big_pool, e->d_walk_seen,
                   e->d_walk_chain, e->d_walk_tmp, e->d_walk_out, e->d_anchor_pool, e->d_anchor_range,
                   e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits, e->d_inactive_bits, e->d_res_bits, e->d_logpos, e->d_lrm_blk,
                   e->d_lrm_stamp, e->d_mig_frames, e->d_mig_src, e->d_mig_blocks, e->d_state, e->d_qkern,
@@ -244,7 +248,8 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
     // their CTAs go ahead of the block-table apply they overlap
     int lo = 0, hi = 0;
     cudaDeviceGetStreamPriorityRange(&lo, &hi);
-    A_(cudaStreamCreateWithPriority(&e->side, cudaStreamNonBlocking, hi));
+    const char *jm = getenv("DUM_JUMP_MODE");
+    A_(cudaStreamCreateWithPriority(&e->side, cudaStreamNonBlocking, (jm && jm[0] == '1') ? lo : hi));
   }
   A_(cudaEventCreateWithFlags(&e->ev_fork, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_join, cudaEventDisableTiming));
@@ -267,6 +272,13 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_next, e->stage_launch_cap));
   A_(dmalloc(&e->d_order, 3ull * e->stage_launch_cap));
   A_(dmalloc(&e->d_slow_list, e->stage_launch_cap));
+  A_(dmalloc(&e->d_e_ops, g.Emax));
+  A_(dmalloc(&e->d_e_last, g.Emax));
+  A_(dmalloc(&e->d_lead, 8ull * e->stage_launch_cap));  // k_build.cu LeadDesc (32 B)
+  // apply items: sum over groups of ceil(ops / 256) <= launches + faults / 256
+  e->items_cap = e->stage_launch_cap + e->stage_fault_cap / 256 + 1;
+  A_(dmalloc(&e->d_items, 2 * e->items_cap));
+  A_(dmalloc(&e->d_rowc, e->stage_fault_cap * (1ull + g.S)));
   A_(dmalloc(&e->d_big_pool, 2 * e->big_pool_entries));
   A_(dmalloc(&e->d_walk_seen, (uint64_t)e->n_walk_slots * e->walk_hash_cap));
   A_(dmalloc(&e->d_walk_chain, (uint64_t)e->n_walk_slots * e->walk_hash_cap));
@@ -372,8 +384,11 @@ int dum_record_faults(dum_engine *e, const uint64_t *launch_hash, const uint64_t
     if (launch_off[0] != 0 || launch_off[n_launch] != n_fault) return fail(e, DUM_EINVAL, "batch not launch-aligned");
     for (uint32_t i = 0; i < n_launch; ++i)
       if (launch_off[i + 1] < launch_off[i]) return fail(e, DUM_EINVAL, "launch_off not monotone");
-    for (uint64_t i = 0; i < n_fault; ++i)
-      if (fault_block[i] >= e->g.W) return fail(e, DUM_EINVAL, "block id >= max_blocks");
+    // branch-free max (vectorised by the compiler): the check costs a fraction
+    // of the copy it guards
+    uint32_t mx = 0;
+    for (uint64_t i = 0; i < n_fault; ++i) mx = fault_block[i] > mx ? fault_block[i] : mx;
+    if (n_fault && mx >= e->g.W) return fail(e, DUM_EINVAL, "block id >= max_blocks");
     CK(cudaMemcpyAsync(e->d_in_hash, launch_hash, 8ull * n_launch, cudaMemcpyHostToDevice, s));
     CK(cudaMemcpyAsync(e->d_in_off, launch_off, 8ull * (n_launch + 1), cudaMemcpyHostToDevice, s));
     if (n_fault) CK(cudaMemcpyAsync(e->d_in_faults, fault_block, 4ull * n_fault, cudaMemcpyHostToDevice, s));

@@ -66,6 +66,7 @@ struct DevState {
   uint32_t cls_cnt[4];        // build: faulting launches per size class
   uint32_t q_cls[8];          // predict: queries per window-size class (k_chain)
   uint32_t chain_done;        // predict: k_chain CTAs finished
+  uint32_t n_items, n_leads;  // build: k_apply items / k_walk items (k_plan)
   unsigned long long ctr[DUM_NCOUNTERS];  // work counters (instrumentation)
 };
 
@@ -137,7 +138,7 @@ struct dum_engine {
   cudaEvent_t ev_fork, ev_join;
   // block tables / walk cache
   uint32_t *d_tbl, *d_start_end, *d_walk, *d_walk_len;
-  uint32_t *d_wrun, *d_wrun_len;   // walk as (word, mask) runs (k_apply_walk / k_walk_slow)
+  uint32_t *d_wrun, *d_wrun_len;   // walk as (word, mask) runs (k_walk / k_walk_slow)
   // staging
   uint32_t stage_launch_cap;
   uint64_t stage_fault_cap;
@@ -152,6 +153,11 @@ struct dum_engine {
   uint64_t built_launches;
   // build scratch
   uint32_t *d_head, *d_next, *d_slow_list, *d_order;
+  uint32_t *d_e_ops, *d_e_last;  // per exec ID: group operations / latest launch of the batch
+  uint32_t *d_lead;              // exec IDs with faults of the batch (k_build.cu LeadDesc, 32 B each)
+  uint32_t *d_items;             // apply items, u32 pairs (leader index, partition | P << 16)
+  uint64_t items_cap;
+  uint32_t *d_rowc;              // walk row cache for long walks: (1 + S) u32 per staged record
   uint32_t *d_big_pool;   // u32 pairs for large-walk hash tables
   uint64_t big_pool_entries;
   // walk scratch for the sequential walker (per CTA slot)

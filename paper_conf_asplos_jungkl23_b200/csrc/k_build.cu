@@ -5,19 +5,27 @@
 //                 execution ID correlation table (PAPER.md; D5): key claimed
 //                 with a 128-bit CAS, successor = max(k<<32 | e_k) ("last
 //                 wins"), order = min(k) ("first seen") -- order-independent
-//                 (SURVEY P4).  Links the launch into its exec ID's group.
-//  k_apply_walk   one CTA per exec ID with faults in the batch (the group
-//                 leader).  Applies the block-table operations of all its
-//                 launches (D7-D11): per fault b_j,
-//                 INSERT b_j into row(b_{j-1}) then TOUCH b_j.  Tables of
-//                 different exec IDs are independent (P1) and operations on
-//                 different sets commute (P2), so the ops are counting-sorted by
-//                 set in shared memory and each set's ops are applied in order
-//                 by one thread, with the set held in registers.  Then it
-//                 rebuilds the walk cache WALK(e, NONE) (
-//                 D13) in parallel -- see walk_fast() -- and records Start/End.
+//                 (SURVEY P4).  Links the launch into its exec ID's group and
+//                 sums the group's operations / latest launch.
+//  k_plan         one CTA: the history shift register, and the work lists of
+//                 the two persistent kernels below -- one walk item per exec ID
+//                 with faults (its group leader), and P apply items per exec ID,
+//                 P = ceil(ops / OPP) set partitions (largest groups first).
+//  k_apply        persistent; item (e, c of P): applies the block-table
+//                 operations of exec ID e whose set lies in partition c
+//                 (D7-D10): per fault b_j, INSERT b_j
+//                 into row(b_{j-1}) then TOUCH b_j.  Tables of different exec IDs
+//                 are independent (P1) and operations on different sets commute
+//                 (P2): a CTA owns the sets {s : (s / 32) mod P = c}, selects their
+//                 operations in order, groups them by set through a shared hash,
+//                 and one thread per set applies the set's operations with the set
+//                 held in registers.  Big exec IDs are thereby spread over many
+//                 SMs instead of one.
+//  k_walk         persistent; one exec ID per item: Start/End, then the walk
+//                 cache WALK(e, NONE) (D13) in parallel --
+//                 see the comment above the kernel.
 //  k_walk_slow    sequential one-warp walker; takes the exec IDs whose walk
-//                 exceeded the parallel path's scratch (never on the configs
+//                 the parallel path cannot prove (never on the configs
 //                 measured; kept for exactness on any input).
 #include <cstdio>
 #include <cstdlib>
@@ -30,11 +38,18 @@
 
 namespace dum {
 
-constexpr int BUILD_NT = 512;
-constexpr uint32_t GCAP = 256;    // launches of one exec ID per build batch
-constexpr uint32_t OPCAP = 2048;  // ops per apply round
-constexpr uint32_t QCAP = 4096;   // smem walk-dedupe hash capacity (|Q| <= 2048)
-constexpr uint32_t WCAP = 2048;   // smem per-row counts (latest launch <= 2048 faults)
+constexpr uint32_t GCAP = 256;     // launches of one exec ID per build batch
+constexpr int PLAN_NT = 1024;
+constexpr int AP_NT = 256;         // k_apply threads
+constexpr uint32_t OPP = 256;      // target operations per apply partition
+constexpr uint32_t PMAX = 64;      // partitions per exec ID (<= R / 32)
+constexpr uint32_t AP_OPCAP = 1024;  // selected operations per apply round
+constexpr uint32_t AP_SCAN = 2 * AP_NT;  // operations scanned per selection step
+constexpr uint32_t AP_HCAP = 2 * AP_OPCAP;
+constexpr int WK_NT = 256;         // k_walk threads
+constexpr uint32_t WK_RC = 5120;   // shared row-cache words (n (1 + S) <= WK_RC)
+constexpr uint32_t WK_CQ = 1024;   // shared chain-position words (n <= WK_CQ)
+constexpr uint32_t WK_QCAP = 4096; // shared dedupe-hash capacity (|Q| <= WK_QCAP / 2)
 
 // ---------------------------------------------------------------------------
 // k_build_prep
@@ -42,7 +57,7 @@ constexpr uint32_t WCAP = 2048;   // smem per-row counts (latest launch <= 2048 
 __global__ void k_build_prep(uint32_t n_staged, uint32_t k0, const uint32_t *__restrict__ stage_exec,
                              const uint32_t *__restrict__ stage_cnt, CorrSlot *corr, uint32_t corr_cap,
                              uint32_t *rec_slot, uint32_t *head, uint32_t *__restrict__ next,
-                             uint32_t *__restrict__ order, DevState *st) {
+                             uint32_t *__restrict__ order, uint32_t *e_ops, uint32_t *e_last, DevState *st) {
   const uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
   if (j == 0) {
     st->pool_big = 0;
@@ -61,7 +76,9 @@ __global__ void k_build_prep(uint32_t n_staged, uint32_t k0, const uint32_t *__r
   if ((threadIdx.x & 31) == __ffs(__activemask()) - 1) ctr_add(st, DUM_CTR_CORR_UPSERTS, nup);
   if (e != NONE && stage_cnt[j] > 0) {
     next[j] = atomicExch(&head[e], j);
-    // big launches first, so the longest CTAs of k_apply_walk start earliest
+    atomicAdd(&e_ops[e], stage_cnt[j]);
+    atomicMax(&e_last[e], j);
+    // big launches first (k_plan orders the work lists by this class)
     const uint32_t c = stage_cnt[j] >= 1024 ? 0u : stage_cnt[j] >= 128 ? 1u : 2u;
     order[c * n_staged + atomicAdd(&st->cls_cnt[c], 1u)] = j;
   }
@@ -206,23 +223,36 @@ struct RegSet {
   }
 };
 
+
 // ---------------------------------------------------------------------------
-// k_apply_walk
+// k_plan
 // ---------------------------------------------------------------------------
+// One exec ID with faults in the batch (written by k_plan, read by k_apply / k_walk).
+struct LeadDesc {
+  uint32_t j, e;                // group leader launch (head of the group list), exec ID
+  uint32_t single, n_ops;       // the group is one launch; operations of the group
+  uint32_t n_last, pad;         // faults of the latest launch of the group
+  unsigned long long off_last;  // its staging offset
+};
+
 struct BuildArgs {
   Geo g;
   uint32_t n_staged;
   const uint32_t *stage_exec, *stage_cnt, *stage_norm;
   const uint64_t *stage_off;
   uint32_t *head, *next;
+  uint32_t *e_ops, *e_last;    // per exec ID: operations / latest launch of the batch (k_build_prep)
+  LeadDesc *desc;              // [n_leads] exec IDs with faults, largest launches first
+  uint2 *items;                // [n_items] apply items (leader index, c | P << 16)
   uint32_t *tbl, *start_end, *walk, *walk_len;
+  uint32_t *rowc;              // global row cache for walks too long for shared memory
   uint32_t *big_pool;
   uint64_t big_entries;
   uint32_t *slow_list;
   uint32_t *wrun, *wrun_len;   // walk bitmap runs (read by k_predict)
   const uint32_t *order;       // [3][n_staged] faulting launches by size class
   DevState *st;
-  unsigned long long *cta_clk;  // debug: per-CTA (start, end, n_ops | n << 32) or null
+  unsigned long long *clk;     // debug (DUM_BUILD_CLOCK): per apply item / walk item 4 x u64, or null
 };
 
 __device__ __forceinline__ unsigned long long gtimer() {
@@ -230,52 +260,18 @@ __device__ __forceinline__ unsigned long long gtimer() {
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
-
-// Parallel WALK(e, NONE) right after the build (D13).  Let C = the latest
-// faulting launch of e in this batch (deduplicated, n = |C|); then Start =
-// C[0], End = C[n-1] (D11).  After the build, the row of C[i] (if still
-// present) has C[i+1] as its MRU successor: INSERT(C[i] -> C[i+1]) was the last
-// operation on that row, because C is duplicate-free and no later launch of e
-// is in the batch.  C[i+1] is not among the chained nodes C[0..i], so the
-// sequential walk's next chain node is exactly C[i+1] until the first i at
-// which the row is missing or a successor equals End.  With t that index, the
-// walk is the first-occurrence dedupe of
-//   Q = [C[0]] ++ succ(row C[0]) ++ ... ++ succ(row C[t])   (row C[t] only if
-//                                                            present).
-// The speculation is still verified (succ[0] == C[i+1]); any violation sends e
-// to the sequential walker.
-//
-// Shared-memory plan (u32 words): grp/seg | row cache of C (count + S succ
-// per position, filled by the set owners right after applying the ops, so the
-// walk never re-reads the table) | per-row Q offsets | a union of the apply
-// arrays (per-set counts/offsets, non-empty-set list, ops, op order) and the
-// walk's dedupe hash.
-constexpr uint32_t RCCAP = 10240;  // row-cache words: n * (1 + S) <= RCCAP
-constexpr uint32_t HCAPMAX = 2 * OPCAP;  // set-hash capacity for a full round
-
-__host__ __device__ inline uint32_t apply_union_words(uint32_t) {
-  const uint32_t ap = 2 * HCAPMAX + 3 * OPCAP, wk = 2 * QCAP;
-  return ap > wk ? ap : wk;
+__device__ __forceinline__ uint32_t smid() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
+  return r;
 }
 
-// link op p at the head of its set's list (order fixed up by the owner)
-__device__ __forceinline__ void sorted_link(uint32_t p, uint32_t slot, uint32_t *hh, uint32_t *lnk) {
-  lnk[p] = atomicExch(&hh[slot], p);
-}
-
-template <int MAXA, int MAXS>
-__global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
-  constexpr int OWN_B = (MAXA * (1 + MAXS) <= 10) ? 2 : 1;  // sets loaded per owner batch
-  extern __shared__ uint32_t sm[];
-  __shared__ uint32_t ws[BUILD_NT / 32];
-  __shared__ uint32_t s_ng, s_tev, s_flag, s_sets, s_nnz, s_nrun;
-  __shared__ unsigned long long goff[GCAP];  // stage offset of each group launch
-  const Geo &g = a.g;
+__global__ void __launch_bounds__(PLAN_NT) k_plan(BuildArgs a) {
+  __shared__ uint32_t ws[PLAN_NT / 32];
   const uint32_t tid = threadIdx.x;
-  const unsigned long long t_begin = a.cta_clk ? gtimer() : 0;
-  if (blockIdx.x == 0 && tid == 0) {
+  if (tid == 0) {
     // history shift register after this batch: the last four exec IDs of
-    // (old history ++ staged launches); read by k_build_prep only.
+    // (old history ++ staged launches); read by the next k_build_prep only
     uint32_t h[4];
     for (int q = 0; q < 4; ++q) {
       const long jj = (long)a.n_staged - 4 + q;
@@ -283,32 +279,55 @@ __global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
     }
     for (int q = 0; q < 4; ++q) a.st->hist[q] = h[q];
   }
-  const uint32_t cls = blockIdx.x / a.n_staged, ci = blockIdx.x % a.n_staged;
-  if (ci >= __ldcg(&a.st->cls_cnt[cls])) return;
-  const uint32_t j = a.order[cls * a.n_staged + ci];
-  const uint32_t e = a.stage_exec[j];
-  if (e == NONE || a.stage_cnt[j] == 0) return;
-  // Leader test, decided once per CTA: thread 0 resets head[e] below, so a
-  // per-thread read could see the reset and drop part of the CTA.
-  if (tid == 0) s_flag = __ldcg(&a.head[e]) == j;
-  __syncthreads();
-  if (!s_flag) return;  // not this exec ID's group leader
-
-  const uint32_t R = g.R, A = g.A, S = g.S;
-  uint32_t *grp = sm;             // [GCAP]
-  uint32_t *seg = grp + GCAP;     // [GCAP + 1]
-  uint32_t *rc = seg + GCAP + 1;  // [RCCAP]
-  uint32_t *cqs = rc + RCCAP;     // [WCAP]
-  uint32_t *U = cqs + WCAP;       // union region
-#ifdef DUM_POISON
-  {
-    const uint32_t words = 2 * GCAP + 1 + RCCAP + WCAP + apply_union_words(R);
-    for (uint32_t w = tid; w < words; w += BUILD_NT) sm[w] = 0xDEAD0000u | (w & 0xFFFF);
-    __syncthreads();
+  const uint32_t c0 = a.st->cls_cnt[0], c1 = a.st->cls_cnt[1], c2 = a.st->cls_cnt[2];
+  const uint32_t tot = c0 + c1 + c2;
+  const uint32_t pmax = max(1u, min(PMAX, a.g.R / 32));
+  uint32_t ibase = 0, lbase = 0;
+  for (uint32_t x0 = 0; x0 < tot; x0 += PLAN_NT) {
+    const uint32_t x = x0 + tid;
+    uint32_t P = 0, j = NONE, e = NONE;
+    if (x < tot) {
+      const uint32_t cls = x < c0 ? 0u : x < c0 + c1 ? 1u : 2u;
+      const uint32_t ci = x - (cls == 0 ? 0u : cls == 1 ? c0 : c0 + c1);
+      j = a.order[cls * a.n_staged + ci];
+      e = a.stage_exec[j];
+      if (a.head[e] == j) P = min(pmax, max(1u, (a.e_ops[e] + OPP - 1) / OPP));
+    }
+    uint32_t totP, totL;
+    const uint32_t ip = block_excl_scan(P, ws, &totP);
+    const uint32_t lp = block_excl_scan(P ? 1u : 0u, ws, &totL);
+    if (P) {
+      LeadDesc d;
+      d.j = j;
+      d.e = e;
+      d.single = a.next[j] == NONE;
+      d.n_ops = a.e_ops[e];
+      const uint32_t last = a.e_last[e];
+      d.n_last = a.stage_cnt[last];
+      d.pad = 0;
+      d.off_last = a.stage_off[last];
+      a.desc[lbase + lp] = d;
+      for (uint32_t c = 0; c < P; ++c) a.items[ibase + ip + c] = make_uint2(lbase + lp, c | (P << 16));
+    }
+    ibase += totP;
+    lbase += totL;
   }
-#endif
+  if (tid == 0) {
+    a.st->n_items = ibase;
+    a.st->n_leads = lbase;
+  }
+}
 
-  // ---- collect and order the group's launches ----
+// ---------------------------------------------------------------------------
+// k_apply
+// ---------------------------------------------------------------------------
+// The launches of exec ID e's group (ascending launch index) into grp, their
+// operation offsets into seg and their staging offsets into goff; returns the
+// group size.  j is the group's leader (the head of its list).
+__device__ __forceinline__ uint32_t load_group(const BuildArgs &a, uint32_t j, uint32_t e, uint32_t *grp,
+                                               uint32_t *seg, unsigned long long *goff, uint32_t *tmp,
+                                               uint32_t *s_ng, uint32_t nt) {
+  const uint32_t tid = threadIdx.x;
   if (tid == 0) {
     uint32_t x = j, n = 0;
     while (x != NONE && n < GCAP) {
@@ -317,21 +336,18 @@ __global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
       x = __ldcg(&a.next[x]);
     }
     if (x != NONE) set_err(a.st, ERR_ECAPACITY, GCAP + 1);
-    s_ng = n;
-    s_sets = 0;
-    a.head[e] = NONE;
+    *s_ng = n;
   }
   __syncthreads();
-  const uint32_t ng = s_ng;
-  if (ng > 1) {
-    uint32_t *tmp = U;  // rank sort (ascending launch index)
-    for (uint32_t p = tid; p < ng; p += BUILD_NT) {
+  const uint32_t ng = *s_ng;
+  if (ng > 1) {  // rank sort (ascending launch index)
+    for (uint32_t p = tid; p < ng; p += nt) {
       uint32_t v = grp[p], r = 0;
       for (uint32_t q = 0; q < ng; ++q) r += grp[q] < v;
       tmp[r] = v;
     }
     __syncthreads();
-    for (uint32_t p = tid; p < ng; p += BUILD_NT) grp[p] = tmp[p];
+    for (uint32_t p = tid; p < ng; p += nt) grp[p] = tmp[p];
     __syncthreads();
   }
   if (tid == 0) {
@@ -344,317 +360,398 @@ __global__ void __launch_bounds__(BUILD_NT, 2) k_apply_walk(BuildArgs a) {
     seg[ng] = acc;
   }
   __syncthreads();
-  if (a.cta_clk && tid == 0) a.cta_clk[10 * j + 3] = gtimer();
-  const uint32_t n_ops = seg[ng];
-  const uint32_t last_seg = seg[ng - 1];
-  const uint32_t Llast = grp[ng - 1];
-  const uint32_t n = a.stage_cnt[Llast];
-  const bool single_round = n_ops <= OPCAP;
-  const bool use_rc = single_round && n <= WCAP && n * (1 + S) <= RCCAP;
-  uint32_t *tbl_e = a.tbl + (uint64_t)e * R * g.stride;
+  return ng;
+}
 
-  // ---- apply: rounds of up to OPCAP ops, grouped by set ----
-  // Each op (fused TOUCH b_p + INSERT b_p -> b_{p+1}) is linked into its set's
-  // list through a shared hash keyed by set index (O(ops), independent of R);
-  // the owner of a set collects the set's ops, orders them by position (lists
-  // are tiny), loads the set into registers, applies them and stores it.
-  uint32_t *hk = U, *hh = U + HCAPMAX;          // set key, list head
-  uint32_t *opb = U + 2 * HCAPMAX, *onx = opb + OPCAP;
-  for (uint32_t r0 = 0; r0 < n_ops; r0 += OPCAP) {
-    const uint32_t m = min(OPCAP, n_ops - r0);
-    uint32_t hcap = pow2ceil(2 * m);
-    if (hcap < 64) hcap = 64;
-    for (uint32_t p = tid; p < hcap; p += BUILD_NT) {
-      hk[p] = NONE;
-      hh[p] = NONE;
-    }
-    __syncthreads();
-    // (1) gather the round's op blocks (coalesced, independent loads)
-    for (uint32_t p = tid; p < m; p += BUILD_NT) {
-      const uint32_t gp = r0 + p;
-      uint32_t lo = 0, hi = ng;  // seg[lo] <= gp < seg[lo+1]
-      while (hi - lo > 1) {
-        const uint32_t mid = (lo + hi) >> 1;
-        if (seg[mid] <= gp) lo = mid;
-        else hi = mid;
+template <int MAXA, int MAXS>
+__global__ void __launch_bounds__(AP_NT) k_apply(BuildArgs a) {
+  constexpr int OWN_B = (MAXA * (1 + MAXS) <= 10) ? 2 : 1;  // sets loaded per owner batch
+  __shared__ uint32_t grp[GCAP], seg[GCAP + 1];
+  __shared__ unsigned long long goff[GCAP];
+  __shared__ uint32_t opb[AP_OPCAP], onx[AP_OPCAP], lnk[AP_OPCAP];
+  __shared__ uint32_t hk[AP_HCAP], hh[AP_HCAP];
+  __shared__ uint32_t ws[AP_NT / 32];
+  __shared__ uint32_t s_ng;
+  const Geo &g = a.g;
+  const uint32_t tid = threadIdx.x;
+  const uint32_t A = g.A, S = g.S;
+  // one CTA per item; the grid is the host's upper bound on the item count
+  const uint32_t t = blockIdx.x;
+  if (t >= *(volatile uint32_t *)&a.st->n_items) return;
+  uint32_t nsets = 0;
+  {
+    const uint2 it = a.items[t];
+    const uint32_t c = it.y & 0xFFFFu, P = it.y >> 16;
+    const LeadDesc d = a.desc[it.x];
+    const uint32_t e = d.e;
+    const unsigned long long t0 = a.clk ? gtimer() : 0;
+    uint32_t ng = 1;
+    if (d.single) {  // the common case: no list to chase
+      if (tid == 0) {
+        seg[0] = 0;
+        seg[1] = d.n_ops;
+        goff[0] = d.off_last;
       }
-      const uint64_t base = goff[lo] + (gp - seg[lo]);
-      uint32_t b = a.stage_norm[base];
-      if (!GUARD(a.st, b < g.W, b)) b = 0;
-      opb[p] = b;
-      // successor within the same launch: the next op, or past the round's end
-      // CLAIM marks "the next op of this round" (never a block id: ids < 2^20)
-      onx[p] = (gp + 1 < seg[lo + 1]) ? (p + 1 < m ? (uint32_t)CLAIM : a.stage_norm[base + 1]) : NONE;
-    }
-    __syncthreads();
-    // (2) link each op into its set's list
-    for (uint32_t p = tid; p < m; p += BUILD_NT) {
-      const uint32_t b = opb[p];
-      if (onx[p] == CLAIM) onx[p] = opb[p + 1];
-      const uint32_t key = row_of(g, b);
-      uint32_t sl = hslot(key, hcap);
-      for (;;) {
-        const uint32_t old = atomicCAS(&hk[sl], NONE, key);
-        if (old == NONE || old == key) break;
-        sl = (sl + 1) & (hcap - 1);
-      }
-      sorted_link(p, sl, hh, U + 2 * HCAPMAX + 2 * OPCAP);
-    }
-    __syncthreads();
-  if (a.cta_clk && tid == 0) a.cta_clk[10 * j + 4] = gtimer();
-    uint32_t *lnk = U + 2 * HCAPMAX + 2 * OPCAP;  // per-op next pointer of its set list
-    uint32_t nsets = 0;
-    for (uint32_t k0 = tid; k0 < hcap; k0 += BUILD_NT * OWN_B) {
-      RegSet<MAXA, MAXS> rs[OWN_B];
-      uint32_t sid[OWN_B], head[OWN_B];
-#pragma unroll
-      for (int q = 0; q < OWN_B; ++q) {  // issue every set load of the batch first
-        const uint32_t k = k0 + q * BUILD_NT;
-        sid[q] = k < hcap ? hk[k] : NONE;
-        head[q] = k < hcap ? hh[k] : NONE;
-        if (sid[q] != NONE) rs[q].load(tbl_e + (uint64_t)sid[q] * g.stride, A, S);
-      }
-#pragma unroll
-      for (int q = 0; q < OWN_B; ++q) {
-        if (sid[q] == NONE) continue;
-        ++nsets;
-        // the set's ops in position order: repeatedly take the smallest
-        // remaining position from the (short) list
-        uint32_t last = 0xFFFFFFFFu;
-        for (;;) {
-          uint32_t best = NONE;
-          for (uint32_t x = head[q]; x != NONE; x = lnk[x])
-            if ((last == 0xFFFFFFFFu || x > last) && (best == NONE || x < best)) best = x;
-          if (best == NONE) break;
-          if (!GUARD(a.st, best < m, best)) break;
-          rs[q].touch(opb[best], A);
-          if (onx[best] != NONE) rs[q].insert0(onx[best], S);
-          last = best;
-        }
-        rs[q].store(tbl_e + (uint64_t)sid[q] * g.stride, A, S);
-        if (use_rc) {
-          // row cache for the walk: final rows of the latest launch's blocks
-          for (uint32_t x = head[q]; x != NONE; x = lnk[x]) {
-            if (r0 + x < last_seg) continue;
-            const uint32_t i = r0 + x - last_seg;
-            if (!GUARD(a.st, i < n && (i + 1) * (1 + S) <= RCCAP, i)) continue;
-            rs[q].export_row(opb[x], A, S, rc + i * (1 + S));
-          }
-        }
-      }
-    }
-    if (nsets) atomicAdd(&s_sets, nsets);
-    __syncthreads();
-  }
-  if (tid == 0) {
-    ctr_add(a.st, DUM_CTR_EXEC_BUILT, 1);
-    ctr_add(a.st, DUM_CTR_OPS, n_ops);
-    ctr_add(a.st, DUM_CTR_SETS, s_sets);
-  }
-  if (a.cta_clk && tid == 0) a.cta_clk[10 * j + 5] = gtimer();
-  // ---- Start / End from the latest launch (D11) ----
-  const uint32_t *C = a.stage_norm + a.stage_off[Llast];
-  const uint32_t start = C[0], end = C[n - 1];
-  if (tid == 0) {
-    a.start_end[2 * e] = start;
-    a.start_end[2 * e + 1] = end;
-  }
-  uint32_t *wout = a.walk + (uint64_t)e * g.walk_cap;
-  if (n == 1) {  // x == End: the walk is [Start]
-    if (tid == 0) {
-      wout[0] = start;
-      a.walk_len[e] = 1;
-      reinterpret_cast<uint2 *>(a.wrun)[(uint64_t)e * g.walk_cap] = make_uint2(start >> 5, 1u << (start & 31));
-      a.wrun_len[e] = 1;
-      ctr_add(a.st, DUM_CTR_WALK_OUT, 1);
-    }
-    return;
-  }
-  // row i of the chain: pointer to its successor list (row cache or table)
-  // and its successor count; NONE count = row missing
-  auto row_at = [&](uint32_t i, const uint32_t *&sc) -> uint32_t {
-    if (use_rc) {
-      sc = rc + i * (1 + S) + 1;
-      DCHECK(rc[i * (1 + S)] == NONE || rc[i * (1 + S)] <= S, "rc[%u]=%x n=%u e=%u\n", i, rc[i * (1 + S)], n, e);
-      return rc[i * (1 + S)];
-    }
-    const uint32_t x = C[i];
-    const uint32_t *set = tbl_e + (uint64_t)row_of(g, x) * g.stride;
-    int w = -1;
-    for (uint32_t q = 0; q < A; ++q)
-      if (w < 0 && __ldcg(set + q * (1 + S)) == x) w = (int)q;
-    if (w < 0) return NONE;
-    sc = set + w * (1 + S) + 1;
-    uint32_t cnt = 0;
-    while (cnt < S && __ldcg(sc + cnt) != NONE) ++cnt;
-    return cnt;
-  };
-
-  // ---- pass A: per chain position i < n-1: row present? stop? successor count ----
-  uint32_t *cq;
-  // without the row cache, [rc, end of U) is free for the walk's arrays
-  const uint32_t free_words = RCCAP + WCAP + apply_union_words(R);
-  const uint32_t cq_words = (n + 31) & ~31u;
-  if (n <= WCAP) {
-    cq = use_rc ? cqs : rc;
-  } else if (!use_rc && cq_words + 2 * 1024 <= free_words) {
-    cq = rc;
-  } else {
-    if (tid == 0) {
-      const unsigned long long off = atomicAdd(&a.st->pool_big, (unsigned long long)n);
-      s_flag = off + n <= a.big_entries * 2 ? 0u : 1u;
-      s_tev = (uint32_t)off;
-    }
-    __syncthreads();
-    if (s_flag) {
-      if (tid == 0) a.slow_list[atomicAdd(&a.st->n_slow, 1u)] = e;
-      return;
-    }
-    cq = a.big_pool + s_tev;
-    __syncthreads();
-  }
-  if (tid == 0) s_tev = NONE;
-  __syncthreads();
-  for (uint32_t i = tid; i < n - 1; i += BUILD_NT) {
-    const uint32_t *sc = nullptr;
-    const uint32_t cnt = row_at(i, sc);
-    uint32_t ev = 0;
-    if (cnt == NONE) {
-      ev = 1;  // row missing: stop, nothing emitted at this step
-      cq[i] = 0;
+      __syncthreads();
     } else {
-      bool hit = false;
-      for (uint32_t q = 0; q < cnt; ++q) hit |= sc[q] == end;
-      if (hit) ev = 2;                                   // a successor is End: stop after emitting
-      else if (cnt == 0 || sc[0] != C[i + 1]) ev = 3;    // speculation violated -> sequential walker
-      cq[i] = cnt;
+      ng = load_group(a, d.j, e, grp, seg, goff, hk, &s_ng, AP_NT);
     }
-    if (ev) atomicMin(&s_tev, (i << 2) | ev);
+    const uint32_t n_ops = seg[ng];
+    __syncthreads();  // every thread has read s_ng (load_group)
+    if (tid == 0) s_ng = 0;  // from here on: the CTA's set count
+    uint32_t *tbl_e = a.tbl + (uint64_t)e * g.R * g.stride;
+    uint32_t m = 0;  // selected operations staged in opb / onx (uniform)
+    for (uint32_t g0 = 0; g0 < n_ops; g0 += AP_SCAN) {
+      // ---- select this partition's operations of [g0, g0 + AP_SCAN), in order ----
+#pragma unroll
+      for (uint32_t u = 0; u < AP_SCAN / AP_NT; ++u) {
+        const uint32_t gu = g0 + u * AP_NT, gp = gu + tid;
+        bool sel = false;
+        uint32_t b = NONE, nx = NONE;
+        if (gp < n_ops) {
+          uint32_t lo = 0, hi = ng;  // seg[lo] <= gp < seg[lo+1]
+          while (hi - lo > 1) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (seg[mid] <= gp) lo = mid;
+            else hi = mid;
+          }
+          const uint64_t base = goff[lo] + (gp - seg[lo]);
+          b = a.stage_norm[base];
+          if (!GUARD(a.st, b < g.W, b)) b = 0;
+          sel = P == 1 || ((row_of(g, b) >> 5) % P) == c;
+          // INSERT target: the next fault of the same launch
+          if (sel && gp + 1 < seg[lo + 1]) nx = a.stage_norm[base + 1];
+        }
+        uint32_t pre, tot;
+        if (P == 1) {  // every operation is selected: positions are known
+          pre = tid;
+          tot = n_ops > gu ? min((uint32_t)AP_NT, n_ops - gu) : 0u;
+        } else {
+          pre = block_excl_scan(sel ? 1u : 0u, ws, &tot);
+        }
+        if (sel) {
+          opb[m + pre] = b;
+          onx[m + pre] = nx;
+        }
+        m += tot;
+      }
+      if (m + AP_SCAN <= AP_OPCAP && g0 + AP_SCAN < n_ops) continue;
+      if (m == 0) continue;  // uniform: nothing of this partition in the range
+      // ---- apply the staged operations: grouped by set, one owner per set ----
+      uint32_t hcap = pow2ceil(2 * m);
+      if (hcap < 64) hcap = 64;
+      __syncthreads();
+      for (uint32_t p = tid; p < hcap; p += AP_NT) {
+        hk[p] = NONE;
+        hh[p] = NONE;
+      }
+      __syncthreads();
+      for (uint32_t p = tid; p < m; p += AP_NT) {
+        const uint32_t key = row_of(g, opb[p]);
+        uint32_t sl = hslot(key, hcap);
+        for (;;) {
+          const uint32_t old = atomicCAS(&hk[sl], NONE, key);
+          if (old == NONE || old == key) break;
+          sl = (sl + 1) & (hcap - 1);
+        }
+        lnk[p] = atomicExch(&hh[sl], p);
+      }
+      __syncthreads();
+      for (uint32_t k0 = tid; k0 < hcap; k0 += AP_NT * OWN_B) {
+        RegSet<MAXA, MAXS> rs[OWN_B];
+        uint32_t sid[OWN_B], hd[OWN_B];
+#pragma unroll
+        for (int q = 0; q < OWN_B; ++q) {  // issue every set load of the batch first
+          const uint32_t k = k0 + q * AP_NT;
+          sid[q] = k < hcap ? hk[k] : NONE;
+          hd[q] = k < hcap ? hh[k] : NONE;
+          if (sid[q] != NONE) rs[q].load(tbl_e + (uint64_t)sid[q] * g.stride, A, S);
+        }
+#pragma unroll
+        for (int q = 0; q < OWN_B; ++q) {
+          if (sid[q] == NONE) continue;
+          ++nsets;
+          // the set's operations in position order: repeatedly take the
+          // smallest remaining position from the (short) list
+          uint32_t last = 0xFFFFFFFFu;
+          for (;;) {
+            uint32_t best = NONE;
+            for (uint32_t x = hd[q]; x != NONE; x = lnk[x])
+              if ((last == 0xFFFFFFFFu || x > last) && (best == NONE || x < best)) best = x;
+            if (best == NONE) break;
+            if (!GUARD(a.st, best < m, best)) break;
+            rs[q].touch(opb[best], A);
+            if (onx[best] != NONE) rs[q].insert0(onx[best], S);
+            last = best;
+          }
+          rs[q].store(tbl_e + (uint64_t)sid[q] * g.stride, A, S);
+        }
+      }
+      __syncthreads();
+      m = 0;
+    }
+    if (a.clk && tid == 0) {
+      unsigned long long *c4 = a.clk + 4ull * t;
+      c4[0] = t0;
+      c4[1] = gtimer();
+      c4[2] = smid() | ((unsigned long long)blockIdx.x << 32);
+      c4[3] = n_ops | ((unsigned long long)P << 32);
+    }
   }
+  // one global atomic per CTA (a per-thread atomic on one address serialises
+  // hundreds of thousands of updates in L2)
+  nsets = __reduce_add_sync(0xffffffffu, nsets);
+  if ((tid & 31) == 0 && nsets) atomicAdd(&s_ng, nsets);
   __syncthreads();
-  if (a.cta_clk && tid == 0) a.cta_clk[10 * j + 6] = gtimer();
-  const uint32_t tev = s_tev;
-  if (tev == NONE || (tev & 3) == 3) {
-    if (tid == 0) a.slow_list[atomicAdd(&a.st->n_slow, 1u)] = e;
-    return;
-  }
-  const uint32_t t = tev >> 2;
-  if (!GUARD(a.st, t + 1 < n, t)) {
-    if (tid == 0) a.slow_list[atomicAdd(&a.st->n_slow, 1u)] = e;
-    return;
-  }
-  // ---- pass B: Q positions (qpos[i] = 1 + sum cq[0..i)) in place ----
-  uint32_t run = 1;
-  for (uint32_t c = 0; c <= t; c += BUILD_NT) {
-    const uint32_t i = c + tid;
-    const uint32_t v = i <= t ? cq[i] : 0;
-    uint32_t tot;
-    const uint32_t pre = block_excl_scan(v, ws, &tot);
-    if (i <= t) cq[i] = run + pre;
-    run += tot;
-  }
-  if (a.cta_clk && tid == 0) a.cta_clk[10 * j + 7] = gtimer();
-  const uint32_t qlen = run;  // |Q|
-  if (!GUARD(a.st, qlen <= 1 + (t + 1) * S, qlen)) {
-    if (tid == 0) a.slow_list[atomicAdd(&a.st->n_slow, 1u)] = e;
-    return;
-  }
-  // dedupe map block -> min Q position
-  uint32_t *qk, *qv;
-  const uint32_t qcap = pow2ceil(2 * qlen);
-  const bool cq_in_rc = cq == rc;
-  if (use_rc && qcap <= QCAP) {
-    qk = U;
-    qv = qk + qcap;
-  } else if (!use_rc && (cq_in_rc ? cq_words : 0) + 2 * qcap <= free_words) {
-    qk = rc + (cq_in_rc ? cq_words : 0);
-    qv = qk + qcap;
-  } else {
+  if (tid == 0 && s_ng) ctr_add(a.st, DUM_CTR_SETS, s_ng);
+}
+
+// ---------------------------------------------------------------------------
+// k_walk
+// ---------------------------------------------------------------------------
+// Parallel WALK(e, NONE) after the build (D13).  Let C = the latest faulting
+// launch of e in this batch (deduplicated, n = |C|); then Start = C[0], End =
+// C[n-1] (D11).  After the build, the row of C[i] (if still present) has
+// C[i+1] as its MRU successor: INSERT(C[i] -> C[i+1]) was the last operation
+// on that row, because C is duplicate-free and no later launch of e is in the
+// batch.  C[i+1] is not among the chained nodes C[0..i], so the sequential
+// walk's next chain node is exactly C[i+1] until the first i at which the row
+// is missing or a successor equals End.  With t that index, the walk is the
+// first-occurrence dedupe of
+//   Q = [C[0]] ++ succ(row C[0]) ++ ... ++ succ(row C[t])   (row C[t] only if
+//                                                            present).
+// The speculation is still verified (succ[0] == C[i+1]); any violation sends e
+// to the sequential walker.
+//
+// Pass A reads the rows of C from the table into a row cache (shared memory,
+// or a global scratch for long walks); pass B places the rows' successor
+// lists in Q; a min-position hash keeps first occurrences; pass C compacts
+// them in order and groups them into bitmap runs for k_predict.
+template <int MAXA, int MAXS>
+__global__ void __launch_bounds__(WK_NT) k_walk(BuildArgs a) {
+  extern __shared__ uint32_t sm[];
+  __shared__ uint32_t ws[WK_NT / 32];
+  __shared__ uint32_t s_tev, s_flag, s_off, s_nrun, s_multi;
+  uint32_t *src = sm, *scq = sm + WK_RC, *sqk = scq + WK_CQ;  // row cache | chain positions | hash
+  const Geo &g = a.g;
+  const uint32_t tid = threadIdx.x;
+  const uint32_t A = g.A, S = g.S;
+  // one CTA per exec ID; the grid is the host's upper bound (staged launches)
+  const uint32_t li = blockIdx.x;
+  if (li >= *(volatile uint32_t *)&a.st->n_leads) return;
+  do {  // (breaks = the early ends of the walk)
+    const LeadDesc d = a.desc[li];
+    const uint32_t e = d.e;
+    const uint32_t n = d.n_last;
+    const uint64_t off = d.off_last;
+    const uint32_t *C = a.stage_norm + off;
+    const uint32_t start = C[0], end = C[n - 1];
+    unsigned long long *c4 = a.clk ? a.clk + 4ull * (a.st->n_items + li) : nullptr;
+    if (c4 && tid == 0) {
+      c4[0] = gtimer();
+      c4[2] = smid() | ((unsigned long long)blockIdx.x << 32);
+      c4[3] = n;
+    }
     if (tid == 0) {
-      const unsigned long long off = atomicAdd(&a.st->pool_big, 2ull * qcap);
-      s_flag = off + 2ull * qcap <= a.big_entries * 2 ? 0u : 1u;
-      s_tev = (uint32_t)off;
+      a.start_end[2 * e] = start;
+      a.start_end[2 * e + 1] = end;
+      ctr_add(a.st, DUM_CTR_EXEC_BUILT, 1);
+      ctr_add(a.st, DUM_CTR_OPS, d.n_ops);
+      // the group bookkeeping of this batch is consumed (prep, plan and apply are done)
+      a.head[e] = NONE;
+      a.e_ops[e] = 0;
+      a.e_last[e] = 0;
+      s_tev = NONE;
+      s_nrun = 0;
+      s_multi = NONE;
+    }
+    uint32_t *wout = a.walk + (uint64_t)e * g.walk_cap;
+    uint2 *wrun = reinterpret_cast<uint2 *>(a.wrun) + (uint64_t)e * g.walk_cap;
+    if (n == 1) {  // x == End: the walk is [Start]
+      if (tid == 0) {
+        wout[0] = start;
+        a.walk_len[e] = 1;
+        wrun[0] = make_uint2(start >> 5, 1u << (start & 31));
+        a.wrun_len[e] = 1;
+        ctr_add(a.st, DUM_CTR_WALK_OUT, 1);
+        if (c4) c4[1] = gtimer();
+      }
+      break;
+    }
+    // ---- scratch: shared memory, else the global pools ----
+    const uint32_t rw = 1 + S;
+    uint32_t *rc = n * rw <= WK_RC ? src : a.rowc + off * rw;
+    uint32_t *cq = scq;
+    if (n > WK_CQ) {
+      if (tid == 0) {
+        const unsigned long long o = atomicAdd(&a.st->pool_big, (unsigned long long)n);
+        s_flag = o + n <= a.big_entries * 2 ? 0u : 1u;
+        s_off = (uint32_t)o;
+      }
+      __syncthreads();
+      if (s_flag) {
+        if (tid == 0) a.slow_list[atomicAdd(&a.st->n_slow, 1u)] = e;
+        break;
+      }
+      cq = a.big_pool + s_off;
     }
     __syncthreads();
-    if (s_flag) {
-      if (tid == 0) a.slow_list[atomicAdd(&a.st->n_slow, 1u)] = e;
-      return;
-    }
-    qk = a.big_pool + s_tev;
-    qv = qk + qcap;
-  }
-  for (uint32_t p = tid; p < qcap; p += BUILD_NT) {
-    qk[p] = NONE;
-    qv[p] = NONE;
-  }
-  __syncthreads();
-  if (tid == 0) hmap_insert_min(qk, qv, qcap, start, 0);
-  for (uint32_t i = tid; i <= t; i += BUILD_NT) {
-    const uint32_t q0 = cq[i];
-    const uint32_t qn = (i < t ? cq[i + 1] : qlen) - q0;
-    if (qn == 0) continue;
-    const uint32_t *sc = nullptr;
-    row_at(i, sc);
-    for (uint32_t q = 0; q < qn; ++q) hmap_insert_min(qk, qv, qcap, sc[q], q0 + q);
-  }
-  __syncthreads();
-  if (a.cta_clk && tid == 0) a.cta_clk[10 * j + 8] = gtimer();
-  // ---- pass C: ordered compaction of first occurrences ----
-  // The kept blocks of each warp step are also grouped by bitmap word into
-  // runs (word, mask) for k_predict (any grouping that puts every block in
-  // exactly one run will do; runs of one walk are disjoint).
-  uint32_t outn = 0;
-  uint2 *wrun = reinterpret_cast<uint2 *>(a.wrun) + (uint64_t)e * g.walk_cap;
-  if (tid == 0) s_nrun = 0;
-  for (uint32_t c = 0; c < qlen; c += BUILD_NT) {
-    const uint32_t p = c + tid;
-    uint32_t val = NONE, keep = 0;
-    if (p < qlen) {
-      if (p == 0) {
-        val = start;
+    // ---- pass A: rows of C[0 .. n-2] -> row cache; stop events ----
+    const uint32_t *tbl_e = a.tbl + (uint64_t)e * g.R * g.stride;
+    for (uint32_t i = tid; i < n - 1; i += WK_NT) {
+      RegSet<MAXA, MAXS> rs;
+      rs.load(tbl_e + (uint64_t)row_of(g, C[i]) * g.stride, A, S);
+      uint32_t *row = rc + i * rw;
+      rs.export_row(C[i], A, S, row);
+      const uint32_t cnt = row[0];
+      uint32_t ev = 0;
+      if (cnt == NONE) {
+        ev = 1;  // row missing: stop, nothing emitted at this step
+        cq[i] = 0;
       } else {
-        uint32_t lo = 0, hi = t + 1;  // largest lo with cq[lo] <= p
-        while (hi - lo > 1) {
-          const uint32_t mid = (lo + hi) >> 1;
-          if (cq[mid] <= p) lo = mid;
-          else hi = mid;
-        }
-        const uint32_t *sc = nullptr;
-        const uint32_t cnt_lo = row_at(lo, sc);
-        val = GUARD(a.st, cnt_lo != NONE && p - cq[lo] < cnt_lo, (lo << 16) | (p - cq[lo])) ? sc[p - cq[lo]] : start;
+        bool hit = false;
+        for (uint32_t q = 0; q < cnt; ++q) hit |= row[1 + q] == end;
+        if (hit) ev = 2;                                  // a successor is End: stop after emitting
+        else if (cnt == 0 || row[1] != C[i + 1]) ev = 3;  // speculation violated -> sequential walker
+        cq[i] = cnt;
+        if (cnt > 1) atomicMin(&s_multi, i);
       }
-      keep = hmap_get(qk, qv, qcap, val) == p;
+      if (ev) atomicMin(&s_tev, (i << 2) | ev);
     }
-    uint32_t tot;
-    const uint32_t pre = block_excl_scan(keep, ws, &tot);
-    if (keep && outn + pre < g.walk_cap) wout[outn + pre] = val;
-    {
-      const uint32_t lane = tid & 31;
-      const uint32_t wkey = keep ? val >> 5 : NONE;
-      const uint32_t grp = __match_any_sync(0xffffffffu, wkey);
-      const uint32_t msk = __reduce_or_sync(grp, keep ? 1u << (val & 31) : 0u);
-      const bool lead = keep && lane == (uint32_t)(__ffs(grp) - 1);
-      const uint32_t lm = __ballot_sync(0xffffffffu, lead);
-      uint32_t rb = 0;
-      if (lane == 0 && lm) rb = atomicAdd(&s_nrun, (uint32_t)__popc(lm));
-      rb = __shfl_sync(0xffffffffu, rb, 0) + __popc(lm & ((1u << lane) - 1));
-      if (lead && rb < g.walk_cap) wrun[rb] = make_uint2(wkey, msk);
+    __syncthreads();
+    const uint32_t tev = s_tev;
+    const uint32_t t = tev >> 2;
+    if (tev == NONE || (tev & 3) == 3 || !GUARD(a.st, t + 1 < n, t)) {
+      if (tid == 0) a.slow_list[atomicAdd(&a.st->n_slow, 1u)] = e;
+      break;
     }
-    outn += tot;
-  }
-  __syncthreads();  // every warp's run count is in s_nrun
-  if (tid == 0) {
-    if (outn > g.walk_cap) set_err(a.st, ERR_ECAPACITY, outn);
-    a.walk_len[e] = outn;
-    a.wrun_len[e] = s_nrun;
-    ctr_add(a.st, DUM_CTR_WALK_ROWS, t + 1);
-    ctr_add(a.st, DUM_CTR_WALK_OUT, outn);
-    if (a.cta_clk) {
-      a.cta_clk[10 * j] = t_begin;
-      a.cta_clk[10 * j + 1] = gtimer();
-      a.cta_clk[10 * j + 2] = (unsigned long long)n_ops | ((unsigned long long)n << 32);
+    if (s_multi > t) {
+      // ---- fast path: rows C[0..t] have the single successor C[i+1], so Q =
+      // C[0 .. t+1] (t+1 only when a successor is End), duplicate-free ----
+      const uint32_t qlen = t + 1 + ((tev & 3) == 2 ? 1u : 0u);
+      for (uint32_t c0 = 0; c0 < qlen; c0 += WK_NT) {
+        const uint32_t p = c0 + tid;
+        const bool keep = p < qlen;
+        const uint32_t val = keep ? C[p] : NONE;
+        if (keep && p < g.walk_cap) wout[p] = val;
+        const uint32_t lane = tid & 31;
+        const uint32_t wkey = keep ? val >> 5 : NONE;
+        const uint32_t gm = __match_any_sync(0xffffffffu, wkey);
+        const uint32_t msk = __reduce_or_sync(gm, keep ? 1u << (val & 31) : 0u);
+        const bool lead = keep && lane == (uint32_t)(__ffs(gm) - 1);
+        const uint32_t lm = __ballot_sync(0xffffffffu, lead);
+        uint32_t rb = 0;
+        if (lane == 0 && lm) rb = atomicAdd(&s_nrun, (uint32_t)__popc(lm));
+        rb = __shfl_sync(0xffffffffu, rb, 0) + __popc(lm & ((1u << lane) - 1));
+        if (lead && rb < g.walk_cap) wrun[rb] = make_uint2(wkey, msk);
+      }
+      __syncthreads();
+      if (tid == 0) {
+        if (qlen > g.walk_cap) set_err(a.st, ERR_ECAPACITY, qlen);
+        a.walk_len[e] = qlen;
+        a.wrun_len[e] = s_nrun;
+        ctr_add(a.st, DUM_CTR_WALK_ROWS, t + 1);
+        ctr_add(a.st, DUM_CTR_WALK_OUT, qlen);
+        if (c4) c4[1] = gtimer();
+      }
+      break;
     }
-  }
+    // ---- pass B: Q positions (qpos[i] = 1 + sum cq[0..i)) in place ----
+    uint32_t run = 1;
+    for (uint32_t c0 = 0; c0 <= t; c0 += WK_NT) {
+      const uint32_t i = c0 + tid;
+      const uint32_t v = i <= t ? cq[i] : 0;
+      uint32_t tot;
+      const uint32_t pre = block_excl_scan(v, ws, &tot);
+      if (i <= t) cq[i] = run + pre;
+      run += tot;
+    }
+    const uint32_t qlen = run;  // |Q|
+    if (!GUARD(a.st, qlen <= 1 + (t + 1) * S, qlen)) {
+      if (tid == 0) a.slow_list[atomicAdd(&a.st->n_slow, 1u)] = e;
+      break;
+    }
+    // ---- dedupe map block -> min Q position ----
+    const uint32_t qcap = pow2ceil(2 * qlen);
+    uint32_t *qk = sqk;
+    if (qcap > WK_QCAP) {
+      if (tid == 0) {
+        const unsigned long long o = atomicAdd(&a.st->pool_big, 2ull * qcap);
+        s_flag = o + 2ull * qcap <= a.big_entries * 2 ? 0u : 1u;
+        s_off = (uint32_t)o;
+      }
+      __syncthreads();
+      if (s_flag) {
+        if (tid == 0) a.slow_list[atomicAdd(&a.st->n_slow, 1u)] = e;
+        break;
+      }
+      qk = a.big_pool + s_off;
+    }
+    uint32_t *qv = qk + qcap;
+    for (uint32_t p = tid; p < qcap; p += WK_NT) {
+      qk[p] = NONE;
+      qv[p] = NONE;
+    }
+    __syncthreads();
+    if (tid == 0) hmap_insert_min(qk, qv, qcap, start, 0);
+    for (uint32_t i = tid; i <= t; i += WK_NT) {
+      const uint32_t q0 = cq[i];
+      const uint32_t qn = (i < t ? cq[i + 1] : qlen) - q0;
+      const uint32_t *sc = rc + i * rw + 1;
+      for (uint32_t q = 0; q < qn; ++q) hmap_insert_min(qk, qv, qcap, sc[q], q0 + q);
+    }
+    __syncthreads();
+    // ---- pass C: ordered compaction of first occurrences + bitmap runs ----
+    // The kept blocks of each warp step are grouped by bitmap word into runs
+    // (word, mask) for k_predict (any grouping that puts every block in exactly
+    // one run will do; runs of one walk are disjoint).
+    uint32_t outn = 0;
+    for (uint32_t c0 = 0; c0 < qlen; c0 += WK_NT) {
+      const uint32_t p = c0 + tid;
+      uint32_t val = NONE, keep = 0;
+      if (p < qlen) {
+        if (p == 0) {
+          val = start;
+        } else {
+          uint32_t lo = 0, hi = t + 1;  // largest lo with cq[lo] <= p
+          while (hi - lo > 1) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (cq[mid] <= p) lo = mid;
+            else hi = mid;
+          }
+          const uint32_t *row = rc + lo * rw;
+          val = GUARD(a.st, row[0] != NONE && p - cq[lo] < row[0], (lo << 16) | (p - cq[lo])) ? row[1 + p - cq[lo]]
+                                                                                            : start;
+        }
+        keep = hmap_get(qk, qv, qcap, val) == p;
+      }
+      uint32_t tot;
+      const uint32_t pre = block_excl_scan(keep, ws, &tot);
+      if (keep && outn + pre < g.walk_cap) wout[outn + pre] = val;
+      {
+        const uint32_t lane = tid & 31;
+        const uint32_t wkey = keep ? val >> 5 : NONE;
+        const uint32_t gm = __match_any_sync(0xffffffffu, wkey);
+        const uint32_t msk = __reduce_or_sync(gm, keep ? 1u << (val & 31) : 0u);
+        const bool lead = keep && lane == (uint32_t)(__ffs(gm) - 1);
+        const uint32_t lm = __ballot_sync(0xffffffffu, lead);
+        uint32_t rb = 0;
+        if (lane == 0 && lm) rb = atomicAdd(&s_nrun, (uint32_t)__popc(lm));
+        rb = __shfl_sync(0xffffffffu, rb, 0) + __popc(lm & ((1u << lane) - 1));
+        if (lead && rb < g.walk_cap) wrun[rb] = make_uint2(wkey, msk);
+      }
+      outn += tot;
+    }
+    __syncthreads();  // every warp's run count is in s_nrun
+    if (tid == 0) {
+      if (outn > g.walk_cap) set_err(a.st, ERR_ECAPACITY, outn);
+      a.walk_len[e] = outn;
+      a.wrun_len[e] = s_nrun;
+      ctr_add(a.st, DUM_CTR_WALK_ROWS, t + 1);
+      ctr_add(a.st, DUM_CTR_WALK_OUT, outn);
+      if (c4) c4[1] = gtimer();
+    }
+  } while (false);
 }
 
 __global__ void k_walk_slow(Geo g, const uint32_t *tbl, const uint32_t *start_end, uint32_t *walk,
@@ -674,7 +771,7 @@ __global__ void k_walk_slow(Geo g, const uint32_t *tbl, const uint32_t *start_en
       walk_len[e] = n;
     }
     __syncwarp();
-    // bitmap runs of the new walk (see pass C of k_apply_walk)
+    // bitmap runs of the new walk (see pass C of k_walk)
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t *w = walk + (uint64_t)e * g.walk_cap;
     uint2 *out = reinterpret_cast<uint2 *>(wrun) + (uint64_t)e * g.walk_cap;
@@ -696,35 +793,31 @@ __global__ void k_walk_slow(Geo g, const uint32_t *tbl, const uint32_t *start_en
   }
 }
 
+
 template <int MA, int MS>
-static cudaError_t launch_apply(dum_engine *e, const BuildArgs &ba, cudaStream_t s) {
-  const size_t smem = (size_t)(2 * GCAP + 1 + RCCAP + WCAP + apply_union_words(ba.g.R)) * 4;
-  cudaFuncSetAttribute(k_apply_walk<MA, MS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  cudaFuncSetAttribute(k_apply_walk<MA, MS>, cudaFuncAttributePreferredSharedMemoryCarveout,
-                       cudaSharedmemCarveoutMaxShared);
-  k_apply_walk<MA, MS><<<3 * ba.n_staged, BUILD_NT, smem, s>>>(ba);
+static cudaError_t launch_apply_walk(dum_engine *e, const BuildArgs &ba, cudaStream_t s) {
+  static bool init = false;
+  const size_t wsmem = (size_t)(WK_RC + WK_CQ + 2 * WK_QCAP) * 4;
+  if (!init) {
+    cudaFuncSetAttribute(k_walk<MA, MS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)wsmem);
+    init = true;
+  }
+  // host upper bounds of the device-side counts (the surplus CTAs return at once):
+  // items = sum over exec IDs of ceil(ops / OPP) <= launches + faults / OPP
+  const uint32_t n_items_max = (uint32_t)std::min<uint64_t>(e->items_cap, e->n_staged + e->staged_faults / OPP + 1);
+  {
+    TimerScope t(e, DUM_T_APPLY_WALK, s);
+    k_apply<MA, MS><<<n_items_max, AP_NT, 0, s>>>(ba);
+  }
+  TimerScope t(e, DUM_T_WALK, s);
+  k_walk<MA, MS><<<e->n_staged, WK_NT, wsmem, s>>>(ba);
   return cudaGetLastError();
 }
 
 cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   const uint32_t n = e->n_staged;
   if (n == 0) return cudaSuccess;
-  {
-  TimerScope t(e, DUM_T_BUILD_PREP, s);
-  cudaMemsetAsync(e->d_state->cls_cnt, 0, sizeof(e->d_state->cls_cnt), s);
-  k_build_prep<<<(n + 255) / 256, 256, 0, s>>>(n, (uint32_t)e->built_launches, e->d_stage_exec, e->d_stage_cnt,
-                                                e->d_corr, e->corr_cap, e->d_rec_slot, e->d_head, e->d_next,
-                                                e->d_order,
-                                                e->d_state);
-  }
-  // the jump tables depend only on the correlation table, final here
-  cudaEventRecord(e->ev_fork, s);
-  cudaStreamWaitEvent(e->side, e->ev_fork, 0);
-  {
-    const cudaError_t je = launch_jump_tables(e, e->side);
-    cudaEventRecord(e->ev_join, e->side);
-    if (je != cudaSuccess) return je;
-  }
+  cudaStreamWaitEvent(s, e->ev_join, 0);  // the previous build's jump tables read corr
   BuildArgs ba;
   ba.g = e->g;
   ba.n_staged = n;
@@ -734,10 +827,15 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   ba.stage_off = e->d_stage_off;
   ba.head = e->d_head;
   ba.next = e->d_next;
+  ba.e_ops = e->d_e_ops;
+  ba.e_last = e->d_e_last;
+  ba.desc = reinterpret_cast<LeadDesc *>(e->d_lead);
+  ba.items = reinterpret_cast<uint2 *>(e->d_items);
   ba.tbl = e->d_tbl;
   ba.start_end = e->d_start_end;
   ba.walk = e->d_walk;
   ba.walk_len = e->d_walk_len;
+  ba.rowc = e->d_rowc;
   ba.big_pool = e->d_big_pool;
   ba.big_entries = e->big_pool_entries;
   ba.slow_list = e->d_slow_list;
@@ -745,24 +843,42 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   ba.wrun_len = e->d_wrun_len;
   ba.order = e->d_order;
   ba.st = e->d_state;
-  ba.cta_clk = nullptr;
-  static const char *clk_path = getenv("DUM_CTA_CLOCK");
+  ba.clk = nullptr;
+  static const char *clk_path = getenv("DUM_BUILD_CLOCK");
   static unsigned long long *d_clk = nullptr;
   static int clk_calls = 0;
+  const uint64_t clk_n = 4ull * (e->items_cap + e->stage_launch_cap);
   if (clk_path) {
-    if (!d_clk) cudaMalloc(&d_clk, 10ull * 8 * e->stage_launch_cap);
-    cudaMemsetAsync(d_clk, 0, 10ull * 8 * n, s);
-    ba.cta_clk = d_clk;
+    if (!d_clk) cudaMalloc(&d_clk, 8 * clk_n);
+    cudaMemsetAsync(d_clk, 0, 8 * clk_n, s);
+    ba.clk = d_clk;
+  }
+  {
+    TimerScope t(e, DUM_T_BUILD_PREP, s);
+    cudaMemsetAsync(e->d_state->cls_cnt, 0, sizeof(e->d_state->cls_cnt), s);
+    k_build_prep<<<(n + 255) / 256, 256, 0, s>>>(n, (uint32_t)e->built_launches, e->d_stage_exec, e->d_stage_cnt,
+                                                  e->d_corr, e->corr_cap, e->d_rec_slot, e->d_head, e->d_next,
+                                                  e->d_order, e->d_e_ops, e->d_e_last, e->d_state);
+    k_plan<<<1, PLAN_NT, 0, s>>>(ba);
+  }
+  // the jump tables depend only on the correlation table, final here
+  static const char *jm = getenv("DUM_JUMP_MODE");
+  if (jm && jm[0] == '2') {
+    const cudaError_t je = launch_jump_tables(e, s);
+    if (je != cudaSuccess) return je;
+  } else {
+    cudaEventRecord(e->ev_fork, s);
+    cudaStreamWaitEvent(e->side, e->ev_fork, 0);
+    const cudaError_t je = launch_jump_tables(e, e->side);
+    cudaEventRecord(e->ev_join, e->side);
+    if (je != cudaSuccess) return je;
   }
   cudaError_t err;
-  {
-  TimerScope t(e, DUM_T_APPLY_WALK, s);
-  if (e->g.A <= 2 && e->g.S <= 4) err = launch_apply<2, 4>(e, ba, s);
-  else if (e->g.A == 2 && e->g.S == 8) err = launch_apply<2, 8>(e, ba, s);
-  else if (e->g.A == 4 && e->g.S == 4) err = launch_apply<4, 4>(e, ba, s);
-  else if (e->g.A <= 4 && e->g.S <= 8) err = launch_apply<4, 8>(e, ba, s);
-  else err = launch_apply<32, 32>(e, ba, s);
-  }
+  if (e->g.A <= 2 && e->g.S <= 4) err = launch_apply_walk<2, 4>(e, ba, s);
+  else if (e->g.A == 2 && e->g.S == 8) err = launch_apply_walk<2, 8>(e, ba, s);
+  else if (e->g.A == 4 && e->g.S == 4) err = launch_apply_walk<4, 4>(e, ba, s);
+  else if (e->g.A <= 4 && e->g.S <= 8) err = launch_apply_walk<4, 8>(e, ba, s);
+  else err = launch_apply_walk<32, 32>(e, ba, s);
   if (err != cudaSuccess) return err;
   WalkScratch ws{e->d_walk_seen, e->d_walk_chain, e->d_walk_tmp, e->walk_hash_cap,
                  e->g.walk_cap + e->g.R * e->g.A + 4};
@@ -771,10 +887,17 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
     k_walk_slow<<<e->n_walk_slots, 32, 0, s>>>(e->g, e->d_tbl, e->d_start_end, e->d_walk, e->d_walk_len,
                                                e->d_wrun, e->d_wrun_len, e->d_slow_list, ws, e->d_state);
   }
-  if (clk_path) {
-    std::vector<unsigned long long> h(10ull * n);
+  // no join here: the jump tables keep building on the side stream, past the
+  // end of this call; the next reader of the correlation table (predict's
+  // k_chain, the next build, reset) waits for ev_join
+  e->kernel_launches += 5;
+  if (clk_path) {  // [n_items | n_leads] header, then the stamps
+    DevState hs;
     cudaStreamSynchronize(s);
-    cudaMemcpy(h.data(), d_clk, 8ull * 10 * n, cudaMemcpyDeviceToHost);
+    cudaMemcpy(&hs, e->d_state, sizeof(hs), cudaMemcpyDeviceToHost);
+    std::vector<unsigned long long> h(4ull * (hs.n_items + hs.n_leads) + 1);
+    h[0] = hs.n_items | ((unsigned long long)hs.n_leads << 32);
+    cudaMemcpy(h.data() + 1, d_clk, 8 * (h.size() - 1), cudaMemcpyDeviceToHost);
     char fn[512];
     snprintf(fn, sizeof fn, "%s.%d", clk_path, clk_calls++);
     if (FILE *f = fopen(fn, "wb")) {
@@ -782,8 +905,6 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
       fclose(f);
     }
   }
-  cudaStreamWaitEvent(s, e->ev_join, 0);
-  e->kernel_launches += 3;
   return cudaGetLastError();
 }
 

@@ -8,7 +8,9 @@
 // the chain of a query whose first record is r0 is succ(next^d(r0)) for
 // d = 0, 1, ... until next^d(r0) is absent.  Rebuilt after every build on a
 // side stream (it only reads the correlation table) while the block tables
-// are applied.
+// are applied; the next reader of the correlation table waits for it.
+#include <algorithm>
+
 #include "corr.cuh"
 #include "device_util.cuh"
 #include "kernels.cuh"
@@ -40,10 +42,9 @@ __global__ void __launch_bounds__(JUMP_NT) k_jumpk(uint32_t cap, const uint32_t 
 }
 
 cudaError_t launch_jump_tables(dum_engine *e, cudaStream_t s) {
-  int dev = 0, sms = 148;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  const uint32_t grid = (uint32_t)sms * 4;
+  // records <= launches applied so far (one upsert each); the grid covers them
+  const uint64_t nrec = std::min<uint64_t>(e->built_launches + e->n_staged, e->corr_cap);
+  const uint32_t grid = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>((nrec + JUMP_NT - 1) / JUMP_NT, 4 * 148));
   TimerScope t(e, DUM_T_JUMP, s);
   k_jump0<<<grid, JUMP_NT, 0, s>>>(e->d_corr, e->corr_cap, e->d_rec_slot, e->d_jump, e->d_state);
   for (uint32_t k = 1; k < e->jump_levels; ++k)

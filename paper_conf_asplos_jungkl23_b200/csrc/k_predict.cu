@@ -108,7 +108,7 @@ struct PredArgs {
   uint32_t corr_cap;
   const uint32_t *jump;  // [levels][corr_cap]
   const uint32_t *walk, *walk_len;
-  const uint32_t *wrun, *wrun_len;  // walk bitmap runs (k_apply_walk pass C / k_walk_slow)
+  const uint32_t *wrun, *wrun_len;  // walk bitmap runs (k_walk pass C / k_walk_slow)
   const uint32_t *anchor_pool;
   const uint64_t *anchor_range;
   uint32_t *pairs;
@@ -771,6 +771,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
     cudaMemsetAsync(d_clk, 0, 12ull * 8 * nq, s);
     a.cta_clk = d_clk;
   }
+  cudaStreamWaitEvent(s, e->ev_join, 0);  // jump tables of the last build (side stream)
   {
     TimerScope t(e, DUM_T_CHAIN, s);
     k_chain<<<(nq + CHAIN_WARPS - 1) / CHAIN_WARPS, CHAIN_WARPS * 32, 0, s>>>(a);

@@ -2,7 +2,9 @@
    python tools/pred_clock.py <prefix>"""
 import sys, glob
 import numpy as np
-for fn in sorted(glob.glob(sys.argv[1] + ".*"), key=lambda x: int(x.rsplit(".", 1)[1]))[-1:]:
+_fs = sorted(glob.glob(sys.argv[1] + ".[0-9]*"), key=lambda x: int(x.rsplit(".", 1)[1]))
+_fs = [f for f in _fs if np.fromfile(f, dtype=np.uint64).reshape(-1, 12)[:, 0].max(initial=0) > 0]
+for fn in _fs[-2:-1] or _fs[-1:]:
     a = np.fromfile(fn, dtype=np.uint64).reshape(-1, 12)
     dup = (a[:, 6] >> np.uint64(63)).astype(bool)
     a6 = (a[:, 6] & np.uint64((1 << 63) - 1)).astype(np.int64)

@@ -8,7 +8,7 @@ from collections import defaultdict
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 tag = sys.argv[1]
-kernels = sys.argv[2:] or ["k_predict", "k_apply_walk", "k_chain", "k_ingest"]
+kernels = sys.argv[2:] or ["k_predict", "k_apply", "k_walk", "k_chain", "k_ingest"]
 out_dir = os.path.join(ROOT, "profiles")
 os.makedirs(out_dir, exist_ok=True)
 lines = ["# ncu summary `%s`" % tag, ""]
