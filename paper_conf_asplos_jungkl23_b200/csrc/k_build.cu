@@ -368,10 +368,9 @@ __global__ void __launch_bounds__(AP_NT) k_apply(BuildArgs a) {
   constexpr int OWN_B = (MAXA * (1 + MAXS) <= 10) ? 2 : 1;  // sets loaded per owner batch
   __shared__ uint32_t grp[GCAP], seg[GCAP + 1];
   __shared__ unsigned long long goff[GCAP];
-  __shared__ uint32_t opb[AP_OPCAP], onx[AP_OPCAP], lnk[AP_OPCAP];
+  __shared__ uint32_t opb[AP_OPCAP], onx[AP_OPCAP], opos[AP_OPCAP], lnk[AP_OPCAP], sll[AP_OPCAP];
   __shared__ uint32_t hk[AP_HCAP], hh[AP_HCAP];
-  __shared__ uint32_t ws[AP_NT / 32];
-  __shared__ uint32_t s_ng;
+  __shared__ uint32_t s_ng, s_m, s_nsl;
   const Geo &g = a.g;
   const uint32_t tid = threadIdx.x;
   const uint32_t A = g.A, S = g.S;
@@ -400,72 +399,45 @@ __global__ void __launch_bounds__(AP_NT) k_apply(BuildArgs a) {
     __syncthreads();  // every thread has read s_ng (load_group)
     if (tid == 0) s_ng = 0;  // from here on: the CTA's set count
     uint32_t *tbl_e = a.tbl + (uint64_t)e * g.R * g.stride;
-    uint32_t m = 0;  // selected operations staged in opb / onx (uniform)
-    for (uint32_t g0 = 0; g0 < n_ops; g0 += AP_SCAN) {
-      // ---- select this partition's operations of [g0, g0 + AP_SCAN), in order ----
-#pragma unroll
-      for (uint32_t u = 0; u < AP_SCAN / AP_NT; ++u) {
-        const uint32_t gu = g0 + u * AP_NT, gp = gu + tid;
-        bool sel = false;
-        uint32_t b = NONE, nx = NONE;
-        if (gp < n_ops) {
-          uint32_t lo = 0, hi = ng;  // seg[lo] <= gp < seg[lo+1]
-          while (hi - lo > 1) {
-            const uint32_t mid = (lo + hi) >> 1;
-            if (seg[mid] <= gp) lo = mid;
-            else hi = mid;
-          }
-          const uint64_t base = goff[lo] + (gp - seg[lo]);
-          b = a.stage_norm[base];
-          if (!GUARD(a.st, b < g.W, b)) b = 0;
-          sel = P == 1 || ((row_of(g, b) >> 5) % P) == c;
-          // INSERT target: the next fault of the same launch
-          if (sel && gp + 1 < seg[lo + 1]) nx = a.stage_norm[base + 1];
-        }
-        uint32_t pre, tot;
-        if (P == 1) {  // every operation is selected: positions are known
-          pre = tid;
-          tot = n_ops > gu ? min((uint32_t)AP_NT, n_ops - gu) : 0u;
-        } else {
-          pre = block_excl_scan(sel ? 1u : 0u, ws, &tot);
-        }
-        if (sel) {
-          opb[m + pre] = b;
-          onx[m + pre] = nx;
-        }
-        m += tot;
-      }
-      if (m + AP_SCAN <= AP_OPCAP && g0 + AP_SCAN < n_ops) continue;
-      if (m == 0) continue;  // uniform: nothing of this partition in the range
-      // ---- apply the staged operations: grouped by set, one owner per set ----
+    uint32_t m = 0;  // selected operations staged in opb / onx / opos (uniform)
+    // apply the staged operations: grouped by set through a shared hash, one
+    // owner thread per set applies the set's operations in position order
+    auto apply_staged = [&]() {
       uint32_t hcap = pow2ceil(2 * m);
       if (hcap < 64) hcap = 64;
-      __syncthreads();
       for (uint32_t p = tid; p < hcap; p += AP_NT) {
         hk[p] = NONE;
         hh[p] = NONE;
       }
+      if (tid == 0) s_nsl = 0;
       __syncthreads();
       for (uint32_t p = tid; p < m; p += AP_NT) {
         const uint32_t key = row_of(g, opb[p]);
         uint32_t sl = hslot(key, hcap);
         for (;;) {
           const uint32_t old = atomicCAS(&hk[sl], NONE, key);
+          if (old == NONE) sll[atomicAdd(&s_nsl, 1u)] = sl;  // a new set: list its slot
           if (old == NONE || old == key) break;
           sl = (sl + 1) & (hcap - 1);
         }
         lnk[p] = atomicExch(&hh[sl], p);
       }
       __syncthreads();
-      for (uint32_t k0 = tid; k0 < hcap; k0 += AP_NT * OWN_B) {
+      const uint32_t nsl = s_nsl;
+      for (uint32_t k0 = tid; k0 < nsl; k0 += AP_NT * OWN_B) {
         RegSet<MAXA, MAXS> rs[OWN_B];
         uint32_t sid[OWN_B], hd[OWN_B];
 #pragma unroll
         for (int q = 0; q < OWN_B; ++q) {  // issue every set load of the batch first
           const uint32_t k = k0 + q * AP_NT;
-          sid[q] = k < hcap ? hk[k] : NONE;
-          hd[q] = k < hcap ? hh[k] : NONE;
-          if (sid[q] != NONE) rs[q].load(tbl_e + (uint64_t)sid[q] * g.stride, A, S);
+          sid[q] = NONE;
+          hd[q] = NONE;
+          if (k < nsl) {
+            const uint32_t sl = sll[k];
+            sid[q] = hk[sl];
+            hd[q] = hh[sl];
+            rs[q].load(tbl_e + (uint64_t)sid[q] * g.stride, A, S);
+          }
         }
 #pragma unroll
         for (int q = 0; q < OWN_B; ++q) {
@@ -473,23 +445,82 @@ __global__ void __launch_bounds__(AP_NT) k_apply(BuildArgs a) {
           ++nsets;
           // the set's operations in position order: repeatedly take the
           // smallest remaining position from the (short) list
-          uint32_t last = 0xFFFFFFFFu;
+          uint32_t last = NONE;
           for (;;) {
-            uint32_t best = NONE;
-            for (uint32_t x = hd[q]; x != NONE; x = lnk[x])
-              if ((last == 0xFFFFFFFFu || x > last) && (best == NONE || x < best)) best = x;
+            uint32_t best = NONE, bpos = NONE;
+            for (uint32_t x = hd[q]; x != NONE; x = lnk[x]) {
+              const uint32_t px = opos[x];
+              if ((last == NONE || px > last) && (bpos == NONE || px < bpos)) {
+                best = x;
+                bpos = px;
+              }
+            }
             if (best == NONE) break;
             if (!GUARD(a.st, best < m, best)) break;
             rs[q].touch(opb[best], A);
             if (onx[best] != NONE) rs[q].insert0(onx[best], S);
-            last = best;
+            last = bpos;
           }
           rs[q].store(tbl_e + (uint64_t)sid[q] * g.stride, A, S);
         }
       }
       __syncthreads();
       m = 0;
+      if (tid == 0) s_m = 0;
+    };
+    if (tid == 0) s_m = 0;
+    __syncthreads();
+    for (uint32_t g0 = 0; g0 < n_ops; g0 += AP_SCAN) {
+      if (m + AP_SCAN > AP_OPCAP) apply_staged();  // a chunk never straddles two rounds
+      // ---- select this partition's operations of [g0, g0 + AP_SCAN) ----
+      // Per set, the operations must be applied in position order; across sets
+      // any order will do, so the selected ones are appended in any order with
+      // their position (P > 1), or in place (P == 1).
+      constexpr uint32_t U = AP_SCAN / AP_NT;
+      uint32_t b[U], nx[U], gp[U];
+      bool sel[U];
+#pragma unroll
+      for (uint32_t u = 0; u < U; ++u) {  // issue the loads first
+        gp[u] = g0 + u * AP_NT + tid;
+        b[u] = NONE;
+        nx[u] = NONE;
+        sel[u] = false;
+        if (gp[u] < n_ops) {
+          uint32_t lo = 0, hi = ng;  // seg[lo] <= gp < seg[lo+1]
+          while (hi - lo > 1) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (seg[mid] <= gp[u]) lo = mid;
+            else hi = mid;
+          }
+          const uint64_t base = goff[lo] + (gp[u] - seg[lo]);
+          b[u] = a.stage_norm[base];
+          // INSERT target: the next fault of the same launch
+          if (gp[u] + 1 < seg[lo + 1]) nx[u] = a.stage_norm[base + 1];
+        }
+      }
+#pragma unroll
+      for (uint32_t u = 0; u < U; ++u) {
+        if (gp[u] < n_ops) {
+          if (!GUARD(a.st, b[u] < g.W, b[u])) b[u] = 0;
+          sel[u] = P == 1 || ((row_of(g, b[u]) >> 5) % P) == c;
+        }
+        uint32_t slot = m + u * AP_NT + tid;
+        if (P != 1) {  // warp-aggregated append
+          const uint32_t lane = tid & 31, bal = __ballot_sync(0xffffffffu, sel[u]);
+          uint32_t base = 0;
+          if (lane == 0 && bal) base = atomicAdd(&s_m, (uint32_t)__popc(bal));
+          slot = __shfl_sync(0xffffffffu, base, 0) + __popc(bal & ((1u << lane) - 1));
+        }
+        if (sel[u]) {
+          opb[slot] = b[u];
+          onx[slot] = nx[u];
+          opos[slot] = gp[u];
+        }
+      }
+      __syncthreads();
+      m = P == 1 ? m + min(AP_SCAN, n_ops - g0) : s_m;
     }
+    if (m) apply_staged();
     if (a.clk && tid == 0) {
       unsigned long long *c4 = a.clk + 4ull * t;
       c4[0] = t0;
@@ -598,25 +629,40 @@ __global__ void __launch_bounds__(WK_NT) k_walk(BuildArgs a) {
     __syncthreads();
     // ---- pass A: rows of C[0 .. n-2] -> row cache; stop events ----
     const uint32_t *tbl_e = a.tbl + (uint64_t)e * g.R * g.stride;
-    for (uint32_t i = tid; i < n - 1; i += WK_NT) {
-      RegSet<MAXA, MAXS> rs;
-      rs.load(tbl_e + (uint64_t)row_of(g, C[i]) * g.stride, A, S);
-      uint32_t *row = rc + i * rw;
-      rs.export_row(C[i], A, S, row);
-      const uint32_t cnt = row[0];
-      uint32_t ev = 0;
-      if (cnt == NONE) {
-        ev = 1;  // row missing: stop, nothing emitted at this step
-        cq[i] = 0;
-      } else {
-        bool hit = false;
-        for (uint32_t q = 0; q < cnt; ++q) hit |= row[1 + q] == end;
-        if (hit) ev = 2;                                  // a successor is End: stop after emitting
-        else if (cnt == 0 || row[1] != C[i + 1]) ev = 3;  // speculation violated -> sequential walker
-        cq[i] = cnt;
-        if (cnt > 1) atomicMin(&s_multi, i);
+    constexpr int WB = (MAXA * (1 + MAXS) <= 10) ? 4 : 1;  // rows per thread in flight
+    for (uint32_t i0 = tid; i0 < n - 1; i0 += WK_NT * WB) {
+      uint32_t x[WB], xn[WB];
+      RegSet<MAXA, MAXS> rs[WB];
+#pragma unroll
+      for (int q = 0; q < WB; ++q) {  // issue every load of the batch first
+        const uint32_t i = i0 + q * WK_NT;
+        x[q] = i < n - 1 ? C[i] : NONE;
+        xn[q] = i < n - 1 ? C[i + 1] : NONE;
       }
-      if (ev) atomicMin(&s_tev, (i << 2) | ev);
+#pragma unroll
+      for (int q = 0; q < WB; ++q)
+        if (x[q] != NONE) rs[q].load(tbl_e + (uint64_t)row_of(g, x[q]) * g.stride, A, S);
+#pragma unroll
+      for (int q = 0; q < WB; ++q) {
+        if (x[q] == NONE) continue;
+        const uint32_t i = i0 + q * WK_NT;
+        uint32_t *row = rc + i * rw;
+        rs[q].export_row(x[q], A, S, row);
+        const uint32_t cnt = row[0];
+        uint32_t ev = 0;
+        if (cnt == NONE) {
+          ev = 1;  // row missing: stop, nothing emitted at this step
+          cq[i] = 0;
+        } else {
+          bool hit = false;
+          for (uint32_t k = 0; k < cnt; ++k) hit |= row[1 + k] == end;
+          if (hit) ev = 2;                              // a successor is End: stop after emitting
+          else if (cnt == 0 || row[1] != xn[q]) ev = 3;  // speculation violated -> sequential walker
+          cq[i] = cnt;
+          if (cnt > 1) atomicMin(&s_multi, i);
+        }
+        if (ev) atomicMin(&s_tev, (i << 2) | ev);
+      }
     }
     __syncthreads();
     const uint32_t tev = s_tev;
