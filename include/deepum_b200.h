@@ -119,7 +119,15 @@ int dum_reset(dum_engine *eng, dum_stream_t stream);
  * occurrence of each block per launch (P:L124 step 2; D2).  Exec IDs: same
  * hash -> same ID, else the next dense ID in first-seen order (D3);
  * written to out_exec[i] if out_exec != NULL (device).  Staged launches are
- * applied by the next dum_build_tables. */
+ * applied by the next dum_build_tables.  With DUM_HOST_PTRS the launch
+ * offsets are validated on the host (DUM_EINVAL); block ids >= max_blocks are
+ * detected on the device for both kinds of pointers (sticky DUM_EINVAL from
+ * dum_sync; the offending records are dropped).  DUM_HOST_PTRS uploads run on
+ * the engine's copy stream into one of two staging buffers (the upload of the
+ * next batch overlaps the kernels of this one) and `stream` waits for them:
+ * pinned host inputs must stay unmodified until the call's work on `stream`
+ * has completed, exactly like device inputs (pageable inputs are staged by
+ * the CUDA runtime before the call returns). */
 int dum_record_faults(dum_engine *eng, const uint64_t *launch_hash, const uint64_t *launch_off,
                       uint32_t n_launch, const uint32_t *fault_block, uint64_t n_fault,
                       uint32_t *out_exec, uint32_t flags, dum_stream_t stream);
@@ -318,6 +326,12 @@ const char *dum_last_error(const dum_engine *eng);
 /* Number of the library's own kernel launches issued so far (for bench
  * launch counting). */
 uint64_t dum_kernel_launches(const dum_engine *eng);
+
+/* Memory kind of a pointer as this library's CUDA runtime sees it
+ * (cudaMemoryType: 0 unregistered host, 1 pinned host, 2 device, 3 managed;
+ * -1 on error).  DUM_HOST_PTRS inputs should be pinned (1) for asynchronous
+ * full-bandwidth copies. */
+int dum_host_ptr_kind(const void *ptr);
 
 #ifdef __cplusplus
 }

@@ -98,6 +98,7 @@ def load_library() -> ctypes.CDLL:
         "dum_kernel_launches": (U64, [P]),
         "dum_read_counters": (I, [P, P, I]),
         "dum_set_timing": (I, [P, I]),
+        "dum_host_ptr_kind": (I, [P]),
         "dum_read_timing": (I, [P, P, P, I]),
     }
     for name, (res, args) in sig.items():

@@ -39,6 +39,8 @@ __global__ void k_init_state(DevState *st) {
   st->needed = 0;
   st->pool_pairs = st->pool_wb = st->pool_inv = st->pool_anchor = st->pool_big = 0;
   st->n_slow = 0;
+  st->n_pend = 0;
+  st->n_items = st->n_leads = 0;
   st->corr_used = 0;
   st->mig_ok = 0;
   st->mig_n = 0;
@@ -114,7 +116,7 @@ void free_all(dum_engine *e) {
                   e->d_start_end, e->d_walk, e->d_walk_len, e->d_in_hash, e->d_in_off, e->d_in_faults,
                   e->d_stage_hash, e->d_stage_norm, e->d_stage_cnt, e->d_stage_exec, e->d_stage_slot,
                   e->d_stage_off, e->d_head, e->d_next, e->d_order, e->d_slow_list,
-                  e->d_e_ops, e->d_e_last, e->d_lead, e->d_items, e->d_rowc, e->d_big_pool, e->d_walk_seen,
+                  e->d_e_ops, e->d_e_last, e->d_pend, e->d_lead, e->d_items, e->d_rowc, e->d_big_pool, e->d_walk_seen,
                   e->d_walk_chain, e->d_walk_tmp, e->d_walk_out, e->d_anchor_pool, e->d_anchor_range,
                   e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits, e->d_inactive_bits, e->d_res_bits, e->d_logpos, e->d_lrm_blk,
                   e->d_lrm_stamp, e->d_mig_frames, e->d_mig_src, e->d_mig_blocks, e->d_state, e->d_qkern,
@@ -122,8 +124,13 @@ void free_all(dum_engine *e) {
   for (void *p : ptrs)
     if (p) cudaFree(p);
   if (e->ev_fork) cudaEventDestroy(e->ev_fork);
+  for (int b = 0; b < 2; ++b) {
+    if (e->ev_in_ready[b]) cudaEventDestroy(e->ev_in_ready[b]);
+    if (e->ev_in_free[b]) cudaEventDestroy(e->ev_in_free[b]);
+  }
   if (e->ev_join) cudaEventDestroy(e->ev_join);
   if (e->side) cudaStreamDestroy(e->side);
+  if (e->copy_s) cudaStreamDestroy(e->copy_s);
   if (e->h_state) cudaFreeHost(e->h_state);
   for (auto &t : e->pending) {
     cudaEventDestroy(t.a);
@@ -244,12 +251,14 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_rec_slot, e->corr_cap));
   A_(dmalloc(&e->d_jump, (uint64_t)e->jump_levels * e->corr_cap));
   {
-    // the jump tables are on the critical path of the next predict and tiny:
-    // their CTAs go ahead of the block-table apply they overlap
+    // jump tables (k_jump.cu) overlap the block-table apply/walk here.  Normal
+    // priority: a high-priority side stream stalled the main stream by
+    // ~100 us per step when steps are issued back to back (measured,
+    // tools/e2e_diag.py); DUM_JUMP_MODE=0 restores it for experiments
     int lo = 0, hi = 0;
     cudaDeviceGetStreamPriorityRange(&lo, &hi);
     const char *jm = getenv("DUM_JUMP_MODE");
-    A_(cudaStreamCreateWithPriority(&e->side, cudaStreamNonBlocking, (jm && jm[0] == '1') ? lo : hi));
+    A_(cudaStreamCreateWithPriority(&e->side, cudaStreamNonBlocking, (jm && jm[0] == '0') ? hi : lo));
   }
   A_(cudaEventCreateWithFlags(&e->ev_fork, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_join, cudaEventDisableTiming));
@@ -259,14 +268,22 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_walk_len, g.Emax));
   A_(dmalloc(&e->d_wrun, 2ull * g.Emax * g.walk_cap));
   A_(dmalloc(&e->d_wrun_len, g.Emax));
-  A_(dmalloc(&e->d_in_hash, e->stage_launch_cap));
-  A_(dmalloc(&e->d_in_off, e->stage_launch_cap + 1ull));
-  A_(dmalloc(&e->d_in_faults, e->stage_fault_cap));
+  // host-pointer inputs: two staging buffers, filled on a copy stream so that
+  // the upload of batch i+1 overlaps the kernels of batch i
+  A_(dmalloc(&e->d_in_hash, 2ull * e->stage_launch_cap));
+  A_(dmalloc(&e->d_in_off, 2ull * (e->stage_launch_cap + 1ull)));
+  A_(dmalloc(&e->d_in_faults, 2ull * e->stage_fault_cap));
+  A_(cudaStreamCreateWithFlags(&e->copy_s, cudaStreamNonBlocking));
+  for (int b = 0; b < 2; ++b) {
+    A_(cudaEventCreateWithFlags(&e->ev_in_ready[b], cudaEventDisableTiming));
+    A_(cudaEventCreateWithFlags(&e->ev_in_free[b], cudaEventDisableTiming));
+  }
   A_(dmalloc(&e->d_stage_hash, e->stage_launch_cap));
   A_(dmalloc(&e->d_stage_norm, e->stage_fault_cap));
   A_(dmalloc(&e->d_stage_cnt, e->stage_launch_cap));
   A_(dmalloc(&e->d_stage_exec, e->stage_launch_cap));
   A_(dmalloc(&e->d_stage_slot, e->stage_launch_cap));
+  A_(dmalloc(&e->d_pend, e->stage_launch_cap));
   A_(dmalloc(&e->d_stage_off, e->stage_launch_cap));
   A_(dmalloc(&e->d_head, g.Emax));
   A_(dmalloc(&e->d_next, e->stage_launch_cap));
@@ -386,15 +403,30 @@ int dum_record_faults(dum_engine *e, const uint64_t *launch_hash, const uint64_t
       if (launch_off[i + 1] < launch_off[i]) return fail(e, DUM_EINVAL, "launch_off not monotone");
     // branch-free max (vectorised by the compiler): the check costs a fraction
     // of the copy it guards
-    uint32_t mx = 0;
-    for (uint64_t i = 0; i < n_fault; ++i) mx = fault_block[i] > mx ? fault_block[i] : mx;
-    if (n_fault && mx >= e->g.W) return fail(e, DUM_EINVAL, "block id >= max_blocks");
-    CK(cudaMemcpyAsync(e->d_in_hash, launch_hash, 8ull * n_launch, cudaMemcpyHostToDevice, s));
-    CK(cudaMemcpyAsync(e->d_in_off, launch_off, 8ull * (n_launch + 1), cudaMemcpyHostToDevice, s));
-    if (n_fault) CK(cudaMemcpyAsync(e->d_in_faults, fault_block, 4ull * n_fault, cudaMemcpyHostToDevice, s));
-    h = e->d_in_hash;
-    o = e->d_in_off;
-    f = e->d_in_faults;
+    // block ids are checked on the device, as for device pointers (a host pass
+    // over the records would read them from DRAM a second time)
+    // copy stream: wait until the kernels that last read this staging buffer
+    // are done, upload, and make the compute stream wait for the upload only
+    const int b = e->in_buf;
+    e->in_buf ^= 1;
+    uint64_t *dh = e->d_in_hash + (uint64_t)b * e->stage_launch_cap;
+    uint64_t *doff = e->d_in_off + (uint64_t)b * (e->stage_launch_cap + 1ull);
+    uint32_t *df = e->d_in_faults + (uint64_t)b * e->stage_fault_cap;
+    CK(cudaStreamWaitEvent(e->copy_s, e->ev_in_free[b], 0));
+    CK(cudaMemcpyAsync(dh, launch_hash, 8ull * n_launch, cudaMemcpyHostToDevice, e->copy_s));
+    CK(cudaMemcpyAsync(doff, launch_off, 8ull * (n_launch + 1), cudaMemcpyHostToDevice, e->copy_s));
+    if (n_fault) CK(cudaMemcpyAsync(df, fault_block, 4ull * n_fault, cudaMemcpyHostToDevice, e->copy_s));
+    CK(cudaEventRecord(e->ev_in_ready[b], e->copy_s));
+    CK(cudaStreamWaitEvent(s, e->ev_in_ready[b], 0));
+    h = dh;
+    o = doff;
+    f = df;
+    CK(launch_record(e, h, o, n_launch, f, out_exec, s));
+    CK(cudaEventRecord(e->ev_in_free[b], s));  // k_ingest has read the buffer after this point
+    e->n_staged += n_launch;
+    e->staged_faults += n_fault;
+    e->launches += n_launch;
+    return DUM_OK;
   } else if ((reinterpret_cast<uintptr_t>(launch_hash) | reinterpret_cast<uintptr_t>(launch_off)) & 7 ||
              reinterpret_cast<uintptr_t>(fault_block) & 3) {
     return fail(e, DUM_EINVAL, "unaligned pointer");
@@ -582,6 +614,15 @@ int dum_read_timing(dum_engine *e, double ms[DUM_NTIMERS], uint64_t count[DUM_NT
 }
 
 uint64_t dum_kernel_launches(const dum_engine *e) { return e ? e->kernel_launches : 0; }
+
+int dum_host_ptr_kind(const void *p) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return -1;
+  }
+  return (int)a.type;
+}
 
 // ---------------------------------------------------------------------------
 // canonical dump (host-side canonicalisation of a device snapshot)

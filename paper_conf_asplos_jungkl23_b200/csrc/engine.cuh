@@ -54,6 +54,7 @@ struct DevState {
   unsigned long long pool_anchor;  // anchored-walk scratch bump pointer
   unsigned long long pool_big;     // build-walk global hash scratch bump pointer
   uint32_t n_slow;            // exec IDs queued for the sequential walk
+  uint32_t n_pend;            // record: launches with a hash first seen in the batch (k_ingest -> k_exec_assign)
   uint32_t free_count;        // free HBM frames
   uint32_t mig_counter;       // next migration stamp (D19)
   uint32_t lrm_head, lrm_tail;// LRM log [head, tail)
@@ -142,10 +143,14 @@ struct dum_engine {
   // staging
   uint32_t stage_launch_cap;
   uint64_t stage_fault_cap;
-  uint64_t *d_in_hash, *d_in_off;   // host-pointer inputs are copied here
+  uint64_t *d_in_hash, *d_in_off;   // host-pointer inputs are copied here (two buffers, alternating)
+  cudaStream_t copy_s;              // uploads of host-pointer inputs
+  cudaEvent_t ev_in_ready[2], ev_in_free[2];
+  int in_buf;
   uint32_t *d_in_faults;
   uint64_t *d_stage_hash;
   uint32_t *d_stage_norm, *d_stage_cnt, *d_stage_exec, *d_stage_slot;
+  uint32_t *d_pend;       // [stage_launch_cap] launches queued for k_exec_assign
   uint64_t *d_stage_off;  // offset of launch j's records in d_stage_norm
   uint32_t n_staged;
   uint64_t staged_faults;

@@ -39,7 +39,7 @@
 namespace dum {
 
 constexpr uint32_t GCAP = 256;     // launches of one exec ID per build batch
-constexpr int PLAN_NT = 1024;
+constexpr int PLAN_NT = 256;
 constexpr int AP_NT = 256;         // k_apply threads
 constexpr uint32_t OPP = 256;      // target operations per apply partition
 constexpr uint32_t PMAX = 64;      // partitions per exec ID (<= R / 32)
@@ -62,6 +62,8 @@ __global__ void k_build_prep(uint32_t n_staged, uint32_t k0, const uint32_t *__r
   if (j == 0) {
     st->pool_big = 0;
     st->n_slow = 0;
+    st->n_items = 0;  // k_plan's CTAs reserve their work-list ranges from here
+    st->n_leads = 0;
   }
   if (j >= n_staged) return;
   auto prev = [&](int m) -> uint32_t {
@@ -268,8 +270,9 @@ __device__ __forceinline__ uint32_t smid() {
 
 __global__ void __launch_bounds__(PLAN_NT) k_plan(BuildArgs a) {
   __shared__ uint32_t ws[PLAN_NT / 32];
+  __shared__ uint32_t s_ib, s_lb;
   const uint32_t tid = threadIdx.x;
-  if (tid == 0) {
+  if (blockIdx.x == 0 && tid == 0) {
     // history shift register after this batch: the last four exec IDs of
     // (old history ++ staged launches); read by the next k_build_prep only
     uint32_t h[4];
@@ -282,39 +285,44 @@ __global__ void __launch_bounds__(PLAN_NT) k_plan(BuildArgs a) {
   const uint32_t c0 = a.st->cls_cnt[0], c1 = a.st->cls_cnt[1], c2 = a.st->cls_cnt[2];
   const uint32_t tot = c0 + c1 + c2;
   const uint32_t pmax = max(1u, min(PMAX, a.g.R / 32));
-  uint32_t ibase = 0, lbase = 0;
-  for (uint32_t x0 = 0; x0 < tot; x0 += PLAN_NT) {
+  // one chunk of the class-ordered list per CTA; the CTAs reserve their item
+  // ranges with one atomic each (chunks of the big classes come first in CTA
+  // order, which is all the largest-first scheduling needs)
+  {
+    const uint32_t x0 = blockIdx.x * PLAN_NT;
+    if (x0 >= tot) return;
     const uint32_t x = x0 + tid;
     uint32_t P = 0, j = NONE, e = NONE;
+    LeadDesc d;
     if (x < tot) {
       const uint32_t cls = x < c0 ? 0u : x < c0 + c1 ? 1u : 2u;
       const uint32_t ci = x - (cls == 0 ? 0u : cls == 1 ? c0 : c0 + c1);
       j = a.order[cls * a.n_staged + ci];
       e = a.stage_exec[j];
-      if (a.head[e] == j) P = min(pmax, max(1u, (a.e_ops[e] + OPP - 1) / OPP));
-    }
-    uint32_t totP, totL;
-    const uint32_t ip = block_excl_scan(P, ws, &totP);
-    const uint32_t lp = block_excl_scan(P ? 1u : 0u, ws, &totL);
-    if (P) {
-      LeadDesc d;
+      // the descriptor's loads go out with the leader test (used by leaders only)
+      const uint32_t hd = a.head[e], last = a.e_last[e];
       d.j = j;
       d.e = e;
       d.single = a.next[j] == NONE;
       d.n_ops = a.e_ops[e];
-      const uint32_t last = a.e_last[e];
       d.n_last = a.stage_cnt[last];
       d.pad = 0;
       d.off_last = a.stage_off[last];
+      if (hd == j) P = min(pmax, max(1u, (d.n_ops + OPP - 1) / OPP));
+    }
+    uint32_t totP, totL;
+    const uint32_t ip = block_excl_scan(P, ws, &totP);
+    const uint32_t lp = block_excl_scan(P ? 1u : 0u, ws, &totL);
+    if (tid == 0) {
+      s_ib = totP ? atomicAdd(&a.st->n_items, totP) : 0u;
+      s_lb = totL ? atomicAdd(&a.st->n_leads, totL) : 0u;
+    }
+    __syncthreads();
+    const uint32_t ibase = s_ib, lbase = s_lb;
+    if (P) {
       a.desc[lbase + lp] = d;
       for (uint32_t c = 0; c < P; ++c) a.items[ibase + ip + c] = make_uint2(lbase + lp, c | (P << 16));
     }
-    ibase += totP;
-    lbase += totL;
-  }
-  if (tid == 0) {
-    a.st->n_items = ibase;
-    a.st->n_leads = lbase;
   }
 }
 
@@ -905,7 +913,7 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
     k_build_prep<<<(n + 255) / 256, 256, 0, s>>>(n, (uint32_t)e->built_launches, e->d_stage_exec, e->d_stage_cnt,
                                                   e->d_corr, e->corr_cap, e->d_rec_slot, e->d_head, e->d_next,
                                                   e->d_order, e->d_e_ops, e->d_e_last, e->d_state);
-    k_plan<<<1, PLAN_NT, 0, s>>>(ba);
+    k_plan<<<(n + PLAN_NT - 1) / PLAN_NT, PLAN_NT, 0, s>>>(ba);
   }
   // the jump tables depend only on the correlation table, final here
   static const char *jm = getenv("DUM_JUMP_MODE");

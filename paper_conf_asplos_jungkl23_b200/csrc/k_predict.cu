@@ -130,6 +130,7 @@ struct PredArgs {
   uint64_t big_entries;
   SelectOut so;     // fused a8 outputs (SELECT only)
   unsigned long long *cta_clk;  // debug (DUM_CTA_CLOCK): per CTA 8 x u64 timestamps, or null
+  uint64_t *needed;             // pair-pool size after every reservation (k_chain's last CTA), or null
 };
 
 __device__ __forceinline__ unsigned long long pred_timer() {
@@ -233,24 +234,30 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
       a.qnk[qi] = nk;
     }
   }
-  // CTA-aggregated output reservation
+  // CTA-aggregated output reservation and window-size class counts (one
+  // global atomic per CTA and class instead of one per query)
+  __shared__ uint32_t s_cls[NQCLS], s_cbase[NQCLS], s_wcls[CHAIN_WARPS];
+  // window-size class (largest first) for k_predict's CTA order: the big
+  // windows start first instead of forming the tail
+  const uint32_t cls = U >= 14336 ? 0u : U >= 10240 ? 1u : U >= 6144 ? 2u : U >= 2048 ? 3u : 4u;
+  if (threadIdx.x < NQCLS) s_cls[threadIdx.x] = 0;
   if (lane == 0) s_u[w] = U;
+  __syncthreads();
+  if (qi < a.nq && lane == 0) s_wcls[w] = atomicAdd(&s_cls[cls], 1u);  // rank within the CTA
   __syncthreads();
   if (threadIdx.x == 0) {
     unsigned long long tot = 0;
     for (int i = 0; i < CHAIN_WARPS; ++i) tot += s_u[i];
     s_base = tot ? atomicAdd(&a.st->pool_pairs, tot) : 0ull;
   }
+  if (threadIdx.x < NQCLS) s_cbase[threadIdx.x] = s_cls[threadIdx.x] ? atomicAdd(&a.st->q_cls[threadIdx.x], s_cls[threadIdx.x]) : 0u;
   __syncthreads();
   if (qi < a.nq && lane == 0) {
     unsigned long long base = s_base;
     for (uint32_t i = 0; i < w; ++i) base += s_u[i];
     a.qbase[qi] = base;
     if (base + U > a.cap) set_err(a.st, ERR_ECAPACITY, base + U);
-    // window-size class (largest first) for k_predict's CTA order: the big
-    // windows start first instead of forming the tail
-    const uint32_t c = U >= 14336 ? 0u : U >= 10240 ? 1u : U >= 6144 ? 2u : U >= 2048 ? 3u : 4u;
-    a.qrank[qi] = (c << 24) | atomicAdd(&a.st->q_cls[c], 1u);
+    a.qrank[qi] = (cls << 24) | (s_cbase[cls] + s_wcls[w]);
   }
   // the last CTA turns (class, rank) into the permutation
   __shared__ bool s_last;
@@ -267,14 +274,26 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
       pre[c] = acc;
       acc += *(volatile uint32_t *)&a.st->q_cls[c];
     }
-    for (uint32_t q = threadIdx.x; q < a.nq; q += blockDim.x) {
-      const uint32_t r = __ldcg(a.qrank + q);
-      uint32_t p = r & 0xFFFFFFu;
+    constexpr uint32_t QB = 4;  // queries per thread with their loads in flight together
+    for (uint32_t q0 = threadIdx.x; q0 < a.nq; q0 += blockDim.x * QB) {
+      uint32_t r[QB];
 #pragma unroll
-      for (int c = 0; c < NQCLS; ++c)
-        if ((r >> 24) == (uint32_t)c) p += pre[c];
-      a.qperm[p] = q;
+      for (uint32_t u = 0; u < QB; ++u) {
+        const uint32_t q = q0 + u * blockDim.x;
+        r[u] = q < a.nq ? __ldcg(a.qrank + q) : NONE;
+      }
+#pragma unroll
+      for (uint32_t u = 0; u < QB; ++u) {
+        if (r[u] == NONE) continue;
+        uint32_t p = r[u] & 0xFFFFFFu;
+#pragma unroll
+        for (int c = 0; c < NQCLS; ++c)
+          if ((r[u] >> 24) == (uint32_t)c) p += pre[c];
+        a.qperm[p] = q0 + u * blockDim.x;
+      }
     }
+    // every reservation is made: the pool size is the call's `needed`
+    if (threadIdx.x == 0 && a.needed) *a.needed = *(volatile unsigned long long *)&a.st->pool_pairs;
   }
 }
 
@@ -426,21 +445,37 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
       record_dup(anchor >> 5, atomicOr(&bitmap[anchor >> 5], m) & m);
     }
     uint32_t lo = 0;  // list of run x (x only grows: a running cursor, no search)
-    for (uint32_t x = tid; x < etot; x += GRP_NT) {
-      while (eoff[lo + 1] <= x) ++lo;
-      const uint32_t i = x - eoff[lo];
-      uint32_t w, m;
-      if (lo == 0 && anchored) {
-        const uint32_t b = apool[i];
-        w = b >> 5;
-        m = 1u << (b & 31);
-      } else {
-        const uint2 r = __ldg(reinterpret_cast<const uint2 *>(a.wrun) + (uint64_t)kern[lo] * g.walk_cap + i);
-        w = r.x;
-        m = r.y;
+    constexpr int RB = 4;  // runs per thread with their loads in flight together
+    for (uint32_t x0 = tid; x0 < etot; x0 += GRP_NT * RB) {
+      uint32_t w[RB], m[RB];
+#pragma unroll
+      for (int q = 0; q < RB; ++q) {
+        const uint32_t x = x0 + q * GRP_NT;
+        w[q] = NONE;
+        m[q] = 0;
+        if (x < etot) {
+          while (eoff[lo + 1] <= x) ++lo;
+          const uint32_t i = x - eoff[lo];
+          if (lo == 0 && anchored) {
+            const uint32_t b = apool[i];
+            w[q] = b >> 5;
+            m[q] = 1u << (b & 31);
+          } else {
+            const uint2 r = __ldg(reinterpret_cast<const uint2 *>(a.wrun) + (uint64_t)kern[lo] * g.walk_cap + i);
+            w[q] = r.x;
+            m[q] = r.y;
+          }
+        }
       }
-      record_dup(w, atomicOr(&bitmap[w], m) & m);
-      if (SELECT) nonres += __popc(m & ~__ldg(&a.so.res_bits[w]));
+      uint32_t rb[RB];
+#pragma unroll
+      for (int q = 0; q < RB; ++q) rb[q] = (SELECT && w[q] != NONE) ? __ldg(&a.so.res_bits[w[q]]) : 0u;
+#pragma unroll
+      for (int q = 0; q < RB; ++q) {
+        if (w[q] == NONE) continue;
+        record_dup(w[q], atomicOr(&bitmap[w[q]], m[q]) & m[q]);
+        if (SELECT) nonres += __popc(m[q] & ~rb[q]);
+      }
     }
     if (SELECT) {
 #pragma unroll
@@ -696,7 +731,6 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
   if (clk && tid == 0) clk[6] = pred_timer() | ((unsigned long long)(ndup != 0) << 63);
 }
 
-__global__ void k_copy_counter(const unsigned long long *src, uint64_t *dst) { *dst = *src; }
 __global__ void k_copy_counters2(const unsigned long long *a, const unsigned long long *b, uint64_t *dst) {
   *dst = *a > *b ? *a : *b;
 }
@@ -763,6 +797,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
     a.so.res_bits = e->d_res_bits;
   }
   a.cta_clk = nullptr;
+  a.needed = needed;
   static const char *clk_path = getenv("DUM_PRED_CLOCK");
   static unsigned long long *d_clk = nullptr;
   static int clk_calls = 0;
@@ -797,10 +832,6 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
       fwrite(h.data(), 8, h.size(), f);
       fclose(f);
     }
-  }
-  if (needed) {
-    k_copy_counter<<<1, 1, 0, s>>>(&e->d_state->pool_pairs, needed);
-    e->kernel_launches += 1;
   }
   if (sel && sel_needed) {
     k_copy_counters2<<<1, 1, 0, s>>>(&e->d_state->pool_wb, &e->d_state->pool_inv, sel_needed);

@@ -28,7 +28,8 @@ __global__ void __launch_bounds__(INGEST_NT) k_ingest(
     uint32_t n_launch, uint32_t W, uint32_t l0, uint64_t f0, uint64_t *__restrict__ stage_hash,
     uint64_t *__restrict__ stage_off, uint32_t *__restrict__ stage_norm, uint32_t *__restrict__ stage_cnt,
     uint32_t *__restrict__ stage_slot, unsigned long long *exec_keys, uint32_t *exec_vals, uint32_t *exec_minpos,
-    uint32_t exec_cap, uint32_t *big_pool, uint64_t big_entries, uint32_t bm_words, DevState *st) {
+    uint32_t exec_cap, uint32_t *big_pool, uint64_t big_entries, uint32_t bm_words, uint32_t *__restrict__ stage_exec,
+    uint32_t *__restrict__ out_exec, uint32_t *__restrict__ pend, uint32_t Emax, DevState *st) {
   extern __shared__ uint32_t dyn[];  // hash (2 x INGEST_HCAP) or bitmap + small dup hash
   __shared__ uint32_t ws[INGEST_NT / 32];
   __shared__ uint32_t s_dups, s_ovf;
@@ -41,6 +42,41 @@ __global__ void __launch_bounds__(INGEST_NT) k_ingest(
     stage_off[l0 + i] = f0 + a;
     ctr_add(st, DUM_CTR_LAUNCHES, 1);
     s_dups = 0;
+  }
+  if (threadIdx.x == 0) {
+    // execution ID table probe (insert if absent), PAPER.md L136 -- issued
+    // first so that its atomics overlap the record dedupe below.  A known hash
+    // gets its ID here; a hash first seen in this batch is PENDING and queued
+    // for k_exec_assign.
+    const uint64_t h = hash[i];
+    uint32_t slot = NONE;
+    if (h == EMPTY64) {
+      slot = exec_cap;  // sentinel-key slot; exec_keys[exec_cap] is a presence word
+      atomicCAS(&exec_keys[exec_cap], 0ull, 1ull);
+    } else {
+      uint32_t s = (uint32_t)fmix64(h) & (exec_cap - 1);
+      for (uint32_t p = 0; p < exec_cap; ++p) {
+        const unsigned long long old = atomicCAS(&exec_keys[s], EMPTY64, (unsigned long long)h);
+        if (old == EMPTY64 || old == h) {
+          slot = s;
+          break;
+        }
+        s = (s + 1) & (exec_cap - 1);
+      }
+    }
+    uint32_t id = NONE;
+    if (slot == NONE) {
+      set_err(st, ERR_ECAPACITY, 2ull * exec_cap);
+    } else if ((id = ((volatile uint32_t *)exec_vals)[slot]) == PENDING) {
+      atomicMin(&exec_minpos[slot], i);
+      pend[atomicAdd(&st->n_pend, 1u)] = i;
+    }
+    if (id != PENDING) {
+      if (id != NONE && id >= Emax) id = NONE;
+      stage_exec[l0 + i] = id;
+      if (out_exec) out_exec[i] = id;
+    }
+    stage_slot[l0 + i] = slot;
   }
   // Big launches (> INGEST_HCAP/2 records) dedupe through a bitmap over the
   // block-id space when it fits the shared-memory budget: an order-free
@@ -193,31 +229,6 @@ __global__ void __launch_bounds__(INGEST_NT) k_ingest(
   } else if (n == 0 && threadIdx.x == 0) {
     stage_cnt[l0 + i] = 0;
   }
-  if (threadIdx.x == 0) {
-    // execution ID table probe (insert if absent)
-    const uint64_t h = hash[i];
-    uint32_t slot = NONE;
-    if (h == EMPTY64) {
-      slot = exec_cap;  // sentinel-key slot; exec_keys[exec_cap] is a presence word
-      atomicCAS(&exec_keys[exec_cap], 0ull, 1ull);
-    } else {
-      uint32_t s = (uint32_t)fmix64(h) & (exec_cap - 1);
-      for (uint32_t p = 0; p < exec_cap; ++p) {
-        const unsigned long long old = atomicCAS(&exec_keys[s], EMPTY64, (unsigned long long)h);
-        if (old == EMPTY64 || old == h) {
-          slot = s;
-          break;
-        }
-        s = (s + 1) & (exec_cap - 1);
-      }
-    }
-    if (slot == NONE) {
-      set_err(st, ERR_ECAPACITY, 2ull * exec_cap);
-    } else if (((volatile uint32_t *)exec_vals)[slot] == PENDING) {
-      atomicMin(&exec_minpos[slot], i);
-    }
-    stage_slot[l0 + i] = slot;
-  }
 }
 
 constexpr int ASSIGN_NT = 1024;
@@ -225,9 +236,56 @@ constexpr int ASSIGN_NT = 1024;
 __global__ void __launch_bounds__(ASSIGN_NT) k_exec_assign(
     uint32_t n_launch, uint32_t l0, const uint32_t *__restrict__ stage_slot, const uint64_t *__restrict__ stage_hash,
     uint32_t *exec_vals, uint32_t *exec_minpos, uint64_t *exec_hash, uint32_t *__restrict__ stage_exec,
-    uint32_t *__restrict__ out_exec, uint32_t Emax, DevState *st) {
+    uint32_t *__restrict__ out_exec, const uint32_t *__restrict__ pend, uint32_t Emax, DevState *st) {
   __shared__ uint32_t ws[ASSIGN_NT / 32];
+  __shared__ uint32_t s_first[2 * ASSIGN_NT], s_nf;
   const uint32_t E0 = st->E;
+  const uint32_t npend = *(volatile uint32_t *)&st->n_pend;
+  if (npend <= 2 * ASSIGN_NT) {
+    // Only the launches whose hash was first seen in this batch (k_ingest
+    // queued them).  New IDs go to the first occurrences in launch order:
+    // rank = first occurrences at an earlier position (the queue is short).
+    if (threadIdx.x == 0) s_nf = 0;
+    __syncthreads();
+    uint32_t mine[2], nm = 0;
+    for (uint32_t t = threadIdx.x; t < npend; t += ASSIGN_NT) {
+      const uint32_t i = pend[t], slot = stage_slot[l0 + i];
+      if (slot != NONE && ((volatile uint32_t *)exec_minpos)[slot] == i) {
+        mine[nm++] = i;
+        s_first[atomicAdd(&s_nf, 1u)] = i;
+      }
+    }
+    __syncthreads();
+    const uint32_t nf = s_nf;
+    for (uint32_t k = 0; k < nm; ++k) {
+      const uint32_t i = mine[k], slot = stage_slot[l0 + i];
+      uint32_t r = 0;
+      for (uint32_t q = 0; q < nf; ++q) r += s_first[q] < i;
+      const uint32_t id = E0 + r;
+      exec_vals[slot] = id;
+      exec_minpos[slot] = NONE;
+      if (id < Emax) exec_hash[id] = stage_hash[l0 + i];
+    }
+    __syncthreads();
+    for (uint32_t t = threadIdx.x; t < npend; t += ASSIGN_NT) {
+      const uint32_t i = pend[t], slot = stage_slot[l0 + i];
+      uint32_t id = slot == NONE ? NONE : ((volatile uint32_t *)exec_vals)[slot];
+      if (id != NONE && id >= Emax) id = NONE;
+      stage_exec[l0 + i] = id;
+      if (out_exec) out_exec[i] = id;
+    }
+    if (threadIdx.x == 0) {
+      uint32_t E = E0 + nf;
+      if (E > Emax) {
+        set_err(st, ERR_ECAPACITY, E);
+        E = Emax;
+      }
+      st->E = E;
+      st->n_pend = 0;
+    }
+    return;
+  }
+  // long queue (a first batch): scan every launch of the batch
   uint32_t base = 0;
   for (uint32_t c = 0; c < n_launch; c += ASSIGN_NT) {
     const uint32_t i = c + threadIdx.x;
@@ -263,6 +321,7 @@ __global__ void __launch_bounds__(ASSIGN_NT) k_exec_assign(
       E = Emax;
     }
     st->E = E;
+    st->n_pend = 0;
   }
 }
 
@@ -280,11 +339,11 @@ cudaError_t launch_record(dum_engine *e, const uint64_t *hash, const uint64_t *o
                                              e->d_stage_hash, e->d_stage_off, e->d_stage_norm, e->d_stage_cnt,
                                              e->d_stage_slot, e->d_exec_keys, e->d_exec_vals, e->d_exec_minpos,
                                              e->exec_cap, e->d_big_pool, e->big_pool_entries, bm_ok ? bmw : 0,
-                                             e->d_state);
+                                             e->d_stage_exec, out_exec, e->d_pend, e->g.Emax, e->d_state);
   }
   TimerScope t(e, DUM_T_EXEC_ASSIGN, s);
   k_exec_assign<<<1, ASSIGN_NT, 0, s>>>(n_launch, e->n_staged, e->d_stage_slot, e->d_stage_hash, e->d_exec_vals,
-                                        e->d_exec_minpos, e->d_exec_hash, e->d_stage_exec, out_exec, e->g.Emax,
+                                        e->d_exec_minpos, e->d_exec_hash, e->d_stage_exec, out_exec, e->d_pend, e->g.Emax,
                                         e->d_state);
   e->kernel_launches += 2;
   return cudaGetLastError();

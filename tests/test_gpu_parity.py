@@ -191,8 +191,14 @@ def test_full_batch_of_ten_iterations_in_one_build():
 
 def test_errors_are_reported():
     eng, o = make_pair(W=64, C=8, N=2)
+    with pytest.raises(B.EngineError):  # host offsets not launch-aligned: refused at once
+        eng.record_faults(np.array([1], np.uint64), np.array([0, 2], np.uint64), np.array([3], np.uint32))
+    # out-of-range block id from host memory: detected on the device (sticky)
+    eng.record_faults(np.array([1], np.uint64), np.array([0, 1], np.uint64), np.array([64], np.uint32))
     with pytest.raises(B.EngineError):
-        eng.record_faults(np.array([1], np.uint64), np.array([0, 1], np.uint64), np.array([64], np.uint32))
+        eng.sync()
+    eng.build_tables()
+    eng.sync()
     # device-side detection of an out-of-range block id
     eng.record_faults(dev(np.array([1], np.uint64), np.uint64), dev(np.array([0, 1], np.uint64), np.uint64),
                       dev(np.array([99], np.uint32)))
@@ -212,3 +218,59 @@ def test_errors_are_reported():
     with pytest.raises(B.EngineError) as ei:
         eng2.sync()
     assert getattr(ei.value, "needed", 0) > 1
+
+
+def _big_launch_trace(rng, n_launch, pool, W, lo, hi, repeat_prob):
+    """Launches of thousands of faults: a kernel's list is mostly contiguous
+    tensor ranges (some repeated from its previous launch, some fresh) with
+    random blocks and duplicates mixed in."""
+    hashes, offs, faults = [], [0], []
+    last = {}
+    for _ in range(n_launch):
+        k = int(rng.integers(len(pool)))
+        n = int(rng.integers(lo, hi))
+        if k in last and rng.random() < repeat_prob:
+            lst = list(last[k])
+        else:
+            lst = []
+            while len(lst) < n:
+                start, ln = int(rng.integers(0, W)), int(rng.integers(16, 600))
+                lst += [(start + x) % W for x in range(ln)]
+            lst = lst[:n]
+            for i in range(len(lst)):
+                r = rng.random()
+                if r < 0.05:
+                    lst[i] = int(rng.integers(0, W))
+                elif r < 0.08 and i:
+                    lst[i] = lst[int(rng.integers(0, i))]
+        last[k] = lst
+        hashes.append(pool[k])
+        faults += lst
+        offs.append(len(faults))
+    return (np.array(hashes, dtype=np.uint64), np.array(offs, dtype=np.uint64),
+            np.array(faults, dtype=np.uint32))
+
+
+@pytest.mark.parametrize("R", [2048, 64, 16])
+def test_big_exec_ids_partitioned_apply_and_long_walks(R):
+    """Exec IDs with thousands of operations per batch: the apply is split
+    into up to R/32 set partitions (several launches of one exec ID per batch,
+    several apply rounds per partition), walks longer than the shared-memory
+    scratch (global row cache / positions / dedupe hash), both the
+    duplicate-free fast path and the dedupe path."""
+    rng = np.random.default_rng(77 + R)
+    W = 20000
+    eng, o = make_pair(R=R, A=2, S=4, W=W, C=3000, N=4, max_batch_faults=1 << 18)
+    pool = [wl.fnv1a64(b"big%d" % i) for i in range(4)]
+    ex_all = []
+    for batch in range(4):
+        h, off, f = _big_launch_trace(rng, n_launch=int(rng.integers(3, 9)), pool=pool, W=W, lo=1200, hi=5200,
+                                      repeat_prob=0.5)
+        exo, exg = record_both(eng, o, h, off, f, host_ptrs=bool(batch & 1))
+        assert np.array_equal(exo, exg)
+        ex_all += [int(x) for x in exo]
+        build_both(eng, o)
+        assert_same_state(eng, o, msg="R=%d batch %d" % (R, batch))
+        qs = transition_queries(ex_all, 0, len(ex_all), 4)
+        ro, rg, _ = predict_both(eng, o, qs)
+        assert_same_predictions(ro, rg, msg="R=%d batch %d" % (R, batch))
