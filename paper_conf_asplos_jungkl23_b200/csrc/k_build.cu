@@ -683,10 +683,21 @@ __global__ void __launch_bounds__(WK_NT) k_walk(BuildArgs a) {
       // ---- fast path: rows C[0..t] have the single successor C[i+1], so Q =
       // C[0 .. t+1] (t+1 only when a successor is End), duplicate-free ----
       const uint32_t qlen = t + 1 + ((tev & 3) == 2 ? 1u : 0u);
-      for (uint32_t c0 = 0; c0 < qlen; c0 += WK_NT) {
+      constexpr uint32_t FB = 4;  // steps with their loads in flight together
+      for (uint32_t c00 = 0; c00 < qlen; c00 += WK_NT * FB) {
+       uint32_t vals[FB];
+#pragma unroll
+       for (uint32_t u = 0; u < FB; ++u) {
+         const uint32_t p = c00 + u * WK_NT + tid;
+         vals[u] = p < qlen ? C[p] : NONE;
+       }
+#pragma unroll
+       for (uint32_t u = 0; u < FB; ++u) {
+        const uint32_t c0 = c00 + u * WK_NT;
+        if (c0 >= qlen) break;  // uniform
         const uint32_t p = c0 + tid;
         const bool keep = p < qlen;
-        const uint32_t val = keep ? C[p] : NONE;
+        const uint32_t val = vals[u];
         if (keep && p < g.walk_cap) wout[p] = val;
         const uint32_t lane = tid & 31;
         const uint32_t wkey = keep ? val >> 5 : NONE;
@@ -698,6 +709,7 @@ __global__ void __launch_bounds__(WK_NT) k_walk(BuildArgs a) {
         if (lane == 0 && lm) rb = atomicAdd(&s_nrun, (uint32_t)__popc(lm));
         rb = __shfl_sync(0xffffffffu, rb, 0) + __popc(lm & ((1u << lane) - 1));
         if (lead && rb < g.walk_cap) wrun[rb] = make_uint2(wkey, msk);
+       }
       }
       __syncthreads();
       if (tid == 0) {

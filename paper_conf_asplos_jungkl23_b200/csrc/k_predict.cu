@@ -433,8 +433,8 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
       if (k < DLCAP) s_dup[k] = w * 32 + bit;
     }
   };
-  if (wid < GRP_W) {
-    // ---------------- pass 1: window set, duplicate test, non-resident count ----------------
+  {
+    // ---------------- pass 1 (whole CTA): window set, duplicate test, non-resident count ----------------
     // One shared atomicOr per run.  Within one walk the runs are disjoint, so
     // a bit found already set means the block occurs in two lists of the
     // window, or is the anchor (in the window set, never emitted; D14).
@@ -446,11 +446,11 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
     }
     uint32_t lo = 0;  // list of run x (x only grows: a running cursor, no search)
     constexpr int RB = 4;  // runs per thread with their loads in flight together
-    for (uint32_t x0 = tid; x0 < etot; x0 += GRP_NT * RB) {
+    for (uint32_t x0 = tid; x0 < etot; x0 += PRED_NT * RB) {
       uint32_t w[RB], m[RB];
 #pragma unroll
       for (int q = 0; q < RB; ++q) {
-        const uint32_t x = x0 + q * GRP_NT;
+        const uint32_t x = x0 + q * PRED_NT;
         w[q] = NONE;
         m[q] = 0;
         if (x < etot) {
@@ -481,19 +481,27 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
 #pragma unroll
       for (int o = 16; o; o >>= 1) nonres += __shfl_xor_sync(0xffffffffu, nonres, o);
       if (lane == 0 && nonres) atomicAdd(&s_nonres, nonres);
-      group_sync<1, GRP_NT>();
-      if (clk && tid == 0) clk[2] = pred_timer();
-      if (s_ndup == 0) {  // uniform over the group
+    }
+  }
+  __syncthreads();
+  if (clk && tid == 0) clk[2] = pred_timer();
+  // Duplicates are known now: without them (the normal case) warps
+  // [0, GRP_W) run the selection (a8) while the others stream the pairs; with
+  // them the whole CTA takes the duplicate path below instead.
+  if (s_ndup == 0 && !SELECT) {
+    if (ok) copy_lists(wid, NWARP, loff, nullptr);  // predict only: every warp streams
+  } else if (s_ndup == 0) {
+    if (wid < GRP_W) {
+      {
         if (tid == 0) select_reserve(a.so, s_nonres, a.st, ss);
         group_sync<1, GRP_NT>();
         if (clk && tid == 0) clk[3] = pred_timer();
         select_tail<GRP_NT, 1>(a.so, qi, ss, bitmap, a.st, tid, dk);
       }
+      if (clk && tid == 0) clk[4] = pred_timer();
+    } else if (ok) {
+      copy_lists(wid - GRP_W, NWARP - GRP_W, loff, nullptr);
     }
-    if (clk && tid == 0) clk[4] = pred_timer();
-  } else if (ok) {
-    // ---------------- streaming copy (valid unless pass 1 finds a duplicate) ----------------
-    copy_lists(wid - GRP_W, NWARP - GRP_W, loff, nullptr);
   }
   if (clk && tid == GRP_NT) clk[5] = pred_timer();
   __syncthreads();
