@@ -74,6 +74,8 @@ enum {
 
 /* flags */
 #define DUM_HOST_PTRS 0x1u /* dum_record_faults: inputs are host pointers */
+#define DUM_INPUTS_READY 0x2u /* dum_record_faults: the device inputs do not depend on work
+                                 queued on `stream` (the ingest may start before it) */
 
 typedef struct {
   /* UM block correlation table geometry, Table 6;

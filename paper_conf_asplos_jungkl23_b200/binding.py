@@ -14,6 +14,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 _LIBPATH = os.environ.get("DUM_LIB") or os.path.join(HERE, "libdeepum_b200.so")
 
 DUM_NONE = NONE = 0xFFFFFFFF
+DUM_INPUTS_READY = 2
 DUM_HOST_PTRS = 0x1
 DUMP_EXEC, DUMP_CORR, DUMP_BLK, DUMP_WALK, DUMP_RES, DUMP_HIST = 1, 2, 4, 8, 16, 32
 H2D, D2H, INVALIDATE, D2D = 0, 1, 2, 3
@@ -189,8 +190,11 @@ class Engine:
     def reset(self):
         self._ck(self.lib.dum_reset(self._h, self._stream()), "dum_reset")
 
-    def record_faults(self, hashes, offs, faults, out_exec: Optional[torch.Tensor] = None) -> Optional[torch.Tensor]:
-        """Device tensors -> device path; numpy arrays -> DUM_HOST_PTRS."""
+    def record_faults(self, hashes, offs, faults, out_exec: Optional[torch.Tensor] = None,
+                      ready: bool = False) -> Optional[torch.Tensor]:
+        """Device tensors -> device path; numpy arrays -> DUM_HOST_PTRS.
+        ready=True (device tensors): the inputs do not depend on work queued on
+        the current stream (DUM_INPUTS_READY), so the ingest may overlap it."""
         if isinstance(hashes, np.ndarray):
             h = np.ascontiguousarray(hashes, dtype=np.uint64)
             o = np.ascontiguousarray(offs, dtype=np.uint64)
@@ -202,7 +206,8 @@ class Engine:
             return out_exec
         n = hashes.numel()
         self._ck(self.lib.dum_record_faults(self._h, _dev(hashes, 8), _dev(offs, 8), n, _dev(faults, 4),
-                                            faults.numel(), _dev(out_exec, 4), 0, self._stream()),
+                                            faults.numel(), _dev(out_exec, 4), DUM_INPUTS_READY if ready else 0,
+                                            self._stream()),
                  "dum_record_faults")
         return out_exec
 

@@ -87,6 +87,7 @@ cudaError_t fill(uint32_t *p, uint64_t n, uint32_t v, cudaStream_t s) {
 int reset_state(dum_engine *e, cudaStream_t s) {
   const Geo &g = e->g;
   if (e->ev_join) CK(cudaStreamWaitEvent(s, e->ev_join, 0));  // jump tables still building on the side stream
+  if (e->ev_rec) CK(cudaStreamWaitEvent(s, e->ev_rec, 0));    // record work on the ingest stream
   CK(fill((uint32_t *)e->d_exec_keys, 2ull * (e->exec_cap + 1), NONE, s));
   CK(cudaMemsetAsync(e->d_exec_keys + e->exec_cap, 0, 8, s));  // sentinel slot: absent
   CK(fill(e->d_exec_vals, e->exec_cap + 1, PENDING, s));
@@ -114,9 +115,9 @@ int reset_state(dum_engine *e, cudaStream_t s) {
 void free_all(dum_engine *e) {
   void *ptrs[] = {e->d_exec_keys, e->d_exec_vals, e->d_exec_minpos, e->d_exec_hash, e->d_corr, e->d_tbl,
                   e->d_start_end, e->d_walk, e->d_walk_len, e->d_in_hash, e->d_in_off, e->d_in_faults,
-                  e->d_stage_hash, e->d_stage_norm, e->d_stage_cnt, e->d_stage_exec, e->d_stage_slot,
-                  e->d_stage_off, e->d_head, e->d_next, e->d_order, e->d_slow_list,
-                  e->d_e_ops, e->d_e_last, e->d_pend, e->d_lead, e->d_items, e->d_rowc, e->d_big_pool, e->d_walk_seen,
+                  e->stage_base[0], e->stage_base[1], e->stage_base[2], e->stage_base[3], e->stage_base[4],
+                  e->stage_base[5], e->d_head, e->d_next, e->d_order, e->d_slow_list,
+                  e->d_e_ops, e->d_e_last, e->d_pend, e->d_lead, e->d_items, e->d_rowc, e->d_big_pool, e->d_ingest_pool, e->d_walk_seen,
                   e->d_walk_chain, e->d_walk_tmp, e->d_walk_out, e->d_anchor_pool, e->d_anchor_range,
                   e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits, e->d_inactive_bits, e->d_res_bits, e->d_logpos, e->d_lrm_blk,
                   e->d_lrm_stamp, e->d_mig_frames, e->d_mig_src, e->d_mig_blocks, e->d_state, e->d_qkern,
@@ -130,7 +131,11 @@ void free_all(dum_engine *e) {
   }
   if (e->ev_join) cudaEventDestroy(e->ev_join);
   if (e->side) cudaStreamDestroy(e->side);
-  if (e->copy_s) cudaStreamDestroy(e->copy_s);
+  if (e->rec_s) cudaStreamDestroy(e->rec_s);
+  if (e->ev_rec) cudaEventDestroy(e->ev_rec);
+  if (e->ev_s_now) cudaEventDestroy(e->ev_s_now);
+  for (int b = 0; b < 2; ++b)
+    if (e->ev_stage_free[b]) cudaEventDestroy(e->ev_stage_free[b]);
   if (e->h_state) cudaFreeHost(e->h_state);
   for (auto &t : e->pending) {
     cudaEventDestroy(t.a);
@@ -273,18 +278,29 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_in_hash, 2ull * e->stage_launch_cap));
   A_(dmalloc(&e->d_in_off, 2ull * (e->stage_launch_cap + 1ull)));
   A_(dmalloc(&e->d_in_faults, 2ull * e->stage_fault_cap));
-  A_(cudaStreamCreateWithFlags(&e->copy_s, cudaStreamNonBlocking));
+  A_(cudaStreamCreateWithFlags(&e->rec_s, cudaStreamNonBlocking));
+  e->copy_s = e->rec_s;
+  A_(cudaEventCreateWithFlags(&e->ev_rec, cudaEventDisableTiming));
+  A_(cudaEventCreateWithFlags(&e->ev_s_now, cudaEventDisableTiming));
+  for (int b = 0; b < 2; ++b) A_(cudaEventCreateWithFlags(&e->ev_stage_free[b], cudaEventDisableTiming));
   for (int b = 0; b < 2; ++b) {
     A_(cudaEventCreateWithFlags(&e->ev_in_ready[b], cudaEventDisableTiming));
     A_(cudaEventCreateWithFlags(&e->ev_in_free[b], cudaEventDisableTiming));
   }
-  A_(dmalloc(&e->d_stage_hash, e->stage_launch_cap));
-  A_(dmalloc(&e->d_stage_norm, e->stage_fault_cap));
-  A_(dmalloc(&e->d_stage_cnt, e->stage_launch_cap));
-  A_(dmalloc(&e->d_stage_exec, e->stage_launch_cap));
-  A_(dmalloc(&e->d_stage_slot, e->stage_launch_cap));
+  A_(dmalloc(&e->d_stage_hash, 2ull * e->stage_launch_cap));
+  A_(dmalloc(&e->d_stage_norm, 2ull * e->stage_fault_cap));
+  A_(dmalloc(&e->d_stage_cnt, 2ull * e->stage_launch_cap));
+  A_(dmalloc(&e->d_stage_exec, 2ull * e->stage_launch_cap));
+  A_(dmalloc(&e->d_stage_slot, 2ull * e->stage_launch_cap));
   A_(dmalloc(&e->d_pend, e->stage_launch_cap));
-  A_(dmalloc(&e->d_stage_off, e->stage_launch_cap));
+  A_(dmalloc(&e->d_stage_off, 2ull * e->stage_launch_cap));
+  e->stage_base[0] = e->d_stage_hash;
+  e->stage_base[1] = e->d_stage_norm;
+  e->stage_base[2] = e->d_stage_cnt;
+  e->stage_base[3] = e->d_stage_exec;
+  e->stage_base[4] = e->d_stage_slot;
+  e->stage_base[5] = e->d_stage_off;
+  e->stage_set = 0;
   A_(dmalloc(&e->d_head, g.Emax));
   A_(dmalloc(&e->d_next, e->stage_launch_cap));
   A_(dmalloc(&e->d_order, 3ull * e->stage_launch_cap));
@@ -297,6 +313,7 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_items, 2 * e->items_cap));
   A_(dmalloc(&e->d_rowc, e->stage_fault_cap * (1ull + g.S)));
   A_(dmalloc(&e->d_big_pool, 2 * e->big_pool_entries));
+  A_(dmalloc(&e->d_ingest_pool, 2 * e->big_pool_entries));
   A_(dmalloc(&e->d_walk_seen, (uint64_t)e->n_walk_slots * e->walk_hash_cap));
   A_(dmalloc(&e->d_walk_chain, (uint64_t)e->n_walk_slots * e->walk_hash_cap));
   A_(dmalloc(&e->d_walk_tmp, (uint64_t)e->n_walk_slots * tmp_cap));
@@ -395,43 +412,45 @@ int dum_record_faults(dum_engine *e, const uint64_t *launch_hash, const uint64_t
   if (e->launches + n_launch > 0xFFFFFFFFull) return fail(e, DUM_ECAPACITY, "launch counter exceeds 2^32");
   cudaSetDevice(e->device);
   cudaStream_t s = (cudaStream_t)stream;
+  cudaStream_t r = e->rec_s;
   const uint64_t *h = launch_hash, *o = launch_off;
   const uint32_t *f = fault_block;
   if (flags & DUM_HOST_PTRS) {
     if (launch_off[0] != 0 || launch_off[n_launch] != n_fault) return fail(e, DUM_EINVAL, "batch not launch-aligned");
     for (uint32_t i = 0; i < n_launch; ++i)
       if (launch_off[i + 1] < launch_off[i]) return fail(e, DUM_EINVAL, "launch_off not monotone");
-    // branch-free max (vectorised by the compiler): the check costs a fraction
-    // of the copy it guards
     // block ids are checked on the device, as for device pointers (a host pass
     // over the records would read them from DRAM a second time)
-    // copy stream: wait until the kernels that last read this staging buffer
-    // are done, upload, and make the compute stream wait for the upload only
-    const int b = e->in_buf;
-    e->in_buf ^= 1;
-    uint64_t *dh = e->d_in_hash + (uint64_t)b * e->stage_launch_cap;
-    uint64_t *doff = e->d_in_off + (uint64_t)b * (e->stage_launch_cap + 1ull);
-    uint32_t *df = e->d_in_faults + (uint64_t)b * e->stage_fault_cap;
-    CK(cudaStreamWaitEvent(e->copy_s, e->ev_in_free[b], 0));
-    CK(cudaMemcpyAsync(dh, launch_hash, 8ull * n_launch, cudaMemcpyHostToDevice, e->copy_s));
-    CK(cudaMemcpyAsync(doff, launch_off, 8ull * (n_launch + 1), cudaMemcpyHostToDevice, e->copy_s));
-    if (n_fault) CK(cudaMemcpyAsync(df, fault_block, 4ull * n_fault, cudaMemcpyHostToDevice, e->copy_s));
-    CK(cudaEventRecord(e->ev_in_ready[b], e->copy_s));
-    CK(cudaStreamWaitEvent(s, e->ev_in_ready[b], 0));
-    h = dh;
-    o = doff;
-    f = df;
-    CK(launch_record(e, h, o, n_launch, f, out_exec, s));
-    CK(cudaEventRecord(e->ev_in_free[b], s));  // k_ingest has read the buffer after this point
-    e->n_staged += n_launch;
-    e->staged_faults += n_fault;
-    e->launches += n_launch;
-    return DUM_OK;
   } else if ((reinterpret_cast<uintptr_t>(launch_hash) | reinterpret_cast<uintptr_t>(launch_off)) & 7 ||
              reinterpret_cast<uintptr_t>(fault_block) & 3) {
     return fail(e, DUM_EINVAL, "unaligned pointer");
   }
-  CK(launch_record(e, h, o, n_launch, f, out_exec, s));
+  // The batch is ingested on the engine's record stream: it waits for the
+  // build that last read this staging set (two batches ago), and -- unless
+  // the inputs come from the host or the caller declares them ready -- for
+  // the work already queued on `stream`; `stream` then waits for the
+  // ingest.  The ingest of batch i+1 thereby overlaps the build of batch i
+  // (the paper's fault-handling and table-update threads run concurrently,
+  // P:L140-L158).
+  if (!(flags & (DUM_HOST_PTRS | DUM_INPUTS_READY))) {
+    CK(cudaEventRecord(e->ev_s_now, s));
+    CK(cudaStreamWaitEvent(r, e->ev_s_now, 0));
+  }
+  CK(cudaStreamWaitEvent(r, e->ev_stage_free[e->stage_set], 0));
+  if (flags & DUM_HOST_PTRS) {
+    uint64_t *dh = e->d_in_hash;
+    uint64_t *doff = e->d_in_off;
+    uint32_t *df = e->d_in_faults;
+    CK(cudaMemcpyAsync(dh, launch_hash, 8ull * n_launch, cudaMemcpyHostToDevice, r));
+    CK(cudaMemcpyAsync(doff, launch_off, 8ull * (n_launch + 1), cudaMemcpyHostToDevice, r));
+    if (n_fault) CK(cudaMemcpyAsync(df, fault_block, 4ull * n_fault, cudaMemcpyHostToDevice, r));
+    h = dh;
+    o = doff;
+    f = df;
+  }
+  CK(launch_record(e, h, o, n_launch, f, out_exec, r));
+  CK(cudaEventRecord(e->ev_rec, r));
+  CK(cudaStreamWaitEvent(s, e->ev_rec, 0));
   e->n_staged += n_launch;
   e->staged_faults += n_fault;
   e->launches += n_launch;
@@ -441,7 +460,20 @@ int dum_record_faults(dum_engine *e, const uint64_t *launch_hash, const uint64_t
 int dum_build_tables(dum_engine *e, dum_stream_t stream) {
   if (!e) return DUM_EINVAL;
   cudaSetDevice(e->device);
-  CK(launch_build(e, (cudaStream_t)stream));
+  if (e->n_staged) {
+    CK(cudaStreamWaitEvent((cudaStream_t)stream, e->ev_rec, 0));
+    CK(launch_build(e, (cudaStream_t)stream));
+    // this staging set is free once the build has run; the next batch goes to the other set
+    CK(cudaEventRecord(e->ev_stage_free[e->stage_set], (cudaStream_t)stream));
+    e->stage_set ^= 1;
+    const uint64_t L = e->stage_launch_cap, F = e->stage_fault_cap, k = (uint64_t)e->stage_set;
+    e->d_stage_hash = static_cast<uint64_t *>(e->stage_base[0]) + k * L;
+    e->d_stage_norm = static_cast<uint32_t *>(e->stage_base[1]) + k * F;
+    e->d_stage_cnt = static_cast<uint32_t *>(e->stage_base[2]) + k * L;
+    e->d_stage_exec = static_cast<uint32_t *>(e->stage_base[3]) + k * L;
+    e->d_stage_slot = static_cast<uint32_t *>(e->stage_base[4]) + k * L;
+    e->d_stage_off = static_cast<uint64_t *>(e->stage_base[5]) + k * L;
+  }
   e->n_staged = 0;
   e->staged_faults = 0;
   e->built_launches = e->launches;

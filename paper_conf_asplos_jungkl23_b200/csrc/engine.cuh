@@ -144,7 +144,13 @@ struct dum_engine {
   uint32_t stage_launch_cap;
   uint64_t stage_fault_cap;
   uint64_t *d_in_hash, *d_in_off;   // host-pointer inputs are copied here (two buffers, alternating)
-  cudaStream_t copy_s;              // uploads of host-pointer inputs
+  cudaStream_t copy_s;              // uploads of host-pointer inputs (== rec_s)
+  // record_faults runs on its own stream so that the next batch's ingest
+  // overlaps the current build; the staging arrays alternate between two sets
+  cudaStream_t rec_s;
+  cudaEvent_t ev_rec, ev_s_now, ev_stage_free[2];
+  int stage_set;
+  void *stage_base[6];              // the two-set allocations behind d_stage_*
   cudaEvent_t ev_in_ready[2], ev_in_free[2];
   int in_buf;
   uint32_t *d_in_faults;
@@ -164,6 +170,7 @@ struct dum_engine {
   uint64_t items_cap;
   uint32_t *d_rowc;              // walk row cache for long walks: (1 + S) u32 per staged record
   uint32_t *d_big_pool;   // u32 pairs for large-walk hash tables
+  uint32_t *d_ingest_pool;  // the ingest's own global hash region (it may run concurrently with a build)
   uint64_t big_pool_entries;
   // walk scratch for the sequential walker (per CTA slot)
   uint32_t n_walk_slots;

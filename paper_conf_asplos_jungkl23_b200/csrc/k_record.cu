@@ -338,7 +338,7 @@ cudaError_t launch_record(dum_engine *e, const uint64_t *hash, const uint64_t *o
   k_ingest<<<n_launch, INGEST_NT, smem, s>>>(hash, off, faults, n_launch, e->g.W, e->n_staged, e->staged_faults,
                                              e->d_stage_hash, e->d_stage_off, e->d_stage_norm, e->d_stage_cnt,
                                              e->d_stage_slot, e->d_exec_keys, e->d_exec_vals, e->d_exec_minpos,
-                                             e->exec_cap, e->d_big_pool, e->big_pool_entries, bm_ok ? bmw : 0,
+                                             e->exec_cap, e->d_ingest_pool, e->big_pool_entries, bm_ok ? bmw : 0,
                                              e->d_stage_exec, out_exec, e->d_pend, e->g.Emax, e->d_state);
   }
   TimerScope t(e, DUM_T_EXEC_ASSIGN, s);
