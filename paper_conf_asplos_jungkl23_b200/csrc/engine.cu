@@ -117,7 +117,7 @@ void free_all(dum_engine *e) {
                   e->d_start_end, e->d_walk, e->d_walk_len, e->d_in_hash, e->d_in_off, e->d_in_faults,
                   e->stage_base[0], e->stage_base[1], e->stage_base[2], e->stage_base[3], e->stage_base[4],
                   e->stage_base[5], e->d_head, e->d_next, e->d_order, e->d_slow_list,
-                  e->d_e_ops, e->d_e_last, e->d_pend, e->d_lead, e->d_items, e->d_rowc, e->d_big_pool, e->d_ingest_pool, e->d_walk_seen,
+                  e->d_e_ops, e->d_e_last, e->d_pend, e->d_plan_agg, e->d_lead, e->d_items, e->d_rowc, e->d_big_pool, e->d_ingest_pool, e->d_walk_seen,
                   e->d_walk_chain, e->d_walk_tmp, e->d_walk_out, e->d_anchor_pool, e->d_anchor_range,
                   e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits, e->d_inactive_bits, e->d_res_bits, e->d_logpos, e->d_lrm_blk,
                   e->d_lrm_stamp, e->d_mig_frames, e->d_mig_src, e->d_mig_blocks, e->d_state, e->d_qkern,
@@ -307,7 +307,8 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_slow_list, e->stage_launch_cap));
   A_(dmalloc(&e->d_e_ops, g.Emax));
   A_(dmalloc(&e->d_e_last, g.Emax));
-  A_(dmalloc(&e->d_lead, 8ull * e->stage_launch_cap));  // k_build.cu LeadDesc (32 B)
+  A_(dmalloc(&e->d_lead, 8ull * e->stage_launch_cap));
+  A_(dmalloc(&e->d_plan_agg, e->stage_launch_cap / 256 + 1));  // k_build.cu LeadDesc (32 B)
   // apply items: sum over groups of ceil(ops / 256) <= launches + faults / 256
   e->items_cap = e->stage_launch_cap + e->stage_fault_cap / 256 + 1;
   A_(dmalloc(&e->d_items, 2 * e->items_cap));

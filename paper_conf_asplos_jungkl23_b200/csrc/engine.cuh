@@ -165,6 +165,7 @@ struct dum_engine {
   // build scratch
   uint32_t *d_head, *d_next, *d_slow_list, *d_order;
   uint32_t *d_e_ops, *d_e_last;  // per exec ID: group operations / latest launch of the batch
+  uint64_t *d_plan_agg;          // k_plan look-back slots (one per 256 staged launches)
   uint32_t *d_lead;              // exec IDs with faults of the batch (k_build.cu LeadDesc, 32 B each)
   uint32_t *d_items;             // apply items, u32 pairs (leader index, partition | P << 16)
   uint64_t items_cap;

@@ -57,12 +57,13 @@ constexpr uint32_t WK_QCAP = 4096; // shared dedupe-hash capacity (|Q| <= WK_QCA
 __global__ void k_build_prep(uint32_t n_staged, uint32_t k0, const uint32_t *__restrict__ stage_exec,
                              const uint32_t *__restrict__ stage_cnt, CorrSlot *corr, uint32_t corr_cap,
                              uint32_t *rec_slot, uint32_t *head, uint32_t *__restrict__ next,
-                             uint32_t *__restrict__ order, uint32_t *e_ops, uint32_t *e_last, DevState *st) {
+                             uint32_t *__restrict__ order, uint32_t *e_ops, uint32_t *e_last,
+                             unsigned long long *plan_agg, DevState *st) {
   const uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
   if (j == 0) {
     st->pool_big = 0;
     st->n_slow = 0;
-    st->n_items = 0;  // k_plan's CTAs reserve their work-list ranges from here
+    st->n_items = 0;  // k_plan's last chunk writes the list sizes
     st->n_leads = 0;
   }
   if (j >= n_staged) return;
@@ -70,6 +71,7 @@ __global__ void k_build_prep(uint32_t n_staged, uint32_t k0, const uint32_t *__r
     long jj = (long)j - m;
     return jj >= 0 ? stage_exec[jj] : st->hist[4 + jj];
   };
+  if (j < (n_staged + 255) / 256) plan_agg[j] = 0;  // k_plan's look-back slots
   const uint32_t e = stage_exec[j];
   const uint32_t owner = prev(1);
   const bool up = owner != NONE && e != NONE;
@@ -253,6 +255,7 @@ struct BuildArgs {
   uint32_t *slow_list;
   uint32_t *wrun, *wrun_len;   // walk bitmap runs (read by k_predict)
   const uint32_t *order;       // [3][n_staged] faulting launches by size class
+  unsigned long long *plan_agg;  // [k_plan CTAs] published chunk totals (flag << 63 | leads << 32 | items)
   DevState *st;
   unsigned long long *clk;     // debug (DUM_BUILD_CLOCK): per apply item / walk item 4 x u64, or null
 };
@@ -313,9 +316,35 @@ __global__ void __launch_bounds__(PLAN_NT) k_plan(BuildArgs a) {
     uint32_t totP, totL;
     const uint32_t ip = block_excl_scan(P, ws, &totP);
     const uint32_t lp = block_excl_scan(P ? 1u : 0u, ws, &totL);
-    if (tid == 0) {
-      s_ib = totP ? atomicAdd(&a.st->n_items, totP) : 0u;
-      s_lb = totL ? atomicAdd(&a.st->n_leads, totL) : 0u;
+    // offsets in list order (largest launches keep the lowest item / walk
+    // indices): publish this chunk's totals, then add up the earlier chunks'
+    // (decoupled look-back; CTAs are dispatched in index order, so every
+    // earlier chunk is resident or done)
+    if (tid == 0)
+      atomicExch(&a.plan_agg[blockIdx.x], (1ull << 63) | ((unsigned long long)totL << 32) | totP);
+    if (tid < 32) {
+      uint32_t bp = 0, bl = 0;
+      for (uint32_t q = tid; q < blockIdx.x; q += 32) {
+        unsigned long long v;
+        do {
+          v = *(volatile unsigned long long *)&a.plan_agg[q];
+        } while (!(v >> 63));
+        bp += (uint32_t)(v & 0xFFFFFFFFull);
+        bl += (uint32_t)((v >> 32) & 0x7FFFFFFFull);
+      }
+#pragma unroll
+      for (int o = 16; o; o >>= 1) {
+        bp += __shfl_xor_sync(0xffffffffu, bp, o);
+        bl += __shfl_xor_sync(0xffffffffu, bl, o);
+      }
+      if (tid == 0) {
+        s_ib = bp;
+        s_lb = bl;
+        if (x0 + PLAN_NT >= tot) {  // the last chunk: the list sizes
+          a.st->n_items = bp + totP;
+          a.st->n_leads = bl + totL;
+        }
+      }
     }
     __syncthreads();
     const uint32_t ibase = s_ib, lbase = s_lb;
@@ -908,6 +937,7 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   ba.wrun = e->d_wrun;
   ba.wrun_len = e->d_wrun_len;
   ba.order = e->d_order;
+  ba.plan_agg = reinterpret_cast<unsigned long long *>(e->d_plan_agg);
   ba.st = e->d_state;
   ba.clk = nullptr;
   static const char *clk_path = getenv("DUM_BUILD_CLOCK");
@@ -924,7 +954,7 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
     cudaMemsetAsync(e->d_state->cls_cnt, 0, sizeof(e->d_state->cls_cnt), s);
     k_build_prep<<<(n + 255) / 256, 256, 0, s>>>(n, (uint32_t)e->built_launches, e->d_stage_exec, e->d_stage_cnt,
                                                   e->d_corr, e->corr_cap, e->d_rec_slot, e->d_head, e->d_next,
-                                                  e->d_order, e->d_e_ops, e->d_e_last, e->d_state);
+                                                  e->d_order, e->d_e_ops, e->d_e_last, ba.plan_agg, e->d_state);
     k_plan<<<(n + PLAN_NT - 1) / PLAN_NT, PLAN_NT, 0, s>>>(ba);
   }
   // the jump tables depend only on the correlation table, final here
