@@ -41,6 +41,7 @@ __global__ void k_init_state(DevState *st) {
   st->n_slow = 0;
   st->n_pend = 0;
   st->n_items = st->n_leads = 0;
+  for (int c = 0; c < 4; ++c) st->cls_cnt[c] = 0;
   st->corr_used = 0;
   st->mig_ok = 0;
   st->mig_n = 0;

@@ -606,6 +606,7 @@ __global__ void __launch_bounds__(WK_NT) k_walk(BuildArgs a) {
   const uint32_t A = g.A, S = g.S;
   // one CTA per exec ID; the grid is the host's upper bound (staged launches)
   const uint32_t li = blockIdx.x;
+  if (li == 0 && tid < 4) a.st->cls_cnt[tid] = 0;  // k_plan has read them; zero for the next build
   if (li >= *(volatile uint32_t *)&a.st->n_leads) return;
   do {  // (breaks = the early ends of the walk)
     const LeadDesc d = a.desc[li];
@@ -951,7 +952,6 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   }
   {
     TimerScope t(e, DUM_T_BUILD_PREP, s);
-    cudaMemsetAsync(e->d_state->cls_cnt, 0, sizeof(e->d_state->cls_cnt), s);
     k_build_prep<<<(n + 255) / 256, 256, 0, s>>>(n, (uint32_t)e->built_launches, e->d_stage_exec, e->d_stage_cnt,
                                                   e->d_corr, e->corr_cap, e->d_rec_slot, e->d_head, e->d_next,
                                                   e->d_order, e->d_e_ops, e->d_e_last, ba.plan_agg, e->d_state);

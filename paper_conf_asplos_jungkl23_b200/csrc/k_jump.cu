@@ -31,13 +31,19 @@ __global__ void __launch_bounds__(JUMP_NT) k_jump0(const CorrSlot *corr, uint32_
   }
 }
 
-__global__ void __launch_bounds__(JUMP_NT) k_jumpk(uint32_t cap, const uint32_t *rec_slot, const uint32_t *jprev,
-                                                   uint32_t *jnext, const DevState *st) {
+// Levels 1 .. levels-1 in one launch: J_k(s) = J_0^(2^k)(s), each thread
+// follows J_0 from its record and stores the positions 2, 4, 8, ... (2^(L-1)
+// dependent loads of an L2-resident array instead of one launch per level).
+__global__ void __launch_bounds__(JUMP_NT) k_jumpk(uint32_t cap, const uint32_t *rec_slot, uint32_t *jump,
+                                                   uint32_t levels, const DevState *st) {
   const uint32_t nrec = min(*(const volatile uint32_t *)&st->corr_used, cap);
   for (uint32_t r = blockIdx.x * JUMP_NT + threadIdx.x; r < nrec; r += gridDim.x * JUMP_NT) {
     const uint32_t s = rec_slot[r];
-    const uint32_t m = __ldcg(jprev + s);
-    jnext[s] = m == NONE ? NONE : __ldcg(jprev + m);
+    uint32_t x = __ldcg(jump + s);  // J_0(s)
+    for (uint32_t k = 1, step = 1; k < levels; ++k) {
+      for (const uint32_t target = 1u << k; step < target && x != NONE; ++step) x = __ldcg(jump + x);
+      jump[(uint64_t)k * cap + s] = x;
+    }
   }
 }
 
@@ -47,10 +53,8 @@ cudaError_t launch_jump_tables(dum_engine *e, cudaStream_t s) {
   const uint32_t grid = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>((nrec + JUMP_NT - 1) / JUMP_NT, 4 * 148));
   TimerScope t(e, DUM_T_JUMP, s);
   k_jump0<<<grid, JUMP_NT, 0, s>>>(e->d_corr, e->corr_cap, e->d_rec_slot, e->d_jump, e->d_state);
-  for (uint32_t k = 1; k < e->jump_levels; ++k)
-    k_jumpk<<<grid, JUMP_NT, 0, s>>>(e->corr_cap, e->d_rec_slot, e->d_jump + (uint64_t)(k - 1) * e->corr_cap,
-                                     e->d_jump + (uint64_t)k * e->corr_cap, e->d_state);
-  e->kernel_launches += e->jump_levels;
+  if (e->jump_levels > 1) k_jumpk<<<grid, JUMP_NT, 0, s>>>(e->corr_cap, e->d_rec_slot, e->d_jump, e->jump_levels, e->d_state);
+  e->kernel_launches += e->jump_levels > 1 ? 2 : 1;
   return cudaGetLastError();
 }
 

@@ -739,6 +739,20 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
   if (clk && tid == 0) clk[6] = pred_timer() | ((unsigned long long)(ndup != 0) << 63);
 }
 
+// the call's bump pointers and k_chain's class counters
+__global__ void k_pred_reset(DevState *st) {
+  const uint32_t t = threadIdx.x;
+  if (t == 0) {
+    st->pool_pairs = 0;
+    st->pool_wb = 0;
+    st->pool_inv = 0;
+    st->pool_anchor = 0;
+    st->pool_big = 0;
+    st->chain_done = 0;
+  }
+  if (t < 8) st->q_cls[t] = 0;
+}
+
 __global__ void k_copy_counters2(const unsigned long long *a, const unsigned long long *b, uint64_t *dst) {
   *dst = *a > *b ? *a : *b;
 }
@@ -758,9 +772,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
                            const SelectOut *sel, uint64_t *sel_needed, cudaStream_t s) {
   if (nq == 0) return cudaSuccess;
   if (nq > e->anchor_range_cap) return cudaErrorInvalidValue;
-  cudaMemsetAsync(&e->d_state->pool_pairs, 0, 2 * sizeof(unsigned long long) * 2, s);  // pairs, wb, inv, anchor
-  cudaMemsetAsync(&e->d_state->pool_big, 0, sizeof(unsigned long long), s);
-  cudaMemsetAsync(e->d_state->q_cls, 0, sizeof(e->d_state->q_cls) + sizeof(e->d_state->chain_done), s);
+  k_pred_reset<<<1, 32, 0, s>>>(e->d_state);  // one launch instead of three memsets
   WalkScratch ws{e->d_walk_seen, e->d_walk_chain, e->d_walk_tmp, e->walk_hash_cap,
                  e->g.walk_cap + e->g.R * e->g.A + 4};
   {
@@ -821,11 +833,19 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   }
   const size_t smem = (size_t)((a.nwords + 3) & ~3u) * 4 + 2 * DHCAP * 4;
   if (sel) {
-    cudaFuncSetAttribute(k_predict<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    static size_t set_smem = 0;  // the attribute is per function: raise it once per size
+    if (smem > set_smem) {
+      cudaFuncSetAttribute(k_predict<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      set_smem = smem;
+    }
     TimerScope t(e, DUM_T_PREDICT, s);
     k_predict<true><<<nq, PRED_NT, smem, s>>>(a);
   } else {
-    cudaFuncSetAttribute(k_predict<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    static size_t set_smem = 0;
+    if (smem > set_smem) {
+      cudaFuncSetAttribute(k_predict<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      set_smem = smem;
+    }
     TimerScope t(e, DUM_T_PREDICT, s);
     k_predict<false><<<nq, PRED_NT, smem, s>>>(a);
   }

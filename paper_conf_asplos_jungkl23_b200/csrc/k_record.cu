@@ -334,7 +334,11 @@ cudaError_t launch_record(dum_engine *e, const uint64_t *hash, const uint64_t *o
   const size_t bm_bytes = (size_t)((bmw + 3) & ~3u) * 4 + 2 * IDCAP * 4;
   const bool bm_ok = bm_bytes <= INGEST_SMEM_MAX;
   const size_t smem = std::max<size_t>(2 * INGEST_HCAP * 4, bm_ok ? bm_bytes : 0);
-  cudaFuncSetAttribute(k_ingest, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  static size_t set_smem = 0;  // the attribute is per function: raise it once per size
+  if (smem > set_smem) {
+    cudaFuncSetAttribute(k_ingest, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    set_smem = smem;
+  }
   k_ingest<<<n_launch, INGEST_NT, smem, s>>>(hash, off, faults, n_launch, e->g.W, e->n_staged, e->staged_faults,
                                              e->d_stage_hash, e->d_stage_off, e->d_stage_norm, e->d_stage_cnt,
                                              e->d_stage_slot, e->d_exec_keys, e->d_exec_vals, e->d_exec_minpos,
