@@ -274,3 +274,61 @@ def test_big_exec_ids_partitioned_apply_and_long_walks(R):
         qs = transition_queries(ex_all, 0, len(ex_all), 4)
         ro, rg, _ = predict_both(eng, o, qs)
         assert_same_predictions(ro, rg, msg="R=%d batch %d" % (R, batch))
+
+
+@pytest.mark.parametrize("trace", ["T", "big"])
+def test_overlapped_ingest_no_host_syncs(trace):
+    """The bench schedule issued back to back with no host synchronisation:
+    record(i+1) runs on the engine's ingest stream (DUM_INPUTS_READY, and host
+    pointers) while build(i) runs; every iteration's predictions (kept in
+    their own buffers) and the final tables must equal the oracle's."""
+    rng = np.random.default_rng(5)
+    if trace == "T":
+        tr = wl.make_T()
+        batches = [tr.iteration(i) for i in range(tr.n_iter)]
+        eng, o = make_pair(R=2048, A=2, S=4, W=tr.W, C=tr.C, N=2)
+        N = 2
+    else:
+        W = 20000
+        pool = [wl.fnv1a64(b"ov%d" % i) for i in range(5)]
+        batches = [_big_launch_trace(rng, n_launch=6, pool=pool, W=W, lo=200, hi=3000, repeat_prob=0.6)
+                   for _ in range(6)]
+        eng, o = make_pair(R=64, A=2, S=4, W=W, C=3000, N=3, max_batch_faults=1 << 17)
+        N = 3
+    dev_b = [(dev(h, np.uint64), dev(off, np.uint64), dev(f)) for h, off, f in batches]
+    torch.cuda.synchronize()
+    ex_all, ex_dev, outs, qs_all = [], [], [], []
+    for i, (h, off, f) in enumerate(batches):
+        ex_o = o.record_faults(h, off, f)
+        out = torch.empty(len(h), dtype=torch.int32, device="cuda")
+        if i % 3 == 2:
+            eng.record_faults(np.asarray(h, np.uint64), np.asarray(off, np.uint64), np.asarray(f, np.uint32), out)
+        else:
+            eng.record_faults(*dev_b[i], out, ready=i > 0)
+        ex_dev.append(out)
+        prev = len(ex_all)
+        ex_all += [int(x) for x in ex_o]
+        if i >= 1:
+            qs = transition_queries(ex_all, prev, len(h), N)
+            qd = dev(qs.reshape(-1)).reshape(-1, 6)
+            off_o, pairs_o, ko_o, ch_o = o.predict(np.ascontiguousarray(qs, dtype=np.uint32).reshape(-1, 6))
+            # a window gathers at most N + 1 walks of at most 1 + S (rows) blocks each
+            cap = len(qs) * (N + 1) * 5 * (int(np.diff(off).max()) + 1) + 64
+            gp, grng, gko, gch, _ = eng.predict_prefetch(qd, cap)
+            outs.append((gp, grng, gko, gch, off_o, pairs_o, ko_o, ch_o))
+        o.build_tables()
+        eng.build_tables()
+    eng.sync()
+    for i, (h, _, _) in enumerate(batches):
+        assert np.array_equal(B.u32(ex_dev[i]), np.array(ex_all[sum(len(b[0]) for b in batches[:i]):][:len(h)],
+                                                         dtype=np.uint32)), "exec ids of batch %d" % i
+    for j, (gp, grng, gko, gch, off_o, pairs_o, ko_o, ch_o) in enumerate(outs):
+        gp = B.u32(gp).reshape(-1, 2)
+        grng = B.u64(grng).reshape(-1, 2)
+        gko = B.u32(gko).reshape(len(grng), -1)
+        gch = B.u32(gch).reshape(len(grng), -1)
+        for q in range(len(grng)):
+            assert np.array_equal(gp[int(grng[q, 0]):int(grng[q, 1])], pairs_o[int(off_o[q]):int(off_o[q + 1])]), \
+                "batch %d query %d" % (j + 1, q)
+            assert np.array_equal(gko[q], ko_o[q]) and np.array_equal(gch[q], ch_o[q])
+    assert_same_state(eng, o)
