@@ -126,10 +126,6 @@ void free_all(dum_engine *e) {
   for (void *p : ptrs)
     if (p) cudaFree(p);
   if (e->ev_fork) cudaEventDestroy(e->ev_fork);
-  for (int b = 0; b < 2; ++b) {
-    if (e->ev_in_ready[b]) cudaEventDestroy(e->ev_in_ready[b]);
-    if (e->ev_in_free[b]) cudaEventDestroy(e->ev_in_free[b]);
-  }
   if (e->ev_join) cudaEventDestroy(e->ev_join);
   if (e->side) cudaStreamDestroy(e->side);
   if (e->rec_s) cudaStreamDestroy(e->rec_s);
@@ -274,20 +270,15 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_walk_len, g.Emax));
   A_(dmalloc(&e->d_wrun, 2ull * g.Emax * g.walk_cap));
   A_(dmalloc(&e->d_wrun_len, g.Emax));
-  // host-pointer inputs: two staging buffers, filled on a copy stream so that
-  // the upload of batch i+1 overlaps the kernels of batch i
-  A_(dmalloc(&e->d_in_hash, 2ull * e->stage_launch_cap));
-  A_(dmalloc(&e->d_in_off, 2ull * (e->stage_launch_cap + 1ull)));
-  A_(dmalloc(&e->d_in_faults, 2ull * e->stage_fault_cap));
+  // host-pointer inputs are uploaded here on the ingest stream (in order with
+  // the ingest that reads them)
+  A_(dmalloc(&e->d_in_hash, e->stage_launch_cap));
+  A_(dmalloc(&e->d_in_off, e->stage_launch_cap + 1ull));
+  A_(dmalloc(&e->d_in_faults, e->stage_fault_cap));
   A_(cudaStreamCreateWithFlags(&e->rec_s, cudaStreamNonBlocking));
-  e->copy_s = e->rec_s;
   A_(cudaEventCreateWithFlags(&e->ev_rec, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_s_now, cudaEventDisableTiming));
   for (int b = 0; b < 2; ++b) A_(cudaEventCreateWithFlags(&e->ev_stage_free[b], cudaEventDisableTiming));
-  for (int b = 0; b < 2; ++b) {
-    A_(cudaEventCreateWithFlags(&e->ev_in_ready[b], cudaEventDisableTiming));
-    A_(cudaEventCreateWithFlags(&e->ev_in_free[b], cudaEventDisableTiming));
-  }
   A_(dmalloc(&e->d_stage_hash, 2ull * e->stage_launch_cap));
   A_(dmalloc(&e->d_stage_norm, 2ull * e->stage_fault_cap));
   A_(dmalloc(&e->d_stage_cnt, 2ull * e->stage_launch_cap));

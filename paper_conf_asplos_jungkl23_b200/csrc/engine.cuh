@@ -143,16 +143,13 @@ struct dum_engine {
   // staging
   uint32_t stage_launch_cap;
   uint64_t stage_fault_cap;
-  uint64_t *d_in_hash, *d_in_off;   // host-pointer inputs are copied here (two buffers, alternating)
-  cudaStream_t copy_s;              // uploads of host-pointer inputs (== rec_s)
+  uint64_t *d_in_hash, *d_in_off;   // host-pointer inputs are uploaded here (on rec_s)
   // record_faults runs on its own stream so that the next batch's ingest
   // overlaps the current build; the staging arrays alternate between two sets
   cudaStream_t rec_s;
   cudaEvent_t ev_rec, ev_s_now, ev_stage_free[2];
   int stage_set;
   void *stage_base[6];              // the two-set allocations behind d_stage_*
-  cudaEvent_t ev_in_ready[2], ev_in_free[2];
-  int in_buf;
   uint32_t *d_in_faults;
   uint64_t *d_stage_hash;
   uint32_t *d_stage_norm, *d_stage_cnt, *d_stage_exec, *d_stage_slot;
