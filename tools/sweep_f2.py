@@ -50,7 +50,8 @@ def run(tr, geo, N, it_eval, dev):
     K = tr.K
     eng = Engine(num_rows=R, assoc=A, num_succs=S, degree_n=N, max_blocks=tr.W, max_exec_ids=8192,
                  hbm_frames=tr.C, device=dev.index or 0, corr_capacity=1 << 16,
-                 max_batch_faults=max(1 << 20, int(max(tr.faults_in_iteration(i) for i in range(tr.n_iter)) * 1.2)),
+                 max_batch_faults=max(1 << 22,  # also sizes predict's hash pool (4x) for long N=64 windows
+                                       int(max(tr.faults_in_iteration(i) for i in range(tr.n_iter)) * 1.2)),
                  max_batch_launches=max(2 * K, 4096))
     exec_all = torch.full((tr.n_iter * K + 3,), -1, dtype=torch.int32, device=dev)
     for i in range(it_eval):
