@@ -43,3 +43,31 @@ def test_score_perfect_and_partial_windows():
     # empty windows score 0 / 0 without dividing by zero
     p, r, w = sweep_f2.score(norm, np.zeros(0, np.uint32), np.zeros((tr.K, 2), np.int64), 1, tr.K)
     assert (p, r, w) == (0.0, 0.0, 0.0)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("name,N", [("Config0", 1), ("Config9", 4), ("Config11", 2)])
+def test_sweep_windows_match_oracle_on_T(name, N):
+    """The sweep's engine path (record/build of iterations 0..i-1, then the
+    transition windows of iteration i through the C-ABI) emits the oracle's
+    windows, so its precision/recall are the oracle's."""
+    import torch
+    import oracle as orc
+    from gpu_helpers import transition_queries
+    A, S, R = sweep_f2.TABLE6[name]
+    tr = wl.make_T(n_iter=3, dup_ppm=200_000)
+    pairs_g, rng_g, _, n_exec, _ = sweep_f2.run(tr, (A, S, R), N, 2, torch.device("cuda", 0))
+    o = orc.Oracle(R=R, A=A, S=S, N=N, W=tr.W, C=tr.C)
+    ex = []
+    for i in range(3):
+        ex += [int(x) for x in o.record_faults(*tr.iteration(i))]
+        if i < 2:
+            o.build_tables()
+    off, pairs_o, _, _ = o.predict(transition_queries(ex, 2 * tr.K, tr.K, N))
+    assert n_exec == o.num_exec
+    for k in range(tr.K):
+        assert pairs_g[int(rng_g[k, 0]):int(rng_g[k, 1])].tolist() == \
+            pairs_o[int(off[k]):int(off[k + 1]), 0].tolist(), (name, N, k)
+    norm = sweep_f2.normalised(tr, 2)
+    rng_o = np.stack([off[:-1], off[1:]], axis=1).astype(np.int64)
+    assert sweep_f2.score(norm, pairs_g, rng_g, N, tr.K) == sweep_f2.score(norm, pairs_o[:, 0], rng_o, N, tr.K)
