@@ -32,8 +32,10 @@
  *   - Return 0 (DUM_OK) or a negative DUM_E* code; dum_last_error() has text.
  *   - All calls are asynchronous and stream-ordered on the given CUDA stream
  *     (cudaStream_t passed as dum_stream_t), except dum_create, dum_destroy,
- *     dum_dump_state, dum_sync, dum_get_stats, dum_read_counters and
- *     dum_read_timing, which synchronize.
+ *     dum_dump_state, dum_sync, dum_get_stats, dum_read_counters,
+ *     dum_read_timing and dum_migrate_blocks with method 2 (copy engines:
+ *     the frame plan is read back to the host before the copies are
+ *     issued), which synchronize.
  *   - Ownership: the caller owns every input/output buffer and must keep it
  *     valid until the stream work completes; the engine owns all tables,
  *     residency state and scratch (device memory on cfg.device).
@@ -124,12 +126,14 @@ int dum_reset(dum_engine *eng, dum_stream_t stream);
  * applied by the next dum_build_tables.  With DUM_HOST_PTRS the launch
  * offsets are validated on the host (DUM_EINVAL); block ids >= max_blocks are
  * detected on the device for both kinds of pointers (sticky DUM_EINVAL from
- * dum_sync; the offending records are dropped).  DUM_HOST_PTRS uploads run on
- * the engine's copy stream into one of two staging buffers (the upload of the
- * next batch overlaps the kernels of this one) and `stream` waits for them:
- * pinned host inputs must stay unmodified until the call's work on `stream`
- * has completed, exactly like device inputs (pageable inputs are staged by
- * the CUDA runtime before the call returns). */
+ * dum_sync; the offending records are dropped); so are device-side launch
+ * offsets that are not monotone or run past n_fault (sticky DUM_EINVAL, the
+ * launch is dropped).  DUM_HOST_PTRS uploads run on the engine's ingest stream
+ * into a single upload buffer, in order with the ingest kernels that read it
+ * (the ingest of this batch may overlap the build of the previous one), and
+ * `stream` waits for the ingest: pinned host inputs must stay unmodified until
+ * the call's work on `stream` has completed, exactly like device inputs
+ * (pageable inputs are staged by the CUDA runtime before the call returns). */
 int dum_record_faults(dum_engine *eng, const uint64_t *launch_hash, const uint64_t *launch_off,
                       uint32_t n_launch, const uint32_t *fault_block, uint64_t n_fault,
                       uint32_t *out_exec, uint32_t flags, dum_stream_t stream);

@@ -43,7 +43,7 @@ H2D, D2H, INVALIDATE, D2D = 0, 1, 2, 3
 def build() -> str:
     """Compile the oracle (plain g++, no CUDA)."""
     tmp = _SO + ".tmp%d" % os.getpid()
-    subprocess.check_call(["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-o", tmp, _SRC])
+    subprocess.check_call(["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-pthread", "-o", tmp, _SRC])
     os.replace(tmp, _SO)
     return _SO
 
@@ -74,6 +74,7 @@ def _lib() -> ctypes.CDLL:
     L.orc_free_frames.argtypes = [P]
     L.orc_free_frames.restype = U32
     L.orc_dump.argtypes = [P, U32, P, U64, P]
+    L.orc_set_threads.argtypes = [P, U32]
     _LIB = L
     return L
 
@@ -99,11 +100,19 @@ class Oracle:
     PAPER.md Table 6 (L429-L443); default Config9 = 2048/2/4 (L303)."""
 
     def __init__(self, R: int = 2048, A: int = 2, S: int = 4, N: int = 32, W: int = 256, C: int = 128,
-                 row_index: int = 0):
+                 row_index: int = 0, threads: int = 1):
         self.R, self.A, self.S, self.N, self.W, self.C = R, A, S, N, W, C
         self._h = _lib().orc_create(R, A, S, N, W, C, row_index)
         if not self._h:
             raise OracleError("bad geometry")
+        self._cap_hint = 1 << 16
+        self.set_threads(threads)
+
+    def set_threads(self, n: int) -> None:
+        """predict / select split their (independent) queries over n threads;
+        the outputs are identical for every n (concatenated in query order)."""
+        self.threads = max(1, int(n))
+        _lib().orc_set_threads(self._h, self.threads)
 
     def __del__(self):
         h = getattr(self, "_h", None)
@@ -137,13 +146,14 @@ class Oracle:
         ko = np.zeros((max(nq, 1), self.N + 2), dtype=np.uint32)
         ch = np.zeros((max(nq, 1), self.N + 1), dtype=np.uint32)
         need = np.zeros(1, dtype=np.uint64)
-        cap = 1 << 16
+        cap = self._cap_hint
         while True:
-            pairs = np.zeros((cap, 2), dtype=np.uint32)
+            pairs = np.empty((cap, 2), dtype=np.uint32)
             rc = _lib().orc_predict(self._h, _p(q), nq, _p(off), _p(pairs), cap, _p(ko), _p(ch), _p(need))
             if rc == 0:
                 return off, pairs[: int(need[0])], ko[:nq], ch[:nq]
             cap = int(need[0]) + 1
+            self._cap_hint = max(self._cap_hint, cap)
 
     # a8
     def select(self, qoff, pairs, anchors=None):
@@ -154,15 +164,16 @@ class Oracle:
         wb_off = np.zeros(nq + 1, dtype=np.uint64)
         inv_off = np.zeros(nq + 1, dtype=np.uint64)
         need = np.zeros(1, dtype=np.uint64)
-        cap = 1 << 16
+        cap = self._cap_hint
         while True:
-            wb = np.zeros(cap, dtype=np.uint32)
-            inv = np.zeros(cap, dtype=np.uint32)
+            wb = np.empty(cap, dtype=np.uint32)
+            inv = np.empty(cap, dtype=np.uint32)
             rc = _lib().orc_select(self._h, _p(qoff), _p(pr) if len(pr) else _p(np.zeros(2, np.uint32)), nq,
                                    _p(an), _p(wb), _p(wb_off), _p(inv), _p(inv_off), cap, _p(need))
             if rc == 0:
                 return wb_off, wb[: int(wb_off[-1])], inv_off, inv[: int(inv_off[-1])]
             cap = int(need[0]) + 1
+            self._cap_hint = max(self._cap_hint, cap)
 
     def mark_inactive(self, blocks, inactive: bool = True) -> None:
         b = _u32(blocks)

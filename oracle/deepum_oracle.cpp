@@ -28,6 +28,7 @@
 #include <cstring>
 #include <map>
 #include <set>
+#include <thread>
 #include <unordered_map>
 #include <unordered_set>
 #include <vector>
@@ -77,6 +78,7 @@ struct Oracle {
   std::vector<uint8_t> inactive;
   std::set<uint32_t> free_frames;
   uint64_t mig_counter = 0;
+  uint32_t threads = 1;                          // predict/select query ranges per thread (orc_set_threads)
 
   uint32_t idx(uint32_t b) const {               // D7
     if (row_index == 1) {
@@ -505,18 +507,40 @@ uint32_t orc_num_exec(void *h) { return (uint32_t)static_cast<Oracle *>(h)->exec
 int orc_predict(void *h, const uint32_t *q, uint32_t nq, uint64_t *out_off, uint32_t *out_pairs,
                 uint64_t cap_pairs, uint32_t *kern_off, uint32_t *chain, uint64_t *needed) {
   Oracle *o = static_cast<Oracle *>(h);
-  std::vector<uint32_t> pairs, ko, ch;
+  // queries are independent pure functions of the state (no ordering between
+  // them): with threads > 1 contiguous query ranges run on separate threads
+  // and their outputs are concatenated in query order -- the same bytes.
+  const uint32_t T = std::max<uint32_t>(1, std::min<uint32_t>(o->threads, nq ? nq : 1));
+  std::vector<std::vector<uint32_t>> pairs(T);
+  std::vector<std::vector<uint64_t>> cnt(T);
+  auto run = [&](uint32_t t) {
+    const uint32_t a = (uint64_t)nq * t / T, b = (uint64_t)nq * (t + 1) / T;
+    std::vector<uint32_t> ko, ch;
+    for (uint32_t i = a; i < b; ++i) {
+      const uint32_t *x = q + 6 * i;
+      o->predict_one(x[0], x[1], x[2], x[3], x[4], std::min(x[5], o->N), pairs[t], ko, ch);
+      cnt[t].push_back(pairs[t].size() / 2);
+      std::memcpy(kern_off + (uint64_t)i * (o->N + 2), ko.data(), 4 * (o->N + 2));
+      std::memcpy(chain + (uint64_t)i * (o->N + 1), ch.data(), 4 * (o->N + 1));
+    }
+  };
+  std::vector<std::thread> th;
+  for (uint32_t t = 1; t < T; ++t) th.emplace_back(run, t);
+  run(0);
+  for (auto &x : th) x.join();
   out_off[0] = 0;
-  for (uint32_t i = 0; i < nq; ++i) {
-    const uint32_t *x = q + 6 * i;
-    o->predict_one(x[0], x[1], x[2], x[3], x[4], std::min(x[5], o->N), pairs, ko, ch);
-    out_off[i + 1] = pairs.size() / 2;
-    std::memcpy(kern_off + (uint64_t)i * (o->N + 2), ko.data(), 4 * (o->N + 2));
-    std::memcpy(chain + (uint64_t)i * (o->N + 1), ch.data(), 4 * (o->N + 1));
+  uint64_t base = 0, i = 0;
+  for (uint32_t t = 0; t < T; ++t) {
+    for (uint64_t c : cnt[t]) out_off[++i] = base + c;
+    base += pairs[t].size() / 2;
   }
-  *needed = pairs.size() / 2;
-  if (pairs.size() / 2 > cap_pairs) return ORC_ECAPACITY;
-  std::memcpy(out_pairs, pairs.data(), 4 * pairs.size());
+  *needed = base;
+  if (base > cap_pairs) return ORC_ECAPACITY;
+  uint64_t w = 0;
+  for (uint32_t t = 0; t < T; ++t) {
+    if (!pairs[t].empty()) std::memcpy(out_pairs + w, pairs[t].data(), 4 * pairs[t].size());
+    w += pairs[t].size();
+  }
   return ORC_OK;
 }
 
@@ -525,20 +549,45 @@ int orc_predict(void *h, const uint32_t *q, uint32_t nq, uint64_t *out_off, uint
 int orc_select(void *h, const uint64_t *qoff, const uint32_t *pairs, uint32_t nq, const uint32_t *anchors,
                uint32_t *wb, uint64_t *wb_off, uint32_t *inv, uint64_t *inv_off, uint64_t cap, uint64_t *needed) {
   Oracle *o = static_cast<Oracle *>(h);
-  std::vector<uint32_t> W, I;
+  const uint32_t T = std::max<uint32_t>(1, std::min<uint32_t>(o->threads, nq ? nq : 1));
+  std::vector<std::vector<uint32_t>> W(T), I(T);
+  std::vector<std::vector<std::pair<uint64_t, uint64_t>>> cnt(T);
+  auto run = [&](uint32_t t) {
+    const uint32_t a = (uint64_t)nq * t / T, b = (uint64_t)nq * (t + 1) / T;
+    for (uint32_t i = a; i < b; ++i) {
+      o->select_one(pairs + 2 * qoff[i], qoff[i + 1] - qoff[i], anchors ? anchors[i] : NONE, W[t], I[t]);
+      cnt[t].push_back({W[t].size(), I[t].size()});
+    }
+  };
+  std::vector<std::thread> th;
+  for (uint32_t t = 1; t < T; ++t) th.emplace_back(run, t);
+  run(0);
+  for (auto &x : th) x.join();
   wb_off[0] = 0;
   inv_off[0] = 0;
-  for (uint32_t i = 0; i < nq; ++i) {
-    o->select_one(pairs + 2 * qoff[i], qoff[i + 1] - qoff[i], anchors ? anchors[i] : NONE, W, I);
-    wb_off[i + 1] = W.size();
-    inv_off[i + 1] = I.size();
+  uint64_t bw = 0, bi = 0, i = 0;
+  for (uint32_t t = 0; t < T; ++t) {
+    for (auto &c : cnt[t]) {
+      ++i;
+      wb_off[i] = bw + c.first;
+      inv_off[i] = bi + c.second;
+    }
+    bw += W[t].size();
+    bi += I[t].size();
   }
-  *needed = std::max(W.size(), I.size());
-  if (W.size() > cap || I.size() > cap) return ORC_ECAPACITY;
-  std::memcpy(wb, W.data(), 4 * W.size());
-  std::memcpy(inv, I.data(), 4 * I.size());
+  *needed = std::max(bw, bi);
+  if (bw > cap || bi > cap) return ORC_ECAPACITY;
+  uint64_t pw = 0, pi = 0;
+  for (uint32_t t = 0; t < T; ++t) {
+    if (!W[t].empty()) std::memcpy(wb + pw, W[t].data(), 4 * W[t].size());
+    if (!I[t].empty()) std::memcpy(inv + pi, I[t].data(), 4 * I[t].size());
+    pw += W[t].size();
+    pi += I[t].size();
+  }
   return ORC_OK;
 }
+
+void orc_set_threads(void *h, uint32_t n) { static_cast<Oracle *>(h)->threads = n ? n : 1; }
 
 int orc_mark_inactive(void *h, const uint32_t *blocks, uint32_t n, int flag) {
   Oracle *o = static_cast<Oracle *>(h);

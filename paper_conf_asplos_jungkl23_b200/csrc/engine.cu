@@ -105,6 +105,10 @@ int reset_state(dum_engine *e, cudaStream_t s) {
   k_init_state<<<1, 1, 0, s>>>(e->d_state);
   CK(cudaGetLastError());
   CK(launch_reset_residency(e, s));
+  // the ingest stream waits for the reset: a following dum_record_faults with
+  // DUM_HOST_PTRS / DUM_INPUTS_READY does not order itself after `s`
+  CK(cudaEventRecord(e->ev_s_now, s));
+  CK(cudaStreamWaitEvent(e->rec_s, e->ev_s_now, 0));
   e->n_staged = 0;
   e->staged_faults = 0;
   e->launches = 0;
@@ -164,15 +168,6 @@ TimerScope::TimerScope(dum_engine *e_, int id_, cudaStream_t s_) : e(e_), id(id_
 }
 TimerScope::~TimerScope() {
   if (b) cudaEventRecord(b, s);
-  static const bool sync_each = getenv("DUM_SYNC_EACH") != nullptr;
-  if (sync_each) {
-    cudaError_t err = cudaStreamSynchronize(s);
-    if (err == cudaSuccess) err = cudaGetLastError();
-    if (err != cudaSuccess) {
-      fprintf(stderr, "DUM_SYNC_EACH: kernel timer id %d failed: %s\n", id, cudaGetErrorString(err));
-      fflush(stderr);
-    }
-  }
 }
 }  // namespace dum
 
@@ -255,12 +250,8 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   {
     // jump tables (k_jump.cu) overlap the block-table apply/walk here.  Normal
     // priority: a high-priority side stream stalled the main stream by
-    // ~100 us per step when steps are issued back to back (measured,
-    // tools/e2e_diag.py); DUM_JUMP_MODE=0 restores it for experiments
-    int lo = 0, hi = 0;
-    cudaDeviceGetStreamPriorityRange(&lo, &hi);
-    const char *jm = getenv("DUM_JUMP_MODE");
-    A_(cudaStreamCreateWithPriority(&e->side, cudaStreamNonBlocking, (jm && jm[0] == '0') ? hi : lo));
+    // ~100 us per step when steps are issued back to back (measured in round 1)
+    A_(cudaStreamCreateWithFlags(&e->side, cudaStreamNonBlocking));
   }
   A_(cudaEventCreateWithFlags(&e->ev_fork, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_join, cudaEventDisableTiming));
@@ -441,7 +432,7 @@ int dum_record_faults(dum_engine *e, const uint64_t *launch_hash, const uint64_t
     o = doff;
     f = df;
   }
-  CK(launch_record(e, h, o, n_launch, f, out_exec, r));
+  CK(launch_record(e, h, o, n_launch, f, n_fault, out_exec, r));
   CK(cudaEventRecord(e->ev_rec, r));
   CK(cudaStreamWaitEvent(s, e->ev_rec, 0));
   e->n_staged += n_launch;

@@ -208,5 +208,5 @@ struct dum_engine {
   std::vector<cudaEvent_t> event_pool;
   double t_ms[DUM_NTIMERS];
   uint64_t t_cnt[DUM_NTIMERS];
-  int predict_smem, select_smem, build_smem;
+  int predict_smem, select_smem, build_smem, ingest_smem;  // dynamic smem attributes applied (per engine / device)
 };

@@ -257,19 +257,7 @@ struct BuildArgs {
   const uint32_t *order;       // [3][n_staged] faulting launches by size class
   unsigned long long *plan_agg;  // [k_plan CTAs] published chunk totals (flag << 63 | leads << 32 | items)
   DevState *st;
-  unsigned long long *clk;     // debug (DUM_BUILD_CLOCK): per apply item / walk item 4 x u64, or null
 };
-
-__device__ __forceinline__ unsigned long long gtimer() {
-  unsigned long long t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-  return t;
-}
-__device__ __forceinline__ uint32_t smid() {
-  uint32_t r;
-  asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
-  return r;
-}
 
 __global__ void __launch_bounds__(PLAN_NT) k_plan(BuildArgs a) {
   __shared__ uint32_t ws[PLAN_NT / 32];
@@ -420,7 +408,6 @@ __global__ void __launch_bounds__(AP_NT) k_apply(BuildArgs a) {
     const uint32_t c = it.y & 0xFFFFu, P = it.y >> 16;
     const LeadDesc d = a.desc[it.x];
     const uint32_t e = d.e;
-    const unsigned long long t0 = a.clk ? gtimer() : 0;
     uint32_t ng = 1;
     if (d.single) {  // the common case: no list to chase
       if (tid == 0) {
@@ -558,13 +545,6 @@ __global__ void __launch_bounds__(AP_NT) k_apply(BuildArgs a) {
       m = P == 1 ? m + min(AP_SCAN, n_ops - g0) : s_m;
     }
     if (m) apply_staged();
-    if (a.clk && tid == 0) {
-      unsigned long long *c4 = a.clk + 4ull * t;
-      c4[0] = t0;
-      c4[1] = gtimer();
-      c4[2] = smid() | ((unsigned long long)blockIdx.x << 32);
-      c4[3] = n_ops | ((unsigned long long)P << 32);
-    }
   }
   // one global atomic per CTA (a per-thread atomic on one address serialises
   // hundreds of thousands of updates in L2)
@@ -615,12 +595,6 @@ __global__ void __launch_bounds__(WK_NT) k_walk(BuildArgs a) {
     const uint64_t off = d.off_last;
     const uint32_t *C = a.stage_norm + off;
     const uint32_t start = C[0], end = C[n - 1];
-    unsigned long long *c4 = a.clk ? a.clk + 4ull * (a.st->n_items + li) : nullptr;
-    if (c4 && tid == 0) {
-      c4[0] = gtimer();
-      c4[2] = smid() | ((unsigned long long)blockIdx.x << 32);
-      c4[3] = n;
-    }
     if (tid == 0) {
       a.start_end[2 * e] = start;
       a.start_end[2 * e + 1] = end;
@@ -643,7 +617,6 @@ __global__ void __launch_bounds__(WK_NT) k_walk(BuildArgs a) {
         wrun[0] = make_uint2(start >> 5, 1u << (start & 31));
         a.wrun_len[e] = 1;
         ctr_add(a.st, DUM_CTR_WALK_OUT, 1);
-        if (c4) c4[1] = gtimer();
       }
       break;
     }
@@ -748,7 +721,6 @@ __global__ void __launch_bounds__(WK_NT) k_walk(BuildArgs a) {
         a.wrun_len[e] = s_nrun;
         ctr_add(a.st, DUM_CTR_WALK_ROWS, t + 1);
         ctr_add(a.st, DUM_CTR_WALK_OUT, qlen);
-        if (c4) c4[1] = gtimer();
       }
       break;
     }
@@ -845,7 +817,6 @@ __global__ void __launch_bounds__(WK_NT) k_walk(BuildArgs a) {
       a.wrun_len[e] = s_nrun;
       ctr_add(a.st, DUM_CTR_WALK_ROWS, t + 1);
       ctr_add(a.st, DUM_CTR_WALK_OUT, outn);
-      if (c4) c4[1] = gtimer();
     }
   } while (false);
 }
@@ -892,11 +863,11 @@ __global__ void k_walk_slow(Geo g, const uint32_t *tbl, const uint32_t *start_en
 
 template <int MA, int MS>
 static cudaError_t launch_apply_walk(dum_engine *e, const BuildArgs &ba, cudaStream_t s) {
-  static bool init = false;
   const size_t wsmem = (size_t)(WK_RC + WK_CQ + 2 * WK_QCAP) * 4;
-  if (!init) {
+  // the attribute is per device and function: raised by every engine on its own device
+  if (!e->build_smem) {
     cudaFuncSetAttribute(k_walk<MA, MS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)wsmem);
-    init = true;
+    e->build_smem = (int)wsmem;
   }
   // host upper bounds of the device-side counts (the surplus CTAs return at once):
   // items = sum over exec IDs of ceil(ops / OPP) <= launches + faults / OPP
@@ -940,16 +911,6 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   ba.order = e->d_order;
   ba.plan_agg = reinterpret_cast<unsigned long long *>(e->d_plan_agg);
   ba.st = e->d_state;
-  ba.clk = nullptr;
-  static const char *clk_path = getenv("DUM_BUILD_CLOCK");
-  static unsigned long long *d_clk = nullptr;
-  static int clk_calls = 0;
-  const uint64_t clk_n = 4ull * (e->items_cap + e->stage_launch_cap);
-  if (clk_path) {
-    if (!d_clk) cudaMalloc(&d_clk, 8 * clk_n);
-    cudaMemsetAsync(d_clk, 0, 8 * clk_n, s);
-    ba.clk = d_clk;
-  }
   {
     TimerScope t(e, DUM_T_BUILD_PREP, s);
     k_build_prep<<<(n + 255) / 256, 256, 0, s>>>(n, (uint32_t)e->built_launches, e->d_stage_exec, e->d_stage_cnt,
@@ -958,11 +919,7 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
     k_plan<<<(n + PLAN_NT - 1) / PLAN_NT, PLAN_NT, 0, s>>>(ba);
   }
   // the jump tables depend only on the correlation table, final here
-  static const char *jm = getenv("DUM_JUMP_MODE");
-  if (jm && jm[0] == '2') {
-    const cudaError_t je = launch_jump_tables(e, s);
-    if (je != cudaSuccess) return je;
-  } else {
+  {
     cudaEventRecord(e->ev_fork, s);
     cudaStreamWaitEvent(e->side, e->ev_fork, 0);
     const cudaError_t je = launch_jump_tables(e, e->side);
@@ -987,20 +944,6 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   // end of this call; the next reader of the correlation table (predict's
   // k_chain, the next build, reset) waits for ev_join
   e->kernel_launches += 5;
-  if (clk_path) {  // [n_items | n_leads] header, then the stamps
-    DevState hs;
-    cudaStreamSynchronize(s);
-    cudaMemcpy(&hs, e->d_state, sizeof(hs), cudaMemcpyDeviceToHost);
-    std::vector<unsigned long long> h(4ull * (hs.n_items + hs.n_leads) + 1);
-    h[0] = hs.n_items | ((unsigned long long)hs.n_leads << 32);
-    cudaMemcpy(h.data() + 1, d_clk, 8 * (h.size() - 1), cudaMemcpyDeviceToHost);
-    char fn[512];
-    snprintf(fn, sizeof fn, "%s.%d", clk_path, clk_calls++);
-    if (FILE *f = fopen(fn, "wb")) {
-      fwrite(h.data(), 8, h.size(), f);
-      fclose(f);
-    }
-  }
   return cudaGetLastError();
 }
 

@@ -443,14 +443,16 @@ cudaError_t launch_migrate(dum_engine *e, int dir, const uint32_t *blocks, const
     cudaError_t err = cudaStreamSynchronize(s);
     if (err != cudaSuccess) return err;
     DevState hs;
-    cudaMemcpy(&hs, e->d_state, sizeof(hs), cudaMemcpyDeviceToHost);
+    if ((err = cudaMemcpy(&hs, e->d_state, sizeof(hs), cudaMemcpyDeviceToHost)) != cudaSuccess) return err;
     if (!hs.mig_ok) return cudaSuccess;
     const uint32_t m = hs.mig_n;
     std::vector<uint32_t> fr(m), bl(m), sr(m);
     if (m) {
-      cudaMemcpy(fr.data(), e->d_mig_frames, 4ull * m, cudaMemcpyDeviceToHost);
-      cudaMemcpy(bl.data(), e->d_mig_blocks, 4ull * m, cudaMemcpyDeviceToHost);
-      if (dir == DUM_D2D) cudaMemcpy(sr.data(), e->d_mig_src, 4ull * m, cudaMemcpyDeviceToHost);
+      if ((err = cudaMemcpy(fr.data(), e->d_mig_frames, 4ull * m, cudaMemcpyDeviceToHost)) != cudaSuccess) return err;
+      if ((err = cudaMemcpy(bl.data(), e->d_mig_blocks, 4ull * m, cudaMemcpyDeviceToHost)) != cudaSuccess) return err;
+      if (dir == DUM_D2D &&
+          (err = cudaMemcpy(sr.data(), e->d_mig_src, 4ull * m, cudaMemcpyDeviceToHost)) != cudaSuccess)
+        return err;
     }
     uint32_t i = 0;
     while (i < m) {

@@ -129,15 +129,8 @@ struct PredArgs {
   uint32_t *big_pool;         // scratch for the exact slow path
   uint64_t big_entries;
   SelectOut so;     // fused a8 outputs (SELECT only)
-  unsigned long long *cta_clk;  // debug (DUM_CTA_CLOCK): per CTA 8 x u64 timestamps, or null
   uint64_t *needed;             // pair-pool size after every reservation (k_chain's last CTA), or null
 };
-
-__device__ __forceinline__ unsigned long long pred_timer() {
-  unsigned long long t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-  return t;
-}
 
 constexpr int CHAIN_WARPS = 8;
 constexpr int NQCLS = 5;  // window-size classes of the predict CTA order
@@ -329,13 +322,6 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
   const bool anchored = anchor != NONE;
   const uint32_t nk = a.qnk[qi];
   const unsigned long long base = a.qbase[qi];
-  unsigned long long *clk = a.cta_clk ? a.cta_clk + 12ull * qi : nullptr;
-  if (clk && tid == 0) {
-    unsigned int smid;
-    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-    clk[0] = pred_timer();
-    clk[7] = smid;
-  }
   for (uint32_t w = tid; w < (a.nwords + 3) / 4; w += PRED_NT) sm4[w] = make_uint4(0, 0, 0, 0);
   for (uint32_t d = tid; d <= nk; d += PRED_NT) {
     loff[d] = a.qloff[(uint64_t)qi * (g.N + 2) + d];
@@ -353,7 +339,6 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
   __syncthreads();
   const uint32_t U = nk ? loff[nk] : 0;
   const bool ok = base + U <= a.cap;
-  if (clk && tid == 0) clk[1] = pred_timer();
   const uint32_t *apool = a.anchor_pool + (anchored ? a.anchor_range[2 * qi] : 0);
   auto list_of = [&](uint32_t d) -> const uint32_t * {
     return (d == 0 && anchored) ? apool : a.walk + (uint64_t)kern[d] * g.walk_cap;
@@ -484,7 +469,6 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
     }
   }
   __syncthreads();
-  if (clk && tid == 0) clk[2] = pred_timer();
   // Duplicates are known now: without them (the normal case) warps
   // [0, GRP_W) run the selection (a8) while the others stream the pairs; with
   // them the whole CTA takes the duplicate path below instead.
@@ -495,15 +479,12 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
       {
         if (tid == 0) select_reserve(a.so, s_nonres, a.st, ss);
         group_sync<1, GRP_NT>();
-        if (clk && tid == 0) clk[3] = pred_timer();
         select_tail<GRP_NT, 1>(a.so, qi, ss, bitmap, a.st, tid, dk);
       }
-      if (clk && tid == 0) clk[4] = pred_timer();
     } else if (ok) {
       copy_lists(wid - GRP_W, NWARP - GRP_W, loff, nullptr);
     }
   }
-  if (clk && tid == GRP_NT) clk[5] = pred_timer();
   __syncthreads();
   const uint32_t ndup = s_ndup;
   uint32_t run = U;
@@ -631,7 +612,6 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
         copy_lists(wid, NWARP, noff, kcnt);
       }
       if (SELECT && tid == 0) s_nonres -= s_dnr;
-      if (clk && tid == 0) clk[8] = pred_timer();
     } else {
       // ---------------- fallback: min-position hash over every element ----------------
       const uint32_t hcap = pow2ceil(2 * (U + 1));
@@ -699,14 +679,12 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
       } else {
         run = 0;
       }
-      if (clk && tid == 0) clk[9] = pred_timer();
     }
     __syncthreads();
     if (SELECT) {
       if (tid == 0) select_reserve(a.so, s_nonres, a.st, ss);
       __syncthreads();
       select_tail<PRED_NT, 0>(a.so, qi, ss, bitmap, a.st, tid, dk);
-      if (clk && tid == 0) clk[11] = pred_timer();
     }
   }
   if (tid == 0) {
@@ -736,7 +714,6 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
     uint32_t *ch = a.chain + (uint64_t)qi * (g.N + 1);
     for (uint32_t d = tid; d <= g.N; d += PRED_NT) ch[d] = d < nk ? kern[d] : NONE;
   }
-  if (clk && tid == 0) clk[6] = pred_timer() | ((unsigned long long)(ndup != 0) << 63);
 }
 
 // the call's bump pointers and k_chain's class counters
@@ -816,16 +793,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   } else {
     a.so.res_bits = e->d_res_bits;
   }
-  a.cta_clk = nullptr;
   a.needed = needed;
-  static const char *clk_path = getenv("DUM_PRED_CLOCK");
-  static unsigned long long *d_clk = nullptr;
-  static int clk_calls = 0;
-  if (clk_path) {
-    if (!d_clk) cudaMalloc(&d_clk, 12ull * 8 * e->anchor_range_cap);
-    cudaMemsetAsync(d_clk, 0, 12ull * 8 * nq, s);
-    a.cta_clk = d_clk;
-  }
   cudaStreamWaitEvent(s, e->ev_join, 0);  // jump tables of the last build (side stream)
   {
     TimerScope t(e, DUM_T_CHAIN, s);
@@ -833,34 +801,22 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   }
   const size_t smem = (size_t)((a.nwords + 3) & ~3u) * 4 + 2 * DHCAP * 4;
   if (sel) {
-    static size_t set_smem = 0;  // the attribute is per function: raise it once per size
-    if (smem > set_smem) {
+    // the attribute is per device and function: raised by every engine on its own device
+    if ((int)smem > e->select_smem) {
       cudaFuncSetAttribute(k_predict<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      set_smem = smem;
+      e->select_smem = (int)smem;
     }
     TimerScope t(e, DUM_T_PREDICT, s);
     k_predict<true><<<nq, PRED_NT, smem, s>>>(a);
   } else {
-    static size_t set_smem = 0;
-    if (smem > set_smem) {
+    if ((int)smem > e->predict_smem) {
       cudaFuncSetAttribute(k_predict<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      set_smem = smem;
+      e->predict_smem = (int)smem;
     }
     TimerScope t(e, DUM_T_PREDICT, s);
     k_predict<false><<<nq, PRED_NT, smem, s>>>(a);
   }
   e->kernel_launches += 3;
-  if (clk_path) {
-    std::vector<unsigned long long> h(12ull * nq);
-    cudaStreamSynchronize(s);
-    cudaMemcpy(h.data(), d_clk, 12ull * 8 * nq, cudaMemcpyDeviceToHost);
-    char fn[512];
-    snprintf(fn, sizeof fn, "%s.%d", clk_path, clk_calls++);
-    if (FILE *f = fopen(fn, "wb")) {
-      fwrite(h.data(), 8, h.size(), f);
-      fclose(f);
-    }
-  }
   if (sel && sel_needed) {
     k_copy_counters2<<<1, 1, 0, s>>>(&e->d_state->pool_wb, &e->d_state->pool_inv, sel_needed);
     e->kernel_launches += 1;

@@ -29,13 +29,18 @@ __global__ void __launch_bounds__(INGEST_NT) k_ingest(
     uint64_t *__restrict__ stage_off, uint32_t *__restrict__ stage_norm, uint32_t *__restrict__ stage_cnt,
     uint32_t *__restrict__ stage_slot, unsigned long long *exec_keys, uint32_t *exec_vals, uint32_t *exec_minpos,
     uint32_t exec_cap, uint32_t *big_pool, uint64_t big_entries, uint32_t bm_words, uint32_t *__restrict__ stage_exec,
-    uint32_t *__restrict__ out_exec, uint32_t *__restrict__ pend, uint32_t Emax, DevState *st) {
+    uint32_t *__restrict__ out_exec, uint32_t *__restrict__ pend, uint32_t Emax, uint64_t n_fault, DevState *st) {
   extern __shared__ uint32_t dyn[];  // hash (2 x INGEST_HCAP) or bitmap + small dup hash
   __shared__ uint32_t ws[INGEST_NT / 32];
   __shared__ uint32_t s_dups, s_ovf;
   const uint32_t i = blockIdx.x;
   if (i >= n_launch) return;
-  const uint64_t a = off[i], b = off[i + 1];
+  uint64_t a = off[i], b = off[i + 1];
+  if (b < a || b > n_fault || (i == 0 && a != 0)) {
+    // offsets not monotone / past the batch: the launch is dropped (sticky EINVAL)
+    if (threadIdx.x == 0) set_err(st, ERR_EINVAL);
+    a = b = 0;
+  }
   const uint32_t n = (uint32_t)(b - a);
   if (threadIdx.x == 0) {
     stage_hash[l0 + i] = hash[i];
@@ -326,7 +331,7 @@ __global__ void __launch_bounds__(ASSIGN_NT) k_exec_assign(
 }
 
 cudaError_t launch_record(dum_engine *e, const uint64_t *hash, const uint64_t *off, uint32_t n_launch,
-                          const uint32_t *faults, uint32_t *out_exec, cudaStream_t s) {
+                          const uint32_t *faults, uint64_t n_fault, uint32_t *out_exec, cudaStream_t s) {
   if (n_launch == 0) return cudaSuccess;
   {
   TimerScope t(e, DUM_T_INGEST, s);
@@ -334,16 +339,16 @@ cudaError_t launch_record(dum_engine *e, const uint64_t *hash, const uint64_t *o
   const size_t bm_bytes = (size_t)((bmw + 3) & ~3u) * 4 + 2 * IDCAP * 4;
   const bool bm_ok = bm_bytes <= INGEST_SMEM_MAX;
   const size_t smem = std::max<size_t>(2 * INGEST_HCAP * 4, bm_ok ? bm_bytes : 0);
-  static size_t set_smem = 0;  // the attribute is per function: raise it once per size
-  if (smem > set_smem) {
+  // the attribute is per device and function: raised by every engine on its own device
+  if ((int)smem > e->ingest_smem) {
     cudaFuncSetAttribute(k_ingest, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    set_smem = smem;
+    e->ingest_smem = (int)smem;
   }
   k_ingest<<<n_launch, INGEST_NT, smem, s>>>(hash, off, faults, n_launch, e->g.W, e->n_staged, e->staged_faults,
                                              e->d_stage_hash, e->d_stage_off, e->d_stage_norm, e->d_stage_cnt,
                                              e->d_stage_slot, e->d_exec_keys, e->d_exec_vals, e->d_exec_minpos,
                                              e->exec_cap, e->d_ingest_pool, e->big_pool_entries, bm_ok ? bmw : 0,
-                                             e->d_stage_exec, out_exec, e->d_pend, e->g.Emax, e->d_state);
+                                             e->d_stage_exec, out_exec, e->d_pend, e->g.Emax, n_fault, e->d_state);
   }
   TimerScope t(e, DUM_T_EXEC_ASSIGN, s);
   k_exec_assign<<<1, ASSIGN_NT, 0, s>>>(n_launch, e->n_staged, e->d_stage_slot, e->d_stage_hash, e->d_exec_vals,

@@ -6,7 +6,7 @@ namespace dum {
 
 // k_record.cu  (a1 + a2)
 cudaError_t launch_record(dum_engine *e, const uint64_t *hash, const uint64_t *off, uint32_t n_launch,
-                          const uint32_t *faults, uint32_t *out_exec, cudaStream_t s);
+                          const uint32_t *faults, uint64_t n_fault, uint32_t *out_exec, cudaStream_t s);
 // k_build.cu   (a3 - a6)
 cudaError_t launch_build(dum_engine *e, cudaStream_t s);
 cudaError_t launch_jump_tables(dum_engine *e, cudaStream_t s);

@@ -395,3 +395,76 @@ def test_T_integration_loop(row):
 
     r = il.run_loop(il.OracleLoop(tr, N), tr, N, check=check)
     assert r["faults_per_iter"] == faults and r["h2d"] == h2d and r["d2h"] == d2h
+
+
+# ---------------------------------------------------------------------------
+# D7 row_index = 1: the fmix32 finalizer of MurmurHash3 (Appleby).  Pinned by
+# published MurmurHash3_x86_32 test vectors, not by the oracle's own formula:
+# a plain-Python MurmurHash3_x86_32 is checked against the published values
+# (body, tail and finalizer all take part), and for a key of length 0 the
+# hash is fmix32(seed ^ 0) -- so MurmurHash3("", seed=b) is the set index
+# source of block b.  The published vectors ("" seed 1 = 0x514E28B7, seed
+# 0xffffffff = 0x81F16F39, ...) fix the finalizer's shifts and constants.
+# ---------------------------------------------------------------------------
+def _murmur3_x86_32(data: bytes, seed: int) -> int:
+    c1, c2, M = 0xCC9E2D51, 0x1B873593, 0xFFFFFFFF
+
+    def rotl(x, r):
+        return ((x << r) | (x >> (32 - r))) & M
+
+    h = seed & M
+    nb = len(data) // 4
+    for i in range(nb):
+        k = int.from_bytes(data[4 * i:4 * i + 4], "little")
+        k = rotl((k * c1) & M, 15)
+        h ^= (k * c2) & M
+        h = (rotl(h, 13) * 5 + 0xE6546B64) & M
+    tail = data[4 * nb:]
+    k = 0
+    for j in reversed(range(len(tail))):
+        k = (k << 8) | tail[j]
+    if tail:
+        k = rotl((k * c1) & M, 15)
+        h ^= (k * c2) & M
+    h ^= len(data)
+    h ^= h >> 16
+    h = (h * 0x85EBCA6B) & M
+    h ^= h >> 13
+    h = (h * 0xC2B2AE35) & M
+    h ^= h >> 16
+    return h
+
+
+MURMUR3_VECTORS = [  # (key, seed, MurmurHash3_x86_32) -- published test vectors
+    (b"", 0, 0x00000000), (b"", 1, 0x514E28B7), (b"", 0xFFFFFFFF, 0x81F16F39),
+    (b"\0\0\0\0", 0, 0x2362F9DE), (b"a", 0x9747B28C, 0x7FA09EA6), (b"abc", 0x9747B28C, 0xC84A62DD),
+    (b"aaaa", 0x9747B28C, 0x5A97808A), (b"Hello, world!", 0x9747B28C, 0x24884CBA),
+    (b"The quick brown fox jumps over the lazy dog", 0x9747B28C, 0x2FA826CD),
+]
+
+
+def test_murmur3_reference_vectors():
+    for key, seed, want in MURMUR3_VECTORS:
+        assert _murmur3_x86_32(key, seed) == want, (key, seed)
+
+
+def test_fmix32_row_index_pinned():
+    """Each block b, TOUCHed alone, lands in set MurmurHash3("", seed=b) &
+    (R - 1) under row_index = 1 (D7), and in set b & (R - 1) under the
+    default low-bit index."""
+    R = 8192
+    rng = np.random.default_rng(3)
+    blocks = [1, 2, 3, 255, 4096, 65535, 65536] + [int(x) for x in rng.integers(0, 1 << 20, 40)]
+    blocks = list(dict.fromkeys(blocks))
+    for row_index in (0, 1):
+        o = orc.Oracle(R=R, A=1, S=1, N=1, W=1 << 20, C=4, row_index=row_index)
+        # one launch per block (a fresh exec ID each), so no set conflicts
+        h = np.arange(1, len(blocks) + 1, dtype=np.uint64)
+        off = np.arange(len(blocks) + 1, dtype=np.uint64)
+        o.record_faults(h, off, np.array(blocks, dtype=np.uint32))
+        o.build_tables()
+        d = orc.parse_dump(o.dump(orc.EXEC | orc.BLK), orc.EXEC | orc.BLK, len(blocks), R, 1, 1)
+        for e, b in enumerate(blocks):
+            want = (_murmur3_x86_32(b"", b) if row_index else b) & (R - 1)
+            sets = np.nonzero(d["blk"][e][:, 0, 0] != NONE)[0]
+            assert list(sets) == [want] and d["blk"][e][want, 0, 0] == b, (row_index, b, list(sets))
