@@ -15,12 +15,17 @@ Default workload: G, the GPT-2-XL-shaped 4x-oversubscribed trace
 (BASELINE.json configs[2]; the replicas config configs[4] is G-shaped, so the
 same workload serves N = 1, 2, 4, 8).  B (configs[1]) via --workload B.
 
-Timing: W warm-up steps, then K timed steps; before every step the L2 is
-flushed (512 MiB write) and the step's residency snapshot is loaded, both
-outside the timed region; each step is bracketed by CUDA events on the
-engine's stream; max over ranks.  Multi-GPU = independent replicas (weak
-scaling, seed 3 + 1000 * rank, no data-path collective; NCCL carries only the
-barrier and the max-time reduction).
+Timing: W warm-up steps, then K timed steps issued back to back inside ONE
+CUDA-event region on the engine's stream (the ingest of step i+1 overlaps the
+build of step i; each step loads its iteration-start residency snapshot inside
+the region; engine counters are off).  No L2 flush inside the region: a step
+writes ~200 MB of prefetch / victim lists, more than the 126 MB L2.  A second
+pass over K further iterations brackets every kernel with CUDA events (L2
+flushed before each step) for the per-kernel durations, shares and the
+roofline; its work counters give the SURVEY 8(d) algorithmic bytes.  Max over
+ranks.  Multi-GPU = independent replicas (weak scaling, seed 3 + 1000 * rank,
+no data-path collective; the process group carries only the barrier and the
+max-time reduction).
 """
 from __future__ import annotations
 
@@ -57,6 +62,8 @@ def parse():
     ap.add_argument("--json-out", default="")
     ap.add_argument("--unfused", action="store_true", help="separate predict / select calls")
     ap.add_argument("--debug", action="store_true", help="synchronize and check after every call")
+    ap.add_argument("--verify", action="store_true",
+                    help="check the last timed step's prefetch / victim lists against the oracle")
     return ap.parse_args()
 
 
@@ -116,30 +123,41 @@ class Clocks:
 # ---------------------------------------------------------------------------
 # algorithmic bytes per kernel
 # ---------------------------------------------------------------------------
-def algorithmic_bytes(ctr, geo, N, fused=True):
-    """Bytes each kernel must move at minimum for the work it did (counters
-    from the engine).  DESIGN.md "Roofline accounting" states every term."""
+def algorithmic_bytes(ctr, geo, N):
+    """SURVEY.md 8(d) "Algorithmic bytes per iteration", term by term, from the
+    engine's work counters (dum_read_counters); returns (terms, per_kernel).
+      ingest        4 B per raw record + 4 B per normalised record + 20 B per launch
+      exec map/corr 16 B probe per launch + 2 x 24 B RMW per correlation upsert
+      block tables  2 x set_bytes per (exec, set) touched    (set_bytes = 4 A (1 + S))
+      walk cache    set_bytes per row walked + 4 B per walk entry written
+      predict       4 B per walk entry gathered + 8 B per pair emitted + 4 (N + 2) B per query
+      select        4 B per LRM entry scanned + 4 B per victim
+    Kernel attribution: the exec-map probe runs in k_ingest, the correlation
+    upserts in k_build_prep; k_window / k_predict split predict + select by the
+    fast-path counters (FAST_*)."""
     from paper_conf_asplos_jungkl23_b200.binding import CTR
     c = {k: int(ctr[v]) for k, v in CTR.items()}
-    set_bytes = 4 * geo["A"] * (1 + geo["S"])
-    # predict: minimal HBM traffic = its outputs (pairs, per-query ranges,
-    # kern_off, chain) + the per-query scratch written by k_chain + one read of
-    # each run entry; re-reads of L2-resident shared inputs (walk lists, the
-    # residency bitmap, the LRM log) are not counted (DESIGN.md Sec. 7)
-    predict = (8 * c["EMITTED"] + 8 * c["RUNS"] + 4 * c["CHAIN"]
-               + c["QUERIES"] * (16 + 24 + 12 + 4 * (N + 2) + 4 * (N + 1)))
-    select_core = 4 * c["SEL_VICTIMS"] + 32 * c["QUERIES"]
-    if fused:
-        predict += select_core
-    return {
-        "k_ingest": 4 * c["RAW_RECORDS"] + 4 * c["NORM_RECORDS"] + 28 * c["LAUNCHES"],
-        "k_exec_assign": 16 * c["LAUNCHES"],
-        "k_build_prep": 8 * c["LAUNCHES"] + 2 * 32 * c["CORR_UPSERTS"],
-        "k_apply": 4 * c["OPS"] + 2 * set_bytes * c["SETS"],
-        "k_walk": set_bytes * c["WALK_ROWS"] + 4 * c["WALK_OUT"] + 16 * c["EXEC_BUILT"],
-        "k_predict": predict,
-        "k_select": 8 * c["SEL_WINDOW"] + select_core,
+    sb = 4 * geo["A"] * (1 + geo["S"])
+    scanned = c["SEL_SCANNED"] + c["FAST_SCANNED"]
+    victims = c["SEL_VICTIMS"] + c["FAST_VICTIMS"]
+    terms = {
+        "ingest": 4 * c["RAW_RECORDS"] + 4 * c["NORM_RECORDS"] + 20 * c["LAUNCHES"],
+        "exec_map_corr": 16 * c["LAUNCHES"] + 48 * c["CORR_UPSERTS"],
+        "block_tables": 2 * sb * c["SETS"],
+        "walk_cache": sb * c["WALK_ROWS"] + 4 * c["WALK_OUT"],
+        "predict": 4 * c["GATHERED"] + 8 * c["EMITTED"] + 4 * (N + 2) * c["QUERIES"],
+        "select": 4 * scanned + 4 * victims,
     }
+    fast = (12 * c["FAST_EMITTED"] + 4 * (N + 2) * c["Q_FAST"] + 4 * c["FAST_SCANNED"] + 4 * c["FAST_VICTIMS"])
+    per_kernel = {
+        "k_ingest": terms["ingest"] + 16 * c["LAUNCHES"],
+        "k_build_prep": 48 * c["CORR_UPSERTS"],
+        "k_apply": terms["block_tables"],
+        "k_walk": terms["walk_cache"],
+        "k_window": fast,
+        "k_predict": terms["predict"] + terms["select"] - fast,
+    }
+    return terms, per_kernel, c
 
 
 def load_peaks():
@@ -342,8 +360,8 @@ def run_ours(args, rank, world, local_rank):
     torch.cuda.synchronize()
     if world > 1:
         torch.distributed.barrier()
-    # ---- timed region: the K steps, no per-kernel events ----
-    eng.read_counters(reset=True)
+    # ---- timed region: the K steps, no per-kernel events, no counters ----
+    eng.set_counting(False)  # no instrumentation atomics in the timed region
     launches0 = eng.kernel_launches
     stream = torch.cuda.current_stream(dev)
     # One CUDA-event region over the K steps, issued back to back: the ingest
@@ -378,7 +396,14 @@ def run_ours(args, rank, world, local_rank):
         cap_ok = False
         print("WARNING: device error in timed region: %s" % e, file=sys.stderr)
     tot_ms = a.elapsed_time(b)
-    ctr = eng.read_counters(reset=True)
+    eng.set_counting(True)
+    verify_out = None
+    if args.verify:  # the last timed step's outputs, checked against the oracle below
+        i_v = args.warmup + args.steps
+        verify_out = (i_v, B.u32(pairs[0]).reshape(-1, 2).copy(), B.u64(rng).reshape(-1, 2).copy(),
+                      B.u32(ko).reshape(K, -1).copy(), B.u32(ch).reshape(K, -1).copy(), B.u32(wb[0]).copy(),
+                      B.u32(inv[0]).copy(), B.u64(srng).reshape(-1, 4).copy())
+    eng.read_counters(reset=True)
     # ---- breakdown pass: K further steps (the next trace iterations) with CUDA
     # events around every kernel, for the per-kernel durations / roofline ----
     eng.read_timing(reset=True)
@@ -402,9 +427,9 @@ def run_ours(args, rank, world, local_rank):
     tot_ms_max, records_all = aggregate(tot_ms, records, device=dev)
     value = records_all / (tot_ms_max / 1000.0)
 
-    # ---- roofline of the dominant kernel ----
+    # ---- roofline of the dominant kernel (SURVEY 8(d) bytes, breakdown pass) ----
     peak, peak_src = load_peaks()
-    abytes = algorithmic_bytes(ctr_bk, geo, N, fused=not args.unfused)
+    terms, abytes, craw = algorithmic_bytes(ctr_bk, geo, N)
     per_kernel = {}
     for name, idx in B.TIMER.items():
         if kcnt[idx]:
@@ -425,11 +450,23 @@ def run_ours(args, rank, world, local_rank):
     traffic = load_traffic().get(dom, {}).get("dram_bytes_per_launch")
     roof = {"kernel": dom, "bound": "hbm", "achieved": d.get("achieved_gbs"), "peak": peak, "unit": "GB/s",
             "frac": round(d["achieved_gbs"] / peak, 4) if d.get("achieved_gbs") else None,
-            "traffic": traffic, "alg_bytes_per_launch": d.get("alg_bytes_per_launch"), "peak_source": peak_src}
-    alg_total = sum(algorithmic_bytes(ctr, geo, N, fused=not args.unfused).values())
-    step_roof = {"alg_bytes_per_step": int(alg_total / max(args.steps, 1)),
-                 "achieved_gbs": round(alg_total / (tot_ms / 1000) / 1e9, 1),
-                 "frac": round(alg_total / (tot_ms / 1000) / 1e9 / peak, 4)}
+            "traffic": traffic, "alg_bytes_per_launch": d.get("alg_bytes_per_launch"),
+            "avg_us": d.get("avg_us"), "peak_source": peak_src,
+            "bytes_formula": {
+                "k_window": "12*FAST_EMITTED + 4*(N+2)*Q_FAST + 4*FAST_SCANNED + 4*FAST_VICTIMS "
+                            "(SURVEY 8(d) predict + select terms for the queries k_window answers)",
+                "k_apply": "2*set_bytes*SETS", "k_walk": "set_bytes*WALK_ROWS + 4*WALK_OUT",
+                "k_ingest": "4*RAW + 4*NORM + 20*LAUNCHES + 16*LAUNCHES (exec-map probe)",
+                "k_build_prep": "48*CORR_UPSERTS", "set_bytes": 4 * geo["A"] * (1 + geo["S"]), "N": N},
+            "timing": "avg CUDA-event duration of the kernel on its launching stream, breakdown pass"}
+    alg_step = sum(terms.values()) / max(args.steps, 1)
+    step_roof = {"alg_bytes_per_step": int(alg_step),
+                 "terms_per_step": {k: int(v / max(args.steps, 1)) for k, v in terms.items()},
+                 "achieved_gbs": round(alg_step / (tot_ms / args.steps / 1000) / 1e9, 1),
+                 "frac": round(alg_step / (tot_ms / args.steps / 1000) / 1e9 / peak, 4),
+                 "how": "SURVEY 8(d) bytes of the breakdown pass's steps (counters are off in the timed region) "
+                        "over the timed ms per step"}
+    counters = {k: round(v / max(args.steps, 1), 1) for k, v in craw.items() if v}
 
     # ---- e2e: same steps through the C-ABI with pinned HOST inputs ----
     e2e = None
@@ -456,7 +493,7 @@ def run_ours(args, rank, world, local_rank):
                              "the build of step i); residency snapshot loaded inside every step",
                    "seed": seed},
         "gpu_launches": int(launches),
-        "roofline": roof, "step_roofline": step_roof, "kernels": per_kernel,
+        "roofline": roof, "step_roofline": step_roof, "kernels": per_kernel, "counters_per_step": counters,
         "breakdown": {"ms_per_step": round(bk_ms / max(args.steps, 1), 4),
                       "how": "K further steps (the next trace iterations) with CUDA events around every kernel; "
                              "kernel shares and the roofline come from this pass, the headline from the "
@@ -467,7 +504,49 @@ def run_ours(args, rank, world, local_rank):
         res["e2e"] = e2e
     if mig:
         res["migration"] = mig
+    if verify_out is not None:
+        res["verify"] = verify_step(tr, N, verify_out)
     return res, tr
+
+
+def verify_step(tr, N, out):
+    """The oracle replays iterations 0 .. i-1 (record + build), loads the
+    iteration-start residency snapshot i and answers the same K transition
+    queries; every query's (block, exec) list, kern_off, chain, write-back and
+    invalidate list of the timed step i must be identical."""
+    import oracle as orc
+    i, gp, grng, gko, gch, gwb, ginv, gsr = out
+    t0 = time.perf_counter()
+    o = orc.Oracle(R=2048, A=2, S=4, N=N, W=tr.W, C=tr.C, threads=os.cpu_count() or 1)
+    o.mark_inactive(tr.inactive_blocks, True)
+    ex = []
+    for it in range(i + 1):
+        h, off, f = tr.iteration(it)
+        ex += [int(x) for x in o.record_faults(h, off, f)]
+        if it < i:
+            o.build_tables()
+    o.load_residency(tr.snap_blk[i][: int(tr.snap_cnt[i])])
+    NONE = 0xFFFFFFFF
+    pad = [NONE] * 3 + ex
+    K = tr.K
+    q = np.array([[ex[k], pad[k], pad[k + 1], pad[k + 2], NONE, N] for k in range(i * K, (i + 1) * K)],
+                 dtype=np.uint32)
+    off_o, pairs_o, ko_o, ch_o = o.predict(q)
+    wo, wb_o, io, inv_o = o.select(off_o, pairs_o, q[:, 4])
+    bad = []
+    for qi in range(K):
+        a, b = int(grng[qi, 0]), int(grng[qi, 1])
+        if not np.array_equal(gp[a:b], pairs_o[int(off_o[qi]):int(off_o[qi + 1])]):
+            bad.append(("pairs", qi))
+        if not (np.array_equal(gko[qi], ko_o[qi]) and np.array_equal(gch[qi], ch_o[qi])):
+            bad.append(("kern_off/chain", qi))
+        r = gsr[qi]
+        if not (np.array_equal(gwb[int(r[0]):int(r[1])], wb_o[int(wo[qi]):int(wo[qi + 1])]) and
+                np.array_equal(ginv[int(r[2]):int(r[3])], inv_o[int(io[qi]):int(io[qi + 1])])):
+            bad.append(("victims", qi))
+    return {"iteration": i, "queries": K, "pairs": int(off_o[-1]), "victims": int(len(wb_o) + len(inv_o)),
+            "ok": not bad, "mismatches": bad[:10], "oracle_s": round(time.perf_counter() - t0, 1),
+            "how": "last timed step's outputs vs the oracle (record+build of iterations 0..i-1, snapshot i)"}
 
 
 def run_e2e(args, tr, eng, step, pre_step, exec_all, rng, srng, dev, stream):

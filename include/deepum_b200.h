@@ -103,7 +103,14 @@ typedef struct {
   uint64_t host_arena_bytes;
   void *frame_pool;
   uint64_t frame_pool_bytes;
+  /* DUM_CFG_* bits (0 = production). */
+  uint32_t flags;
 } dum_config;
+
+/* dum_config.flags: build every walk with the sequential one-warp walker
+ * (the literal PAPER.md L218-L224 loop) instead of the parallel k_walk --
+ * a verification mode: both must give identical walk caches. */
+#define DUM_CFG_SEQ_WALKS 0x1u
 
 /* Fill *cfg with the defaults (Config9, N = 32). */
 void dum_config_default(dum_config *cfg);
@@ -239,6 +246,39 @@ typedef enum { DUM_H2D = 0, DUM_D2H = 1, DUM_INVALIDATE = 2, DUM_D2D = 3 } dum_d
 int dum_migrate_blocks(dum_engine *eng, dum_dir dir, const uint32_t *blocks_or_src, const uint32_t *dst_frames,
                        uint32_t n, uint32_t method, dum_stream_t stream);
 
+/* ---- closed-loop replay ------------------------------
+ * dum_simulate replays launches 0 .. n_launch-1 (launch k has hash
+ * launch_hash[k] and accesses the blocks acc_blk[acc_off[k % n_kernels] ..
+ * acc_off[k % n_kernels + 1]), per launch and in order, through the paper's
+ * loop: faults = accesses without a frame (first
+ * occurrence, D2) -> dum_record_faults -> demand eviction when the faults
+ * exceed the free frames (least recently migrated blocks the launch does not
+ * access, D22; inactive ones invalidated with DUM_SIM_INVALIDATE) and H2D of
+ * the faults -> dum_build_tables -> (DUM_SIM_PREFETCH) the transition query of
+ * the next launch (its exec ID if its hash is known, the last three exec IDs
+ * as history, degree n) -> (DUM_SIM_PREEVICT) pre-eviction of the window's
+ * victims (L236-L243) -> H2D of the window's non-resident prefix that fits the
+ * free frames (L156-L158).  Every step runs in this library's kernels, list
+ * sizes stay on the device.  Without a data plane the migrations move the
+ * residency only (metadata-only engine: B/G scale); with one the bytes move.
+ * Per-launch statistics go to stats[k] (device).  launch_hash, acc_blk, stats:
+ * device; acc_off: HOST (n_kernels + 1 entries, <= 4096 accesses per launch).
+ * Requires an empty staging area (call after dum_build_tables). */
+typedef struct {
+  uint32_t faults;      /* demand faults of the launch (blocks migrated on demand) */
+  uint32_t demand_wb;   /* demand-path victims written back */
+  uint32_t demand_inv;  /* demand-path victims invalidated (D20) */
+  uint32_t pre_wb;      /* pre-evicted blocks written back */
+  uint32_t pre_inv;     /* pre-evicted blocks invalidated */
+  uint32_t prefetched;  /* window blocks migrated ahead of use */
+} dum_sim_stats;
+#define DUM_SIM_PREFETCH 0x1u   /* query + prefetch the window (else naive UM: demand only) */
+#define DUM_SIM_PREEVICT 0x2u   /* pre-evict for the window */
+#define DUM_SIM_INVALIDATE 0x4u /* inactive victims are invalidated, not written back (L285) */
+int dum_simulate(dum_engine *eng, const uint64_t *launch_hash, uint32_t n_launch, const uint64_t *acc_off,
+                 const uint32_t *acc_blk, uint32_t n_kernels, uint32_t degree, uint32_t flags,
+                 dum_sim_stats *stats, dum_stream_t stream);
+
 /* 64-bit position-weighted checksums (sum_w word_w * (2w+1) mod 2^64) of 2 MiB
  * blocks: where = 0 -> HBM frames ids[i]; 1 -> host-arena blocks ids[i]. */
 int dum_block_checksums(dum_engine *eng, int where, const uint32_t *ids, uint32_t n, uint64_t *out,
@@ -299,8 +339,26 @@ enum {
   DUM_CTR_SEL_VICTIMS,      /* victims selected                          */
   DUM_CTR_MIG_BLOCKS,       /* 2 MiB blocks copied                       */
   DUM_CTR_RUNS,             /* walk bitmap runs inserted by predict      */
-  DUM_NCOUNTERS = 24
+  /* which code path answered each unit of work (tests assert every path is
+   * exercised; the bench reports them) */
+  DUM_CTR_Q_NODUP,          /* predict queries: window-bitmap path, no duplicate found    */
+  DUM_CTR_Q_DUP,            /* predict queries: duplicate path (occurrence lists)         */
+  DUM_CTR_Q_FALLBACK,       /* predict queries: min-position hash over every element      */
+  DUM_CTR_WALK_PREFIX,      /* walks proved to be a prefix of the latest launch           */
+  DUM_CTR_WALK_DEDUPE,      /* walks built by the parallel min-position dedupe            */
+  DUM_CTR_WALK_SLOW,        /* walks built by the sequential walker                       */
+  DUM_CTR_Q_FAST,           /* predict queries: conflict-free window (no bitmap)          */
+  DUM_CTR_ANCHOR_WALKS,     /* fault-anchored walks (WALK(e, anchor))                     */
+  DUM_CTR_INGEST_DUP,       /* launches whose records held duplicates                     */
+  DUM_CTR_Q_SLOW,           /* predict queries sent to the exact (bitmap) kernel          */
+  DUM_CTR_FAST_EMITTED,     /* pairs emitted by k_window (= walk entries it gathered)      */
+  DUM_CTR_FAST_SCANNED,     /* LRM-log entries scanned by k_window's selection             */
+  DUM_CTR_FAST_VICTIMS,     /* victims selected by k_window                                */
+  DUM_NCOUNTERS = 32
 };
+/* Counters accumulate only while counting is on (the default); the bench turns
+ * it off for its timed region (no instrumentation atomics there). */
+int dum_set_counting(dum_engine *eng, int enable);
 int dum_read_counters(dum_engine *eng, uint64_t out[DUM_NCOUNTERS], int reset);
 
 /* Per-kernel CUDA-event timing on the launching stream (off by default).
@@ -322,7 +380,10 @@ enum {
   DUM_T_CHAIN,
   DUM_T_JUMP,         /* jump tables over the correlation table (side stream, in dum_build_tables) */
   DUM_T_WALK,         /* parallel walk-cache rebuild (in dum_build_tables) */
-  DUM_NTIMERS = 16
+  DUM_T_EXACT,        /* exact-path predict kernel k_predict (side stream, beside k_window) */
+  DUM_T_WALK_INDEX,   /* walk index: holders per block, conflicts per walk (build end) */
+  DUM_T_WALK_RES,     /* residency facts per walk (predict) */
+  DUM_NTIMERS = 24
 };
 int dum_set_timing(dum_engine *eng, int enable);
 int dum_read_timing(dum_engine *eng, double ms[DUM_NTIMERS], uint64_t count[DUM_NTIMERS], int reset);

@@ -16,22 +16,31 @@ _LIBPATH = os.environ.get("DUM_LIB") or os.path.join(HERE, "libdeepum_b200.so")
 DUM_NONE = NONE = 0xFFFFFFFF
 DUM_INPUTS_READY = 2
 DUM_HOST_PTRS = 0x1
+DUM_CFG_SEQ_WALKS = 0x1
+SIM_PREFETCH, SIM_PREEVICT, SIM_INVALIDATE = 0x1, 0x2, 0x4
+SIM_FIELDS = ("faults", "demand_wb", "demand_inv", "pre_wb", "pre_inv", "prefetched")
 DUMP_EXEC, DUMP_CORR, DUMP_BLK, DUMP_WALK, DUMP_RES, DUMP_HIST = 1, 2, 4, 8, 16, 32
 H2D, D2H, INVALIDATE, D2D = 0, 1, 2, 3
-NCOUNTERS, NTIMERS = 24, 16
+NCOUNTERS, NTIMERS = 32, 24
 CTR = {n: i for i, n in enumerate(["RAW_RECORDS", "NORM_RECORDS", "LAUNCHES", "CORR_UPSERTS", "EXEC_BUILT", "OPS",
                                    "SETS", "WALK_ROWS", "WALK_OUT", "QUERIES", "CHAIN", "GATHERED", "EMITTED",
-                                   "SEL_WINDOW", "SEL_SCANNED", "SEL_VICTIMS", "MIG_BLOCKS", "RUNS"])}
+                                   "SEL_WINDOW", "SEL_SCANNED", "SEL_VICTIMS", "MIG_BLOCKS", "RUNS",
+                                   "Q_NODUP", "Q_DUP", "Q_FALLBACK", "WALK_PREFIX", "WALK_DEDUPE", "WALK_SLOW",
+                                   "Q_FAST", "ANCHOR_WALKS", "INGEST_DUP", "Q_SLOW", "FAST_EMITTED", "FAST_SCANNED",
+                                   "FAST_VICTIMS"])}
 TIMER = {n: i for i, n in enumerate(["INGEST", "EXEC_ASSIGN", "BUILD_PREP", "APPLY_WALK", "WALK_SLOW",
                                      "MAKE_QUERIES", "ANCHOR_WALK", "PREDICT", "SELECT", "MIG_PLAN", "COPY",
-                                     "RESIDENCY", "CHAIN", "JUMP", "WALK"])}
+                                     "RESIDENCY", "CHAIN", "JUMP", "WALK", "EXACT", "WALK_INDEX", "WALK_RES"])}
 KERNEL_OF_TIMER = {"INGEST": "k_ingest", "EXEC_ASSIGN": "k_exec_assign", "BUILD_PREP": "k_build_prep",
                    "APPLY_WALK": "k_apply", "WALK": "k_walk", "WALK_SLOW": "k_walk_slow", "MAKE_QUERIES": "k_make_queries",
-                   "ANCHOR_WALK": "k_anchor_walk", "PREDICT": "k_predict", "SELECT": "k_select",
+                   "ANCHOR_WALK": "k_anchor_walk", "PREDICT": "k_copy_fast", "SELECT": "k_select_fast",
                    "MIG_PLAN": "k_mig_plan", "COPY": "k_copy_blocks", "RESIDENCY": "k_load_res",
-                   "CHAIN": "k_chain", "JUMP": "k_jump0"}
-# timers of kernels launched on the engine's side stream (overlapping others)
-SIDE_TIMERS = {"JUMP": "side stream, overlaps k_apply / k_walk (k_jump0 + k_jumpk levels)"}
+                   "CHAIN": "k_chain", "JUMP": "k_jump0", "EXACT": "k_predict", "WALK_INDEX": "k_walk_index",
+                   "WALK_RES": "k_walk_res"}
+# timers of kernels launched on the engine's side streams (overlapping others)
+SIDE_TIMERS = {"JUMP": "side stream, overlaps k_apply / k_walk (k_jump0 + k_jumpk levels)",
+               "EXACT": "second side stream, beside the fast path (exact-path queries)",
+               "SELECT": "third side stream, beside k_copy_fast (fast-path selection)"}
 _ERR = {0: "DUM_OK", -1: "DUM_EINVAL", -2: "DUM_ECAPACITY", -3: "DUM_ENOMEM", -4: "DUM_ECUDA", -5: "DUM_ESTATE"}
 
 
@@ -49,6 +58,7 @@ class DumConfig(ctypes.Structure):
         ("max_batch_faults", ctypes.c_uint64), ("corr_capacity", ctypes.c_uint32), ("device", ctypes.c_int),
         ("host_arena", ctypes.c_void_p), ("host_arena_bytes", ctypes.c_uint64),
         ("frame_pool", ctypes.c_void_p), ("frame_pool_bytes", ctypes.c_uint64),
+        ("flags", ctypes.c_uint32),
     ]
 
 
@@ -98,9 +108,11 @@ def load_library() -> ctypes.CDLL:
         "dum_last_error": (ctypes.c_char_p, [P]),
         "dum_kernel_launches": (U64, [P]),
         "dum_read_counters": (I, [P, P, I]),
+        "dum_set_counting": (I, [P, I]),
         "dum_set_timing": (I, [P, I]),
         "dum_host_ptr_kind": (I, [P]),
         "dum_read_timing": (I, [P, P, P, I]),
+        "dum_simulate": (I, [P, P, U32, P, P, U32, U32, U32, P, P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -146,7 +158,7 @@ class Engine:
     def __init__(self, num_rows=2048, assoc=2, num_succs=4, degree_n=32, max_blocks=1 << 16, max_exec_ids=8192,
                  hbm_frames=1024, row_index=0, max_batch_launches=0, max_batch_faults=0, corr_capacity=0,
                  device: int = 0, host_arena: Optional[torch.Tensor] = None,
-                 frame_pool: Optional[torch.Tensor] = None):
+                 frame_pool: Optional[torch.Tensor] = None, flags: int = 0):
         self.lib = load_library()
         self.device = torch.device("cuda", device)
         c = DumConfig()
@@ -155,6 +167,7 @@ class Engine:
         c.max_blocks, c.max_exec_ids, c.hbm_frames, c.row_index = max_blocks, max_exec_ids, hbm_frames, row_index
         c.max_batch_launches, c.max_batch_faults, c.corr_capacity, c.device = (
             max_batch_launches, max_batch_faults, corr_capacity, device)
+        c.flags = flags
         if host_arena is not None:
             c.host_arena, c.host_arena_bytes = host_arena.data_ptr(), host_arena.numel() * host_arena.element_size()
         if frame_pool is not None:
@@ -292,6 +305,20 @@ class Engine:
                                              self._stream()), "dum_predict_select")
         return pairs, rng, kern_off, chain, needed, wb, inv, sel_rng, sel_needed
 
+    def simulate(self, launch_hash: torch.Tensor, acc_off: np.ndarray, acc_blk: torch.Tensor, degree: int,
+                 flags: int, stats: Optional[torch.Tensor] = None) -> torch.Tensor:
+        """dum_simulate: the closed loop over len(launch_hash) launches; launch k
+        accesses acc_blk[acc_off[k % K] : acc_off[k % K + 1]] (K = len(acc_off) - 1).
+        Returns the per-launch statistics, a [n_launch, 6] int32 device tensor
+        (columns SIM_FIELDS)."""
+        n = launch_hash.numel()
+        off = np.ascontiguousarray(acc_off, dtype=np.uint64)
+        if stats is None:
+            stats = torch.zeros((n, len(SIM_FIELDS)), dtype=torch.int32, device=self.device)
+        self._ck(self.lib.dum_simulate(self._h, _dev(launch_hash, 8), n, off.ctypes.data, _dev(acc_blk, 4),
+                                       len(off) - 1, degree, flags, _dev(stats, 4), self._stream()), "dum_simulate")
+        return stats
+
     def mark_inactive(self, blocks: torch.Tensor, inactive: bool = True):
         self._ck(self.lib.dum_mark_inactive(self._h, _dev(blocks, 4), blocks.numel(), 1 if inactive else 0,
                                             self._stream()), "dum_mark_inactive")
@@ -337,6 +364,13 @@ class Engine:
         out = np.zeros(NCOUNTERS, dtype=np.uint64)
         self._ck(self.lib.dum_read_counters(self._h, out.ctypes.data, 1 if reset else 0), "dum_read_counters")
         return out
+
+    def set_counting(self, on: bool):
+        self._ck(self.lib.dum_set_counting(self._h, 1 if on else 0), "dum_set_counting")
+
+    def counters(self, reset: bool = False) -> dict:
+        c = self.read_counters(reset)
+        return {k: int(c[v]) for k, v in CTR.items()}
 
     def set_timing(self, on: bool):
         self._ck(self.lib.dum_set_timing(self._h, 1 if on else 0), "dum_set_timing")

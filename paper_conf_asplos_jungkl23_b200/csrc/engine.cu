@@ -13,6 +13,7 @@
 
 #include "device_util.cuh"
 #include "kernels.cuh"
+#include "predict.cuh"
 #include "select_tail.cuh"
 
 using namespace dum;
@@ -37,7 +38,11 @@ __global__ void k_init_state(DevState *st) {
   for (int q = 0; q < 4; ++q) st->hist[q] = NONE;
   st->err = 0;
   st->needed = 0;
-  st->pool_pairs = st->pool_wb = st->pool_inv = st->pool_anchor = st->pool_big = 0;
+  st->pool_pairs = st->pool_wb = st->pool_inv = st->pool_anchor = st->pool_big = st->pool_chunks = 0;
+  st->chain_done = 0;
+  for (int c = 0; c < 16; ++c) st->q_cls[c] = 0;
+  st->n_fast = 0;
+  st->n_dd = 0;
   st->n_slow = 0;
   st->n_pend = 0;
   st->n_items = st->n_leads = 0;
@@ -47,6 +52,7 @@ __global__ void k_init_state(DevState *st) {
   st->mig_n = 0;
   st->dbg_line = st->dbg_val = 0;
   for (int c = 0; c < DUM_NCOUNTERS; ++c) st->ctr[c] = 0;
+  st->counting = 1;
 }
 
 uint32_t pow2ceil_h(uint64_t x) {
@@ -88,6 +94,9 @@ cudaError_t fill(uint32_t *p, uint64_t n, uint32_t v, cudaStream_t s) {
 int reset_state(dum_engine *e, cudaStream_t s) {
   const Geo &g = e->g;
   if (e->ev_join) CK(cudaStreamWaitEvent(s, e->ev_join, 0));  // jump tables still building on the side stream
+  if (e->ev_join2) CK(cudaStreamWaitEvent(s, e->ev_join2, 0));  // exact-path predict kernel
+  if (e->ev_join3) CK(cudaStreamWaitEvent(s, e->ev_join3, 0));  // fast-path selection
+  if (e->ev_widx) CK(cudaStreamWaitEvent(s, e->ev_widx, 0));    // walk index
   if (e->ev_rec) CK(cudaStreamWaitEvent(s, e->ev_rec, 0));    // record work on the ingest stream
   CK(fill((uint32_t *)e->d_exec_keys, 2ull * (e->exec_cap + 1), NONE, s));
   CK(cudaMemsetAsync(e->d_exec_keys + e->exec_cap, 0, 8, s));  // sentinel slot: absent
@@ -99,6 +108,8 @@ int reset_state(dum_engine *e, cudaStream_t s) {
   CK(fill(e->d_start_end, 2ull * g.Emax, NONE, s));
   CK(cudaMemsetAsync(e->d_walk_len, 0, 4ull * g.Emax, s));
   CK(cudaMemsetAsync(e->d_wrun_len, 0, 4ull * g.Emax, s));
+  CK(cudaMemsetAsync(e->d_conf_n, 0, 4ull * g.Emax, s));  // no walks: no conflicts
+  CK(cudaMemsetAsync(e->d_bcnt, 0, 4ull * g.W, s));
   CK(fill(e->d_head, g.Emax, NONE, s));
   CK(cudaMemsetAsync(e->d_e_ops, 0, 4ull * g.Emax, s));
   CK(cudaMemsetAsync(e->d_e_last, 0, 4ull * g.Emax, s));
@@ -126,12 +137,21 @@ void free_all(dum_engine *e) {
                   e->d_walk_chain, e->d_walk_tmp, e->d_walk_out, e->d_anchor_pool, e->d_anchor_range,
                   e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits, e->d_inactive_bits, e->d_res_bits, e->d_logpos, e->d_lrm_blk,
                   e->d_lrm_stamp, e->d_mig_frames, e->d_mig_src, e->d_mig_blocks, e->d_state, e->d_qkern,
-                  e->d_qloff, e->d_qnk, e->d_qbase, e->d_rec_slot, e->d_jump, e->d_wrun, e->d_wrun_len, e->d_qeoff, e->d_qgoff, e->d_qrank, e->d_qperm};
+                  e->d_qloff, e->d_qnk, e->d_qbase, e->d_rec_slot, e->d_jump, e->d_wrun, e->d_wrun_len, e->d_qeoff, e->d_qgoff, e->d_qrank, e->d_qperm,
+                  e->d_bcnt, e->d_bhold, e->d_conf, e->d_conf_n, e->d_wnr, e->d_wnres, e->d_respos, e->d_qroff, e->d_qneed, e->d_qvb, e->d_chunk_map, e->d_dd_list,
+                  e->sim_acc_bits, e->sim_faults, e->sim_pairs, e->sim_wb, e->sim_inv, e->sim_pf, e->sim_foff,
+                  e->sim_ranges, e->sim_q};
   for (void *p : ptrs)
     if (p) cudaFree(p);
   if (e->ev_fork) cudaEventDestroy(e->ev_fork);
   if (e->ev_join) cudaEventDestroy(e->ev_join);
   if (e->side) cudaStreamDestroy(e->side);
+  if (e->side2) cudaStreamDestroy(e->side2);
+  if (e->side3) cudaStreamDestroy(e->side3);
+  if (e->ev_join3) cudaEventDestroy(e->ev_join3);
+  if (e->ev_widx) cudaEventDestroy(e->ev_widx);
+  if (e->ev_fork2) cudaEventDestroy(e->ev_fork2);
+  if (e->ev_join2) cudaEventDestroy(e->ev_join2);
   if (e->rec_s) cudaStreamDestroy(e->rec_s);
   if (e->ev_rec) cudaEventDestroy(e->ev_rec);
   if (e->ev_s_now) cudaEventDestroy(e->ev_s_now);
@@ -253,6 +273,12 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
     // ~100 us per step when steps are issued back to back (measured in round 1)
     A_(cudaStreamCreateWithFlags(&e->side, cudaStreamNonBlocking));
   }
+  A_(cudaStreamCreateWithFlags(&e->side2, cudaStreamNonBlocking));
+  A_(cudaStreamCreateWithFlags(&e->side3, cudaStreamNonBlocking));
+  A_(cudaEventCreateWithFlags(&e->ev_join3, cudaEventDisableTiming));
+  A_(cudaEventCreateWithFlags(&e->ev_widx, cudaEventDisableTiming));
+  A_(cudaEventCreateWithFlags(&e->ev_fork2, cudaEventDisableTiming));
+  A_(cudaEventCreateWithFlags(&e->ev_join2, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_fork, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_join, cudaEventDisableTiming));
   A_(dmalloc(&e->d_tbl, (uint64_t)g.Emax * g.R * g.stride));
@@ -288,6 +314,7 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_next, e->stage_launch_cap));
   A_(dmalloc(&e->d_order, 3ull * e->stage_launch_cap));
   A_(dmalloc(&e->d_slow_list, e->stage_launch_cap));
+  A_(dmalloc(&e->d_dd_list, e->stage_launch_cap));
   A_(dmalloc(&e->d_e_ops, g.Emax));
   A_(dmalloc(&e->d_e_last, g.Emax));
   A_(dmalloc(&e->d_lead, 8ull * e->stage_launch_cap));
@@ -309,9 +336,23 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_qeoff, (uint64_t)e->anchor_range_cap * (g.N + 2)));
   A_(dmalloc(&e->d_qgoff, (uint64_t)e->anchor_range_cap * (g.N + 2)));
   A_(dmalloc(&e->d_qrank, e->anchor_range_cap));
-  A_(dmalloc(&e->d_qperm, e->anchor_range_cap));
+  A_(dmalloc(&e->d_qperm, 10ull * e->anchor_range_cap));  // k_chain's class lists (2 NQCLS x queries)
   A_(dmalloc(&e->d_qnk, e->anchor_range_cap));
   A_(dmalloc(&e->d_qbase, e->anchor_range_cap));
+  A_(dmalloc(&e->d_bcnt, g.W));
+  A_(dmalloc(&e->d_bhold, (uint64_t)g.W * HOLD_MAX));
+  A_(dmalloc(&e->d_conf, (uint64_t)g.Emax * CONF_MAX));
+  A_(dmalloc(&e->d_conf_n, g.Emax));
+  A_(dmalloc(&e->d_wnr, g.Emax));
+  A_(dmalloc(&e->d_wnres, g.Emax));
+  A_(dmalloc(&e->d_respos, (uint64_t)g.Emax * g.walk_cap));
+  A_(dmalloc(&e->d_qroff, (uint64_t)e->anchor_range_cap * (g.N + 2)));
+  A_(dmalloc(&e->d_qneed, e->anchor_range_cap));
+  A_(dmalloc(&e->d_qvb, 2ull * e->anchor_range_cap));
+  // copy chunks of one predict call <= out_cap_pairs / 128 + queries x (N + 1); grown by
+  // launch_predict when a call's bound exceeds it
+  e->chunk_cap = 1u << 20;
+  A_(dmalloc(&e->d_chunk_map, e->chunk_cap));
   A_(dmalloc(&e->d_frame_of, g.W));
   A_(dmalloc(&e->d_stamp_of, g.W));
   A_(dmalloc(&e->d_block_of, g.C));
@@ -514,6 +555,26 @@ int dum_select_evictions(dum_engine *e, const uint64_t *query_range, const uint3
   return DUM_OK;
 }
 
+int dum_simulate(dum_engine *e, const uint64_t *launch_hash, uint32_t n_launch, const uint64_t *acc_off,
+                 const uint32_t *acc_blk, uint32_t n_kernels, uint32_t degree, uint32_t flags, dum_sim_stats *stats,
+                 dum_stream_t stream) {
+  if (!e) return DUM_EINVAL;
+  if (n_launch == 0) return DUM_OK;
+  if (!launch_hash || !acc_off || !acc_blk || !stats || n_kernels == 0 || flags > 7)
+    return fail(e, DUM_EINVAL, "null argument / bad flags");
+  if (e->n_staged) return fail(e, DUM_ESTATE, "dum_simulate needs an empty staging area (call dum_build_tables)");
+  for (uint32_t j = 0; j < n_kernels; ++j)
+    if (acc_off[j + 1] < acc_off[j] || acc_off[j + 1] - acc_off[j] > 4096)
+      return fail(e, DUM_EINVAL, "acc_off not monotone or a launch with more than 4096 accesses");
+  if (e->launches + n_launch > 0xFFFFFFFFull) return fail(e, DUM_ECAPACITY, "launch counter exceeds 2^32");
+  cudaSetDevice(e->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  // the ingest stream's pending work (a record call before) is ordered before the loop
+  CK(cudaStreamWaitEvent(s, e->ev_rec, 0));
+  CK(launch_simulate(e, launch_hash, n_launch, acc_off, acc_blk, n_kernels, degree, flags, stats, s));
+  return DUM_OK;
+}
+
 int dum_mark_inactive(dum_engine *e, const uint32_t *blocks, uint32_t n, int inactive, dum_stream_t stream) {
   if (!e || (n && !blocks)) return DUM_EINVAL;
   cudaSetDevice(e->device);
@@ -596,6 +657,16 @@ int dum_read_counters(dum_engine *e, uint64_t out[DUM_NCOUNTERS], int reset) {
   CK(cudaDeviceSynchronize());
   CK(cudaMemcpy(out, e->d_state->ctr, sizeof(uint64_t) * DUM_NCOUNTERS, cudaMemcpyDeviceToHost));
   if (reset) CK(cudaMemset(e->d_state->ctr, 0, sizeof(uint64_t) * DUM_NCOUNTERS));
+  return DUM_OK;
+}
+
+int dum_set_counting(dum_engine *e, int enable) {
+  if (!e) return DUM_EINVAL;
+  cudaSetDevice(e->device);
+  const uint32_t v = enable ? 1u : 0u;
+  // stream-ordered with the caller's legacy default stream and every engine stream (a plain store)
+  CK(cudaDeviceSynchronize());
+  CK(cudaMemcpy(&e->d_state->counting, &v, 4, cudaMemcpyHostToDevice));
   return DUM_OK;
 }
 

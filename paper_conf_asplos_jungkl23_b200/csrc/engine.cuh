@@ -53,6 +53,7 @@ struct DevState {
   unsigned long long pool_wb, pool_inv;
   unsigned long long pool_anchor;  // anchored-walk scratch bump pointer
   unsigned long long pool_big;     // build-walk global hash scratch bump pointer
+  unsigned long long pool_chunks;  // predict: k_copy_fast chunk-map bump pointer
   uint32_t n_slow;            // exec IDs queued for the sequential walk
   uint32_t n_pend;            // record: launches with a hash first seen in the batch (k_ingest -> k_exec_assign)
   uint32_t free_count;        // free HBM frames
@@ -65,9 +66,12 @@ struct DevState {
   uint32_t log_dirty;         // LRM log may hold entries of evicted blocks
   uint32_t dbg_line, dbg_val; // first failed internal guard (GUARD macro)
   uint32_t cls_cnt[4];        // build: faulting launches per size class
-  uint32_t q_cls[8];          // predict: queries per window-size class (k_chain)
+  uint32_t q_cls[16];         // predict: queries per (fast/exact, window-size) class (k_chain)
+  uint32_t n_fast;            // predict: queries answered by k_window (the first n_fast of qperm)
   uint32_t chain_done;        // predict: k_chain CTAs finished
-  uint32_t n_items, n_leads;  // build: k_apply items / k_walk items (k_plan)
+  uint32_t n_items, n_leads;  // build: k_apply items / exec IDs with faults (k_plan)
+  uint32_t n_dd;              // build: walks left to k_walk's dedupe (k_build_exec)
+  uint32_t counting;          // ctr_add is live (dum_set_counting)
   unsigned long long ctr[DUM_NCOUNTERS];  // work counters (instrumentation)
 };
 
@@ -101,7 +105,9 @@ __host__ __device__ inline uint32_t row_of(const Geo &g, uint32_t b) {
 
 __device__ __forceinline__ void ctr_add(DevState *st, int c, unsigned long long v) {
 #ifdef __CUDA_ARCH__
-  if (v) atomicAdd(&st->ctr[c], v);
+  // `counting` only changes between calls (dum_set_counting synchronizes): a
+  // read-only-cache load, no L2 round trip per call site
+  if (v && __ldg(&st->counting)) atomicAdd(&st->ctr[c], v);
 #endif
 }
 
@@ -161,6 +167,7 @@ struct dum_engine {
   uint64_t built_launches;
   // build scratch
   uint32_t *d_head, *d_next, *d_slow_list, *d_order;
+  uint32_t *d_dd_list;           // k_build_exec -> k_walk: walks needing the dedupe
   uint32_t *d_e_ops, *d_e_last;  // per exec ID: group operations / latest launch of the batch
   uint64_t *d_plan_agg;          // k_plan look-back slots (one per 256 staged launches)
   uint32_t *d_lead;              // exec IDs with faults of the batch (k_build.cu LeadDesc, 32 B each)
@@ -182,6 +189,27 @@ struct dum_engine {
   uint32_t *d_qkern, *d_qloff, *d_qeoff, *d_qgoff, *d_qnk;
   uint32_t *d_qrank, *d_qperm;  // window-size class rank per query; predict CTA order (largest first)  // per-query chain scratch (k_chain -> k_predict)
   unsigned long long *d_qbase;
+  // walk index (k_window.cu): holders per block, conflicts per walk (build
+  // end); residency facts per walk (predict time); fast/exact split
+  uint32_t *d_bcnt, *d_bhold;   // [W], [W][HOLD_MAX]
+  uint32_t *d_conf, *d_conf_n;  // [Emax][CONF_MAX], [Emax] (NONE = not recorded)
+  uint32_t *d_wnr, *d_wnres;    // [Emax] walk blocks without / with a frame
+  uint32_t *d_respos;           // [Emax][walk_cap] log positions of the latter
+  uint32_t *d_qroff, *d_qneed;  // [max queries][N+2], [max queries] (k_chain -> k_window)
+  unsigned long long *d_qvb;    // [max queries][2] victim-range bases (k_chain -> k_window)
+  unsigned long long *d_chunk_map;  // [chunk_cap] (q << 40 | list << 32 | chunk) of the fast queries' windows
+  uint64_t chunk_cap;
+  cudaStream_t side2;           // exact-path predict kernel beside the fast path
+  cudaEvent_t ev_fork2, ev_join2;
+  cudaStream_t side3;           // walk index (build end) and the fast-path selection
+  cudaEvent_t ev_join3, ev_widx;
+  // closed-loop replay scratch (k_sim.cu, allocated by the first dum_simulate)
+  bool sim_ready;
+  uint32_t sim_acc_cap;
+  uint64_t sim_pair_cap;
+  uint32_t *sim_acc_bits, *sim_faults, *sim_pairs, *sim_wb, *sim_inv, *sim_pf;
+  uint64_t *sim_foff, *sim_ranges;
+  dum_query *sim_q;
   // residency
   uint32_t *d_frame_of, *d_stamp_of, *d_block_of, *d_free_bits, *d_inactive_bits, *d_res_bits;
   uint32_t *d_lrm_blk, *d_lrm_stamp;   // LRM log: block | inactive << 31, migration stamp
@@ -208,5 +236,7 @@ struct dum_engine {
   std::vector<cudaEvent_t> event_pool;
   double t_ms[DUM_NTIMERS];
   uint64_t t_cnt[DUM_NTIMERS];
-  int predict_smem, select_smem, build_smem, ingest_smem;  // dynamic smem attributes applied (per engine / device)
+  int predict_smem, select_smem, build_smem, ingest_smem;
+  uint32_t apply_grid, walk_grid;  // persistent build grids (occupancy x SMs), set on first build
+  uint32_t copy_grid, sel_grid;    // persistent predict grids (k_window.cu)  // dynamic smem attributes applied (per engine / device)
 };

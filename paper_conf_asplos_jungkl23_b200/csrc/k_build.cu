@@ -27,6 +27,7 @@
 //  k_walk_slow    sequential one-warp walker; takes the exec IDs whose walk
 //                 the parallel path cannot prove (never on the configs
 //                 measured; kept for exactness on any input).
+#include <algorithm>
 #include <cstdio>
 #include <cstdlib>
 #include <vector>
@@ -34,6 +35,7 @@
 #include "device_util.cuh"
 #include "kernels.cuh"
 #include "corr.cuh"
+#include "predict.cuh"
 #include "walk_seq.cuh"
 
 namespace dum {
@@ -41,7 +43,7 @@ namespace dum {
 constexpr uint32_t GCAP = 256;     // launches of one exec ID per build batch
 constexpr int PLAN_NT = 256;
 constexpr int AP_NT = 256;         // k_apply threads
-constexpr uint32_t OPP = 256;      // target operations per apply partition
+constexpr uint32_t OPP = 1024;     // target operations per apply partition
 constexpr uint32_t PMAX = 64;      // partitions per exec ID (<= R / 32)
 constexpr uint32_t AP_OPCAP = 1024;  // selected operations per apply round
 constexpr uint32_t AP_SCAN = 2 * AP_NT;  // operations scanned per selection step
@@ -63,6 +65,7 @@ __global__ void k_build_prep(uint32_t n_staged, uint32_t k0, const uint32_t *__r
   if (j == 0) {
     st->pool_big = 0;
     st->n_slow = 0;
+    st->n_dd = 0;
     st->n_items = 0;  // k_plan's last chunk writes the list sizes
     st->n_leads = 0;
   }
@@ -108,13 +111,15 @@ struct RegSet {
     const int w = k / (1 + MAXS), r = k % (1 + MAXS);
     return r == 0 ? tag[w] : sc[w][r - 1];
   }
+  // CG: load through L2 only (sets written earlier by this CTA, k_build_exec)
+  template <bool CG = false>
   __device__ __forceinline__ void load(const uint32_t *p, uint32_t A, uint32_t S) {
     if (A == MAXA && S == MAXS) {
       // exact geometry: a few 16 B vector loads instead of A(1+S) scalar ones
       const uint4 *p4 = reinterpret_cast<const uint4 *>(p);
       uint4 v[NV];
 #pragma unroll
-      for (int i = 0; i < NV; ++i) v[i] = p4[i];
+      for (int i = 0; i < NV; ++i) v[i] = CG ? __ldcg(p4 + i) : p4[i];
 #pragma unroll
       for (int k = 0; k < NW; ++k) {
         const uint4 &x = v[k / 4];
@@ -128,10 +133,10 @@ struct RegSet {
 #pragma unroll
       for (int j = 0; j < MAXS; ++j) sc[w][j] = NONE;
       if (w < (int)A) {
-        tag[w] = p[w * (1 + S)];
+        tag[w] = CG ? __ldcg(p + w * (1 + S)) : p[w * (1 + S)];
 #pragma unroll
         for (int j = 0; j < MAXS; ++j)
-          if (j < (int)S) sc[w][j] = p[w * (1 + S) + 1 + j];
+          if (j < (int)S) sc[w][j] = CG ? __ldcg(p + w * (1 + S) + 1 + j) : p[w * (1 + S) + 1 + j];
       }
     }
   }
@@ -257,6 +262,8 @@ struct BuildArgs {
   const uint32_t *order;       // [3][n_staged] faulting launches by size class
   unsigned long long *plan_agg;  // [k_plan CTAs] published chunk totals (flag << 63 | leads << 32 | items)
   DevState *st;
+  uint32_t seq_walks;          // DUM_CFG_SEQ_WALKS
+  uint32_t *dd_list;           // k_build_exec -> k_walk: walks that need the min-position dedupe (desc indices)
 };
 
 __global__ void __launch_bounds__(PLAN_NT) k_plan(BuildArgs a) {
@@ -400,10 +407,10 @@ __global__ void __launch_bounds__(AP_NT) k_apply(BuildArgs a) {
   const uint32_t tid = threadIdx.x;
   const uint32_t A = g.A, S = g.S;
   // one CTA per item; the grid is the host's upper bound on the item count
-  const uint32_t t = blockIdx.x;
-  if (t >= *(volatile uint32_t *)&a.st->n_items) return;
+  // persistent: the grid is sized by occupancy, the item count is on the device
+  const uint32_t n_items = *(volatile uint32_t *)&a.st->n_items;
   uint32_t nsets = 0;
-  {
+  for (uint32_t t = blockIdx.x; t < n_items; t += gridDim.x) {
     const uint2 it = a.items[t];
     const uint32_t c = it.y & 0xFFFFu, P = it.y >> 16;
     const LeadDesc d = a.desc[it.x];
@@ -545,13 +552,246 @@ __global__ void __launch_bounds__(AP_NT) k_apply(BuildArgs a) {
       m = P == 1 ? m + min(AP_SCAN, n_ops - g0) : s_m;
     }
     if (m) apply_staged();
+    __syncthreads();  // the next item reuses the shared state
   }
   // one global atomic per CTA (a per-thread atomic on one address serialises
   // hundreds of thousands of updates in L2)
-  nsets = __reduce_add_sync(0xffffffffu, nsets);
-  if ((tid & 31) == 0 && nsets) atomicAdd(&s_ng, nsets);
+  __shared__ uint32_t s_sets;
+  if (tid == 0) s_sets = 0;
   __syncthreads();
-  if (tid == 0 && s_ng) ctr_add(a.st, DUM_CTR_SETS, s_ng);
+  nsets = __reduce_add_sync(0xffffffffu, nsets);
+  if ((tid & 31) == 0 && nsets) atomicAdd(&s_sets, nsets);
+  __syncthreads();
+  if (tid == 0 && s_sets) ctr_add(a.st, DUM_CTR_SETS, s_sets);
+}
+
+// ---------------------------------------------------------------------------
+// k_build_exec: a4 + a5 + a6 of one exec ID per item (persistent, largest
+// exec IDs first), fused so that the walk reads the sets its own apply just
+// wrote (L2-hot) and one kernel replaces the partitioned apply and the walk.
+//  apply  the exec ID's operations (INSERT b_j into row(b_{j-1}), TOUCH b_j;
+//         PAPER.md L168, L174, L216; D7-D10) in rounds of BX_RC in position
+//         order; per round the operations are linked per set (shared head
+//         table over the R sets) and one owner thread applies a set's
+//         operations in position order with the set in registers (SURVEY P2:
+//         operations on different sets commute).
+//  walk   Start/End (D11) and WALK(e, NONE) (L218-L224; D13) as k_walk's fast
+//         path: the walk is the prefix C[0 .. t+1] of the latest launch when
+//         rows C[0..t] each hold the single successor C[i+1] (see k_walk);
+//         any other walk goes to k_walk's exact dedupe (dd_list) or the
+//         sequential walker (slow_list).
+// ---------------------------------------------------------------------------
+constexpr int BX_NT = 256;
+constexpr uint32_t BX_RC = 1024;  // operations per apply round
+
+template <int MAXA, int MAXS>
+__global__ void __launch_bounds__(BX_NT, 4) k_build_exec(BuildArgs a) {
+  extern __shared__ uint32_t bx[];  // set heads [R] | opb | onx | lnk | sll [BX_RC each]
+  __shared__ uint32_t grp[GCAP], seg[GCAP + 1];
+  __shared__ unsigned long long goff[GCAP];
+  __shared__ uint32_t s_ng, s_nsl, s_tev, s_multi, s_nrun, s_sets;
+  const Geo &g = a.g;
+  const uint32_t tid = threadIdx.x, lane = tid & 31;
+  const uint32_t A = g.A, S = g.S, R = g.R;
+  uint32_t *shead = bx, *opb = bx + R, *onx = opb + BX_RC, *lnk = onx + BX_RC, *sll = lnk + BX_RC;
+  if (blockIdx.x == 0 && tid < 4) a.st->cls_cnt[tid] = 0;  // k_plan has read them; zero for the next build
+  for (uint32_t x = tid; x < R; x += BX_NT) shead[x] = NONE;  // kept clean by the owners
+  if (tid == 0) s_sets = 0;
+  const uint32_t n_leads = *(volatile uint32_t *)&a.st->n_leads;
+  uint32_t nsets = 0;
+  for (uint32_t li = blockIdx.x; li < n_leads; li += gridDim.x) {
+    const LeadDesc d = a.desc[li];
+    const uint32_t e = d.e;
+    uint32_t ng = 1;
+    if (d.single) {  // the common case: no list to chase
+      if (tid == 0) {
+        seg[0] = 0;
+        seg[1] = d.n_ops;
+        goff[0] = d.off_last;
+        s_nsl = 0;
+      }
+      __syncthreads();
+    } else {
+      if (tid == 0) s_nsl = 0;
+      ng = load_group(a, d.j, e, grp, seg, goff, sll, &s_ng, BX_NT);
+    }
+    const uint32_t n_ops = seg[ng];
+    uint32_t *tbl_e = a.tbl + (uint64_t)e * R * g.stride;
+    // ---- a4: the operations, BX_RC per round (rounds in position order) ----
+    for (uint32_t g0 = 0; g0 < n_ops; g0 += BX_RC) {
+      const uint32_t m = min(BX_RC, n_ops - g0);
+      for (uint32_t p = tid; p < m; p += BX_NT) {
+        const uint32_t gp = g0 + p;
+        uint32_t lo = 0, hi = ng;  // seg[lo] <= gp < seg[lo+1]
+        while (hi - lo > 1) {
+          const uint32_t mid = (lo + hi) >> 1;
+          if (seg[mid] <= gp) lo = mid;
+          else hi = mid;
+        }
+        const uint64_t base = goff[lo] + (gp - seg[lo]);
+        uint32_t b = a.stage_norm[base];
+        // INSERT target: the next fault of the same launch
+        const uint32_t nx = gp + 1 < seg[lo + 1] ? a.stage_norm[base + 1] : NONE;
+        if (!GUARD(a.st, b < g.W, b)) b = 0;
+        opb[p] = b;
+        onx[p] = nx;
+        const uint32_t sx = row_of(g, b);
+        const uint32_t old = atomicExch(&shead[sx], p);
+        lnk[p] = old;
+        if (old == NONE) sll[atomicAdd(&s_nsl, 1u)] = sx;  // a set touched first in this round
+      }
+      __syncthreads();
+      const uint32_t nsl = s_nsl;
+      constexpr int OWN = (MAXA * (1 + MAXS) <= 10) ? 2 : 1;  // sets per owner with loads in flight
+      for (uint32_t k0 = tid; k0 < nsl; k0 += BX_NT * OWN) {
+        RegSet<MAXA, MAXS> rs[OWN];
+        uint32_t sx[OWN], hd[OWN];
+#pragma unroll
+        for (int q = 0; q < OWN; ++q) {
+          const uint32_t k = k0 + q * BX_NT;
+          sx[q] = k < nsl ? sll[k] : NONE;
+          hd[q] = NONE;
+          if (sx[q] != NONE) {
+            hd[q] = shead[sx[q]];
+            rs[q].template load<true>(tbl_e + (uint64_t)sx[q] * g.stride, A, S);
+          }
+        }
+#pragma unroll
+        for (int q = 0; q < OWN; ++q) {
+          if (sx[q] == NONE) continue;
+          ++nsets;
+          // the set's operations in position order: repeatedly the smallest
+          // remaining position of its (short) list
+          uint32_t last = NONE;
+          for (;;) {
+            uint32_t best = NONE;
+            for (uint32_t x = hd[q]; x != NONE; x = lnk[x])
+              if ((last == NONE || x > last) && (best == NONE || x < best)) best = x;
+            if (best == NONE) break;
+            rs[q].touch(opb[best], A);
+            if (onx[best] != NONE) rs[q].insert0(onx[best], S);
+            last = best;
+          }
+          rs[q].store(tbl_e + (uint64_t)sx[q] * g.stride, A, S);
+          shead[sx[q]] = NONE;
+        }
+      }
+      if (tid == 0) s_nsl = 0;
+      __syncthreads();  // the round's sets are written; the next round may link them again
+    }
+    // ---- a5 + a6: Start/End and the walk of the post-build table ----
+    const uint32_t n = d.n_last;
+    const uint32_t *C = a.stage_norm + d.off_last;
+    const uint32_t start = C[0], end = C[n - 1];
+    if (tid == 0) {
+      a.start_end[2 * e] = start;
+      a.start_end[2 * e + 1] = end;
+      ctr_add(a.st, DUM_CTR_EXEC_BUILT, 1);
+      ctr_add(a.st, DUM_CTR_OPS, d.n_ops);
+      // the group bookkeeping of this batch is consumed (prep and plan are done)
+      a.head[e] = NONE;
+      a.e_ops[e] = 0;
+      a.e_last[e] = 0;
+      s_tev = NONE;
+      s_nrun = 0;
+      s_multi = NONE;
+    }
+    uint32_t *wout = a.walk + (uint64_t)e * g.walk_cap;
+    uint2 *wrun = reinterpret_cast<uint2 *>(a.wrun) + (uint64_t)e * g.walk_cap;
+    if (n == 1 || (a.seq_walks && n > 1)) {
+      if (tid == 0) {
+        if (n == 1) {  // x == End: the walk is [Start]
+          wout[0] = start;
+          a.walk_len[e] = 1;
+          wrun[0] = make_uint2(start >> 5, 1u << (start & 31));
+          a.wrun_len[e] = 1;
+          ctr_add(a.st, DUM_CTR_WALK_OUT, 1);
+          ctr_add(a.st, DUM_CTR_WALK_PREFIX, 1);
+        } else {  // DUM_CFG_SEQ_WALKS: the sequential walker builds every walk
+          a.slow_list[atomicAdd(&a.st->n_slow, 1u)] = e;
+        }
+      }
+      __syncthreads();
+      continue;
+    }
+    __syncthreads();
+    // pass A: rows of C[0 .. n-2] (written above by this CTA: L2) -> stop events
+    constexpr int WB = (MAXA * (1 + MAXS) <= 10) ? 2 : 1;  // rows per thread in flight
+    for (uint32_t i0 = tid; i0 < n - 1; i0 += BX_NT * WB) {
+      uint32_t x[WB], xn[WB];
+      RegSet<MAXA, MAXS> rs[WB];
+#pragma unroll
+      for (int q = 0; q < WB; ++q) {
+        const uint32_t i = i0 + q * BX_NT;
+        x[q] = i < n - 1 ? C[i] : NONE;
+        xn[q] = i < n - 1 ? C[i + 1] : NONE;
+      }
+#pragma unroll
+      for (int q = 0; q < WB; ++q)
+        if (x[q] != NONE) rs[q].template load<true>(tbl_e + (uint64_t)row_of(g, x[q]) * g.stride, A, S);
+#pragma unroll
+      for (int q = 0; q < WB; ++q) {
+        if (x[q] == NONE) continue;
+        const uint32_t i = i0 + q * BX_NT;
+        uint32_t row[1 + MAXS];
+        rs[q].export_row(x[q], A, S, row);
+        const uint32_t cnt = row[0];
+        uint32_t ev = 0;
+        if (cnt == NONE) {
+          ev = 1;  // row missing: stop, nothing emitted at this step
+        } else {
+          bool hit = false;
+#pragma unroll
+          for (int k = 0; k < MAXS; ++k) hit |= (uint32_t)k < cnt && row[1 + k] == end;
+          if (hit) ev = 2;                              // a successor is End: stop after emitting
+          else if (cnt == 0 || row[1] != xn[q]) ev = 3;  // speculation violated -> sequential walker
+          if (cnt > 1) atomicMin(&s_multi, i);
+        }
+        if (ev) atomicMin(&s_tev, (i << 2) | ev);
+      }
+    }
+    __syncthreads();
+    const uint32_t tev = s_tev;
+    const uint32_t t = tev >> 2;
+    if (tev == NONE || (tev & 3) == 3 || !GUARD(a.st, t + 1 < n, t)) {
+      if (tid == 0) a.slow_list[atomicAdd(&a.st->n_slow, 1u)] = e;
+    } else if (s_multi <= t) {
+      if (tid == 0) a.dd_list[atomicAdd(&a.st->n_dd, 1u)] = li;  // k_walk: min-position dedupe
+    } else {
+      // fast path: the walk is C[0 .. t] (+ C[t+1] when a successor is End),
+      // duplicate-free; written with its bitmap runs for k_predict
+      const uint32_t qlen = t + 1 + ((tev & 3) == 2 ? 1u : 0u);
+      for (uint32_t c0 = 0; c0 < qlen; c0 += BX_NT) {
+        const uint32_t p = c0 + tid;
+        const bool keep = p < qlen;
+        const uint32_t val = keep ? C[p] : NONE;
+        if (keep && p < g.walk_cap) wout[p] = val;
+        const uint32_t wkey = keep ? val >> 5 : NONE;
+        const uint32_t gm = __match_any_sync(0xffffffffu, wkey);
+        const uint32_t msk = __reduce_or_sync(gm, keep ? 1u << (val & 31) : 0u);
+        const bool lead = keep && lane == (uint32_t)(__ffs(gm) - 1);
+        const uint32_t lm = __ballot_sync(0xffffffffu, lead);
+        uint32_t rb = 0;
+        if (lane == 0 && lm) rb = atomicAdd(&s_nrun, (uint32_t)__popc(lm));
+        rb = __shfl_sync(0xffffffffu, rb, 0) + __popc(lm & ((1u << lane) - 1));
+        if (lead && rb < g.walk_cap) wrun[rb] = make_uint2(wkey, msk);
+      }
+      __syncthreads();
+      if (tid == 0) {
+        if (qlen > g.walk_cap) set_err(a.st, ERR_ECAPACITY, qlen);
+        a.walk_len[e] = qlen;
+        a.wrun_len[e] = s_nrun;
+        ctr_add(a.st, DUM_CTR_WALK_ROWS, t + 1);
+        ctr_add(a.st, DUM_CTR_WALK_OUT, qlen);
+        ctr_add(a.st, DUM_CTR_WALK_PREFIX, 1);
+      }
+    }
+    __syncthreads();  // the next item reuses the shared state
+  }
+  nsets = __reduce_add_sync(0xffffffffu, nsets);
+  if (lane == 0 && nsets) atomicAdd(&s_sets, nsets);
+  __syncthreads();
+  if (tid == 0 && s_sets) ctr_add(a.st, DUM_CTR_SETS, s_sets);
 }
 
 // ---------------------------------------------------------------------------
@@ -585,9 +825,12 @@ __global__ void __launch_bounds__(WK_NT) k_walk(BuildArgs a) {
   const uint32_t tid = threadIdx.x;
   const uint32_t A = g.A, S = g.S;
   // one CTA per exec ID; the grid is the host's upper bound (staged launches)
-  const uint32_t li = blockIdx.x;
-  if (li == 0 && tid < 4) a.st->cls_cnt[tid] = 0;  // k_plan has read them; zero for the next build
-  if (li >= *(volatile uint32_t *)&a.st->n_leads) return;
+  if (blockIdx.x == 0 && tid < 4) a.st->cls_cnt[tid] = 0;  // k_plan has read them; zero for the next build
+  // persistent over the walks k_build_exec could not prove to be a prefix of
+  // the latest launch (dd_list), grid sized by occupancy
+  const uint32_t n_dd = *(volatile uint32_t *)&a.st->n_dd;
+  for (uint32_t xi = blockIdx.x; xi < n_dd; xi += gridDim.x) {
+  const uint32_t li = a.dd_list[xi];
   do {  // (breaks = the early ends of the walk)
     const LeadDesc d = a.desc[li];
     const uint32_t e = d.e;
@@ -610,6 +853,10 @@ __global__ void __launch_bounds__(WK_NT) k_walk(BuildArgs a) {
     }
     uint32_t *wout = a.walk + (uint64_t)e * g.walk_cap;
     uint2 *wrun = reinterpret_cast<uint2 *>(a.wrun) + (uint64_t)e * g.walk_cap;
+    if (a.seq_walks && n > 1) {  // DUM_CFG_SEQ_WALKS: the sequential walker builds every walk
+      if (tid == 0) a.slow_list[atomicAdd(&a.st->n_slow, 1u)] = e;
+      break;
+    }
     if (n == 1) {  // x == End: the walk is [Start]
       if (tid == 0) {
         wout[0] = start;
@@ -617,6 +864,7 @@ __global__ void __launch_bounds__(WK_NT) k_walk(BuildArgs a) {
         wrun[0] = make_uint2(start >> 5, 1u << (start & 31));
         a.wrun_len[e] = 1;
         ctr_add(a.st, DUM_CTR_WALK_OUT, 1);
+        ctr_add(a.st, DUM_CTR_WALK_PREFIX, 1);
       }
       break;
     }
@@ -721,6 +969,7 @@ __global__ void __launch_bounds__(WK_NT) k_walk(BuildArgs a) {
         a.wrun_len[e] = s_nrun;
         ctr_add(a.st, DUM_CTR_WALK_ROWS, t + 1);
         ctr_add(a.st, DUM_CTR_WALK_OUT, qlen);
+        ctr_add(a.st, DUM_CTR_WALK_PREFIX, 1);
       }
       break;
     }
@@ -817,8 +1066,11 @@ __global__ void __launch_bounds__(WK_NT) k_walk(BuildArgs a) {
       a.wrun_len[e] = s_nrun;
       ctr_add(a.st, DUM_CTR_WALK_ROWS, t + 1);
       ctr_add(a.st, DUM_CTR_WALK_OUT, outn);
+      ctr_add(a.st, DUM_CTR_WALK_DEDUPE, 1);
     }
   } while (false);
+  __syncthreads();  // the next item reuses the shared state
+  }
 }
 
 __global__ void k_walk_slow(Geo g, const uint32_t *tbl, const uint32_t *start_end, uint32_t *walk,
@@ -836,6 +1088,7 @@ __global__ void k_walk_slow(Geo g, const uint32_t *tbl, const uint32_t *start_en
         n = 0;
       }
       walk_len[e] = n;
+      ctr_add(st, DUM_CTR_WALK_SLOW, 1);
     }
     __syncwarp();
     // bitmap runs of the new walk (see pass C of k_walk)
@@ -864,20 +1117,27 @@ __global__ void k_walk_slow(Geo g, const uint32_t *tbl, const uint32_t *start_en
 template <int MA, int MS>
 static cudaError_t launch_apply_walk(dum_engine *e, const BuildArgs &ba, cudaStream_t s) {
   const size_t wsmem = (size_t)(WK_RC + WK_CQ + 2 * WK_QCAP) * 4;
-  // the attribute is per device and function: raised by every engine on its own device
+  const size_t bsmem = (size_t)(e->g.R + 4 * BX_RC) * 4;
+  // the attributes are per device and function: raised by every engine on its own device;
+  // persistent grids: resident CTAs per SM x SMs (the item counts are on the device)
   if (!e->build_smem) {
     cudaFuncSetAttribute(k_walk<MA, MS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)wsmem);
-    e->build_smem = (int)wsmem;
+    cudaFuncSetAttribute(k_build_exec<MA, MS>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bsmem);
+    e->build_smem = (int)std::max(wsmem, bsmem);
+    int dev = 0, sms = 148, nb = 1, nw = 1;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_build_exec<MA, MS>, BX_NT, bsmem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nw, k_walk<MA, MS>, WK_NT, wsmem);
+    e->apply_grid = (uint32_t)std::max(1, nb * sms);
+    e->walk_grid = (uint32_t)std::max(1, std::min(nw * sms, 2 * sms));
   }
-  // host upper bounds of the device-side counts (the surplus CTAs return at once):
-  // items = sum over exec IDs of ceil(ops / OPP) <= launches + faults / OPP
-  const uint32_t n_items_max = (uint32_t)std::min<uint64_t>(e->items_cap, e->n_staged + e->staged_faults / OPP + 1);
   {
     TimerScope t(e, DUM_T_APPLY_WALK, s);
-    k_apply<MA, MS><<<n_items_max, AP_NT, 0, s>>>(ba);
+    k_build_exec<MA, MS><<<std::min(e->n_staged, e->apply_grid), BX_NT, bsmem, s>>>(ba);
   }
   TimerScope t(e, DUM_T_WALK, s);
-  k_walk<MA, MS><<<e->n_staged, WK_NT, wsmem, s>>>(ba);
+  k_walk<MA, MS><<<std::min(e->n_staged, e->walk_grid), WK_NT, wsmem, s>>>(ba);  // dd_list only
   return cudaGetLastError();
 }
 
@@ -885,6 +1145,7 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   const uint32_t n = e->n_staged;
   if (n == 0) return cudaSuccess;
   cudaStreamWaitEvent(s, e->ev_join, 0);  // the previous build's jump tables read corr
+  cudaStreamWaitEvent(s, e->ev_widx, 0);  // the previous build's walk index reads the walk cache
   BuildArgs ba;
   ba.g = e->g;
   ba.n_staged = n;
@@ -911,6 +1172,8 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   ba.order = e->d_order;
   ba.plan_agg = reinterpret_cast<unsigned long long *>(e->d_plan_agg);
   ba.st = e->d_state;
+  ba.seq_walks = (e->cfg.flags & DUM_CFG_SEQ_WALKS) ? 1u : 0u;
+  ba.dd_list = e->d_dd_list;
   {
     TimerScope t(e, DUM_T_BUILD_PREP, s);
     k_build_prep<<<(n + 255) / 256, 256, 0, s>>>(n, (uint32_t)e->built_launches, e->d_stage_exec, e->d_stage_cnt,
@@ -939,6 +1202,10 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
     TimerScope t(e, DUM_T_WALK_SLOW, s);
     k_walk_slow<<<e->n_walk_slots, 32, 0, s>>>(e->g, e->d_tbl, e->d_start_end, e->d_walk, e->d_walk_len,
                                                e->d_wrun, e->d_wrun_len, e->d_slow_list, ws, e->d_state);
+  }
+  {
+    const cudaError_t we = launch_walk_index(e, s);  // k_window.cu: conflicts between the new walks
+    if (we != cudaSuccess) return we;
   }
   // no join here: the jump tables keep building on the side stream, past the
   // end of this call; the next reader of the correlation table (predict's

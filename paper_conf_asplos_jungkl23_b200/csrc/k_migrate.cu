@@ -100,6 +100,7 @@ struct MigArgs {
   int dir;
   const uint32_t *blocks, *dst;
   uint32_t n;
+  const uint64_t *rng;  // device (begin, end) into blocks: the list is blocks[begin, end), n caps it (closed loop)
   uint32_t W, C;
   uint32_t *frame_of, *stamp_of, *block_of, *free_bits, *lrm_blk, *lrm_stamp, *res_bits, *logpos;
   const uint32_t *inactive;
@@ -144,7 +145,15 @@ __global__ void __launch_bounds__(PLAN_NT) k_mig_plan(MigArgs a) {
     st->mig_ok = 0;
   }
   __syncthreads();
-  const uint32_t n = a.n;
+  uint32_t n = a.n;
+  const uint32_t *blocks_in = a.blocks;
+  if (a.rng) {  // a device-sized list (dum_simulate): blocks[rng[0], rng[1])
+    const uint64_t b0 = a.rng[0], b1 = a.rng[1];
+    const uint64_t len = b1 > b0 ? b1 - b0 : 0;
+    if (len < n) n = (uint32_t)len;
+    blocks_in += b0;
+  }
+  a.blocks = blocks_in;
   if (a.dir == DUM_H2D) {
     if (n > st->free_count) {
       if (tid == 0) set_err(st, ERR_ECAPACITY, n);
@@ -409,12 +418,13 @@ static int copy_grid(uint32_t n) {
 }
 
 cudaError_t launch_migrate(dum_engine *e, int dir, const uint32_t *blocks, const uint32_t *dst, uint32_t n,
-                           uint32_t method, cudaStream_t s) {
+                           uint32_t method, cudaStream_t s, const uint64_t *rng) {
   MigArgs a;
   a.dir = dir;
   a.blocks = blocks;
   a.dst = dst;
   a.n = n;
+  a.rng = rng;
   a.W = e->g.W;
   a.C = e->g.C;
   a.frame_of = e->d_frame_of;
@@ -437,6 +447,8 @@ cudaError_t launch_migrate(dum_engine *e, int dir, const uint32_t *blocks, const
   }
   e->kernel_launches += 1;
   if (dir == DUM_INVALIDATE) return cudaGetLastError();
+  // metadata-only engines (dum_simulate at B/G scale): the residency moves, no bytes
+  if (!e->frame_pool || (dir != DUM_D2D && !e->host_arena)) return cudaGetLastError();
   const bool compaction = dir == DUM_D2D && blocks == nullptr;
   if (method == 2) {
     // copy-engine baseline: needs the plan on the host

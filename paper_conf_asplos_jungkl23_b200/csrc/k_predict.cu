@@ -22,6 +22,7 @@
 //                  re-compaction overwrite the output.
 //                  SELECT: the fused pre-eviction selection of a8 reuses the
 //                  window bitmap (select_tail.cuh).
+#include <algorithm>
 #include <cstdio>
 #include <cstdlib>
 #include <vector>
@@ -29,6 +30,7 @@
 #include "corr.cuh"
 #include "device_util.cuh"
 #include "kernels.cuh"
+#include "predict.cuh"
 #include "select_tail.cuh"
 #include "walk_seq.cuh"
 
@@ -36,7 +38,6 @@ namespace dum {
 
 constexpr int PRED_NT = 512;
 constexpr int NWARP = PRED_NT / 32;
-constexpr uint32_t MAXN = 128;   // degree_n limit
 constexpr uint32_t DLCAP = 512;   // duplicated blocks recorded by pass 1 (more: hash every element)
 constexpr uint32_t DHCAP = 2048;  // shared hash of the duplicated blocks (block -> min position + 1)
 static_assert(2 * DHCAP >= SEL_CHUNK, "the dup hash region doubles as the selection stage");
@@ -83,6 +84,7 @@ __global__ void k_anchor_walk(Geo g, const dum_query *__restrict__ q, uint32_t n
         n = 0;
       }
     }
+    if (threadIdx.x == 0) ctr_add(st, DUM_CTR_ANCHOR_WALKS, 1);
     unsigned long long base = 0;
     if (threadIdx.x == 0 && n) base = atomicAdd(&st->pool_anchor, (unsigned long long)n);
     base = __shfl_sync(0xffffffffu, base, 0);
@@ -100,51 +102,22 @@ __global__ void k_anchor_walk(Geo g, const dum_query *__restrict__ q, uint32_t n
   }
 }
 
-struct PredArgs {
-  Geo g;
-  const dum_query *q;
-  uint32_t nq;
-  const CorrSlot *corr;
-  uint32_t corr_cap;
-  const uint32_t *jump;  // [levels][corr_cap]
-  const uint32_t *walk, *walk_len;
-  const uint32_t *wrun, *wrun_len;  // walk bitmap runs (k_walk pass C / k_walk_slow)
-  const uint32_t *anchor_pool;
-  const uint64_t *anchor_range;
-  uint32_t *pairs;
-  uint64_t cap;
-  uint64_t *range;
-  uint32_t *kern_off, *chain;
-  DevState *st;
-  uint32_t nwords;  // bitmap words
-  // per-query scratch written by k_chain
-  uint32_t *qkern;  // [nq][N+1]
-  uint32_t *qloff;  // [nq][N+2]
-  uint32_t *qeoff;  // [nq][N+2] run-entry offsets of the window's lists
-  uint32_t *qgoff;  // [nq][N+2] 128-block copy-chunk offsets of the window's lists
-  uint32_t *qnk;    // [nq]
-  uint32_t *qrank;  // [nq] class << 24 | rank within the window-size class
-  uint32_t *qperm;  // [nq] k_predict CTA b answers query qperm[b] (largest windows first)
-  unsigned long long *qbase;  // [nq]
-  uint32_t *big_pool;         // scratch for the exact slow path
-  uint64_t big_entries;
-  SelectOut so;     // fused a8 outputs (SELECT only)
-  uint64_t *needed;             // pair-pool size after every reservation (k_chain's last CTA), or null
-};
+
 
 constexpr int CHAIN_WARPS = 8;
-constexpr int NQCLS = 5;  // window-size classes of the predict CTA order
-constexpr uint32_t CHUNK_B = 128;  // window blocks per copy chunk (one warp: 4 coalesced steps)
 
 __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
-  __shared__ uint32_t skern[CHAIN_WARPS][MAXN + 1];
-  __shared__ uint32_t s_u[CHAIN_WARPS];
-  __shared__ unsigned long long s_base;
+  __shared__ uint32_t skern[CHAIN_WARPS][MAXN + 1], sgoff[CHAIN_WARPS][MAXN + 2];
+  __shared__ uint32_t s_u[CHAIN_WARPS], s_need[CHAIN_WARPS], s_gu[CHAIN_WARPS];
+  __shared__ unsigned long long s_base, s_wbase, s_ibase, s_gbase;
   const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const uint32_t qi = blockIdx.x * CHAIN_WARPS + w;
   const uint32_t below = (1u << lane) - 1;
   const Geo &g = a.g;
   uint32_t U = 0;
+  bool slow = false;   // the query goes to the exact kernel (k_predict) instead of k_window
+  uint32_t qneed = 0;  // fast query, fused select: victims to reserve in each output list
+  uint32_t GUq = 0;    // copy chunks of the window (k_copy_fast)
   if (qi < a.nq) {
     const dum_query Q = a.q[qi];
     const bool anchored = Q.anchor != NONE;
@@ -181,6 +154,10 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
     uint32_t *goff = a.qgoff + (uint64_t)qi * (g.N + 2);
     uint32_t RU = 0;  // bitmap-run entries of the window (k_predict pass 1)
     uint32_t GU = 0;  // 128-block copy chunks of the window (k_predict copy)
+    uint32_t *roff = a.qroff + (uint64_t)qi * (g.N + 2);  // prefix of the lists' resident blocks
+    bool conflict = false;
+    uint32_t nonres = 0;  // (per lane) window blocks without a frame
+    uint32_t nwres = 0;   // (warp-uniform) window blocks with a frame
     for (uint32_t d0 = 0; d0 < nk; d0 += 32) {
       const uint32_t d = d0 + lane;
       const bool v = d < nk, anc0 = d == 0 && anchored;
@@ -195,19 +172,43 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
             len = 0;
             break;
           }
+      // fast-path test (k_window.cu): a walk whose recorded conflicts meet
+      // the chain, or whose conflicts were too many to record
+      uint32_t wres = 0;  // this step's resident window blocks (k_window marks their log positions)
+      if (len && !anc0) {
+        const uint32_t cn = __ldg(a.conf_n + e);
+        if (cn == NONE) {
+          conflict = true;
+        } else {
+          // the conflict row, 4 entries per 16 B load (CONF_MAX words, 16 B aligned)
+          const uint4 *cr = reinterpret_cast<const uint4 *>(a.conf + (uint64_t)e * CONF_MAX);
+          for (uint32_t k0 = 0; k0 < cn; k0 += 4) {
+            const uint4 x = __ldg(cr + k0 / 4);
+            const uint32_t c4[4] = {x.x, x.y, x.z, x.w};
+            for (uint32_t k = 0; k < 4 && k0 + k < cn; ++k)
+              for (uint32_t y = 0; y < nk; ++y) conflict |= kern[y] == c4[k];
+          }
+        }
+        if (a.select) {
+          nonres += __ldg(a.wnr + e);
+          wres = __ldg(a.wnres + e);
+        }
+      }
       // an anchored query's own walk has no runs: its blocks enter one by one
       const uint32_t rl = len ? (anc0 ? len : __ldg(a.wrun_len + e)) : 0u;
       const uint32_t gl = (len + CHUNK_B - 1) / CHUNK_B;
-      uint32_t incl = len, rincl = rl, gincl = gl;
+      uint32_t incl = len, rincl = rl, gincl = gl, wincl = wres;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
         const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
         const uint32_t z = __shfl_up_sync(0xffffffffu, rincl, o);
         const uint32_t u = __shfl_up_sync(0xffffffffu, gincl, o);
+        const uint32_t t = __shfl_up_sync(0xffffffffu, wincl, o);
         if (lane >= (uint32_t)o) {
           incl += y;
           rincl += z;
           gincl += u;
+          wincl += t;
         }
       }
       if (v) {
@@ -215,26 +216,53 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
         loff[d + 1] = U + incl;
         eoff[d + 1] = RU + rincl;
         goff[d + 1] = GU + gincl;
+        sgoff[w][d + 1] = GU + gincl;
+        if (a.select) roff[d + 1] = nwres + wincl;
       }
       U += __shfl_sync(0xffffffffu, incl, 31);
       RU += __shfl_sync(0xffffffffu, rincl, 31);
       GU += __shfl_sync(0xffffffffu, gincl, 31);
+      nwres += __shfl_sync(0xffffffffu, wincl, 31);
     }
     if (lane == 0) {
       loff[0] = 0;
       eoff[0] = 0;
       goff[0] = 0;
+      sgoff[w][0] = 0;
+      roff[0] = 0;
       a.qnk[qi] = nk;
     }
+    slow = anchored || __any_sync(0xffffffffu, conflict);
+    nonres = __reduce_add_sync(0xffffffffu, nonres);
+    if (a.select && !slow) {
+      // need = max(0, window blocks without a frame - free frames) (D18);
+      // k_window's selection scans log positions [head, head + need + nwres +
+      // stale entries) at most: it must stay inside its position bitmap
+      const uint32_t nfree = *(volatile uint32_t *)&a.st->free_count;
+      qneed = nonres > nfree ? nonres - nfree : 0;
+      const uint32_t span = *(volatile uint32_t *)&a.st->lrm_tail - *(volatile uint32_t *)&a.st->lrm_head;
+      const uint32_t stale = span - *(volatile uint32_t *)&a.st->n_resident;
+      if ((uint64_t)qneed + nwres + stale > POS_WORDS * 32ull) slow = true;
+    }
+    if (slow) qneed = 0;  // the exact kernel reserves its own victim ranges
+    GUq = slow ? 0u : GU;
   }
   // CTA-aggregated output reservation and window-size class counts (one
   // global atomic per CTA and class instead of one per query)
-  __shared__ uint32_t s_cls[NQCLS], s_cbase[NQCLS], s_wcls[CHAIN_WARPS];
-  // window-size class (largest first) for k_predict's CTA order: the big
-  // windows start first instead of forming the tail
-  const uint32_t cls = U >= 14336 ? 0u : U >= 10240 ? 1u : U >= 6144 ? 2u : U >= 2048 ? 3u : 4u;
-  if (threadIdx.x < NQCLS) s_cls[threadIdx.x] = 0;
-  if (lane == 0) s_u[w] = U;
+  __shared__ uint32_t s_cls[2 * NQCLS], s_cbase[2 * NQCLS], s_wcls[CHAIN_WARPS];
+  // window-size class (largest first) for the CTA order of k_window / k_predict:
+  // the big windows start first instead of forming the tail; fast-path
+  // queries (classes 0 .. NQCLS-1) before exact-path ones
+  // (fast queries of a fused select: ordered by `need`, the length of their selection)
+  const uint32_t key = (a.select && !slow) ? 2 * qneed : U;
+  const uint32_t cls = (key >= 14336 ? 0u : key >= 10240 ? 1u : key >= 6144 ? 2u : key >= 2048 ? 3u : 4u) +
+                       (slow ? (uint32_t)NQCLS : 0u);
+  if (threadIdx.x < 2 * NQCLS) s_cls[threadIdx.x] = 0;
+  if (lane == 0) {
+    s_u[w] = U;
+    s_need[w] = qneed;
+    s_gu[w] = GUq;  // copy chunks of k_copy_fast
+  }
   __syncthreads();
   if (qi < a.nq && lane == 0) s_wcls[w] = atomicAdd(&s_cls[cls], 1u);  // rank within the CTA
   __syncthreads();
@@ -242,51 +270,75 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
     unsigned long long tot = 0;
     for (int i = 0; i < CHAIN_WARPS; ++i) tot += s_u[i];
     s_base = tot ? atomicAdd(&a.st->pool_pairs, tot) : 0ull;
+  } else if (threadIdx.x == 64) {
+    unsigned long long tot = 0;
+    for (int i = 0; i < CHAIN_WARPS; ++i) tot += s_gu[i];
+    s_gbase = tot ? atomicAdd(&a.st->pool_chunks, tot) : 0ull;
+  } else if (threadIdx.x == 32 && a.select) {
+    // victim ranges of the fast queries: `need` entries in each list (D18-D20)
+    unsigned long long tot = 0;
+    for (int i = 0; i < CHAIN_WARPS; ++i) tot += s_need[i];
+    s_wbase = tot ? atomicAdd(&a.st->pool_wb, tot) : 0ull;
+    s_ibase = tot ? atomicAdd(&a.st->pool_inv, tot) : 0ull;
   }
-  if (threadIdx.x < NQCLS) s_cbase[threadIdx.x] = s_cls[threadIdx.x] ? atomicAdd(&a.st->q_cls[threadIdx.x], s_cls[threadIdx.x]) : 0u;
+  if (threadIdx.x < 2 * NQCLS)
+    s_cbase[threadIdx.x] = s_cls[threadIdx.x] ? atomicAdd(&a.st->q_cls[threadIdx.x], s_cls[threadIdx.x]) : 0u;
   __syncthreads();
   if (qi < a.nq && lane == 0) {
-    unsigned long long base = s_base;
-    for (uint32_t i = 0; i < w; ++i) base += s_u[i];
+    unsigned long long base = s_base, nb = 0;
+    for (uint32_t i = 0; i < w; ++i) {
+      base += s_u[i];
+      nb += s_need[i];
+    }
     a.qbase[qi] = base;
+    if (a.select) {
+      a.qneed[qi] = qneed;
+      a.qvb[2 * qi] = s_wbase + nb;
+      a.qvb[2 * qi + 1] = s_ibase + nb;
+      if (qneed && (s_wbase + nb + qneed > a.so.cap || s_ibase + nb + qneed > a.so.cap))
+        set_err(a.st, ERR_ECAPACITY, (s_wbase > s_ibase ? s_wbase : s_ibase) + nb + qneed);
+    }
     if (base + U > a.cap) set_err(a.st, ERR_ECAPACITY, base + U);
-    a.qrank[qi] = (cls << 24) | (s_cbase[cls] + s_wcls[w]);
+    // class lists: query order for k_select_fast / k_predict = class by class
+    // (fast classes 0 .. NQCLS-1 largest first, then the exact-path ones)
+    a.qperm[(uint64_t)cls * a.nq + s_cbase[cls] + s_wcls[w]] = qi;
   }
-  // the last CTA turns (class, rank) into the permutation
-  __shared__ bool s_last;
-  __threadfence();
-  __syncthreads();
-  if (threadIdx.x == 0) s_last = atomicAdd(&a.st->chain_done, 1u) == gridDim.x - 1;
-  __syncthreads();
-  if (s_last) {
-    __threadfence();
-    uint32_t pre[NQCLS];
-    uint32_t acc = 0;
-#pragma unroll
-    for (int c = 0; c < NQCLS; ++c) {
-      pre[c] = acc;
-      acc += *(volatile uint32_t *)&a.st->q_cls[c];
+  // fast queries: the per-query outputs are known here (k_copy_fast writes the pairs)
+  if (qi < a.nq && !slow) {
+    __syncwarp();
+    const unsigned long long base = a.qbase[qi];
+    const uint32_t nk = a.qnk[qi];
+    const bool ok = base + U <= a.cap;
+    if (lane == 0) {
+      a.range[2 * qi] = base;
+      a.range[2 * qi + 1] = base + (ok ? U : 0);
+      ctr_add(a.st, DUM_CTR_QUERIES, 1);
+      ctr_add(a.st, DUM_CTR_Q_FAST, 1);
+      ctr_add(a.st, DUM_CTR_CHAIN, nk);
     }
-    constexpr uint32_t QB = 4;  // queries per thread with their loads in flight together
-    for (uint32_t q0 = threadIdx.x; q0 < a.nq; q0 += blockDim.x * QB) {
-      uint32_t r[QB];
-#pragma unroll
-      for (uint32_t u = 0; u < QB; ++u) {
-        const uint32_t q = q0 + u * blockDim.x;
-        r[u] = q < a.nq ? __ldcg(a.qrank + q) : NONE;
-      }
-#pragma unroll
-      for (uint32_t u = 0; u < QB; ++u) {
-        if (r[u] == NONE) continue;
-        uint32_t p = r[u] & 0xFFFFFFu;
-#pragma unroll
-        for (int c = 0; c < NQCLS; ++c)
-          if ((r[u] >> 24) == (uint32_t)c) p += pre[c];
-        a.qperm[p] = q0 + u * blockDim.x;
-      }
+    if (a.kern_off) {
+      const uint32_t *lo = a.qloff + (uint64_t)qi * (g.N + 2);
+      uint32_t *ko = a.kern_off + (uint64_t)qi * (g.N + 2);
+      for (uint32_t d = lane; d <= g.N + 1; d += 32) ko[d] = d <= nk ? __ldcg(lo + d) : U;
     }
-    // every reservation is made: the pool size is the call's `needed`
-    if (threadIdx.x == 0 && a.needed) *a.needed = *(volatile unsigned long long *)&a.st->pool_pairs;
+    if (a.chain) {
+      uint32_t *ch = a.chain + (uint64_t)qi * (g.N + 1);
+      for (uint32_t d = lane; d <= g.N; d += 32) ch[d] = d < nk ? skern[w][d] : NONE;
+    }
+  }
+  // the chunk map of k_copy_fast: chunk j of list d of a fast query -> (q, d, j)
+  if (qi < a.nq && s_gu[w]) {
+    unsigned long long gb = s_gbase;
+    for (uint32_t i = 0; i < w; ++i) gb += s_gu[i];
+    const uint32_t G = s_gu[w], nk = a.qnk[qi];
+    uint32_t d = 0;
+    for (uint32_t x = lane; x < G; x += 32) {
+      while (sgoff[w][d + 1] <= x) ++d;
+      if (gb + x < a.chunk_cap)
+        a.chunk_map[gb + x] = ((unsigned long long)qi << 40) | ((unsigned long long)d << 32) | (x - sgoff[w][d]);
+    }
+    if (lane == 0 && gb + G > a.chunk_cap) set_err(a.st, ERR_ECAPACITY, gb + G);
+    (void)nk;
   }
 }
 
@@ -316,7 +368,23 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
   __shared__ uint32_t s_dup[2 * OCCAP];  // pass 1: duplicated blocks; duplicate path: occurrences (list, block)
   __shared__ unsigned long long s_hoff;
   const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  const uint32_t qi = a.qperm[blockIdx.x];
+  // persistent over the exact-path queries (class lists NQCLS .. 2 NQCLS-1 of
+  // k_chain, largest windows first; the fast path answers the others)
+  uint32_t ccnt[NQCLS];
+#pragma unroll
+  for (int c = 0; c < NQCLS; ++c) ccnt[c] = *(volatile uint32_t *)&a.st->q_cls[NQCLS + c];
+  uint32_t nslow = 0;
+#pragma unroll
+  for (int c = 0; c < NQCLS; ++c) nslow += ccnt[c];
+  for (uint32_t bq = blockIdx.x; bq < nslow; bq += gridDim.x) {
+  uint32_t cq = NQCLS, rq = bq;
+#pragma unroll
+  for (int c = 0; c < NQCLS; ++c)
+    if (cq == NQCLS) {
+      if (rq < ccnt[c]) cq = c;
+      else rq -= ccnt[c];
+    }
+  const uint32_t qi = a.qperm[(uint64_t)(NQCLS + cq) * a.nq + rq];
   const Geo &g = a.g;
   const uint32_t anchor = a.q[qi].anchor;
   const bool anchored = anchor != NONE;
@@ -479,7 +547,7 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
       {
         if (tid == 0) select_reserve(a.so, s_nonres, a.st, ss);
         group_sync<1, GRP_NT>();
-        select_tail<GRP_NT, 1>(a.so, qi, ss, bitmap, a.st, tid, dk);
+        select_tail<GRP_NT, 1>(a.so, qi, ss, InBlockBitmap{bitmap}, a.st, tid, dk);
       }
     } else if (ok) {
       copy_lists(wid - GRP_W, NWARP - GRP_W, loff, nullptr);
@@ -587,35 +655,47 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
       __syncthreads();
       run = noff[nk];
       if (ok) {
-        // lists that lose blocks: one warp each, ordered ballot compaction
-        for (uint32_t d = wid; d < nk; d += NWARP) {
+        // lists that lose blocks: ordered compaction by the whole CTA, chunks
+        // of 4 * PRED_NT elements (thread tid owns 4 consecutive ones), one
+        // block scan of the keep counts per chunk
+        for (uint32_t d = 0; d < nk; ++d) {
           if (!kcnt[d]) continue;
           const uint32_t *lst = list_of(d);
           const uint32_t L = loff[d + 1] - loff[d], kd = kern[d];
           uint2 *o = reinterpret_cast<uint2 *>(a.pairs) + base + noff[d];
           uint32_t pos = 0;
-          for (uint32_t c = 0; c < L; c += 32) {
-            const uint32_t i = c + lane;
-            uint32_t b = NONE;
-            bool keep = false;
-            if (i < L) {
-              b = __ldg(lst + i);
-              const uint32_t f = hmap_get(bk, bv, DBCAP, b);
-              keep = f == NONE || f == d + 1;
+          for (uint32_t c = 0; c < L; c += 4 * PRED_NT) {
+            uint32_t bb[4], keep = 0;
+#pragma unroll
+            for (uint32_t u = 0; u < 4; ++u) {
+              const uint32_t i = c + 4 * tid + u;
+              bb[u] = i < L ? __ldg(lst + i) : NONE;
             }
-            const uint32_t mask = __ballot_sync(0xffffffffu, keep);
-            if (keep) __stcs(o + pos + __popc(mask & ((1u << lane) - 1)), make_uint2(b, kd));
-            pos += __popc(mask);
+#pragma unroll
+            for (uint32_t u = 0; u < 4; ++u) {
+              if (c + 4 * tid + u >= L) continue;
+              const uint32_t f = hmap_get(bk, bv, DBCAP, bb[u]);
+              if (f == NONE || f == d + 1) keep |= 1u << u;
+            }
+            uint32_t tot;
+            const uint32_t pre = block_excl_scan(__popc(keep), ws, &tot);
+            uint32_t r = 0;
+#pragma unroll
+            for (uint32_t u = 0; u < 4; ++u)
+              if ((keep >> u) & 1u) __stcs(o + pos + pre + r++, make_uint2(bb[u], kd));
+            pos += tot;
           }
         }
         // the other lists at their shifted offsets
         copy_lists(wid, NWARP, noff, kcnt);
       }
       if (SELECT && tid == 0) s_nonres -= s_dnr;
+      if (tid == 0) ctr_add(a.st, DUM_CTR_Q_DUP, 1);
     } else {
       // ---------------- fallback: min-position hash over every element ----------------
       const uint32_t hcap = pow2ceil(2 * (U + 1));
       if (tid == 0) {
+        ctr_add(a.st, DUM_CTR_Q_FALLBACK, 1);
         s_nonres = 0;
         const unsigned long long o = atomicAdd(&a.st->pool_big, 2ull * hcap);
         s_flag = o + 2ull * hcap <= a.big_entries * 2;
@@ -684,7 +764,7 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
     if (SELECT) {
       if (tid == 0) select_reserve(a.so, s_nonres, a.st, ss);
       __syncthreads();
-      select_tail<PRED_NT, 0>(a.so, qi, ss, bitmap, a.st, tid, dk);
+      select_tail<PRED_NT, 0>(a.so, qi, ss, InBlockBitmap{bitmap}, a.st, tid, dk);
     }
   }
   if (tid == 0) {
@@ -695,6 +775,7 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
     ctr_add(a.st, DUM_CTR_GATHERED, U);
     ctr_add(a.st, DUM_CTR_EMITTED, run);
     ctr_add(a.st, DUM_CTR_RUNS, nk ? eoff[nk] : 0);
+    if (ndup == 0) ctr_add(a.st, DUM_CTR_Q_NODUP, 1);
   }
   if (a.kern_off) {
     // kern_off[d] = pairs emitted before kernel d (kcnt = occurrences dropped per list)
@@ -714,24 +795,28 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
     uint32_t *ch = a.chain + (uint64_t)qi * (g.N + 1);
     for (uint32_t d = tid; d <= g.N; d += PRED_NT) ch[d] = d < nk ? kern[d] : NONE;
   }
+  if (tid == 0) ctr_add(a.st, DUM_CTR_Q_SLOW, 1);
+  __syncthreads();  // the next query reuses the shared state
+  }
 }
 
-// the call's bump pointers and k_chain's class counters
-__global__ void k_pred_reset(DevState *st) {
+// Predict epilogue: the selection pools' size for the caller, then the call's
+// bump pointers and k_chain's class counters are cleared for the next call
+// (they start cleared: k_init_state).
+__global__ void k_pred_epilogue(DevState *st, uint64_t *needed, uint64_t *sel_needed) {
   const uint32_t t = threadIdx.x;
   if (t == 0) {
+    if (needed) *needed = st->pool_pairs;  // every reservation is made: the pool size is the call's `needed`
+    if (sel_needed) *sel_needed = st->pool_wb > st->pool_inv ? st->pool_wb : st->pool_inv;
     st->pool_pairs = 0;
+    st->pool_chunks = 0;
     st->pool_wb = 0;
     st->pool_inv = 0;
     st->pool_anchor = 0;
     st->pool_big = 0;
     st->chain_done = 0;
   }
-  if (t < 8) st->q_cls[t] = 0;
-}
-
-__global__ void k_copy_counters2(const unsigned long long *a, const unsigned long long *b, uint64_t *dst) {
-  *dst = *a > *b ? *a : *b;
+  if (t < 16) st->q_cls[t] = 0;
 }
 
 cudaError_t launch_make_queries(dum_engine *e, const uint32_t *exec_seq, uint32_t n_seq, uint32_t first,
@@ -749,7 +834,6 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
                            const SelectOut *sel, uint64_t *sel_needed, cudaStream_t s) {
   if (nq == 0) return cudaSuccess;
   if (nq > e->anchor_range_cap) return cudaErrorInvalidValue;
-  k_pred_reset<<<1, 32, 0, s>>>(e->d_state);  // one launch instead of three memsets
   WalkScratch ws{e->d_walk_seen, e->d_walk_chain, e->d_walk_tmp, e->walk_hash_cap,
                  e->g.walk_cap + e->g.R * e->g.A + 4};
   {
@@ -794,33 +878,69 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
     a.so.res_bits = e->d_res_bits;
   }
   a.needed = needed;
+  a.select = sel ? 1u : 0u;
+  a.conf = e->d_conf;
+  a.conf_n = e->d_conf_n;
+  a.wnr = e->d_wnr;
+  a.wnres = e->d_wnres;
+  a.respos = e->d_respos;
+  a.qroff = e->d_qroff;
+  a.qneed = e->d_qneed;
+  a.qvb = e->d_qvb;
+  {
+    // the chunk map holds every copy chunk of the call: <= cap / 128 + nq (N + 1)
+    const uint64_t bound = cap / CHUNK_B + (uint64_t)nq * (e->g.N + 1) + 1;
+    if (bound > e->chunk_cap) {
+      cudaError_t ce = cudaStreamSynchronize(s);  // growth only: the old map may be in use
+      if (ce == cudaSuccess) ce = cudaFree(e->d_chunk_map);
+      e->d_chunk_map = nullptr;
+      if (ce == cudaSuccess) ce = cudaMalloc((void **)&e->d_chunk_map, 8 * bound);
+      if (ce != cudaSuccess) return ce;
+      e->chunk_cap = bound;
+    }
+  }
+  a.chunk_map = e->d_chunk_map;
+  a.chunk_cap = e->chunk_cap;
+  cudaError_t err;
+  if (sel && (err = launch_walk_res(e, s)) != cudaSuccess) return err;  // residency facts per walk
   cudaStreamWaitEvent(s, e->ev_join, 0);  // jump tables of the last build (side stream)
+  cudaStreamWaitEvent(s, e->ev_widx, 0);  // walk index of the last build (third side stream)
   {
     TimerScope t(e, DUM_T_CHAIN, s);
     k_chain<<<(nq + CHAIN_WARPS - 1) / CHAIN_WARPS, CHAIN_WARPS * 32, 0, s>>>(a);
   }
+  // exact path (windows that may hold duplicates, anchored queries) on the
+  // engine's second side stream, beside the fast path on `s`
+  cudaEventRecord(e->ev_fork2, s);
+  cudaStreamWaitEvent(e->side2, e->ev_fork2, 0);
   const size_t smem = (size_t)((a.nwords + 3) & ~3u) * 4 + 2 * DHCAP * 4;
+  const uint32_t pgrid = std::min<uint32_t>(nq, 2 * 148);
   if (sel) {
     // the attribute is per device and function: raised by every engine on its own device
     if ((int)smem > e->select_smem) {
       cudaFuncSetAttribute(k_predict<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       e->select_smem = (int)smem;
     }
-    TimerScope t(e, DUM_T_PREDICT, s);
-    k_predict<true><<<nq, PRED_NT, smem, s>>>(a);
+    TimerScope t(e, DUM_T_EXACT, e->side2);
+    k_predict<true><<<pgrid, PRED_NT, smem, e->side2>>>(a);
   } else {
     if ((int)smem > e->predict_smem) {
       cudaFuncSetAttribute(k_predict<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       e->predict_smem = (int)smem;
     }
-    TimerScope t(e, DUM_T_PREDICT, s);
-    k_predict<false><<<nq, PRED_NT, smem, s>>>(a);
+    TimerScope t(e, DUM_T_EXACT, e->side2);
+    k_predict<false><<<pgrid, PRED_NT, smem, e->side2>>>(a);
   }
+  cudaEventRecord(e->ev_join2, e->side2);
+  // fast path: the flat copy on `s`, the selection on the third side stream
+  cudaStreamWaitEvent(e->side3, e->ev_fork2, 0);
+  if ((err = launch_window(e, a, sel != nullptr, s, e->side3)) != cudaSuccess) return err;
+  cudaEventRecord(e->ev_join3, e->side3);
+  cudaStreamWaitEvent(s, e->ev_join2, 0);
+  cudaStreamWaitEvent(s, e->ev_join3, 0);
   e->kernel_launches += 3;
-  if (sel && sel_needed) {
-    k_copy_counters2<<<1, 1, 0, s>>>(&e->d_state->pool_wb, &e->d_state->pool_inv, sel_needed);
-    e->kernel_launches += 1;
-  }
+  k_pred_epilogue<<<1, 32, 0, s>>>(e->d_state, needed, sel ? sel_needed : nullptr);
+  e->kernel_launches += 1;
   return cudaGetLastError();
 }
 

@@ -114,6 +114,7 @@ __global__ void __launch_bounds__(INGEST_NT) k_ingest(
     }
     if (ndup) s_dups = 1;
     __syncthreads();
+    if (threadIdx.x == 0 && s_dups) ctr_add(st, DUM_CTR_INGEST_DUP, 1);
     uint32_t run = n;
     if (!s_dups) {
       for (uint32_t j = threadIdx.x; j < n; j += INGEST_NT) stage_norm[f0 + a + j] = faults[a + j];
@@ -203,6 +204,7 @@ __global__ void __launch_bounds__(INGEST_NT) k_ingest(
       }
       if (dup) s_dups = 1;
       __syncthreads();
+      if (threadIdx.x == 0 && s_dups) ctr_add(st, DUM_CTR_INGEST_DUP, 1);
       uint32_t run = n;
       if (!s_dups) {
         // no duplicate record in this launch: the normalised list is the input

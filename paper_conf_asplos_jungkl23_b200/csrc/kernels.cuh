@@ -26,9 +26,14 @@ cudaError_t launch_reset_residency(dum_engine *e, cudaStream_t s);
 cudaError_t launch_load_residency(dum_engine *e, const uint32_t *lrm, uint32_t n, cudaStream_t s);
 cudaError_t launch_mark_inactive(dum_engine *e, const uint32_t *blocks, uint32_t n, int flag, cudaStream_t s);
 cudaError_t launch_migrate(dum_engine *e, int dir, const uint32_t *blocks, const uint32_t *dst, uint32_t n,
-                           uint32_t method, cudaStream_t s);
+                           uint32_t method, cudaStream_t s, const uint64_t *rng = nullptr);
 cudaError_t launch_checksums(dum_engine *e, int where, const uint32_t *ids, uint32_t n, uint64_t *out,
                              cudaStream_t s);
+
+// k_sim.cu
+cudaError_t launch_simulate(dum_engine *e, const uint64_t *hash, uint32_t n_launch, const uint64_t *acc_off,
+                            const uint32_t *acc_blk, uint32_t n_kernels, uint32_t degree, uint32_t flags,
+                            dum_sim_stats *stats, cudaStream_t s);
 
 // walk geometry helpers shared by k_build.cu and k_predict.cu
 struct WalkScratch {

@@ -66,11 +66,30 @@ __device__ __forceinline__ void group_sync() {
 // costs two barriers (three in the last one).
 constexpr uint32_t SEL_CHUNK = 4096;  // stage capacity (words); a chunk is NT * IT <= SEL_CHUNK entries
 
-template <int NT, int BAR>
-__device__ void select_tail(const SelectOut &so, uint32_t qi, const SelShared &ss, const uint32_t *bitmap,
+// Window membership of a log entry (block b at log position p): the window
+// set as a bitmap over the block-id space (built from the window's blocks).
+struct InBlockBitmap {
+  const uint32_t *bitmap;
+  __device__ __forceinline__ uint32_t operator()(uint32_t b, uint32_t) const { return bitmap[b >> 5] >> (b & 31); }
+};
+// ... or as a bitmap over log positions [head, head + 32 * words) holding the
+// positions of the window's resident blocks (k_window.cu fast path; the scan
+// never passes head + 32 * words there).
+struct InPosBitmap {
+  const uint32_t *bits;
+  uint32_t head, words;
+  __device__ __forceinline__ uint32_t operator()(uint32_t, uint32_t p) const {
+    const uint32_t r = p - head;
+    return (p >= head && (r >> 5) < words) ? bits[r >> 5] >> (r & 31) : 0u;
+  }
+};
+
+template <int NT, int BAR, class InWin, int CTR_SCAN = DUM_CTR_SEL_SCANNED, int CTR_VICT = DUM_CTR_SEL_VICTIMS,
+          int ITP = 0>
+__device__ void select_tail(const SelectOut &so, uint32_t qi, const SelShared &ss, const InWin &inwin,
                             DevState *st, uint32_t tid, uint32_t *stage /* SEL_CHUNK words of shared memory */) {
   constexpr int NW = NT / 32;
-  constexpr uint32_t IT = NT >= 512 ? 8 : NT >= 320 ? 12 : 16;
+  constexpr uint32_t IT = ITP ? ITP : NT >= 512 ? 8 : NT >= 320 ? 12 : 16;  // entries per thread per chunk
   constexpr uint32_t CHUNK = NT * IT;
   static_assert(NW <= 32 && IT % 4 == 0 && CHUNK <= SEL_CHUNK, "one warp scans the warp totals; 16 B loads");
   __shared__ uint32_t s_wt[2][NW], s_tw, s_ti;
@@ -105,7 +124,7 @@ __device__ void select_tail(const SelectOut &so, uint32_t qi, const SelShared &s
 #pragma unroll
     for (uint32_t k = 0; k < IT; ++k) {
       const uint32_t b = v[k] & 0x7FFFFFFFu;
-      uint32_t e = ((valid >> k) & 1u) & ~(bitmap[b >> 5] >> (b & 31));
+      uint32_t e = ((valid >> k) & 1u) & ~inwin(b, i0 + k);
       if (!clean && (e & 1u))
         e = __ldg(&so.frame_of[b]) != NONE && __ldg(&so.stamp_of[b]) == so.lrm_stamp[i0 + k];
       const uint32_t ina = v[k] >> 31;
@@ -186,8 +205,8 @@ __device__ void select_tail(const SelectOut &so, uint32_t qi, const SelShared &s
     o[1] = bwb + (ok ? run_wb : 0);
     o[2] = binv;
     o[3] = binv + (ok ? run_inv : 0);
-    ctr_add(st, DUM_CTR_SEL_SCANNED, scanned);
-    ctr_add(st, DUM_CTR_SEL_VICTIMS, run_wb + run_inv);
+    ctr_add(st, CTR_SCAN, scanned);
+    ctr_add(st, CTR_VICT, run_wb + run_inv);
   }
 }
 

@@ -15,9 +15,14 @@ NONE = 0xFFFFFFFF
 ALL_TABLES = orc.EXEC | orc.CORR | orc.BLK | orc.WALK | orc.HIST
 
 
+# engines created by the current test (conftest reads their path counters at teardown)
+LIVE_ENGINES: list = []
+
+
 def make_pair(R=2048, A=2, S=4, N=32, W=256, C=128, row_index=0, Emax=1024, **kw):
     eng = Engine(num_rows=R, assoc=A, num_succs=S, degree_n=N, max_blocks=W, max_exec_ids=Emax, hbm_frames=C,
                  row_index=row_index, **kw)
+    LIVE_ENGINES.append(eng)
     o = orc.Oracle(R=R, A=A, S=S, N=N, W=W, C=C, row_index=row_index)
     return eng, o
 

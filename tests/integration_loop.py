@@ -41,19 +41,30 @@ class LoopEngine:
     def snapshot(self) -> bytes: ...
 
 
-def run_loop(eng: LoopEngine, tr, N: int, inactive: set = frozenset(), check=None) -> Dict[str, object]:
+def run_loop(eng: LoopEngine, tr, N: int, inactive: set = frozenset(), check=None, preevict: bool = True,
+             invalidate: bool = True, n_launch: int = None, per_launch: list = None) -> Dict[str, object]:
+    """N < 0: no queries (naive UM, demand path only).  preevict=False: the
+    window is prefetched into free frames only.  invalidate=False: inactive
+    victims are written back too.  Faults are the first occurrence of each
+    non-resident access of the launch (D2; the T trace has no repeats).
+    per_launch (a list) receives (faults, demand_wb, demand_inv, pre_wb,
+    pre_inv, prefetched) per launch."""
     ids: Dict[int, int] = {}
     execs: List[int] = []
     faults_per_iter = [0] * tr.n_iter
     h2d = d2h = inv = 0
     K = tr.K
+    total = tr.n_iter * K if n_launch is None else n_launch
     for it in range(tr.n_iter):
         for j in range(K):
             k = it * K + j
+            if k >= total:
+                break
             acc = [int(b) for b in tr.access_blk[int(tr.access_off[j]):int(tr.access_off[j + 1])]]
             res = eng.resident()
             rset = set(res)
-            faults = [b for b in acc if b not in rset]
+            faults = [b for b in dict.fromkeys(acc) if b not in rset]
+            st = [len(faults), 0, 0, 0, 0, 0]
             faults_per_iter[it] += len(faults)
             h = int(tr.launch_hash[k])
             e = eng.record(h, faults)
@@ -67,6 +78,9 @@ def run_loop(eng: LoopEngine, tr, N: int, inactive: set = frozenset(), check=Non
                 victims = [b for b in res if b not in aset][:need]
                 wb = [b for b in victims if b not in inactive]
                 iv = [b for b in victims if b in inactive]
+                if not invalidate:
+                    wb, iv = wb + iv, []  # (the engine writes the inactive list back after the active one)
+                st[1], st[2] = len(wb), len(iv)
                 if wb:
                     eng.migrate(D2H, wb); d2h += len(wb)
                 if iv:
@@ -76,31 +90,40 @@ def run_loop(eng: LoopEngine, tr, N: int, inactive: set = frozenset(), check=Non
             eng.build()
             # transition query for the next launch
             k1 = k + 1
-            if k1 < tr.n_iter * K and N >= 0:
+            if k1 < total and N >= 0:
                 h1 = int(tr.launch_hash[k1])
                 if h1 in ids:
                     hist = ([NONE, NONE, NONE] + execs)[-3:]
                     q = [ids[h1], hist[0], hist[1], hist[2], NONE, N]
                     window = eng.predict1(q)
-                    wb, iv = eng.select1(window, NONE)
-                    if wb:
-                        eng.migrate(D2H, wb); d2h += len(wb)
-                    if iv:
-                        eng.migrate(INVALIDATE, iv); inv += len(iv)
+                    if preevict:
+                        wb, iv = eng.select1(window, NONE)
+                        if not invalidate:
+                            wb, iv = wb + iv, []
+                        st[3], st[4] = len(wb), len(iv)
+                        if wb:
+                            eng.migrate(D2H, wb); d2h += len(wb)
+                        if iv:
+                            eng.migrate(INVALIDATE, iv); inv += len(iv)
                     rset = set(eng.resident())
                     todo = [b for b in window if b not in rset][: eng.free()]
+                    st[5] = len(todo)
                     if todo:
                         eng.migrate(H2D, todo); h2d += len(todo)
+            if per_launch is not None:
+                per_launch.append(tuple(st))
             if check is not None:
                 check(k, eng)
     return {"faults_per_iter": faults_per_iter, "h2d": h2d, "d2h": d2h, "inv": inv}
 
 
 class OracleLoop(LoopEngine):
-    def __init__(self, tr, N: int, R=2048, A=2, S=4):
+    def __init__(self, tr, N: int, R=2048, A=2, S=4, inactive=None):
         import oracle as orc
         self.orc = orc
         self.o = orc.Oracle(R=R, A=A, S=S, N=max(N, 0), W=tr.W, C=tr.C)
+        if inactive is not None and len(inactive):
+            self.o.mark_inactive(np.asarray(sorted(inactive), np.uint32), True)
 
     def record(self, h, faults):
         return int(self.o.record_faults(np.array([h], np.uint64), np.array([0, len(faults)], np.uint64),

@@ -332,3 +332,27 @@ def test_overlapped_ingest_no_host_syncs(trace):
                 "batch %d query %d" % (j + 1, q)
             assert np.array_equal(gko[q], ko_o[q]) and np.array_equal(gch[q], ch_o[q])
     assert_same_state(eng, o)
+
+
+@pytest.mark.parametrize("R", [2048, 16])
+def test_sequential_walker_mode_builds_identical_walks(R):
+    """DUM_CFG_SEQ_WALKS: every walk is built by the sequential one-warp walker
+    (k_walk_slow, the literal PAPER.md L218-L224 loop); the walk cache and the
+    windows must equal the oracle's exactly as with the parallel walker."""
+    rng = np.random.default_rng(900 + R)
+    W = 5000
+    eng, o = make_pair(R=R, A=2, S=4, W=W, C=800, N=4, max_batch_faults=1 << 17, flags=B.DUM_CFG_SEQ_WALKS)
+    pool = [wl.fnv1a64(b"sq%d" % i) for i in range(6)]
+    ex_all = []
+    for batch in range(3):
+        h, off, f = _big_launch_trace(rng, n_launch=8, pool=pool, W=W, lo=20, hi=1500, repeat_prob=0.5)
+        exo, exg = record_both(eng, o, h, off, f)
+        assert np.array_equal(exo, exg)
+        ex_all += [int(x) for x in exo]
+        build_both(eng, o)
+        assert_same_state(eng, o, msg="batch %d" % batch)
+        qs = transition_queries(ex_all, 0, len(ex_all), 4)
+        ro, rg, _ = predict_both(eng, o, qs)
+        assert_same_predictions(ro, rg)
+    c = eng.counters()
+    assert c["WALK_SLOW"] > 0 and c["WALK_DEDUPE"] == 0, c
