@@ -54,7 +54,7 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="G", choices=["G", "B", "T"])
     ap.add_argument("--degree", type=int, default=32)
-    ap.add_argument("--mig-blocks", type=int, default=1024)
+    ap.add_argument("--mig-blocks", type=int, default=4096)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-migration", action="store_true")
@@ -62,6 +62,9 @@ def parse():
     ap.add_argument("--json-out", default="")
     ap.add_argument("--unfused", action="store_true", help="separate predict / select calls")
     ap.add_argument("--debug", action="store_true", help="synchronize and check after every call")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="process group of the N>1 replicas (barrier + reductions only); gloo lets several ranks "
+                         "share one GPU (tests)")
     ap.add_argument("--verify", action="store_true",
                     help="check the last timed step's prefetch / victim lists against the oracle")
     return ap.parse_args()
@@ -178,13 +181,13 @@ def load_traffic():
 # ---------------------------------------------------------------------------
 # oracle timing (cpu_baseline and --impl reference)
 # ---------------------------------------------------------------------------
-def oracle_sample(tr, n_launch: int, degree: int, start_launch: int = None):
+def oracle_sample(tr, n_launch: int, degree: int, start_launch: int = None, threads: int = 1):
     """Time the oracle on a bounded sample: n_launch consecutive launches of
     iteration 1 (iteration 0 is built untimed first), each with its full
     per-launch work: record + transition query (predict) + select + build.
     Returns (records, seconds)."""
     import oracle as orc
-    o = orc.Oracle(R=2048, A=2, S=4, N=degree, W=tr.W, C=tr.C)
+    o = orc.Oracle(R=2048, A=2, S=4, N=degree, W=tr.W, C=tr.C, threads=threads)
     h, off, f = tr.iteration(0)
     ex = list(o.record_faults(h, off, f))
     o.build_tables()
@@ -207,10 +210,6 @@ def oracle_sample(tr, n_launch: int, degree: int, start_launch: int = None):
     o.build_tables()
     dt = time.perf_counter() - t0
     return int(off[-1]), dt
-
-
-def cpu_cores_used():
-    return 1  # the oracle is single-threaded
 
 
 def run_reference(args, rank):
@@ -236,7 +235,7 @@ def run_reference(args, rank):
         "vs_baseline": None, "dtype": "u32", "data": "synthetic",
         "config": {"workload": args.workload, "sample": "%d consecutive launches per step" % L,
                    "degree_n": args.degree, "geometry": "Config9 (2048 rows, 2-way, 4 succ)"},
-        "cpu_baseline": {"value": value, "unit": "records/s", "cores": cpu_cores_used(), "kind": "oracle",
+        "cpu_baseline": {"value": value, "unit": "records/s", "cores": 1, "kind": "oracle",
                          "sample": "per step: record+predict+select+build of %d consecutive launches of "
                                    "iteration 1 of %s (iteration 0 built untimed)" % (L, args.workload)},
         "e2e": {"value": value, "unit": "records/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -469,14 +468,26 @@ def run_ours(args, rank, world, local_rank):
     counters = {k: round(v / max(args.steps, 1), 1) for k, v in craw.items() if v}
 
     # ---- e2e: same steps through the C-ABI with pinned HOST inputs ----
+    from paper_conf_asplos_jungkl23_b200.replicas import aggregate_many, barrier
     e2e = None
     if not args.no_e2e:
-        e2e = run_e2e(args, tr, eng, step, pre_step, exec_all, rng, srng, dev, stream)
+        barrier()  # every replica's e2e leg starts together
+        e2e = run_e2e(args, tr, eng, dev, stream, cap[0], cap[0])
+        if world > 1:  # whole-job: records summed, time max over ranks
+            ms_max, = aggregate_many([e2e["ms_per_step"]], device=dev, op="max")
+            recs_all, = aggregate_many([e2e["value"] * e2e["ms_per_step"] / 1000.0], device=dev)
+            e2e["value"] = recs_all / (ms_max / 1000.0)
+            e2e["ms_per_step"] = ms_max
 
     # ---- migration (a9) vs host-link peak ----
     mig = None
     if not args.no_migration:
+        barrier()  # all replicas on their host links at once (the link may be shared)
         mig = run_migration(args, dev, local_rank)
+        if world > 1:
+            for d in ("h2d", "d2h"):
+                tot, = aggregate_many([mig[d + "_gbs"]], device=dev)
+                mig["aggregate_" + d + "_gbs"] = tot
 
     res = {
         "metric": "fault records/s (table build+predict)",
@@ -549,41 +560,39 @@ def verify_step(tr, N, out):
             "how": "last timed step's outputs vs the oracle (record+build of iterations 0..i-1, snapshot i)"}
 
 
-def run_e2e(args, tr, eng, step, pre_step, exec_all, rng, srng, dev, stream):
+def run_e2e(args, tr, eng, dev, stream, cap, sel_cap):
     """The same steps through the public C-ABI with every per-step input in
-    pinned HOST memory: the launch records (DUM_HOST_PTRS copies inside
-    dum_record_faults) and the iteration-start residency snapshot (copied to
-    the device inside the timed region, then dum_load_residency); each step's
-    per-query predict / select ranges are copied back to pinned host memory.
-    Steps are issued back to back (the host does not wait for step i before
-    issuing step i+1; every D2H result lands in its own pinned buffer) and one
-    CUDA-event region spans all K steps.  No L2 flush: the step itself moves
-    several hundred MB (tables, walk lists, prefetch lists) through L2."""
+    pinned HOST memory, one call per step: dum_step(DUM_HOST_PTRS) uploads the
+    launch records on the engine's ingest stream and runs record -> queries ->
+    predict+select -> build; the iteration-start residency snapshot is copied
+    up (copy stream) and loaded with dum_load_residency; each step's per-query
+    prefetch / victim ranges are copied back to pinned host memory.  Steps are
+    issued back to back (every D2H result has its own buffer) under one
+    CUDA-event region that ends after the last read-back.  The prefetch and
+    victim lists themselves stay in HBM: their consumer is dum_migrate_blocks
+    (the closed loop, dum_simulate)."""
     import torch
     K = tr.K
     n_iter = 1 + args.warmup + args.steps
-    hh, ho, hf, hs, keep = [], [], [], [], []
+    hh, ho, hf, hs = [], [], [], []
     for i in range(n_iter):
         h, off, f = tr.iteration(i)
         th = torch.from_numpy(h.view(np.int64)).pin_memory()
         to = torch.from_numpy(off.view(np.int64)).pin_memory()
         tf = torch.from_numpy(f.view(np.int32)).pin_memory()
         ts = torch.from_numpy(np.ascontiguousarray(tr.snap_blk[i][: int(tr.snap_cnt[i])]).view(np.int32)).pin_memory()
-        keep.append((th, to, tf))
-        hh.append(th.numpy().view(np.uint64))
-        ho.append(to.numpy().view(np.uint64))
-        hf.append(tf.numpy().view(np.uint32))
+        hh.append((th, th.numpy().view(np.uint64)))
+        ho.append((to, to.numpy().view(np.uint64)))
+        hf.append((tf, tf.numpy().view(np.uint32)))
         hs.append(ts)
     snap_dev = [torch.empty(tr.C, dtype=torch.int32, device=dev) for _ in range(2)]
     out_r = [torch.empty((K, 2), dtype=torch.int64).pin_memory() for _ in range(args.steps)]
     out_s = [torch.empty((K, 4), dtype=torch.int64).pin_memory() for _ in range(args.steps)]
-    # host<->device copies of the bench's own I/O on a copy stream, so that they
-    # overlap the engine's kernels (the engine uploads the records itself)
-    cs = torch.cuda.Stream(device=dev)
-    snap_used = [None, None]  # event: load_residency consumed snap_dev[k]
-    d2h_done = [None]         # event: the last result read-back finished
+    cs = torch.cuda.Stream(device=dev)  # host<->device copies of the bench's own I/O
+    snap_used = [None, None]
+    d2h_done = [None]
+    outs = {}
     eng.reset()
-    exec_all.fill_(-1)
     eng.mark_inactive(torch.from_numpy(tr.inactive_blocks.view(np.int32)).to(dev), True)
 
     def host_step(i, s=None):
@@ -599,22 +608,18 @@ def run_e2e(args, tr, eng, step, pre_step, exec_all, rng, srng, dev, stream):
         eng.load_residency(snap_dev[k][:n])
         snap_used[k] = torch.cuda.Event()
         snap_used[k].record(stream)
-
-        def read_back():
-            if s is None:
-                return
+        if d2h_done[0] is not None:
+            stream.wait_event(d2h_done[0])  # the previous read-back is done before predict overwrites the ranges
+        eng.step(hh[i][1], ho[i][1], hf[i][1], cap, sel_cap, outs)
+        if s is not None:
             ev = torch.cuda.Event()
             ev.record(stream)
             with torch.cuda.stream(cs):
                 cs.wait_event(ev)
-                out_r[s].copy_(rng, non_blocking=True)
-                out_s[s].copy_(srng, non_blocking=True)
+                out_r[s].copy_(outs["rng"], non_blocking=True)
+                out_s[s].copy_(outs["sel_rng"], non_blocking=True)
                 d2h_done[0] = torch.cuda.Event()
                 d2h_done[0].record(cs)
-
-        if d2h_done[0] is not None:
-            stream.wait_event(d2h_done[0])  # the previous read-back is done before predict overwrites the ranges
-        step(i, host=(hh, ho, hf), after_predict=read_back)
 
     for i in range(0, 1 + args.warmup):
         host_step(i)
@@ -639,27 +644,35 @@ def run_e2e(args, tr, eng, step, pre_step, exec_all, rng, srng, dev, stream):
     wall = time.perf_counter() - t0
     tot = a.elapsed_time(b)
     eng.sync()
-    h2d = int(np.mean([hh[i].nbytes + ho[i].nbytes + hf[i].nbytes + hs[i].numel() * 4 for i in range(1, n_iter)]))
+    h2d = int(np.mean([hh[i][1].nbytes + ho[i][1].nbytes + hf[i][1].nbytes + hs[i].numel() * 4
+                       for i in range(1, n_iter)]))
     d2h = out_r[0].numel() * 8 + out_s[0].numel() * 8
     return {"value": records / (tot / 1000.0), "unit": "records/s", "h2d_bytes_per_step": h2d,
             "d2h_bytes_per_step": d2h, "ms_per_step": tot / args.steps,
             "host_wall_ms_per_step": 1000 * wall / args.steps,
             "host_issue_us_per_step": [round(1e6 * x, 1) for x in issue],
-            "note": "public C-ABI with pinned HOST inputs per step (launch records via DUM_HOST_PTRS on the "
-                    "engine's ingest stream; the residency snapshot uploaded on a copy stream) and per-query "
-                    "predict/select ranges read back per step on the copy stream; steps issued back to back, one "
-                    "CUDA-event region over the K steps (it ends after the last read-back); prefetch/victim lists "
-                    "stay in HBM for dum_migrate_blocks"}
+            "note": "public C-ABI, one dum_step call per step with pinned HOST launch records (DUM_HOST_PTRS, "
+                    "uploaded on the engine's ingest stream) + the iteration-start residency snapshot uploaded "
+                    "(copy stream) and loaded + the per-query prefetch/victim ranges read back per step; steps "
+                    "issued back to back, one CUDA-event region over the K steps (it ends after the last "
+                    "read-back); the lists stay in HBM for their consumer dum_migrate_blocks (closed loop: "
+                    "dum_simulate)"}
 
 
 def run_migration(args, dev, local_rank):
+    """Config M in brief (the full sweep: tools/migration_sweep.py): 2 MiB
+    blocks through dum_migrate_blocks H2D and D2H with the SM copy kernel
+    (method 1), TMA bulk copies (3) and the copy engines (2, one cudaMemcpyAsync
+    per contiguous run), at n = 1, 4, 16, 64, 256, 1024 and --mig-blocks
+    (default 4096 = 8 GiB) contiguous blocks; median of 3 after 1 warm-up,
+    against the host-link peak measured here (cudaMemcpyAsync 1 GiB pinned,
+    best of 10, per direction)."""
     import torch
     from paper_conf_asplos_jungkl23_b200 import Engine, binding as B
-    n = args.mig_blocks
-    nbytes = n * BLOCK
+    nmax = args.mig_blocks
+    nbytes = nmax * BLOCK
     host = torch.empty(nbytes, dtype=torch.uint8).pin_memory()
     pool = torch.empty(nbytes, dtype=torch.uint8, device=dev)
-    # host-link peak: cudaMemcpyAsync of 1 GiB pinned, best of 10 per direction
     gib = min(1 << 30, nbytes)
     stream = torch.cuda.current_stream(dev)
 
@@ -680,43 +693,53 @@ def run_migration(args, dev, local_rank):
     peak = {"h2d_gbs": gib / t_h2d / 1e9, "d2h_gbs": gib / t_d2h / 1e9,
             "how": "cudaMemcpyAsync 1 GiB pinned, best of 10"}
     host[: 4 * BLOCK].view(torch.int64).copy_(torch.arange(4 * BLOCK // 8, dtype=torch.int64))
-    eng = Engine(max_blocks=n, hbm_frames=n, max_exec_ids=16, device=local_rank, host_arena=host, frame_pool=pool)
-    blocks = torch.arange(n, dtype=torch.int32, device=dev)
-    out = {"blocks": n, "bytes": nbytes, "host_link_peak": peak}
-    for method, mname in ((1, "sm_copy_kernel"), (2, "copy_engine")):
+    eng = Engine(max_blocks=nmax, hbm_frames=nmax, max_exec_ids=16, device=local_rank, host_arena=host,
+                 frame_pool=pool)
+    empty = torch.empty(0, dtype=torch.int32, device=dev)
+    out = {"blocks": nmax, "bytes": nbytes, "host_link_peak": peak, "curve": {}}
+    sizes = sorted(set([1, 4, 16, 64, 256, 1024, nmax]))
+    for method, mname in ((1, "sm_copy_kernel"), (3, "tma_bulk"), (2, "copy_engine")):
         r = {}
         for d, dname in ((B.H2D, "h2d"), (B.D2H, "d2h")):
-            ts = []
-            for rep in range(4):
-                if d == B.H2D:
-                    eng.load_residency(torch.empty(0, dtype=torch.int32, device=dev))
-                else:
-                    eng.load_residency(blocks)
-                torch.cuda.synchronize()
-                a = torch.cuda.Event(enable_timing=True)
-                b = torch.cuda.Event(enable_timing=True)
-                a.record(stream)
-                eng.migrate_blocks(d, blocks, method=method)
-                b.record(stream)
-                b.synchronize()
-                ts.append(a.elapsed_time(b) / 1000)
-            eng.sync()
-            t = min(ts[1:])
-            r[dname + "_gbs"] = nbytes / t / 1e9
-            r[dname + "_frac"] = r[dname + "_gbs"] / peak[dname + "_gbs"]
+            curve = []
+            for n in sizes:
+                blocks = torch.arange(n, dtype=torch.int32, device=dev)
+                ts = []
+                for rep in range(4):
+                    eng.load_residency(empty if d == B.H2D else blocks)
+                    torch.cuda.synchronize()
+                    a = torch.cuda.Event(enable_timing=True)
+                    b = torch.cuda.Event(enable_timing=True)
+                    a.record(stream)
+                    eng.migrate_blocks(d, blocks, method=method)
+                    b.record(stream)
+                    b.synchronize()
+                    ts.append(a.elapsed_time(b) / 1000)
+                eng.sync()
+                gbs = n * BLOCK / statistics.median(ts[1:]) / 1e9
+                curve.append((n, round(gbs, 2), round(gbs / peak[dname + "_gbs"], 4)))
+            r[dname + "_gbs"] = curve[-1][1]
+            r[dname + "_frac"] = curve[-1][2]
+            reach = [c[0] for c in curve if c[2] >= 0.8]
+            r[dname + "_smallest_n_at_0.8"] = reach[0] if reach else None
+            out["curve"][mname + "_" + dname] = curve
         out[mname] = r
-    # correctness spot check: H2D then compare bytes of a few frames
-    eng.load_residency(torch.empty(0, dtype=torch.int32, device=dev))
-    eng.migrate_blocks(B.H2D, blocks, method=1)
-    eng.sync()
-    ok = bool(torch.equal(pool[: 4 * BLOCK].cpu(), host[: 4 * BLOCK]))
+    # correctness spot check (untimed): H2D with each method, frames equal the host blocks
+    ok = True
+    for method in (1, 3, 2):
+        eng.load_residency(empty)
+        pool[: 4 * BLOCK].zero_()
+        eng.migrate_blocks(B.H2D, torch.arange(4, dtype=torch.int32, device=dev), method=method)
+        eng.sync()
+        ok &= bool(torch.equal(pool[: 4 * BLOCK].cpu(), host[: 4 * BLOCK]))
     out["bytes_verified"] = ok
-    best_m = max(("sm_copy_kernel", "copy_engine"), key=lambda m: out[m]["h2d_gbs"] + out[m]["d2h_gbs"])
-    out["best_method"] = best_m
-    out["h2d_gbs"] = out[best_m]["h2d_gbs"]
-    out["d2h_gbs"] = out[best_m]["d2h_gbs"]
-    out["h2d_frac"] = out[best_m]["h2d_frac"]
-    out["d2h_frac"] = out[best_m]["d2h_frac"]
+    kernels = ("sm_copy_kernel", "tma_bulk")  # the repo's own copy kernels
+    best_k = max(kernels, key=lambda m: out[m]["h2d_gbs"] + out[m]["d2h_gbs"])
+    out["best_kernel_method"] = best_k
+    for k in ("h2d_gbs", "d2h_gbs", "h2d_frac", "d2h_frac", "h2d_smallest_n_at_0.8", "d2h_smallest_n_at_0.8"):
+        out[k] = out[best_k][k]
+    out["note"] = ("headline h2d/d2h = the best of the repo's copy kernels (SM 16 B vector, TMA bulk); "
+                   "copy_engine = cudaMemcpyAsync runs for comparison (a library copy)")
     eng.close()
     return out
 
@@ -732,17 +755,31 @@ def main():
             print(json.dumps(line))
         return
     import torch
+    from paper_conf_asplos_jungkl23_b200.replicas import bind_to_gpu_node
+    gpu = local_rank % max(torch.cuda.device_count(), 1)  # gloo test: several ranks may share one GPU
+    numa = bind_to_gpu_node(gpu)  # before the pinned host allocations (first touch)
     if world > 1:
-        torch.cuda.set_device(local_rank)
-        torch.distributed.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
-    res, tr = run_ours(args, rank, world, local_rank)
+        torch.cuda.set_device(gpu)
+        if args.dist_backend == "nccl":
+            torch.distributed.init_process_group("nccl", device_id=torch.device("cuda", gpu))
+        else:
+            torch.distributed.init_process_group("gloo")
+    res, tr = run_ours(args, rank, world, gpu)
+    res["config"]["numa"] = numa
+    res["config"]["dist_backend"] = args.dist_backend if world > 1 else None
     if rank == 0 and not args.no_cpu_baseline:
         L = args.cpu_launches or 600
         recs, dt = oracle_sample(tr, L, args.degree)
-        res["cpu_baseline"] = {"value": recs / dt, "unit": "records/s", "cores": cpu_cores_used(), "kind": "oracle",
+        res["cpu_baseline"] = {"value": recs / dt, "unit": "records/s", "cores": 1, "kind": "oracle",
                                "sample": "record+predict+select+build of %d consecutive launches (%d records) of "
-                                         "iteration 1 of %s, after an untimed cold build of iteration 0; %.1f s"
-                                         % (L, recs, args.workload, dt)}
+                                         "iteration 1 of %s, after an untimed cold build of iteration 0; %.1f s; "
+                                         "single-threaded (the canonical baseline)" % (L, recs, args.workload, dt)}
+        nt = os.cpu_count() or 1
+        recs, dt = oracle_sample(tr, L, args.degree, threads=nt)
+        res["cpu_baseline_mt"] = {"value": recs / dt, "unit": "records/s", "cores": nt, "kind": "oracle",
+                                  "sample": "the same sample with the oracle's predict / select split over %d "
+                                            "threads (record and build are sequential by definition); %.1f s"
+                                            % (nt, dt)}
     if world > 1:
         torch.distributed.barrier()
         torch.distributed.destroy_process_group()

@@ -219,6 +219,21 @@ int dum_predict_select(dum_engine *eng, const dum_query *queries, uint32_t n_que
                        uint64_t *out_needed, uint32_t *out_writeback, uint32_t *out_invalidate, uint64_t sel_cap,
                        uint64_t *sel_range, uint64_t *sel_needed, dum_stream_t stream);
 
+/* ---- one step ------------------------------------------------------------
+ * The whole hot path of one batch in one call (SURVEY 8d schedule):
+ * dum_record_faults(batch, flags: DUM_HOST_PTRS / DUM_INPUTS_READY) -> one
+ * transition query per launch of the batch ({its exec ID, the three exec IDs
+ * before it -- across steps --, DUM_NONE, degree}) -> dum_predict_select on the
+ * state built by the previous steps -> dum_build_tables(batch).  Outputs and
+ * their layouts are dum_predict_select's, one query per launch in launch
+ * order.  The engine keeps the last three exec IDs of the previous step
+ * (DUM_NONE after dum_reset).  Requires no batch staged by dum_record_faults. */
+int dum_step(dum_engine *eng, const uint64_t *launch_hash, const uint64_t *launch_off, uint32_t n_launch,
+             const uint32_t *fault_block, uint64_t n_fault, uint32_t flags, uint32_t degree, uint32_t *out_pairs,
+             uint64_t out_cap_pairs, uint64_t *out_range, uint32_t *out_kern_off, uint32_t *out_chain,
+             uint64_t *out_needed, uint32_t *out_writeback, uint32_t *out_invalidate, uint64_t sel_cap,
+             uint64_t *sel_range, uint64_t *sel_needed, dum_stream_t stream);
+
 /* Mark UM blocks as belonging to inactive (inactive != 0) or active PyTorch
  * blocks (D20: a block is invalidatable iff every PT block overlapping
  * it is inactive -- the caller resolves overlap). */
@@ -239,7 +254,12 @@ int dum_load_residency(dum_engine *eng, const uint32_t *lrm_blocks, uint32_t n_r
  *                 the highest frames move into the lowest free frames until
  *                 the free frames form a contiguous tail; otherwise block
  *                 blocks_or_src[i] moves to the free frame dst_frames[i].
- * method: 0 = auto, 1 = SM copy kernel, 2 = copy engines (cudaMemcpyAsync runs).
+ * method: 0 = auto (SM copy kernel), 1 = SM copy kernel (16 B vector loads /
+ *         stores, host memory through its mapped address), 2 = copy engines
+ *         (one cudaMemcpyAsync per run contiguous on both sides; synchronizes:
+ *         the frame plan is read back first), 3 = TMA bulk copies
+ *         (cp.async.bulk global -> shared -> global, 32 KiB tiles, one CTA per
+ *         SM).
  * Invalid lists (duplicates, wrong residency, not enough free frames) set a
  * sticky DUM_EINVAL / DUM_ECAPACITY and move nothing. */
 typedef enum { DUM_H2D = 0, DUM_D2H = 1, DUM_INVALIDATE = 2, DUM_D2D = 3 } dum_dir;
@@ -262,7 +282,7 @@ int dum_migrate_blocks(dum_engine *eng, dum_dir dir, const uint32_t *blocks_or_s
  * sizes stay on the device.  Without a data plane the migrations move the
  * residency only (metadata-only engine: B/G scale); with one the bytes move.
  * Per-launch statistics go to stats[k] (device).  launch_hash, acc_blk, stats:
- * device; acc_off: HOST (n_kernels + 1 entries, <= 4096 accesses per launch).
+ * device; acc_off: HOST (n_kernels + 1 entries, <= 8192 accesses per launch).
  * Requires an empty staging area (call after dum_build_tables). */
 typedef struct {
   uint32_t faults;      /* demand faults of the launch (blocks migrated on demand) */
@@ -351,10 +371,15 @@ enum {
   DUM_CTR_ANCHOR_WALKS,     /* fault-anchored walks (WALK(e, anchor))                     */
   DUM_CTR_INGEST_DUP,       /* launches whose records held duplicates                     */
   DUM_CTR_Q_SLOW,           /* predict queries sent to the exact (bitmap) kernel          */
-  DUM_CTR_FAST_EMITTED,     /* pairs emitted by k_window (= walk entries it gathered)      */
-  DUM_CTR_FAST_SCANNED,     /* LRM-log entries scanned by k_window's selection             */
-  DUM_CTR_FAST_VICTIMS,     /* victims selected by k_window                                */
-  DUM_NCOUNTERS = 32
+  DUM_CTR_FAST_EMITTED,     /* pairs emitted by the fast path (= walk entries it gathered)      */
+  DUM_CTR_FAST_SCANNED,     /* LRM-log entries scanned by the fast path's selection             */
+  DUM_CTR_FAST_VICTIMS,     /* victims selected by the fast path                                */
+  DUM_CTR_SLOW_CONFLICT,    /* exact path: two walks of the chain share a block            */
+  DUM_CTR_SLOW_UNRECORDED,  /* exact path: a walk's conflicts were too many to record      */
+  DUM_CTR_SLOW_SPAN,        /* exact path: the selection could pass the position bitmap   */
+  DUM_CTR_SLOW_ANCHOR,      /* exact path: fault-anchored query                            */
+  DUM_CTR_FAST_DIRTY,       /* fast selections over a log with stale entries               */
+  DUM_NCOUNTERS = 40
 };
 /* Counters accumulate only while counting is on (the default); the bench turns
  * it off for its timed region (no instrumentation atomics there). */
@@ -380,7 +405,7 @@ enum {
   DUM_T_CHAIN,
   DUM_T_JUMP,         /* jump tables over the correlation table (side stream, in dum_build_tables) */
   DUM_T_WALK,         /* parallel walk-cache rebuild (in dum_build_tables) */
-  DUM_T_EXACT,        /* exact-path predict kernel k_predict (side stream, beside k_window) */
+  DUM_T_EXACT,        /* exact-path predict kernel k_predict (side stream, beside the fast path) */
   DUM_T_WALK_INDEX,   /* walk index: holders per block, conflicts per walk (build end) */
   DUM_T_WALK_RES,     /* residency facts per walk (predict) */
   DUM_NTIMERS = 24

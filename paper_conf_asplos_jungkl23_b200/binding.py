@@ -21,13 +21,14 @@ SIM_PREFETCH, SIM_PREEVICT, SIM_INVALIDATE = 0x1, 0x2, 0x4
 SIM_FIELDS = ("faults", "demand_wb", "demand_inv", "pre_wb", "pre_inv", "prefetched")
 DUMP_EXEC, DUMP_CORR, DUMP_BLK, DUMP_WALK, DUMP_RES, DUMP_HIST = 1, 2, 4, 8, 16, 32
 H2D, D2H, INVALIDATE, D2D = 0, 1, 2, 3
-NCOUNTERS, NTIMERS = 32, 24
+NCOUNTERS, NTIMERS = 40, 24
 CTR = {n: i for i, n in enumerate(["RAW_RECORDS", "NORM_RECORDS", "LAUNCHES", "CORR_UPSERTS", "EXEC_BUILT", "OPS",
                                    "SETS", "WALK_ROWS", "WALK_OUT", "QUERIES", "CHAIN", "GATHERED", "EMITTED",
                                    "SEL_WINDOW", "SEL_SCANNED", "SEL_VICTIMS", "MIG_BLOCKS", "RUNS",
                                    "Q_NODUP", "Q_DUP", "Q_FALLBACK", "WALK_PREFIX", "WALK_DEDUPE", "WALK_SLOW",
                                    "Q_FAST", "ANCHOR_WALKS", "INGEST_DUP", "Q_SLOW", "FAST_EMITTED", "FAST_SCANNED",
-                                   "FAST_VICTIMS"])}
+                                   "FAST_VICTIMS", "SLOW_CONFLICT", "SLOW_UNRECORDED", "SLOW_SPAN",
+                                   "SLOW_ANCHOR", "FAST_DIRTY"])}
 TIMER = {n: i for i, n in enumerate(["INGEST", "EXEC_ASSIGN", "BUILD_PREP", "APPLY_WALK", "WALK_SLOW",
                                      "MAKE_QUERIES", "ANCHOR_WALK", "PREDICT", "SELECT", "MIG_PLAN", "COPY",
                                      "RESIDENCY", "CHAIN", "JUMP", "WALK", "EXACT", "WALK_INDEX", "WALK_RES"])}
@@ -113,6 +114,7 @@ def load_library() -> ctypes.CDLL:
         "dum_host_ptr_kind": (I, [P]),
         "dum_read_timing": (I, [P, P, P, I]),
         "dum_simulate": (I, [P, P, U32, P, P, U32, U32, U32, P, P]),
+        "dum_step": (I, [P, P, P, U32, P, U64, U32, U32, P, U64, P, P, P, P, P, P, U64, P, P, P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -318,6 +320,38 @@ class Engine:
         self._ck(self.lib.dum_simulate(self._h, _dev(launch_hash, 8), n, off.ctypes.data, _dev(acc_blk, 4),
                                        len(off) - 1, degree, flags, _dev(stats, 4), self._stream()), "dum_simulate")
         return stats
+
+    def step(self, hashes, offs, faults, cap: int, sel_cap: int, out: dict, degree: Optional[int] = None,
+             ready: bool = False):
+        """dum_step: record -> one transition query per launch -> predict+select
+        -> build, in one C call.  numpy inputs -> DUM_HOST_PTRS (pinned arrays
+        upload asynchronously); device tensors otherwise.  `out` holds the
+        output tensors (pairs, rng, kern_off, chain, needed, wb, inv, sel_rng,
+        sel_needed), allocated on first use for the batch size."""
+        n = len(hashes) if isinstance(hashes, np.ndarray) else hashes.numel()
+        d = self.device
+        if out.get("n") != n or out.get("cap") != cap or out.get("sel_cap") != sel_cap:
+            out.update(n=n, cap=cap, sel_cap=sel_cap,
+                       pairs=torch.empty((max(cap, 1), 2), dtype=torch.int32, device=d),
+                       rng=torch.empty((n, 2), dtype=torch.int64, device=d),
+                       kern_off=torch.empty((n, self.N + 2), dtype=torch.int32, device=d),
+                       chain=torch.empty((n, self.N + 1), dtype=torch.int32, device=d),
+                       needed=torch.zeros(1, dtype=torch.int64, device=d),
+                       wb=torch.empty(max(sel_cap, 1), dtype=torch.int32, device=d),
+                       inv=torch.empty(max(sel_cap, 1), dtype=torch.int32, device=d),
+                       sel_rng=torch.empty((n, 4), dtype=torch.int64, device=d),
+                       sel_needed=torch.zeros(1, dtype=torch.int64, device=d))
+        if isinstance(hashes, np.ndarray):
+            h, o, f = hashes, offs, faults
+            args = (h.ctypes.data, o.ctypes.data, n, f.ctypes.data if len(f) else None, len(f), DUM_HOST_PTRS)
+        else:
+            args = (_dev(hashes, 8), _dev(offs, 8), n, _dev(faults, 4), faults.numel(),
+                    DUM_INPUTS_READY if ready else 0)
+        self._ck(self.lib.dum_step(self._h, *args, self.N if degree is None else degree, _dev(out["pairs"], 4), cap,
+                                   _dev(out["rng"], 8), _dev(out["kern_off"], 4), _dev(out["chain"], 4),
+                                   _dev(out["needed"], 8), _dev(out["wb"], 4), _dev(out["inv"], 4), sel_cap,
+                                   _dev(out["sel_rng"], 8), _dev(out["sel_needed"], 8), self._stream()), "dum_step")
+        return out
 
     def mark_inactive(self, blocks: torch.Tensor, inactive: bool = True):
         self._ck(self.lib.dum_mark_inactive(self._h, _dev(blocks, 4), blocks.numel(), 1 if inactive else 0,

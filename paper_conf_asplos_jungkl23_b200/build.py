@@ -9,6 +9,7 @@ import glob
 import os
 import subprocess
 import sys
+import time
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
@@ -45,6 +46,7 @@ def build(force: bool = False, verbose: bool = False, ptxas_v: bool = False, che
     objs = []
 
     hdr_t = max(os.path.getmtime(p) for p in _deps() if not p.endswith(".cu"))
+    start = time.time()
 
     def one(src):
         obj = os.path.join(bdir, os.path.basename(src) + ".o")
@@ -59,6 +61,9 @@ def build(force: bool = False, verbose: bool = False, ptxas_v: bool = False, che
             raise RuntimeError("nvcc failed for %s:\n%s\n%s" % (src, r.stdout, r.stderr))
         if verbose and (r.stderr or r.stdout):
             sys.stderr.write(r.stdout + r.stderr)
+        # stamp the object with the build's start time: a source or header edited
+        # while it compiled is newer than the object, so the next build redoes it
+        os.utime(obj, (start, start))
         return obj
 
     with cf.ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 2)) as ex:

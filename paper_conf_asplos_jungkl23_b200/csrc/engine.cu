@@ -109,6 +109,7 @@ int reset_state(dum_engine *e, cudaStream_t s) {
   CK(cudaMemsetAsync(e->d_walk_len, 0, 4ull * g.Emax, s));
   CK(cudaMemsetAsync(e->d_wrun_len, 0, 4ull * g.Emax, s));
   CK(cudaMemsetAsync(e->d_conf_n, 0, 4ull * g.Emax, s));  // no walks: no conflicts
+  CK(fill(e->d_step_exec, 3, NONE, s));  // dum_step: no history
   CK(cudaMemsetAsync(e->d_bcnt, 0, 4ull * g.W, s));
   CK(fill(e->d_head, g.Emax, NONE, s));
   CK(cudaMemsetAsync(e->d_e_ops, 0, 4ull * g.Emax, s));
@@ -138,9 +139,9 @@ void free_all(dum_engine *e) {
                   e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits, e->d_inactive_bits, e->d_res_bits, e->d_logpos, e->d_lrm_blk,
                   e->d_lrm_stamp, e->d_mig_frames, e->d_mig_src, e->d_mig_blocks, e->d_state, e->d_qkern,
                   e->d_qloff, e->d_qnk, e->d_qbase, e->d_rec_slot, e->d_jump, e->d_wrun, e->d_wrun_len, e->d_qeoff, e->d_qgoff, e->d_qrank, e->d_qperm,
-                  e->d_bcnt, e->d_bhold, e->d_conf, e->d_conf_n, e->d_wnr, e->d_wnres, e->d_respos, e->d_qroff, e->d_qneed, e->d_qvb, e->d_chunk_map, e->d_dd_list,
+                  e->d_bcnt, e->d_bhold, e->d_conf, e->d_conf_n, e->d_wnr, e->d_wnres, e->d_respos, e->d_qroff, e->d_qneed, e->d_qvb, e->d_chunk_map, e->d_dd_list, e->d_log_bits,
                   e->sim_acc_bits, e->sim_faults, e->sim_pairs, e->sim_wb, e->sim_inv, e->sim_pf, e->sim_foff,
-                  e->sim_ranges, e->sim_q};
+                  e->sim_ranges, e->sim_q, e->d_step_exec, e->d_step_q};
   for (void *p : ptrs)
     if (p) cudaFree(p);
   if (e->ev_fork) cudaEventDestroy(e->ev_fork);
@@ -315,6 +316,8 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_order, 3ull * e->stage_launch_cap));
   A_(dmalloc(&e->d_slow_list, e->stage_launch_cap));
   A_(dmalloc(&e->d_dd_list, e->stage_launch_cap));
+  A_(dmalloc(&e->d_step_exec, 3ull + e->stage_launch_cap));
+  A_(dmalloc(&e->d_step_q, e->stage_launch_cap));
   A_(dmalloc(&e->d_e_ops, g.Emax));
   A_(dmalloc(&e->d_e_last, g.Emax));
   A_(dmalloc(&e->d_lead, 8ull * e->stage_launch_cap));
@@ -346,6 +349,7 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_wnr, g.Emax));
   A_(dmalloc(&e->d_wnres, g.Emax));
   A_(dmalloc(&e->d_respos, (uint64_t)g.Emax * g.walk_cap));
+  A_(dmalloc(&e->d_log_bits, 4 * g.C / 32 + 1024 / 32 + 2));  // lrm_cap / 32 + 1 (lrm_cap = 4 C + 1024)
   A_(dmalloc(&e->d_qroff, (uint64_t)e->anchor_range_cap * (g.N + 2)));
   A_(dmalloc(&e->d_qneed, e->anchor_range_cap));
   A_(dmalloc(&e->d_qvb, 2ull * e->anchor_range_cap));
@@ -505,6 +509,41 @@ int dum_build_tables(dum_engine *e, dum_stream_t stream) {
   return DUM_OK;
 }
 
+__global__ void k_step_shift(uint32_t *ex, uint32_t n) {
+  // the last three exec IDs of [previous three | batch] become the next step's history
+  if (threadIdx.x == 0) {
+    const uint32_t a = ex[n], b = ex[n + 1], c = ex[n + 2];
+    ex[0] = a;
+    ex[1] = b;
+    ex[2] = c;
+  }
+}
+
+int dum_step(dum_engine *e, const uint64_t *launch_hash, const uint64_t *launch_off, uint32_t n_launch,
+             const uint32_t *fault_block, uint64_t n_fault, uint32_t flags, uint32_t degree, uint32_t *out_pairs,
+             uint64_t out_cap_pairs, uint64_t *out_range, uint32_t *out_kern_off, uint32_t *out_chain,
+             uint64_t *out_needed, uint32_t *out_writeback, uint32_t *out_invalidate, uint64_t sel_cap,
+             uint64_t *sel_range, uint64_t *sel_needed, dum_stream_t stream) {
+  if (!e) return DUM_EINVAL;
+  if (n_launch == 0) return DUM_OK;
+  if (e->n_staged) return fail(e, DUM_ESTATE, "dum_step: a batch is already staged (call dum_build_tables)");
+  if (n_launch > e->anchor_range_cap) return fail(e, DUM_EINVAL, "too many launches in one step (max 65536)");
+  int rc = dum_record_faults(e, launch_hash, launch_off, n_launch, fault_block, n_fault, e->d_step_exec + 3, flags,
+                             stream);
+  if (rc) return rc;
+  cudaStream_t s = (cudaStream_t)stream;
+  CK(launch_make_queries(e, e->d_step_exec, 3 + n_launch, 3, degree, e->d_step_q, s));
+  rc = dum_predict_select(e, e->d_step_q, n_launch, out_pairs, out_cap_pairs, out_range, out_kern_off, out_chain,
+                          out_needed, out_writeback, out_invalidate, sel_cap, sel_range, sel_needed, stream);
+  if (rc) return rc;
+  rc = dum_build_tables(e, stream);
+  if (rc) return rc;
+  k_step_shift<<<1, 32, 0, s>>>(e->d_step_exec, n_launch);
+  e->kernel_launches += 1;
+  CK(cudaGetLastError());
+  return DUM_OK;
+}
+
 int dum_make_queries(dum_engine *e, const uint32_t *exec_seq, uint32_t n_seq, uint32_t first, uint32_t degree,
                      dum_query *out, dum_stream_t stream) {
   if (!e || (!exec_seq && n_seq) || (!out && first < n_seq)) return DUM_EINVAL;
@@ -564,8 +603,8 @@ int dum_simulate(dum_engine *e, const uint64_t *launch_hash, uint32_t n_launch, 
     return fail(e, DUM_EINVAL, "null argument / bad flags");
   if (e->n_staged) return fail(e, DUM_ESTATE, "dum_simulate needs an empty staging area (call dum_build_tables)");
   for (uint32_t j = 0; j < n_kernels; ++j)
-    if (acc_off[j + 1] < acc_off[j] || acc_off[j + 1] - acc_off[j] > 4096)
-      return fail(e, DUM_EINVAL, "acc_off not monotone or a launch with more than 4096 accesses");
+    if (acc_off[j + 1] < acc_off[j] || acc_off[j + 1] - acc_off[j] > 8192)
+      return fail(e, DUM_EINVAL, "acc_off not monotone or a launch with more than 8192 accesses");
   if (e->launches + n_launch > 0xFFFFFFFFull) return fail(e, DUM_ECAPACITY, "launch counter exceeds 2^32");
   cudaSetDevice(e->device);
   cudaStream_t s = (cudaStream_t)stream;
@@ -593,7 +632,7 @@ int dum_load_residency(dum_engine *e, const uint32_t *lrm_blocks, uint32_t n_res
 int dum_migrate_blocks(dum_engine *e, dum_dir dir, const uint32_t *blocks_or_src, const uint32_t *dst_frames,
                        uint32_t n, uint32_t method, dum_stream_t stream) {
   if (!e) return DUM_EINVAL;
-  if ((int)dir < 0 || (int)dir > 3 || method > 2) return fail(e, DUM_EINVAL, "bad direction or method");
+  if ((int)dir < 0 || (int)dir > 3 || method > 3) return fail(e, DUM_EINVAL, "bad direction or method");
   if (n > e->g.C) return fail(e, DUM_EINVAL, "list longer than the frame count");
   if (dir != DUM_D2D && n && !blocks_or_src) return fail(e, DUM_EINVAL, "null block list");
   if (dir == DUM_D2D && blocks_or_src && !dst_frames) return fail(e, DUM_EINVAL, "D2D needs dst_frames");

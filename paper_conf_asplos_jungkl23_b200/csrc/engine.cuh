@@ -195,6 +195,7 @@ struct dum_engine {
   uint32_t *d_conf, *d_conf_n;  // [Emax][CONF_MAX], [Emax] (NONE = not recorded)
   uint32_t *d_wnr, *d_wnres;    // [Emax] walk blocks without / with a frame
   uint32_t *d_respos;           // [Emax][walk_cap] log positions of the latter
+  uint32_t *d_log_bits;         // [lrm_cap / 32 + 1] inactive log entries by position from head (k_log_bits)
   uint32_t *d_qroff, *d_qneed;  // [max queries][N+2], [max queries] (k_chain -> k_window)
   unsigned long long *d_qvb;    // [max queries][2] victim-range bases (k_chain -> k_window)
   unsigned long long *d_chunk_map;  // [chunk_cap] (q << 40 | list << 32 | chunk) of the fast queries' windows
@@ -203,6 +204,9 @@ struct dum_engine {
   cudaEvent_t ev_fork2, ev_join2;
   cudaStream_t side3;           // walk index (build end) and the fast-path selection
   cudaEvent_t ev_join3, ev_widx;
+  // dum_step: exec IDs [last 3 of the previous step | this batch] and the batch's queries
+  uint32_t *d_step_exec;
+  dum_query *d_step_q;
   // closed-loop replay scratch (k_sim.cu, allocated by the first dum_simulate)
   bool sim_ready;
   uint32_t sim_acc_cap;
@@ -238,5 +242,7 @@ struct dum_engine {
   uint64_t t_cnt[DUM_NTIMERS];
   int predict_smem, select_smem, build_smem, ingest_smem;
   uint32_t apply_grid, walk_grid;  // persistent build grids (occupancy x SMs), set on first build
-  uint32_t copy_grid, sel_grid;    // persistent predict grids (k_window.cu)  // dynamic smem attributes applied (per engine / device)
+  uint32_t copy_grid, sel_grid;    // persistent predict grids (k_window.cu)
+  int chain_smem;                  // k_chain dynamic smem attribute applied
+  int bulk_smem;                   // k_copy_bulk dynamic smem attribute applied  // dynamic smem attributes applied (per engine / device)
 };

@@ -363,6 +363,88 @@ __global__ void __launch_bounds__(COPY_NT) k_copy_blocks(int dir, const uint32_t
   }
 }
 
+// TMA bulk path (method 3): one elected thread per CTA moves 32 KiB tiles
+// with the bulk-copy engine -- cp.async.bulk global -> shared (completion on an
+// mbarrier), then cp.async.bulk shared -> global -- NBULK tiles in flight per
+// CTA, one CTA per SM; the same (block i, tile) work split as k_copy_blocks.
+constexpr uint32_t BULK_TILE = 32u << 10;
+constexpr uint32_t NBULK = 4;
+constexpr uint32_t BULK_TILES = (uint32_t)(BLK / BULK_TILE);
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+__global__ void __launch_bounds__(32) k_copy_bulk(int dir, const uint32_t *__restrict__ blocks,
+                                                  const uint32_t *__restrict__ src_frames,
+                                                  const uint32_t *__restrict__ frames, char *host, char *pool,
+                                                  const DevState *st) {
+  extern __shared__ __align__(128) unsigned char tiles[];  // NBULK x BULK_TILE
+  __shared__ __align__(8) unsigned long long bar[NBULK];
+  if (!st->mig_ok || dir == DUM_INVALIDATE) return;
+  if (threadIdx.x != 0) return;
+  const uint32_t n = st->mig_n;
+  const uint64_t items = (uint64_t)n * BULK_TILES;
+  if (blockIdx.x == 0) ctr_add(const_cast<DevState *>(st), DUM_CTR_MIG_BLOCKS, n);
+  for (uint32_t s = 0; s < NBULK; ++s)
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&bar[s])));
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  auto addr = [&](uint64_t it, const char *&src, char *&dst) {
+    const uint32_t i = (uint32_t)(it / BULK_TILES), c = (uint32_t)(it % BULK_TILES);
+    if (dir == DUM_H2D) {
+      src = host + (uint64_t)blocks[i] * BLK;
+      dst = pool + (uint64_t)frames[i] * BLK;
+    } else if (dir == DUM_D2H) {
+      src = pool + (uint64_t)frames[i] * BLK;
+      dst = host + (uint64_t)blocks[i] * BLK;
+    } else {
+      src = pool + (uint64_t)src_frames[i] * BLK;
+      dst = pool + (uint64_t)frames[i] * BLK;
+    }
+    src += (uint64_t)c * BULK_TILE;
+    dst += (uint64_t)c * BULK_TILE;
+  };
+  auto load = [&](uint64_t it, uint32_t s) {
+    const char *src;
+    char *dst;
+    addr(it, src, dst);
+    const uint32_t b = smem_u32(&bar[s]), t = smem_u32(tiles + (uint64_t)s * BULK_TILE);
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(b), "r"(BULK_TILE) : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(t), "l"(src), "r"(BULK_TILE), "r"(b) : "memory");
+  };
+  // tiles of this CTA: it = blockIdx.x + j * gridDim.x; ring of NBULK stages
+  uint32_t phase[NBULK] = {0, 0, 0, 0};
+  uint64_t j = 0;
+  for (uint32_t s = 0; s < NBULK; ++s) {
+    const uint64_t it = blockIdx.x + (uint64_t)s * gridDim.x;
+    if (it < items) load(it, s);
+  }
+  for (uint64_t it = blockIdx.x; it < items; it += gridDim.x, ++j) {
+    const uint32_t s = (uint32_t)(j % NBULK);
+    const uint32_t b = smem_u32(&bar[s]), t = smem_u32(tiles + (uint64_t)s * BULK_TILE);
+    // the tile has landed
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tWAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT_%=;\n\t}" ::"r"(b), "r"(phase[s]) : "memory");
+    phase[s] ^= 1u;
+    const char *src;
+    char *dst;
+    addr(it, src, dst);
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(t), "r"(BULK_TILE)
+                 : "memory");
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    // refill this stage once its store has read the tile
+    const uint64_t nxt = it + (uint64_t)NBULK * gridDim.x;
+    if (nxt < items) {
+      asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+      load(nxt, s);
+    }
+  }
+  asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+}
+
 constexpr int SUM_NT = 512;
 __global__ void __launch_bounds__(SUM_NT) k_checksums(const uint32_t *__restrict__ ids, const char *base,
                                                       unsigned long long *out) {
@@ -482,6 +564,21 @@ cudaError_t launch_migrate(dum_engine *e, int dir, const uint32_t *blocks, const
       i = j;
     }
     return cudaSuccess;
+  }
+  if (method == 3) {  // TMA bulk copies: one CTA per SM, NBULK tiles in flight
+    const size_t bsm = (size_t)NBULK * BULK_TILE;
+    if (!e->bulk_smem) {
+      cudaFuncSetAttribute(k_copy_bulk, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bsm);
+      e->bulk_smem = 1;
+    }
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    TimerScope t(e, DUM_T_COPY, s);
+    k_copy_bulk<<<sms, 32, bsm, s>>>(dir, e->d_mig_blocks, e->d_mig_src, e->d_mig_frames, e->host_arena_dev,
+                                     e->frame_pool, e->d_state);
+    e->kernel_launches += 1;
+    return cudaGetLastError();
   }
   const int grid = copy_grid(compaction ? e->g.C : n);
   TimerScope t(e, DUM_T_COPY, s);

@@ -107,6 +107,12 @@ __global__ void k_anchor_walk(Geo g, const dum_query *__restrict__ q, uint32_t n
 constexpr int CHAIN_WARPS = 8;
 
 __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
+  extern __shared__ uint32_t cbits_dyn[];  // [CHAIN_WARPS][cwords] chain bitsets (when Emax fits)
+  const uint32_t cwords = (a.g.Emax + 31) / 32;
+  uint32_t *cbits = a.chain_bitset ? cbits_dyn : nullptr;
+  if (cbits)
+    for (uint32_t x = threadIdx.x; x < CHAIN_WARPS * cwords; x += blockDim.x) cbits[x] = 0;
+  __syncthreads();
   __shared__ uint32_t skern[CHAIN_WARPS][MAXN + 1], sgoff[CHAIN_WARPS][MAXN + 2];
   __shared__ uint32_t s_u[CHAIN_WARPS], s_need[CHAIN_WARPS], s_gu[CHAIN_WARPS];
   __shared__ unsigned long long s_base, s_wbase, s_ibase, s_gbase;
@@ -146,6 +152,11 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
       }
     }
     __syncwarp();
+    // the chain as a bitset over exec IDs (conflict test below), if it fits
+    uint32_t *cset = cbits ? cbits + (uint64_t)w * cwords : nullptr;
+    if (cset)
+      for (uint32_t d = lane; d < nk; d += 32) atomicOr(&cset[kern[d] >> 5], 1u << (kern[d] & 31));
+    __syncwarp();
     // window layout: walk lengths; a kernel met earlier in the chain with the
     // same (unanchored) walk adds nothing (exact; keeps the reservation tight)
     uint32_t *gkern = a.qkern + (uint64_t)qi * (g.N + 1);
@@ -155,7 +166,7 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
     uint32_t RU = 0;  // bitmap-run entries of the window (k_predict pass 1)
     uint32_t GU = 0;  // 128-block copy chunks of the window (k_predict copy)
     uint32_t *roff = a.qroff + (uint64_t)qi * (g.N + 2);  // prefix of the lists' resident blocks
-    bool conflict = false;
+    bool conflict = false, unrec = false;
     uint32_t nonres = 0;  // (per lane) window blocks without a frame
     uint32_t nwres = 0;   // (warp-uniform) window blocks with a frame
     for (uint32_t d0 = 0; d0 < nk; d0 += 32) {
@@ -179,14 +190,21 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
         const uint32_t cn = __ldg(a.conf_n + e);
         if (cn == NONE) {
           conflict = true;
+          unrec = true;
         } else {
           // the conflict row, 4 entries per 16 B load (CONF_MAX words, 16 B aligned)
           const uint4 *cr = reinterpret_cast<const uint4 *>(a.conf + (uint64_t)e * CONF_MAX);
           for (uint32_t k0 = 0; k0 < cn; k0 += 4) {
             const uint4 x = __ldg(cr + k0 / 4);
             const uint32_t c4[4] = {x.x, x.y, x.z, x.w};
-            for (uint32_t k = 0; k < 4 && k0 + k < cn; ++k)
-              for (uint32_t y = 0; y < nk; ++y) conflict |= kern[y] == c4[k];
+            for (uint32_t k = 0; k < 4 && k0 + k < cn; ++k) {
+              const uint32_t c = c4[k];
+              if (cset) {  // the chain's exec-ID bitset (one shared load)
+                conflict |= c < a.g.Emax && ((cset[c >> 5] >> (c & 31)) & 1u);
+              } else {
+                for (uint32_t y = 0; y < nk; ++y) conflict |= kern[y] == c;
+              }
+            }
           }
         }
         if (a.select) {
@@ -233,6 +251,9 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
       a.qnk[qi] = nk;
     }
     slow = anchored || __any_sync(0xffffffffu, conflict);
+    const bool s_unrec = __any_sync(0xffffffffu, unrec);
+    if (lane == 0 && slow) ctr_add(a.st, anchored ? DUM_CTR_SLOW_ANCHOR : s_unrec ? DUM_CTR_SLOW_UNRECORDED
+                                                                           : DUM_CTR_SLOW_CONFLICT, 1);
     nonres = __reduce_add_sync(0xffffffffu, nonres);
     if (a.select && !slow) {
       // need = max(0, window blocks without a frame - free frames) (D18);
@@ -242,10 +263,16 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
       qneed = nonres > nfree ? nonres - nfree : 0;
       const uint32_t span = *(volatile uint32_t *)&a.st->lrm_tail - *(volatile uint32_t *)&a.st->lrm_head;
       const uint32_t stale = span - *(volatile uint32_t *)&a.st->n_resident;
-      if ((uint64_t)qneed + nwres + stale > POS_WORDS * 32ull) slow = true;
+      if ((uint64_t)qneed + nwres + stale > POS_WORDS * 32ull) {
+        slow = true;
+        if (lane == 0) ctr_add(a.st, DUM_CTR_SLOW_SPAN, 1);
+      }
     }
     if (slow) qneed = 0;  // the exact kernel reserves its own victim ranges
     GUq = slow ? 0u : GU;
+    __syncwarp();
+    if (cset)
+      for (uint32_t d = lane; d < nk; d += 32) cset[kern[d] >> 5] = 0;
   }
   // CTA-aggregated output reservation and window-size class counts (one
   // global atomic per CTA and class instead of one per query)
@@ -331,14 +358,13 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
     unsigned long long gb = s_gbase;
     for (uint32_t i = 0; i < w; ++i) gb += s_gu[i];
     const uint32_t G = s_gu[w], nk = a.qnk[qi];
-    uint32_t d = 0;
-    for (uint32_t x = lane; x < G; x += 32) {
-      while (sgoff[w][d + 1] <= x) ++d;
-      if (gb + x < a.chunk_cap)
-        a.chunk_map[gb + x] = ((unsigned long long)qi << 40) | ((unsigned long long)d << 32) | (x - sgoff[w][d]);
+    for (uint32_t d = lane; d < nk; d += 32) {  // lane d: the chunks of list d
+      const uint32_t g0 = sgoff[w][d], g1 = sgoff[w][d + 1];
+      for (uint32_t x = g0; x < g1; ++x)
+        if (gb + x < a.chunk_cap)
+          a.chunk_map[gb + x] = ((unsigned long long)qi << 40) | ((unsigned long long)d << 32) | (x - g0);
     }
     if (lane == 0 && gb + G > a.chunk_cap) set_err(a.st, ERR_ECAPACITY, gb + G);
-    (void)nk;
   }
 }
 
@@ -884,6 +910,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   a.wnr = e->d_wnr;
   a.wnres = e->d_wnres;
   a.respos = e->d_respos;
+  a.inact_bits = sel ? e->d_log_bits : nullptr;
   a.qroff = e->d_qroff;
   a.qneed = e->d_qneed;
   a.qvb = e->d_qvb;
@@ -907,7 +934,15 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   cudaStreamWaitEvent(s, e->ev_widx, 0);  // walk index of the last build (third side stream)
   {
     TimerScope t(e, DUM_T_CHAIN, s);
-    k_chain<<<(nq + CHAIN_WARPS - 1) / CHAIN_WARPS, CHAIN_WARPS * 32, 0, s>>>(a);
+    // chain bitsets in shared memory when max_exec_ids fits (<= 8 KB per warp)
+    const uint32_t cwords = (e->g.Emax + 31) / 32;
+    a.chain_bitset = cwords <= 2048 ? 1u : 0u;
+    const size_t csmem = a.chain_bitset ? (size_t)CHAIN_WARPS * cwords * 4 : 0;
+    if ((int)csmem > e->chain_smem) {
+      cudaFuncSetAttribute(k_chain, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)csmem);
+      e->chain_smem = (int)csmem;
+    }
+    k_chain<<<(nq + CHAIN_WARPS - 1) / CHAIN_WARPS, CHAIN_WARPS * 32, csmem, s>>>(a);
   }
   // exact path (windows that may hold duplicates, anchored queries) on the
   // engine's second side stream, beside the fast path on `s`

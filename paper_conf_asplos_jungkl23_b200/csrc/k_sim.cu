@@ -34,7 +34,7 @@
 namespace dum {
 
 constexpr int SIM_NT = 1024;
-constexpr uint32_t SIM_HCAP = 8192;  // launch accesses <= SIM_HCAP / 2 (shared first-position hash)
+constexpr uint32_t SIM_HCAP = 16384;  // launch accesses <= SIM_HCAP / 2 (shared first-position hash, 128 KiB)
 
 // 1. faults of one launch: its accesses without a frame, first occurrence,
 // in access order; marks the launch's access set in acc_bits (demand rule D22).
@@ -295,7 +295,8 @@ cudaError_t launch_simulate(dum_engine *e, const uint64_t *hash, uint32_t n_laun
       k_sim_prefetch<<<1, SIM_NT, 0, s>>>(e->sim_pairs, r_pairs, e->d_res_bits, e->sim_pf, r_pf, e->d_state);
       if ((err = launch_migrate(e, DUM_H2D, e->sim_pf, nullptr, g.C, 1, s, r_pf)) != cudaSuccess) return err;
     }
-    k_sim_close<<<8, 256, 0, s>>>(acc, n, g.W, e->sim_acc_bits, r_dem, r_pre, r_pf, preevict ? 1u : 0u,
+    k_sim_close<<<8, 256, 0, s>>>(acc, n, g.W, e->sim_acc_bits, r_dem, r_pre, r_pf,
+                                  (preevict && k + 1 < n_launch) ? 1u : 0u,
                                   (prefetch && k + 1 < n_launch) ? 1u : 0u, invalidate ? 1u : 0u, stats + k);
     e->kernel_launches += 8;
   }

@@ -42,7 +42,7 @@ namespace dum {
 
 constexpr int IX_NT = 512;
 constexpr int IX_U = 4;              // walk entries per thread with their loads in flight together
-constexpr uint32_t CONF_HCAP = 128;  // shared hash of one walk's conflicts (> CONF_MAX)
+constexpr uint32_t CONF_HCAP = 256;  // shared hash of one walk's conflicts (> CONF_MAX)
 
 __global__ void __launch_bounds__(IX_NT) k_walk_count(const uint32_t *__restrict__ walk,
                                                       const uint32_t *__restrict__ walk_len, uint32_t walk_cap,
@@ -98,7 +98,7 @@ __global__ void __launch_bounds__(IX_NT) k_walk_conf(const uint32_t *__restrict_
         for (uint32_t k = 0; k < c[u]; ++k) {
           const uint32_t h = bhold[(uint64_t)b[u] * HOLD_MAX + k];
           if (h == e) continue;
-          uint32_t sl = (h * 0x9E3779B1u) >> 25;  // 7 bits: CONF_HCAP = 128
+          uint32_t sl = (h * 0x9E3779B1u) >> 24;  // 8 bits: CONF_HCAP = 256
           bool placed = false;
           for (uint32_t p = 0; p < CONF_HCAP; ++p, sl = (sl + 1) & (CONF_HCAP - 1)) {
             // most inserts repeat a recorded conflict: a plain read first (no
@@ -264,44 +264,32 @@ constexpr uint32_t FSEG = 1024;                 // log entries per segment (32 p
 constexpr uint32_t FSEG_MAX = POS_WORDS * 32 / FSEG;
 static_assert(FSEG_MAX <= 32, "one warp scans the segment counts");
 
-// Eligibility masks of one segment's entries for the calling lane: entries
-// p0 + 128 k + 4 lane + u (u < 4) -> bit u of am[k] (active) / im[k]
-// (inactive); eligible = inside [head, tail), not a resident window block
-// (posmap over positions from head), still resident with its stamp.
-constexpr uint32_t FHALF = FSEG / 256;  // 16 B loads per lane per half segment
-
-__device__ __forceinline__ void seg_masks(const SelectOut &so, const uint32_t *posmap, uint32_t p0, uint32_t head,
-                                          uint32_t tail, bool clean, uint32_t lane, uint32_t *am, uint32_t *im,
-                                          uint4 *vout = nullptr) {
-  uint4 v[FHALF];
-#pragma unroll
-  for (uint32_t k = 0; k < FHALF; ++k) {
-    const uint32_t p = p0 + 128 * k + 4 * lane;
-    v[k] = p < tail ? __ldcg(reinterpret_cast<const uint4 *>(so.lrm_blk + p)) : make_uint4(0, 0, 0, 0);
+// One warp step of the selection: the 32 log entries at positions
+// head + r0 + lane (r0 a multiple of 32 relative to head, so that one
+// broadcast word of the position bitmap covers them).  Eligible = inside the
+// log, not a resident window block, still resident with its stamp; returns the
+// active / inactive eligible ballots.  v = the entry (block | inactive << 31).
+__device__ __forceinline__ void step_masks(const SelectOut &so, const uint32_t *posmap, uint32_t head,
+                                           uint32_t tail, bool clean, uint32_t lane, uint32_t r0, uint32_t v,
+                                           uint32_t &ma, uint32_t &mi) {
+  const uint32_t p = head + r0 + lane;
+  const uint32_t w = (r0 >> 5) < POS_WORDS ? posmap[r0 >> 5] : 0xFFFFFFFFu;  // beyond the map: never reached
+  bool el = p < tail && !((w >> lane) & 1u);
+  if (!clean && el) {
+    const uint32_t b = v & 0x7FFFFFFFu;
+    el = __ldg(&so.frame_of[b]) != NONE && __ldg(&so.stamp_of[b]) == __ldcg(so.lrm_stamp + p);
   }
-#pragma unroll
-  for (uint32_t k = 0; k < FHALF; ++k) {
-    const uint32_t vv[4] = {v[k].x, v[k].y, v[k].z, v[k].w};
-    uint32_t a = 0, in = 0;
-#pragma unroll
-    for (uint32_t u = 0; u < 4; ++u) {
-      const uint32_t p = p0 + 128 * k + 4 * lane + u;
-      const uint32_t b = vv[u] & 0x7FFFFFFFu, r = p - head;
-      bool el = p >= head && p < tail && r < POS_WORDS * 32 && !((posmap[r >> 5] >> (r & 31)) & 1u);
-      if (!clean && el) el = __ldg(&so.frame_of[b]) != NONE && __ldg(&so.stamp_of[b]) == __ldcg(so.lrm_stamp + p);
-      a |= (el && !(vv[u] >> 31)) ? 1u << u : 0u;
-      in |= (el && (vv[u] >> 31)) ? 1u << u : 0u;
-    }
-    am[k] = a;
-    im[k] = in;
-    if (vout) vout[k] = v[k];
-  }
+  ma = __ballot_sync(0xffffffffu, el && !(v >> 31));
+  mi = __ballot_sync(0xffffffffu, el && (v >> 31));
 }
 
-__global__ void __launch_bounds__(WSEL_NT, 4) k_select_fast(PredArgs a) {
+constexpr uint32_t FB = 8;  // warp steps with their entry loads in flight together
+
+__global__ void __launch_bounds__(WSEL_NT, 8) k_select_fast(PredArgs a) {
   __shared__ uint32_t kern[MAXN + 1], roff[MAXN + 2];
   __shared__ uint32_t posmap[POS_WORDS];
   __shared__ uint32_t seg_cnt[FSEG_MAX], seg_pre[FSEG_MAX];
+  __shared__ uint32_t wem[POS_WORDS], wim[POS_WORDS], wpre[POS_WORDS];  // clean-log word path
   __shared__ uint32_t s_need, s_head, s_tail, s_clean, s_ok, s_tw, s_ti, s_nres;
   __shared__ unsigned long long s_bwb, s_binv;
   constexpr uint32_t NW = WSEL_NT / 32;
@@ -371,28 +359,112 @@ __global__ void __launch_bounds__(WSEL_NT, 4) k_select_fast(PredArgs a) {
         }
       }
       const uint32_t stale = tail - head - s_nres;
-      const uint32_t span = min(tail - head, min(need + R + stale, POS_WORDS * 32 - 4));
+      const uint32_t span = min(tail - head, min(need + R + stale, POS_WORDS * 32));
       __syncthreads();
-      // Segments start at absolute positions multiple of 4 (16 B loads); lane
-      // l owns entries base + 128 k + 4 l .. +3 (k < 8); all 8 loads of a
-      // segment are issued together.
-      const uint32_t hb = head & ~3u;
-      nseg = (span + (head - hb) + FSEG - 1) / FSEG;
+      if (clean && a.inact_bits) {
+        // ---- clean log: word-level selection.  Every entry of [head, tail) is
+        // valid, so a 32-position word's eligible entries are ~excluded & valid,
+        // split by the log's inactive-entry bitmap (k_log_bits): counts and
+        // ranks come from popcounts; only the taken entries are read. ----
+        const uint32_t nw = (span + 31) / 32;
+        uint32_t ca[4], ci[4], em[4], imk[4];
+        uint32_t tot = 0;
+#pragma unroll
+        for (uint32_t u = 0; u < 4; ++u) {  // thread t owns words 4t .. 4t+3 (nw <= POS_WORDS = 4 * WSEL_NT)
+          const uint32_t w = 4 * tid + u;
+          em[u] = imk[u] = 0;
+          if (w < nw) {
+            const uint32_t lo = w * 32, valid = span - lo >= 32 ? 0xFFFFFFFFu : (1u << (span - lo)) - 1u;
+            const uint32_t ib = __ldg(a.inact_bits + w);
+            const uint32_t e = valid & ~posmap[w];
+            em[u] = e & ~ib;
+            imk[u] = e & ib;
+          }
+          ca[u] = __popc(em[u]);
+          ci[u] = __popc(imk[u]);
+          tot += ca[u] | (ci[u] << 16);
+        }
+        uint32_t tsum;
+        const uint32_t tpre = block_excl_scan(tot, seg_pre, &tsum);  // packed (inactive << 16 | active)
+        {
+          uint32_t pre = tpre;
+#pragma unroll
+          for (uint32_t u = 0; u < 4; ++u) {
+            const uint32_t w = 4 * tid + u;
+            if (w < nw) {
+              wem[w] = em[u];
+              wim[w] = imk[u];
+              wpre[w] = pre;
+            }
+            pre += ca[u] | (ci[u] << 16);
+          }
+        }
+        __syncthreads();
+        // a warp per word, a lane per position: the eligible entries of
+        // combined rank < need, written at their list ranks (4 words in flight)
+        const uint32_t lt = (1u << lane) - 1;
+        uint32_t tw = 0, ti = 0;
+        for (uint32_t w0 = wid; w0 < nw; w0 += NW * 4) {
+          uint32_t v[4], mA[4], mI[4], pr[4];
+#pragma unroll
+          for (uint32_t u = 0; u < 4; ++u) {
+            const uint32_t w = w0 + u * NW;
+            mA[u] = mI[u] = 0;
+            pr[u] = 0;
+            v[u] = 0;
+            if (w < nw) {
+              pr[u] = wpre[w];
+              if ((pr[u] & 0xFFFFu) + (pr[u] >> 16) < need) {
+                mA[u] = wem[w];
+                mI[u] = wim[w];
+                if (((mA[u] | mI[u]) >> lane) & 1u) v[u] = __ldcg(so.lrm_blk + head + w * 32 + lane);
+              }
+            }
+          }
+#pragma unroll
+          for (uint32_t u = 0; u < 4; ++u) {
+            const bool ea = (mA[u] >> lane) & 1u, ei = (mI[u] >> lane) & 1u;
+            const uint32_t ra = (pr[u] & 0xFFFFu) + __popc(mA[u] & lt), rr = (pr[u] >> 16) + __popc(mI[u] & lt);
+            if ((ea || ei) && ra + rr < need) {
+              if (ok) {
+                if (ei) so.inv[binv + rr] = v[u] & 0x7FFFFFFFu;
+                else so.wb[bwb + ra] = v[u];
+              }
+              tw += ea;
+              ti += ei;
+            }
+          }
+        }
+        tw = __reduce_add_sync(0xffffffffu, tw);
+        ti = __reduce_add_sync(0xffffffffu, ti);
+        if (lane == 0 && (tw | ti)) {
+          atomicAdd(&s_tw, tw);
+          atomicAdd(&s_ti, ti);
+        }
+        nseg = (span + FSEG - 1) / FSEG;  // (reported as scanned)
+        __syncthreads();
+      } else {
+      // segments of FSEG positions relative to head; a warp step covers 32
+      nseg = (span + FSEG - 1) / FSEG;
       __syncthreads();
       // 2. pass 1: eligible entries per segment (active | inactive << 16)
       for (uint32_t sg = wid; sg < nseg; sg += NW) {
         uint32_t na = 0, ni = 0;
-        for (uint32_t h = 0; h < 2; ++h) {
-          uint32_t am[FHALF], im[FHALF];
-          seg_masks(so, posmap, hb + sg * FSEG + h * (FSEG / 2), head, tail, clean, lane, am, im);
+        for (uint32_t k0 = 0; k0 < FSEG / 32; k0 += FB) {
+          uint32_t v[FB];
 #pragma unroll
-          for (uint32_t k = 0; k < FHALF; ++k) {
-            na += __popc(am[k]);
-            ni += __popc(im[k]);
+          for (uint32_t u = 0; u < FB; ++u) {
+            const uint32_t p = head + sg * FSEG + 32 * (k0 + u) + lane;
+            v[u] = p < tail ? __ldcg(so.lrm_blk + p) : 0u;
+          }
+#pragma unroll
+          for (uint32_t u = 0; u < FB; ++u) {
+            uint32_t ma, mi;
+            step_masks(so, posmap, head, tail, clean, lane, sg * FSEG + 32 * (k0 + u), v[u], ma, mi);
+            na += __popc(ma);
+            ni += __popc(mi);
           }
         }
-        na = __reduce_add_sync(0xffffffffu, na);
-        ni = __reduce_add_sync(0xffffffffu, ni);
         if (lane == 0) seg_cnt[sg] = na | (ni << 16);
       }
       __syncthreads();
@@ -409,45 +481,35 @@ __global__ void __launch_bounds__(WSEL_NT, 4) k_select_fast(PredArgs a) {
       }
       __syncthreads();
       // 4. pass 2: the entries of combined rank < need, at their list ranks
+      const uint32_t lt = (1u << lane) - 1;
       uint32_t tw = 0, ti = 0;
       for (uint32_t sg = wid; sg < nseg; sg += NW) {
         const uint32_t pre = seg_pre[sg];
         uint32_t rw = pre & 0xFFFFu, ri = pre >> 16;
-        if (rw + ri >= need) continue;
-        for (uint32_t h = 0; h < 2 && rw + ri < need; ++h) {
-        uint32_t am[FHALF], im[FHALF];
-        uint4 v[FHALF];
-        seg_masks(so, posmap, hb + sg * FSEG + h * (FSEG / 2), head, tail, clean, lane, am, im, v);
+        for (uint32_t k0 = 0; k0 < FSEG / 32 && rw + ri < need; k0 += FB) {
+          uint32_t v[FB];
 #pragma unroll
-        for (uint32_t k = 0; k < FHALF; ++k) {
-          // lane-exclusive prefix of the eligible counts (active | inactive << 16)
-          const uint32_t c = __popc(am[k]) | (__popc(im[k]) << 16);
-          uint32_t x = c;
-#pragma unroll
-          for (int o = 1; o < 32; o <<= 1) {
-            const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-            if (lane >= (uint32_t)o) x += y;
+          for (uint32_t u = 0; u < FB; ++u) {
+            const uint32_t p = head + sg * FSEG + 32 * (k0 + u) + lane;
+            v[u] = p < tail ? __ldcg(so.lrm_blk + p) : 0u;
           }
-          const uint32_t tot = __shfl_sync(0xffffffffu, x, 31);
-          uint32_t ra = rw + ((x - c) & 0xFFFFu), rr = ri + ((x - c) >> 16);
-          const uint32_t vv[4] = {v[k].x, v[k].y, v[k].z, v[k].w};
 #pragma unroll
-          for (uint32_t u = 0; u < 4; ++u) {
-            const bool ea = (am[k] >> u) & 1u, ei = (im[k] >> u) & 1u;
+          for (uint32_t u = 0; u < FB; ++u) {
+            uint32_t ma, mi;
+            step_masks(so, posmap, head, tail, clean, lane, sg * FSEG + 32 * (k0 + u), v[u], ma, mi);
+            const uint32_t ra = rw + __popc(ma & lt), rr = ri + __popc(mi & lt);
+            const bool ea = (ma >> lane) & 1u, ei = (mi >> lane) & 1u;
             if ((ea || ei) && ra + rr < need) {
               if (ok) {
-                if (ei) so.inv[binv + rr] = vv[u] & 0x7FFFFFFFu;
-                else so.wb[bwb + ra] = vv[u];
+                if (ei) so.inv[binv + rr] = v[u] & 0x7FFFFFFFu;
+                else so.wb[bwb + ra] = v[u];
               }
               tw += ea;
               ti += ei;
             }
-            ra += ea;
-            rr += ei;
+            rw += __popc(ma);
+            ri += __popc(mi);
           }
-          rw += tot & 0xFFFFu;
-          ri += tot >> 16;
-        }
         }
       }
       tw = __reduce_add_sync(0xffffffffu, tw);
@@ -457,6 +519,7 @@ __global__ void __launch_bounds__(WSEL_NT, 4) k_select_fast(PredArgs a) {
         atomicAdd(&s_ti, ti);
       }
       __syncthreads();
+      }  // per-entry path (stale log entries)
     }
     if (tid == 0) {
       uint64_t *o = so.out_range + 4ull * qi;
@@ -465,8 +528,9 @@ __global__ void __launch_bounds__(WSEL_NT, 4) k_select_fast(PredArgs a) {
       o[2] = binv;
       o[3] = binv + (ok ? s_ti : 0);
       // log entries read by the selection: the segments (each pass reads them)
-      ctr_add(a.st, DUM_CTR_FAST_SCANNED, need ? min(tail - head, nseg * FSEG) : 0u);
+      ctr_add(a.st, DUM_CTR_FAST_SCANNED, need ? min(tail - head, nseg * FSEG) : 0u);  // (both passes read these)
       ctr_add(a.st, DUM_CTR_FAST_VICTIMS, s_tw + s_ti);
+      if (!clean) ctr_add(a.st, DUM_CTR_FAST_DIRTY, 1);
     }
     __syncthreads();  // the next query reuses the shared state
   }
@@ -494,12 +558,28 @@ cudaError_t launch_walk_index(dum_engine *e, cudaStream_t main) {
   return cudaGetLastError();
 }
 
+// The LRM log's inactive entries as a bitmap over positions relative to the
+// head (bit l of word w = entry head + 32 w + l is inactive): the fast
+// selection's clean-log path splits write-back / invalidate by popcounts.
+__global__ void __launch_bounds__(256) k_log_bits(const uint32_t *__restrict__ lrm_blk, const DevState *st,
+                                                  uint32_t *bits) {
+  const uint32_t head = *(const volatile uint32_t *)&st->lrm_head, tail = *(const volatile uint32_t *)&st->lrm_tail;
+  const uint32_t nw = (tail - head + 31) / 32, lane = threadIdx.x & 31;
+  for (uint32_t w = (blockIdx.x * 256 + threadIdx.x) >> 5; w < nw; w += gridDim.x * 8) {
+    const uint32_t p = head + 32 * w + lane;
+    const uint32_t m = __ballot_sync(0xffffffffu, p < tail && (__ldg(lrm_blk + p) >> 31));
+    if (lane == 0) bits[w] = m;
+  }
+}
+
 // Predict time: per-walk residency facts for the fast selection.
 cudaError_t launch_walk_res(dum_engine *e, cudaStream_t s) {
   TimerScope t(e, DUM_T_WALK_RES, s);
   k_walk_res<<<index_grid(e), IX_NT, 0, s>>>(e->d_walk, e->d_walk_len, e->g.walk_cap, e->d_state, e->d_res_bits,
                                              e->d_logpos, e->d_wnr, e->d_wnres, e->d_respos);
-  e->kernel_launches += 1;
+  k_log_bits<<<std::min<uint32_t>(e->lrm_cap / 256 + 1, 148 * 4), 256, 0, s>>>(e->d_lrm_blk, e->d_state,
+                                                                              e->d_log_bits);
+  e->kernel_launches += 2;
   return cudaGetLastError();
 }
 

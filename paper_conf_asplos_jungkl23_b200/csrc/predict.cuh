@@ -10,7 +10,7 @@ namespace dum {
 constexpr uint32_t MAXN = 128;      // degree_n limit
 constexpr int NQCLS = 5;            // window-size classes of k_chain's query order
 constexpr uint32_t HOLD_MAX = 16;   // walk index: holders recorded per block
-constexpr uint32_t CONF_MAX = 32;   // walk index: conflicting exec IDs recorded per walk
+constexpr uint32_t CONF_MAX = 64;   // walk index: conflicting exec IDs recorded per walk
 constexpr uint32_t CHUNK_B = 128;   // window blocks per copy chunk (one warp: 4 coalesced steps)
 constexpr int COPY_NT = 256;        // k_copy_fast threads
 constexpr int WSEL_NT = 256;        // k_select_fast threads
@@ -22,6 +22,7 @@ struct PredArgs {
   const dum_query *q;
   uint32_t nq;
   uint32_t select;       // a8 fused (dum_predict_select)
+  uint32_t chain_bitset; // k_chain tests conflicts against a shared bitset of the chain
   const CorrSlot *corr;
   uint32_t corr_cap;
   const uint32_t *jump;  // [levels][corr_cap]
@@ -38,6 +39,7 @@ struct PredArgs {
   // walk index (k_window.cu): conflicts per walk; residency facts per walk
   const uint32_t *conf, *conf_n;
   const uint32_t *wnr, *wnres, *respos;
+  const uint32_t *inact_bits;  // the LRM log's inactive entries by position from head (k_log_bits), or null
   // per-query scratch written by k_chain
   uint32_t *qkern;  // [nq][N+1]
   uint32_t *qloff;  // [nq][N+2]

@@ -356,3 +356,42 @@ def test_sequential_walker_mode_builds_identical_walks(R):
         assert_same_predictions(ro, rg)
     c = eng.counters()
     assert c["WALK_SLOW"] > 0 and c["WALK_DEDUPE"] == 0, c
+
+
+@pytest.mark.parametrize("host", [True, False])
+def test_dum_step_equals_the_separate_calls(host):
+    """dum_step (record -> queries -> predict+select -> build in one call) on
+    Config T with a residency snapshot and inactive blocks: every iteration's
+    windows, victims and the final tables equal the oracle's."""
+    tr = wl.make_T(dup_ppm=100_000)
+    N = 2
+    eng, o = make_pair(W=tr.W, C=tr.C, N=N)
+    snap = tr.snap_blk[4][: int(tr.snap_cnt[4])]
+    o.load_residency(snap)
+    eng.load_residency(dev(snap))
+    inact = np.arange(0, tr.W, 5, dtype=np.uint32)
+    o.mark_inactive(inact, True)
+    eng.mark_inactive(dev(inact), True)
+    out = {}
+    ex_all = []
+    for i in range(tr.n_iter):
+        h, off, f = tr.iteration(i)
+        ex_all += [int(x) for x in o.record_faults(h, off, f)]
+        qs = transition_queries(ex_all, i * tr.K, tr.K, N)
+        off_o, pairs_o, ko_o, ch_o = o.predict(qs)
+        wo, wb_o, io, iv_o = o.select(off_o, pairs_o, qs[:, 4])
+        o.build_tables()
+        if host:
+            eng.step(np.asarray(h, np.uint64), np.asarray(off, np.uint64), np.asarray(f, np.uint32), 4096, 4096, out)
+        else:
+            eng.step(dev(h, np.uint64), dev(off, np.uint64), dev(f), 4096, 4096, out)
+        eng.sync()
+        gp, rg = B.u32(out["pairs"]).reshape(-1, 2), B.u64(out["rng"]).reshape(-1, 2)
+        sr = B.u64(out["sel_rng"]).reshape(-1, 4)
+        gwb, giv = B.u32(out["wb"]), B.u32(out["inv"])
+        for q in range(tr.K):
+            assert np.array_equal(gp[rg[q, 0]:rg[q, 1]], pairs_o[off_o[q]:off_o[q + 1]]), (i, q)
+            assert np.array_equal(B.u32(out["kern_off"])[q], ko_o[q]) and np.array_equal(B.u32(out["chain"])[q], ch_o[q])
+            assert np.array_equal(gwb[sr[q, 0]:sr[q, 1]], wb_o[wo[q]:wo[q + 1]]), (i, q)
+            assert np.array_equal(giv[sr[q, 2]:sr[q, 3]], iv_o[io[q]:io[q + 1]]), (i, q)
+    assert_same_state(eng, o)

@@ -1,0 +1,106 @@
+#!/usr/bin/env python
+"""SURVEY.md 8(f) rows 1-2 on the GPU: the closed loop (dum_simulate) at B / G
+scale, metadata-only, and its sweeps.
+
+    python tools/sim_f1.py [--configs B,G] [--iters 10] [--out profiles/r02_f1.json]
+
+  * Table 5 shape: demand faults per iteration, naive UM
+    (no prefetch) vs the engine (prefetch + pre-eviction + invalidation).
+  * Fig. 10 ablation: naive / prefetch / + pre-eviction /
+    + invalidation: faults, blocks migrated in (demand, prefetch), written back,
+    invalidated -- per iteration, steady state = mean of iterations 1..
+  * Fig. 11: degree N in {1, 2, 4, 8, 16, 32, 64} (B).
+  * Fig. 12 / Table 6: Config0 - Config12 (B).
+  * Cross-check: naive UM here == the generator's naive-UM fault trace
+    (workloads/um_sim.c, independent code).
+Every number comes from the engine's kernels; the host only launches."""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import workloads as wl  # noqa: E402
+from paper_conf_asplos_jungkl23_b200 import Engine, binding as B  # noqa: E402
+
+TABLE6 = {  # PAPER.md Table 6 (L429-L443): name -> (Assoc, NumSuccs, NumRows)
+    "Config0": (2, 4, 128), "Config1": (2, 8, 128), "Config2": (4, 4, 128), "Config3": (2, 4, 512),
+    "Config4": (2, 8, 512), "Config5": (4, 4, 512), "Config6": (2, 4, 1024), "Config7": (2, 8, 1024),
+    "Config8": (4, 4, 1024), "Config9": (2, 4, 2048), "Config10": (2, 8, 2048), "Config11": (4, 4, 2048),
+    "Config12": (2, 4, 4096),
+}
+ABLATIONS = {"naive_um": 0, "prefetch": B.SIM_PREFETCH, "prefetch+preevict": B.SIM_PREFETCH | B.SIM_PREEVICT,
+             "prefetch+preevict+invalidate": B.SIM_PREFETCH | B.SIM_PREEVICT | B.SIM_INVALIDATE}
+
+
+def run(tr, dev, flags, N=32, geo=(2, 4, 2048)):
+    A, S, R = geo
+    eng = Engine(num_rows=R, assoc=A, num_succs=S, degree_n=max(N, 1), max_blocks=tr.W, max_exec_ids=8192,
+                 hbm_frames=tr.C, corr_capacity=1 << 16, device=dev.index or 0)
+    eng.mark_inactive(torch.from_numpy(tr.inactive_blocks.view(np.int32)).to(dev), True)
+    h = torch.from_numpy(np.ascontiguousarray(tr.launch_hash).view(np.int64)).to(dev)
+    acc = torch.from_numpy(np.ascontiguousarray(tr.access_blk).view(np.int32)).to(dev)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    st = eng.simulate(h, np.asarray(tr.access_off, np.uint64), acc, N, flags)
+    eng.sync()
+    dt = time.perf_counter() - t0
+    s = st.cpu().numpy().view(np.uint32).reshape(tr.n_iter, tr.K, -1).astype(np.int64).sum(axis=1)
+    eng.close()
+    cols = {f: s[:, i].tolist() for i, f in enumerate(B.SIM_FIELDS)}
+    steady = {f: float(np.mean(v[1:])) for f, v in cols.items()}
+    return {"per_iteration": cols, "steady_mean": steady, "wall_s": round(dt, 2),
+            "launches": tr.n_iter * tr.K, "launches_per_s": round(tr.n_iter * tr.K / dt)}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--configs", default="B,G")
+    ap.add_argument("--iters", type=int, default=10)
+    ap.add_argument("--out", default="")
+    ap.add_argument("--no-sweeps", action="store_true")
+    args = ap.parse_args()
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(dev)
+    out = {"how": __doc__.split("\n\n")[1], "configs": {}}
+    for cfg in args.configs.split(","):
+        tr = wl.make(cfg, n_iter=args.iters)
+        res = {"trace_naive_um_faults": [int(tr.faults_in_iteration(i)) for i in range(tr.n_iter)],
+               "W": tr.W, "C": tr.C, "K": tr.K, "ablation": {}}
+        for name, fl in ABLATIONS.items():
+            res["ablation"][name] = run(tr, dev, fl, N=32 if fl else -1)
+            print(cfg, name, res["ablation"][name]["steady_mean"], res["ablation"][name]["wall_s"], file=sys.stderr)
+        naive = res["ablation"]["naive_um"]["per_iteration"]["faults"]
+        res["naive_equals_trace"] = naive == res["trace_naive_um_faults"]
+        full = res["ablation"]["prefetch+preevict+invalidate"]["steady_mean"]["faults"]
+        res["table5_shape"] = {"naive_um_faults_per_iter": float(np.mean(naive[1:])),
+                               "engine_faults_per_iter": full,
+                               "ratio": full / max(float(np.mean(naive[1:])), 1.0)}
+        if cfg == "B" and not args.no_sweeps:
+            res["degree_sweep"] = {}
+            for N in (1, 2, 4, 8, 16, 32, 64):
+                r = run(tr, dev, B.SIM_PREFETCH | B.SIM_PREEVICT | B.SIM_INVALIDATE, N=N)
+                res["degree_sweep"][N] = r["steady_mean"]
+                print(cfg, "N", N, r["steady_mean"], file=sys.stderr)
+            res["geometry_sweep"] = {}
+            for name, geo in TABLE6.items():
+                r = run(tr, dev, B.SIM_PREFETCH | B.SIM_PREEVICT | B.SIM_INVALIDATE, N=32, geo=geo)
+                res["geometry_sweep"][name] = r["steady_mean"]
+                print(cfg, name, r["steady_mean"], file=sys.stderr)
+        out["configs"][cfg] = res
+    s = json.dumps(out)
+    if args.out:
+        open(args.out, "w").write(s + "\n")
+    print(s)
+
+
+if __name__ == "__main__":
+    main()
