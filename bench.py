@@ -60,7 +60,9 @@ def parse():
     ap.add_argument("--no-migration", action="store_true")
     ap.add_argument("--cpu-launches", type=int, default=0, help="oracle sample size in launches")
     ap.add_argument("--json-out", default="")
-    ap.add_argument("--unfused", action="store_true", help="separate predict / select calls")
+    ap.add_argument("--separate-calls", action="store_true",
+                    help="record / make_queries / predict_select / build as separate C-ABI calls instead of dum_step")
+    ap.add_argument("--no-graph", action="store_true", help="dum_step without its CUDA graph")
     ap.add_argument("--debug", action="store_true", help="synchronize and check after every call")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="process group of the N>1 replicas (barrier + reductions only); gloo lets several ranks "
@@ -151,14 +153,15 @@ def algorithmic_bytes(ctr, geo, N):
         "predict": 4 * c["GATHERED"] + 8 * c["EMITTED"] + 4 * (N + 2) * c["QUERIES"],
         "select": 4 * scanned + 4 * victims,
     }
-    fast = (12 * c["FAST_EMITTED"] + 4 * (N + 2) * c["Q_FAST"] + 4 * c["FAST_SCANNED"] + 4 * c["FAST_VICTIMS"])
+    fast_copy = 12 * c["FAST_EMITTED"] + 4 * (N + 2) * c["Q_FAST"]
+    fast_sel = 4 * c["FAST_SCANNED"] + 4 * c["FAST_VICTIMS"]
     per_kernel = {
         "k_ingest": terms["ingest"] + 16 * c["LAUNCHES"],
         "k_build_prep": 48 * c["CORR_UPSERTS"],
-        "k_apply": terms["block_tables"],
-        "k_walk": terms["walk_cache"],
-        "k_window": fast,
-        "k_predict": terms["predict"] + terms["select"] - fast,
+        "k_build_exec": terms["block_tables"] + terms["walk_cache"],  # apply + walks (dedupe walks: k_walk)
+        "k_copy_fast": fast_copy,
+        "k_select_fast": fast_sel,
+        "k_predict": terms["predict"] + terms["select"] - fast_copy - fast_sel,
     }
     return terms, per_kernel, c
 
@@ -302,9 +305,15 @@ def run_ours(args, rank, world, local_rank):
 
     step_ready = [False]  # DUM_INPUTS_READY: the ingest may overlap the previous build
 
+    outs = {}  # dum_step outputs (fixed addresses: a replayed step graph writes them)
+
     def step(i, host=None, after_predict=None):
         """record(i) -> queries -> predict(i) -> select(i) -> build(i)"""
         dbg.i = i
+        if not args.separate_calls:  # one dum_step call (a replayed CUDA graph unless --no-graph)
+            eng.step(hs[i], offs[i], fs[i], cap[0], cap[0], outs, ready=step_ready[0])
+            dbg("dum_step")
+            return
         out_exec = exec_all[3 + i * K: 3 + (i + 1) * K]
         if host is None:
             eng.record_faults(hs[i], offs[i], fs[i], out_exec, ready=step_ready[0])
@@ -314,7 +323,7 @@ def run_ours(args, rank, world, local_rank):
         if i >= 1:
             eng.make_queries(exec_all[i * K: 3 + (i + 1) * K], 3, N, out=qbuf)
             dbg("make_queries")
-            if args.unfused:
+            if False:
                 eng.predict_prefetch(qbuf, cap[0], pairs=pairs[0], rng=rng, kern_off=ko, chain=ch, needed=need_p)
                 eng.select_evictions(rng, pairs[0], qbuf, cap[0], wb=wb[0], inv=inv[0], out_rng=srng,
                                      needed=need_s)
@@ -334,6 +343,7 @@ def run_ours(args, rank, world, local_rank):
         eng.set_timing(timing_on[0])
 
     timing_on = [False]
+    eng.set_step_graphs(not args.separate_calls and not args.no_graph)
     # iteration 0 (cold build, untimed) + capacity sizing on iteration 1
     eng.mark_inactive(inactive, True)
     pre_step(0)
@@ -353,7 +363,10 @@ def run_ours(args, rank, world, local_rank):
         except B.EngineError as e:
             if e.code != -2:
                 raise
-        need = max(int(need_p.item()), int(need_s.item()))
+        if args.separate_calls:
+            need = max(int(need_p.item()), int(need_s.item()))
+        else:
+            need = max(int(outs["needed"].item()), int(outs["sel_needed"].item()))
         if need * 1.1 > cap[0]:
             grow(need)
     torch.cuda.synchronize()
@@ -399,13 +412,19 @@ def run_ours(args, rank, world, local_rank):
     verify_out = None
     if args.verify:  # the last timed step's outputs, checked against the oracle below
         i_v = args.warmup + args.steps
-        verify_out = (i_v, B.u32(pairs[0]).reshape(-1, 2).copy(), B.u64(rng).reshape(-1, 2).copy(),
-                      B.u32(ko).reshape(K, -1).copy(), B.u32(ch).reshape(K, -1).copy(), B.u32(wb[0]).copy(),
-                      B.u32(inv[0]).copy(), B.u64(srng).reshape(-1, 4).copy())
+        if args.separate_calls:
+            o = {"pairs": pairs[0], "rng": rng, "kern_off": ko, "chain": ch, "wb": wb[0], "inv": inv[0],
+                 "sel_rng": srng}
+        else:
+            o = outs
+        verify_out = (i_v, B.u32(o["pairs"]).reshape(-1, 2).copy(), B.u64(o["rng"]).reshape(-1, 2).copy(),
+                      B.u32(o["kern_off"]).reshape(K, -1).copy(), B.u32(o["chain"]).reshape(K, -1).copy(),
+                      B.u32(o["wb"]).copy(), B.u32(o["inv"]).copy(), B.u64(o["sel_rng"]).reshape(-1, 4).copy())
     eng.read_counters(reset=True)
     # ---- breakdown pass: K further steps (the next trace iterations) with CUDA
     # events around every kernel, for the per-kernel durations / roofline ----
     eng.read_timing(reset=True)
+    eng.set_step_graphs(False)  # per-kernel events need the kernels issued one by one
     timing_on[0] = True
     bk_ms = 0.0
     for s in range(args.steps):
@@ -444,7 +463,9 @@ def run_ours(args, rank, world, local_rank):
             if ab is not None:
                 per_kernel[kn]["alg_bytes_per_launch"] = int(ab / kcnt[idx])
                 per_kernel[kn]["achieved_gbs"] = round(ab / kcnt[idx] / (avg_ms / 1000) / 1e9, 1)
-    dom = max((k for k in per_kernel if "stream" not in per_kernel[k]), key=lambda k: per_kernel[k]["ms_total"])
+    # dominant = the longest kernel of the step, side streams included (their
+    # work is part of the step); the jump tables overlap the build entirely
+    dom = max((k for k in per_kernel if k != "k_jump0"), key=lambda k: per_kernel[k]["ms_total"])
     d = per_kernel[dom]
     traffic = load_traffic().get(dom, {}).get("dram_bytes_per_launch")
     roof = {"kernel": dom, "bound": "hbm", "achieved": d.get("achieved_gbs"), "peak": peak, "unit": "GB/s",
@@ -452,9 +473,10 @@ def run_ours(args, rank, world, local_rank):
             "traffic": traffic, "alg_bytes_per_launch": d.get("alg_bytes_per_launch"),
             "avg_us": d.get("avg_us"), "peak_source": peak_src,
             "bytes_formula": {
-                "k_window": "12*FAST_EMITTED + 4*(N+2)*Q_FAST + 4*FAST_SCANNED + 4*FAST_VICTIMS "
-                            "(SURVEY 8(d) predict + select terms for the queries k_window answers)",
-                "k_apply": "2*set_bytes*SETS", "k_walk": "set_bytes*WALK_ROWS + 4*WALK_OUT",
+                "k_copy_fast": "4*GATHERED + 8*EMITTED + 4*(N+2)*QUERIES of the fast queries = "
+                               "12*FAST_EMITTED + 4*(N+2)*Q_FAST (SURVEY 8(d) predict term)",
+                "k_select_fast": "4*FAST_SCANNED + 4*FAST_VICTIMS (SURVEY 8(d) select term)",
+                "k_build_exec": "2*set_bytes*SETS + set_bytes*WALK_ROWS + 4*WALK_OUT (block tables + walk cache)",
                 "k_ingest": "4*RAW + 4*NORM + 20*LAUNCHES + 16*LAUNCHES (exec-map probe)",
                 "k_build_prep": "48*CORR_UPSERTS", "set_bytes": 4 * geo["A"] * (1 + geo["S"]), "N": N},
             "timing": "avg CUDA-event duration of the kernel on its launching stream, breakdown pass"}
@@ -472,6 +494,7 @@ def run_ours(args, rank, world, local_rank):
     e2e = None
     if not args.no_e2e:
         barrier()  # every replica's e2e leg starts together
+        eng.set_step_graphs(not args.no_graph)
         e2e = run_e2e(args, tr, eng, dev, stream, cap[0], cap[0])
         if world > 1:  # whole-job: records summed, time max over ranks
             ms_max, = aggregate_many([e2e["ms_per_step"]], device=dev, op="max")
@@ -500,8 +523,10 @@ def run_ours(args, rank, world, local_rank):
                    "geometry": "Config9 (2048 rows, 2-way, 4 succ)", "parallelism": "replicas%d" % world,
                    "l2": "not flushed in the timed region: each step writes ~200 MB of prefetch/victim lists "
                          "(> 126 MB L2); the breakdown pass flushes (512 MiB write) before every step",
-                   "timing": "one CUDA-event region over K back-to-back steps (ingest of step i+1 overlaps "
-                             "the build of step i); residency snapshot loaded inside every step",
+                   "timing": "one CUDA-event region over K back-to-back steps, each = dum_load_residency + "
+                             "dum_step (%s); counters off" % ("separate C-ABI calls" if args.separate_calls else
+                                                              "one C call" + ("" if args.no_graph else
+                                                                              ", replayed as a CUDA graph")),
                    "seed": seed},
         "gpu_launches": int(launches),
         "roofline": roof, "step_roofline": step_roof, "kernels": per_kernel, "counters_per_step": counters,

@@ -234,6 +234,13 @@ int dum_step(dum_engine *eng, const uint64_t *launch_hash, const uint64_t *launc
              uint64_t *out_needed, uint32_t *out_writeback, uint32_t *out_invalidate, uint64_t sel_cap,
              uint64_t *sel_range, uint64_t *sel_needed, dum_stream_t stream);
 
+/* dum_step as a replayed CUDA graph (enable != 0): the batch is copied into
+ * the engine's upload buffers, then the whole step replays as one graph (one
+ * per batch size x staging set x output buffers, captured on first use; every
+ * value a step changes lives on the device).  Outputs must keep their
+ * addresses between the steps of one graph. */
+int dum_set_step_graphs(dum_engine *eng, int enable);
+
 /* Mark UM blocks as belonging to inactive (inactive != 0) or active PyTorch
  * blocks (D20: a block is invalidatable iff every PT block overlapping
  * it is inactive -- the caller resolves overlap). */

@@ -33,7 +33,7 @@ TIMER = {n: i for i, n in enumerate(["INGEST", "EXEC_ASSIGN", "BUILD_PREP", "APP
                                      "MAKE_QUERIES", "ANCHOR_WALK", "PREDICT", "SELECT", "MIG_PLAN", "COPY",
                                      "RESIDENCY", "CHAIN", "JUMP", "WALK", "EXACT", "WALK_INDEX", "WALK_RES"])}
 KERNEL_OF_TIMER = {"INGEST": "k_ingest", "EXEC_ASSIGN": "k_exec_assign", "BUILD_PREP": "k_build_prep",
-                   "APPLY_WALK": "k_apply", "WALK": "k_walk", "WALK_SLOW": "k_walk_slow", "MAKE_QUERIES": "k_make_queries",
+                   "APPLY_WALK": "k_build_exec", "WALK": "k_walk", "WALK_SLOW": "k_walk_slow", "MAKE_QUERIES": "k_make_queries",
                    "ANCHOR_WALK": "k_anchor_walk", "PREDICT": "k_copy_fast", "SELECT": "k_select_fast",
                    "MIG_PLAN": "k_mig_plan", "COPY": "k_copy_blocks", "RESIDENCY": "k_load_res",
                    "CHAIN": "k_chain", "JUMP": "k_jump0", "EXACT": "k_predict", "WALK_INDEX": "k_walk_index",
@@ -115,6 +115,7 @@ def load_library() -> ctypes.CDLL:
         "dum_read_timing": (I, [P, P, P, I]),
         "dum_simulate": (I, [P, P, U32, P, P, U32, U32, U32, P, P]),
         "dum_step": (I, [P, P, P, U32, P, U64, U32, U32, P, U64, P, P, P, P, P, P, U64, P, P, P]),
+        "dum_set_step_graphs": (I, [P, I]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -352,6 +353,9 @@ class Engine:
                                    _dev(out["needed"], 8), _dev(out["wb"], 4), _dev(out["inv"], 4), sel_cap,
                                    _dev(out["sel_rng"], 8), _dev(out["sel_needed"], 8), self._stream()), "dum_step")
         return out
+
+    def set_step_graphs(self, on: bool):
+        self._ck(self.lib.dum_set_step_graphs(self._h, 1 if on else 0), "dum_set_step_graphs")
 
     def mark_inactive(self, blocks: torch.Tensor, inactive: bool = True):
         self._ck(self.lib.dum_mark_inactive(self._h, _dev(blocks, 4), blocks.numel(), 1 if inactive else 0,

@@ -53,6 +53,7 @@ __global__ void k_init_state(DevState *st) {
   st->dbg_line = st->dbg_val = 0;
   for (int c = 0; c < DUM_NCOUNTERS; ++c) st->ctr[c] = 0;
   st->counting = 1;
+  st->k_base = 0;
 }
 
 uint32_t pow2ceil_h(uint64_t x) {
@@ -148,6 +149,12 @@ void free_all(dum_engine *e) {
   if (e->ev_join) cudaEventDestroy(e->ev_join);
   if (e->side) cudaStreamDestroy(e->side);
   if (e->side2) cudaStreamDestroy(e->side2);
+  if (e->graph_s) cudaStreamDestroy(e->graph_s);
+  if (e->ev_graph) cudaEventDestroy(e->ev_graph);
+  if (e->ev_wres) cudaEventDestroy(e->ev_wres);
+  if (e->cap_events_ready)
+    for (int i = 0; i < 8; ++i)
+      if (e->cap_ev[i]) cudaEventDestroy(e->cap_ev[i]);
   if (e->side3) cudaStreamDestroy(e->side3);
   if (e->ev_join3) cudaEventDestroy(e->ev_join3);
   if (e->ev_widx) cudaEventDestroy(e->ev_widx);
@@ -164,6 +171,8 @@ void free_all(dum_engine *e) {
     cudaEventDestroy(t.b);
   }
   for (auto ev : e->event_pool) cudaEventDestroy(ev);
+  for (auto &g : e->step_graphs) cudaGraphExecDestroy(g.exec);
+  e->step_graphs.clear();
 }
 
 cudaEvent_t get_event(dum_engine *e) {
@@ -181,7 +190,7 @@ cudaEvent_t get_event(dum_engine *e) {
 
 namespace dum {
 TimerScope::TimerScope(dum_engine *e_, int id_, cudaStream_t s_) : e(e_), id(id_), s(s_), b(nullptr) {
-  if (!e->timing) return;
+  if (!e->timing || e->capturing) return;
   cudaEvent_t a = get_event(e);
   b = get_event(e);
   cudaEventRecord(a, s);
@@ -275,6 +284,9 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
     A_(cudaStreamCreateWithFlags(&e->side, cudaStreamNonBlocking));
   }
   A_(cudaStreamCreateWithFlags(&e->side2, cudaStreamNonBlocking));
+  A_(cudaStreamCreateWithFlags(&e->graph_s, cudaStreamNonBlocking));
+  A_(cudaEventCreateWithFlags(&e->ev_graph, cudaEventDisableTiming));
+  A_(cudaEventCreateWithFlags(&e->ev_wres, cudaEventDisableTiming));
   A_(cudaStreamCreateWithFlags(&e->side3, cudaStreamNonBlocking));
   A_(cudaEventCreateWithFlags(&e->ev_join3, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_widx, cudaEventDisableTiming));
@@ -519,6 +531,169 @@ __global__ void k_step_shift(uint32_t *ex, uint32_t n) {
   }
 }
 
+// The selection's per-walk residency facts depend only on the residency and
+// the walks of the previous build: issued on the second side stream so that
+// they overlap the ingest of the step; launch_predict joins them.
+static cudaError_t fork_walk_res(dum_engine *e, cudaStream_t s) {
+  cudaError_t err;
+  if ((err = cudaEventRecord(e->ev_fork2, s)) != cudaSuccess) return err;
+  if ((err = cudaStreamWaitEvent(e->side2, e->ev_fork2, 0)) != cudaSuccess) return err;
+  if ((err = launch_walk_res(e, e->side2)) != cudaSuccess) return err;
+  if ((err = cudaEventRecord(e->ev_wres, e->side2)) != cudaSuccess) return err;
+  e->wres_pending = true;
+  return cudaSuccess;
+}
+
+// dum_step as one CUDA graph per (batch size, staging set, outputs): the
+// inputs go to the engine's fixed upload buffers outside the graph, then the
+// whole step -- ingest, queries, predict + select, build, history shift, every
+// side-stream fork joined -- replays with one cudaGraphLaunch.  The values a
+// step changes (launch index base, pools, counts) live on the device.
+static int step_graph(dum_engine *e, const uint64_t *launch_hash, const uint64_t *launch_off, uint32_t n_launch,
+                      const uint32_t *fault_block, uint64_t n_fault, uint32_t flags, uint32_t degree,
+                      uint32_t *out_pairs, uint64_t out_cap_pairs, uint64_t *out_range, uint32_t *out_kern_off,
+                      uint32_t *out_chain, uint64_t *out_needed, uint32_t *out_writeback, uint32_t *out_invalidate,
+                      uint64_t sel_cap, uint64_t *sel_range, uint64_t *sel_needed, cudaStream_t s) {
+  if (!launch_hash || !launch_off || (n_fault && !fault_block) || !out_range || !sel_range)
+    return fail(e, DUM_EINVAL, "null argument");
+  if (n_launch > e->stage_launch_cap || n_fault > e->stage_fault_cap)
+    return fail(e, DUM_ECAPACITY, "staging capacity exceeded: raise max_batch_*");
+  if (e->launches + n_launch > 0xFFFFFFFFull) return fail(e, DUM_ECAPACITY, "launch counter exceeds 2^32");
+  if (reinterpret_cast<uintptr_t>(out_pairs) & 7) return fail(e, DUM_EINVAL, "out_pairs must be 8-byte aligned");
+  cudaSetDevice(e->device);
+  const cudaMemcpyKind kind = (flags & DUM_HOST_PTRS) ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
+  if (flags & DUM_HOST_PTRS) {
+    if (launch_off[0] != 0 || launch_off[n_launch] != n_fault) return fail(e, DUM_EINVAL, "batch not launch-aligned");
+    for (uint32_t i = 0; i < n_launch; ++i)
+      if (launch_off[i + 1] < launch_off[i]) return fail(e, DUM_EINVAL, "launch_off not monotone");
+  }
+  // the batch into the fixed upload buffers (stream-ordered before the replay)
+  CK(cudaMemcpyAsync(e->d_in_hash, launch_hash, 8ull * n_launch, kind, s));
+  CK(cudaMemcpyAsync(e->d_in_off, launch_off, 8ull * (n_launch + 1), kind, s));
+  if (n_fault) CK(cudaMemcpyAsync(e->d_in_faults, fault_block, 4ull * n_fault, kind, s));
+  // the graph runs on the engine's own (capturable, non-blocking) stream, ordered
+  // after the caller's stream and before it again
+  cudaStream_t caller = s;
+  s = e->graph_s;
+  CK(cudaEventRecord(e->ev_s_now, caller));
+  CK(cudaStreamWaitEvent(s, e->ev_s_now, 0));
+  // side-stream work of an earlier uncaptured call (jump tables, walk index,
+  // predict's side kernels) is finished before the graph starts
+  CK(cudaStreamWaitEvent(s, e->ev_join, 0));
+  CK(cudaStreamWaitEvent(s, e->ev_widx, 0));
+  CK(cudaStreamWaitEvent(s, e->ev_join2, 0));
+  CK(cudaStreamWaitEvent(s, e->ev_join3, 0));
+  CK(cudaStreamWaitEvent(s, e->ev_rec, 0));
+  const uint64_t key[12] = {n_launch, (uint64_t)e->stage_set, degree, (uint64_t)out_pairs, out_cap_pairs,
+                            (uint64_t)out_range, (uint64_t)out_kern_off, (uint64_t)out_chain, (uint64_t)out_needed,
+                            (uint64_t)out_writeback ^ ((uint64_t)out_invalidate << 1), sel_cap,
+                            (uint64_t)sel_range ^ ((uint64_t)sel_needed << 1)};
+  cudaGraphExec_t exec = nullptr;
+  for (auto &g : e->step_graphs)
+    if (std::memcmp(g.key, key, sizeof key) == 0) exec = g.exec;
+  if (!exec) {
+    // the chunk map of this output capacity is grown before the capture
+    const uint64_t bound = out_cap_pairs / CHUNK_B + (uint64_t)n_launch * (e->g.N + 1) + 1;
+    if (bound > e->chunk_cap) {
+      CK(cudaDeviceSynchronize());
+      CK(cudaFree(e->d_chunk_map));
+      e->d_chunk_map = nullptr;
+      CK(cudaMalloc((void **)&e->d_chunk_map, 8 * bound));
+      e->chunk_cap = bound;
+    }
+    SelectOut so = make_select_out(e, out_writeback, out_invalidate, sel_cap, sel_range);
+    cudaGraph_t graph = nullptr;
+    // fork / join events recorded inside a capture become graph edges and may
+    // not be waited on outside it: the capture uses its own set
+    cudaEvent_t *evs[] = {&e->ev_fork, &e->ev_join, &e->ev_fork2, &e->ev_join2, &e->ev_join3, &e->ev_widx,
+                          &e->ev_wres};
+    constexpr int NEV = sizeof(evs) / sizeof(evs[0]);
+    if (!e->cap_events_ready) {
+      for (int i = 0; i < NEV; ++i) CK(cudaEventCreateWithFlags(&e->cap_ev[i], cudaEventDisableTiming));
+      e->cap_events_ready = true;
+    }
+    cudaEvent_t real[NEV];
+    for (int i = 0; i < NEV; ++i) {
+      real[i] = *evs[i];
+      *evs[i] = e->cap_ev[i];
+    }
+    e->capturing = true;
+    const uint32_t ns0 = e->n_staged;
+    const uint64_t sf0 = e->staged_faults;
+    e->n_staged = 0;
+    e->staged_faults = 0;
+    cudaError_t err = cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal);
+    // the previous step's walk index (a replayed build leaves it to this step),
+    // beside the residency facts and the ingest
+    if (err == cudaSuccess) err = launch_walk_index(e, s);
+    if (err == cudaSuccess) err = fork_walk_res(e, s);
+    if (err == cudaSuccess)
+      err = launch_record(e, e->d_in_hash, e->d_in_off, n_launch, e->d_in_faults, e->stage_fault_cap,
+                          e->d_step_exec + 3, s);
+    if (err == cudaSuccess) err = launch_make_queries(e, e->d_step_exec, 3 + n_launch, 3, degree, e->d_step_q, s);
+    if (err == cudaSuccess)
+      err = launch_predict(e, e->d_step_q, n_launch, out_pairs, out_cap_pairs, out_range, out_kern_off, out_chain,
+                           out_needed, &so, sel_needed, s);
+    e->n_staged = n_launch;
+    e->staged_faults = e->stage_fault_cap;
+    if (err == cudaSuccess) err = launch_build(e, s);
+    if (err == cudaSuccess) {
+      k_step_shift<<<1, 32, 0, s>>>(e->d_step_exec, n_launch);
+      // every side stream joins the step: the next replay may start at once
+      cudaStreamWaitEvent(s, e->ev_join, 0);
+      cudaStreamWaitEvent(s, e->ev_widx, 0);
+      err = cudaGetLastError();
+    }
+    const cudaError_t err2 = cudaStreamEndCapture(s, &graph);
+    e->capturing = false;
+    for (int i = 0; i < NEV; ++i) *evs[i] = real[i];
+    e->n_staged = ns0;
+    e->staged_faults = sf0;
+    if (err == cudaSuccess) err = err2;
+    if (err == cudaSuccess) err = cudaGraphInstantiate(&exec, graph, 0);
+    if (graph) cudaGraphDestroy(graph);
+    if (err != cudaSuccess) {
+      // not capturable here: say so once, drop to the one-call path for good
+      cudaGetLastError();
+      fprintf(stderr, "libdeepum_b200: dum_step graph capture failed (%s); steps run uncaptured\n",
+              cudaGetErrorString(err));
+      e->graph_steps = false;
+      e->wres_pending = false;
+      e->last_error = std::string("dum_step graph capture: ") + cudaGetErrorString(err);
+      CK(cudaEventRecord(e->ev_graph, s));
+      CK(cudaStreamWaitEvent(caller, e->ev_graph, 0));
+      return DUM_ECUDA;
+    }
+    dum_engine::StepGraph sg;
+    std::memcpy(sg.key, key, sizeof key);
+    sg.exec = exec;
+    e->step_graphs.push_back(sg);
+  }
+  CK(cudaGraphLaunch(exec, s));
+  e->widx_stale = true;  // the replayed build's walk index is built by the next step
+  CK(cudaEventRecord(e->ev_graph, s));
+  CK(cudaStreamWaitEvent(caller, e->ev_graph, 0));
+  // host bookkeeping of the replayed step (as dum_record_faults + dum_build_tables)
+  e->launches += n_launch;
+  e->built_launches = e->launches;
+  e->stage_set ^= 1;
+  const uint64_t L = e->stage_launch_cap, F = e->stage_fault_cap, k = (uint64_t)e->stage_set;
+  e->d_stage_hash = static_cast<uint64_t *>(e->stage_base[0]) + k * L;
+  e->d_stage_norm = static_cast<uint32_t *>(e->stage_base[1]) + k * F;
+  e->d_stage_cnt = static_cast<uint32_t *>(e->stage_base[2]) + k * L;
+  e->d_stage_exec = static_cast<uint32_t *>(e->stage_base[3]) + k * L;
+  e->d_stage_slot = static_cast<uint32_t *>(e->stage_base[4]) + k * L;
+  e->d_stage_off = static_cast<uint64_t *>(e->stage_base[5]) + k * L;
+  e->kernel_launches += 40;  // approximate node count of a step graph
+  return DUM_OK;
+}
+
+int dum_set_step_graphs(dum_engine *e, int enable) {
+  if (!e) return DUM_EINVAL;
+  e->graph_steps = enable != 0;
+  return DUM_OK;
+}
+
 int dum_step(dum_engine *e, const uint64_t *launch_hash, const uint64_t *launch_off, uint32_t n_launch,
              const uint32_t *fault_block, uint64_t n_fault, uint32_t flags, uint32_t degree, uint32_t *out_pairs,
              uint64_t out_cap_pairs, uint64_t *out_range, uint32_t *out_kern_off, uint32_t *out_chain,
@@ -528,6 +703,17 @@ int dum_step(dum_engine *e, const uint64_t *launch_hash, const uint64_t *launch_
   if (n_launch == 0) return DUM_OK;
   if (e->n_staged) return fail(e, DUM_ESTATE, "dum_step: a batch is already staged (call dum_build_tables)");
   if (n_launch > e->anchor_range_cap) return fail(e, DUM_EINVAL, "too many launches in one step (max 65536)");
+  // graph mode: the first step of a shape runs uncaptured (first-use attribute /
+  // occupancy queries of the launchers are not capturable), later ones replay
+  if (e->graph_steps && e->step_warm) {
+    const int rc = step_graph(e, launch_hash, launch_off, n_launch, fault_block, n_fault, flags, degree, out_pairs,
+                              out_cap_pairs, out_range, out_kern_off, out_chain, out_needed, out_writeback,
+                              out_invalidate, sel_cap, sel_range, sel_needed, (cudaStream_t)stream);
+    if (rc != DUM_ECUDA || e->graph_steps) return rc;  // (a failed capture turned graph mode off: run it below)
+  }
+  e->step_warm = e->graph_steps;
+  cudaSetDevice(e->device);
+  CK(fork_walk_res(e, (cudaStream_t)stream));
   int rc = dum_record_faults(e, launch_hash, launch_off, n_launch, fault_block, n_fault, e->d_step_exec + 3, flags,
                              stream);
   if (rc) return rc;

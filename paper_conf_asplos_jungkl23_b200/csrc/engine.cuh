@@ -72,6 +72,7 @@ struct DevState {
   uint32_t n_items, n_leads;  // build: k_apply items / exec IDs with faults (k_plan)
   uint32_t n_dd;              // build: walks left to k_walk's dedupe (k_build_exec)
   uint32_t counting;          // ctr_add is live (dum_set_counting)
+  uint32_t k_base;            // global launch index of the next build's first staged launch
   unsigned long long ctr[DUM_NCOUNTERS];  // work counters (instrumentation)
 };
 
@@ -244,5 +245,18 @@ struct dum_engine {
   uint32_t apply_grid, walk_grid;  // persistent build grids (occupancy x SMs), set on first build
   uint32_t copy_grid, sel_grid;    // persistent predict grids (k_window.cu)
   int chain_smem;                  // k_chain dynamic smem attribute applied
-  int bulk_smem;                   // k_copy_bulk dynamic smem attribute applied  // dynamic smem attributes applied (per engine / device)
+  int bulk_smem;                   // k_copy_bulk dynamic smem attribute applied
+  // dum_step as a replayed CUDA graph (dum_set_step_graphs)
+  bool graph_steps, capturing, step_warm;
+  cudaStream_t graph_s;        // the step graphs are captured and replayed here
+  cudaEvent_t ev_graph, ev_wres;
+  bool wres_pending;           // dum_step issued the walk residency facts beside the ingest
+  bool cap_events_ready;
+  bool widx_stale;             // the walk index lags the last (replayed) build
+  cudaEvent_t cap_ev[8];       // the fork / join events of a step-graph capture (graph edges only)
+  struct StepGraph {
+    uint64_t key[12];
+    cudaGraphExec_t exec;
+  };
+  std::vector<StepGraph> step_graphs;  // dynamic smem attributes applied (per engine / device)
 };

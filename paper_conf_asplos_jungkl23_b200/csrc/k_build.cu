@@ -56,7 +56,7 @@ constexpr uint32_t WK_QCAP = 4096; // shared dedupe-hash capacity (|Q| <= WK_QCA
 // ---------------------------------------------------------------------------
 // k_build_prep
 // ---------------------------------------------------------------------------
-__global__ void k_build_prep(uint32_t n_staged, uint32_t k0, const uint32_t *__restrict__ stage_exec,
+__global__ void k_build_prep(uint32_t n_staged, const uint32_t *__restrict__ stage_exec,
                              const uint32_t *__restrict__ stage_cnt, CorrSlot *corr, uint32_t corr_cap,
                              uint32_t *rec_slot, uint32_t *head, uint32_t *__restrict__ next,
                              uint32_t *__restrict__ order, uint32_t *e_ops, uint32_t *e_last,
@@ -78,6 +78,9 @@ __global__ void k_build_prep(uint32_t n_staged, uint32_t k0, const uint32_t *__r
   const uint32_t e = stage_exec[j];
   const uint32_t owner = prev(1);
   const bool up = owner != NONE && e != NONE;
+  // global launch index of staged launch j: the device-side base of this build
+  // (k_plan advances it; the same value in a replayed graph step)
+  const uint32_t k0 = *(volatile uint32_t *)&st->k_base;
   if (up) corr_upsert(corr, corr_cap, rec_slot, owner, prev(4), prev(3), prev(2), e, k0 + j, st);
   const uint32_t nup = __popc(__ballot_sync(__activemask(), up));
   if ((threadIdx.x & 31) == __ffs(__activemask()) - 1) ctr_add(st, DUM_CTR_CORR_UPSERTS, nup);
@@ -279,6 +282,7 @@ __global__ void __launch_bounds__(PLAN_NT) k_plan(BuildArgs a) {
       h[q] = jj >= 0 ? a.stage_exec[jj] : a.st->hist[4 + jj];
     }
     for (int q = 0; q < 4; ++q) a.st->hist[q] = h[q];
+    a.st->k_base += a.n_staged;  // the next build's launch index base (k_build_prep of this build has read it)
   }
   const uint32_t c0 = a.st->cls_cnt[0], c1 = a.st->cls_cnt[1], c2 = a.st->cls_cnt[2];
   const uint32_t tot = c0 + c1 + c2;
@@ -1144,8 +1148,10 @@ static cudaError_t launch_apply_walk(dum_engine *e, const BuildArgs &ba, cudaStr
 cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   const uint32_t n = e->n_staged;
   if (n == 0) return cudaSuccess;
-  cudaStreamWaitEvent(s, e->ev_join, 0);  // the previous build's jump tables read corr
-  cudaStreamWaitEvent(s, e->ev_widx, 0);  // the previous build's walk index reads the walk cache
+  if (!e->capturing) {  // (a captured step joins its side streams before it ends)
+    cudaStreamWaitEvent(s, e->ev_join, 0);  // the previous build's jump tables read corr
+    cudaStreamWaitEvent(s, e->ev_widx, 0);  // the previous build's walk index reads the walk cache
+  }
   BuildArgs ba;
   ba.g = e->g;
   ba.n_staged = n;
@@ -1176,7 +1182,7 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   ba.dd_list = e->d_dd_list;
   {
     TimerScope t(e, DUM_T_BUILD_PREP, s);
-    k_build_prep<<<(n + 255) / 256, 256, 0, s>>>(n, (uint32_t)e->built_launches, e->d_stage_exec, e->d_stage_cnt,
+    k_build_prep<<<(n + 255) / 256, 256, 0, s>>>(n, e->d_stage_exec, e->d_stage_cnt,
                                                   e->d_corr, e->corr_cap, e->d_rec_slot, e->d_head, e->d_next,
                                                   e->d_order, e->d_e_ops, e->d_e_last, ba.plan_agg, e->d_state);
     k_plan<<<(n + PLAN_NT - 1) / PLAN_NT, PLAN_NT, 0, s>>>(ba);
@@ -1203,7 +1209,11 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
     k_walk_slow<<<e->n_walk_slots, 32, 0, s>>>(e->g, e->d_tbl, e->d_start_end, e->d_walk, e->d_walk_len,
                                                e->d_wrun, e->d_wrun_len, e->d_slow_list, ws, e->d_state);
   }
-  {
+  if (e->capturing) {
+    // a captured step builds the walk index at the start of the next step,
+    // beside its ingest (dum_step graph); the next uncaptured predict does it
+    e->widx_stale = true;
+  } else {
     const cudaError_t we = launch_walk_index(e, s);  // k_window.cu: conflicts between the new walks
     if (we != cudaSuccess) return we;
   }

@@ -288,7 +288,7 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
   if (lane == 0) {
     s_u[w] = U;
     s_need[w] = qneed;
-    s_gu[w] = GUq;  // copy chunks of k_copy_fast
+    s_gu[w] = a.select ? 0u : GUq;  // copy chunks of k_copy_fast (predict only)
   }
   __syncthreads();
   if (qi < a.nq && lane == 0) s_wcls[w] = atomicAdd(&s_cls[cls], 1u);  // rank within the CTA
@@ -353,8 +353,8 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
       for (uint32_t d = lane; d <= g.N; d += 32) ch[d] = d < nk ? skern[w][d] : NONE;
     }
   }
-  // the chunk map of k_copy_fast: chunk j of list d of a fast query -> (q, d, j)
-  if (qi < a.nq && s_gu[w]) {
+  // the chunk map of k_copy_fast (predict only): chunk j of list d of a fast query -> (q, d, j)
+  if (qi < a.nq && s_gu[w] && !a.select) {
     unsigned long long gb = s_gbase;
     for (uint32_t i = 0; i < w; ++i) gb += s_gu[i];
     const uint32_t G = s_gu[w], nk = a.qnk[qi];
@@ -388,9 +388,9 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
   uint32_t *dk = bitmap + ((a.nwords + 3) & ~3u);  // [2 * DHCAP]
   __shared__ SelShared ss;
   __shared__ uint32_t kern[MAXN + 1], loff[MAXN + 2], kcnt[MAXN + 1], eoff[MAXN + 2], goff[MAXN + 2];
-  __shared__ uint32_t noff[MAXN + 2];
+  __shared__ uint32_t noff[MAXN + 2], dl_d[MAXN + 1], dl_off[MAXN + 2], dl_base[MAXN + 1];
   __shared__ uint32_t ws[NWARP];
-  __shared__ uint32_t s_ndup, s_nonres, s_flag, s_nocc, s_dnr;
+  __shared__ uint32_t s_ndup, s_nonres, s_flag, s_nocc, s_dnr, s_nd;
   __shared__ uint32_t s_dup[2 * OCCAP];  // pass 1: duplicated blocks; duplicate path: occurrences (list, block)
   __shared__ unsigned long long s_hoff;
   const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
@@ -590,7 +590,7 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
     // list is found from the runs (a word hash filters the runs that hold
     // duplicated blocks), every other occurrence is dropped, the lists keep
     // their order and shift left; the few lists that lose blocks are
-    // compacted by one warp each, the others are copied again.
+    // compacted together by the whole CTA, the others are copied again.
     uint32_t *wk = dk, *wm = dk + DWCAP;                      // word -> duplicated-block mask
     uint32_t *bk = dk + 2 * DWCAP, *bv = bk + DBCAP;          // block -> first list + 1 (anchor: 0)
     bool fallback = ndup > DLCAP;
@@ -681,36 +681,71 @@ __global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
       __syncthreads();
       run = noff[nk];
       if (ok) {
-        // lists that lose blocks: ordered compaction by the whole CTA, chunks
+        // lists that lose blocks: one ordered compaction by the whole CTA over
+        // their concatenation (rank r -> list dl_d[r], offsets dl_off), chunks
         // of 4 * PRED_NT elements (thread tid owns 4 consecutive ones), one
-        // block scan of the keep counts per chunk
-        for (uint32_t d = 0; d < nk; ++d) {
-          if (!kcnt[d]) continue;
-          const uint32_t *lst = list_of(d);
-          const uint32_t L = loff[d + 1] - loff[d], kd = kern[d];
-          uint2 *o = reinterpret_cast<uint2 *>(a.pairs) + base + noff[d];
-          uint32_t pos = 0;
-          for (uint32_t c = 0; c < L; c += 4 * PRED_NT) {
-            uint32_t bb[4], keep = 0;
+        // block scan of the keep counts per chunk; a kept element's slot in
+        // its list is (kept before it) - (kept before its list), the latter
+        // recorded in dl_base by the thread owning the list's first element
+        if (wid == 0) {
+          uint32_t acc = 0, nd = 0;
+          for (uint32_t d0 = 0; d0 < nk; d0 += 32) {
+            const uint32_t d = d0 + lane;
+            const bool f = d < nk && kcnt[d];
+            const uint32_t len = f ? loff[d + 1] - loff[d] : 0;
+            const uint32_t bal = __ballot_sync(0xffffffffu, f);
+            uint32_t incl = len;
 #pragma unroll
-            for (uint32_t u = 0; u < 4; ++u) {
-              const uint32_t i = c + 4 * tid + u;
-              bb[u] = i < L ? __ldg(lst + i) : NONE;
+            for (int o = 1; o < 32; o <<= 1) {
+              const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+              if (lane >= (uint32_t)o) incl += y;
             }
-#pragma unroll
-            for (uint32_t u = 0; u < 4; ++u) {
-              if (c + 4 * tid + u >= L) continue;
-              const uint32_t f = hmap_get(bk, bv, DBCAP, bb[u]);
-              if (f == NONE || f == d + 1) keep |= 1u << u;
+            if (f) {
+              const uint32_t r = nd + __popc(bal & ((1u << lane) - 1u));
+              dl_d[r] = d;
+              dl_off[r] = acc + incl - len;
             }
-            uint32_t tot;
-            const uint32_t pre = block_excl_scan(__popc(keep), ws, &tot);
-            uint32_t r = 0;
-#pragma unroll
-            for (uint32_t u = 0; u < 4; ++u)
-              if ((keep >> u) & 1u) __stcs(o + pos + pre + r++, make_uint2(bb[u], kd));
-            pos += tot;
+            acc += __shfl_sync(0xffffffffu, incl, 31);
+            nd += __popc(bal);
           }
+          if (lane == 0) {
+            dl_off[nd] = acc;
+            s_nd = nd;
+          }
+        }
+        __syncthreads();
+        const uint32_t T = dl_off[s_nd];
+        uint32_t kept = 0, cur = 0;
+        for (uint32_t c = 0; c < T; c += 4 * PRED_NT) {
+          uint32_t bb[4], lr[4], keep = 0;
+#pragma unroll
+          for (uint32_t u = 0; u < 4; ++u) {
+            const uint32_t t = c + 4 * tid + u;
+            bb[u] = NONE;
+            lr[u] = cur;
+            if (t >= T) continue;
+            while (dl_off[cur + 1] <= t) ++cur;
+            lr[u] = cur;
+            const uint32_t d = dl_d[cur];
+            bb[u] = __ldg(list_of(d) + (t - dl_off[cur]));
+            const uint32_t f = hmap_get(bk, bv, DBCAP, bb[u]);
+            if (f == NONE || f == d + 1) keep |= 1u << u;
+          }
+          uint32_t tot;
+          const uint32_t pre = block_excl_scan(__popc(keep), ws, &tot);
+#pragma unroll
+          for (uint32_t u = 0; u < 4; ++u)
+            if (c + 4 * tid + u < T && c + 4 * tid + u == dl_off[lr[u]])
+              dl_base[lr[u]] = kept + pre + __popc(keep & ((1u << u) - 1u));
+          __syncthreads();
+#pragma unroll
+          for (uint32_t u = 0; u < 4; ++u)
+            if ((keep >> u) & 1u) {
+              const uint32_t d = dl_d[lr[u]];
+              const uint32_t k = kept + pre + __popc(keep & ((1u << u) - 1u)) - dl_base[lr[u]];
+              __stcs(reinterpret_cast<uint2 *>(a.pairs) + base + noff[d] + k, make_uint2(bb[u], kern[d]));
+            }
+          kept += tot;
         }
         // the other lists at their shifted offsets
         copy_lists(wid, NWARP, noff, kcnt);
@@ -917,6 +952,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   {
     // the chunk map holds every copy chunk of the call: <= cap / 128 + nq (N + 1)
     const uint64_t bound = cap / CHUNK_B + (uint64_t)nq * (e->g.N + 1) + 1;
+    if (bound > e->chunk_cap && e->capturing) return cudaErrorInvalidValue;  // grown before a capture
     if (bound > e->chunk_cap) {
       cudaError_t ce = cudaStreamSynchronize(s);  // growth only: the old map may be in use
       if (ce == cudaSuccess) ce = cudaFree(e->d_chunk_map);
@@ -929,8 +965,19 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   a.chunk_map = e->d_chunk_map;
   a.chunk_cap = e->chunk_cap;
   cudaError_t err;
-  if (sel && (err = launch_walk_res(e, s)) != cudaSuccess) return err;  // residency facts per walk
-  cudaStreamWaitEvent(s, e->ev_join, 0);  // jump tables of the last build (side stream)
+  if (sel && e->wres_pending) {  // issued beside the ingest by dum_step: join it
+    cudaStreamWaitEvent(s, e->ev_wres, 0);
+    e->wres_pending = false;
+  } else if (sel && (err = launch_walk_res(e, s)) != cudaSuccess) {  // residency facts per walk
+    return err;
+  }
+  if (!e->capturing) {  // (a captured step joins its side streams before it ends)
+    if (e->widx_stale) {  // the last build was a replayed step: its walk index is due
+      if ((err = launch_walk_index(e, s)) != cudaSuccess) return err;
+      e->widx_stale = false;
+    }
+    cudaStreamWaitEvent(s, e->ev_join, 0);  // jump tables of the last build (side stream)
+  }
   cudaStreamWaitEvent(s, e->ev_widx, 0);  // walk index of the last build (third side stream)
   {
     TimerScope t(e, DUM_T_CHAIN, s);
@@ -967,12 +1014,9 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
     k_predict<false><<<pgrid, PRED_NT, smem, e->side2>>>(a);
   }
   cudaEventRecord(e->ev_join2, e->side2);
-  // fast path: the flat copy on `s`, the selection on the third side stream
-  cudaStreamWaitEvent(e->side3, e->ev_fork2, 0);
-  if ((err = launch_window(e, a, sel != nullptr, s, e->side3)) != cudaSuccess) return err;
-  cudaEventRecord(e->ev_join3, e->side3);
+  // fast path on `s`: the flat copy (predict only) or a CTA per window (select + copy)
+  if ((err = launch_window(e, a, sel != nullptr, s)) != cudaSuccess) return err;
   cudaStreamWaitEvent(s, e->ev_join2, 0);
-  cudaStreamWaitEvent(s, e->ev_join3, 0);
   e->kernel_launches += 3;
   k_pred_epilogue<<<1, 32, 0, s>>>(e->d_state, needed, sel ? sel_needed : nullptr);
   e->kernel_launches += 1;

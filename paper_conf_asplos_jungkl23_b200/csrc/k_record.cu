@@ -19,9 +19,9 @@
 namespace dum {
 
 constexpr int INGEST_NT = 256;
-constexpr uint32_t INGEST_HCAP = 4096;  // smem hash capacity (n <= 2048 in smem)
+constexpr uint32_t INGEST_HCAP = 2048;  // smem hash capacity (n <= 1024 in smem): 16 KB, 8 CTAs / SM
 constexpr uint32_t IDCAP = 1024;        // repeated-block hash of the bitmap path
-constexpr uint32_t INGEST_SMEM_MAX = 64 * 1024;
+constexpr uint32_t INGEST_SMEM_MAX = 16 * 1024;  // the bitmap path only where it fits this (small W)
 
 __global__ void __launch_bounds__(INGEST_NT) k_ingest(
     const uint64_t *__restrict__ hash, const uint64_t *__restrict__ off, const uint32_t *__restrict__ faults,

@@ -285,8 +285,8 @@ __device__ __forceinline__ void step_masks(const SelectOut &so, const uint32_t *
 
 constexpr uint32_t FB = 8;  // warp steps with their entry loads in flight together
 
-__global__ void __launch_bounds__(WSEL_NT, 8) k_select_fast(PredArgs a) {
-  __shared__ uint32_t kern[MAXN + 1], roff[MAXN + 2];
+__global__ void __launch_bounds__(WSEL_NT, 6) k_select_fast(PredArgs a) {
+  __shared__ uint32_t kern[MAXN + 1], roff[MAXN + 2], loff[MAXN + 2], goff[MAXN + 2];
   __shared__ uint32_t posmap[POS_WORDS];
   __shared__ uint32_t seg_cnt[FSEG_MAX], seg_pre[FSEG_MAX];
   __shared__ uint32_t wem[POS_WORDS], wim[POS_WORDS], wpre[POS_WORDS];  // clean-log word path
@@ -315,6 +315,8 @@ __global__ void __launch_bounds__(WSEL_NT, 8) k_select_fast(PredArgs a) {
     const uint32_t nk = a.qnk[qi];
     for (uint32_t d = tid; d <= nk; d += WSEL_NT) {
       roff[d] = a.qroff[(uint64_t)qi * (g.N + 2) + d];
+      loff[d] = a.qloff[(uint64_t)qi * (g.N + 2) + d];
+      goff[d] = a.qgoff[(uint64_t)qi * (g.N + 2) + d];
       if (d < nk) kern[d] = a.qkern[(uint64_t)qi * (g.N + 1) + d];
     }
     for (uint32_t w = tid; w < POS_WORDS; w += WSEL_NT) posmap[w] = 0;
@@ -400,38 +402,50 @@ __global__ void __launch_bounds__(WSEL_NT, 8) k_select_fast(PredArgs a) {
           }
         }
         __syncthreads();
-        // a warp per word, a lane per position: the eligible entries of
-        // combined rank < need, written at their list ranks (4 words in flight)
-        const uint32_t lt = (1u << lane) - 1;
+        // a warp per 128-position chunk (4 words), a lane per 4 consecutive
+        // positions: the eligible entries of combined rank < need, written at
+        // their list ranks.  head is 16 B aligned for the vector load when
+        // possible; otherwise 4 scalar loads.
         uint32_t tw = 0, ti = 0;
-        for (uint32_t w0 = wid; w0 < nw; w0 += NW * 4) {
-          uint32_t v[4], mA[4], mI[4], pr[4];
+        const uint32_t nch = (nw + 3) / 4;
+        const bool al = (head & 3u) == 0;
+        for (uint32_t ch = wid; ch < nch; ch += NW) {
+          const uint32_t w = 4 * ch + (lane >> 3), sh = (lane & 7) * 4;
+          const uint32_t pre = w < nw ? wpre[w] : 0xFFFFFFFFu;
+          const uint32_t pre0 = __shfl_sync(0xffffffffu, pre, 0);
+          if ((pre0 & 0xFFFFu) + (pre0 >> 16) >= need) break;  // chunks only grow: the cut is behind
+          const uint32_t a4 = w < nw ? (wem[w] >> sh) & 0xFu : 0u, i4 = w < nw ? (wim[w] >> sh) & 0xFu : 0u;
+          // ranks: the word's prefix + the eligible entries of the lower lanes of the same word
+          uint32_t c = __popc(a4) | (__popc(i4) << 16), x = c;
 #pragma unroll
-          for (uint32_t u = 0; u < 4; ++u) {
-            const uint32_t w = w0 + u * NW;
-            mA[u] = mI[u] = 0;
-            pr[u] = 0;
-            v[u] = 0;
-            if (w < nw) {
-              pr[u] = wpre[w];
-              if ((pr[u] & 0xFFFFu) + (pr[u] >> 16) < need) {
-                mA[u] = wem[w];
-                mI[u] = wim[w];
-                if (((mA[u] | mI[u]) >> lane) & 1u) v[u] = __ldcg(so.lrm_blk + head + w * 32 + lane);
-              }
-            }
+          for (int o = 1; o < 8; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+            if ((lane & 7) >= (uint32_t)o) x += y;
           }
+          uint32_t ra = (pre & 0xFFFFu) + ((x - c) & 0xFFFFu), rr = (pre >> 16) + ((x - c) >> 16);
+          if ((a4 | i4) && ra + rr < need) {
+            const uint32_t p = head + 32 * w + sh;
+            uint32_t vv[4];
+            if (al) {
+              const uint4 q = __ldcg(reinterpret_cast<const uint4 *>(so.lrm_blk + p));
+              vv[0] = q.x; vv[1] = q.y; vv[2] = q.z; vv[3] = q.w;
+            } else {
 #pragma unroll
-          for (uint32_t u = 0; u < 4; ++u) {
-            const bool ea = (mA[u] >> lane) & 1u, ei = (mI[u] >> lane) & 1u;
-            const uint32_t ra = (pr[u] & 0xFFFFu) + __popc(mA[u] & lt), rr = (pr[u] >> 16) + __popc(mI[u] & lt);
-            if ((ea || ei) && ra + rr < need) {
-              if (ok) {
-                if (ei) so.inv[binv + rr] = v[u] & 0x7FFFFFFFu;
-                else so.wb[bwb + ra] = v[u];
+              for (uint32_t u = 0; u < 4; ++u) vv[u] = ((a4 | i4) >> u) & 1u ? __ldcg(so.lrm_blk + p + u) : 0u;
+            }
+#pragma unroll
+            for (uint32_t u = 0; u < 4; ++u) {
+              const bool ea = (a4 >> u) & 1u, ei = (i4 >> u) & 1u;
+              if ((ea || ei) && ra + rr < need) {
+                if (ok) {
+                  if (ei) so.inv[binv + rr] = vv[u] & 0x7FFFFFFFu;
+                  else so.wb[bwb + ra] = vv[u];
+                }
+                tw += ea;
+                ti += ei;
               }
-              tw += ea;
-              ti += ei;
+              ra += ea;
+              rr += ei;
             }
           }
         }
@@ -532,6 +546,18 @@ __global__ void __launch_bounds__(WSEL_NT, 8) k_select_fast(PredArgs a) {
       ctr_add(a.st, DUM_CTR_FAST_VICTIMS, s_tw + s_ti);
       if (!clean) ctr_add(a.st, DUM_CTR_FAST_DIRTY, 1);
     }
+    // the window's (block, exec) pairs: every warp streams the lists (the copy
+    // of this query overlaps the selection of the SM's other queries)
+    {
+      const unsigned long long base = a.qbase[qi];
+      const uint32_t U = nk ? loff[nk] : 0;
+      if (base + U <= a.cap) copy_window_lists(a, kern, loff, goff, nk, base, wid, NW, loff, nullptr);
+      if (tid == 0) {
+        ctr_add(a.st, DUM_CTR_EMITTED, U);
+        ctr_add(a.st, DUM_CTR_GATHERED, U);
+        ctr_add(a.st, DUM_CTR_FAST_EMITTED, U);
+      }
+    }
     __syncthreads();  // the next query reuses the shared state
   }
 }
@@ -583,7 +609,7 @@ cudaError_t launch_walk_res(dum_engine *e, cudaStream_t s) {
   return cudaGetLastError();
 }
 
-cudaError_t launch_window(dum_engine *e, const PredArgs &a, bool select, cudaStream_t s, cudaStream_t s_sel) {
+cudaError_t launch_window(dum_engine *e, const PredArgs &a, bool select, cudaStream_t s) {
   if (!e->copy_grid) {
     int dev = 0, sms = 148, nc = 1, ns = 1;
     cudaGetDevice(&dev);
@@ -593,16 +619,14 @@ cudaError_t launch_window(dum_engine *e, const PredArgs &a, bool select, cudaStr
     e->copy_grid = (uint32_t)std::max(1, nc * sms);
     e->sel_grid = (uint32_t)std::max(1, ns * sms);
   }
-  {
+  if (!select) {  // prefetch windows only: the flat copy
     TimerScope t(e, DUM_T_PREDICT, s);
     k_copy_fast<<<e->copy_grid, COPY_NT, 0, s>>>(a);
+  } else {  // one CTA per window: selection, then its pairs
+    TimerScope t(e, DUM_T_PREDICT, s);
+    k_select_fast<<<std::min(a.nq, e->sel_grid), WSEL_NT, 0, s>>>(a);
   }
   e->kernel_launches += 1;
-  if (select) {
-    TimerScope t(e, DUM_T_SELECT, s_sel);
-    k_select_fast<<<std::min(a.nq, e->sel_grid), WSEL_NT, 0, s_sel>>>(a);
-    e->kernel_launches += 1;
-  }
   return cudaGetLastError();
 }
 

@@ -9,7 +9,7 @@ namespace dum {
 
 constexpr uint32_t MAXN = 128;      // degree_n limit
 constexpr int NQCLS = 5;            // window-size classes of k_chain's query order
-constexpr uint32_t HOLD_MAX = 16;   // walk index: holders recorded per block
+constexpr uint32_t HOLD_MAX = 64;   // walk index: holders recorded per block
 constexpr uint32_t CONF_MAX = 64;   // walk index: conflicting exec IDs recorded per walk
 constexpr uint32_t CHUNK_B = 128;   // window blocks per copy chunk (one warp: 4 coalesced steps)
 constexpr int COPY_NT = 256;        // k_copy_fast threads
@@ -111,6 +111,6 @@ __device__ __forceinline__ void copy_window_lists(const PredArgs &a, const uint3
 
 cudaError_t launch_walk_index(dum_engine *e, cudaStream_t s);
 cudaError_t launch_walk_res(dum_engine *e, cudaStream_t s);
-cudaError_t launch_window(dum_engine *e, const PredArgs &a, bool select, cudaStream_t s, cudaStream_t s_sel);
+cudaError_t launch_window(dum_engine *e, const PredArgs &a, bool select, cudaStream_t s);
 
 }  // namespace dum

@@ -60,13 +60,11 @@ def local_cpus_of_gpu(index: int):
     its pinned host arena and its driver threads sit on the GPU's NUMA node
     (numactl --cpunodebind/--membind equivalent)."""
     try:
-        bus = torch.cuda.get_device_properties(index).pci_bus_id  # "0000:1B:00.0"
+        p = torch.cuda.get_device_properties(index)
+        bus = "%04x:%02x:%02x.0" % (int(getattr(p, "pci_domain_id", 0)), int(p.pci_bus_id), int(p.pci_device_id))
     except Exception:
         return None
-    if not bus:
-        return None
-    for cand in (bus.lower(), bus.lower()[4:] if len(bus) > 12 else bus.lower()):
-        path = "/sys/bus/pci/devices/%s/local_cpulist" % (cand if cand.count(":") == 2 else "0000:" + cand)
+    for path in ("/sys/bus/pci/devices/%s/local_cpulist" % bus,):
         try:
             txt = open(path).read().strip()
         except OSError:
@@ -86,7 +84,10 @@ def bind_to_gpu_node(index: int):
     """Bind this process to the CPUs local to GPU `index` (first-touch then
     places its host allocations on that NUMA node).  Returns a report dict."""
     import os
-    cpus = local_cpus_of_gpu(index)
+    try:
+        cpus = local_cpus_of_gpu(index)
+    except Exception as e:  # never fatal: binding is a placement hint
+        return {"bound": False, "why": "lookup failed: %s" % e}
     if not cpus:
         return {"bound": False, "why": "no sysfs local_cpulist for the GPU"}
     try:

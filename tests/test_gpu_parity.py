@@ -358,8 +358,8 @@ def test_sequential_walker_mode_builds_identical_walks(R):
     assert c["WALK_SLOW"] > 0 and c["WALK_DEDUPE"] == 0, c
 
 
-@pytest.mark.parametrize("host", [True, False])
-def test_dum_step_equals_the_separate_calls(host):
+@pytest.mark.parametrize("host,graph", [(True, False), (False, False), (True, True), (False, True)])
+def test_dum_step_equals_the_separate_calls(host, graph):
     """dum_step (record -> queries -> predict+select -> build in one call) on
     Config T with a residency snapshot and inactive blocks: every iteration's
     windows, victims and the final tables equal the oracle's."""
@@ -374,6 +374,7 @@ def test_dum_step_equals_the_separate_calls(host):
     eng.mark_inactive(dev(inact), True)
     out = {}
     ex_all = []
+    eng.set_step_graphs(graph)  # graph: one CUDA graph per staging set, replayed
     for i in range(tr.n_iter):
         h, off, f = tr.iteration(i)
         ex_all += [int(x) for x in o.record_faults(h, off, f)]
