@@ -159,8 +159,8 @@ def algorithmic_bytes(ctr, geo, N):
         "k_ingest": terms["ingest"] + 16 * c["LAUNCHES"],
         "k_build_prep": 48 * c["CORR_UPSERTS"],
         "k_build_exec": terms["block_tables"] + terms["walk_cache"],  # apply + walks (dedupe walks: k_walk)
-        "k_copy_fast": fast_copy,
-        "k_select_fast": fast_sel,
+        "k_copy_fast": fast_copy,             # predict only: the flat copy of the fast windows
+        "k_select_fast": fast_copy + fast_sel,  # with selection: a CTA per window selects, then copies
         "k_predict": terms["predict"] + terms["select"] - fast_copy - fast_sel,
     }
     return terms, per_kernel, c
@@ -475,7 +475,8 @@ def run_ours(args, rank, world, local_rank):
             "bytes_formula": {
                 "k_copy_fast": "4*GATHERED + 8*EMITTED + 4*(N+2)*QUERIES of the fast queries = "
                                "12*FAST_EMITTED + 4*(N+2)*Q_FAST (SURVEY 8(d) predict term)",
-                "k_select_fast": "4*FAST_SCANNED + 4*FAST_VICTIMS (SURVEY 8(d) select term)",
+                "k_select_fast": "12*FAST_EMITTED + 4*(N+2)*Q_FAST + 4*FAST_SCANNED + 4*FAST_VICTIMS "
+                                 "(SURVEY 8(d) predict + select terms of the fast queries)",
                 "k_build_exec": "2*set_bytes*SETS + set_bytes*WALK_ROWS + 4*WALK_OUT (block tables + walk cache)",
                 "k_ingest": "4*RAW + 4*NORM + 20*LAUNCHES + 16*LAUNCHES (exec-map probe)",
                 "k_build_prep": "48*CORR_UPSERTS", "set_bytes": 4 * geo["A"] * (1 + geo["S"]), "N": N},

@@ -415,6 +415,7 @@ enum {
   DUM_T_EXACT,        /* exact-path predict kernel k_predict (side stream, beside the fast path) */
   DUM_T_WALK_INDEX,   /* walk index: holders per block, conflicts per walk (build end) */
   DUM_T_WALK_RES,     /* residency facts per walk (predict) */
+  DUM_T_SELECT_FAST,  /* fast path with selection: k_select_fast (a CTA per window: victims, then pairs) */
   DUM_NTIMERS = 24
 };
 int dum_set_timing(dum_engine *eng, int enable);

@@ -598,7 +598,7 @@ static int step_graph(dum_engine *e, const uint64_t *launch_hash, const uint64_t
       CK(cudaDeviceSynchronize());
       CK(cudaFree(e->d_chunk_map));
       e->d_chunk_map = nullptr;
-      CK(cudaMalloc((void **)&e->d_chunk_map, 8 * bound));
+      CK(cudaMalloc((void **)&e->d_chunk_map, 16 * bound));
       e->chunk_cap = bound;
     }
     SelectOut so = make_select_out(e, out_writeback, out_invalidate, sel_cap, sel_range);

@@ -199,7 +199,7 @@ struct dum_engine {
   uint32_t *d_log_bits;         // [lrm_cap / 32 + 1] inactive log entries by position from head (k_log_bits)
   uint32_t *d_qroff, *d_qneed;  // [max queries][N+2], [max queries] (k_chain -> k_window)
   unsigned long long *d_qvb;    // [max queries][2] victim-range bases (k_chain -> k_window)
-  unsigned long long *d_chunk_map;  // [chunk_cap] (q << 40 | list << 32 | chunk) of the fast queries' windows
+  uint4 *d_chunk_map;  // [chunk_cap] copy chunks of the fast queries' windows: {exec, first, dst lo, dst hi | n << 16}
   uint64_t chunk_cap;
   cudaStream_t side2;           // exact-path predict kernel beside the fast path
   cudaEvent_t ev_fork2, ev_join2;
@@ -243,7 +243,8 @@ struct dum_engine {
   uint64_t t_cnt[DUM_NTIMERS];
   int predict_smem, select_smem, build_smem, ingest_smem;
   uint32_t apply_grid, walk_grid;  // persistent build grids (occupancy x SMs), set on first build
-  uint32_t copy_grid, sel_grid;    // persistent predict grids (k_window.cu)
+  uint32_t copy_grid, sel_grid, stale_grid;  // persistent predict grids (k_window.cu)
+  int sel_smem;                              // k_select_fast dynamic shared memory (k_window.cu)
   int chain_smem;                  // k_chain dynamic smem attribute applied
   int bulk_smem;                   // k_copy_bulk dynamic smem attribute applied
   // dum_step as a replayed CUDA graph (dum_set_step_graphs)

@@ -124,6 +124,7 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
   bool slow = false;   // the query goes to the exact kernel (k_predict) instead of k_window
   uint32_t qneed = 0;  // fast query, fused select: victims to reserve in each output list
   uint32_t GUq = 0;    // copy chunks of the window (k_copy_fast)
+  uint32_t qres = 0;   // fast query, fused select: resident window blocks (marks of the selection)
   if (qi < a.nq) {
     const dum_query Q = a.q[qi];
     const bool anchored = Q.anchor != NONE;
@@ -269,6 +270,7 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
       }
     }
     if (slow) qneed = 0;  // the exact kernel reserves its own victim ranges
+    qres = nwres;
     GUq = slow ? 0u : GU;
     __syncwarp();
     if (cset)
@@ -280,15 +282,17 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
   // window-size class (largest first) for the CTA order of k_window / k_predict:
   // the big windows start first instead of forming the tail; fast-path
   // queries (classes 0 .. NQCLS-1) before exact-path ones
-  // (fast queries of a fused select: ordered by `need`, the length of their selection)
-  const uint32_t key = (a.select && !slow) ? 2 * qneed : U;
+  // (fast queries of a fused select: by their selection work -- the marks of
+  // the resident window blocks plus the log entries up to the cut, need +
+  // resident ones at most -- which also picks k_select_fast's CTA items)
+  const uint32_t key = (a.select && !slow) ? (qneed ? qneed + 2 * qres : 0u) : U;
   const uint32_t cls = (key >= 14336 ? 0u : key >= 10240 ? 1u : key >= 6144 ? 2u : key >= 2048 ? 3u : 4u) +
                        (slow ? (uint32_t)NQCLS : 0u);
   if (threadIdx.x < 2 * NQCLS) s_cls[threadIdx.x] = 0;
   if (lane == 0) {
     s_u[w] = U;
     s_need[w] = qneed;
-    s_gu[w] = a.select ? 0u : GUq;  // copy chunks of k_copy_fast (predict only)
+    s_gu[w] = GUq;  // copy chunks of k_copy_fast
   }
   __syncthreads();
   if (qi < a.nq && lane == 0) s_wcls[w] = atomicAdd(&s_cls[cls], 1u);  // rank within the CTA
@@ -353,16 +357,27 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
       for (uint32_t d = lane; d <= g.N; d += 32) ch[d] = d < nk ? skern[w][d] : NONE;
     }
   }
-  // the chunk map of k_copy_fast (predict only): chunk j of list d of a fast query -> (q, d, j)
-  if (qi < a.nq && s_gu[w] && !a.select) {
-    unsigned long long gb = s_gbase;
-    for (uint32_t i = 0; i < w; ++i) gb += s_gu[i];
+  // the chunk map of k_copy_fast: chunk j of list d of a fast query -> its
+  // source (walk, first entry), destination slot and length; a query whose
+  // pairs do not fit the pool gets empty chunks (capacity error raised above)
+  if (qi < a.nq && s_gu[w]) {
+    __syncwarp();  // the lanes' qloff entries
+    unsigned long long gb = s_gbase, base = s_base;
+    for (uint32_t i = 0; i < w; ++i) {
+      gb += s_gu[i];
+      base += s_u[i];
+    }
     const uint32_t G = s_gu[w], nk = a.qnk[qi];
+    const bool fits = base + s_u[w] <= a.cap;
+    const uint32_t *lo = a.qloff + (uint64_t)qi * (g.N + 2);
     for (uint32_t d = lane; d < nk; d += 32) {  // lane d: the chunks of list d
-      const uint32_t g0 = sgoff[w][d], g1 = sgoff[w][d + 1];
+      const uint32_t g0 = sgoff[w][d], g1 = sgoff[w][d + 1], l0 = lo[d], L = lo[d + 1] - l0, e = skern[w][d];
       for (uint32_t x = g0; x < g1; ++x)
-        if (gb + x < a.chunk_cap)
-          a.chunk_map[gb + x] = ((unsigned long long)qi << 40) | ((unsigned long long)d << 32) | (x - g0);
+        if (gb + x < a.chunk_cap) {
+          const uint32_t i0 = (x - g0) * CHUNK_B, n = fits ? min(CHUNK_B, L - i0) : 0u;
+          const unsigned long long dst = base + l0 + i0;
+          a.chunk_map[gb + x] = make_uint4(e, i0, (uint32_t)dst, (uint32_t)(dst >> 32) | (n << 16));
+        }
     }
     if (lane == 0 && gb + G > a.chunk_cap) set_err(a.st, ERR_ECAPACITY, gb + G);
   }
@@ -382,7 +397,7 @@ static_assert(2 * DWCAP + 2 * DBCAP <= 2 * DHCAP, "duplicate hashes live in the 
 static_assert(OCCAP >= DLCAP, "s_dup doubles as the occurrence list");
 
 template <bool SELECT>
-__global__ void __launch_bounds__(PRED_NT, 3) k_predict(PredArgs a) {
+__global__ void __launch_bounds__(PRED_NT, 2) k_predict(PredArgs a) {
   extern __shared__ uint4 sm4[];  // [nwords rounded up to 4] window set bitmap | dup hashes / select stage
   uint32_t *bitmap = reinterpret_cast<uint32_t *>(sm4);
   uint32_t *dk = bitmap + ((a.nwords + 3) & ~3u);  // [2 * DHCAP]
@@ -957,7 +972,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
       cudaError_t ce = cudaStreamSynchronize(s);  // growth only: the old map may be in use
       if (ce == cudaSuccess) ce = cudaFree(e->d_chunk_map);
       e->d_chunk_map = nullptr;
-      if (ce == cudaSuccess) ce = cudaMalloc((void **)&e->d_chunk_map, 8 * bound);
+      if (ce == cudaSuccess) ce = cudaMalloc((void **)&e->d_chunk_map, 16 * bound);
       if (ce != cudaSuccess) return ce;
       e->chunk_cap = bound;
     }

@@ -21,14 +21,23 @@ namespace dum {
 constexpr int INGEST_NT = 256;
 constexpr uint32_t INGEST_HCAP = 2048;  // smem hash capacity (n <= 1024 in smem): 16 KB, 8 CTAs / SM
 constexpr uint32_t IDCAP = 1024;        // repeated-block hash of the bitmap path
-constexpr uint32_t INGEST_SMEM_MAX = 16 * 1024;  // the bitmap path only where it fits this (small W)
+constexpr uint32_t INGEST_SMEM_MAX = 24 * 1024;  // bitmap (exact for small W, else hashed) + dup hash
+
+// bit of block b in a hashed bitmap of 2^k bits: runs of consecutive blocks
+// stay consecutive (the warp's word grouping), far regions land at
+// pseudo-random offsets.  A shared bit is only a candidate repeat: the
+// min-position hash then settles it exactly.
+__device__ __forceinline__ uint32_t bm_bit(uint32_t b, uint32_t nbits) {
+  return (b + (b / nbits) * 0x9E3779B1u) & (nbits - 1);
+}
 
 __global__ void __launch_bounds__(INGEST_NT) k_ingest(
     const uint64_t *__restrict__ hash, const uint64_t *__restrict__ off, const uint32_t *__restrict__ faults,
     uint32_t n_launch, uint32_t W, uint32_t l0, uint64_t f0, uint64_t *__restrict__ stage_hash,
     uint64_t *__restrict__ stage_off, uint32_t *__restrict__ stage_norm, uint32_t *__restrict__ stage_cnt,
     uint32_t *__restrict__ stage_slot, unsigned long long *exec_keys, uint32_t *exec_vals, uint32_t *exec_minpos,
-    uint32_t exec_cap, uint32_t *big_pool, uint64_t big_entries, uint32_t bm_words, uint32_t *__restrict__ stage_exec,
+    uint32_t exec_cap, uint32_t *big_pool, uint64_t big_entries, uint32_t bm_words, bool bm_hashed,
+    uint32_t *__restrict__ stage_exec,
     uint32_t *__restrict__ out_exec, uint32_t *__restrict__ pend, uint32_t Emax, uint64_t n_fault, DevState *st) {
   extern __shared__ uint32_t dyn[];  // hash (2 x INGEST_HCAP) or bitmap + small dup hash
   __shared__ uint32_t ws[INGEST_NT / 32];
@@ -83,11 +92,13 @@ __global__ void __launch_bounds__(INGEST_NT) k_ingest(
     }
     stage_slot[l0 + i] = slot;
   }
-  // Big launches (> INGEST_HCAP/2 records) dedupe through a bitmap over the
-  // block-id space when it fits the shared-memory budget: an order-free
-  // warp-aggregated test-and-set finds whether any block repeats (normally
-  // not: the input is then copied), and only repeated blocks go through a
-  // small min-position hash.  Otherwise a private global-pool hash is used.
+  // Big launches (> INGEST_HCAP/2 records) dedupe through a bitmap: over the
+  // block-id space when it fits the shared-memory budget, else hashed
+  // (bm_bit).  An order-free warp-aggregated test-and-set finds the records
+  // whose bit was already set (normally none: the input is then copied);
+  // only those blocks go through a small min-position hash, which keeps the
+  // first occurrence of each.  A private global-pool hash takes launches
+  // whose candidates overflow it.
   const bool use_bitmap = n > INGEST_HCAP / 2 && bm_words != 0;
   if (n > 0 && use_bitmap) {
     uint32_t *bm = dyn, *dk = dyn + ((bm_words + 3) & ~3u), *dv = dk + IDCAP;
@@ -107,14 +118,13 @@ __global__ void __launch_bounds__(INGEST_NT) k_ingest(
         set_err(st, ERR_EINVAL);
         ++ndup;  // dropped: take the compaction path
       }
-      if (warp_test_and_set(bm, blk, inr)) {
+      if (warp_test_and_set(bm, bm_hashed && inr ? bm_bit(blk, bm_words * 32) : blk, inr)) {
         ++ndup;
         if (!hmap_insert_min(dk, dv, IDCAP, blk, j)) s_ovf = 1;
       }
     }
     if (ndup) s_dups = 1;
     __syncthreads();
-    if (threadIdx.x == 0 && s_dups) ctr_add(st, DUM_CTR_INGEST_DUP, 1);
     uint32_t run = n;
     if (!s_dups) {
       for (uint32_t j = threadIdx.x; j < n; j += INGEST_NT) stage_norm[f0 + a + j] = faults[a + j];
@@ -152,6 +162,7 @@ __global__ void __launch_bounds__(INGEST_NT) k_ingest(
     }
     if (!s_dups || !s_ovf) {
       if (threadIdx.x == 0) {
+        if (run < n) ctr_add(st, DUM_CTR_INGEST_DUP, 1);
         stage_cnt[l0 + i] = run;
         ctr_add(st, DUM_CTR_RAW_RECORDS, n);
         ctr_add(st, DUM_CTR_NORM_RECORDS, run);
@@ -337,10 +348,16 @@ cudaError_t launch_record(dum_engine *e, const uint64_t *hash, const uint64_t *o
   if (n_launch == 0) return cudaSuccess;
   {
   TimerScope t(e, DUM_T_INGEST, s);
-  const uint32_t bmw = (e->g.W + 31) / 32;
+  // the bitmap: exact over [0, W) when it fits, else the largest power-of-two
+  // word count that does (hashed)
+  uint32_t bmw = (e->g.W + 31) / 32;
+  const bool bm_hashed = (size_t)((bmw + 3) & ~3u) * 4 + 2 * IDCAP * 4 > INGEST_SMEM_MAX;
+  if (bm_hashed) {
+    bmw = 1;
+    while ((size_t)(2 * bmw) * 4 + 2 * IDCAP * 4 <= INGEST_SMEM_MAX) bmw *= 2;
+  }
   const size_t bm_bytes = (size_t)((bmw + 3) & ~3u) * 4 + 2 * IDCAP * 4;
-  const bool bm_ok = bm_bytes <= INGEST_SMEM_MAX;
-  const size_t smem = std::max<size_t>(2 * INGEST_HCAP * 4, bm_ok ? bm_bytes : 0);
+  const size_t smem = std::max<size_t>(2 * INGEST_HCAP * 4, bm_bytes);
   // the attribute is per device and function: raised by every engine on its own device
   if ((int)smem > e->ingest_smem) {
     cudaFuncSetAttribute(k_ingest, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -349,7 +366,7 @@ cudaError_t launch_record(dum_engine *e, const uint64_t *hash, const uint64_t *o
   k_ingest<<<n_launch, INGEST_NT, smem, s>>>(hash, off, faults, n_launch, e->g.W, e->n_staged, e->staged_faults,
                                              e->d_stage_hash, e->d_stage_off, e->d_stage_norm, e->d_stage_cnt,
                                              e->d_stage_slot, e->d_exec_keys, e->d_exec_vals, e->d_exec_minpos,
-                                             e->exec_cap, e->d_ingest_pool, e->big_pool_entries, bm_ok ? bmw : 0,
+                                             e->exec_cap, e->d_ingest_pool, e->big_pool_entries, bmw, bm_hashed,
                                              e->d_stage_exec, out_exec, e->d_pend, e->g.Emax, n_fault, e->d_state);
   }
   TimerScope t(e, DUM_T_EXEC_ASSIGN, s);

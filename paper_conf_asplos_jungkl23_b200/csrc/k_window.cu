@@ -21,7 +21,7 @@
 //                                     of a resident block of one of its walks.
 // k_walk_res computes, per walk, the non-resident count and the log positions
 // of its resident blocks (after every residency change, at predict time);
-// k_window marks those positions in a shared-memory bitmap over
+// the selection kernels mark those positions in a shared-memory bitmap over
 // [head, head + POS_BITS) of the LRM log and runs the same ordered selection
 // as the exact path (select_tail.cuh) on it.  k_chain only routes a query
 // here when the selection provably ends inside that range.
@@ -30,7 +30,9 @@
 //  k_walk_conf   (build end)   conflicts of each walk: conf[e][..], conf_n[e]
 //  k_walk_res    (predict)     per walk: non-resident count, resident positions
 //  k_copy_fast   (predict)     flat copy of every fast window (chunk map from k_chain)
-//  k_select_fast (predict)     one CTA per fast query: marking + ordered selection
+//  k_select_fast (predict)     clean log: a CTA per big window, a warp per small one;
+//                              marking + word-level selection
+//  k_select_stale (predict)    stale log entries: a CTA per window, per-entry selection
 #include <algorithm>
 
 #include "device_util.cuh"
@@ -183,59 +185,43 @@ __global__ void __launch_bounds__(IX_NT) k_walk_res(const uint32_t *__restrict__
   }
 }
 
-// Flat copy of every fast query's window: warp-granular work items of 128
-// window blocks (one list of one query; chunk map from k_chain), two in flight
-// per warp, lane-consecutive 4 B loads of the cached walk and 8 B streaming
-// stores of the (block, exec) pairs.  Persistent grid over the device count.
+// Flat copy of every fast query's window: warp-granular work items of <= 128
+// window blocks of one list of one query, each a 16 B descriptor written by
+// k_chain (source walk + first entry, destination pair slot, length: one
+// dependent load before the data), four in flight per warp, lane-consecutive
+// 4 B loads of the cached walk and 8 B streaming stores of the (block, exec)
+// pairs.  Persistent grid over the device count.
 __global__ void __launch_bounds__(COPY_NT) k_copy_fast(PredArgs a) {
-  constexpr uint32_t UN = 2;
+  constexpr uint32_t UN = 4;  // chunks per warp step, their loads in flight together
   const uint32_t lane = threadIdx.x & 31;
   const uint64_t G = *(volatile unsigned long long *)&a.st->pool_chunks;
   const uint64_t nw = (uint64_t)gridDim.x * (COPY_NT / 32);
-  const uint32_t N = a.g.N;
   uint2 *out = reinterpret_cast<uint2 *>(a.pairs);
   unsigned long long emitted = 0;
   for (uint64_t c0 = (uint64_t)blockIdx.x * (COPY_NT / 32) + (threadIdx.x >> 5); c0 < G; c0 += nw * UN) {
-    unsigned long long m[UN];
+    uint4 m[UN];
 #pragma unroll
-    for (uint32_t u = 0; u < UN; ++u) m[u] = c0 + u * nw < G ? __ldcg(a.chunk_map + c0 + u * nw) : ~0ull;
-    uint32_t kd[UN], lo[UN], L[UN], i0[UN];
-    unsigned long long base[UN];
-#pragma unroll
-    for (uint32_t u = 0; u < UN; ++u) {
-      if (m[u] == ~0ull) continue;
-      const uint32_t q = (uint32_t)(m[u] >> 40), d = (uint32_t)(m[u] >> 32) & 0xFFu;
-      i0[u] = (uint32_t)(m[u] & 0xFFFFFFFFu) * CHUNK_B;
-      kd[u] = __ldcg(a.qkern + (uint64_t)q * (N + 1) + d);
-      lo[u] = __ldcg(a.qloff + (uint64_t)q * (N + 2) + d);
-      L[u] = __ldcg(a.qloff + (uint64_t)q * (N + 2) + d + 1) - lo[u];
-      base[u] = __ldcg(a.qbase + q);
-    }
+    for (uint32_t u = 0; u < UN; ++u)
+      m[u] = c0 + u * nw < G ? __ldcg(a.chunk_map + c0 + u * nw) : make_uint4(0, 0, 0, 0);
     uint32_t b[UN][4];
 #pragma unroll
     for (uint32_t u = 0; u < UN; ++u) {
-      if (m[u] == ~0ull) continue;
-      const uint32_t *lst = a.walk + (uint64_t)kd[u] * a.g.walk_cap;
+      const uint32_t n = m[u].w >> 16;
+      const uint32_t *lst = a.walk + (uint64_t)m[u].x * a.g.walk_cap + m[u].y;
 #pragma unroll
-      for (uint32_t k = 0; k < 4; ++k) {
-        const uint32_t i = i0[u] + 32 * k + lane;
-        b[u][k] = i < L[u] ? __ldg(lst + i) : NONE;
-      }
+      for (uint32_t k = 0; k < 4; ++k) b[u][k] = 32 * k + lane < n ? __ldg(lst + 32 * k + lane) : NONE;
     }
 #pragma unroll
     for (uint32_t u = 0; u < UN; ++u) {
-      if (m[u] == ~0ull) continue;
-      if (base[u] + lo[u] + L[u] > a.cap) continue;  // capacity error raised by k_chain
-      uint2 *o = out + base[u] + lo[u];
+      const uint32_t n = m[u].w >> 16;
+      uint2 *o = out + ((unsigned long long)(m[u].w & 0xFFFFu) << 32 | m[u].z);
 #pragma unroll
-      for (uint32_t k = 0; k < 4; ++k) {
-        const uint32_t i = i0[u] + 32 * k + lane;
-        if (i < L[u]) __stcs(o + i, make_uint2(b[u][k], kd[u]));
-      }
-      if (lane == 0) emitted += min(CHUNK_B, L[u] - i0[u]);
+      for (uint32_t k = 0; k < 4; ++k)
+        if (32 * k + lane < n) __stcs(o + 32 * k + lane, make_uint2(b[u][k], m[u].x));
+      emitted += n;
     }
   }
-  emitted = __reduce_add_sync(0xffffffffu, (unsigned)emitted);
+  emitted = __reduce_add_sync(0xffffffffu, (unsigned)emitted) / 32;
   if (lane == 0 && emitted) {
     ctr_add(a.st, DUM_CTR_EMITTED, emitted);
     ctr_add(a.st, DUM_CTR_GATHERED, emitted);
@@ -243,39 +229,380 @@ __global__ void __launch_bounds__(COPY_NT) k_copy_fast(PredArgs a) {
   }
 }
 
-// Fused a8 of one fast query per CTA (k_chain's order: fast queries by
-// decreasing `need`).  need = max(0, window blocks without a frame - free
-// frames) and the victim ranges come from k_chain (D18).  The victims are the
-// first `need` entries of the LRM log, oldest first, that are still resident
-// with their stamp and not in the window, split by the
-// inactive bit of the entry into invalidate / write-back (L285; D19, D20).
-//   1. mark the log positions of the window's resident blocks (flat over the
-//      lists' respos entries, prefix qroff from k_chain) in a bitmap over
-//      [head, head + 32 POS_WORDS);
-//   2. the log prefix [head, head + span) (span = need + resident window
-//      blocks + stale entries: the selection provably ends inside) is cut
-//      into 1024-entry segments; pass 1: each warp counts the eligible
-//      active / inactive entries of its segments;
-//   3. one warp scans the segment counts;
-//   4. pass 2: each warp re-reads its segments and writes the entries of
-//      combined rank < need at their ranks in the two lists (LRM order).
-// Two CTA barriers per query instead of two per 2048-entry chunk.
+// a8 of the fast queries (k_chain's order: by decreasing `need`).  need =
+// max(0, window blocks without a frame - free frames) and the victim ranges
+// come from k_chain (D18).  The victims are the first `need` entries of the
+// LRM log, oldest first, that are still resident with their stamp and not in
+// the window, split by the inactive bit of the entry into
+// invalidate / write-back (L285; D19, D20).  Every variant marks the log
+// positions of the window's resident blocks (flat over the lists' respos
+// entries, prefix qroff from k_chain) in a bitmap over [head, head + 32
+// POS_WORDS) and selects in the log prefix [head, head + span), span = need +
+// resident window blocks + stale entries (k_chain routes a query here only
+// when the selection provably ends inside).  The window's pairs are written
+// by k_copy_fast, concurrently.
+//
+// Clean log (every entry of [head, tail) valid, the normal case):
+// k_select_fast.  A 32-position word's eligible entries are ~marked & valid,
+// split by the log's inactive-entry bitmap (k_log_bits) into write-back /
+// invalidate; a scan of the packed popcounts gives every word its rank base;
+// then 4-word chunks (a lane per 4 consecutive entries, 16 B loads of the
+// log) write the entries of combined rank < need at their ranks.  Work items
+// in k_chain's class order: a big window (classes 0-2, need-key >= 6144) is
+// one CTA item (all warps mark, one block scan, the warps split the chunks);
+// the small ones go WSEL_NT / 32 to an item, a warp each (32-word groups, a
+// warp scan per group, no CTA barrier).  A warp per window alone leaves the
+// few biggest windows as a serial tail; a CTA per window leaves the SMs
+// waiting on barriers for the many small ones.
+//
+// Stale entries (a log not compacted since an eviction): k_select_stale, a CTA
+// per query, per-entry eligibility (frame + stamp check):
+//   1. marks as above;  2. pass 1: eligible active / inactive entries per
+//   1024-entry segment, a warp per segment;  3. one warp scans the segment
+//   counts;  4. pass 2: each warp re-reads its segments and writes the
+//   entries of combined rank < need.
 constexpr uint32_t FSEG = 1024;                 // log entries per segment (32 per lane)
 constexpr uint32_t FSEG_MAX = POS_WORDS * 32 / FSEG;
 static_assert(FSEG_MAX <= 32, "one warp scans the segment counts");
+constexpr uint32_t SEL_NW = WSEL_NT / 32;  // warps per selection CTA
+constexpr uint32_t SW_KB = 2;              // warp path: 4-word chunks with their log loads in flight together
+constexpr uint32_t BIG_CLS = 3;            // classes [0, BIG_CLS) take a CTA per window
 
-// One warp step of the selection: the 32 log entries at positions
+__host__ __device__ constexpr uint32_t sw_words(uint32_t N) {  // shared words of one warp's window (16 B multiple)
+  return (POS_WORDS + (N + 2) + (N + 1) + 3) & ~3u;
+}
+__host__ __device__ constexpr uint32_t sel_smem_words(uint32_t N) {  // k_select_fast dynamic shared memory
+  return SEL_NW * sw_words(N) > 4 * POS_WORDS + sw_words(N) - POS_WORDS
+             ? SEL_NW * sw_words(N)
+             : 4 * POS_WORDS + sw_words(N) - POS_WORDS;
+}
+
+// the fast query of rank bq in k_chain's class lists
+__device__ __forceinline__ uint32_t fast_query(const PredArgs &a, const uint32_t *ccnt, uint32_t bq) {
+  uint32_t cq = NQCLS, rq = bq;
+#pragma unroll
+  for (int c = 0; c < NQCLS; ++c)
+    if (cq == NQCLS) {
+      if (rq < ccnt[c]) cq = c;
+      else rq -= ccnt[c];
+    }
+  return __ldg(a.qperm + (uint64_t)cq * a.nq + rq);
+}
+
+struct SelLog {  // the log, fixed during the kernel
+  uint32_t head, tail, stale;
+  bool al;       // head 16 B aligned: vector loads of the log
+};
+
+struct SelQuery {
+  uint32_t qi, nk, need;
+  unsigned long long bwb, binv;
+  bool ok;
+};
+
+__device__ __forceinline__ SelQuery load_query(const PredArgs &a, uint32_t qi) {
+  SelQuery q;
+  q.qi = qi;
+  q.nk = __ldg(a.qnk + qi);
+  q.need = __ldg(a.qneed + qi);
+  q.bwb = __ldg(a.qvb + 2 * qi);
+  q.binv = __ldg(a.qvb + 2 * qi + 1);
+  q.ok = q.bwb + q.need <= a.so.cap && q.binv + q.need <= a.so.cap;
+  return q;
+}
+
+__device__ __forceinline__ void write_range(const PredArgs &a, const SelQuery &q, uint32_t tw, uint32_t ti) {
+  uint64_t *o = a.so.out_range + 4ull * q.qi;
+  o[0] = q.bwb;
+  o[1] = q.bwb + (q.ok ? tw : 0);
+  o[2] = q.binv;
+  o[3] = q.binv + (q.ok ? ti : 0);
+}
+
+// Marks: the log positions (relative to head) of the window's resident blocks
+// below nbits, by threads t = t0, t0 + nt, ... (MU loads in flight each).
+template <uint32_t MU>
+__device__ __forceinline__ void mark_window(const PredArgs &a, const uint32_t *roff, const uint32_t *kern, uint32_t R,
+                                            uint32_t head, uint32_t nbits, uint32_t *posmap, uint32_t t0,
+                                            uint32_t nt) {
+  uint32_t lo = 0;
+  for (uint32_t x0 = t0; x0 < R; x0 += nt * MU) {
+    uint32_t r[MU];
+#pragma unroll
+    for (uint32_t u = 0; u < MU; ++u) {
+      const uint32_t x = x0 + u * nt;
+      r[u] = NONE;
+      if (x < R) {
+        while (roff[lo + 1] <= x) ++lo;
+        r[u] = __ldg(a.respos + (uint64_t)kern[lo] * a.g.walk_cap + (x - roff[lo])) - head;
+      }
+    }
+#pragma unroll
+    for (uint32_t u = 0; u < MU; ++u)
+      if (r[u] < nbits) atomicOr(&posmap[r[u] >> 5], 1u << (r[u] & 31));
+  }
+}
+
+// The eligible entries of UC 4-word chunks of one warp (a lane per 4
+// consecutive entries): chunk u covers words wd[u] .. +3 relative to w0 (lane
+// >> 3 picks the word), with em / im / pre the word's masks and rank base
+// (packed inactive << 16 | active).  Entries of combined rank < need go to
+// their ranks; returns the counts written (tw, ti).
+template <uint32_t UC>
+__device__ __forceinline__ void emit_chunks(const PredArgs &a, const SelQuery &q, const SelLog &lg, uint32_t lane,
+                                            const uint32_t *wpos, const uint32_t *em, const uint32_t *im,
+                                            const uint32_t *pre, uint32_t &tw, uint32_t &ti) {
+  const SelectOut &so = a.so;
+  uint32_t a4[UC], i4[UC], ra[UC], rr[UC], vv[UC][4];
+  const uint32_t sh = (lane & 7) * 4;
+#pragma unroll
+  for (uint32_t u = 0; u < UC; ++u) {
+    a4[u] = (em[u] >> sh) & 0xFu;
+    i4[u] = (im[u] >> sh) & 0xFu;
+    // ranks: the word's base + the eligible entries of the lower lanes of the same word
+    const uint32_t cc = __popc(a4[u]) | (__popc(i4[u]) << 16);
+    uint32_t y = cc;
+#pragma unroll
+    for (int o = 1; o < 8; o <<= 1) {
+      const uint32_t t = __shfl_up_sync(0xffffffffu, y, o);
+      if ((lane & 7) >= (uint32_t)o) y += t;
+    }
+    ra[u] = (pre[u] & 0xFFFFu) + ((y - cc) & 0xFFFFu);
+    rr[u] = (pre[u] >> 16) + ((y - cc) >> 16);
+    if (ra[u] + rr[u] >= q.need) a4[u] = i4[u] = 0;
+    if (a4[u] | i4[u]) {
+      const uint32_t p = lg.head + 32 * wpos[u] + sh;
+      if (lg.al) {
+        const uint4 v = __ldcg(reinterpret_cast<const uint4 *>(so.lrm_blk + p));
+        vv[u][0] = v.x; vv[u][1] = v.y; vv[u][2] = v.z; vv[u][3] = v.w;
+      } else {
+#pragma unroll
+        for (uint32_t k = 0; k < 4; ++k) vv[u][k] = ((a4[u] | i4[u]) >> k) & 1u ? __ldcg(so.lrm_blk + p + k) : 0u;
+      }
+    }
+  }
+#pragma unroll
+  for (uint32_t u = 0; u < UC; ++u) {
+    if (!(a4[u] | i4[u])) continue;
+#pragma unroll
+    for (uint32_t k = 0; k < 4; ++k) {
+      const bool ea = (a4[u] >> k) & 1u, ei = (i4[u] >> k) & 1u;
+      if ((ea || ei) && ra[u] + rr[u] < q.need) {
+        if (q.ok) {
+          if (ei) so.inv[q.binv + rr[u]] = vv[u][k] & 0x7FFFFFFFu;
+          else so.wb[q.bwb + ra[u]] = vv[u][k];
+        }
+        tw += ea;
+        ti += ei;
+      }
+      ra[u] += ea;
+      rr[u] += ei;
+    }
+  }
+}
+
+// A small window, one warp: marks in the warp's bitmap, then 32-word groups
+// (lane l: word w0 + l) with a warp scan each, until the cut.
+__device__ __forceinline__ void warp_window(const PredArgs &a, const SelLog &lg, uint32_t qi, uint32_t *wsm,
+                                            unsigned long long &scanned, unsigned long long &victims) {
+  const uint32_t lane = threadIdx.x & 31;
+  const Geo &g = a.g;
+  uint32_t *posmap = wsm, *roff = wsm + POS_WORDS, *kern = roff + g.N + 2;
+  const SelQuery q = load_query(a, qi);
+  for (uint32_t d = lane; d <= q.nk; d += 32) {
+    roff[d] = __ldg(a.qroff + (uint64_t)qi * (g.N + 2) + d);
+    if (d < q.nk) kern[d] = __ldg(a.qkern + (uint64_t)qi * (g.N + 1) + d);
+  }
+  __syncwarp();
+  const uint32_t R = roff[q.nk];
+  const uint32_t span = min(lg.tail - lg.head, min(q.need + R + lg.stale, POS_WORDS * 32));
+  const uint32_t nw = (span + 31) / 32;
+  uint32_t tw = 0, ti = 0;
+  if (q.need) {
+    for (uint32_t w = lane; w < nw; w += 32) posmap[w] = 0;
+    __syncwarp();
+    mark_window<8>(a, roff, kern, R, lg.head, nw * 32, posmap, lane, 32);
+    __syncwarp();
+    uint32_t ba = 0, bi = 0, w0 = 0;
+    for (; w0 < nw && ba + bi < q.need; w0 += 32) {
+      const uint32_t w = w0 + lane;
+      uint32_t em = 0, im = 0;
+      if (w < nw) {
+        const uint32_t lo = w * 32, valid = span - lo >= 32 ? 0xFFFFFFFFu : (1u << (span - lo)) - 1u;
+        const uint32_t ib = __ldg(a.inact_bits + w), e = valid & ~posmap[w];
+        em = e & ~ib;
+        im = e & ib;
+      }
+      const uint32_t c = __popc(em) | (__popc(im) << 16);
+      uint32_t x = c;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= (uint32_t)o) x += y;
+      }
+      const uint32_t wpre = (ba | (bi << 16)) + x - c;  // packed ranks: both < 2^15
+      for (uint32_t k0 = 0; k0 < 8; k0 += SW_KB) {
+        const uint32_t pre0 = __shfl_sync(0xffffffffu, wpre, 4 * k0);
+        if (w0 + 4 * k0 >= nw || (pre0 & 0xFFFFu) + (pre0 >> 16) >= q.need) break;
+        uint32_t wp[SW_KB], e32[SW_KB], i32[SW_KB], p32[SW_KB];
+#pragma unroll
+        for (uint32_t u = 0; u < SW_KB; ++u) {
+          const uint32_t wd = 4 * (k0 + u) + (lane >> 3);
+          wp[u] = w0 + wd;
+          e32[u] = __shfl_sync(0xffffffffu, em, wd);
+          i32[u] = __shfl_sync(0xffffffffu, im, wd);
+          p32[u] = __shfl_sync(0xffffffffu, wpre, wd);
+        }
+        emit_chunks<SW_KB>(a, q, lg, lane, wp, e32, i32, p32, tw, ti);
+      }
+      const uint32_t tot = __shfl_sync(0xffffffffu, x, 31);
+      ba += tot & 0xFFFFu;
+      bi += tot >> 16;
+    }
+    tw = __reduce_add_sync(0xffffffffu, tw);
+    ti = __reduce_add_sync(0xffffffffu, ti);
+    if (lane == 0) scanned += min(span, 32 * w0);
+  }
+  if (lane == 0) {
+    write_range(a, q, tw, ti);
+    victims += tw + ti;
+  }
+}
+
+// A big window, the whole CTA: marks, one block scan over the words (thread t
+// owns words 4t .. 4t+3), the warps split the chunks.
+__device__ __forceinline__ void cta_window(const PredArgs &a, const SelLog &lg, uint32_t qi, uint32_t *sm,
+                                           uint32_t *ws, uint32_t *s_cnt, unsigned long long &scanned,
+                                           unsigned long long &victims) {
+  const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const Geo &g = a.g;
+  uint32_t *posmap = sm, *wem = sm + POS_WORDS, *wim = wem + POS_WORDS, *wpre = wim + POS_WORDS;
+  uint32_t *roff = wpre + POS_WORDS, *kern = roff + g.N + 2;
+  const SelQuery q = load_query(a, qi);
+  for (uint32_t d = tid; d <= q.nk; d += WSEL_NT) {
+    roff[d] = __ldg(a.qroff + (uint64_t)qi * (g.N + 2) + d);
+    if (d < q.nk) kern[d] = __ldg(a.qkern + (uint64_t)qi * (g.N + 1) + d);
+  }
+  for (uint32_t w = tid; w < POS_WORDS; w += WSEL_NT) posmap[w] = 0;
+  if (tid == 0) s_cnt[0] = s_cnt[1] = 0;
+  __syncthreads();
+  const uint32_t R = roff[q.nk];
+  const uint32_t span = min(lg.tail - lg.head, min(q.need + R + lg.stale, POS_WORDS * 32));
+  const uint32_t nw = (span + 31) / 32;
+  if (q.need) {
+    mark_window<4>(a, roff, kern, R, lg.head, POS_WORDS * 32, posmap, tid, WSEL_NT);
+    __syncthreads();
+    uint32_t ca[4], ci[4], em[4], imk[4], tot = 0;
+#pragma unroll
+    for (uint32_t u = 0; u < 4; ++u) {  // nw <= POS_WORDS = 4 * WSEL_NT
+      const uint32_t w = 4 * tid + u;
+      em[u] = imk[u] = 0;
+      if (w < nw) {
+        const uint32_t lo = w * 32, valid = span - lo >= 32 ? 0xFFFFFFFFu : (1u << (span - lo)) - 1u;
+        const uint32_t ib = __ldg(a.inact_bits + w), e = valid & ~posmap[w];
+        em[u] = e & ~ib;
+        imk[u] = e & ib;
+      }
+      ca[u] = __popc(em[u]);
+      ci[u] = __popc(imk[u]);
+      tot += ca[u] | (ci[u] << 16);
+    }
+    uint32_t tsum;
+    uint32_t pre = block_excl_scan(tot, ws, &tsum);  // packed (inactive << 16 | active)
+#pragma unroll
+    for (uint32_t u = 0; u < 4; ++u) {
+      const uint32_t w = 4 * tid + u;
+      if (w < nw) {
+        wem[w] = em[u];
+        wim[w] = imk[u];
+        wpre[w] = pre;
+      }
+      pre += ca[u] | (ci[u] << 16);
+    }
+    __syncthreads();
+    constexpr uint32_t UC = 2;
+    uint32_t tw = 0, ti = 0;
+    const uint32_t nch = (nw + 3) / 4;
+    for (uint32_t ch0 = wid; ch0 < nch; ch0 += SEL_NW * UC) {
+      {
+        const uint32_t p0 = wpre[4 * ch0];  // the step's first chunk starts past the cut: so do the rest
+        if ((p0 & 0xFFFFu) + (p0 >> 16) >= q.need) break;
+      }
+      uint32_t wp[UC], e32[UC], i32[UC], p32[UC];
+#pragma unroll
+      for (uint32_t u = 0; u < UC; ++u) {
+        const uint32_t w = 4 * (ch0 + u * SEL_NW) + (lane >> 3);
+        wp[u] = w;
+        e32[u] = w < nw ? wem[w] : 0u;
+        i32[u] = w < nw ? wim[w] : 0u;
+        p32[u] = w < nw ? wpre[w] : 0xFFFFFFFFu;
+      }
+      emit_chunks<UC>(a, q, lg, lane, wp, e32, i32, p32, tw, ti);
+    }
+    tw = __reduce_add_sync(0xffffffffu, tw);
+    ti = __reduce_add_sync(0xffffffffu, ti);
+    if (lane == 0 && (tw | ti)) {
+      atomicAdd(&s_cnt[0], tw);
+      atomicAdd(&s_cnt[1], ti);
+    }
+    __syncthreads();
+  }
+  if (tid == 0) {
+    write_range(a, q, s_cnt[0], s_cnt[1]);
+    victims += s_cnt[0] + s_cnt[1];
+    if (q.need) scanned += span;
+  }
+}
+
+__global__ void __launch_bounds__(WSEL_NT, 4) k_select_fast(PredArgs a) {
+  extern __shared__ uint4 sel4[];
+  __shared__ uint32_t ws[SEL_NW], s_cnt[2];
+  const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  if (*(const volatile uint32_t *)&a.st->log_dirty) return;  // k_select_stale's case
+  uint32_t *sm = reinterpret_cast<uint32_t *>(sel4);
+  uint32_t ccnt[NQCLS], nfast = 0, nbig = 0;
+#pragma unroll
+  for (int c = 0; c < NQCLS; ++c) {
+    ccnt[c] = *(const volatile uint32_t *)&a.st->q_cls[c];
+    nfast += ccnt[c];
+    if (c < (int)BIG_CLS) nbig += ccnt[c];
+  }
+  SelLog lg;
+  lg.head = *(const volatile uint32_t *)&a.st->lrm_head;
+  lg.tail = *(const volatile uint32_t *)&a.st->lrm_tail;
+  lg.stale = lg.tail - lg.head - *(const volatile uint32_t *)&a.st->n_resident;
+  lg.al = (lg.head & 3u) == 0;
+  const uint32_t nitems = nbig + (nfast - nbig + SEL_NW - 1) / SEL_NW;
+  unsigned long long scanned = 0, victims = 0;
+  for (uint32_t it = blockIdx.x; it < nitems; it += gridDim.x) {
+    if (it < nbig) {
+      cta_window(a, lg, fast_query(a, ccnt, it), sm, ws, s_cnt, scanned, victims);
+    } else {
+      const uint32_t j = nbig + (it - nbig) * SEL_NW + wid;
+      if (j < nfast) warp_window(a, lg, fast_query(a, ccnt, j), sm + wid * sw_words(a.g.N), scanned, victims);
+    }
+    __syncthreads();  // the next item reuses the shared state
+  }
+  scanned = __reduce_add_sync(0xffffffffu, (unsigned)scanned);
+  victims = __reduce_add_sync(0xffffffffu, (unsigned)victims);
+  if (lane == 0 && (scanned | victims)) {
+    ctr_add(a.st, DUM_CTR_FAST_SCANNED, scanned);
+    ctr_add(a.st, DUM_CTR_FAST_VICTIMS, victims);
+  }
+}
+
+// One warp step of the stale-entry path: the 32 log entries at positions
 // head + r0 + lane (r0 a multiple of 32 relative to head, so that one
 // broadcast word of the position bitmap covers them).  Eligible = inside the
 // log, not a resident window block, still resident with its stamp; returns the
 // active / inactive eligible ballots.  v = the entry (block | inactive << 31).
 __device__ __forceinline__ void step_masks(const SelectOut &so, const uint32_t *posmap, uint32_t head,
-                                           uint32_t tail, bool clean, uint32_t lane, uint32_t r0, uint32_t v,
-                                           uint32_t &ma, uint32_t &mi) {
+                                           uint32_t tail, uint32_t lane, uint32_t r0, uint32_t v, uint32_t &ma,
+                                           uint32_t &mi) {
   const uint32_t p = head + r0 + lane;
   const uint32_t w = (r0 >> 5) < POS_WORDS ? posmap[r0 >> 5] : 0xFFFFFFFFu;  // beyond the map: never reached
   bool el = p < tail && !((w >> lane) & 1u);
-  if (!clean && el) {
+  if (el) {
     const uint32_t b = v & 0x7FFFFFFFu;
     el = __ldg(&so.frame_of[b]) != NONE && __ldg(&so.stamp_of[b]) == __ldcg(so.lrm_stamp + p);
   }
@@ -285,58 +612,41 @@ __device__ __forceinline__ void step_masks(const SelectOut &so, const uint32_t *
 
 constexpr uint32_t FB = 8;  // warp steps with their entry loads in flight together
 
-__global__ void __launch_bounds__(WSEL_NT, 6) k_select_fast(PredArgs a) {
-  __shared__ uint32_t kern[MAXN + 1], roff[MAXN + 2], loff[MAXN + 2], goff[MAXN + 2];
+__global__ void __launch_bounds__(WSEL_NT) k_select_stale(PredArgs a) {
+  __shared__ uint32_t kern[MAXN + 1], roff[MAXN + 2];
   __shared__ uint32_t posmap[POS_WORDS];
   __shared__ uint32_t seg_cnt[FSEG_MAX], seg_pre[FSEG_MAX];
-  __shared__ uint32_t wem[POS_WORDS], wim[POS_WORDS], wpre[POS_WORDS];  // clean-log word path
-  __shared__ uint32_t s_need, s_head, s_tail, s_clean, s_ok, s_tw, s_ti, s_nres;
-  __shared__ unsigned long long s_bwb, s_binv;
+  __shared__ uint32_t s_tw, s_ti;
   constexpr uint32_t NW = WSEL_NT / 32;
   const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const Geo &g = a.g;
   const SelectOut &so = a.so;
-  // the fast queries, class by class (k_chain: by decreasing `need`)
-  uint32_t ccnt[NQCLS];
+  if (!*(const volatile uint32_t *)&a.st->log_dirty) return;  // k_select_fast's case
+  uint32_t ccnt[NQCLS], nfast = 0;
 #pragma unroll
-  for (int c = 0; c < NQCLS; ++c) ccnt[c] = *(volatile uint32_t *)&a.st->q_cls[c];
-  uint32_t nfast = 0;
-#pragma unroll
-  for (int c = 0; c < NQCLS; ++c) nfast += ccnt[c];
+  for (int c = 0; c < NQCLS; ++c) {
+    ccnt[c] = *(const volatile uint32_t *)&a.st->q_cls[c];
+    nfast += ccnt[c];
+  }
+  const uint32_t head = *(const volatile uint32_t *)&a.st->lrm_head;
+  const uint32_t tail = *(const volatile uint32_t *)&a.st->lrm_tail;
+  const uint32_t stale = tail - head - *(const volatile uint32_t *)&a.st->n_resident;
   for (uint32_t bq = blockIdx.x; bq < nfast; bq += gridDim.x) {
-    uint32_t cq = NQCLS, rq = bq;
-#pragma unroll
-    for (int c = 0; c < NQCLS; ++c)
-      if (cq == NQCLS) {
-        if (rq < ccnt[c]) cq = c;
-        else rq -= ccnt[c];
-      }
-    const uint32_t qi = a.qperm[(uint64_t)cq * a.nq + rq];
-    const uint32_t nk = a.qnk[qi];
+    const uint32_t qi = fast_query(a, ccnt, bq);
+    const uint32_t nk = __ldg(a.qnk + qi);
     for (uint32_t d = tid; d <= nk; d += WSEL_NT) {
-      roff[d] = a.qroff[(uint64_t)qi * (g.N + 2) + d];
-      loff[d] = a.qloff[(uint64_t)qi * (g.N + 2) + d];
-      goff[d] = a.qgoff[(uint64_t)qi * (g.N + 2) + d];
-      if (d < nk) kern[d] = a.qkern[(uint64_t)qi * (g.N + 1) + d];
+      roff[d] = __ldg(a.qroff + (uint64_t)qi * (g.N + 2) + d);
+      if (d < nk) kern[d] = __ldg(a.qkern + (uint64_t)qi * (g.N + 1) + d);
     }
     for (uint32_t w = tid; w < POS_WORDS; w += WSEL_NT) posmap[w] = 0;
     if (tid == 0) {
-      const uint32_t need = a.qneed[qi];
-      s_need = need;
-      s_bwb = a.qvb[2 * qi];
-      s_binv = a.qvb[2 * qi + 1];
-      s_ok = s_bwb + need <= so.cap && s_binv + need <= so.cap;
-      s_head = *(volatile uint32_t *)&a.st->lrm_head;
-      s_tail = *(volatile uint32_t *)&a.st->lrm_tail;
-      s_clean = *(volatile uint32_t *)&a.st->log_dirty == 0;
-      s_nres = *(volatile uint32_t *)&a.st->n_resident;
       s_tw = 0;
       s_ti = 0;
     }
+    const uint32_t need = __ldg(a.qneed + qi);
+    const unsigned long long bwb = __ldg(a.qvb + 2 * qi), binv = __ldg(a.qvb + 2 * qi + 1);
+    const bool ok = bwb + need <= so.cap && binv + need <= so.cap;
     __syncthreads();
-    const uint32_t need = s_need, head = s_head, tail = s_tail;
-    const bool clean = s_clean, ok = s_ok;
-    const unsigned long long bwb = s_bwb, binv = s_binv;
     const uint32_t R = nk ? roff[nk] : 0;
     uint32_t nseg = 0;
     if (need) {
@@ -360,104 +670,7 @@ __global__ void __launch_bounds__(WSEL_NT, 6) k_select_fast(PredArgs a) {
             if (r[u] < POS_WORDS * 32) atomicOr(&posmap[r[u] >> 5], 1u << (r[u] & 31));
         }
       }
-      const uint32_t stale = tail - head - s_nres;
       const uint32_t span = min(tail - head, min(need + R + stale, POS_WORDS * 32));
-      __syncthreads();
-      if (clean && a.inact_bits) {
-        // ---- clean log: word-level selection.  Every entry of [head, tail) is
-        // valid, so a 32-position word's eligible entries are ~excluded & valid,
-        // split by the log's inactive-entry bitmap (k_log_bits): counts and
-        // ranks come from popcounts; only the taken entries are read. ----
-        const uint32_t nw = (span + 31) / 32;
-        uint32_t ca[4], ci[4], em[4], imk[4];
-        uint32_t tot = 0;
-#pragma unroll
-        for (uint32_t u = 0; u < 4; ++u) {  // thread t owns words 4t .. 4t+3 (nw <= POS_WORDS = 4 * WSEL_NT)
-          const uint32_t w = 4 * tid + u;
-          em[u] = imk[u] = 0;
-          if (w < nw) {
-            const uint32_t lo = w * 32, valid = span - lo >= 32 ? 0xFFFFFFFFu : (1u << (span - lo)) - 1u;
-            const uint32_t ib = __ldg(a.inact_bits + w);
-            const uint32_t e = valid & ~posmap[w];
-            em[u] = e & ~ib;
-            imk[u] = e & ib;
-          }
-          ca[u] = __popc(em[u]);
-          ci[u] = __popc(imk[u]);
-          tot += ca[u] | (ci[u] << 16);
-        }
-        uint32_t tsum;
-        const uint32_t tpre = block_excl_scan(tot, seg_pre, &tsum);  // packed (inactive << 16 | active)
-        {
-          uint32_t pre = tpre;
-#pragma unroll
-          for (uint32_t u = 0; u < 4; ++u) {
-            const uint32_t w = 4 * tid + u;
-            if (w < nw) {
-              wem[w] = em[u];
-              wim[w] = imk[u];
-              wpre[w] = pre;
-            }
-            pre += ca[u] | (ci[u] << 16);
-          }
-        }
-        __syncthreads();
-        // a warp per 128-position chunk (4 words), a lane per 4 consecutive
-        // positions: the eligible entries of combined rank < need, written at
-        // their list ranks.  head is 16 B aligned for the vector load when
-        // possible; otherwise 4 scalar loads.
-        uint32_t tw = 0, ti = 0;
-        const uint32_t nch = (nw + 3) / 4;
-        const bool al = (head & 3u) == 0;
-        for (uint32_t ch = wid; ch < nch; ch += NW) {
-          const uint32_t w = 4 * ch + (lane >> 3), sh = (lane & 7) * 4;
-          const uint32_t pre = w < nw ? wpre[w] : 0xFFFFFFFFu;
-          const uint32_t pre0 = __shfl_sync(0xffffffffu, pre, 0);
-          if ((pre0 & 0xFFFFu) + (pre0 >> 16) >= need) break;  // chunks only grow: the cut is behind
-          const uint32_t a4 = w < nw ? (wem[w] >> sh) & 0xFu : 0u, i4 = w < nw ? (wim[w] >> sh) & 0xFu : 0u;
-          // ranks: the word's prefix + the eligible entries of the lower lanes of the same word
-          uint32_t c = __popc(a4) | (__popc(i4) << 16), x = c;
-#pragma unroll
-          for (int o = 1; o < 8; o <<= 1) {
-            const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-            if ((lane & 7) >= (uint32_t)o) x += y;
-          }
-          uint32_t ra = (pre & 0xFFFFu) + ((x - c) & 0xFFFFu), rr = (pre >> 16) + ((x - c) >> 16);
-          if ((a4 | i4) && ra + rr < need) {
-            const uint32_t p = head + 32 * w + sh;
-            uint32_t vv[4];
-            if (al) {
-              const uint4 q = __ldcg(reinterpret_cast<const uint4 *>(so.lrm_blk + p));
-              vv[0] = q.x; vv[1] = q.y; vv[2] = q.z; vv[3] = q.w;
-            } else {
-#pragma unroll
-              for (uint32_t u = 0; u < 4; ++u) vv[u] = ((a4 | i4) >> u) & 1u ? __ldcg(so.lrm_blk + p + u) : 0u;
-            }
-#pragma unroll
-            for (uint32_t u = 0; u < 4; ++u) {
-              const bool ea = (a4 >> u) & 1u, ei = (i4 >> u) & 1u;
-              if ((ea || ei) && ra + rr < need) {
-                if (ok) {
-                  if (ei) so.inv[binv + rr] = vv[u] & 0x7FFFFFFFu;
-                  else so.wb[bwb + ra] = vv[u];
-                }
-                tw += ea;
-                ti += ei;
-              }
-              ra += ea;
-              rr += ei;
-            }
-          }
-        }
-        tw = __reduce_add_sync(0xffffffffu, tw);
-        ti = __reduce_add_sync(0xffffffffu, ti);
-        if (lane == 0 && (tw | ti)) {
-          atomicAdd(&s_tw, tw);
-          atomicAdd(&s_ti, ti);
-        }
-        nseg = (span + FSEG - 1) / FSEG;  // (reported as scanned)
-        __syncthreads();
-      } else {
       // segments of FSEG positions relative to head; a warp step covers 32
       nseg = (span + FSEG - 1) / FSEG;
       __syncthreads();
@@ -474,7 +687,7 @@ __global__ void __launch_bounds__(WSEL_NT, 6) k_select_fast(PredArgs a) {
 #pragma unroll
           for (uint32_t u = 0; u < FB; ++u) {
             uint32_t ma, mi;
-            step_masks(so, posmap, head, tail, clean, lane, sg * FSEG + 32 * (k0 + u), v[u], ma, mi);
+            step_masks(so, posmap, head, tail, lane, sg * FSEG + 32 * (k0 + u), v[u], ma, mi);
             na += __popc(ma);
             ni += __popc(mi);
           }
@@ -510,7 +723,7 @@ __global__ void __launch_bounds__(WSEL_NT, 6) k_select_fast(PredArgs a) {
 #pragma unroll
           for (uint32_t u = 0; u < FB; ++u) {
             uint32_t ma, mi;
-            step_masks(so, posmap, head, tail, clean, lane, sg * FSEG + 32 * (k0 + u), v[u], ma, mi);
+            step_masks(so, posmap, head, tail, lane, sg * FSEG + 32 * (k0 + u), v[u], ma, mi);
             const uint32_t ra = rw + __popc(ma & lt), rr = ri + __popc(mi & lt);
             const bool ea = (ma >> lane) & 1u, ei = (mi >> lane) & 1u;
             if ((ea || ei) && ra + rr < need) {
@@ -533,7 +746,6 @@ __global__ void __launch_bounds__(WSEL_NT, 6) k_select_fast(PredArgs a) {
         atomicAdd(&s_ti, ti);
       }
       __syncthreads();
-      }  // per-entry path (stale log entries)
     }
     if (tid == 0) {
       uint64_t *o = so.out_range + 4ull * qi;
@@ -542,21 +754,9 @@ __global__ void __launch_bounds__(WSEL_NT, 6) k_select_fast(PredArgs a) {
       o[2] = binv;
       o[3] = binv + (ok ? s_ti : 0);
       // log entries read by the selection: the segments (each pass reads them)
-      ctr_add(a.st, DUM_CTR_FAST_SCANNED, need ? min(tail - head, nseg * FSEG) : 0u);  // (both passes read these)
+      ctr_add(a.st, DUM_CTR_FAST_SCANNED, need ? min(tail - head, nseg * FSEG) : 0u);
       ctr_add(a.st, DUM_CTR_FAST_VICTIMS, s_tw + s_ti);
-      if (!clean) ctr_add(a.st, DUM_CTR_FAST_DIRTY, 1);
-    }
-    // the window's (block, exec) pairs: every warp streams the lists (the copy
-    // of this query overlaps the selection of the SM's other queries)
-    {
-      const unsigned long long base = a.qbase[qi];
-      const uint32_t U = nk ? loff[nk] : 0;
-      if (base + U <= a.cap) copy_window_lists(a, kern, loff, goff, nk, base, wid, NW, loff, nullptr);
-      if (tid == 0) {
-        ctr_add(a.st, DUM_CTR_EMITTED, U);
-        ctr_add(a.st, DUM_CTR_GATHERED, U);
-        ctr_add(a.st, DUM_CTR_FAST_EMITTED, U);
-      }
+      ctr_add(a.st, DUM_CTR_FAST_DIRTY, 1);
     }
     __syncthreads();  // the next query reuses the shared state
   }
@@ -610,23 +810,40 @@ cudaError_t launch_walk_res(dum_engine *e, cudaStream_t s) {
 }
 
 cudaError_t launch_window(dum_engine *e, const PredArgs &a, bool select, cudaStream_t s) {
-  if (!e->copy_grid) {
-    int dev = 0, sms = 148, nc = 1, ns = 1;
+  const int ssmem = (int)(sel_smem_words(e->g.N) * 4);
+  if (!e->copy_grid || e->sel_smem != ssmem) {
+    int dev = 0, sms = 148, nc = 1, ns = 1, nt = 1;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    // the attribute is per device and function: raised by every engine on its own device
+    if (ssmem > 48 * 1024) cudaFuncSetAttribute(k_select_fast, cudaFuncAttributeMaxDynamicSharedMemorySize, ssmem);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nc, k_copy_fast, COPY_NT, 0);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ns, k_select_fast, WSEL_NT, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ns, k_select_fast, WSEL_NT, ssmem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nt, k_select_stale, WSEL_NT, 0);
     e->copy_grid = (uint32_t)std::max(1, nc * sms);
     e->sel_grid = (uint32_t)std::max(1, ns * sms);
+    e->stale_grid = (uint32_t)std::max(1, nt * sms);
+    e->sel_smem = ssmem;
   }
-  if (!select) {  // prefetch windows only: the flat copy
+  if (select) {
+    // the selection on the third side stream, beside the copy (each kernel
+    // exits at once in the other's case: clean log / stale entries)
+    cudaEventRecord(e->ev_fork2, s);
+    cudaStreamWaitEvent(e->side3, e->ev_fork2, 0);
+    {
+      TimerScope t(e, DUM_T_SELECT_FAST, e->side3);
+      k_select_fast<<<std::min(a.nq, e->sel_grid), WSEL_NT, ssmem, e->side3>>>(a);
+      k_select_stale<<<std::min(a.nq, e->stale_grid), WSEL_NT, 0, e->side3>>>(a);
+    }
+    cudaEventRecord(e->ev_join3, e->side3);
+    e->kernel_launches += 2;
+  }
+  {  // every fast window's pairs: the flat copy over k_chain's chunk map
     TimerScope t(e, DUM_T_PREDICT, s);
     k_copy_fast<<<e->copy_grid, COPY_NT, 0, s>>>(a);
-  } else {  // one CTA per window: selection, then its pairs
-    TimerScope t(e, DUM_T_PREDICT, s);
-    k_select_fast<<<std::min(a.nq, e->sel_grid), WSEL_NT, 0, s>>>(a);
   }
   e->kernel_launches += 1;
+  if (select) cudaStreamWaitEvent(s, e->ev_join3, 0);
   return cudaGetLastError();
 }
 

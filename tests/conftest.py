@@ -19,7 +19,7 @@ def pytest_configure(config):
 # (tests/gpu_helpers.make_pair) report which code paths answered its work
 # (DUM_CTR_Q_*, DUM_CTR_WALK_*, ...); the totals are written at session end
 # to gpurun_out/path_counters.json (or $DUM_PATHS_OUT) and checked by
-# test_gpu_paths.py::test_every_path_taken_in_the_suite when it runs last.
+# test_gpu_zz_paths.py::test_every_path_taken_in_the_suite (runs last).
 # ---------------------------------------------------------------------------
 import collections  # noqa: E402
 import json  # noqa: E402
@@ -27,7 +27,7 @@ import json  # noqa: E402
 import pytest  # noqa: E402
 
 PATHS = ["Q_FAST", "Q_NODUP", "Q_DUP", "Q_FALLBACK", "WALK_PREFIX", "WALK_DEDUPE", "WALK_SLOW", "ANCHOR_WALKS",
-         "INGEST_DUP", "Q_SLOW"]
+         "INGEST_DUP", "Q_SLOW", "FAST_DIRTY"]
 PATH_TOTALS = collections.Counter()
 PATH_BY_TEST = {}
 

@@ -134,6 +134,38 @@ def test_block_ids_near_limit_and_fmix_index():
     assert_same_predictions(ro, rg)
 
 
+
+@pytest.mark.parametrize("dup_frac", [0.0, 0.05])
+def test_big_launches_hashed_ingest_bitmap(dup_frac):
+    """W = 2^20: big launches (> 1024 records) dedupe through a hashed
+    shared-memory bitmap; shared bits are only candidates, settled by the
+    min-position hash (D2: first occurrence kept, order preserved).  The
+    12000-record launch has more candidates than that hash holds and takes
+    the global-pool path."""
+    W = 1 << 20
+    rng = np.random.default_rng(11 + int(100 * dup_frac))
+    eng, o = make_pair(R=64, A=2, S=4, W=W, C=64, N=4)
+    sizes = [1500, 3000, 4000, 12000, 700, 3345]
+    lists = []
+    for n in sizes:
+        x = rng.choice(W, n, replace=False)
+        k = int(dup_frac * n)
+        if k:
+            x[rng.integers(1, n, k)] = x[rng.integers(0, n // 2, k)]
+        lists.append([int(v) for v in x])
+    lists.append(list(range(5000, 7000)) + list(range(5000 + W // 2, 6000 + W // 2)))  # runs, far regions
+    h = np.array([wl.fnv1a64(b"big%d" % (i % 3)) for i in range(len(lists))], dtype=np.uint64)
+    off = np.zeros(len(lists) + 1, dtype=np.uint64)
+    off[1:] = np.cumsum([len(x) for x in lists])
+    f = np.array([b for x in lists for b in x], dtype=np.uint32)
+    exo, exg = record_both(eng, o, h, off, f)
+    assert np.array_equal(exo, exg)
+    build_both(eng, o)
+    assert_same_state(eng, o)
+    c = eng.counters()
+    assert c["NORM_RECORDS"] == sum(len(dict.fromkeys(x)) for x in lists)
+    assert (c["INGEST_DUP"] > 0) == (dup_frac > 0)
+
 def test_hash_sentinel_and_collisions():
     """Two launches with the same hash share an ID; the all-ones hash is a
     legal key (D3)."""
@@ -396,3 +428,60 @@ def test_dum_step_equals_the_separate_calls(host, graph):
             assert np.array_equal(gwb[sr[q, 0]:sr[q, 1]], wb_o[wo[q]:wo[q + 1]]), (i, q)
             assert np.array_equal(giv[sr[q, 2]:sr[q, 3]], iv_o[io[q]:io[q + 1]]), (i, q)
     assert_same_state(eng, o)
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_fast_selection_on_a_log_with_stale_entries(seed):
+    """Write-backs leave stale entries in the LRM log (PAPER.md L238-L241:
+    the victims are resident blocks; a logged block that left HBM is skipped)
+    until the next compaction: the fast path's per-entry selection
+    (k_select_fast) must give the oracle's victims.  The clean-log path
+    (k_select_warp) answers the same queries after the log is reloaded."""
+    W, C = 96, 40
+    rng = np.random.default_rng(77 + seed)
+    arena = torch.zeros(W * (2 << 20), dtype=torch.uint8).pin_memory()
+    pool = torch.zeros(C * (2 << 20), dtype=torch.uint8, device="cuda")
+    eng, o = make_pair(R=16, A=2, S=4, W=W, C=C, N=6, host_arena=arena, frame_pool=pool)
+    # kernels with disjoint block ranges (16 blocks each): their walks share no
+    # block, so the windows take the fast path
+    ex_all = []
+    for _ in range(3):
+        ks = [k % 6 for k in range(30)]
+        h = np.array([wl.fnv1a64(b"dk%d" % k) for k in ks], dtype=np.uint64)
+        lists = [[16 * k + int(x) for x in rng.permutation(16)[: int(rng.integers(4, 17))]] for k in ks]
+        off = np.zeros(len(ks) + 1, dtype=np.uint64)
+        off[1:] = np.cumsum([len(x) for x in lists])
+        f = np.array([b for x in lists for b in x], dtype=np.uint32)
+        exo, exg = record_both(eng, o, h, off, f)
+        assert np.array_equal(exo, exg)
+        ex_all += [int(x) for x in exo]
+    build_both(eng, o)
+    qs = transition_queries(ex_all, 0, len(ex_all), 6)
+    inact = rng.permutation(W)[: W // 3].astype(np.uint32)
+    o.mark_inactive(inact, True)
+    eng.mark_inactive(dev(inact), True)
+    snap = rng.permutation(W)[:C].astype(np.uint32)
+    o.load_residency(snap)
+    eng.load_residency(dev(snap))
+    # write back blocks from the middle of the log, then fault others in
+    for d, blocks in ((B.D2H, snap[3:15:2]), (B.H2D, [b for b in rng.permutation(W) if b not in set(snap)][:4])):
+        blocks = np.asarray(blocks, np.uint32)
+        assert o.migrate(d, blocks) == 0
+        eng.migrate_blocks(d, dev(blocks))
+        eng.sync()
+    assert eng.dump_state(orc.RES) == o.dump(orc.RES)
+    c0 = eng.counters()
+    fused_both(eng, o, qs)
+    c1 = eng.counters()
+    assert c1.get("FAST_DIRTY", 0) > c0.get("FAST_DIRTY", 0), "the stale-entry path did not run"
+    # the same queries on a compacted (clean) log: the live entries, log order
+    rs = orc.parse_dump(o.dump(orc.RES), orc.RES, 0, 1, 1, 1)
+    live = set(int(b) for b in rs["block_of_frame"] if b != orc.NONE)
+    res = np.asarray([b for b in rs["lrm"] if (int(b) & 0x7FFFFFFF) in live], np.uint32) & 0x7FFFFFFF
+    assert len(res) == len(live)
+    o.load_residency(res)
+    eng.load_residency(dev(res))
+    c0 = eng.counters()
+    fused_both(eng, o, qs)
+    c1 = eng.counters()
+    assert c1["Q_FAST"] > c0["Q_FAST"] and c1["FAST_DIRTY"] == c0["FAST_DIRTY"]
