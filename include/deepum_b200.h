@@ -272,6 +272,11 @@ int dum_load_residency(dum_engine *eng, const uint32_t *lrm_blocks, uint32_t n_r
 typedef enum { DUM_H2D = 0, DUM_D2H = 1, DUM_INVALIDATE = 2, DUM_D2D = 3 } dum_dir;
 int dum_migrate_blocks(dum_engine *eng, dum_dir dir, const uint32_t *blocks_or_src, const uint32_t *dst_frames,
                        uint32_t n, uint32_t method, dum_stream_t stream);
+/* The copy kernels (methods 0, 1, 3) of this engine use at most n_sms SMs'
+ * worth of CTAs (0 = every SM, the default): two engines whose copies run
+ * concurrently -- write-back on one, fetch on another -- each take a share
+ * instead of queueing behind each other.  No synchronization. */
+int dum_set_copy_sms(dum_engine *eng, uint32_t n_sms);
 
 /* ---- closed-loop replay ------------------------------
  * dum_simulate replays launches 0 .. n_launch-1 (launch k has hash
@@ -285,7 +290,10 @@ int dum_migrate_blocks(dum_engine *eng, dum_dir dir, const uint32_t *blocks_or_s
  * the next launch (its exec ID if its hash is known, the last three exec IDs
  * as history, degree n) -> (DUM_SIM_PREEVICT) pre-eviction of the window's
  * victims (L236-L243) -> H2D of the window's non-resident prefix that fits the
- * free frames (L156-L158).  Every step runs in this library's kernels, list
+ * free frames (L156-L158); without DUM_SIM_PREEVICT every non-resident window
+ * block is prefetched and the driver evicts the least recently migrated
+ * blocks, window or not, for those beyond the free frames (L236-L238; the
+ * evictions are reported as pre_wb / pre_inv).  Every step runs in this library's kernels, list
  * sizes stay on the device.  Without a data plane the migrations move the
  * residency only (metadata-only engine: B/G scale); with one the bytes move.
  * Per-launch statistics go to stats[k] (device).  launch_hash, acc_blk, stats:
@@ -295,8 +303,8 @@ typedef struct {
   uint32_t faults;      /* demand faults of the launch (blocks migrated on demand) */
   uint32_t demand_wb;   /* demand-path victims written back */
   uint32_t demand_inv;  /* demand-path victims invalidated (D20) */
-  uint32_t pre_wb;      /* pre-evicted blocks written back */
-  uint32_t pre_inv;     /* pre-evicted blocks invalidated */
+  uint32_t pre_wb;      /* pre-evicted (prefetch only: driver-evicted) blocks written back */
+  uint32_t pre_inv;     /* pre-evicted (prefetch only: driver-evicted) blocks invalidated */
   uint32_t prefetched;  /* window blocks migrated ahead of use */
 } dum_sim_stats;
 #define DUM_SIM_PREFETCH 0x1u   /* query + prefetch the window (else naive UM: demand only) */

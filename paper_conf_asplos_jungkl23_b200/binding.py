@@ -40,7 +40,10 @@ KERNEL_OF_TIMER = {"INGEST": "k_ingest", "EXEC_ASSIGN": "k_exec_assign", "BUILD_
                    "WALK_RES": "k_walk_res"}
 # timers of kernels launched on the engine's side streams (overlapping others)
 SIDE_TIMERS = {"JUMP": "side stream, overlaps k_apply / k_walk (k_jump0 + k_jumpk levels)",
-               "EXACT": "second side stream, beside the fast path (exact-path queries)"}
+               "EXACT": "second side stream, beside the fast path (exact-path queries)",
+               "SELECT_FAST": "third side stream, beside k_copy_fast (fast-path selection: k_select_fast + k_select_stale)",
+               "WALK_RES": "ingest-side fork in dum_step (beside k_ingest .. k_anchor_walk)",
+               "WALK_INDEX": "third side stream after the build (replayed step graphs: at the start of the next step, beside its ingest)"}
 _ERR = {0: "DUM_OK", -1: "DUM_EINVAL", -2: "DUM_ECAPACITY", -3: "DUM_ENOMEM", -4: "DUM_ECUDA", -5: "DUM_ESTATE"}
 
 
@@ -109,6 +112,7 @@ def load_library() -> ctypes.CDLL:
         "dum_kernel_launches": (U64, [P]),
         "dum_read_counters": (I, [P, P, I]),
         "dum_set_counting": (I, [P, I]),
+        "dum_set_copy_sms": (I, [P, ctypes.c_uint32]),
         "dum_set_timing": (I, [P, I]),
         "dum_host_ptr_kind": (I, [P]),
         "dum_read_timing": (I, [P, P, P, I]),
@@ -408,6 +412,10 @@ class Engine:
     def counters(self, reset: bool = False) -> dict:
         c = self.read_counters(reset)
         return {k: int(c[v]) for k, v in CTR.items()}
+
+    def set_copy_sms(self, n_sms: int):
+        """Cap the copy kernels of this engine at n_sms SMs' worth of CTAs (0 = all)."""
+        self._ck(self.lib.dum_set_copy_sms(self._h, int(n_sms)), "dum_set_copy_sms")
 
     def set_timing(self, on: bool):
         self._ck(self.lib.dum_set_timing(self._h, 1 if on else 0), "dum_set_timing")

@@ -301,10 +301,11 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_wrun, 2ull * g.Emax * g.walk_cap));
   A_(dmalloc(&e->d_wrun_len, g.Emax));
   // host-pointer inputs are uploaded here on the ingest stream (in order with
-  // the ingest that reads them)
-  A_(dmalloc(&e->d_in_hash, e->stage_launch_cap));
-  A_(dmalloc(&e->d_in_off, e->stage_launch_cap + 1ull));
-  A_(dmalloc(&e->d_in_faults, e->stage_fault_cap));
+  // the ingest that reads them), one buffer per staging set: the upload of
+  // batch i+1 overlaps the work on batch i
+  A_(dmalloc(&e->d_in_hash, 2ull * e->stage_launch_cap));
+  A_(dmalloc(&e->d_in_off, 2ull * (e->stage_launch_cap + 1ull)));
+  A_(dmalloc(&e->d_in_faults, 2ull * e->stage_fault_cap));
   A_(cudaStreamCreateWithFlags(&e->rec_s, cudaStreamNonBlocking));
   A_(cudaEventCreateWithFlags(&e->ev_rec, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_s_now, cudaEventDisableTiming));
@@ -479,9 +480,9 @@ int dum_record_faults(dum_engine *e, const uint64_t *launch_hash, const uint64_t
   }
   CK(cudaStreamWaitEvent(r, e->ev_stage_free[e->stage_set], 0));
   if (flags & DUM_HOST_PTRS) {
-    uint64_t *dh = e->d_in_hash;
-    uint64_t *doff = e->d_in_off;
-    uint32_t *df = e->d_in_faults;
+    uint64_t *dh = in_hash(e);
+    uint64_t *doff = in_off(e);
+    uint32_t *df = in_faults(e);
     CK(cudaMemcpyAsync(dh, launch_hash, 8ull * n_launch, cudaMemcpyHostToDevice, r));
     CK(cudaMemcpyAsync(doff, launch_off, 8ull * (n_launch + 1), cudaMemcpyHostToDevice, r));
     if (n_fault) CK(cudaMemcpyAsync(df, fault_block, 4ull * n_fault, cudaMemcpyHostToDevice, r));
@@ -567,15 +568,21 @@ static int step_graph(dum_engine *e, const uint64_t *launch_hash, const uint64_t
     for (uint32_t i = 0; i < n_launch; ++i)
       if (launch_off[i + 1] < launch_off[i]) return fail(e, DUM_EINVAL, "launch_off not monotone");
   }
-  // the batch into the fixed upload buffers (stream-ordered before the replay)
-  CK(cudaMemcpyAsync(e->d_in_hash, launch_hash, 8ull * n_launch, kind, s));
-  CK(cudaMemcpyAsync(e->d_in_off, launch_off, 8ull * (n_launch + 1), kind, s));
-  if (n_fault) CK(cudaMemcpyAsync(e->d_in_faults, fault_block, 4ull * n_fault, kind, s));
-  // the graph runs on the engine's own (capturable, non-blocking) stream, ordered
-  // after the caller's stream and before it again
+  // the batch into this staging set's upload buffers, on the record stream:
+  // after the replay that last read them (two steps ago) -- and, for device
+  // inputs, after the caller's stream -- so that it overlaps the previous step
   cudaStream_t caller = s;
-  s = e->graph_s;
+  const int set = e->stage_set;
   CK(cudaEventRecord(e->ev_s_now, caller));
+  if (!(flags & DUM_HOST_PTRS)) CK(cudaStreamWaitEvent(e->rec_s, e->ev_s_now, 0));
+  CK(cudaStreamWaitEvent(e->rec_s, e->ev_stage_free[set], 0));
+  CK(cudaMemcpyAsync(in_hash(e), launch_hash, 8ull * n_launch, kind, e->rec_s));
+  CK(cudaMemcpyAsync(in_off(e), launch_off, 8ull * (n_launch + 1), kind, e->rec_s));
+  if (n_fault) CK(cudaMemcpyAsync(in_faults(e), fault_block, 4ull * n_fault, kind, e->rec_s));
+  CK(cudaEventRecord(e->ev_rec, e->rec_s));
+  // the graph runs on the engine's own (capturable, non-blocking) stream, ordered
+  // after the caller's stream (and the upload) and before it again
+  s = e->graph_s;
   CK(cudaStreamWaitEvent(s, e->ev_s_now, 0));
   // side-stream work of an earlier uncaptured call (jump tables, walk index,
   // predict's side kernels) is finished before the graph starts
@@ -628,7 +635,7 @@ static int step_graph(dum_engine *e, const uint64_t *launch_hash, const uint64_t
     if (err == cudaSuccess) err = launch_walk_index(e, s);
     if (err == cudaSuccess) err = fork_walk_res(e, s);
     if (err == cudaSuccess)
-      err = launch_record(e, e->d_in_hash, e->d_in_off, n_launch, e->d_in_faults, e->stage_fault_cap,
+      err = launch_record(e, in_hash(e), in_off(e), n_launch, in_faults(e), e->stage_fault_cap,
                           e->d_step_exec + 3, s);
     if (err == cudaSuccess) err = launch_make_queries(e, e->d_step_exec, 3 + n_launch, 3, degree, e->d_step_q, s);
     if (err == cudaSuccess)
@@ -672,6 +679,7 @@ static int step_graph(dum_engine *e, const uint64_t *launch_hash, const uint64_t
   CK(cudaGraphLaunch(exec, s));
   e->widx_stale = true;  // the replayed build's walk index is built by the next step
   CK(cudaEventRecord(e->ev_graph, s));
+  CK(cudaEventRecord(e->ev_stage_free[set], s));  // this set's staging and upload buffers are free again
   CK(cudaStreamWaitEvent(caller, e->ev_graph, 0));
   // host bookkeeping of the replayed step (as dum_record_faults + dum_build_tables)
   e->launches += n_launch;
@@ -882,6 +890,12 @@ int dum_read_counters(dum_engine *e, uint64_t out[DUM_NCOUNTERS], int reset) {
   CK(cudaDeviceSynchronize());
   CK(cudaMemcpy(out, e->d_state->ctr, sizeof(uint64_t) * DUM_NCOUNTERS, cudaMemcpyDeviceToHost));
   if (reset) CK(cudaMemset(e->d_state->ctr, 0, sizeof(uint64_t) * DUM_NCOUNTERS));
+  return DUM_OK;
+}
+
+int dum_set_copy_sms(dum_engine *e, uint32_t n_sms) {
+  if (!e) return DUM_EINVAL;
+  e->copy_sms = n_sms;
   return DUM_OK;
 }
 

@@ -150,7 +150,7 @@ struct dum_engine {
   // staging
   uint32_t stage_launch_cap;
   uint64_t stage_fault_cap;
-  uint64_t *d_in_hash, *d_in_off;   // host-pointer inputs are uploaded here (on rec_s)
+  uint64_t *d_in_hash, *d_in_off;   // host-pointer inputs are uploaded here (on rec_s), two sets
   // record_faults runs on its own stream so that the next batch's ingest
   // overlaps the current build; the staging arrays alternate between two sets
   cudaStream_t rec_s;
@@ -247,6 +247,7 @@ struct dum_engine {
   int sel_smem;                              // k_select_fast dynamic shared memory (k_window.cu)
   int chain_smem;                  // k_chain dynamic smem attribute applied
   int bulk_smem;                   // k_copy_bulk dynamic smem attribute applied
+  uint32_t copy_sms;               // copy kernels: SMs' worth of CTAs (0 = all; dum_set_copy_sms)
   // dum_step as a replayed CUDA graph (dum_set_step_graphs)
   bool graph_steps, capturing, step_warm;
   cudaStream_t graph_s;        // the step graphs are captured and replayed here
@@ -261,3 +262,10 @@ struct dum_engine {
   };
   std::vector<StepGraph> step_graphs;  // dynamic smem attributes applied (per engine / device)
 };
+
+// this staging set's upload buffers for host-pointer / step inputs
+inline uint64_t *in_hash(const dum_engine *e) { return e->d_in_hash + (uint64_t)e->stage_set * e->stage_launch_cap; }
+inline uint64_t *in_off(const dum_engine *e) {
+  return e->d_in_off + (uint64_t)e->stage_set * (e->stage_launch_cap + 1ull);
+}
+inline uint32_t *in_faults(const dum_engine *e) { return e->d_in_faults + (uint64_t)e->stage_set * e->stage_fault_cap; }

@@ -490,10 +490,15 @@ cudaError_t launch_mark_inactive(dum_engine *e, const uint32_t *blocks, uint32_t
   return cudaGetLastError();
 }
 
-static int copy_grid(uint32_t n) {
+static int copy_sms(const dum_engine *e) {
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  return e->copy_sms && (int)e->copy_sms < sms ? (int)e->copy_sms : sms;
+}
+
+static int copy_grid(const dum_engine *e, uint32_t n) {
+  const int sms = copy_sms(e);
   const uint64_t items = (uint64_t)(n ? n : 1) * CHUNKS;
   const uint64_t g = std::min<uint64_t>(items, (uint64_t)sms * 8);
   return (int)g;
@@ -571,16 +576,14 @@ cudaError_t launch_migrate(dum_engine *e, int dir, const uint32_t *blocks, const
       cudaFuncSetAttribute(k_copy_bulk, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bsm);
       e->bulk_smem = 1;
     }
-    int dev = 0, sms = 148;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int sms = copy_sms(e);
     TimerScope t(e, DUM_T_COPY, s);
     k_copy_bulk<<<sms, 32, bsm, s>>>(dir, e->d_mig_blocks, e->d_mig_src, e->d_mig_frames, e->host_arena_dev,
                                      e->frame_pool, e->d_state);
     e->kernel_launches += 1;
     return cudaGetLastError();
   }
-  const int grid = copy_grid(compaction ? e->g.C : n);
+  const int grid = copy_grid(e, compaction ? e->g.C : n);
   TimerScope t(e, DUM_T_COPY, s);
   k_copy_blocks<<<grid, COPY_NT, 0, s>>>(dir, e->d_mig_blocks, e->d_mig_src, e->d_mig_frames, e->host_arena_dev,
                                          e->frame_pool, e->d_state);

@@ -59,7 +59,7 @@ __global__ void k_make_queries(const uint32_t *__restrict__ seq, uint32_t n_seq,
 __global__ void k_anchor_walk(Geo g, const dum_query *__restrict__ q, uint32_t nq, const uint32_t *tbl,
                               const uint32_t *start_end, uint32_t *slot_out, uint32_t *pool, uint64_t pool_cap,
                               uint64_t *range, WalkScratch ws, DevState *st) {
-  const uint32_t E = *(volatile uint32_t *)&st->E;
+  const uint32_t E = __ldcg(&st->E);
   uint32_t *out = slot_out + (uint64_t)blockIdx.x * g.walk_cap;
   const uint32_t lane = threadIdx.x & 31;
   for (uint32_t q0 = blockIdx.x * 32; q0 < nq; q0 += gridDim.x * 32) {
@@ -128,7 +128,7 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
   if (qi < a.nq) {
     const dum_query Q = a.q[qi];
     const bool anchored = Q.anchor != NONE;
-    const uint32_t E = *(volatile uint32_t *)&a.st->E;
+    const uint32_t E = __ldcg(&a.st->E);
     uint32_t *kern = skern[w];
     uint32_t nk = 0;
     if (Q.exec < E) {
@@ -260,10 +260,10 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
       // need = max(0, window blocks without a frame - free frames) (D18);
       // k_window's selection scans log positions [head, head + need + nwres +
       // stale entries) at most: it must stay inside its position bitmap
-      const uint32_t nfree = *(volatile uint32_t *)&a.st->free_count;
+      const uint32_t nfree = __ldcg(&a.st->free_count);
       qneed = nonres > nfree ? nonres - nfree : 0;
-      const uint32_t span = *(volatile uint32_t *)&a.st->lrm_tail - *(volatile uint32_t *)&a.st->lrm_head;
-      const uint32_t stale = span - *(volatile uint32_t *)&a.st->n_resident;
+      const uint32_t span = __ldcg(&a.st->lrm_tail) - __ldcg(&a.st->lrm_head);
+      const uint32_t stale = span - __ldcg(&a.st->n_resident);
       if ((uint64_t)qneed + nwres + stale > POS_WORDS * 32ull) {
         slow = true;
         if (lane == 0) ctr_add(a.st, DUM_CTR_SLOW_SPAN, 1);
@@ -413,7 +413,7 @@ __global__ void __launch_bounds__(PRED_NT, 2) k_predict(PredArgs a) {
   // k_chain, largest windows first; the fast path answers the others)
   uint32_t ccnt[NQCLS];
 #pragma unroll
-  for (int c = 0; c < NQCLS; ++c) ccnt[c] = *(volatile uint32_t *)&a.st->q_cls[NQCLS + c];
+  for (int c = 0; c < NQCLS; ++c) ccnt[c] = __ldcg(&a.st->q_cls[NQCLS + c]);
   uint32_t nslow = 0;
 #pragma unroll
   for (int c = 0; c < NQCLS; ++c) nslow += ccnt[c];
@@ -1011,7 +1011,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   cudaEventRecord(e->ev_fork2, s);
   cudaStreamWaitEvent(e->side2, e->ev_fork2, 0);
   const size_t smem = (size_t)((a.nwords + 3) & ~3u) * 4 + 2 * DHCAP * 4;
-  const uint32_t pgrid = std::min<uint32_t>(nq, 2 * 148);
+  const uint32_t pgrid = std::min<uint32_t>(nq, 148);  // persistent over the exact-path classes; few queries
   if (sel) {
     // the attribute is per device and function: raised by every engine on its own device
     if ((int)smem > e->select_smem) {

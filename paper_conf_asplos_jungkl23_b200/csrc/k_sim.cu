@@ -18,7 +18,12 @@
 //   5. transition query for the next launch (its exec ID if its hash is
 //      known; the last three exec IDs as history)             (a7)
 //   6. pre-eviction of the window (DUM_SIM_PREEVICT)          (a8)
-//   7. H2D of the window's non-resident prefix that fits the free frames
+//   7. H2D of the window's non-resident blocks: with pre-eviction the prefix
+//      that fits the free frames; without it (prefetch only) all of them, the
+//      driver evicting least-recently-migrated blocks for those beyond the
+//      free frames, window or not (the driver's policy
+//      "evicts pages that are least recently migrated", which is what
+//      pre-eviction avoids)
 // Without a data plane (B/G: 720 GB do not fit host memory) the migrations
 // move the residency only; with one (T) the bytes move too.  Flags select the
 // Fig. 10 ablation: no prefetch (naive UM), prefetch,
@@ -151,16 +156,16 @@ __global__ void k_sim_query(const uint64_t *hash_next, const unsigned long long 
   *q = Q;
 }
 
-// 7. the window's blocks without a frame, in window order, as many as there
-// are free frames; and the launch's statistics.
+// 7. the window's blocks without a frame, in window order: as many as there
+// are free frames, or (driver eviction) as there are frames.
 __global__ void __launch_bounds__(SIM_NT) k_sim_prefetch(const uint32_t *__restrict__ pairs,
                                                          const uint64_t *__restrict__ prange,
                                                          const uint32_t *__restrict__ res_bits, uint32_t *pf,
-                                                         uint64_t *pf_range, DevState *st) {
+                                                         uint64_t *pf_range, uint32_t driver_evict, DevState *st) {
   __shared__ uint32_t ws[SIM_NT / 32];
   const uint32_t tid = threadIdx.x;
   const uint64_t a = prange[0], b = prange[1];
-  const uint32_t nfree = *(volatile uint32_t *)&st->free_count;
+  const uint32_t nfree = __ldcg(&st->free_count) + (driver_evict ? __ldcg(&st->n_resident) : 0u);
   uint32_t run = 0;
   for (uint64_t c = a; c < b && run < nfree; c += SIM_NT) {
     const uint64_t i = c + tid;
@@ -180,10 +185,36 @@ __global__ void __launch_bounds__(SIM_NT) k_sim_prefetch(const uint32_t *__restr
   }
 }
 
+// 7'. prefetch only: the driver's victims for the prefetched blocks beyond the
+// free frames -- the first entries of the LRM log, no exclusion.
+struct NoneExcluded {
+  __device__ __forceinline__ uint32_t operator()(uint32_t, uint32_t) const { return 0u; }
+};
+
+__global__ void __launch_bounds__(DEM_NT) k_sim_driver_evict(SelectOut so, const uint64_t *pf_range, DevState *st) {
+  __shared__ SelShared ss;
+  __shared__ uint32_t stage[SEL_CHUNK];
+  const uint32_t tid = threadIdx.x;
+  if (tid == 0) {
+    const uint32_t npf = (uint32_t)(pf_range[1] - pf_range[0]);
+    const uint32_t nfree = __ldcg(&st->free_count);
+    const uint32_t need = npf > nfree ? npf - nfree : 0;
+    ss.need = need;
+    ss.ok = need <= so.cap;
+    ss.bwb = ss.binv = 0;
+    ss.head = __ldcg(&st->lrm_head);
+    ss.tail = __ldcg(&st->lrm_tail);
+    ss.clean = __ldcg(&st->log_dirty) == 0;
+    if (!ss.ok) set_err(st, ERR_ECAPACITY, need);
+  }
+  __syncthreads();
+  select_tail<DEM_NT, 0>(so, 0, ss, NoneExcluded{}, st, tid, stage);
+}
+
 // launch statistics from the lists' ranges; clears the launch's access set
 __global__ void k_sim_close(const uint32_t *__restrict__ acc, uint32_t n, uint32_t W, uint32_t *acc_bits,
                             const uint64_t *dem_rng, const uint64_t *pre_rng, const uint64_t *pf_range,
-                            uint32_t preevict, uint32_t prefetch, uint32_t invalidate, dum_sim_stats *stats) {
+                            uint32_t evicted, uint32_t prefetch, uint32_t invalidate, dum_sim_stats *stats) {
   const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
   for (uint32_t j = tid; j < n; j += gridDim.x * blockDim.x) {
     const uint32_t b = acc[j];
@@ -192,8 +223,9 @@ __global__ void k_sim_close(const uint32_t *__restrict__ acc, uint32_t n, uint32
   if (tid == 0) {
     // without DUM_SIM_INVALIDATE the inactive victims were written back too
     const uint32_t dw = (uint32_t)(dem_rng[1] - dem_rng[0]), di = (uint32_t)(dem_rng[3] - dem_rng[2]);
-    const uint32_t pw = preevict ? (uint32_t)(pre_rng[1] - pre_rng[0]) : 0u;
-    const uint32_t pi = preevict ? (uint32_t)(pre_rng[3] - pre_rng[2]) : 0u;
+    // pre-eviction (or, prefetch only, the driver's evictions for the prefetch)
+    const uint32_t pw = evicted ? (uint32_t)(pre_rng[1] - pre_rng[0]) : 0u;
+    const uint32_t pi = evicted ? (uint32_t)(pre_rng[3] - pre_rng[2]) : 0u;
     stats->demand_wb = invalidate ? dw : dw + di;
     stats->demand_inv = invalidate ? di : 0u;
     stats->pre_wb = invalidate ? pw : pw + pi;
@@ -292,11 +324,19 @@ cudaError_t launch_simulate(dum_engine *e, const uint64_t *hash, uint32_t n_laun
                                   r_pre + 2)) != cudaSuccess)
           return err;
       }
-      k_sim_prefetch<<<1, SIM_NT, 0, s>>>(e->sim_pairs, r_pairs, e->d_res_bits, e->sim_pf, r_pf, e->d_state);
+      k_sim_prefetch<<<1, SIM_NT, 0, s>>>(e->sim_pairs, r_pairs, e->d_res_bits, e->sim_pf, r_pf, preevict ? 0u : 1u,
+                                          e->d_state);
+      if (!preevict) {  // prefetch only: the driver evicts for the blocks beyond the free frames
+        k_sim_driver_evict<<<1, DEM_NT, 0, s>>>(pre, r_pf, e->d_state);
+        if ((err = launch_migrate(e, DUM_D2H, e->sim_wb, nullptr, g.C, 1, s, r_pre)) != cudaSuccess) return err;
+        if ((err = launch_migrate(e, invalidate ? DUM_INVALIDATE : DUM_D2H, e->sim_inv, nullptr, g.C, 1, s,
+                                  r_pre + 2)) != cudaSuccess)
+          return err;
+      }
       if ((err = launch_migrate(e, DUM_H2D, e->sim_pf, nullptr, g.C, 1, s, r_pf)) != cudaSuccess) return err;
     }
     k_sim_close<<<8, 256, 0, s>>>(acc, n, g.W, e->sim_acc_bits, r_dem, r_pre, r_pf,
-                                  (preevict && k + 1 < n_launch) ? 1u : 0u,
+                                  (prefetch && k + 1 < n_launch) ? 1u : 0u,
                                   (prefetch && k + 1 < n_launch) ? 1u : 0u, invalidate ? 1u : 0u, stats + k);
     e->kernel_launches += 8;
   }

@@ -49,7 +49,7 @@ constexpr uint32_t CONF_HCAP = 256;  // shared hash of one walk's conflicts (> C
 __global__ void __launch_bounds__(IX_NT) k_walk_count(const uint32_t *__restrict__ walk,
                                                       const uint32_t *__restrict__ walk_len, uint32_t walk_cap,
                                                       const DevState *st, uint32_t *bcnt, uint32_t *bhold) {
-  const uint32_t E = *(const volatile uint32_t *)&st->E;
+  const uint32_t E = __ldcg(&st->E);
   for (uint32_t e = blockIdx.x; e < E; e += gridDim.x) {
     const uint32_t n = walk_len[e];
     const uint32_t *w = walk + (uint64_t)e * walk_cap;
@@ -73,7 +73,7 @@ __global__ void __launch_bounds__(IX_NT) k_walk_conf(const uint32_t *__restrict_
                                                      uint32_t *conf_n) {
   __shared__ uint32_t hs[CONF_HCAP];
   __shared__ uint32_t s_n, s_ovf;
-  const uint32_t E = *(const volatile uint32_t *)&st->E;
+  const uint32_t E = __ldcg(&st->E);
   const uint32_t tid = threadIdx.x;
   for (uint32_t e = blockIdx.x; e < E; e += gridDim.x) {
     for (uint32_t k = tid; k < CONF_HCAP; k += IX_NT) hs[k] = NONE;
@@ -141,7 +141,7 @@ __global__ void __launch_bounds__(IX_NT) k_walk_res(const uint32_t *__restrict__
                                                     const uint32_t *__restrict__ logpos, uint32_t *wnr,
                                                     uint32_t *wnres, uint32_t *respos) {
   __shared__ uint32_t s_nres, s_nr;
-  const uint32_t E = *(const volatile uint32_t *)&st->E;
+  const uint32_t E = __ldcg(&st->E);
   const uint32_t tid = threadIdx.x, lane = tid & 31;
   for (uint32_t e = blockIdx.x; e < E; e += gridDim.x) {
     if (tid == 0) {
@@ -194,7 +194,7 @@ __global__ void __launch_bounds__(IX_NT) k_walk_res(const uint32_t *__restrict__
 __global__ void __launch_bounds__(COPY_NT) k_copy_fast(PredArgs a) {
   constexpr uint32_t UN = 4;  // chunks per warp step, their loads in flight together
   const uint32_t lane = threadIdx.x & 31;
-  const uint64_t G = *(volatile unsigned long long *)&a.st->pool_chunks;
+  const uint64_t G = __ldcg(&a.st->pool_chunks);
   const uint64_t nw = (uint64_t)gridDim.x * (COPY_NT / 32);
   uint2 *out = reinterpret_cast<uint2 *>(a.pairs);
   unsigned long long emitted = 0;
@@ -558,19 +558,19 @@ __global__ void __launch_bounds__(WSEL_NT, 4) k_select_fast(PredArgs a) {
   extern __shared__ uint4 sel4[];
   __shared__ uint32_t ws[SEL_NW], s_cnt[2];
   const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  if (*(const volatile uint32_t *)&a.st->log_dirty) return;  // k_select_stale's case
+  if (__ldcg(&a.st->log_dirty)) return;  // k_select_stale's case
   uint32_t *sm = reinterpret_cast<uint32_t *>(sel4);
   uint32_t ccnt[NQCLS], nfast = 0, nbig = 0;
 #pragma unroll
   for (int c = 0; c < NQCLS; ++c) {
-    ccnt[c] = *(const volatile uint32_t *)&a.st->q_cls[c];
+    ccnt[c] = __ldcg(&a.st->q_cls[c]);
     nfast += ccnt[c];
     if (c < (int)BIG_CLS) nbig += ccnt[c];
   }
   SelLog lg;
-  lg.head = *(const volatile uint32_t *)&a.st->lrm_head;
-  lg.tail = *(const volatile uint32_t *)&a.st->lrm_tail;
-  lg.stale = lg.tail - lg.head - *(const volatile uint32_t *)&a.st->n_resident;
+  lg.head = __ldcg(&a.st->lrm_head);
+  lg.tail = __ldcg(&a.st->lrm_tail);
+  lg.stale = lg.tail - lg.head - __ldcg(&a.st->n_resident);
   lg.al = (lg.head & 3u) == 0;
   const uint32_t nitems = nbig + (nfast - nbig + SEL_NW - 1) / SEL_NW;
   unsigned long long scanned = 0, victims = 0;
@@ -621,16 +621,16 @@ __global__ void __launch_bounds__(WSEL_NT) k_select_stale(PredArgs a) {
   const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const Geo &g = a.g;
   const SelectOut &so = a.so;
-  if (!*(const volatile uint32_t *)&a.st->log_dirty) return;  // k_select_fast's case
+  if (!__ldcg(&a.st->log_dirty)) return;  // k_select_fast's case
   uint32_t ccnt[NQCLS], nfast = 0;
 #pragma unroll
   for (int c = 0; c < NQCLS; ++c) {
-    ccnt[c] = *(const volatile uint32_t *)&a.st->q_cls[c];
+    ccnt[c] = __ldcg(&a.st->q_cls[c]);
     nfast += ccnt[c];
   }
-  const uint32_t head = *(const volatile uint32_t *)&a.st->lrm_head;
-  const uint32_t tail = *(const volatile uint32_t *)&a.st->lrm_tail;
-  const uint32_t stale = tail - head - *(const volatile uint32_t *)&a.st->n_resident;
+  const uint32_t head = __ldcg(&a.st->lrm_head);
+  const uint32_t tail = __ldcg(&a.st->lrm_tail);
+  const uint32_t stale = tail - head - __ldcg(&a.st->n_resident);
   for (uint32_t bq = blockIdx.x; bq < nfast; bq += gridDim.x) {
     const uint32_t qi = fast_query(a, ccnt, bq);
     const uint32_t nk = __ldg(a.qnk + qi);
@@ -789,7 +789,7 @@ cudaError_t launch_walk_index(dum_engine *e, cudaStream_t main) {
 // selection's clean-log path splits write-back / invalidate by popcounts.
 __global__ void __launch_bounds__(256) k_log_bits(const uint32_t *__restrict__ lrm_blk, const DevState *st,
                                                   uint32_t *bits) {
-  const uint32_t head = *(const volatile uint32_t *)&st->lrm_head, tail = *(const volatile uint32_t *)&st->lrm_tail;
+  const uint32_t head = __ldcg(&st->lrm_head), tail = __ldcg(&st->lrm_tail);
   const uint32_t nw = (tail - head + 31) / 32, lane = threadIdx.x & 31;
   for (uint32_t w = (blockIdx.x * 256 + threadIdx.x) >> 5; w < nw; w += gridDim.x * 8) {
     const uint32_t p = head + 32 * w + lane;

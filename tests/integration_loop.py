@@ -43,8 +43,9 @@ class LoopEngine:
 
 def run_loop(eng: LoopEngine, tr, N: int, inactive: set = frozenset(), check=None, preevict: bool = True,
              invalidate: bool = True, n_launch: int = None, per_launch: list = None) -> Dict[str, object]:
-    """N < 0: no queries (naive UM, demand path only).  preevict=False: the
-    window is prefetched into free frames only.  invalidate=False: inactive
+    """N < 0: no queries (naive UM, demand path only).  preevict=False
+    (prefetch only): the whole non-resident window is prefetched, the driver
+    evicting the least recently migrated blocks beyond the free frames.  invalidate=False: inactive
     victims are written back too.  Faults are the first occurrence of each
     non-resident access of the launch (D2; the T trace has no repeats).
     per_launch (a list) receives (faults, demand_wb, demand_inv, pre_wb,
@@ -105,8 +106,27 @@ def run_loop(eng: LoopEngine, tr, N: int, inactive: set = frozenset(), check=Non
                             eng.migrate(D2H, wb); d2h += len(wb)
                         if iv:
                             eng.migrate(INVALIDATE, iv); inv += len(iv)
-                    rset = set(eng.resident())
-                    todo = [b for b in window if b not in rset][: eng.free()]
+                    res = eng.resident()
+                    rset = set(res)
+                    if preevict:
+                        todo = [b for b in window if b not in rset][: eng.free()]
+                    else:
+                        # prefetch only: the whole non-resident window; the driver
+                        # evicts least recently migrated blocks (any) beyond the
+                        # free frames
+                        todo = [b for b in window if b not in rset][: eng.free() + len(res)]
+                        extra = len(todo) - eng.free()
+                        if extra > 0:
+                            victims = res[:extra]
+                            wb = [b for b in victims if b not in inactive]
+                            iv = [b for b in victims if b in inactive]
+                            if not invalidate:
+                                wb, iv = wb + iv, []
+                            st[3], st[4] = len(wb), len(iv)
+                            if wb:
+                                eng.migrate(D2H, wb); d2h += len(wb)
+                            if iv:
+                                eng.migrate(INVALIDATE, iv); inv += len(iv)
                     st[5] = len(todo)
                     if todo:
                         eng.migrate(H2D, todo); h2d += len(todo)

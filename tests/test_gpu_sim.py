@@ -64,7 +64,8 @@ def test_T_closed_loop_matches_reference_and_closed_form(N):
 
 @pytest.mark.parametrize("flags", [B.SIM_PREFETCH, B.SIM_PREFETCH | B.SIM_PREEVICT])
 def test_T_closed_loop_ablations_match_reference(flags):
-    """Fig. 10's intermediate configurations: prefetch only, + pre-eviction."""
+    """Fig. 10's intermediate configurations: prefetch only (the driver evicts
+    least recently migrated blocks for the prefetch), + pre-eviction."""
     tr = wl.make_T()
     N = 2
     eng = Engine(num_rows=2048, assoc=2, num_succs=4, degree_n=N, max_blocks=tr.W, max_exec_ids=64, hbm_frames=tr.C)
@@ -77,7 +78,7 @@ def test_T_closed_loop_ablations_match_reference(flags):
     assert eng.dump_state(orc.RES) == ref.o.dump(orc.RES)
 
 
-@pytest.mark.parametrize("flags", [0, ALL])
+@pytest.mark.parametrize("flags", [0, B.SIM_PREFETCH, ALL])
 def test_B_closed_loop_sample_matches_reference(flags):
     """BERT-large-shaped trace (configs[1]), 1.5 iterations, metadata-only."""
     tr = wl.make("B", n_iter=2)

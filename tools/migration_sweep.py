@@ -9,7 +9,9 @@ frame pool, for
   order:     contiguous blocks -> contiguous frames, and a random permutation
              of blocks (frames still assigned lowest-free-first, D21);
   direction: H2D, D2H, H2D || D2H concurrently (two engines on two streams,
-             disjoint halves of the arena / pool), D2D compaction (HBM);
+             disjoint halves of the arena / pool, half of the SMs each for
+             the copy kernels; method 2 synchronizes per call, so its pair
+             runs one after the other), D2D compaction (HBM);
   method:    1 = SM copy kernel, 3 = TMA bulk copies, 2 = copy engines (one
              cudaMemcpyAsync per contiguous run).
 Per point: W warm-up + R timed repetitions (CUDA events on the engine's
@@ -96,6 +98,11 @@ def main():
                   frame_pool=pool[: half * BLOCK])
     engB = Engine(max_blocks=half, hbm_frames=half, max_exec_ids=16, host_arena=host[half * BLOCK:],
                   frame_pool=pool[half * BLOCK:])
+    # the concurrent pair splits the SMs: each engine's copy kernels take half
+    # (dum_set_copy_sms), so the write-back and the fetch run side by side
+    nsm = torch.cuda.get_device_properties(dev).multi_processor_count
+    engA.set_copy_sms(nsm // 2)
+    engB.set_copy_sms(nsm - nsm // 2)
     sB = torch.cuda.Stream(device=dev)
     rng = np.random.default_rng(4)
     methods = [int(m) for m in args.methods.split(",")]

@@ -11,8 +11,8 @@ scale, metadata-only, and its sweeps.
     invalidated -- per iteration, steady state = mean of iterations 1..
   * Fig. 11: degree N in {1, 2, 4, 8, 16, 32, 64} (B).
   * Fig. 12 / Table 6: Config0 - Config12 (B).
-  * Cross-check: naive UM here == the generator's naive-UM fault trace
-    (workloads/um_sim.c, independent code).
+  * Cross-check: naive UM here vs the generator's naive-UM fault trace
+    (workloads/um_sim.c, independent code; differs by the demand rule D22).
 Every number comes from the engine's kernels; the host only launches."""
 from __future__ import annotations
 
@@ -79,7 +79,15 @@ def main():
             res["ablation"][name] = run(tr, dev, fl, N=32 if fl else -1)
             print(cfg, name, res["ablation"][name]["steady_mean"], res["ablation"][name]["wall_s"], file=sys.stderr)
         naive = res["ablation"]["naive_um"]["per_iteration"]["faults"]
-        res["naive_equals_trace"] = naive == res["trace_naive_um_faults"]
+        # the generator's naive-UM model (workloads/um_sim.c) evicts one block per
+        # fault, possibly one the faulting launch touches; the engine's demand
+        # path takes a launch's faults together and never evicts a block the
+        # launch accesses (reading D22): the two fault counts differ by that
+        res["naive_um_vs_trace"] = {"engine": naive, "um_sim": res["trace_naive_um_faults"],
+                                    "rel_diff_steady": float(np.mean(naive[1:])) /
+                                    max(float(np.mean(res["trace_naive_um_faults"][1:])), 1.0) - 1.0,
+                                    "why": "D22: demand victims exclude the faulting launch's blocks; um_sim.c "
+                                           "evicts fault by fault in LRM order"}
         full = res["ablation"]["prefetch+preevict+invalidate"]["steady_mean"]["faults"]
         res["table5_shape"] = {"naive_um_faults_per_iter": float(np.mean(naive[1:])),
                                "engine_faults_per_iter": full,
