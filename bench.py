@@ -56,6 +56,7 @@ def parse():
     ap.add_argument("--degree", type=int, default=32)
     ap.add_argument("--mig-blocks", type=int, default=4096)
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--timeline", default=None, help="write the last breakdown step's per-kernel timeline (JSON)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-migration", action="store_true")
     ap.add_argument("--cpu-launches", type=int, default=0, help="oracle sample size in launches")
@@ -159,8 +160,8 @@ def algorithmic_bytes(ctr, geo, N):
         "k_ingest": terms["ingest"] + 16 * c["LAUNCHES"],
         "k_build_prep": 48 * c["CORR_UPSERTS"],
         "k_build_exec": terms["block_tables"] + terms["walk_cache"],  # apply + walks (dedupe walks: k_walk)
-        "k_copy_fast": fast_copy,    # the flat copy of the fast windows
-        "k_select_fast": fast_sel,   # their selection (beside the copy)
+        "k_copy_fast": fast_copy,    # the flat copy of the fast windows (predict-only calls)
+        "k_window_fast": fast_copy + fast_sel,  # copy + selection of the fast windows in one kernel
         "k_predict": terms["predict"] + terms["select"] - fast_copy - fast_sel,
     }
     return terms, per_kernel, c
@@ -427,8 +428,11 @@ def run_ours(args, rank, world, local_rank):
     eng.set_step_graphs(False)  # per-kernel events need the kernels issued one by one
     timing_on[0] = True
     bk_ms = 0.0
+    timeline = None
     for s in range(args.steps):
         i = 1 + args.warmup + args.steps + s
+        if args.timeline and s == args.steps - 1:
+            eng.read_timeline(0)  # the earlier steps' regions go to the sums only
         pre_step(i)
         a = torch.cuda.Event(enable_timing=True)
         b = torch.cuda.Event(enable_timing=True)
@@ -437,6 +441,13 @@ def run_ours(args, rank, world, local_rank):
         b.record(stream)
         b.synchronize()
         bk_ms += a.elapsed_time(b)
+        if args.timeline and s == args.steps - 1:  # the last step's kernels: (name, start, end) in us
+            names = {v: k for k, v in B.TIMER.items()}
+            ids, t0, t1 = eng.read_timeline()
+            timeline = [(names.get(int(x), str(int(x))), round(1000 * float(u), 1), round(1000 * float(v), 1))
+                        for x, u, v in zip(ids, t0, t1)]
+            with open(args.timeline, "w") as f:
+                json.dump({"step_us": round(1000 * a.elapsed_time(b), 1), "regions": timeline}, f, indent=0)
     timing_on[0] = False
     eng.set_timing(False)
     ctr_bk = eng.read_counters(reset=True)
@@ -475,7 +486,8 @@ def run_ours(args, rank, world, local_rank):
             "bytes_formula": {
                 "k_copy_fast": "4*GATHERED + 8*EMITTED + 4*(N+2)*QUERIES of the fast queries = "
                                "12*FAST_EMITTED + 4*(N+2)*Q_FAST (SURVEY 8(d) predict term)",
-                "k_select_fast": "4*FAST_SCANNED + 4*FAST_VICTIMS (SURVEY 8(d) select term of the fast queries)",
+                "k_window_fast": "12*FAST_EMITTED + 4*(N+2)*Q_FAST + 4*FAST_SCANNED + 4*FAST_VICTIMS (SURVEY 8(d) "
+                                 "predict + select terms of the fast queries)",
                 "k_build_exec": "2*set_bytes*SETS + set_bytes*WALK_ROWS + 4*WALK_OUT (block tables + walk cache)",
                 "k_ingest": "4*RAW + 4*NORM + 20*LAUNCHES + 16*LAUNCHES (exec-map probe)",
                 "k_build_prep": "48*CORR_UPSERTS", "set_bytes": 4 * geo["A"] * (1 + geo["S"]), "N": N},

@@ -420,14 +420,20 @@ enum {
   DUM_T_CHAIN,
   DUM_T_JUMP,         /* jump tables over the correlation table (side stream, in dum_build_tables) */
   DUM_T_WALK,         /* parallel walk-cache rebuild (in dum_build_tables) */
-  DUM_T_EXACT,        /* exact-path predict kernel k_predict (side stream, beside the fast path) */
+  DUM_T_EXACT,        /* exact-path predict kernel k_predict (the fast path runs beside it on a side stream) */
   DUM_T_WALK_INDEX,   /* walk index: holders per block, conflicts per walk (build end) */
   DUM_T_WALK_RES,     /* residency facts per walk (predict) */
-  DUM_T_SELECT_FAST,  /* fast path with selection: k_select_fast (a CTA per window: victims, then pairs) */
+  DUM_T_SELECT_FAST,  /* fast path with selection: k_window_fast (pairs + selection, one persistent kernel) */
   DUM_NTIMERS = 24
 };
 int dum_set_timing(dum_engine *eng, int enable);
 int dum_read_timing(dum_engine *eng, double ms[DUM_NTIMERS], uint64_t count[DUM_NTIMERS], int reset);
+/* The same timed regions as a timeline: synchronizes, then for each region
+ * recorded since the last dum_read_timing / dum_read_timeline (in issue order,
+ * at most cap) writes its timer id and its start / end in ms relative to the
+ * first region's start; returns the number written (>= 0) or a negative
+ * DUM_* code.  The regions are consumed (and added to dum_read_timing's sums). */
+int dum_read_timeline(dum_engine *eng, int cap, int *ids, float *t0, float *t1);
 
 const char *dum_last_error(const dum_engine *eng);
 

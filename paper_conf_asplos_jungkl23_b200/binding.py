@@ -34,16 +34,15 @@ TIMER = {n: i for i, n in enumerate(["INGEST", "EXEC_ASSIGN", "BUILD_PREP", "APP
                                      "RESIDENCY", "CHAIN", "JUMP", "WALK", "EXACT", "WALK_INDEX", "WALK_RES", "SELECT_FAST"])}
 KERNEL_OF_TIMER = {"INGEST": "k_ingest", "EXEC_ASSIGN": "k_exec_assign", "BUILD_PREP": "k_build_prep",
                    "APPLY_WALK": "k_build_exec", "WALK": "k_walk", "WALK_SLOW": "k_walk_slow", "MAKE_QUERIES": "k_make_queries",
-                   "ANCHOR_WALK": "k_anchor_walk", "PREDICT": "k_copy_fast", "SELECT": "k_select", "SELECT_FAST": "k_select_fast",
+                   "ANCHOR_WALK": "k_anchor_walk", "PREDICT": "k_copy_fast", "SELECT": "k_select", "SELECT_FAST": "k_window_fast",
                    "MIG_PLAN": "k_mig_plan", "COPY": "k_copy_blocks", "RESIDENCY": "k_load_res",
                    "CHAIN": "k_chain", "JUMP": "k_jump0", "EXACT": "k_predict", "WALK_INDEX": "k_walk_index",
                    "WALK_RES": "k_walk_res"}
 # timers of kernels launched on the engine's side streams (overlapping others)
 SIDE_TIMERS = {"JUMP": "side stream, overlaps k_apply / k_walk (k_jump0 + k_jumpk levels)",
-               "EXACT": "second side stream, beside the fast path (exact-path queries)",
-               "SELECT_FAST": "third side stream, beside k_copy_fast (fast-path selection: k_select_fast + k_select_stale)",
+               "SELECT_FAST": "second side stream, beside the exact path (k_window_fast: pairs + selection of the fast windows)",
                "WALK_RES": "ingest-side fork in dum_step (beside k_ingest .. k_anchor_walk)",
-               "WALK_INDEX": "third side stream after the build (replayed step graphs: at the start of the next step, beside its ingest)"}
+               "WALK_INDEX": "third side stream (high priority) after the build (replayed step graphs: at the start of the next step, beside its ingest)"}
 _ERR = {0: "DUM_OK", -1: "DUM_EINVAL", -2: "DUM_ECAPACITY", -3: "DUM_ENOMEM", -4: "DUM_ECUDA", -5: "DUM_ESTATE"}
 
 
@@ -116,6 +115,7 @@ def load_library() -> ctypes.CDLL:
         "dum_set_timing": (I, [P, I]),
         "dum_host_ptr_kind": (I, [P]),
         "dum_read_timing": (I, [P, P, P, I]),
+        "dum_read_timeline": (I, [P, I, P, P, P]),
         "dum_simulate": (I, [P, P, U32, P, P, U32, U32, U32, P, P]),
         "dum_step": (I, [P, P, P, U32, P, U64, U32, U32, P, U64, P, P, P, P, P, P, U64, P, P, P]),
         "dum_set_step_graphs": (I, [P, I]),
@@ -426,6 +426,16 @@ class Engine:
         self._ck(self.lib.dum_read_timing(self._h, ms.ctypes.data, cnt.ctypes.data, 1 if reset else 0),
                  "dum_read_timing")
         return ms, cnt
+
+    def read_timeline(self, cap: int = 4096):
+        """(timer ids, start ms, end ms) of the timed regions since the last read, issue order."""
+        ids = np.zeros(cap, dtype=np.int32)
+        t0 = np.zeros(cap, dtype=np.float32)
+        t1 = np.zeros(cap, dtype=np.float32)
+        n = int(self.lib.dum_read_timeline(self._h, cap, ids.ctypes.data, t0.ctypes.data, t1.ctypes.data))
+        if n < 0:
+            self._ck(n, "dum_read_timeline")
+        return ids[:n], t0[:n], t1[:n]
 
     @property
     def kernel_launches(self) -> int:

@@ -39,6 +39,8 @@ __global__ void k_init_state(DevState *st) {
   st->err = 0;
   st->needed = 0;
   st->pool_pairs = st->pool_wb = st->pool_inv = st->pool_anchor = st->pool_big = st->pool_chunks = 0;
+  st->sel_queue = 0;
+  st->copy_queue = 0;
   st->chain_done = 0;
   for (int c = 0; c < 16; ++c) st->q_cls[c] = 0;
   st->n_fast = 0;
@@ -96,7 +98,6 @@ int reset_state(dum_engine *e, cudaStream_t s) {
   const Geo &g = e->g;
   if (e->ev_join) CK(cudaStreamWaitEvent(s, e->ev_join, 0));  // jump tables still building on the side stream
   if (e->ev_join2) CK(cudaStreamWaitEvent(s, e->ev_join2, 0));  // exact-path predict kernel
-  if (e->ev_join3) CK(cudaStreamWaitEvent(s, e->ev_join3, 0));  // fast-path selection
   if (e->ev_widx) CK(cudaStreamWaitEvent(s, e->ev_widx, 0));    // walk index
   if (e->ev_rec) CK(cudaStreamWaitEvent(s, e->ev_rec, 0));    // record work on the ingest stream
   CK(fill((uint32_t *)e->d_exec_keys, 2ull * (e->exec_cap + 1), NONE, s));
@@ -140,7 +141,7 @@ void free_all(dum_engine *e) {
                   e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits, e->d_inactive_bits, e->d_res_bits, e->d_logpos, e->d_lrm_blk,
                   e->d_lrm_stamp, e->d_mig_frames, e->d_mig_src, e->d_mig_blocks, e->d_state, e->d_qkern,
                   e->d_qloff, e->d_qnk, e->d_qbase, e->d_rec_slot, e->d_jump, e->d_wrun, e->d_wrun_len, e->d_qeoff, e->d_qgoff, e->d_qrank, e->d_qperm,
-                  e->d_bcnt, e->d_bhold, e->d_conf, e->d_conf_n, e->d_wnr, e->d_wnres, e->d_respos, e->d_qroff, e->d_qneed, e->d_qvb, e->d_chunk_map, e->d_dd_list, e->d_log_bits,
+                  e->d_bcnt, e->d_bhold, e->d_conf, e->d_conf_n, e->d_wnr, e->d_wnres, e->d_respos, e->d_qroff, e->d_qneed, e->d_qvb, e->d_chunk_map, e->d_selrec, e->d_dd_list, e->d_log_bits,
                   e->sim_acc_bits, e->sim_faults, e->sim_pairs, e->sim_wb, e->sim_inv, e->sim_pf, e->sim_foff,
                   e->sim_ranges, e->sim_q, e->d_step_exec, e->d_step_q};
   for (void *p : ptrs)
@@ -156,7 +157,9 @@ void free_all(dum_engine *e) {
     for (int i = 0; i < 8; ++i)
       if (e->cap_ev[i]) cudaEventDestroy(e->cap_ev[i]);
   if (e->side3) cudaStreamDestroy(e->side3);
-  if (e->ev_join3) cudaEventDestroy(e->ev_join3);
+  if (e->side4) cudaStreamDestroy(e->side4);
+  if (e->ev_fork4) cudaEventDestroy(e->ev_fork4);
+  if (e->ev_bhead) cudaEventDestroy(e->ev_bhead);
   if (e->ev_widx) cudaEventDestroy(e->ev_widx);
   if (e->ev_fork2) cudaEventDestroy(e->ev_fork2);
   if (e->ev_join2) cudaEventDestroy(e->ev_join2);
@@ -287,8 +290,15 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(cudaStreamCreateWithFlags(&e->graph_s, cudaStreamNonBlocking));
   A_(cudaEventCreateWithFlags(&e->ev_graph, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_wres, cudaEventDisableTiming));
-  A_(cudaStreamCreateWithFlags(&e->side3, cudaStreamNonBlocking));
-  A_(cudaEventCreateWithFlags(&e->ev_join3, cudaEventDisableTiming));
+  {  // the walk index runs here beside the next step's ingest and gates its k_chain:
+     // high priority, so that its CTAs are dispatched first
+    int lo = 0, hi = 0;
+    cudaDeviceGetStreamPriorityRange(&lo, &hi);
+    A_(cudaStreamCreateWithPriority(&e->side3, cudaStreamNonBlocking, hi));
+  }
+  A_(cudaStreamCreateWithFlags(&e->side4, cudaStreamNonBlocking));
+  A_(cudaEventCreateWithFlags(&e->ev_fork4, cudaEventDisableTiming));
+  A_(cudaEventCreateWithFlags(&e->ev_bhead, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_widx, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_fork2, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_join2, cudaEventDisableTiming));
@@ -362,7 +372,8 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_wnr, g.Emax));
   A_(dmalloc(&e->d_wnres, g.Emax));
   A_(dmalloc(&e->d_respos, (uint64_t)g.Emax * g.walk_cap));
-  A_(dmalloc(&e->d_log_bits, 4 * g.C / 32 + 1024 / 32 + 2));  // lrm_cap / 32 + 1 (lrm_cap = 4 C + 1024)
+  // lrm_cap / 32 + 1 (lrm_cap = 4 C + 1024), + slack: k_window_fast bulk-loads whole 16 B
+  A_(dmalloc(&e->d_log_bits, 4 * g.C / 32 + 1024 / 32 + 8));
   A_(dmalloc(&e->d_qroff, (uint64_t)e->anchor_range_cap * (g.N + 2)));
   A_(dmalloc(&e->d_qneed, e->anchor_range_cap));
   A_(dmalloc(&e->d_qvb, 2ull * e->anchor_range_cap));
@@ -370,6 +381,7 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   // launch_predict when a call's bound exceeds it
   e->chunk_cap = 1u << 20;
   A_(dmalloc(&e->d_chunk_map, e->chunk_cap));
+  A_(dmalloc(&e->d_selrec, 3ull * NQCLS * e->anchor_range_cap));
   A_(dmalloc(&e->d_frame_of, g.W));
   A_(dmalloc(&e->d_stamp_of, g.W));
   A_(dmalloc(&e->d_block_of, g.C));
@@ -383,6 +395,7 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_mig_src, e->mig_cap));
   A_(dmalloc(&e->d_mig_blocks, e->mig_cap));
   A_(dmalloc(&e->d_state, 1));
+  A_(cudaMemset(e->d_state, 0, sizeof(DevState)));
   A_(cudaMallocHost((void **)&e->h_state, sizeof(DevState)));
   if (err != cudaSuccess) {
     free_all(e);
@@ -589,7 +602,6 @@ static int step_graph(dum_engine *e, const uint64_t *launch_hash, const uint64_t
   CK(cudaStreamWaitEvent(s, e->ev_join, 0));
   CK(cudaStreamWaitEvent(s, e->ev_widx, 0));
   CK(cudaStreamWaitEvent(s, e->ev_join2, 0));
-  CK(cudaStreamWaitEvent(s, e->ev_join3, 0));
   CK(cudaStreamWaitEvent(s, e->ev_rec, 0));
   const uint64_t key[12] = {n_launch, (uint64_t)e->stage_set, degree, (uint64_t)out_pairs, out_cap_pairs,
                             (uint64_t)out_range, (uint64_t)out_kern_off, (uint64_t)out_chain, (uint64_t)out_needed,
@@ -612,8 +624,8 @@ static int step_graph(dum_engine *e, const uint64_t *launch_hash, const uint64_t
     cudaGraph_t graph = nullptr;
     // fork / join events recorded inside a capture become graph edges and may
     // not be waited on outside it: the capture uses its own set
-    cudaEvent_t *evs[] = {&e->ev_fork, &e->ev_join, &e->ev_fork2, &e->ev_join2, &e->ev_join3, &e->ev_widx,
-                          &e->ev_wres};
+    cudaEvent_t *evs[] = {&e->ev_fork, &e->ev_join, &e->ev_fork2, &e->ev_join2, &e->ev_widx,
+                          &e->ev_wres, &e->ev_fork4, &e->ev_bhead};
     constexpr int NEV = sizeof(evs) / sizeof(evs[0]);
     if (!e->cap_events_ready) {
       for (int i = 0; i < NEV; ++i) CK(cudaEventCreateWithFlags(&e->cap_ev[i], cudaEventDisableTiming));
@@ -638,9 +650,11 @@ static int step_graph(dum_engine *e, const uint64_t *launch_hash, const uint64_t
       err = launch_record(e, in_hash(e), in_off(e), n_launch, in_faults(e), e->stage_fault_cap,
                           e->d_step_exec + 3, s);
     if (err == cudaSuccess) err = launch_make_queries(e, e->d_step_exec, 3 + n_launch, 3, degree, e->d_step_q, s);
+    e->bhead_n = n_launch;  // the build's head goes beside the predict kernels
     if (err == cudaSuccess)
       err = launch_predict(e, e->d_step_q, n_launch, out_pairs, out_cap_pairs, out_range, out_kern_off, out_chain,
                            out_needed, &so, sel_needed, s);
+    e->bhead_n = 0;
     e->n_staged = n_launch;
     e->staged_faults = e->stage_fault_cap;
     if (err == cudaSuccess) err = launch_build(e, s);
@@ -657,7 +671,7 @@ static int step_graph(dum_engine *e, const uint64_t *launch_hash, const uint64_t
     e->n_staged = ns0;
     e->staged_faults = sf0;
     if (err == cudaSuccess) err = err2;
-    if (err == cudaSuccess) err = cudaGraphInstantiate(&exec, graph, 0);
+    if (err == cudaSuccess) err = cudaGraphInstantiate(&exec, graph, cudaGraphInstantiateFlagUseNodePriority);
     if (graph) cudaGraphDestroy(graph);
     if (err != cudaSuccess) {
       // not capturable here: say so once, drop to the one-call path for good
@@ -727,9 +741,14 @@ int dum_step(dum_engine *e, const uint64_t *launch_hash, const uint64_t *launch_
   if (rc) return rc;
   cudaStream_t s = (cudaStream_t)stream;
   CK(launch_make_queries(e, e->d_step_exec, 3 + n_launch, 3, degree, e->d_step_q, s));
+  e->bhead_n = e->n_staged;  // the build's head goes beside the predict kernels
   rc = dum_predict_select(e, e->d_step_q, n_launch, out_pairs, out_cap_pairs, out_range, out_kern_off, out_chain,
                           out_needed, out_writeback, out_invalidate, sel_cap, sel_range, sel_needed, stream);
-  if (rc) return rc;
+  e->bhead_n = 0;
+  if (rc) {
+    e->bhead_pending = false;
+    return rc;
+  }
   rc = dum_build_tables(e, stream);
   if (rc) return rc;
   k_step_shift<<<1, 32, 0, s>>>(e->d_step_exec, n_launch);
@@ -937,6 +956,33 @@ int dum_read_timing(dum_engine *e, double ms[DUM_NTIMERS], uint64_t count[DUM_NT
     }
   }
   return DUM_OK;
+}
+
+int dum_read_timeline(dum_engine *e, int cap, int *ids, float *t0, float *t1) {
+  if (!e || cap < 0 || (cap && (!ids || !t0 || !t1))) return DUM_EINVAL;
+  cudaSetDevice(e->device);
+  CK(cudaDeviceSynchronize());
+  int n = 0;
+  for (auto &t : e->pending) {
+    float x = 0.f, a = 0.f, b = 0.f;
+    CK(cudaEventElapsedTime(&x, t.a, t.b));
+    CK(cudaEventElapsedTime(&a, e->pending[0].a, t.a));
+    CK(cudaEventElapsedTime(&b, e->pending[0].a, t.b));
+    e->t_ms[t.id] += x;
+    e->t_cnt[t.id] += 1;
+    if (n < cap) {
+      ids[n] = t.id;
+      t0[n] = a;
+      t1[n] = b;
+      ++n;
+    }
+  }
+  for (auto &t : e->pending) {
+    e->event_pool.push_back(t.a);
+    e->event_pool.push_back(t.b);
+  }
+  e->pending.clear();
+  return n;
 }
 
 uint64_t dum_kernel_launches(const dum_engine *e) { return e ? e->kernel_launches : 0; }

@@ -54,6 +54,8 @@ struct DevState {
   unsigned long long pool_anchor;  // anchored-walk scratch bump pointer
   unsigned long long pool_big;     // build-walk global hash scratch bump pointer
   unsigned long long pool_chunks;  // predict: k_copy_fast chunk-map bump pointer
+  uint32_t sel_queue;         // predict: k_window_fast selection-item queue head
+  unsigned long long copy_queue;  // predict: k_window_fast copy-chunk queue head
   uint32_t n_slow;            // exec IDs queued for the sequential walk
   uint32_t n_pend;            // record: launches with a hash first seen in the batch (k_ingest -> k_exec_assign)
   uint32_t free_count;        // free HBM frames
@@ -199,12 +201,17 @@ struct dum_engine {
   uint32_t *d_log_bits;         // [lrm_cap / 32 + 1] inactive log entries by position from head (k_log_bits)
   uint32_t *d_qroff, *d_qneed;  // [max queries][N+2], [max queries] (k_chain -> k_window)
   unsigned long long *d_qvb;    // [max queries][2] victim-range bases (k_chain -> k_window)
+  uint4 *d_selrec;  // [NQCLS][max queries][3] k_window_fast selection records, k_chain's class order
   uint4 *d_chunk_map;  // [chunk_cap] copy chunks of the fast queries' windows: {exec, first, dst lo, dst hi | n << 16}
   uint64_t chunk_cap;
   cudaStream_t side2;           // exact-path predict kernel beside the fast path
   cudaEvent_t ev_fork2, ev_join2;
-  cudaStream_t side3;           // walk index (build end) and the fast-path selection
-  cudaEvent_t ev_join3, ev_widx;
+  cudaStream_t side3;           // walk index (build end)
+  cudaStream_t side4;           // dum_step: the build's head (k_build_prep, k_plan) beside the predict kernels
+  cudaEvent_t ev_fork4, ev_bhead;
+  uint32_t bhead_n;             // dum_step: launches whose build head launch_predict issues after k_chain
+  bool bhead_pending;           // the head was issued early: launch_build waits for ev_bhead
+  cudaEvent_t ev_widx;
   // dum_step: exec IDs [last 3 of the previous step | this batch] and the batch's queries
   uint32_t *d_step_exec;
   dum_query *d_step_q;
@@ -243,8 +250,7 @@ struct dum_engine {
   uint64_t t_cnt[DUM_NTIMERS];
   int predict_smem, select_smem, build_smem, ingest_smem;
   uint32_t apply_grid, walk_grid;  // persistent build grids (occupancy x SMs), set on first build
-  uint32_t copy_grid, sel_grid, stale_grid;  // persistent predict grids (k_window.cu)
-  int sel_smem;                              // k_select_fast dynamic shared memory (k_window.cu)
+  uint32_t copy_grid, sel_grid;  // persistent predict grids (k_window.cu)
   int chain_smem;                  // k_chain dynamic smem attribute applied
   int bulk_smem;                   // k_copy_bulk dynamic smem attribute applied
   uint32_t copy_sms;               // copy kernels: SMs' worth of CTAs (0 = all; dum_set_copy_sms)

@@ -60,10 +60,10 @@ __global__ void k_build_prep(uint32_t n_staged, const uint32_t *__restrict__ sta
                              const uint32_t *__restrict__ stage_cnt, CorrSlot *corr, uint32_t corr_cap,
                              uint32_t *rec_slot, uint32_t *head, uint32_t *__restrict__ next,
                              uint32_t *__restrict__ order, uint32_t *e_ops, uint32_t *e_last,
-                             unsigned long long *plan_agg, DevState *st) {
+                             unsigned long long *plan_agg, DevState *st, uint32_t reset_pool) {
   const uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
   if (j == 0) {
-    st->pool_big = 0;
+    if (reset_pool) st->pool_big = 0;
     st->n_slow = 0;
     st->n_dd = 0;
     st->n_items = 0;  // k_plan's last chunk writes the list sizes
@@ -1145,13 +1145,7 @@ static cudaError_t launch_apply_walk(dum_engine *e, const BuildArgs &ba, cudaStr
   return cudaGetLastError();
 }
 
-cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
-  const uint32_t n = e->n_staged;
-  if (n == 0) return cudaSuccess;
-  if (!e->capturing) {  // (a captured step joins its side streams before it ends)
-    cudaStreamWaitEvent(s, e->ev_join, 0);  // the previous build's jump tables read corr
-    cudaStreamWaitEvent(s, e->ev_widx, 0);  // the previous build's walk index reads the walk cache
-  }
+static BuildArgs build_args(dum_engine *e, uint32_t n) {
   BuildArgs ba;
   ba.g = e->g;
   ba.n_staged = n;
@@ -1180,20 +1174,63 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   ba.st = e->d_state;
   ba.seq_walks = (e->cfg.flags & DUM_CFG_SEQ_WALKS) ? 1u : 0u;
   ba.dd_list = e->d_dd_list;
+  return ba;
+}
+
+// The build's head: correlation upserts + work lists (k_build_prep, k_plan) on
+// `s`, the jump tables forked to the side stream.  reset_pool: k_build_prep
+// clears the walk-scratch bump pointer (pool_big) -- not when it runs beside
+// the predict kernels, whose exact path allocates from it (k_pred_epilogue
+// clears it before the build's tail then).
+static cudaError_t build_head(dum_engine *e, const BuildArgs &ba, cudaStream_t s, uint32_t reset_pool) {
+  const uint32_t n = ba.n_staged;
   {
     TimerScope t(e, DUM_T_BUILD_PREP, s);
     k_build_prep<<<(n + 255) / 256, 256, 0, s>>>(n, e->d_stage_exec, e->d_stage_cnt,
                                                   e->d_corr, e->corr_cap, e->d_rec_slot, e->d_head, e->d_next,
-                                                  e->d_order, e->d_e_ops, e->d_e_last, ba.plan_agg, e->d_state);
+                                                  e->d_order, e->d_e_ops, e->d_e_last, ba.plan_agg, e->d_state,
+                                                  reset_pool);
     k_plan<<<(n + PLAN_NT - 1) / PLAN_NT, PLAN_NT, 0, s>>>(ba);
   }
   // the jump tables depend only on the correlation table, final here
-  {
-    cudaEventRecord(e->ev_fork, s);
-    cudaStreamWaitEvent(e->side, e->ev_fork, 0);
-    const cudaError_t je = launch_jump_tables(e, e->side);
-    cudaEventRecord(e->ev_join, e->side);
-    if (je != cudaSuccess) return je;
+  cudaEventRecord(e->ev_fork, s);
+  cudaStreamWaitEvent(e->side, e->ev_fork, 0);
+  const cudaError_t je = launch_jump_tables(e, e->side);
+  cudaEventRecord(e->ev_join, e->side);
+  return je;
+}
+
+// dum_step: the head of the build of the n staged launches, issued by
+// launch_predict right after k_chain (the last reader of the correlation and
+// jump tables) on a side stream beside the exact / fast predict kernels; the
+// build's tail (launch_build) waits for it.
+cudaError_t launch_build_head(dum_engine *e, uint32_t n, cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  cudaEventRecord(e->ev_fork4, s);
+  cudaStreamWaitEvent(e->side4, e->ev_fork4, 0);
+  const BuildArgs ba = build_args(e, n);
+  const cudaError_t err = build_head(e, ba, e->side4, 0u);
+  cudaEventRecord(e->ev_bhead, e->side4);
+  e->bhead_pending = true;
+  e->kernel_launches += 2;
+  return err;
+}
+
+cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
+  const uint32_t n = e->n_staged;
+  if (n == 0) return cudaSuccess;
+  if (!e->capturing) {  // (a captured step joins its side streams before it ends)
+    cudaStreamWaitEvent(s, e->ev_join, 0);  // the previous build's jump tables read corr
+    cudaStreamWaitEvent(s, e->ev_widx, 0);  // the previous build's walk index reads the walk cache
+  }
+  const BuildArgs ba = build_args(e, n);
+  const bool was_early = e->bhead_pending;
+  if (e->bhead_pending) {  // the head ran beside the predict kernels (launch_build_head)
+    cudaStreamWaitEvent(s, e->ev_bhead, 0);
+    e->bhead_pending = false;
+  } else {
+    const cudaError_t he = build_head(e, ba, s, 1u);
+    if (he != cudaSuccess) return he;
   }
   cudaError_t err;
   if (e->g.A <= 2 && e->g.S <= 4) err = launch_apply_walk<2, 4>(e, ba, s);
@@ -1220,7 +1257,8 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   // no join here: the jump tables keep building on the side stream, past the
   // end of this call; the next reader of the correlation table (predict's
   // k_chain, the next build, reset) waits for ev_join
-  e->kernel_launches += 5;
+  if (!was_early) e->kernel_launches += 2;  // the head
+  e->kernel_launches += 3;
   return cudaGetLastError();
 }
 

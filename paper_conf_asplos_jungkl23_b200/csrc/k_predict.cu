@@ -125,6 +125,7 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
   uint32_t qneed = 0;  // fast query, fused select: victims to reserve in each output list
   uint32_t GUq = 0;    // copy chunks of the window (k_copy_fast)
   uint32_t qres = 0;   // fast query, fused select: resident window blocks (marks of the selection)
+  uint32_t qnw = 0;    // fast query, fused select: log-bitmap words k_window_fast scans at most
   if (qi < a.nq) {
     const dum_query Q = a.q[qi];
     const bool anchored = Q.anchor != NONE;
@@ -267,9 +268,11 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
       if ((uint64_t)qneed + nwres + stale > POS_WORDS * 32ull) {
         slow = true;
         if (lane == 0) ctr_add(a.st, DUM_CTR_SLOW_SPAN, 1);
+      } else if (qneed) {
+        qnw = (min(span, qneed + nwres + stale) + 31) / 32;
       }
     }
-    if (slow) qneed = 0;  // the exact kernel reserves its own victim ranges
+    if (slow) qneed = qnw = 0;  // the exact kernel reserves its own victim ranges
     qres = nwres;
     GUq = slow ? 0u : GU;
     __syncwarp();
@@ -284,7 +287,7 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
   // queries (classes 0 .. NQCLS-1) before exact-path ones
   // (fast queries of a fused select: by their selection work -- the marks of
   // the resident window blocks plus the log entries up to the cut, need +
-  // resident ones at most -- which also picks k_select_fast's CTA items)
+  // resident ones at most -- the selection items' order in k_window_fast)
   const uint32_t key = (a.select && !slow) ? (qneed ? qneed + 2 * qres : 0u) : U;
   const uint32_t cls = (key >= 14336 ? 0u : key >= 10240 ? 1u : key >= 6144 ? 2u : key >= 2048 ? 3u : 4u) +
                        (slow ? (uint32_t)NQCLS : 0u);
@@ -330,7 +333,7 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
         set_err(a.st, ERR_ECAPACITY, (s_wbase > s_ibase ? s_wbase : s_ibase) + nb + qneed);
     }
     if (base + U > a.cap) set_err(a.st, ERR_ECAPACITY, base + U);
-    // class lists: query order for k_select_fast / k_predict = class by class
+    // class lists: query order for k_window_fast / k_predict = class by class
     // (fast classes 0 .. NQCLS-1 largest first, then the exact-path ones)
     a.qperm[(uint64_t)cls * a.nq + s_cbase[cls] + s_wcls[w]] = qi;
   }
@@ -356,6 +359,17 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
       uint32_t *ch = a.chain + (uint64_t)qi * (g.N + 1);
       for (uint32_t d = lane; d <= g.N; d += 32) ch[d] = d < nk ? skern[w][d] : NONE;
     }
+  }
+  // k_window_fast's selection record of a fast query (at its class position, like qperm)
+  if (qi < a.nq && a.select && !slow && lane == 0) {
+    unsigned long long nb = 0;
+    for (uint32_t i = 0; i < w; ++i) nb += s_need[i];
+    const unsigned long long bwb = s_wbase + nb, binv = s_ibase + nb;
+    const uint32_t ok = bwb + qneed <= a.so.cap && binv + qneed <= a.so.cap;
+    uint4 *r = a.selrec + 3 * ((uint64_t)cls * a.nq + s_cbase[cls] + s_wcls[w]);
+    r[0] = make_uint4(qi, __ldcg(a.qnk + qi), qneed, qnw);
+    r[1] = make_uint4(0u, ok, 0u, 0u);
+    r[2] = make_uint4((uint32_t)bwb, (uint32_t)(bwb >> 32), (uint32_t)binv, (uint32_t)(binv >> 32));
   }
   // the chunk map of k_copy_fast: chunk j of list d of a fast query -> its
   // source (walk, first entry), destination slot and length; a query whose
@@ -886,6 +900,8 @@ __global__ void k_pred_epilogue(DevState *st, uint64_t *needed, uint64_t *sel_ne
     if (sel_needed) *sel_needed = st->pool_wb > st->pool_inv ? st->pool_wb : st->pool_inv;
     st->pool_pairs = 0;
     st->pool_chunks = 0;
+    st->sel_queue = 0;
+    st->copy_queue = 0;
     st->pool_wb = 0;
     st->pool_inv = 0;
     st->pool_anchor = 0;
@@ -964,6 +980,8 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   a.qroff = e->d_qroff;
   a.qneed = e->d_qneed;
   a.qvb = e->d_qvb;
+  a.selrec = e->d_selrec;
+  a.lrm_cap = e->lrm_cap;
   {
     // the chunk map holds every copy chunk of the call: <= cap / 128 + nq (N + 1)
     const uint64_t bound = cap / CHUNK_B + (uint64_t)nq * (e->g.N + 1) + 1;
@@ -1006,8 +1024,12 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
     }
     k_chain<<<(nq + CHAIN_WARPS - 1) / CHAIN_WARPS, CHAIN_WARPS * 32, csmem, s>>>(a);
   }
-  // exact path (windows that may hold duplicates, anchored queries) on the
-  // engine's second side stream, beside the fast path on `s`
+  if (e->bhead_n) {  // dum_step: the staged batch's build head beside the predict kernels (k_build.cu)
+    if ((err = launch_build_head(e, e->bhead_n, s)) != cudaSuccess) return err;
+  }
+  // exact path (windows that may hold duplicates, anchored queries) first on
+  // `s` -- its few CTAs are dispatched before the fast path's persistent grid
+  // fills the SMs -- and the fast path beside it on the second side stream
   cudaEventRecord(e->ev_fork2, s);
   cudaStreamWaitEvent(e->side2, e->ev_fork2, 0);
   const size_t smem = (size_t)((a.nwords + 3) & ~3u) * 4 + 2 * DHCAP * 4;
@@ -1018,21 +1040,20 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
       cudaFuncSetAttribute(k_predict<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       e->select_smem = (int)smem;
     }
-    TimerScope t(e, DUM_T_EXACT, e->side2);
-    k_predict<true><<<pgrid, PRED_NT, smem, e->side2>>>(a);
+    TimerScope t(e, DUM_T_EXACT, s);
+    k_predict<true><<<pgrid, PRED_NT, smem, s>>>(a);
   } else {
     if ((int)smem > e->predict_smem) {
       cudaFuncSetAttribute(k_predict<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
       e->predict_smem = (int)smem;
     }
-    TimerScope t(e, DUM_T_EXACT, e->side2);
-    k_predict<false><<<pgrid, PRED_NT, smem, e->side2>>>(a);
+    TimerScope t(e, DUM_T_EXACT, s);
+    k_predict<false><<<pgrid, PRED_NT, smem, s>>>(a);
   }
+  if ((err = launch_window(e, a, sel != nullptr, e->side2)) != cudaSuccess) return err;
   cudaEventRecord(e->ev_join2, e->side2);
-  // fast path on `s`: the flat copy (predict only) or a CTA per window (select + copy)
-  if ((err = launch_window(e, a, sel != nullptr, s)) != cudaSuccess) return err;
   cudaStreamWaitEvent(s, e->ev_join2, 0);
-  e->kernel_launches += 3;
+  e->kernel_launches += 2;
   k_pred_epilogue<<<1, 32, 0, s>>>(e->d_state, needed, sel ? sel_needed : nullptr);
   e->kernel_launches += 1;
   return cudaGetLastError();

@@ -30,15 +30,34 @@
 //  k_walk_conf   (build end)   conflicts of each walk: conf[e][..], conf_n[e]
 //  k_walk_res    (predict)     per walk: non-resident count, resident positions
 //  k_copy_fast   (predict)     flat copy of every fast window (chunk map from k_chain)
-//  k_select_fast (predict)     clean log: a CTA per big window, a warp per small one;
-//                              marking + word-level selection
-//  k_select_stale (predict)    stale log entries: a CTA per window, per-entry selection
+//  k_window_fast (predict+select) one persistent kernel, a work queue: the
+//                              flat copy interleaved with the selection (clean
+//                              log: marking + word-level ranks, then emit
+//                              groups; stale entries: per-entry selection)
 #include <algorithm>
 
 #include "device_util.cuh"
 #include "kernels.cuh"
 #include "predict.cuh"
 #include "select_tail.cuh"
+
+#ifdef EXP_TRACE
+// experiment builds only: globaltimer stamps of k_window_fast's work items
+__device__ unsigned long long g_tr[4096 * 4 + 8 * 65536];
+__device__ __forceinline__ unsigned long long gtime() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+#define TR(i, v) (g_tr[(i)] = (v))
+static void *g_tr_ptr() {
+  void *p = nullptr;
+  cudaGetSymbolAddress(&p, g_tr);
+  return p;
+}
+#else
+#define TR(i, v) ((void)0)
+#endif
 
 namespace dum {
 
@@ -242,21 +261,19 @@ __global__ void __launch_bounds__(COPY_NT) k_copy_fast(PredArgs a) {
 // when the selection provably ends inside).  The window's pairs are written
 // by k_copy_fast, concurrently.
 //
-// Clean log (every entry of [head, tail) valid, the normal case):
-// k_select_fast.  A 32-position word's eligible entries are ~marked & valid,
-// split by the log's inactive-entry bitmap (k_log_bits) into write-back /
-// invalidate; a scan of the packed popcounts gives every word its rank base;
-// then 4-word chunks (a lane per 4 consecutive entries, 16 B loads of the
-// log) write the entries of combined rank < need at their ranks.  Work items
-// in k_chain's class order: a big window (classes 0-2, need-key >= 6144) is
-// one CTA item (all warps mark, one block scan, the warps split the chunks);
-// the small ones go WSEL_NT / 32 to an item, a warp each (32-word groups, a
-// warp scan per group, no CTA barrier).  A warp per window alone leaves the
-// few biggest windows as a serial tail; a CTA per window leaves the SMs
-// waiting on barriers for the many small ones.
+// Clean log (every entry of [head, tail) valid, the normal case): sel_staged,
+// a query per item of the selection group (4 warps of a k_window_fast CTA).
+// The window's resident-position lists, the log's inactive-entry words and the
+// log prefix are staged in shared memory by TMA bulk copies; the positions
+// are marked in a bitmap; a 32-position word's eligible entries are ~marked &
+// valid, split by the inactive bits into write-back / invalidate; one group
+// scan of the packed popcounts gives every word its rank base and locates the
+// cut (the need-th eligible entry); then a lane per 4 consecutive entries of a
+// word writes the entries of combined rank < need at their ranks, reading the
+// log from the staged segments.
 //
-// Stale entries (a log not compacted since an eviction): k_select_stale, a CTA
-// per query, per-entry eligibility (frame + stamp check):
+// Stale entries (a log not compacted since an eviction): sel_stale, a CTA
+// item per query (same queue), per-entry eligibility (frame + stamp check):
 //   1. marks as above;  2. pass 1: eligible active / inactive entries per
 //   1024-entry segment, a warp per segment;  3. one warp scans the segment
 //   counts;  4. pass 2: each warp re-reads its segments and writes the
@@ -264,30 +281,6 @@ __global__ void __launch_bounds__(COPY_NT) k_copy_fast(PredArgs a) {
 constexpr uint32_t FSEG = 1024;                 // log entries per segment (32 per lane)
 constexpr uint32_t FSEG_MAX = POS_WORDS * 32 / FSEG;
 static_assert(FSEG_MAX <= 32, "one warp scans the segment counts");
-constexpr uint32_t SEL_NW = WSEL_NT / 32;  // warps per selection CTA
-constexpr uint32_t SW_KB = 2;              // warp path: 4-word chunks with their log loads in flight together
-constexpr uint32_t BIG_CLS = 3;            // classes [0, BIG_CLS) take a CTA per window
-
-__host__ __device__ constexpr uint32_t sw_words(uint32_t N) {  // shared words of one warp's window (16 B multiple)
-  return (POS_WORDS + (N + 2) + (N + 1) + 3) & ~3u;
-}
-__host__ __device__ constexpr uint32_t sel_smem_words(uint32_t N) {  // k_select_fast dynamic shared memory
-  return SEL_NW * sw_words(N) > 4 * POS_WORDS + sw_words(N) - POS_WORDS
-             ? SEL_NW * sw_words(N)
-             : 4 * POS_WORDS + sw_words(N) - POS_WORDS;
-}
-
-// the fast query of rank bq in k_chain's class lists
-__device__ __forceinline__ uint32_t fast_query(const PredArgs &a, const uint32_t *ccnt, uint32_t bq) {
-  uint32_t cq = NQCLS, rq = bq;
-#pragma unroll
-  for (int c = 0; c < NQCLS; ++c)
-    if (cq == NQCLS) {
-      if (rq < ccnt[c]) cq = c;
-      else rq -= ccnt[c];
-    }
-  return __ldg(a.qperm + (uint64_t)cq * a.nq + rq);
-}
 
 struct SelLog {  // the log, fixed during the kernel
   uint32_t head, tail, stale;
@@ -299,17 +292,6 @@ struct SelQuery {
   unsigned long long bwb, binv;
   bool ok;
 };
-
-__device__ __forceinline__ SelQuery load_query(const PredArgs &a, uint32_t qi) {
-  SelQuery q;
-  q.qi = qi;
-  q.nk = __ldg(a.qnk + qi);
-  q.need = __ldg(a.qneed + qi);
-  q.bwb = __ldg(a.qvb + 2 * qi);
-  q.binv = __ldg(a.qvb + 2 * qi + 1);
-  q.ok = q.bwb + q.need <= a.so.cap && q.binv + q.need <= a.so.cap;
-  return q;
-}
 
 __device__ __forceinline__ void write_range(const PredArgs &a, const SelQuery &q, uint32_t tw, uint32_t ti) {
   uint64_t *o = a.so.out_range + 4ull * q.qi;
@@ -343,253 +325,297 @@ __device__ __forceinline__ void mark_window(const PredArgs &a, const uint32_t *r
   }
 }
 
-// The eligible entries of UC 4-word chunks of one warp (a lane per 4
-// consecutive entries): chunk u covers words wd[u] .. +3 relative to w0 (lane
-// >> 3 picks the word), with em / im / pre the word's masks and rank base
-// (packed inactive << 16 | active).  Entries of combined rank < need go to
-// their ranks; returns the counts written (tw, ti).
-template <uint32_t UC>
-__device__ __forceinline__ void emit_chunks(const PredArgs &a, const SelQuery &q, const SelLog &lg, uint32_t lane,
-                                            const uint32_t *wpos, const uint32_t *em, const uint32_t *im,
-                                            const uint32_t *pre, uint32_t &tw, uint32_t &ti) {
-  const SelectOut &so = a.so;
-  uint32_t a4[UC], i4[UC], ra[UC], rr[UC], vv[UC][4];
-  const uint32_t sh = (lane & 7) * 4;
+// The selection group of k_window_fast: warps [0, SG_NT / 32) of the CTA,
+// synchronised by named barrier 1; the other warps copy pairs meanwhile.
+constexpr uint32_t SG_NT = 128;
+constexpr uint32_t SG_WPT = POS_WORDS / SG_NT;  // bitmap words per group thread
+__device__ __forceinline__ void gsync() { asm volatile("bar.sync 1, %0;" ::"n"(SG_NT) : "memory"); }
+
+// Exclusive scan of one value per group thread; ws holds SG_NT / 32 words.
+__device__ __forceinline__ uint32_t group_excl_scan(uint32_t v, uint32_t *ws, uint32_t *total) {
+  const uint32_t t = threadIdx.x, lane = t & 31, wid = t >> 5;
+  uint32_t x = v;
 #pragma unroll
-  for (uint32_t u = 0; u < UC; ++u) {
-    a4[u] = (em[u] >> sh) & 0xFu;
-    i4[u] = (im[u] >> sh) & 0xFu;
-    // ranks: the word's base + the eligible entries of the lower lanes of the same word
-    const uint32_t cc = __popc(a4[u]) | (__popc(i4[u]) << 16);
-    uint32_t y = cc;
-#pragma unroll
-    for (int o = 1; o < 8; o <<= 1) {
-      const uint32_t t = __shfl_up_sync(0xffffffffu, y, o);
-      if ((lane & 7) >= (uint32_t)o) y += t;
-    }
-    ra[u] = (pre[u] & 0xFFFFu) + ((y - cc) & 0xFFFFu);
-    rr[u] = (pre[u] >> 16) + ((y - cc) >> 16);
-    if (ra[u] + rr[u] >= q.need) a4[u] = i4[u] = 0;
-    if (a4[u] | i4[u]) {
-      const uint32_t p = lg.head + 32 * wpos[u] + sh;
-      if (lg.al) {
-        const uint4 v = __ldcg(reinterpret_cast<const uint4 *>(so.lrm_blk + p));
-        vv[u][0] = v.x; vv[u][1] = v.y; vv[u][2] = v.z; vv[u][3] = v.w;
-      } else {
-#pragma unroll
-        for (uint32_t k = 0; k < 4; ++k) vv[u][k] = ((a4[u] | i4[u]) >> k) & 1u ? __ldcg(so.lrm_blk + p + k) : 0u;
-      }
-    }
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= (uint32_t)o) x += y;
   }
+  if (lane == 31) ws[wid] = x;
+  gsync();
+  uint32_t base = 0, tot = 0;
 #pragma unroll
-  for (uint32_t u = 0; u < UC; ++u) {
-    if (!(a4[u] | i4[u])) continue;
-#pragma unroll
-    for (uint32_t k = 0; k < 4; ++k) {
-      const bool ea = (a4[u] >> k) & 1u, ei = (i4[u] >> k) & 1u;
-      if ((ea || ei) && ra[u] + rr[u] < q.need) {
-        if (q.ok) {
-          if (ei) so.inv[q.binv + rr[u]] = vv[u][k] & 0x7FFFFFFFu;
-          else so.wb[q.bwb + ra[u]] = vv[u][k];
-        }
-        tw += ea;
-        ti += ei;
-      }
-      ra[u] += ea;
-      rr[u] += ei;
-    }
+  for (uint32_t k = 0; k < SG_NT / 32; ++k) {
+    const uint32_t c = ws[k];
+    if (k < wid) base += c;
+    tot += c;
   }
+  gsync();  // ws is reused by the next call
+  *total = tot;
+  return base + x - v;
 }
 
-// A small window, one warp: marks in the warp's bitmap, then 32-word groups
-// (lane l: word w0 + l) with a warp scan each, until the cut.
-__device__ __forceinline__ void warp_window(const PredArgs &a, const SelLog &lg, uint32_t qi, uint32_t *wsm,
-                                            unsigned long long &scanned, unsigned long long &victims) {
-  const uint32_t lane = threadIdx.x & 31;
+// A selection item's record (k_chain): {qi, nk, need, nw}, {first emit group,
+// ok, -, -}, {wb base, inv base}.
+struct SelRec {
+  uint4 x, y, z;
+};
+__device__ __forceinline__ SelQuery rec_query(const SelRec &r) {
+  SelQuery q;
+  q.qi = r.x.x;
+  q.nk = r.x.y;
+  q.need = r.x.z;
+  q.ok = r.y.y != 0;
+  q.bwb = (unsigned long long)r.z.y << 32 | r.z.x;
+  q.binv = (unsigned long long)r.z.w << 32 | r.z.z;
+  return q;
+}
+
+// ---------------------------------------------------------------------------
+// The clean-log selection of one fast query by the selection group.  The log
+// prefix it scans is staged in shared memory by TMA bulk copies
+// (cp.async.bulk, one mbarrier per buffer) in segments of SR_SEG entries,
+// double-buffered so that the next segment lands while the current one is
+// emitted, and so are the log's inactive-entry words; both are issued before
+// the marking starts and land meanwhile.  (The resident-position lists are
+// loaded with plain coalesced loads: one bulk copy per list -- ~33 small ones
+// per query -- measured slower, 5-28 us to land.)
+constexpr uint32_t SR_SEG = 4096;        // log entries per segment
+constexpr uint32_t SR_SEGW = SR_SEG / 32;
+constexpr uint32_t SR_SMEM_WORDS = POS_WORDS /*ibits*/ + POS_WORDS /*wpre*/ + 2 * (SR_SEG + 4);
+
+__device__ __forceinline__ uint32_t sm_addr(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(unsigned long long *b) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(sm_addr(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_expect(unsigned long long *b, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(sm_addr(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, unsigned long long *b) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               ::"r"(sm_addr(dst)), "l"(src), "r"(bytes), "r"(sm_addr(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long *b, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tWAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n\t}" ::"r"(sm_addr(b)), "r"(parity) : "memory");
+}
+
+struct StageSm {
+  uint32_t *ibits, *wpre, *lbuf;  // dynamic shared memory (SR_SMEM_WORDS)
+  unsigned long long *bar;               // [3]: inactive-entry words, segment buffers 0 / 1
+};
+
+// Thread 0: the log segment k into buffer k & 1 (16 B aligned source; entries
+// [k SR_SEG, min(span, (k + 1) SR_SEG)) relative to head, at offset head & 3).
+__device__ __forceinline__ void issue_segment(const PredArgs &a, const SelLog &lg, const StageSm &S, uint32_t k,
+                                              uint32_t span) {
+  const uint32_t base = (lg.head + k * SR_SEG) & ~3u, o = (lg.head + k * SR_SEG) - base;
+  uint32_t n = (min(SR_SEG, span - k * SR_SEG) + o + 3) & ~3u;
+  n = min(n, a.lrm_cap - base);
+  unsigned long long *b = S.bar + 1 + (k & 1);
+  mbar_expect(b, 4 * n);
+  bulk_g2s(S.lbuf + (k & 1) * (SR_SEG + 4), a.so.lrm_blk + base, 4 * n, b);
+}
+
+// Thread 0: the log's inactive-entry words [0, nw) (one bulk copy).
+__device__ __forceinline__ void issue_bits(const PredArgs &a, const StageSm &S, uint32_t nw) {
+  const uint32_t bytes = 4 * ((nw + 3) & ~3u);
+  mbar_expect(S.bar, bytes);
+  bulk_g2s(S.ibits, a.inact_bits, bytes, S.bar);
+}
+
+__device__ __forceinline__ void sel_staged(const PredArgs &a, const SelLog &lg, const SelRec &r, const StageSm &S,
+                                           uint32_t *posmap, uint32_t *roff, uint32_t *kern, uint32_t *ws,
+                                           uint32_t *s_cut, uint32_t (&ph)[3], unsigned long long &scanned,
+                                           unsigned long long &victims, uint32_t it) {
+  const uint32_t t = threadIdx.x, lane = t & 31, wid = t >> 5;  // t < SG_NT
+#ifdef EXP_TRACE
+#define TRI(j) if (t == 0) TR(4 * 4096 + 8 * it + (j), gtime())
+#else
+#define TRI(j) ((void)it)
+#endif
   const Geo &g = a.g;
-  uint32_t *posmap = wsm, *roff = wsm + POS_WORDS, *kern = roff + g.N + 2;
-  const SelQuery q = load_query(a, qi);
-  for (uint32_t d = lane; d <= q.nk; d += 32) {
+  const SelQuery q = rec_query(r);
+  const uint32_t qi = q.qi, nw = q.need ? r.x.w : 0u;
+  if (!nw) {  // nothing to evict: an empty range
+    if (t == 0) write_range(a, q, 0, 0);
+    return;
+  }
+  for (uint32_t d = t; d <= q.nk; d += SG_NT) {
     roff[d] = __ldg(a.qroff + (uint64_t)qi * (g.N + 2) + d);
     if (d < q.nk) kern[d] = __ldg(a.qkern + (uint64_t)qi * (g.N + 1) + d);
   }
-  __syncwarp();
+  for (uint32_t w = t; w < nw; w += SG_NT) posmap[w] = 0;
+  gsync();
+  TRI(2);
   const uint32_t R = roff[q.nk];
   const uint32_t span = min(lg.tail - lg.head, min(q.need + R + lg.stale, POS_WORDS * 32));
-  const uint32_t nw = (span + 31) / 32;
-  uint32_t tw = 0, ti = 0;
-  if (q.need) {
-    for (uint32_t w = lane; w < nw; w += 32) posmap[w] = 0;
-    __syncwarp();
-    mark_window<8>(a, roff, kern, R, lg.head, nw * 32, posmap, lane, 32);
-    __syncwarp();
-    uint32_t ba = 0, bi = 0, w0 = 0;
-    for (; w0 < nw && ba + bi < q.need; w0 += 32) {
-      const uint32_t w = w0 + lane;
-      uint32_t em = 0, im = 0;
-      if (w < nw) {
-        const uint32_t lo = w * 32, valid = span - lo >= 32 ? 0xFFFFFFFFu : (1u << (span - lo)) - 1u;
-        const uint32_t ib = __ldg(a.inact_bits + w), e = valid & ~posmap[w];
-        em = e & ~ib;
-        im = e & ib;
-      }
-      const uint32_t c = __popc(em) | (__popc(im) << 16);
-      uint32_t x = c;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-        if (lane >= (uint32_t)o) x += y;
-      }
-      const uint32_t wpre = (ba | (bi << 16)) + x - c;  // packed ranks: both < 2^15
-      for (uint32_t k0 = 0; k0 < 8; k0 += SW_KB) {
-        const uint32_t pre0 = __shfl_sync(0xffffffffu, wpre, 4 * k0);
-        if (w0 + 4 * k0 >= nw || (pre0 & 0xFFFFu) + (pre0 >> 16) >= q.need) break;
-        uint32_t wp[SW_KB], e32[SW_KB], i32[SW_KB], p32[SW_KB];
-#pragma unroll
-        for (uint32_t u = 0; u < SW_KB; ++u) {
-          const uint32_t wd = 4 * (k0 + u) + (lane >> 3);
-          wp[u] = w0 + wd;
-          e32[u] = __shfl_sync(0xffffffffu, em, wd);
-          i32[u] = __shfl_sync(0xffffffffu, im, wd);
-          p32[u] = __shfl_sync(0xffffffffu, wpre, wd);
-        }
-        emit_chunks<SW_KB>(a, q, lg, lane, wp, e32, i32, p32, tw, ti);
-      }
-      const uint32_t tot = __shfl_sync(0xffffffffu, x, 31);
-      ba += tot & 0xFFFFu;
-      bi += tot >> 16;
-    }
-    tw = __reduce_add_sync(0xffffffffu, tw);
-    ti = __reduce_add_sync(0xffffffffu, ti);
-    if (lane == 0) scanned += min(span, 32 * w0);
+  const uint32_t nseg = (span + SR_SEG - 1) / SR_SEG;
+  if (t == 0) {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // earlier generic accesses of the buffers
+    issue_segment(a, lg, S, 0, span);
+    if (nseg > 1) issue_segment(a, lg, S, 1, span);
+    issue_bits(a, S, nw);
   }
-  if (lane == 0) {
+  // marks: the window's resident positions below nw * 32, flat over the lists'
+  // entries (coalesced loads, MU in flight per thread); a walk's resident
+  // blocks sit mostly at consecutive log positions, so the lanes hitting one
+  // bitmap word combine their bits first (one shared atomic per word)
+  {
+    constexpr uint32_t MU = 8;
+    uint32_t lo = 0;
+    for (uint32_t xb = 0; xb < R; xb += SG_NT * MU) {  // (warp-uniform trip count: the warp intrinsics below)
+      uint32_t rv[MU];
+#pragma unroll
+      for (uint32_t u = 0; u < MU; ++u) {
+        const uint32_t x = xb + u * SG_NT + t;
+        rv[u] = NONE;
+        if (x < R) {
+          while (roff[lo + 1] <= x) ++lo;
+          rv[u] = __ldg(a.respos + (uint64_t)kern[lo] * g.walk_cap + (x - roff[lo])) - lg.head;
+        }
+      }
+#pragma unroll
+      for (uint32_t u = 0; u < MU; ++u) {
+        const uint32_t wd = rv[u] < nw * 32 ? rv[u] >> 5 : NONE;
+        const uint32_t m = __match_any_sync(0xffffffffu, wd);
+        const uint32_t bits = __reduce_or_sync(m, wd != NONE ? 1u << (rv[u] & 31) : 0u);
+        if (wd != NONE && lane == (uint32_t)__ffs(m) - 1) atomicOr(&posmap[wd], bits);
+      }
+    }
+  }
+  TRI(3);
+  mbar_wait(S.bar, ph[0]);  // the inactive-entry words
+  ph[0] ^= 1u;
+  TRI(5);
+  gsync();
+  // eligible entries per word (~marked & valid, split by the inactive bits),
+  // rank bases by one group scan, the cut
+  uint32_t em[SG_WPT], im[SG_WPT], tot = 0;
+#pragma unroll
+  for (uint32_t u = 0; u < SG_WPT; ++u) {
+    const uint32_t w = SG_WPT * t + u;
+    em[u] = im[u] = 0;
+    if (w < nw) {
+      const uint32_t lo = w * 32, valid = span - lo >= 32 ? 0xFFFFFFFFu : (1u << (span - lo)) - 1u;
+      const uint32_t e = valid & ~posmap[w], ib = S.ibits[w];
+      em[u] = e & ~ib;
+      im[u] = e & ib;
+    }
+    tot += __popc(em[u]) | (__popc(im[u]) << 16);
+  }
+  if (t == 0) s_cut[0] = s_cut[1] = s_cut[2] = NONE;  // (ordered by the scan's barriers)
+  uint32_t tsum;
+  uint32_t pre = group_excl_scan(tot, ws, &tsum);  // packed (inactive << 16 | active); both <= 32768
+#pragma unroll
+  for (uint32_t u = 0; u < SG_WPT; ++u) {
+    const uint32_t w = SG_WPT * t + u;
+    if (w < nw) {
+      S.wpre[w] = pre;
+      posmap[w] = em[u];  // from here posmap holds the eligible write-back entries, ibits the invalidate ones
+      S.ibits[w] = im[u];
+      const uint32_t before = (pre & 0xFFFFu) + (pre >> 16), here = __popc(em[u] | im[u]);
+      if (before < q.need && before + here >= q.need) {  // the cut is in this word: take k more entries
+        uint32_t x = em[u] | im[u], mask = 0;
+        for (uint32_t k = q.need - before; k; --k) {
+          const uint32_t low = x & (0u - x);
+          mask |= low;
+          x ^= low;
+        }
+        s_cut[0] = (pre & 0xFFFFu) + __popc(em[u] & mask);  // taken write-back entries
+        s_cut[1] = (pre >> 16) + __popc(im[u] & mask);     // taken invalidate entries
+        s_cut[2] = w;
+      }
+    }
+    pre += __popc(em[u]) | (__popc(im[u]) << 16);
+  }
+  gsync();
+  TRI(4);
+  const uint32_t wcut = s_cut[2] == NONE ? nw - 1 : s_cut[2];  // the last word with victims
+  const uint32_t kend = (wcut * 32) / SR_SEG;                  // the last segment needed
+  // emit, segment by segment: a lane per 4 consecutive entries of a word
+  const uint32_t sh = (lane & 7) * 4, below = (1u << sh) - 1u;
+  for (uint32_t k = 0; k <= kend; ++k) {
+    mbar_wait(S.bar + 1 + (k & 1), ph[1 + (k & 1)]);
+    ph[1 + (k & 1)] ^= 1u;
+    const uint32_t *lb = S.lbuf + (k & 1) * (SR_SEG + 4) + ((lg.head + k * SR_SEG) & 3u);
+    const uint32_t w0 = k * SR_SEGW, w1 = min(wcut + 1, w0 + SR_SEGW);
+    for (uint32_t w = w0 + 4 * wid + (lane >> 3); w < w1; w += 4 * (SG_NT / 32)) {
+      const uint32_t ea4 = posmap[w], ei4 = S.ibits[w], pw = S.wpre[w];
+      uint32_t ra = (pw & 0xFFFFu) + __popc(ea4 & below), rr = (pw >> 16) + __popc(ei4 & below);
+      const uint32_t am = (ea4 >> sh) & 0xFu, imk = (ei4 >> sh) & 0xFu;
+      if (!(am | imk) || ra + rr >= q.need) continue;
+      const uint32_t *e4 = lb + 32 * (w - w0) + sh;  // (the segment's start may not be 16 B aligned)
+#pragma unroll
+      for (uint32_t j = 0; j < 4; ++j) {
+        const bool ea = (am >> j) & 1u, ei = (imk >> j) & 1u;
+        if ((ea || ei) && ra + rr < q.need && q.ok) {
+          if (ei) a.so.inv[q.binv + rr] = e4[j] & 0x7FFFFFFFu;
+          else a.so.wb[q.bwb + ra] = e4[j];
+        }
+        ra += ea;
+        rr += ei;
+      }
+    }
+    if (k + 2 <= kend) {
+      gsync();  // buffer k & 1 is read
+      if (t == 0) {
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        issue_segment(a, lg, S, k + 2, span);
+      }
+    }
+  }
+  // segments issued but not needed (the cut came early): wait for them so
+  // that the barriers' phases stay in step with the parities
+  for (uint32_t k = kend + 1; k < min(nseg, 2u); ++k) {
+    mbar_wait(S.bar + 1 + (k & 1), ph[1 + (k & 1)]);
+    ph[1 + (k & 1)] ^= 1u;
+  }
+  if (t == 0) {
+    uint32_t tw = s_cut[0], ti = s_cut[1];
+    if (s_cut[2] == NONE) {  // fewer eligible entries than need: all of them
+      tw = tsum & 0xFFFFu;
+      ti = tsum >> 16;
+    }
     write_range(a, q, tw, ti);
     victims += tw + ti;
+    scanned += s_cut[2] == NONE ? span : min(span, 32 * (s_cut[2] + 1));
   }
 }
 
-// A big window, the whole CTA: marks, one block scan over the words (thread t
-// owns words 4t .. 4t+3), the warps split the chunks.
-__device__ __forceinline__ void cta_window(const PredArgs &a, const SelLog &lg, uint32_t qi, uint32_t *sm,
-                                           uint32_t *ws, uint32_t *s_cnt, unsigned long long &scanned,
-                                           unsigned long long &victims) {
-  const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  const Geo &g = a.g;
-  uint32_t *posmap = sm, *wem = sm + POS_WORDS, *wim = wem + POS_WORDS, *wpre = wim + POS_WORDS;
-  uint32_t *roff = wpre + POS_WORDS, *kern = roff + g.N + 2;
-  const SelQuery q = load_query(a, qi);
-  for (uint32_t d = tid; d <= q.nk; d += WSEL_NT) {
-    roff[d] = __ldg(a.qroff + (uint64_t)qi * (g.N + 2) + d);
-    if (d < q.nk) kern[d] = __ldg(a.qkern + (uint64_t)qi * (g.N + 1) + d);
-  }
-  for (uint32_t w = tid; w < POS_WORDS; w += WSEL_NT) posmap[w] = 0;
-  if (tid == 0) s_cnt[0] = s_cnt[1] = 0;
-  __syncthreads();
-  const uint32_t R = roff[q.nk];
-  const uint32_t span = min(lg.tail - lg.head, min(q.need + R + lg.stale, POS_WORDS * 32));
-  const uint32_t nw = (span + 31) / 32;
-  if (q.need) {
-    mark_window<4>(a, roff, kern, R, lg.head, POS_WORDS * 32, posmap, tid, WSEL_NT);
-    __syncthreads();
-    uint32_t ca[4], ci[4], em[4], imk[4], tot = 0;
+// Copy chunks [c0, c1) of the chunk map, one warp (k_copy_fast's body over a
+// contiguous range): four descriptors, then their walk loads, in flight together.
+__device__ __forceinline__ void copy_range(const PredArgs &a, uint64_t c0, uint64_t c1,
+                                           unsigned long long &emitted) {
+  constexpr uint32_t UN = 4;
+  const uint32_t lane = threadIdx.x & 31;
+  uint2 *out = reinterpret_cast<uint2 *>(a.pairs);
+  for (uint64_t c = c0; c < c1; c += UN) {
+    uint4 m[UN];
 #pragma unroll
-    for (uint32_t u = 0; u < 4; ++u) {  // nw <= POS_WORDS = 4 * WSEL_NT
-      const uint32_t w = 4 * tid + u;
-      em[u] = imk[u] = 0;
-      if (w < nw) {
-        const uint32_t lo = w * 32, valid = span - lo >= 32 ? 0xFFFFFFFFu : (1u << (span - lo)) - 1u;
-        const uint32_t ib = __ldg(a.inact_bits + w), e = valid & ~posmap[w];
-        em[u] = e & ~ib;
-        imk[u] = e & ib;
-      }
-      ca[u] = __popc(em[u]);
-      ci[u] = __popc(imk[u]);
-      tot += ca[u] | (ci[u] << 16);
-    }
-    uint32_t tsum;
-    uint32_t pre = block_excl_scan(tot, ws, &tsum);  // packed (inactive << 16 | active)
+    for (uint32_t u = 0; u < UN; ++u) m[u] = c + u < c1 ? __ldcg(a.chunk_map + c + u) : make_uint4(0, 0, 0, 0);
+    uint32_t b[UN][4];
 #pragma unroll
-    for (uint32_t u = 0; u < 4; ++u) {
-      const uint32_t w = 4 * tid + u;
-      if (w < nw) {
-        wem[w] = em[u];
-        wim[w] = imk[u];
-        wpre[w] = pre;
-      }
-      pre += ca[u] | (ci[u] << 16);
-    }
-    __syncthreads();
-    constexpr uint32_t UC = 2;
-    uint32_t tw = 0, ti = 0;
-    const uint32_t nch = (nw + 3) / 4;
-    for (uint32_t ch0 = wid; ch0 < nch; ch0 += SEL_NW * UC) {
-      {
-        const uint32_t p0 = wpre[4 * ch0];  // the step's first chunk starts past the cut: so do the rest
-        if ((p0 & 0xFFFFu) + (p0 >> 16) >= q.need) break;
-      }
-      uint32_t wp[UC], e32[UC], i32[UC], p32[UC];
+    for (uint32_t u = 0; u < UN; ++u) {
+      const uint32_t n = m[u].w >> 16;
+      const uint32_t *lst = a.walk + (uint64_t)m[u].x * a.g.walk_cap + m[u].y;
 #pragma unroll
-      for (uint32_t u = 0; u < UC; ++u) {
-        const uint32_t w = 4 * (ch0 + u * SEL_NW) + (lane >> 3);
-        wp[u] = w;
-        e32[u] = w < nw ? wem[w] : 0u;
-        i32[u] = w < nw ? wim[w] : 0u;
-        p32[u] = w < nw ? wpre[w] : 0xFFFFFFFFu;
-      }
-      emit_chunks<UC>(a, q, lg, lane, wp, e32, i32, p32, tw, ti);
+      for (uint32_t k = 0; k < 4; ++k) b[u][k] = 32 * k + lane < n ? __ldg(lst + 32 * k + lane) : NONE;
     }
-    tw = __reduce_add_sync(0xffffffffu, tw);
-    ti = __reduce_add_sync(0xffffffffu, ti);
-    if (lane == 0 && (tw | ti)) {
-      atomicAdd(&s_cnt[0], tw);
-      atomicAdd(&s_cnt[1], ti);
+#pragma unroll
+    for (uint32_t u = 0; u < UN; ++u) {
+      const uint32_t n = m[u].w >> 16;
+      uint2 *o = out + ((unsigned long long)(m[u].w & 0xFFFFu) << 32 | m[u].z);
+#pragma unroll
+      for (uint32_t k = 0; k < 4; ++k)
+        if (32 * k + lane < n) __stcs(o + 32 * k + lane, make_uint2(b[u][k], m[u].x));
+      emitted += n;
     }
-    __syncthreads();
-  }
-  if (tid == 0) {
-    write_range(a, q, s_cnt[0], s_cnt[1]);
-    victims += s_cnt[0] + s_cnt[1];
-    if (q.need) scanned += span;
   }
 }
 
-__global__ void __launch_bounds__(WSEL_NT, 4) k_select_fast(PredArgs a) {
-  extern __shared__ uint4 sel4[];
-  __shared__ uint32_t ws[SEL_NW], s_cnt[2];
-  const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  if (__ldcg(&a.st->log_dirty)) return;  // k_select_stale's case
-  uint32_t *sm = reinterpret_cast<uint32_t *>(sel4);
-  uint32_t ccnt[NQCLS], nfast = 0, nbig = 0;
-#pragma unroll
-  for (int c = 0; c < NQCLS; ++c) {
-    ccnt[c] = __ldcg(&a.st->q_cls[c]);
-    nfast += ccnt[c];
-    if (c < (int)BIG_CLS) nbig += ccnt[c];
-  }
-  SelLog lg;
-  lg.head = __ldcg(&a.st->lrm_head);
-  lg.tail = __ldcg(&a.st->lrm_tail);
-  lg.stale = lg.tail - lg.head - __ldcg(&a.st->n_resident);
-  lg.al = (lg.head & 3u) == 0;
-  const uint32_t nitems = nbig + (nfast - nbig + SEL_NW - 1) / SEL_NW;
-  unsigned long long scanned = 0, victims = 0;
-  for (uint32_t it = blockIdx.x; it < nitems; it += gridDim.x) {
-    if (it < nbig) {
-      cta_window(a, lg, fast_query(a, ccnt, it), sm, ws, s_cnt, scanned, victims);
-    } else {
-      const uint32_t j = nbig + (it - nbig) * SEL_NW + wid;
-      if (j < nfast) warp_window(a, lg, fast_query(a, ccnt, j), sm + wid * sw_words(a.g.N), scanned, victims);
-    }
-    __syncthreads();  // the next item reuses the shared state
-  }
-  scanned = __reduce_add_sync(0xffffffffu, (unsigned)scanned);
-  victims = __reduce_add_sync(0xffffffffu, (unsigned)victims);
-  if (lane == 0 && (scanned | victims)) {
-    ctr_add(a.st, DUM_CTR_FAST_SCANNED, scanned);
-    ctr_add(a.st, DUM_CTR_FAST_VICTIMS, victims);
-  }
-}
+constexpr uint32_t CPW = 8;  // k_window_fast: copy chunks per claim of a copy warp
 
 // One warp step of the stale-entry path: the 32 log entries at positions
 // head + r0 + lane (r0 a multiple of 32 relative to head, so that one
@@ -612,153 +638,252 @@ __device__ __forceinline__ void step_masks(const SelectOut &so, const uint32_t *
 
 constexpr uint32_t FB = 8;  // warp steps with their entry loads in flight together
 
-__global__ void __launch_bounds__(WSEL_NT) k_select_stale(PredArgs a) {
-  __shared__ uint32_t kern[MAXN + 1], roff[MAXN + 2];
-  __shared__ uint32_t posmap[POS_WORDS];
-  __shared__ uint32_t seg_cnt[FSEG_MAX], seg_pre[FSEG_MAX];
-  __shared__ uint32_t s_tw, s_ti;
-  constexpr uint32_t NW = WSEL_NT / 32;
+// The selection of one fast query over a log with stale entries (the selection group; see
+// above): marks, pass 1 per-segment counts, segment prefix, pass 2 emit.
+__device__ __forceinline__ void sel_stale(const PredArgs &a, uint32_t qi, uint32_t head, uint32_t tail,
+                                        uint32_t stale, uint32_t *kern, uint32_t *roff, uint32_t *posmap,
+                                        uint32_t *seg_cnt, uint32_t *seg_pre, uint32_t &s_tw, uint32_t &s_ti) {
+  constexpr uint32_t NW = SG_NT / 32;
   const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const Geo &g = a.g;
   const SelectOut &so = a.so;
-  if (!__ldcg(&a.st->log_dirty)) return;  // k_select_fast's case
-  uint32_t ccnt[NQCLS], nfast = 0;
-#pragma unroll
-  for (int c = 0; c < NQCLS; ++c) {
-    ccnt[c] = __ldcg(&a.st->q_cls[c]);
-    nfast += ccnt[c];
+  const uint32_t nk = __ldg(a.qnk + qi);
+  for (uint32_t d = tid; d <= nk; d += SG_NT) {
+    roff[d] = __ldg(a.qroff + (uint64_t)qi * (g.N + 2) + d);
+    if (d < nk) kern[d] = __ldg(a.qkern + (uint64_t)qi * (g.N + 1) + d);
   }
-  const uint32_t head = __ldcg(&a.st->lrm_head);
-  const uint32_t tail = __ldcg(&a.st->lrm_tail);
-  const uint32_t stale = tail - head - __ldcg(&a.st->n_resident);
-  for (uint32_t bq = blockIdx.x; bq < nfast; bq += gridDim.x) {
-    const uint32_t qi = fast_query(a, ccnt, bq);
-    const uint32_t nk = __ldg(a.qnk + qi);
-    for (uint32_t d = tid; d <= nk; d += WSEL_NT) {
-      roff[d] = __ldg(a.qroff + (uint64_t)qi * (g.N + 2) + d);
-      if (d < nk) kern[d] = __ldg(a.qkern + (uint64_t)qi * (g.N + 1) + d);
-    }
-    for (uint32_t w = tid; w < POS_WORDS; w += WSEL_NT) posmap[w] = 0;
-    if (tid == 0) {
-      s_tw = 0;
-      s_ti = 0;
-    }
-    const uint32_t need = __ldg(a.qneed + qi);
-    const unsigned long long bwb = __ldg(a.qvb + 2 * qi), binv = __ldg(a.qvb + 2 * qi + 1);
-    const bool ok = bwb + need <= so.cap && binv + need <= so.cap;
-    __syncthreads();
-    const uint32_t R = nk ? roff[nk] : 0;
-    uint32_t nseg = 0;
-    if (need) {
-      // 1. the window's resident blocks: their log positions into the bitmap
-      {
-        constexpr uint32_t MU = 4;  // loads in flight per thread
-        uint32_t lo = 0;
-        for (uint32_t x0 = tid; x0 < R; x0 += WSEL_NT * MU) {
-          uint32_t r[MU];
+  for (uint32_t w = tid; w < POS_WORDS; w += SG_NT) posmap[w] = 0;
+  if (tid == 0) {
+    s_tw = 0;
+    s_ti = 0;
+  }
+  const uint32_t need = __ldg(a.qneed + qi);
+  const unsigned long long bwb = __ldg(a.qvb + 2 * qi), binv = __ldg(a.qvb + 2 * qi + 1);
+  const bool ok = bwb + need <= so.cap && binv + need <= so.cap;
+  gsync();
+  const uint32_t R = nk ? roff[nk] : 0;
+  uint32_t nseg = 0;
+  if (need) {
+    // 1. the window's resident blocks: their log positions into the bitmap
+    {
+      constexpr uint32_t MU = 4;  // loads in flight per thread
+      uint32_t lo = 0;
+      for (uint32_t x0 = tid; x0 < R; x0 += SG_NT * MU) {
+        uint32_t r[MU];
 #pragma unroll
-          for (uint32_t u = 0; u < MU; ++u) {
-            const uint32_t x = x0 + u * WSEL_NT;
-            r[u] = NONE;
-            if (x < R) {
-              while (roff[lo + 1] <= x) ++lo;
-              r[u] = __ldg(a.respos + (uint64_t)kern[lo] * g.walk_cap + (x - roff[lo])) - head;
+        for (uint32_t u = 0; u < MU; ++u) {
+          const uint32_t x = x0 + u * SG_NT;
+          r[u] = NONE;
+          if (x < R) {
+            while (roff[lo + 1] <= x) ++lo;
+            r[u] = __ldg(a.respos + (uint64_t)kern[lo] * g.walk_cap + (x - roff[lo])) - head;
+          }
+        }
+#pragma unroll
+        for (uint32_t u = 0; u < MU; ++u)
+          if (r[u] < POS_WORDS * 32) atomicOr(&posmap[r[u] >> 5], 1u << (r[u] & 31));
+      }
+    }
+    const uint32_t span = min(tail - head, min(need + R + stale, POS_WORDS * 32));
+    // segments of FSEG positions relative to head; a warp step covers 32
+    nseg = (span + FSEG - 1) / FSEG;
+    gsync();
+    // 2. pass 1: eligible entries per segment (active | inactive << 16)
+    for (uint32_t sg = wid; sg < nseg; sg += NW) {
+      uint32_t na = 0, ni = 0;
+      for (uint32_t k0 = 0; k0 < FSEG / 32; k0 += FB) {
+        uint32_t v[FB];
+#pragma unroll
+        for (uint32_t u = 0; u < FB; ++u) {
+          const uint32_t p = head + sg * FSEG + 32 * (k0 + u) + lane;
+          v[u] = p < tail ? __ldcg(so.lrm_blk + p) : 0u;
+        }
+#pragma unroll
+        for (uint32_t u = 0; u < FB; ++u) {
+          uint32_t ma, mi;
+          step_masks(so, posmap, head, tail, lane, sg * FSEG + 32 * (k0 + u), v[u], ma, mi);
+          na += __popc(ma);
+          ni += __popc(mi);
+        }
+      }
+      if (lane == 0) seg_cnt[sg] = na | (ni << 16);
+    }
+    gsync();
+    // 3. segment prefix (one warp; nseg <= 32)
+    if (wid == 0) {
+      const uint32_t c = lane < nseg ? seg_cnt[lane] : 0u;
+      uint32_t x = c;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= (uint32_t)o) x += y;
+      }
+      if (lane < nseg) seg_pre[lane] = x - c;
+    }
+    gsync();
+    // 4. pass 2: the entries of combined rank < need, at their list ranks
+    const uint32_t lt = (1u << lane) - 1;
+    uint32_t tw = 0, ti = 0;
+    for (uint32_t sg = wid; sg < nseg; sg += NW) {
+      const uint32_t pre = seg_pre[sg];
+      uint32_t rw = pre & 0xFFFFu, ri = pre >> 16;
+      for (uint32_t k0 = 0; k0 < FSEG / 32 && rw + ri < need; k0 += FB) {
+        uint32_t v[FB];
+#pragma unroll
+        for (uint32_t u = 0; u < FB; ++u) {
+          const uint32_t p = head + sg * FSEG + 32 * (k0 + u) + lane;
+          v[u] = p < tail ? __ldcg(so.lrm_blk + p) : 0u;
+        }
+#pragma unroll
+        for (uint32_t u = 0; u < FB; ++u) {
+          uint32_t ma, mi;
+          step_masks(so, posmap, head, tail, lane, sg * FSEG + 32 * (k0 + u), v[u], ma, mi);
+          const uint32_t ra = rw + __popc(ma & lt), rr = ri + __popc(mi & lt);
+          const bool ea = (ma >> lane) & 1u, ei = (mi >> lane) & 1u;
+          if ((ea || ei) && ra + rr < need) {
+            if (ok) {
+              if (ei) so.inv[binv + rr] = v[u] & 0x7FFFFFFFu;
+              else so.wb[bwb + ra] = v[u];
             }
+            tw += ea;
+            ti += ei;
           }
-#pragma unroll
-          for (uint32_t u = 0; u < MU; ++u)
-            if (r[u] < POS_WORDS * 32) atomicOr(&posmap[r[u] >> 5], 1u << (r[u] & 31));
+          rw += __popc(ma);
+          ri += __popc(mi);
         }
       }
-      const uint32_t span = min(tail - head, min(need + R + stale, POS_WORDS * 32));
-      // segments of FSEG positions relative to head; a warp step covers 32
-      nseg = (span + FSEG - 1) / FSEG;
-      __syncthreads();
-      // 2. pass 1: eligible entries per segment (active | inactive << 16)
-      for (uint32_t sg = wid; sg < nseg; sg += NW) {
-        uint32_t na = 0, ni = 0;
-        for (uint32_t k0 = 0; k0 < FSEG / 32; k0 += FB) {
-          uint32_t v[FB];
-#pragma unroll
-          for (uint32_t u = 0; u < FB; ++u) {
-            const uint32_t p = head + sg * FSEG + 32 * (k0 + u) + lane;
-            v[u] = p < tail ? __ldcg(so.lrm_blk + p) : 0u;
-          }
-#pragma unroll
-          for (uint32_t u = 0; u < FB; ++u) {
-            uint32_t ma, mi;
-            step_masks(so, posmap, head, tail, lane, sg * FSEG + 32 * (k0 + u), v[u], ma, mi);
-            na += __popc(ma);
-            ni += __popc(mi);
-          }
-        }
-        if (lane == 0) seg_cnt[sg] = na | (ni << 16);
-      }
-      __syncthreads();
-      // 3. segment prefix (one warp; nseg <= 32)
-      if (wid == 0) {
-        const uint32_t c = lane < nseg ? seg_cnt[lane] : 0u;
-        uint32_t x = c;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-          if (lane >= (uint32_t)o) x += y;
-        }
-        if (lane < nseg) seg_pre[lane] = x - c;
-      }
-      __syncthreads();
-      // 4. pass 2: the entries of combined rank < need, at their list ranks
-      const uint32_t lt = (1u << lane) - 1;
-      uint32_t tw = 0, ti = 0;
-      for (uint32_t sg = wid; sg < nseg; sg += NW) {
-        const uint32_t pre = seg_pre[sg];
-        uint32_t rw = pre & 0xFFFFu, ri = pre >> 16;
-        for (uint32_t k0 = 0; k0 < FSEG / 32 && rw + ri < need; k0 += FB) {
-          uint32_t v[FB];
-#pragma unroll
-          for (uint32_t u = 0; u < FB; ++u) {
-            const uint32_t p = head + sg * FSEG + 32 * (k0 + u) + lane;
-            v[u] = p < tail ? __ldcg(so.lrm_blk + p) : 0u;
-          }
-#pragma unroll
-          for (uint32_t u = 0; u < FB; ++u) {
-            uint32_t ma, mi;
-            step_masks(so, posmap, head, tail, lane, sg * FSEG + 32 * (k0 + u), v[u], ma, mi);
-            const uint32_t ra = rw + __popc(ma & lt), rr = ri + __popc(mi & lt);
-            const bool ea = (ma >> lane) & 1u, ei = (mi >> lane) & 1u;
-            if ((ea || ei) && ra + rr < need) {
-              if (ok) {
-                if (ei) so.inv[binv + rr] = v[u] & 0x7FFFFFFFu;
-                else so.wb[bwb + ra] = v[u];
-              }
-              tw += ea;
-              ti += ei;
-            }
-            rw += __popc(ma);
-            ri += __popc(mi);
-          }
-        }
-      }
-      tw = __reduce_add_sync(0xffffffffu, tw);
-      ti = __reduce_add_sync(0xffffffffu, ti);
-      if (lane == 0 && (tw | ti)) {
-        atomicAdd(&s_tw, tw);
-        atomicAdd(&s_ti, ti);
-      }
-      __syncthreads();
     }
-    if (tid == 0) {
-      uint64_t *o = so.out_range + 4ull * qi;
-      o[0] = bwb;
-      o[1] = bwb + (ok ? s_tw : 0);
-      o[2] = binv;
-      o[3] = binv + (ok ? s_ti : 0);
-      // log entries read by the selection: the segments (each pass reads them)
-      ctr_add(a.st, DUM_CTR_FAST_SCANNED, need ? min(tail - head, nseg * FSEG) : 0u);
-      ctr_add(a.st, DUM_CTR_FAST_VICTIMS, s_tw + s_ti);
-      ctr_add(a.st, DUM_CTR_FAST_DIRTY, 1);
+    tw = __reduce_add_sync(0xffffffffu, tw);
+    ti = __reduce_add_sync(0xffffffffu, ti);
+    if (lane == 0 && (tw | ti)) {
+      atomicAdd(&s_tw, tw);
+      atomicAdd(&s_ti, ti);
     }
-    __syncthreads();  // the next query reuses the shared state
+    gsync();
+  }
+  if (tid == 0) {
+    uint64_t *o = so.out_range + 4ull * qi;
+    o[0] = bwb;
+    o[1] = bwb + (ok ? s_tw : 0);
+    o[2] = binv;
+    o[3] = binv + (ok ? s_ti : 0);
+    // log entries read by the selection: the segments (each pass reads them)
+    ctr_add(a.st, DUM_CTR_FAST_SCANNED, need ? min(tail - head, nseg * FSEG) : 0u);
+    ctr_add(a.st, DUM_CTR_FAST_VICTIMS, s_tw + s_ti);
+    ctr_add(a.st, DUM_CTR_FAST_DIRTY, 1);
+  }
+}
+
+
+// a7 + a8 of every fast query in one persistent, warp-specialised kernel.
+// Warps [0, SG_NT / 32) of each CTA form the selection group: it claims
+// queries (k_chain's class order, biggest selection first; sel_staged on a
+// clean log, sel_stale on a log with stale entries) until the selection queue
+// is empty, then joins the copy.  The other warps claim copy items (CPW
+// chunks of k_chain's chunk map each) from the start, so that the pair stream
+// keeps HBM busy while the selection waits on its staged loads.  Queues: the
+// DevState counters sel_queue / copy_queue (k_pred_epilogue clears them).
+__global__ void __launch_bounds__(WSEL_NT, 3) k_window_fast(PredArgs a) {
+  extern __shared__ uint4 stage4[];  // SR_SMEM_WORDS: the staged selection's buffers
+  __shared__ uint32_t posmap[POS_WORDS], roff[MAXN + 2], kern[MAXN + 1], ws[SG_NT / 32], s_cut[3], s_item;
+  __shared__ uint32_t seg_cnt[FSEG_MAX], seg_pre[FSEG_MAX], s_tw, s_ti;
+  __shared__ __align__(8) unsigned long long bar[3];
+  const uint32_t tid = threadIdx.x, lane = tid & 31;
+  StageSm S;
+  S.ibits = reinterpret_cast<uint32_t *>(stage4);
+  S.wpre = S.ibits + POS_WORDS;
+  S.lbuf = S.wpre + POS_WORDS;
+  S.bar = bar;
+  if (tid == 0) {
+    for (int i = 0; i < 3; ++i) mbar_init(&bar[i]);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  uint32_t ph[3] = {0, 0, 0};  // the barriers' phase parities (every selection-group thread in step)
+#ifdef EXP_TRACE
+  if (tid == 0) TR(4 * blockIdx.x, gtime());
+#endif
+  const bool sel = __ldcg(&a.st->log_dirty) == 0;  // a clean log: sel_staged; else sel_stale
+  SelLog lg;
+  lg.head = __ldcg(&a.st->lrm_head);
+  lg.tail = __ldcg(&a.st->lrm_tail);
+  lg.stale = lg.tail - lg.head - __ldcg(&a.st->n_resident);
+  lg.al = (lg.head & 3u) == 0;
+  unsigned long long scanned = 0, victims = 0, emitted = 0;
+  if (tid < SG_NT) {  // the selection group: a query per item
+#ifdef EXP_COPY_ONLY
+    return;
+#endif
+    uint32_t ccnt[NQCLS], n1 = 0;
+#pragma unroll
+    for (int c = 0; c < NQCLS; ++c) {
+      ccnt[c] = __ldcg(&a.st->q_cls[c]);
+      n1 += ccnt[c];
+    }
+    for (;;) {
+      if (tid == 0) s_item = atomicAdd(&a.st->sel_queue, 1u);
+      gsync();
+      const uint32_t it = s_item;
+      if (it >= n1) break;
+      SelRec r;
+      {  // the item's record: class-order position -> (class, rank) as in qperm
+        uint32_t cq = NQCLS, rq = it;
+#pragma unroll
+        for (int c = 0; c < NQCLS; ++c)
+          if (cq == NQCLS) {
+            if (rq < ccnt[c]) cq = c;
+            else rq -= ccnt[c];
+          }
+        const uint4 *p = a.selrec + 3 * ((uint64_t)cq * a.nq + rq);
+        r.x = __ldcg(p);
+        r.y = __ldcg(p + 1);
+        r.z = __ldcg(p + 2);
+      }
+#ifdef EXP_TRACE
+      if (tid == 0) TR(4 * 4096 + 8 * it, gtime());
+#endif
+      if (sel)
+        sel_staged(a, lg, r, S, posmap, roff, kern, ws, s_cut, ph, scanned, victims, it);
+      else
+        sel_stale(a, r.x.x, lg.head, lg.tail, lg.stale, kern, roff, posmap, seg_cnt, seg_pre, s_tw, s_ti);
+#ifdef EXP_TRACE
+      if (tid == 0) TR(4 * 4096 + 8 * it + 1, gtime());
+#endif
+      gsync();  // the next item reuses the shared state
+    }
+#ifdef EXP_TRACE
+    if (tid == 0) TR(4 * blockIdx.x + 1, gtime());
+#endif
+  }
+  {  // the copy warps; the selection group joins them once its queue is empty
+#ifdef EXP_SEL_ONLY
+    const unsigned long long G = 0;
+#else
+    const unsigned long long G = min((unsigned long long)a.chunk_cap, __ldcg(&a.st->pool_chunks));
+#endif
+    for (;;) {
+      unsigned long long c0 = 0;
+      if (lane == 0) c0 = atomicAdd(&a.st->copy_queue, (unsigned long long)CPW);
+      c0 = __shfl_sync(0xffffffffu, c0, 0);
+      if (c0 >= G) break;
+      copy_range(a, c0, min((unsigned long long)G, c0 + CPW), emitted);
+    }
+#ifdef EXP_TRACE
+    if (tid == SG_NT) TR(4 * blockIdx.x + 2, gtime());  // (a copy warp's end)
+#endif
+  }
+#ifdef EXP_TRACE
+  if (lane == 0) atomicMax(&g_tr[4 * blockIdx.x + 3], gtime());
+#endif
+  emitted = __reduce_add_sync(0xffffffffu, (unsigned)emitted) / 32;
+  if (lane == 0 && emitted) {
+    ctr_add(a.st, DUM_CTR_EMITTED, emitted);
+    ctr_add(a.st, DUM_CTR_GATHERED, emitted);
+    ctr_add(a.st, DUM_CTR_FAST_EMITTED, emitted);
+  }
+  if (tid == 0 && (scanned | victims)) {
+    ctr_add(a.st, DUM_CTR_FAST_SCANNED, scanned);
+    ctr_add(a.st, DUM_CTR_FAST_VICTIMS, victims);
   }
 }
 
@@ -810,41 +935,33 @@ cudaError_t launch_walk_res(dum_engine *e, cudaStream_t s) {
 }
 
 cudaError_t launch_window(dum_engine *e, const PredArgs &a, bool select, cudaStream_t s) {
-  const int ssmem = (int)(sel_smem_words(e->g.N) * 4);
-  if (!e->copy_grid || e->sel_smem != ssmem) {
-    int dev = 0, sms = 148, nc = 1, ns = 1, nt = 1;
+  if (!e->copy_grid) {
+    int dev = 0, sms = 148, nc = 1, ns = 1;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    // the attribute is per device and function: raised by every engine on its own device
-    if (ssmem > 48 * 1024) cudaFuncSetAttribute(k_select_fast, cudaFuncAttributeMaxDynamicSharedMemorySize, ssmem);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nc, k_copy_fast, COPY_NT, 0);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ns, k_select_fast, WSEL_NT, ssmem);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nt, k_select_stale, WSEL_NT, 0);
+    // the attribute is per device and function: every engine sets it on its own device
+    cudaFuncSetAttribute(k_window_fast, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(SR_SMEM_WORDS * 4));
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ns, k_window_fast, WSEL_NT, SR_SMEM_WORDS * 4);
     e->copy_grid = (uint32_t)std::max(1, nc * sms);
     e->sel_grid = (uint32_t)std::max(1, ns * sms);
-    e->stale_grid = (uint32_t)std::max(1, nt * sms);
-    e->sel_smem = ssmem;
   }
-  if (select) {
-    // the selection on the third side stream, beside the copy (each kernel
-    // exits at once in the other's case: clean log / stale entries)
-    cudaEventRecord(e->ev_fork2, s);
-    cudaStreamWaitEvent(e->side3, e->ev_fork2, 0);
-    {
-      TimerScope t(e, DUM_T_SELECT_FAST, e->side3);
-      k_select_fast<<<std::min(a.nq, e->sel_grid), WSEL_NT, ssmem, e->side3>>>(a);
-      k_select_stale<<<std::min(a.nq, e->stale_grid), WSEL_NT, 0, e->side3>>>(a);
-    }
-    cudaEventRecord(e->ev_join3, e->side3);
-    e->kernel_launches += 2;
-  }
-  {  // every fast window's pairs: the flat copy over k_chain's chunk map
+  if (select) {  // the pairs and the selection of the fast windows: one persistent kernel
+    TimerScope t(e, DUM_T_SELECT_FAST, s);
+    k_window_fast<<<e->sel_grid, WSEL_NT, SR_SMEM_WORDS * 4, s>>>(a);
+  } else {  // the pairs only: the flat copy over k_chain's chunk map
     TimerScope t(e, DUM_T_PREDICT, s);
     k_copy_fast<<<e->copy_grid, COPY_NT, 0, s>>>(a);
   }
   e->kernel_launches += 1;
-  if (select) cudaStreamWaitEvent(s, e->ev_join3, 0);
   return cudaGetLastError();
 }
 
 }  // namespace dum
+
+#ifdef EXP_TRACE
+extern "C" int dum_exp_trace(void *dst, unsigned long long bytes, int clear) {
+  if (clear) return (int)cudaMemset(g_tr_ptr(), 0, sizeof(g_tr));
+  return (int)cudaMemcpyFromSymbol(dst, g_tr, bytes < sizeof(g_tr) ? bytes : sizeof(g_tr));
+}
+#endif

@@ -13,7 +13,7 @@ constexpr uint32_t HOLD_MAX = 64;   // walk index: holders recorded per block
 constexpr uint32_t CONF_MAX = 64;   // walk index: conflicting exec IDs recorded per walk
 constexpr uint32_t CHUNK_B = 128;   // window blocks per copy chunk (one warp: 4 coalesced steps)
 constexpr int COPY_NT = 256;        // k_copy_fast threads
-constexpr int WSEL_NT = 256;        // k_select_fast threads
+constexpr int WSEL_NT = 256;        // k_window_fast threads
 constexpr uint32_t POS_WORDS = 1024;  // k_window position bitmap: log positions [head, head + 32768)
 
 struct PredArgs {
@@ -50,6 +50,10 @@ struct PredArgs {
   uint32_t *qroff;    // [nq][N+2] prefix of the lists' resident blocks (fast queries, select)
   uint32_t *qneed;    // [nq] victims to find (fast queries, select)
   unsigned long long *qvb;  // [nq][2] reserved write-back / invalidate offsets (fast queries, select)
+  // k_window_fast: per fast query (class order, like qperm) a 48 B record
+  //   {qi, nk, need, nw}, {-, ok, -, -}, {wb base, inv base}
+  uint4 *selrec;
+  uint32_t lrm_cap;  // LRM log entries allocated (k_window_fast clamps its bulk loads to it)
   uint4 *chunk_map;  // [chunk_cap] copy chunks of the fast queries (k_chain -> k_copy_fast):
                     // {exec ID, first list entry, pair slot lo 32, pair slot hi 16 | entries << 16}
   uint64_t chunk_cap;

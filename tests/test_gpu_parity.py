@@ -435,8 +435,8 @@ def test_fast_selection_on_a_log_with_stale_entries(seed):
     """Write-backs leave stale entries in the LRM log (PAPER.md L238-L241:
     the victims are resident blocks; a logged block that left HBM is skipped)
     until the next compaction: the fast path's per-entry selection
-    (k_select_fast) must give the oracle's victims.  The clean-log path
-    (k_select_warp) answers the same queries after the log is reloaded."""
+    (k_select_stale) must give the oracle's victims.  The clean-log path
+    (k_window_fast) answers the same queries after the log is reloaded."""
     W, C = 96, 40
     rng = np.random.default_rng(77 + seed)
     arena = torch.zeros(W * (2 << 20), dtype=torch.uint8).pin_memory()

@@ -1,6 +1,6 @@
 """Path coverage of the GPU suite (runs last: file order).  Every code path
 that answers the engine's work must have answered some of the suite's:
-  Q_FAST / Q_SLOW        fast windows (k_copy_fast + k_select_warp / k_select_fast)
+  Q_FAST / Q_SLOW        fast windows (k_window_fast: pairs + selection; k_copy_fast without selection)
                          and the exact kernel (k_predict)
   Q_NODUP / Q_DUP / Q_FALLBACK  the exact kernel's window-set, duplicate and
                          fallback paths
