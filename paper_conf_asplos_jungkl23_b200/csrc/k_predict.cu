@@ -253,6 +253,9 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
       a.qnk[qi] = nk;
     }
     slow = anchored || __any_sync(0xffffffffu, conflict);
+#ifdef EXP_ALL_EXACT
+    slow = true;
+#endif
     const bool s_unrec = __any_sync(0xffffffffu, unrec);
     if (lane == 0 && slow) ctr_add(a.st, anchored ? DUM_CTR_SLOW_ANCHOR : s_unrec ? DUM_CTR_SLOW_UNRECORDED
                                                                            : DUM_CTR_SLOW_CONFLICT, 1);

@@ -450,6 +450,10 @@ __device__ __forceinline__ void sel_staged(const PredArgs &a, const SelLog &lg, 
   gsync();
   TRI(2);
   const uint32_t R = roff[q.nk];
+#ifdef EXP_TRACE
+  if (t == 0) TR(4 * 4096 + 8 * it + 6, (unsigned long long)R << 32 | nw);
+  if (t == 0) TR(4 * 4096 + 8 * it + 7, (unsigned long long)q.nk << 32 | q.need);
+#endif
   const uint32_t span = min(lg.tail - lg.head, min(q.need + R + lg.stale, POS_WORDS * 32));
   const uint32_t nseg = (span + SR_SEG - 1) / SR_SEG;
   if (t == 0) {
@@ -458,37 +462,47 @@ __device__ __forceinline__ void sel_staged(const PredArgs &a, const SelLog &lg, 
     if (nseg > 1) issue_segment(a, lg, S, 1, span);
     issue_bits(a, S, nw);
   }
+  TRI(5);
   // marks: the window's resident positions below nw * 32, flat over the lists'
-  // entries (coalesced loads, MU in flight per thread); a walk's resident
-  // blocks sit mostly at consecutive log positions, so the lanes hitting one
-  // bitmap word combine their bits first (one shared atomic per word)
+  // entries.  A walk's resident blocks sit mostly at consecutive log
+  // positions: each lane takes ML consecutive entries (all loads in flight,
+  // L1-served), ORs the bits of one bitmap word in a register and flushes it
+  // with one shared atomic when the word changes.  (Measured against coalesced
+  // loads + a warp match / reduce or a segmented shuffle OR per word: slower.)
   {
-    constexpr uint32_t MU = 8;
+    constexpr uint32_t ML = 16;
     uint32_t lo = 0;
-    for (uint32_t xb = 0; xb < R; xb += SG_NT * MU) {  // (warp-uniform trip count: the warp intrinsics below)
-      uint32_t rv[MU];
+    for (uint32_t xb = 0; xb < R; xb += SG_NT * ML) {
+      const uint32_t x0 = xb + t * ML;
+      uint32_t rv[ML];
+      uint32_t l2 = lo;
 #pragma unroll
-      for (uint32_t u = 0; u < MU; ++u) {
-        const uint32_t x = xb + u * SG_NT + t;
-        rv[u] = NONE;
+      for (uint32_t j = 0; j < ML; ++j) {
+        const uint32_t x = x0 + j;
+        rv[j] = NONE;
         if (x < R) {
-          while (roff[lo + 1] <= x) ++lo;
-          rv[u] = __ldg(a.respos + (uint64_t)kern[lo] * g.walk_cap + (x - roff[lo])) - lg.head;
+          while (roff[l2 + 1] <= x) ++l2;
+          rv[j] = __ldg(a.respos + (uint64_t)kern[l2] * g.walk_cap + (x - roff[l2])) - lg.head;
         }
       }
+      lo = l2;
+      uint32_t cw = NONE, cb = 0;
 #pragma unroll
-      for (uint32_t u = 0; u < MU; ++u) {
-        const uint32_t wd = rv[u] < nw * 32 ? rv[u] >> 5 : NONE;
-        const uint32_t m = __match_any_sync(0xffffffffu, wd);
-        const uint32_t bits = __reduce_or_sync(m, wd != NONE ? 1u << (rv[u] & 31) : 0u);
-        if (wd != NONE && lane == (uint32_t)__ffs(m) - 1) atomicOr(&posmap[wd], bits);
+      for (uint32_t j = 0; j < ML; ++j) {
+        const uint32_t wd = rv[j] < nw * 32 ? rv[j] >> 5 : NONE;
+        if (wd != cw) {
+          if (cw != NONE) atomicOr(&posmap[cw], cb);
+          cw = wd;
+          cb = 0;
+        }
+        if (wd != NONE) cb |= 1u << (rv[j] & 31);
       }
+      if (cw != NONE) atomicOr(&posmap[cw], cb);
     }
   }
   TRI(3);
   mbar_wait(S.bar, ph[0]);  // the inactive-entry words
   ph[0] ^= 1u;
-  TRI(5);
   gsync();
   // eligible entries per word (~marked & valid, split by the inactive bits),
   // rank bases by one group scan, the cut
@@ -893,6 +907,9 @@ static uint32_t index_grid(const dum_engine *e) {
 
 // Build end: the walk index of the walks just rebuilt (k_walk / k_walk_slow).
 cudaError_t launch_walk_index(dum_engine *e, cudaStream_t main) {
+#ifdef EXP_ALL_EXACT
+  return cudaSuccess;
+#endif
   // on the third side stream: the next predict's prelude (residency load, ingest,
   // queries, walk residency facts) overlaps it; k_chain waits for ev_widx
   cudaEventRecord(e->ev_fork2, main);
@@ -925,6 +942,9 @@ __global__ void __launch_bounds__(256) k_log_bits(const uint32_t *__restrict__ l
 
 // Predict time: per-walk residency facts for the fast selection.
 cudaError_t launch_walk_res(dum_engine *e, cudaStream_t s) {
+#ifdef EXP_ALL_EXACT
+  return cudaSuccess;
+#endif
   TimerScope t(e, DUM_T_WALK_RES, s);
   k_walk_res<<<index_grid(e), IX_NT, 0, s>>>(e->d_walk, e->d_walk_len, e->g.walk_cap, e->d_state, e->d_res_bits,
                                              e->d_logpos, e->d_wnr, e->d_wnres, e->d_respos);

@@ -50,9 +50,20 @@ st = p1[p1[:, 2] > 0]
 if len(st):
     res["to_roff_us"] = pc((st[:, 2] - st[:, 0]) / 1000.0)
     res["to_marks_us"] = pc((st[:, 3] - st[:, 2]) / 1000.0)
-    res["lists_land_us"] = pc((st[:, 5] - st[:, 2]) / 1000.0)
+    res["tma_issue_us"] = pc((st[:, 5] - st[:, 2]) / 1000.0)
     res["to_scan_us"] = pc((st[:, 4] - st[:, 3]) / 1000.0)
     res["emit_us"] = pc((st[:, 1] - st[:, 4]) / 1000.0)
     res["staged_items"] = len(st)
+    R = (st[:, 6] >> 32).astype(np.int64)
+    nw = (st[:, 6] & 0xFFFFFFFF).astype(np.int64)
+    nk = (st[:, 7] >> 32).astype(np.int64)
+    need = (st[:, 7] & 0xFFFFFFFF).astype(np.int64)
+    res["R"] = pc(R)
+    res["nw"] = pc(nw)
+    res["nk"] = pc(nk)
+    res["need"] = pc(need)
+    top = np.argsort(-(st[:, 3] - st[:, 2]).astype(np.int64))[:8]
+    res["slowest_marks"] = [[float((st[k, 3] - st[k, 2]) / 1000.0), int(R[k]), int(nw[k]), int(nk[k]), int(need[k])]
+                            for k in top]
 json.dump(res, open(sys.argv[1], "w"), indent=1)
 print(json.dumps(res, indent=1))
