@@ -77,6 +77,37 @@ def build(force: bool = False, verbose: bool = False, ptxas_v: bool = False, che
     return out
 
 
+HOOK_SRC = os.path.join(CSRC, "alloc_hook.cpp")
+HOOK_OUT = os.path.join(HERE, "libdeepum_hook.so")
+
+
+def build_hook(force: bool = False) -> str:
+    """libdeepum_hook.so: host C++ against PyTorch's c10 /
+    c10_cuda (its CUDA caching allocator's trace tracker) and libdeepum_b200.so."""
+    import torch
+    import torch.utils.cpp_extension as ce
+    deps = [HOOK_SRC, os.path.join(HERE, "..", "include", "deepum_hook.h"),
+            os.path.join(HERE, "..", "include", "deepum_b200.h")]
+    if not force and os.path.exists(HOOK_OUT) and all(os.path.getmtime(p) <= os.path.getmtime(HOOK_OUT)
+                                                      for p in deps):
+        return HOOK_OUT
+    tlib = os.path.join(os.path.dirname(torch.__file__), "lib")
+    abi = int(torch._C._GLIBCXX_USE_CXX11_ABI)
+    tmp = HOOK_OUT + ".tmp%d" % os.getpid()
+    cmd = ["g++", "-O2", "-std=c++17", "-fPIC", "-shared", "-D_GLIBCXX_USE_CXX11_ABI=%d" % abi,
+           "-I" + os.path.join(HERE, "..", "include"), "-I/usr/local/cuda/include",
+           *["-I" + p for p in ce.include_paths()], HOOK_SRC, "-o", tmp,
+           "-L" + tlib, "-lc10", "-lc10_cuda", "-L/usr/local/cuda/lib64", "-lcudart",
+           "-L" + HERE, "-ldeepum_b200", "-Wl,-rpath,$ORIGIN", "-Wl,-rpath," + tlib]
+    r = subprocess.run(cmd, capture_output=True, text=True)
+    if r.returncode != 0:
+        raise RuntimeError("g++ failed for alloc_hook.cpp:\n%s\n%s" % (r.stdout, r.stderr))
+    os.replace(tmp, HOOK_OUT)
+    return HOOK_OUT
+
+
 if __name__ == "__main__":
     print(build(force="--force" in sys.argv, verbose="--verbose" in sys.argv, ptxas_v="-v" in sys.argv,
                 checks="--checks" in sys.argv))
+    if "--checks" not in sys.argv:
+        print(build_hook(force="--force" in sys.argv))

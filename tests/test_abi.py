@@ -1,5 +1,5 @@
-"""The C-ABI library loads and exports every symbol include/deepum_b200.h
-declares (no compute calls: CPU only)."""
+"""The C-ABI libraries load and export every symbol include/deepum_b200.h and
+include/deepum_hook.h declare (no compute calls: CPU only)."""
 import ctypes
 import os
 import re
@@ -8,10 +8,11 @@ import pytest
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 HDR = os.path.join(ROOT, "include", "deepum_b200.h")
+HOOK_HDR = os.path.join(ROOT, "include", "deepum_hook.h")
 
 
-def _declared():
-    txt = open(HDR).read()
+def _declared(hdr=HDR):
+    txt = open(hdr).read()
     txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
     return sorted(set(re.findall(r"\b(dum_[a-z_0-9]+)\s*\(", txt)))
 
@@ -28,6 +29,17 @@ def test_library_exports_every_declared_symbol():
     so = bld.build()
     lib = ctypes.CDLL(so)
     missing = [n for n in _declared() if not hasattr(lib, n)]
+    assert not missing, missing
+
+
+def test_hook_library_exports_every_declared_symbol():
+    from paper_conf_asplos_jungkl23_b200 import build as bld
+    bld.build()
+    import torch  # noqa: F401  (libc10 / libc10_cuda)
+    lib = ctypes.CDLL(bld.build_hook())
+    names = _declared(HOOK_HDR)
+    assert "dum_hook_flush" in names
+    missing = [n for n in names if not hasattr(lib, n)]
     assert not missing, missing
 
 
