@@ -106,8 +106,31 @@ def build_hook(force: bool = False) -> str:
     return HOOK_OUT
 
 
+UM_SRC = os.path.join(CSRC, "um", "um_runtime.cu")
+UM_OUT = os.path.join(HERE, "libdeepum_um.so")
+
+
+def build_um(force: bool = False) -> str:
+    """libdeepum_um.so: the real-UM runtime -- managed
+    arena, CUPTI launch interposition / fault records, cudaMemPrefetchAsync --
+    with the shared CUDA runtime (the process's other launches go through it)."""
+    deps = [UM_SRC, os.path.join(HERE, "..", "include", "deepum_um.h"),
+            os.path.join(HERE, "..", "include", "deepum_b200.h")]
+    if not force and os.path.exists(UM_OUT) and all(os.path.getmtime(p) <= os.path.getmtime(UM_OUT) for p in deps):
+        return UM_OUT
+    tmp = UM_OUT + ".tmp%d" % os.getpid()
+    cmd = [NVCC, *ARCH, *FLAGS, "-shared", "-cudart", "shared", UM_SRC, "-o", tmp,
+           "-L/usr/local/cuda/lib64", "-lcupti", "-lcuda", "-Xlinker", "-rpath=/usr/local/cuda/lib64"]
+    r = subprocess.run(cmd, capture_output=True, text=True)
+    if r.returncode != 0:
+        raise RuntimeError("nvcc failed for um_runtime.cu:\n%s\n%s" % (r.stdout, r.stderr))
+    os.replace(tmp, UM_OUT)
+    return UM_OUT
+
+
 if __name__ == "__main__":
     print(build(force="--force" in sys.argv, verbose="--verbose" in sys.argv, ptxas_v="-v" in sys.argv,
                 checks="--checks" in sys.argv))
     if "--checks" not in sys.argv:
         print(build_hook(force="--force" in sys.argv))
+        print(build_um(force="--force" in sys.argv))
