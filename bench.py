@@ -56,6 +56,8 @@ def parse():
     ap.add_argument("--degree", type=int, default=32)
     ap.add_argument("--mig-blocks", type=int, default=4096)
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--fast-windows", action="store_true",
+                    help="DUM_CFG_FAST_WINDOWS: conflict-free windows on the fast path (walk index + k_window_fast)")
     ap.add_argument("--timeline", default=None, help="write the last breakdown step's per-kernel timeline (JSON)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-migration", action="store_true")
@@ -266,7 +268,7 @@ def run_ours(args, rank, world, local_rank):
     eng = Engine(num_rows=2048, assoc=2, num_succs=4, degree_n=N, max_blocks=tr.W, max_exec_ids=8192,
                  hbm_frames=tr.C, device=local_rank, corr_capacity=1 << 16,
                  max_batch_faults=max(1 << 20, int(max(tr.faults_in_iteration(i) for i in range(n_iter)) * 1.2)),
-                 max_batch_launches=max(K * 2, 4096))
+                 max_batch_launches=max(K * 2, 4096), flags=B.DUM_CFG_FAST_WINDOWS if args.fast_windows else 0)
     geo = {"A": 2, "S": 4, "R": 2048}
     # ---- device-resident inputs (uploaded before timing) ----
     hs, offs, fs = [], [], []
@@ -535,6 +537,9 @@ def run_ours(args, rank, world, local_rank):
                    % ({"G": "GPT-2-XL", "B": "BERT-large", "T": "tiny"}[args.workload], tr.W, tr.C, K),
                    "records_per_step": records // args.steps, "queries_per_step": K, "degree_n": N,
                    "geometry": "Config9 (2048 rows, 2-way, 4 succ)", "parallelism": "replicas%d" % world,
+                   "windows": ("fast path for conflict-free windows (DUM_CFG_FAST_WINDOWS: walk index + "
+                               "k_window_fast), exact kernel for the rest" if args.fast_windows else
+                               "exact kernel k_predict, a CTA per query (library default)"),
                    "l2": "not flushed in the timed region: each step writes ~200 MB of prefetch/victim lists "
                          "(> 126 MB L2); the breakdown pass flushes (512 MiB write) before every step",
                    "timing": "one CUDA-event region over K back-to-back steps, each = dum_load_residency + "

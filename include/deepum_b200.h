@@ -111,6 +111,14 @@ typedef struct {
  * (the literal PAPER.md L218-L224 loop) instead of the parallel k_walk --
  * a verification mode: both must give identical walk caches. */
 #define DUM_CFG_SEQ_WALKS 0x1u
+/* dum_config.flags: answer the windows whose kernels' walks share no block
+ * on the fast path (walk index at build end, per-walk residency facts, the
+ * persistent copy + staged-selection kernel k_window_fast) and only the rest
+ * on the exact kernel.  Without it (the default) every query takes the exact
+ * kernel k_predict, one CTA per query, and the walk index is not built.  Both
+ * give identical outputs; the default is the faster one on the G workload
+ * (DESIGN.md 7). */
+#define DUM_CFG_FAST_WINDOWS 0x2u
 
 /* Fill *cfg with the defaults (Config9, N = 32). */
 void dum_config_default(dum_config *cfg);

@@ -17,6 +17,7 @@ DUM_NONE = NONE = 0xFFFFFFFF
 DUM_INPUTS_READY = 2
 DUM_HOST_PTRS = 0x1
 DUM_CFG_SEQ_WALKS = 0x1
+DUM_CFG_FAST_WINDOWS = 0x2
 SIM_PREFETCH, SIM_PREEVICT, SIM_INVALIDATE = 0x1, 0x2, 0x4
 SIM_FIELDS = ("faults", "demand_wb", "demand_inv", "pre_wb", "pre_inv", "prefetched")
 DUMP_EXEC, DUMP_CORR, DUMP_BLK, DUMP_WALK, DUMP_RES, DUMP_HIST = 1, 2, 4, 8, 16, 32

@@ -230,6 +230,7 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   dum_engine *e = new (std::nothrow) dum_engine();
   if (!e) return DUM_ENOMEM;
   e->cfg = *cfg;
+  e->fast_windows = (cfg->flags & DUM_CFG_FAST_WINDOWS) != 0;
   e->device = cfg->device;
   e->timing = false;
   for (int i = 0; i < DUM_NTIMERS; ++i) {
@@ -296,7 +297,11 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
     cudaDeviceGetStreamPriorityRange(&lo, &hi);
     A_(cudaStreamCreateWithPriority(&e->side3, cudaStreamNonBlocking, hi));
   }
-  A_(cudaStreamCreateWithFlags(&e->side4, cudaStreamNonBlocking));
+  {  // the build head beside the exact predict kernel: its few CTAs are dispatched first
+    int lo = 0, hi = 0;
+    cudaDeviceGetStreamPriorityRange(&lo, &hi);
+    A_(cudaStreamCreateWithPriority(&e->side4, cudaStreamNonBlocking, hi));
+  }
   A_(cudaEventCreateWithFlags(&e->ev_fork4, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_bhead, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_widx, cudaEventDisableTiming));

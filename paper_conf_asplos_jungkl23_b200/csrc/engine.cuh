@@ -211,6 +211,7 @@ struct dum_engine {
   cudaEvent_t ev_fork4, ev_bhead;
   uint32_t bhead_n;             // dum_step: launches whose build head launch_predict issues after k_chain
   bool bhead_pending;           // the head was issued early: launch_build waits for ev_bhead
+  bool fast_windows;            // DUM_CFG_FAST_WINDOWS
   cudaEvent_t ev_widx;
   // dum_step: exec IDs [last 3 of the previous step | this batch] and the batch's queries
   uint32_t *d_step_exec;

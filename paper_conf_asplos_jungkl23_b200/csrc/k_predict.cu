@@ -188,7 +188,7 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
       // fast-path test (k_window.cu): a walk whose recorded conflicts meet
       // the chain, or whose conflicts were too many to record
       uint32_t wres = 0;  // this step's resident window blocks (k_window marks their log positions)
-      if (len && !anc0) {
+      if (len && !anc0 && a.fast) {
         const uint32_t cn = __ldg(a.conf_n + e);
         if (cn == NONE) {
           conflict = true;
@@ -252,12 +252,9 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
       roff[0] = 0;
       a.qnk[qi] = nk;
     }
-    slow = anchored || __any_sync(0xffffffffu, conflict);
-#ifdef EXP_ALL_EXACT
-    slow = true;
-#endif
+    slow = anchored || __any_sync(0xffffffffu, conflict) || !a.fast;
     const bool s_unrec = __any_sync(0xffffffffu, unrec);
-    if (lane == 0 && slow) ctr_add(a.st, anchored ? DUM_CTR_SLOW_ANCHOR : s_unrec ? DUM_CTR_SLOW_UNRECORDED
+    if (lane == 0 && slow && (a.fast || anchored)) ctr_add(a.st, anchored ? DUM_CTR_SLOW_ANCHOR : s_unrec ? DUM_CTR_SLOW_UNRECORDED
                                                                            : DUM_CTR_SLOW_CONFLICT, 1);
     nonres = __reduce_add_sync(0xffffffffu, nonres);
     if (a.select && !slow) {
@@ -984,6 +981,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   a.qneed = e->d_qneed;
   a.qvb = e->d_qvb;
   a.selrec = e->d_selrec;
+  a.fast = e->fast_windows ? 1u : 0u;
   a.lrm_cap = e->lrm_cap;
   {
     // the chunk map holds every copy chunk of the call: <= cap / 128 + nq (N + 1)
@@ -1036,7 +1034,8 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   cudaEventRecord(e->ev_fork2, s);
   cudaStreamWaitEvent(e->side2, e->ev_fork2, 0);
   const size_t smem = (size_t)((a.nwords + 3) & ~3u) * 4 + 2 * DHCAP * 4;
-  const uint32_t pgrid = std::min<uint32_t>(nq, 148);  // persistent over the exact-path classes; few queries
+  // fast windows: persistent over the few exact-path queries; else a CTA per query
+  const uint32_t pgrid = e->fast_windows ? std::min<uint32_t>(nq, 148) : nq;
   if (sel) {
     // the attribute is per device and function: raised by every engine on its own device
     if ((int)smem > e->select_smem) {
@@ -1053,7 +1052,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
     TimerScope t(e, DUM_T_EXACT, s);
     k_predict<false><<<pgrid, PRED_NT, smem, s>>>(a);
   }
-  if ((err = launch_window(e, a, sel != nullptr, e->side2)) != cudaSuccess) return err;
+  if (e->fast_windows && (err = launch_window(e, a, sel != nullptr, e->side2)) != cudaSuccess) return err;
   cudaEventRecord(e->ev_join2, e->side2);
   cudaStreamWaitEvent(s, e->ev_join2, 0);
   e->kernel_launches += 2;

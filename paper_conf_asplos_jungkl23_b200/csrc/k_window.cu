@@ -907,9 +907,7 @@ static uint32_t index_grid(const dum_engine *e) {
 
 // Build end: the walk index of the walks just rebuilt (k_walk / k_walk_slow).
 cudaError_t launch_walk_index(dum_engine *e, cudaStream_t main) {
-#ifdef EXP_ALL_EXACT
-  return cudaSuccess;
-#endif
+  if (!e->fast_windows) return cudaSuccess;  // every window takes the exact kernel: no conflicts needed
   // on the third side stream: the next predict's prelude (residency load, ingest,
   // queries, walk residency facts) overlaps it; k_chain waits for ev_widx
   cudaEventRecord(e->ev_fork2, main);
@@ -942,9 +940,7 @@ __global__ void __launch_bounds__(256) k_log_bits(const uint32_t *__restrict__ l
 
 // Predict time: per-walk residency facts for the fast selection.
 cudaError_t launch_walk_res(dum_engine *e, cudaStream_t s) {
-#ifdef EXP_ALL_EXACT
-  return cudaSuccess;
-#endif
+  if (!e->fast_windows) return cudaSuccess;
   TimerScope t(e, DUM_T_WALK_RES, s);
   k_walk_res<<<index_grid(e), IX_NT, 0, s>>>(e->d_walk, e->d_walk_len, e->g.walk_cap, e->d_state, e->d_res_bits,
                                              e->d_logpos, e->d_wnr, e->d_wnres, e->d_respos);

@@ -22,6 +22,7 @@ struct PredArgs {
   uint32_t nq;
   uint32_t select;       // a8 fused (dum_predict_select)
   uint32_t chain_bitset; // k_chain tests conflicts against a shared bitset of the chain
+  uint32_t fast;         // DUM_CFG_FAST_WINDOWS: conflict-free windows take k_window_fast
   const CorrSlot *corr;
   uint32_t corr_cap;
   const uint32_t *jump;  // [levels][corr_cap]

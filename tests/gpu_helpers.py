@@ -19,7 +19,13 @@ ALL_TABLES = orc.EXEC | orc.CORR | orc.BLK | orc.WALK | orc.HIST
 LIVE_ENGINES: list = []
 
 
-def make_pair(R=2048, A=2, S=4, N=32, W=256, C=128, row_index=0, Emax=1024, **kw):
+def make_pair(R=2048, A=2, S=4, N=32, W=256, C=128, row_index=0, Emax=1024, fast=True, **kw):
+    """An engine and the oracle on the same geometry.  fast: the engine answers
+    conflict-free windows on the fast path (DUM_CFG_FAST_WINDOWS) -- the suite's
+    default, so that both predict paths are covered; False: every window on the
+    exact kernel (the library default, what bench.py times)."""
+    if fast:
+        kw["flags"] = kw.get("flags", 0) | B.DUM_CFG_FAST_WINDOWS
     eng = Engine(num_rows=R, assoc=A, num_succs=S, degree_n=N, max_blocks=W, max_exec_ids=Emax, hbm_frames=C,
                  row_index=row_index, **kw)
     LIVE_ENGINES.append(eng)

@@ -32,12 +32,13 @@ from paper_conf_asplos_jungkl23_b200 import Engine, binding as B  # noqa: E402
 N = 32
 
 
-def bench_engine(tr, n_iter):
-    """The engine configuration bench.py times (Config9, N = 32)."""
+def bench_engine(tr, n_iter, fast=False):
+    """The engine configuration bench.py times (Config9, N = 32; exact windows
+    unless fast)."""
     mf = max(1 << 20, int(max(tr.faults_in_iteration(i) for i in range(n_iter)) * 1.2))
     return Engine(num_rows=2048, assoc=2, num_succs=4, degree_n=N, max_blocks=tr.W, max_exec_ids=8192,
                   hbm_frames=tr.C, corr_capacity=1 << 16, max_batch_faults=mf,
-                  max_batch_launches=max(tr.K * 2, 4096))
+                  max_batch_launches=max(tr.K * 2, 4096), flags=B.DUM_CFG_FAST_WINDOWS if fast else 0)
 
 
 def anchored_sample(tr, i, ex_all, rng, frac=0.01):
@@ -82,11 +83,12 @@ def compare_predict_select(out, ref, nq, msg):
     assert np.array_equal(ioff, io.astype(np.int64)) and np.array_equal(gi, inv_o), "%s: invalidate lists" % msg
 
 
+@pytest.mark.parametrize("windows", ["exact", "fast"])
 @pytest.mark.parametrize("config", ["B", "G"])
-def test_ten_iterations_every_query_matches_oracle(config):
+def test_ten_iterations_every_query_matches_oracle(config, windows):
     n_iter = 10
     tr = wl.make(config, n_iter=n_iter)
-    eng = bench_engine(tr, n_iter)
+    eng = bench_engine(tr, n_iter, fast=windows == "fast")
     LIVE_ENGINES.append(eng)
     o = orc.Oracle(R=2048, A=2, S=4, N=N, W=tr.W, C=tr.C, threads=os.cpu_count() or 1)
     o.mark_inactive(tr.inactive_blocks, True)
@@ -146,6 +148,9 @@ def test_ten_iterations_every_query_matches_oracle(config):
     assert c["Q_DUP"] + c["Q_FALLBACK"] > 0, c          # windows whose kernels share blocks
     assert c["Q_FAST"] + c["Q_NODUP"] > 0, c
     assert c["WALK_PREFIX"] > 0, c
-    assert c["Q_FAST"] > 0 and c["Q_SLOW"] > 0, c     # both predict kernels answered queries
+    if windows == "fast":
+        assert c["Q_FAST"] > 0 and c["Q_SLOW"] > 0, c  # both predict kernels answered queries
+    else:
+        assert c["Q_FAST"] == 0 and c["Q_SLOW"] > 0, c  # every query on the exact kernel
     if config == "B":  # B's windows reach the min-position fallback and the walk dedupe
         assert c["Q_FALLBACK"] > 0 and c["WALK_DEDUPE"] > 0, c
