@@ -638,6 +638,8 @@ def run_e2e(args, tr, eng, dev, stream, cap, sel_cap):
     outs = {}
     eng.reset()
     eng.mark_inactive(torch.from_numpy(tr.inactive_blocks.view(np.int32)).to(dev), True)
+    # the timed steps' mode (the breakdown pass before this turned the step graphs off)
+    eng.set_step_graphs(not args.separate_calls and not args.no_graph)
 
     def host_step(i, s=None):
         n = hs[i].numel()

@@ -9,7 +9,7 @@
 set -u
 TAG=${1:-r02}
 shift
-KERNELS=${*:-"k_window k_apply k_walk k_chain k_ingest"}
+KERNELS=${*:-"k_predict k_build_exec k_chain k_ingest k_build_prep"}
 B="python bench.py --steps 2 --warmup 3 --no-e2e --no-migration --no-cpu-baseline"
 timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv \
     --log-file gpurun_out/${TAG}_launches.csv $B > gpurun_out/${TAG}_launches.log 2>&1
