@@ -632,7 +632,9 @@ def run_e2e(args, tr, eng, dev, stream, cap, sel_cap):
     snap_dev = [torch.empty(tr.C, dtype=torch.int32, device=dev) for _ in range(2)]
     out_r = [torch.empty((K, 2), dtype=torch.int64).pin_memory() for _ in range(args.steps)]
     out_s = [torch.empty((K, 4), dtype=torch.int64).pin_memory() for _ in range(args.steps)]
-    cs = torch.cuda.Stream(device=dev)  # host<->device copies of the bench's own I/O
+    cs = torch.cuda.Stream(device=dev)  # uploads of the residency snapshots
+    ds = torch.cuda.Stream(device=dev)  # read-backs of the results (a stream of their own: the next
+    #                                      snapshot upload must not queue behind this step's read-back)
     snap_used = [None, None]
     d2h_done = [None]
     outs = {}
@@ -660,12 +662,12 @@ def run_e2e(args, tr, eng, dev, stream, cap, sel_cap):
         if s is not None:
             ev = torch.cuda.Event()
             ev.record(stream)
-            with torch.cuda.stream(cs):
-                cs.wait_event(ev)
+            with torch.cuda.stream(ds):
+                ds.wait_event(ev)
                 out_r[s].copy_(outs["rng"], non_blocking=True)
                 out_s[s].copy_(outs["sel_rng"], non_blocking=True)
                 d2h_done[0] = torch.cuda.Event()
-                d2h_done[0].record(cs)
+                d2h_done[0].record(ds)
 
     for i in range(0, 1 + args.warmup):
         host_step(i)

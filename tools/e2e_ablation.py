@@ -43,7 +43,7 @@ for i in range(n_iter):
     ds.append(hs[-1].to(dev))
 cap = 24 << 20
 res = {}
-for mode in ["full", "dev_inputs", "no_snap_upload", "no_d2h", "plain"]:
+for mode in ["full", "one_copy_stream", "dev_inputs", "no_snap_upload", "no_d2h", "plain"]:
     host_in = mode not in ("dev_inputs", "plain")
     snap_up = mode not in ("no_snap_upload", "plain")
     d2h = mode not in ("no_d2h", "plain")
@@ -55,6 +55,7 @@ for mode in ["full", "dev_inputs", "no_snap_upload", "no_d2h", "plain"]:
     out_r = [torch.empty((K, 2), dtype=torch.int64).pin_memory() for _ in range(args.steps)]
     out_s = [torch.empty((K, 4), dtype=torch.int64).pin_memory() for _ in range(args.steps)]
     cs = torch.cuda.Stream(device=dev)
+    dstr = torch.cuda.Stream(device=dev) if mode != "one_copy_stream" else cs
     snap_used = [None, None]
     d2h_done = [None]
 
@@ -83,12 +84,12 @@ for mode in ["full", "dev_inputs", "no_snap_upload", "no_d2h", "plain"]:
         if d2h and s is not None:
             ev = torch.cuda.Event()
             ev.record(stream)
-            with torch.cuda.stream(cs):
-                cs.wait_event(ev)
+            with torch.cuda.stream(dstr):
+                dstr.wait_event(ev)
                 out_r[s].copy_(outs["rng"], non_blocking=True)
                 out_s[s].copy_(outs["sel_rng"], non_blocking=True)
                 d2h_done[0] = torch.cuda.Event()
-                d2h_done[0].record(cs)
+                d2h_done[0].record(dstr)
 
     for i in range(0, 1 + args.warmup):
         host_step(i)
