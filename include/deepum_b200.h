@@ -432,6 +432,7 @@ enum {
   DUM_T_WALK_INDEX,   /* walk index: holders per block, conflicts per walk (build end) */
   DUM_T_WALK_RES,     /* residency facts per walk (predict) */
   DUM_T_SELECT_FAST,  /* fast path with selection: k_window_fast (pairs + selection, one persistent kernel) */
+  DUM_T_COMMIT,       /* k_walk_commit: the rebuilt walks published after predict (dum_build_tables) */
   DUM_NTIMERS = 24
 };
 int dum_set_timing(dum_engine *eng, int enable);

@@ -32,13 +32,13 @@ CTR = {n: i for i, n in enumerate(["RAW_RECORDS", "NORM_RECORDS", "LAUNCHES", "C
                                    "SLOW_ANCHOR", "FAST_DIRTY"])}
 TIMER = {n: i for i, n in enumerate(["INGEST", "EXEC_ASSIGN", "BUILD_PREP", "APPLY_WALK", "WALK_SLOW",
                                      "MAKE_QUERIES", "ANCHOR_WALK", "PREDICT", "SELECT", "MIG_PLAN", "COPY",
-                                     "RESIDENCY", "CHAIN", "JUMP", "WALK", "EXACT", "WALK_INDEX", "WALK_RES", "SELECT_FAST"])}
+                                     "RESIDENCY", "CHAIN", "JUMP", "WALK", "EXACT", "WALK_INDEX", "WALK_RES", "SELECT_FAST", "COMMIT"])}
 KERNEL_OF_TIMER = {"INGEST": "k_ingest", "EXEC_ASSIGN": "k_exec_assign", "BUILD_PREP": "k_build_prep",
                    "APPLY_WALK": "k_build_exec", "WALK": "k_walk", "WALK_SLOW": "k_walk_slow", "MAKE_QUERIES": "k_make_queries",
                    "ANCHOR_WALK": "k_anchor_walk", "PREDICT": "k_copy_fast", "SELECT": "k_select", "SELECT_FAST": "k_window_fast",
                    "MIG_PLAN": "k_mig_plan", "COPY": "k_copy_blocks", "RESIDENCY": "k_load_res",
                    "CHAIN": "k_chain", "JUMP": "k_jump0", "EXACT": "k_predict", "WALK_INDEX": "k_walk_index",
-                   "WALK_RES": "k_walk_res"}
+                   "WALK_RES": "k_walk_res", "COMMIT": "k_walk_commit"}
 # timers of kernels launched on the engine's side streams (overlapping others)
 SIDE_TIMERS = {"JUMP": "side stream, overlaps k_apply / k_walk (k_jump0 + k_jumpk levels)",
                "SELECT_FAST": "second side stream, beside the exact path (k_window_fast: pairs + selection of the fast windows)",

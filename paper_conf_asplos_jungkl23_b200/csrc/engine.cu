@@ -39,6 +39,7 @@ __global__ void k_init_state(DevState *st) {
   st->err = 0;
   st->needed = 0;
   st->pool_pairs = st->pool_wb = st->pool_inv = st->pool_anchor = st->pool_big = st->pool_chunks = 0;
+  st->pool_bigb = 0;
   st->sel_queue = 0;
   st->copy_queue = 0;
   st->chain_done = 0;
@@ -133,10 +134,11 @@ int reset_state(dum_engine *e, cudaStream_t s) {
 
 void free_all(dum_engine *e) {
   void *ptrs[] = {e->d_exec_keys, e->d_exec_vals, e->d_exec_minpos, e->d_exec_hash, e->d_corr, e->d_tbl,
-                  e->d_start_end, e->d_walk, e->d_walk_len, e->d_in_hash, e->d_in_off, e->d_in_faults,
+                  e->d_start_end, e->d_walk, e->d_walk_len, e->d_walk_n, e->d_walk_len_n, e->d_wrun_n,
+                  e->d_wrun_len_n, e->d_in_hash, e->d_in_off, e->d_in_faults,
                   e->stage_base[0], e->stage_base[1], e->stage_base[2], e->stage_base[3], e->stage_base[4],
                   e->stage_base[5], e->d_head, e->d_next, e->d_order, e->d_slow_list,
-                  e->d_e_ops, e->d_e_last, e->d_pend, e->d_plan_agg, e->d_lead, e->d_items, e->d_rowc, e->d_big_pool, e->d_ingest_pool, e->d_walk_seen,
+                  e->d_e_ops, e->d_e_last, e->d_pend, e->d_plan_agg, e->d_lead, e->d_items, e->d_rowc, e->d_big_pool, e->d_big_pool_b, e->d_ingest_pool, e->d_walk_seen,
                   e->d_walk_chain, e->d_walk_tmp, e->d_walk_out, e->d_anchor_pool, e->d_anchor_range,
                   e->d_frame_of, e->d_stamp_of, e->d_block_of, e->d_free_bits, e->d_inactive_bits, e->d_res_bits, e->d_logpos, e->d_lrm_blk,
                   e->d_lrm_stamp, e->d_mig_frames, e->d_mig_src, e->d_mig_blocks, e->d_state, e->d_qkern,
@@ -315,6 +317,10 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_walk_len, g.Emax));
   A_(dmalloc(&e->d_wrun, 2ull * g.Emax * g.walk_cap));
   A_(dmalloc(&e->d_wrun_len, g.Emax));
+  A_(dmalloc(&e->d_walk_n, (uint64_t)g.Emax * g.walk_cap));
+  A_(dmalloc(&e->d_walk_len_n, g.Emax));
+  A_(dmalloc(&e->d_wrun_n, 2ull * g.Emax * g.walk_cap));
+  A_(dmalloc(&e->d_wrun_len_n, g.Emax));
   // host-pointer inputs are uploaded here on the ingest stream (in order with
   // the ingest that reads them), one buffer per staging set: the upload of
   // batch i+1 overlaps the work on batch i
@@ -355,6 +361,7 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(dmalloc(&e->d_items, 2 * e->items_cap));
   A_(dmalloc(&e->d_rowc, e->stage_fault_cap * (1ull + g.S)));
   A_(dmalloc(&e->d_big_pool, 2 * e->big_pool_entries));
+  A_(dmalloc(&e->d_big_pool_b, 2 * e->big_pool_entries));
   A_(dmalloc(&e->d_ingest_pool, 2 * e->big_pool_entries));
   A_(dmalloc(&e->d_walk_seen, (uint64_t)e->n_walk_slots * e->walk_hash_cap));
   A_(dmalloc(&e->d_walk_chain, (uint64_t)e->n_walk_slots * e->walk_hash_cap));

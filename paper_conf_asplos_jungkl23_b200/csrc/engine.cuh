@@ -52,7 +52,8 @@ struct DevState {
   unsigned long long pool_pairs;   // predict output bump pointer
   unsigned long long pool_wb, pool_inv;
   unsigned long long pool_anchor;  // anchored-walk scratch bump pointer
-  unsigned long long pool_big;     // build-walk global hash scratch bump pointer
+  unsigned long long pool_big;     // exact-predict global hash scratch bump pointer (d_big_pool)
+  unsigned long long pool_bigb;    // build-walk global hash scratch bump pointer (d_big_pool_b)
   unsigned long long pool_chunks;  // predict: k_copy_fast chunk-map bump pointer
   uint32_t sel_queue;         // predict: k_window_fast selection-item queue head
   unsigned long long copy_queue;  // predict: k_window_fast copy-chunk queue head
@@ -177,7 +178,12 @@ struct dum_engine {
   uint32_t *d_items;             // apply items, u32 pairs (leader index, partition | P << 16)
   uint64_t items_cap;
   uint32_t *d_rowc;              // walk row cache for long walks: (1 + S) u32 per staged record
-  uint32_t *d_big_pool;   // u32 pairs for large-walk hash tables
+  uint32_t *d_big_pool;   // u32 pairs for large-window hash tables (exact predict)
+  uint32_t *d_big_pool_b; // the same for the build's large walks (the build may run beside predict)
+  // the build writes the walks of the exec IDs it rebuilds here, beside the
+  // predict kernels that read the live walk cache; k_walk_commit copies them
+  // into the live arrays once predict is done (D12)
+  uint32_t *d_walk_n, *d_walk_len_n, *d_wrun_n, *d_wrun_len_n;
   uint32_t *d_ingest_pool;  // the ingest's own global hash region (it may run concurrently with a build)
   uint64_t big_pool_entries;
   // walk scratch for the sequential walker (per CTA slot)

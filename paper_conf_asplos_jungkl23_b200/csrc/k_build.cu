@@ -60,10 +60,10 @@ __global__ void k_build_prep(uint32_t n_staged, const uint32_t *__restrict__ sta
                              const uint32_t *__restrict__ stage_cnt, CorrSlot *corr, uint32_t corr_cap,
                              uint32_t *rec_slot, uint32_t *head, uint32_t *__restrict__ next,
                              uint32_t *__restrict__ order, uint32_t *e_ops, uint32_t *e_last,
-                             unsigned long long *plan_agg, DevState *st, uint32_t reset_pool) {
+                             unsigned long long *plan_agg, DevState *st) {
   const uint32_t j = blockIdx.x * blockDim.x + threadIdx.x;
   if (j == 0) {
-    if (reset_pool) st->pool_big = 0;
+    st->pool_bigb = 0;  // the build's own scratch (the exact predict kernel may run beside it)
     st->n_slow = 0;
     st->n_dd = 0;
     st->n_items = 0;  // k_plan's last chunk writes the list sizes
@@ -878,7 +878,7 @@ __global__ void __launch_bounds__(WK_NT) k_walk(BuildArgs a) {
     uint32_t *cq = scq;
     if (n > WK_CQ) {
       if (tid == 0) {
-        const unsigned long long o = atomicAdd(&a.st->pool_big, (unsigned long long)n);
+        const unsigned long long o = atomicAdd(&a.st->pool_bigb, (unsigned long long)n);
         s_flag = o + n <= a.big_entries * 2 ? 0u : 1u;
         s_off = (uint32_t)o;
       }
@@ -997,7 +997,7 @@ __global__ void __launch_bounds__(WK_NT) k_walk(BuildArgs a) {
     uint32_t *qk = sqk;
     if (qcap > WK_QCAP) {
       if (tid == 0) {
-        const unsigned long long o = atomicAdd(&a.st->pool_big, 2ull * qcap);
+        const unsigned long long o = atomicAdd(&a.st->pool_bigb, 2ull * qcap);
         s_flag = o + 2ull * qcap <= a.big_entries * 2 ? 0u : 1u;
         s_off = (uint32_t)o;
       }
@@ -1161,14 +1161,14 @@ static BuildArgs build_args(dum_engine *e, uint32_t n) {
   ba.items = reinterpret_cast<uint2 *>(e->d_items);
   ba.tbl = e->d_tbl;
   ba.start_end = e->d_start_end;
-  ba.walk = e->d_walk;
-  ba.walk_len = e->d_walk_len;
+  ba.walk = e->d_walk_n;  // staged: k_walk_commit publishes them (the build may run beside predict)
+  ba.walk_len = e->d_walk_len_n;
   ba.rowc = e->d_rowc;
-  ba.big_pool = e->d_big_pool;
+  ba.big_pool = e->d_big_pool_b;
   ba.big_entries = e->big_pool_entries;
   ba.slow_list = e->d_slow_list;
-  ba.wrun = e->d_wrun;
-  ba.wrun_len = e->d_wrun_len;
+  ba.wrun = e->d_wrun_n;
+  ba.wrun_len = e->d_wrun_len_n;
   ba.order = e->d_order;
   ba.plan_agg = reinterpret_cast<unsigned long long *>(e->d_plan_agg);
   ba.st = e->d_state;
@@ -1177,62 +1177,56 @@ static BuildArgs build_args(dum_engine *e, uint32_t n) {
   return ba;
 }
 
-// The build's head: correlation upserts + work lists (k_build_prep, k_plan) on
-// `s`, the jump tables forked to the side stream.  reset_pool: k_build_prep
-// clears the walk-scratch bump pointer (pool_big) -- not when it runs beside
-// the predict kernels, whose exact path allocates from it (k_pred_epilogue
-// clears it before the build's tail then).
-static cudaError_t build_head(dum_engine *e, const BuildArgs &ba, cudaStream_t s, uint32_t reset_pool) {
+// The published walks of the exec IDs a build rebuilt: the build writes them
+// to the staging arrays (d_*_n) -- possibly while the predict kernels of the
+// same step still read the live walk cache -- and this copies them over once
+// predict is done.  A CTA per rebuilt exec ID (the build's leads).
+__global__ void __launch_bounds__(256) k_walk_commit(const LeadDesc *__restrict__ desc, const DevState *st,
+                                                     uint32_t walk_cap, const uint32_t *__restrict__ walk_n,
+                                                     const uint32_t *__restrict__ len_n,
+                                                     const uint2 *__restrict__ wrun_n,
+                                                     const uint32_t *__restrict__ rlen_n, uint32_t *walk,
+                                                     uint32_t *len, uint2 *wrun, uint32_t *rlen) {
+  const uint32_t n_leads = *(volatile const uint32_t *)&st->n_leads;
+  for (uint32_t li = blockIdx.x; li < n_leads; li += gridDim.x) {
+    const uint32_t e = desc[li].e;
+    const uint32_t L = len_n[e], RL = rlen_n[e];
+    const uint64_t r0 = (uint64_t)e * walk_cap;  // rows are 32 B aligned (walk_cap % 8 == 0)
+    const uint4 *ws = reinterpret_cast<const uint4 *>(walk_n + r0);
+    uint4 *wd = reinterpret_cast<uint4 *>(walk + r0);
+    for (uint32_t i = threadIdx.x; i < (L + 3) / 4; i += blockDim.x) wd[i] = __ldcs(ws + i);
+    const uint4 *rs = reinterpret_cast<const uint4 *>(wrun_n + r0);
+    uint4 *rd = reinterpret_cast<uint4 *>(wrun + r0);
+    for (uint32_t i = threadIdx.x; i < (RL + 1) / 2; i += blockDim.x) rd[i] = __ldcs(rs + i);
+    if (threadIdx.x == 0) {
+      len[e] = L;
+      rlen[e] = RL;
+    }
+  }
+}
+
+// The build of the n staged launches into the staging walk arrays: the head
+// (correlation upserts + work lists, k_build_prep / k_plan; the jump tables
+// forked to the side stream), the table apply + walks (k_build_exec, k_walk)
+// and the sequential walks (k_walk_slow), all on `s`.  Everything it writes
+// is read by the next predict only through k_chain (corr / jump, already
+// read) or after k_walk_commit (walks), so it may run beside this step's
+// predict kernels (D12 holds: predict reads the walks of the last build).
+static cudaError_t build_body(dum_engine *e, const BuildArgs &ba, cudaStream_t s) {
   const uint32_t n = ba.n_staged;
   {
     TimerScope t(e, DUM_T_BUILD_PREP, s);
     k_build_prep<<<(n + 255) / 256, 256, 0, s>>>(n, e->d_stage_exec, e->d_stage_cnt,
                                                   e->d_corr, e->corr_cap, e->d_rec_slot, e->d_head, e->d_next,
-                                                  e->d_order, e->d_e_ops, e->d_e_last, ba.plan_agg, e->d_state,
-                                                  reset_pool);
+                                                  e->d_order, e->d_e_ops, e->d_e_last, ba.plan_agg, e->d_state);
     k_plan<<<(n + PLAN_NT - 1) / PLAN_NT, PLAN_NT, 0, s>>>(ba);
   }
   // the jump tables depend only on the correlation table, final here
   cudaEventRecord(e->ev_fork, s);
   cudaStreamWaitEvent(e->side, e->ev_fork, 0);
-  const cudaError_t je = launch_jump_tables(e, e->side);
+  cudaError_t err = launch_jump_tables(e, e->side);
   cudaEventRecord(e->ev_join, e->side);
-  return je;
-}
-
-// dum_step: the head of the build of the n staged launches, issued by
-// launch_predict right after k_chain (the last reader of the correlation and
-// jump tables) on a side stream beside the exact / fast predict kernels; the
-// build's tail (launch_build) waits for it.
-cudaError_t launch_build_head(dum_engine *e, uint32_t n, cudaStream_t s) {
-  if (n == 0) return cudaSuccess;
-  cudaEventRecord(e->ev_fork4, s);
-  cudaStreamWaitEvent(e->side4, e->ev_fork4, 0);
-  const BuildArgs ba = build_args(e, n);
-  const cudaError_t err = build_head(e, ba, e->side4, 0u);
-  cudaEventRecord(e->ev_bhead, e->side4);
-  e->bhead_pending = true;
-  e->kernel_launches += 2;
-  return err;
-}
-
-cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
-  const uint32_t n = e->n_staged;
-  if (n == 0) return cudaSuccess;
-  if (!e->capturing) {  // (a captured step joins its side streams before it ends)
-    cudaStreamWaitEvent(s, e->ev_join, 0);  // the previous build's jump tables read corr
-    cudaStreamWaitEvent(s, e->ev_widx, 0);  // the previous build's walk index reads the walk cache
-  }
-  const BuildArgs ba = build_args(e, n);
-  const bool was_early = e->bhead_pending;
-  if (e->bhead_pending) {  // the head ran beside the predict kernels (launch_build_head)
-    cudaStreamWaitEvent(s, e->ev_bhead, 0);
-    e->bhead_pending = false;
-  } else {
-    const cudaError_t he = build_head(e, ba, s, 1u);
-    if (he != cudaSuccess) return he;
-  }
-  cudaError_t err;
+  if (err != cudaSuccess) return err;
   if (e->g.A <= 2 && e->g.S <= 4) err = launch_apply_walk<2, 4>(e, ba, s);
   else if (e->g.A == 2 && e->g.S == 8) err = launch_apply_walk<2, 8>(e, ba, s);
   else if (e->g.A == 4 && e->g.S == 4) err = launch_apply_walk<4, 4>(e, ba, s);
@@ -1243,8 +1237,49 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
                  e->g.walk_cap + e->g.R * e->g.A + 4};
   {
     TimerScope t(e, DUM_T_WALK_SLOW, s);
-    k_walk_slow<<<e->n_walk_slots, 32, 0, s>>>(e->g, e->d_tbl, e->d_start_end, e->d_walk, e->d_walk_len,
-                                               e->d_wrun, e->d_wrun_len, e->d_slow_list, ws, e->d_state);
+    k_walk_slow<<<e->n_walk_slots, 32, 0, s>>>(e->g, e->d_tbl, e->d_start_end, ba.walk, ba.walk_len, ba.wrun,
+                                               ba.wrun_len, e->d_slow_list, ws, e->d_state);
+  }
+  e->kernel_launches += 4;
+  return cudaGetLastError();
+}
+
+// dum_step: the build of the n staged launches, issued by launch_predict right
+// after k_chain (the last reader of the correlation and jump tables) on a
+// high-priority side stream beside the predict kernels; launch_build (after
+// predict) waits for it and publishes the walks.
+cudaError_t launch_build_head(dum_engine *e, uint32_t n, cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  cudaEventRecord(e->ev_fork4, s);
+  cudaStreamWaitEvent(e->side4, e->ev_fork4, 0);
+  const BuildArgs ba = build_args(e, n);
+  const cudaError_t err = build_body(e, ba, e->side4);
+  cudaEventRecord(e->ev_bhead, e->side4);
+  e->bhead_pending = true;
+  return err;
+}
+
+cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
+  const uint32_t n = e->n_staged;
+  if (n == 0) return cudaSuccess;
+  if (!e->capturing) {  // (a captured step joins its side streams before it ends)
+    cudaStreamWaitEvent(s, e->ev_join, 0);  // the previous build's jump tables read corr
+    cudaStreamWaitEvent(s, e->ev_widx, 0);  // the previous build's walk index reads the walk cache
+  }
+  if (e->bhead_pending) {  // built beside the predict kernels (launch_build_head)
+    cudaStreamWaitEvent(s, e->ev_bhead, 0);
+    e->bhead_pending = false;
+  } else {
+    const BuildArgs ba = build_args(e, n);
+    const cudaError_t be = build_body(e, ba, s);
+    if (be != cudaSuccess) return be;
+  }
+  {  // publish the rebuilt walks (predict, the only other reader, is ordered before)
+    TimerScope t(e, DUM_T_COMMIT, s);
+    k_walk_commit<<<std::max<uint32_t>(1, std::min<uint32_t>(e->g.Emax, 148 * 8)), 256, 0, s>>>(
+        reinterpret_cast<const LeadDesc *>(e->d_lead), e->d_state, e->g.walk_cap, e->d_walk_n, e->d_walk_len_n,
+        reinterpret_cast<const uint2 *>(e->d_wrun_n), e->d_wrun_len_n, e->d_walk, e->d_walk_len,
+        reinterpret_cast<uint2 *>(e->d_wrun), e->d_wrun_len);
   }
   if (e->capturing) {
     // a captured step builds the walk index at the start of the next step,
@@ -1257,8 +1292,7 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   // no join here: the jump tables keep building on the side stream, past the
   // end of this call; the next reader of the correlation table (predict's
   // k_chain, the next build, reset) waits for ev_join
-  if (!was_early) e->kernel_launches += 2;  // the head
-  e->kernel_launches += 3;
+  e->kernel_launches += 1;
   return cudaGetLastError();
 }
 
