@@ -65,14 +65,19 @@ def parse():
     ap.add_argument("--json-out", default="")
     ap.add_argument("--separate-calls", action="store_true",
                     help="record / make_queries / predict_select / build as separate C-ABI calls instead of dum_step")
-    ap.add_argument("--no-graph", action="store_true", help="dum_step without its CUDA graph")
+    ap.add_argument("--graph", action="store_true",
+                    help="replay each dum_step as a CUDA graph (dum_set_step_graphs); default: one uncaptured "
+                         "dum_step call per step, whose next ingest overlaps the previous step's tail (faster on G)")
+    ap.add_argument("--no-graph", action="store_true", help=argparse.SUPPRESS)  # (the default; kept for old scripts)
     ap.add_argument("--debug", action="store_true", help="synchronize and check after every call")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="process group of the N>1 replicas (barrier + reductions only); gloo lets several ranks "
                          "share one GPU (tests)")
     ap.add_argument("--verify", action="store_true",
                     help="check the last timed step's prefetch / victim lists against the oracle")
-    return ap.parse_args()
+    args = ap.parse_args()
+    args.no_graph = not args.graph
+    return args
 
 
 # ---------------------------------------------------------------------------

@@ -97,6 +97,8 @@ cudaError_t fill(uint32_t *p, uint64_t n, uint32_t v, cudaStream_t s) {
 
 int reset_state(dum_engine *e, cudaStream_t s) {
   const Geo &g = e->g;
+  e->commit_stale = false;  // (the walks are cleared below)
+  e->jump_stale = false;
   if (e->ev_join) CK(cudaStreamWaitEvent(s, e->ev_join, 0));  // jump tables still building on the side stream
   if (e->ev_join2) CK(cudaStreamWaitEvent(s, e->ev_join2, 0));  // exact-path predict kernel
   if (e->ev_widx) CK(cudaStreamWaitEvent(s, e->ev_widx, 0));    // walk index
@@ -653,23 +655,42 @@ static int step_graph(dum_engine *e, const uint64_t *launch_hash, const uint64_t
     const uint64_t sf0 = e->staged_faults;
     e->n_staged = 0;
     e->staged_faults = 0;
+    // an error left by an earlier uncaptured launch is not this capture's
+    const cudaError_t pending = cudaGetLastError();
+    if (pending != cudaSuccess) {
+      e->last_error = std::string("pending before a dum_step capture: ") + cudaGetErrorString(pending);
+      return DUM_ECUDA;
+    }
+    const char *stage = "begin capture";
     cudaError_t err = cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal);
     // the previous step's walk index (a replayed build leaves it to this step),
     // beside the residency facts and the ingest
-    if (err == cudaSuccess) err = launch_walk_index(e, s);
-    if (err == cudaSuccess) err = fork_walk_res(e, s);
-    if (err == cudaSuccess)
+    if (err == cudaSuccess && (stage = "jump tables", true)) {
+      // the previous build's jump tables (a captured build leaves them to the
+      // next step), on the side stream beside the ingest; k_chain joins them
+      cudaEventRecord(e->ev_fork, s);
+      cudaStreamWaitEvent(e->side, e->ev_fork, 0);
+      err = launch_jump_tables(e, e->side);
+      // ... and its walks (exact windows: k_chain is their first reader; a
+      // fast-window build published them itself, for the walk index)
+      if (err == cudaSuccess && !e->fast_windows) err = launch_walk_commit(e, e->side);
+      cudaEventRecord(e->ev_join, e->side);
+    }
+    if (err == cudaSuccess && (stage = "walk index", true)) err = launch_walk_index(e, s);
+    if (err == cudaSuccess && (stage = "walk residency", true)) err = fork_walk_res(e, s);
+    if (err == cudaSuccess && (stage = "record", true))
       err = launch_record(e, in_hash(e), in_off(e), n_launch, in_faults(e), e->stage_fault_cap,
                           e->d_step_exec + 3, s);
-    if (err == cudaSuccess) err = launch_make_queries(e, e->d_step_exec, 3 + n_launch, 3, degree, e->d_step_q, s);
-    e->bhead_n = n_launch;  // the build's head goes beside the predict kernels
-    if (err == cudaSuccess)
+    if (err == cudaSuccess && (stage = "queries", true))
+      err = launch_make_queries(e, e->d_step_exec, 3 + n_launch, 3, degree, e->d_step_q, s);
+    e->bhead_n = n_launch;  // the build goes beside the predict kernels
+    if (err == cudaSuccess && (stage = "predict + build", true))
       err = launch_predict(e, e->d_step_q, n_launch, out_pairs, out_cap_pairs, out_range, out_kern_off, out_chain,
                            out_needed, &so, sel_needed, s);
     e->bhead_n = 0;
     e->n_staged = n_launch;
     e->staged_faults = e->stage_fault_cap;
-    if (err == cudaSuccess) err = launch_build(e, s);
+    if (err == cudaSuccess && (stage = "build commit", true)) err = launch_build(e, s);
     if (err == cudaSuccess) {
       k_step_shift<<<1, 32, 0, s>>>(e->d_step_exec, n_launch);
       // every side stream joins the step: the next replay may start at once
@@ -688,7 +709,7 @@ static int step_graph(dum_engine *e, const uint64_t *launch_hash, const uint64_t
     if (err != cudaSuccess) {
       // not capturable here: say so once, drop to the one-call path for good
       cudaGetLastError();
-      fprintf(stderr, "libdeepum_b200: dum_step graph capture failed (%s); steps run uncaptured\n",
+      fprintf(stderr, "libdeepum_b200: dum_step graph capture failed at %s (%s); steps run uncaptured\n", stage,
               cudaGetErrorString(err));
       e->graph_steps = false;
       e->wres_pending = false;
@@ -704,6 +725,8 @@ static int step_graph(dum_engine *e, const uint64_t *launch_hash, const uint64_t
   }
   CK(cudaGraphLaunch(exec, s));
   e->widx_stale = true;  // the replayed build's walk index is built by the next step
+  e->jump_stale = true;  // and so are its jump tables
+  e->commit_stale = !e->fast_windows;  // and, with exact windows, the publishing of its walks
   CK(cudaEventRecord(e->ev_graph, s));
   CK(cudaEventRecord(e->ev_stage_free[set], s));  // this set's staging and upload buffers are free again
   CK(cudaStreamWaitEvent(caller, e->ev_graph, 0));
@@ -1025,6 +1048,7 @@ static void put64(std::vector<uint8_t> &o, uint64_t v) {
 int dum_dump_state(dum_engine *e, uint32_t what, void *host_buf, uint64_t cap, uint64_t *needed) {
   if (!e) return DUM_EINVAL;
   cudaSetDevice(e->device);
+  if (e->commit_stale) CK(launch_walk_commit(e, e->graph_s));  // the last replayed build's walks
   CK(cudaDeviceSynchronize());
   DevState st;
   CK(cudaMemcpy(&st, e->d_state, sizeof(st), cudaMemcpyDeviceToHost));

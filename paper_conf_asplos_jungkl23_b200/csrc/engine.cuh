@@ -268,6 +268,8 @@ struct dum_engine {
   bool wres_pending;           // dum_step issued the walk residency facts beside the ingest
   bool cap_events_ready;
   bool widx_stale;             // the walk index lags the last (replayed) build
+  bool jump_stale;             // the jump tables lag the last (captured / replayed) build
+  bool commit_stale;           // the walks of the last (captured / replayed) build are not yet published
   cudaEvent_t cap_ev[8];       // the fork / join events of a step-graph capture (graph edges only)
   struct StepGraph {
     uint64_t key[12];

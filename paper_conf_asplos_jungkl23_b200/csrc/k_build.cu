@@ -1138,10 +1138,10 @@ static cudaError_t launch_apply_walk(dum_engine *e, const BuildArgs &ba, cudaStr
   }
   {
     TimerScope t(e, DUM_T_APPLY_WALK, s);
-    k_build_exec<MA, MS><<<std::min(e->n_staged, e->apply_grid), BX_NT, bsmem, s>>>(ba);
+    k_build_exec<MA, MS><<<std::min(ba.n_staged, e->apply_grid), BX_NT, bsmem, s>>>(ba);
   }
   TimerScope t(e, DUM_T_WALK, s);
-  k_walk<MA, MS><<<std::min(e->n_staged, e->walk_grid), WK_NT, wsmem, s>>>(ba);  // dd_list only
+  k_walk<MA, MS><<<std::min(ba.n_staged, e->walk_grid), WK_NT, wsmem, s>>>(ba);  // dd_list only
   return cudaGetLastError();
 }
 
@@ -1205,6 +1205,17 @@ __global__ void __launch_bounds__(256) k_walk_commit(const LeadDesc *__restrict_
   }
 }
 
+cudaError_t launch_walk_commit(dum_engine *e, cudaStream_t s) {
+  TimerScope t(e, DUM_T_COMMIT, s);
+  k_walk_commit<<<std::max<uint32_t>(1, std::min<uint32_t>(e->g.Emax, 148 * 8)), 256, 0, s>>>(
+      reinterpret_cast<const LeadDesc *>(e->d_lead), e->d_state, e->g.walk_cap, e->d_walk_n, e->d_walk_len_n,
+      reinterpret_cast<const uint2 *>(e->d_wrun_n), e->d_wrun_len_n, e->d_walk, e->d_walk_len,
+      reinterpret_cast<uint2 *>(e->d_wrun), e->d_wrun_len);
+  e->commit_stale = false;
+  e->kernel_launches += 1;
+  return cudaGetLastError();
+}
+
 // The build of the n staged launches into the staging walk arrays: the head
 // (correlation upserts + work lists, k_build_prep / k_plan; the jump tables
 // forked to the side stream), the table apply + walks (k_build_exec, k_walk)
@@ -1221,12 +1232,20 @@ static cudaError_t build_body(dum_engine *e, const BuildArgs &ba, cudaStream_t s
                                                   e->d_order, e->d_e_ops, e->d_e_last, ba.plan_agg, e->d_state);
     k_plan<<<(n + PLAN_NT - 1) / PLAN_NT, PLAN_NT, 0, s>>>(ba);
   }
-  // the jump tables depend only on the correlation table, final here
-  cudaEventRecord(e->ev_fork, s);
-  cudaStreamWaitEvent(e->side, e->ev_fork, 0);
-  cudaError_t err = launch_jump_tables(e, e->side);
-  cudaEventRecord(e->ev_join, e->side);
-  if (err != cudaSuccess) return err;
+  // the jump tables depend only on the correlation table, final here; a
+  // captured step leaves them to the start of the next step (beside its
+  // ingest) instead of joining them at its end
+  cudaError_t err = cudaSuccess;
+  if (e->capturing) {
+    e->jump_stale = true;
+  } else {
+    cudaEventRecord(e->ev_fork, s);
+    cudaStreamWaitEvent(e->side, e->ev_fork, 0);
+    err = launch_jump_tables(e, e->side);
+    cudaEventRecord(e->ev_join, e->side);
+    e->jump_stale = false;
+    if (err != cudaSuccess) return err;
+  }
   if (e->g.A <= 2 && e->g.S <= 4) err = launch_apply_walk<2, 4>(e, ba, s);
   else if (e->g.A == 2 && e->g.S == 8) err = launch_apply_walk<2, 8>(e, ba, s);
   else if (e->g.A == 4 && e->g.S == 4) err = launch_apply_walk<4, 4>(e, ba, s);
@@ -1270,16 +1289,22 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
     cudaStreamWaitEvent(s, e->ev_bhead, 0);
     e->bhead_pending = false;
   } else {
+    // the staging arrays still hold the last replayed build's unpublished walks
+    if (!e->capturing && e->commit_stale) {
+      const cudaError_t ce = launch_walk_commit(e, s);
+      if (ce != cudaSuccess) return ce;
+    }
     const BuildArgs ba = build_args(e, n);
     const cudaError_t be = build_body(e, ba, s);
     if (be != cudaSuccess) return be;
   }
-  {  // publish the rebuilt walks (predict, the only other reader, is ordered before)
-    TimerScope t(e, DUM_T_COMMIT, s);
-    k_walk_commit<<<std::max<uint32_t>(1, std::min<uint32_t>(e->g.Emax, 148 * 8)), 256, 0, s>>>(
-        reinterpret_cast<const LeadDesc *>(e->d_lead), e->d_state, e->g.walk_cap, e->d_walk_n, e->d_walk_len_n,
-        reinterpret_cast<const uint2 *>(e->d_wrun_n), e->d_wrun_len_n, e->d_walk, e->d_walk_len,
-        reinterpret_cast<uint2 *>(e->d_wrun), e->d_wrun_len);
+  if (e->capturing && !e->fast_windows) {
+    // a captured step publishes its walks at the start of the next step, beside
+    // its ingest (before k_chain, their first reader)
+    e->commit_stale = true;
+  } else {  // publish the rebuilt walks (predict, the only other reader, is ordered before)
+    const cudaError_t ce = launch_walk_commit(e, s);
+    if (ce != cudaSuccess) return ce;
   }
   if (e->capturing) {
     // a captured step builds the walk index at the start of the next step,

@@ -1008,13 +1008,23 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   } else if (sel && (err = launch_walk_res(e, s)) != cudaSuccess) {  // residency facts per walk
     return err;
   }
+  if (!e->capturing && e->commit_stale && (err = launch_walk_commit(e, s)) != cudaSuccess) return err;
   if (!e->capturing) {  // (a captured step joins its side streams before it ends)
     if (e->widx_stale) {  // the last build was a replayed step: its walk index is due
       if ((err = launch_walk_index(e, s)) != cudaSuccess) return err;
       e->widx_stale = false;
     }
-    cudaStreamWaitEvent(s, e->ev_join, 0);  // jump tables of the last build (side stream)
+    if (e->jump_stale) {  // ... and so are its jump tables
+      cudaEventRecord(e->ev_fork, s);
+      cudaStreamWaitEvent(e->side, e->ev_fork, 0);
+      if ((err = launch_jump_tables(e, e->side)) != cudaSuccess) return err;
+      cudaEventRecord(e->ev_join, e->side);
+      e->jump_stale = false;
+    }
   }
+  // jump tables of the last build (side stream; in a captured step: forked at
+  // its start, beside the ingest)
+  cudaStreamWaitEvent(s, e->ev_join, 0);
   cudaStreamWaitEvent(s, e->ev_widx, 0);  // walk index of the last build (third side stream)
   {
     TimerScope t(e, DUM_T_CHAIN, s);

@@ -10,6 +10,7 @@ cudaError_t launch_record(dum_engine *e, const uint64_t *hash, const uint64_t *o
 // k_build.cu   (a3 - a6)
 cudaError_t launch_build(dum_engine *e, cudaStream_t s);
 cudaError_t launch_build_head(dum_engine *e, uint32_t n, cudaStream_t s);
+cudaError_t launch_walk_commit(dum_engine *e, cudaStream_t s);
 cudaError_t launch_jump_tables(dum_engine *e, cudaStream_t s);
 // k_predict.cu (a6 + a7)
 cudaError_t launch_make_queries(dum_engine *e, const uint32_t *exec_seq, uint32_t n_seq, uint32_t first,

@@ -43,13 +43,14 @@ for i in range(n_iter):
     ds.append(hs[-1].to(dev))
 cap = 24 << 20
 res = {}
-for mode in ["full", "one_copy_stream", "dev_inputs", "no_snap_upload", "no_d2h", "plain"]:
+for mode in ["full", "counting_off", "one_copy_stream", "dev_inputs", "no_snap_upload", "no_d2h", "plain"]:
     host_in = mode not in ("dev_inputs", "plain")
     snap_up = mode not in ("no_snap_upload", "plain")
     d2h = mode not in ("no_d2h", "plain")
     eng.reset()
     eng.mark_inactive(B.as_u32_tensor(tr.inactive_blocks, dev), True)
     eng.set_step_graphs(True)
+    eng.set_counting(mode != "counting_off")
     outs = {}
     snap_dev = [torch.empty(tr.C, dtype=torch.int32, device=dev) for _ in range(2)]
     out_r = [torch.empty((K, 2), dtype=torch.int64).pin_memory() for _ in range(args.steps)]

@@ -66,6 +66,12 @@ if bf:
     out += ["## The fast-window mode (`bench.py --fast-windows`)", "",
             "%.3g records/s (%.4f ms/step); dominant kernel %s %.1f us" % (
                 bf["value"], bf["ms_per_step"], bf["roofline"].get("kernel"), bf["roofline"].get("avg_us") or 0), ""]
+bg = line(os.path.join(G, tag + "_bench_graph.log"))
+if bg:
+    json.dump(bg, open(os.path.join(P, "bench_graph_%s.json" % tag), "w"), indent=1)
+    out += ["## Steps replayed as CUDA graphs (`bench.py --graph`)", "",
+            "%.3g records/s (%.4f ms/step); e2e %.3g records/s (%.4f ms/step)" % (
+                bg["value"], bg["ms_per_step"], bg["e2e"]["value"], bg["e2e"]["ms_per_step"]), ""]
 br = line(os.path.join(G, tag + "_ref.log"))
 if br:
     json.dump(br, open(os.path.join(P, "bench_ref_%s.json" % tag), "w"), indent=1)
