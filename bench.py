@@ -513,7 +513,9 @@ def run_ours(args, rank, world, local_rank):
     e2e = None
     if not args.no_e2e:
         barrier()  # every replica's e2e leg starts together
-        eng.set_step_graphs(not args.no_graph)
+        # host inputs: each step replays as a CUDA graph (uncaptured, the host
+        # issue of a step's ~40 launches would bound it; --separate-calls: no graphs)
+        eng.set_step_graphs(not args.separate_calls)
         eng.set_counting(False)  # as in the timed region: no instrumentation atomics
         e2e = run_e2e(args, tr, eng, dev, stream, cap[0], cap[0])
         eng.set_counting(True)
@@ -611,7 +613,9 @@ def verify_step(tr, N, out):
 
 def run_e2e(args, tr, eng, dev, stream, cap, sel_cap):
     """The same steps through the public C-ABI with every per-step input in
-    pinned HOST memory, one call per step: dum_step(DUM_HOST_PTRS) uploads the
+    pinned HOST memory, one call per step, replayed as a CUDA graph
+    (dum_set_step_graphs: the host issue of an uncaptured step, ~40 launches,
+    would bound a host-fed loop): dum_step(DUM_HOST_PTRS) uploads the
     launch records on the engine's ingest stream and runs record -> queries ->
     predict+select -> build; the iteration-start residency snapshot is copied
     up (copy stream) and loaded with dum_load_residency; each step's per-query
@@ -645,8 +649,8 @@ def run_e2e(args, tr, eng, dev, stream, cap, sel_cap):
     outs = {}
     eng.reset()
     eng.mark_inactive(torch.from_numpy(tr.inactive_blocks.view(np.int32)).to(dev), True)
-    # the timed steps' mode (the breakdown pass before this turned the step graphs off)
-    eng.set_step_graphs(not args.separate_calls and not args.no_graph)
+    # replayed step graphs (the breakdown pass before this turned them off)
+    eng.set_step_graphs(not args.separate_calls)
 
     def host_step(i, s=None):
         n = hs[i].numel()
@@ -704,7 +708,7 @@ def run_e2e(args, tr, eng, dev, stream, cap, sel_cap):
             "d2h_bytes_per_step": d2h, "ms_per_step": tot / args.steps,
             "host_wall_ms_per_step": 1000 * wall / args.steps,
             "host_issue_us_per_step": [round(1e6 * x, 1) for x in issue],
-            "note": "public C-ABI, one dum_step call per step with pinned HOST launch records (DUM_HOST_PTRS, "
+            "note": "public C-ABI, one dum_step call per step (replayed CUDA graph) with pinned HOST launch records (DUM_HOST_PTRS, "
                     "uploaded on the engine's ingest stream) + the iteration-start residency snapshot uploaded "
                     "(copy stream) and loaded + the per-query prefetch/victim ranges read back per step; steps "
                     "issued back to back, one CUDA-event region over the K steps (it ends after the last "

@@ -235,7 +235,10 @@ int dum_predict_select(dum_engine *eng, const dum_query *queries, uint32_t n_que
  * state built by the previous steps -> dum_build_tables(batch).  Outputs and
  * their layouts are dum_predict_select's, one query per launch in launch
  * order.  The engine keeps the last three exec IDs of the previous step
- * (DUM_NONE after dum_reset).  Requires no batch staged by dum_record_faults. */
+ * (DUM_NONE after dum_reset).  Requires no batch staged by dum_record_faults.
+ * The build of the batch runs beside the predict kernels (side stream, issued
+ * after the chain step); its rebuilt walks are published after predict, so
+ * predict sees the tables and walks of the previous steps only (D12). */
 int dum_step(dum_engine *eng, const uint64_t *launch_hash, const uint64_t *launch_off, uint32_t n_launch,
              const uint32_t *fault_block, uint64_t n_fault, uint32_t flags, uint32_t degree, uint32_t *out_pairs,
              uint64_t out_cap_pairs, uint64_t *out_range, uint32_t *out_kern_off, uint32_t *out_chain,
@@ -246,7 +249,9 @@ int dum_step(dum_engine *eng, const uint64_t *launch_hash, const uint64_t *launc
  * the engine's upload buffers, then the whole step replays as one graph (one
  * per batch size x staging set x output buffers, captured on first use; every
  * value a step changes lives on the device).  Outputs must keep their
- * addresses between the steps of one graph. */
+ * addresses between the steps of one graph.  A captured build leaves its
+ * jump tables and the publishing of its walks to the start of the next step
+ * (or to the next predict / build / dum_dump_state call). */
 int dum_set_step_graphs(dum_engine *eng, int enable);
 
 /* Mark UM blocks as belonging to inactive (inactive != 0) or active PyTorch
