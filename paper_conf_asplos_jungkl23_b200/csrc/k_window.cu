@@ -825,9 +825,6 @@ __global__ void __launch_bounds__(WSEL_NT, 3) k_window_fast(PredArgs a) {
   lg.al = (lg.head & 3u) == 0;
   unsigned long long scanned = 0, victims = 0, emitted = 0;
   if (tid < SG_NT) {  // the selection group: a query per item
-#ifdef EXP_COPY_ONLY
-    return;
-#endif
     uint32_t ccnt[NQCLS], n1 = 0;
 #pragma unroll
     for (int c = 0; c < NQCLS; ++c) {
@@ -870,11 +867,7 @@ __global__ void __launch_bounds__(WSEL_NT, 3) k_window_fast(PredArgs a) {
 #endif
   }
   {  // the copy warps; the selection group joins them once its queue is empty
-#ifdef EXP_SEL_ONLY
-    const unsigned long long G = 0;
-#else
     const unsigned long long G = min((unsigned long long)a.chunk_cap, __ldcg(&a.st->pool_chunks));
-#endif
     for (;;) {
       unsigned long long c0 = 0;
       if (lane == 0) c0 = atomicAdd(&a.st->copy_queue, (unsigned long long)CPW);
