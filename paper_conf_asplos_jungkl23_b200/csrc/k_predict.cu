@@ -541,24 +541,25 @@ __global__ void __launch_bounds__(PRED_NT, 2) k_predict(PredArgs a) {
       if (k < DLCAP) s_dup[k] = w * 32 + bit;
     }
   };
-  {
-    // ---------------- pass 1 (whole CTA): window set, duplicate test, non-resident count ----------------
-    // One shared atomicOr per run.  Within one walk the runs are disjoint, so
-    // a bit found already set means the block occurs in two lists of the
-    // window, or is the anchor (in the window set, never emitted; D14).
+  // ---------------- pass 1: window set, duplicate test, non-resident count ----------------
+  // by threads t = [0, nt): one shared atomicOr per run.  Within one walk the
+  // runs are disjoint, so a bit found already set means the block occurs in
+  // two lists of the window, or is the anchor (in the window set, never
+  // emitted; D14).
+  auto pass1 = [&](uint32_t t, uint32_t nt) {
     const uint32_t etot = nk ? eoff[nk] : 0;
     uint32_t nonres = 0;
-    if (tid == 0 && anchored && anchor < g.W) {
+    if (t == 0 && anchored && anchor < g.W) {
       const uint32_t m = 1u << (anchor & 31);
       record_dup(anchor >> 5, atomicOr(&bitmap[anchor >> 5], m) & m);
     }
     uint32_t lo = 0;  // list of run x (x only grows: a running cursor, no search)
     constexpr int RB = 4;  // runs per thread with their loads in flight together
-    for (uint32_t x0 = tid; x0 < etot; x0 += PRED_NT * RB) {
+    for (uint32_t x0 = t; x0 < etot; x0 += nt * RB) {
       uint32_t w[RB], m[RB];
 #pragma unroll
       for (int q = 0; q < RB; ++q) {
-        const uint32_t x = x0 + q * PRED_NT;
+        const uint32_t x = x0 + q * nt;
         w[q] = NONE;
         m[q] = 0;
         if (x < etot) {
@@ -590,16 +591,16 @@ __global__ void __launch_bounds__(PRED_NT, 2) k_predict(PredArgs a) {
       for (int o = 16; o; o >>= 1) nonres += __shfl_xor_sync(0xffffffffu, nonres, o);
       if (lane == 0 && nonres) atomicAdd(&s_nonres, nonres);
     }
-  }
-  __syncthreads();
-  // Duplicates are known now: without them (the normal case) warps
-  // [0, GRP_W) run the selection (a8) while the others stream the pairs; with
-  // them the whole CTA takes the duplicate path below instead.
-  if (s_ndup == 0 && !SELECT) {
-    if (ok) copy_lists(wid, NWARP, loff, nullptr);  // predict only: every warp streams
-  } else if (s_ndup == 0) {
+  };
+  if (SELECT) {
+    // warps [0, GRP_W): pass 1, then -- without duplicates, the normal case --
+    // the selection (a8); warps [GRP_W, NWARP) stream the pairs meanwhile,
+    // speculatively: a window with duplicates is rewritten by the duplicate
+    // path below (whole CTA), which also redoes the selection
     if (wid < GRP_W) {
-      {
+      pass1(tid, GRP_NT);
+      group_sync<1, GRP_NT>();
+      if (s_ndup == 0) {
         if (tid == 0) select_reserve(a.so, s_nonres, a.st, ss);
         group_sync<1, GRP_NT>();
         select_tail<GRP_NT, 1>(a.so, qi, ss, InBlockBitmap{bitmap}, a.st, tid, dk);
@@ -607,6 +608,10 @@ __global__ void __launch_bounds__(PRED_NT, 2) k_predict(PredArgs a) {
     } else if (ok) {
       copy_lists(wid - GRP_W, NWARP - GRP_W, loff, nullptr);
     }
+  } else {  // predict only: pass 1 by the whole CTA, then every warp streams (no duplicates)
+    pass1(tid, PRED_NT);
+    __syncthreads();
+    if (s_ndup == 0 && ok) copy_lists(wid, NWARP, loff, nullptr);
   }
   __syncthreads();
   const uint32_t ndup = s_ndup;
