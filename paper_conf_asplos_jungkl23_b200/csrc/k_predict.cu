@@ -402,7 +402,7 @@ __global__ void __launch_bounds__(CHAIN_WARPS * 32) k_chain(PredArgs a) {
 // the (block, exec) pairs meanwhile.  Duplicates (rare) are only known after
 // pass 1: the duplicate path then rewrites the pairs and redoes the selection
 // with the whole CTA.
-constexpr int GRP_W = 10;  // window set + selection warps; the other NWARP - GRP_W copy (6, 8, 12 measured: no better)
+constexpr int GRP_W = 10;  // window set + selection warps; the other NWARP - GRP_W copy (6, 8 measured: slower)
 constexpr int GRP_NT = GRP_W * 32;
 constexpr uint32_t OCCAP = 1024;   // duplicate occurrences (list, block) tracked by the duplicate path
 constexpr uint32_t DWCAP = 1024;   // duplicate-word hash slots (word -> mask of duplicated blocks)
