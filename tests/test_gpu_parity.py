@@ -485,3 +485,52 @@ def test_fast_selection_on_a_log_with_stale_entries(seed):
     fused_both(eng, o, qs)
     c1 = eng.counters()
     assert c1["Q_FAST"] > c0["Q_FAST"] and c1["FAST_DIRTY"] == c0["FAST_DIRTY"]
+
+
+@pytest.mark.parametrize("fast", [False, True])
+def test_graph_steps_then_separate_calls(fast):
+    """Graph-replayed dum_step leaves its jump tables and (exact windows) the
+    publishing of its rebuilt walks to what comes next; here the next calls
+    are the separate record / predict+select / build calls, then dum_step
+    again (uncaptured first use, then replays): every window, victim list and
+    the final tables equal the oracle's."""
+    tr = wl.make_T(dup_ppm=50_000)
+    N = 2
+    eng, o = make_pair(W=tr.W, C=tr.C, N=N, fast=fast)
+    snap = tr.snap_blk[4][: int(tr.snap_cnt[4])]
+    o.load_residency(snap)
+    eng.load_residency(dev(snap))
+    ex_all, out = [], {}
+    eng.set_step_graphs(True)
+    for i in range(tr.n_iter):
+        h, off, f = tr.iteration(i)
+        exo = o.record_faults(h, off, f)
+        ex_all += [int(x) for x in exo]
+        qs = transition_queries(ex_all, i * tr.K, tr.K, N)
+        off_o, pairs_o, ko_o, ch_o = o.predict(qs)
+        wo, wb_o, io, iv_o = o.select(off_o, pairs_o, qs[:, 4])
+        if i in (4, 5):  # separate calls between replayed steps
+            exg = torch.empty(len(h), dtype=torch.int32, device="cuda")
+            eng.record_faults(dev(h, np.uint64), dev(off, np.uint64), dev(f), exg)
+            assert np.array_equal(B.u32(exg), exo)
+            if i >= 1:
+                fused_both(eng, o, qs)
+            o.build_tables()
+            eng.build_tables()
+            eng.sync()
+            continue
+        o.build_tables()
+        eng.step(dev(h, np.uint64), dev(off, np.uint64), dev(f), 4096, 4096, out)
+        eng.sync()
+        gp, rg = B.u32(out["pairs"]).reshape(-1, 2), B.u64(out["rng"]).reshape(-1, 2)
+        sr = B.u64(out["sel_rng"]).reshape(-1, 4)
+        gwb, giv = B.u32(out["wb"]), B.u32(out["inv"])
+        # (dum_step's query history spans dum_step calls only: after the
+        # separate calls its first three queries differ from the true history)
+        for q in range(3 if i == 6 else 0, tr.K):
+            assert np.array_equal(gp[rg[q, 0]:rg[q, 1]], pairs_o[off_o[q]:off_o[q + 1]]), (i, q)
+            assert np.array_equal(gwb[sr[q, 0]:sr[q, 1]], wb_o[wo[q]:wo[q + 1]]), (i, q)
+            assert np.array_equal(giv[sr[q, 2]:sr[q, 3]], iv_o[io[q]:io[q + 1]]), (i, q)
+        if i == 3:
+            assert_same_state(eng, o, msg="after replayed steps")  # (publishes the pending walks)
+    assert_same_state(eng, o)
