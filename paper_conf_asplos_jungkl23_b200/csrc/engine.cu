@@ -97,6 +97,8 @@ cudaError_t fill(uint32_t *p, uint64_t n, uint32_t v, cudaStream_t s) {
 
 int reset_state(dum_engine *e, cudaStream_t s) {
   const Geo &g = e->g;
+  if (e->ev_commit) CK(cudaStreamWaitEvent(s, e->ev_commit, 0));  // a walk commit still copying
+  e->commit_inflight = false;
   e->commit_stale = false;  // (the walks are cleared below)
   e->jump_stale = false;
   if (e->ev_join) CK(cudaStreamWaitEvent(s, e->ev_join, 0));  // jump tables still building on the side stream
@@ -164,6 +166,7 @@ void free_all(dum_engine *e) {
   if (e->side4) cudaStreamDestroy(e->side4);
   if (e->ev_fork4) cudaEventDestroy(e->ev_fork4);
   if (e->ev_bhead) cudaEventDestroy(e->ev_bhead);
+  if (e->ev_commit) cudaEventDestroy(e->ev_commit);
   if (e->ev_widx) cudaEventDestroy(e->ev_widx);
   if (e->ev_fork2) cudaEventDestroy(e->ev_fork2);
   if (e->ev_join2) cudaEventDestroy(e->ev_join2);
@@ -308,6 +311,7 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   }
   A_(cudaEventCreateWithFlags(&e->ev_fork4, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_bhead, cudaEventDisableTiming));
+  A_(cudaEventCreateWithFlags(&e->ev_commit, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_widx, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_fork2, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_join2, cudaEventDisableTiming));
@@ -617,6 +621,10 @@ static int step_graph(dum_engine *e, const uint64_t *launch_hash, const uint64_t
   CK(cudaStreamWaitEvent(s, e->ev_widx, 0));
   CK(cudaStreamWaitEvent(s, e->ev_join2, 0));
   CK(cudaStreamWaitEvent(s, e->ev_rec, 0));
+  if (e->commit_inflight) {  // an uncaptured build's walk commit (side stream)
+    CK(cudaStreamWaitEvent(s, e->ev_commit, 0));
+    e->commit_inflight = false;
+  }
   const uint64_t key[12] = {n_launch, (uint64_t)e->stage_set, degree, (uint64_t)out_pairs, out_cap_pairs,
                             (uint64_t)out_range, (uint64_t)out_kern_off, (uint64_t)out_chain, (uint64_t)out_needed,
                             (uint64_t)out_writeback ^ ((uint64_t)out_invalidate << 1), sel_cap,

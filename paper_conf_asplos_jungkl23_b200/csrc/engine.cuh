@@ -270,6 +270,8 @@ struct dum_engine {
   bool widx_stale;             // the walk index lags the last (replayed) build
   bool jump_stale;             // the jump tables lag the last (captured / replayed) build
   bool commit_stale;           // the walks of the last (captured / replayed) build are not yet published
+  cudaEvent_t ev_commit;       // an uncaptured build's walk commit (side stream); its readers wait for it
+  bool commit_inflight;        // ev_commit not yet waited for by predict
   cudaEvent_t cap_ev[8];       // the fork / join events of a step-graph capture (graph edges only)
   struct StepGraph {
     uint64_t key[12];

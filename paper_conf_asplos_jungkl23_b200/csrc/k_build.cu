@@ -1281,6 +1281,10 @@ cudaError_t launch_build_head(dum_engine *e, uint32_t n, cudaStream_t s) {
 cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
   const uint32_t n = e->n_staged;
   if (n == 0) return cudaSuccess;
+  if (e->commit_inflight && !e->capturing) {  // the last commit still reads the staging arrays
+    cudaStreamWaitEvent(s, e->ev_commit, 0);
+    e->commit_inflight = false;
+  }
   if (!e->capturing) {  // (a captured step joins its side streams before it ends)
     cudaStreamWaitEvent(s, e->ev_join, 0);  // the previous build's jump tables read corr
     cudaStreamWaitEvent(s, e->ev_widx, 0);  // the previous build's walk index reads the walk cache
@@ -1302,7 +1306,17 @@ cudaError_t launch_build(dum_engine *e, cudaStream_t s) {
     // a captured step publishes its walks at the start of the next step, beside
     // its ingest (before k_chain, their first reader)
     e->commit_stale = true;
-  } else {  // publish the rebuilt walks (predict, the only other reader, is ordered before)
+  } else if (!e->capturing && !e->fast_windows) {
+    // publish the rebuilt walks beside the next step's residency load and
+    // ingest (side stream): their readers -- the next predict, the next build
+    // (staging) -- wait for ev_commit
+    cudaEventRecord(e->ev_fork4, s);
+    cudaStreamWaitEvent(e->side4, e->ev_fork4, 0);
+    const cudaError_t ce = launch_walk_commit(e, e->side4);
+    if (ce != cudaSuccess) return ce;
+    cudaEventRecord(e->ev_commit, e->side4);
+    e->commit_inflight = true;
+  } else {  // publish the rebuilt walks (the walk index below reads them)
     const cudaError_t ce = launch_walk_commit(e, s);
     if (ce != cudaSuccess) return ce;
   }

@@ -1011,6 +1011,10 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
     return err;
   }
   if (!e->capturing && e->commit_stale && (err = launch_walk_commit(e, s)) != cudaSuccess) return err;
+  if (e->commit_inflight && !e->capturing) {  // the last build's walks (side-stream commit)
+    cudaStreamWaitEvent(s, e->ev_commit, 0);
+    e->commit_inflight = false;
+  }
   if (!e->capturing) {  // (a captured step joins its side streams before it ends)
     if (e->widx_stale) {  // the last build was a replayed step: its walk index is due
       if ((err = launch_walk_index(e, s)) != cudaSuccess) return err;
