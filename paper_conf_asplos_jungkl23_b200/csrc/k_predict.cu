@@ -933,7 +933,7 @@ cudaError_t launch_predict(dum_engine *e, const dum_query *q, uint32_t nq, uint3
   if (nq > e->anchor_range_cap) return cudaErrorInvalidValue;
   WalkScratch ws{e->d_walk_seen, e->d_walk_chain, e->d_walk_tmp, e->walk_hash_cap,
                  e->g.walk_cap + e->g.R * e->g.A + 4};
-  {
+  if (!e->bhead_n) {  // (dum_step's queries are transition queries: no anchors, no anchored walks)
     TimerScope t(e, DUM_T_ANCHOR_WALK, s);
     k_anchor_walk<<<e->n_walk_slots, 32, 0, s>>>(e->g, q, nq, e->d_tbl, e->d_start_end, e->d_walk_out,
                                                  e->d_anchor_pool, e->anchor_pool_entries, e->d_anchor_range, ws,
