@@ -167,6 +167,8 @@ void free_all(dum_engine *e) {
   if (e->ev_fork4) cudaEventDestroy(e->ev_fork4);
   if (e->ev_bhead) cudaEventDestroy(e->ev_bhead);
   if (e->ev_commit) cudaEventDestroy(e->ev_commit);
+  if (e->ev_wslow_fork) cudaEventDestroy(e->ev_wslow_fork);
+  if (e->ev_wslow) cudaEventDestroy(e->ev_wslow);
   if (e->ev_widx) cudaEventDestroy(e->ev_widx);
   if (e->ev_fork2) cudaEventDestroy(e->ev_fork2);
   if (e->ev_join2) cudaEventDestroy(e->ev_join2);
@@ -312,6 +314,8 @@ int dum_create(const dum_config *cfg, dum_engine **out) {
   A_(cudaEventCreateWithFlags(&e->ev_fork4, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_bhead, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_commit, cudaEventDisableTiming));
+  A_(cudaEventCreateWithFlags(&e->ev_wslow_fork, cudaEventDisableTiming));
+  A_(cudaEventCreateWithFlags(&e->ev_wslow, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_widx, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_fork2, cudaEventDisableTiming));
   A_(cudaEventCreateWithFlags(&e->ev_join2, cudaEventDisableTiming));
@@ -647,7 +651,7 @@ static int step_graph(dum_engine *e, const uint64_t *launch_hash, const uint64_t
     // fork / join events recorded inside a capture become graph edges and may
     // not be waited on outside it: the capture uses its own set
     cudaEvent_t *evs[] = {&e->ev_fork, &e->ev_join, &e->ev_fork2, &e->ev_join2, &e->ev_widx,
-                          &e->ev_wres, &e->ev_fork4, &e->ev_bhead};
+                          &e->ev_wres, &e->ev_fork4, &e->ev_bhead, &e->ev_wslow_fork, &e->ev_wslow};
     constexpr int NEV = sizeof(evs) / sizeof(evs[0]);
     if (!e->cap_events_ready) {
       for (int i = 0; i < NEV; ++i) CK(cudaEventCreateWithFlags(&e->cap_ev[i], cudaEventDisableTiming));

@@ -215,6 +215,7 @@ struct dum_engine {
   cudaStream_t side3;           // walk index (build end)
   cudaStream_t side4;           // dum_step: the build's head (k_build_prep, k_plan) beside the predict kernels
   cudaEvent_t ev_fork4, ev_bhead;
+  cudaEvent_t ev_wslow_fork, ev_wslow;  // the build's sequential walks beside its parallel ones (third side stream)
   uint32_t bhead_n;             // dum_step: launches whose build head launch_predict issues after k_chain
   bool bhead_pending;           // the head was issued early: launch_build waits for ev_bhead
   bool fast_windows;            // DUM_CFG_FAST_WINDOWS
@@ -272,7 +273,7 @@ struct dum_engine {
   bool commit_stale;           // the walks of the last (captured / replayed) build are not yet published
   cudaEvent_t ev_commit;       // an uncaptured build's walk commit (side stream); its readers wait for it
   bool commit_inflight;        // ev_commit not yet waited for by predict
-  cudaEvent_t cap_ev[8];       // the fork / join events of a step-graph capture (graph edges only)
+  cudaEvent_t cap_ev[12];       // the fork / join events of a step-graph capture (graph edges only)
   struct StepGraph {
     uint64_t key[12];
     cudaGraphExec_t exec;

@@ -1140,8 +1140,23 @@ static cudaError_t launch_apply_walk(dum_engine *e, const BuildArgs &ba, cudaStr
     TimerScope t(e, DUM_T_APPLY_WALK, s);
     k_build_exec<MA, MS><<<std::min(ba.n_staged, e->apply_grid), BX_NT, bsmem, s>>>(ba);
   }
-  TimerScope t(e, DUM_T_WALK, s);
-  k_walk<MA, MS><<<std::min(ba.n_staged, e->walk_grid), WK_NT, wsmem, s>>>(ba);  // dd_list only
+  // the sequential walks (slow list) on the third side stream, beside the
+  // parallel ones (dedupe list): disjoint exec IDs, separate scratch
+  cudaEventRecord(e->ev_wslow_fork, s);
+  cudaStreamWaitEvent(e->side3, e->ev_wslow_fork, 0);
+  {
+    WalkScratch ws{e->d_walk_seen, e->d_walk_chain, e->d_walk_tmp, e->walk_hash_cap,
+                   e->g.walk_cap + e->g.R * e->g.A + 4};
+    TimerScope t(e, DUM_T_WALK_SLOW, e->side3);
+    k_walk_slow<<<e->n_walk_slots, 32, 0, e->side3>>>(e->g, e->d_tbl, e->d_start_end, ba.walk, ba.walk_len, ba.wrun,
+                                                     ba.wrun_len, e->d_slow_list, ws, e->d_state);
+  }
+  cudaEventRecord(e->ev_wslow, e->side3);
+  {
+    TimerScope t(e, DUM_T_WALK, s);
+    k_walk<MA, MS><<<std::min(ba.n_staged, e->walk_grid), WK_NT, wsmem, s>>>(ba);  // dd_list only
+  }
+  cudaStreamWaitEvent(s, e->ev_wslow, 0);
   return cudaGetLastError();
 }
 
@@ -1252,13 +1267,6 @@ static cudaError_t build_body(dum_engine *e, const BuildArgs &ba, cudaStream_t s
   else if (e->g.A <= 4 && e->g.S <= 8) err = launch_apply_walk<4, 8>(e, ba, s);
   else err = launch_apply_walk<32, 32>(e, ba, s);
   if (err != cudaSuccess) return err;
-  WalkScratch ws{e->d_walk_seen, e->d_walk_chain, e->d_walk_tmp, e->walk_hash_cap,
-                 e->g.walk_cap + e->g.R * e->g.A + 4};
-  {
-    TimerScope t(e, DUM_T_WALK_SLOW, s);
-    k_walk_slow<<<e->n_walk_slots, 32, 0, s>>>(e->g, e->d_tbl, e->d_start_end, ba.walk, ba.walk_len, ba.wrun,
-                                               ba.wrun_len, e->d_slow_list, ws, e->d_state);
-  }
   e->kernel_launches += 4;
   return cudaGetLastError();
 }
